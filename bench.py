@@ -1,0 +1,391 @@
+#!/usr/bin/env python
+"""Benchmark: BASELINE.json metric "gates/s and achieved HBM GB/s (% of B200 peak)".
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--impl lfqs|reference] [--n 30]
+
+Workload at N = 1 (BASELINE.json configs[1]): the 30-qubit single-gate sweep --
+every gate class (diagonal Z/S/T/Rz/Phase/CZ/CPhase, permutation X/Y/CNOT/SWAP/
+Toffoli, dense H/Rx/Ry/U3 and 4x4 UNITARY2 on adjacent and distant pairs) on
+every target qubit, 18 x 30 = 540 gates, applied in place to a 16 GiB
+complex128 state resident in HBM.  One "step" = one pass of the whole sweep.
+The state (16 GiB) is >> the 126 MB L2, so no L2 flush is needed.
+
+N > 1 (torchrun, one rank per GPU): weak scaling, 2^30 amplitudes per GPU,
+n = 30 + log2 N, the same sweep over all n qubits (gates on the top log2 N
+"global" qubits go through the NCCL half-shard exchange).
+
+--impl reference: the CPU oracle (oracle/, tier B index loop with OpenMP on
+all host cores) on a bounded sample of the same sweep, rank 0 only.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import math
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import workloads as W  # noqa: E402
+
+METRIC = "gates/s and achieved HBM GB/s (% of B200 peak) at 30-36 qubits, 1/2/4/8 GPUs"
+UNIT = "gates/s"
+
+
+def peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    try:
+        with open(p) as f:
+            d = json.load(f)
+        return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs)"
+    except Exception:
+        return 6650.0, "fallback (B200_PROFILING.md)"
+
+
+# ----------------------------------------------------------------------------
+# clocks sampling during the timed region
+# ----------------------------------------------------------------------------
+_REASONS = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+
+
+class ClockSampler:
+    def __init__(self, device: int):
+        self.device = device
+        self.proc = None
+        self.lines = []
+
+    def __enter__(self):
+        q = ("clocks.sm,clocks.max.sm,power.draw,utilization.gpu,"
+             "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+             "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", "-i", str(self.device), f"--query-gpu={q}",
+                 "--format=csv,noheader,nounits", "-lms", "200"],
+                stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except Exception:
+            self.proc = None
+        return self
+
+    def _read(self):
+        for ln in self.proc.stdout:
+            self.lines.append(ln.strip())
+
+    def __exit__(self, *exc):
+        if self.proc:
+            self.proc.terminate()
+            try:
+                self.proc.wait(timeout=5)
+            except Exception:
+                self.proc.kill()
+
+    def summary(self):
+        sm, mx, reasons = [], [], set()
+        for ln in self.lines:
+            f = [x.strip() for x in ln.split(",")]
+            if len(f) < 8:
+                continue
+            try:
+                s, m, util = float(f[0]), float(f[1]), float(f[3])
+            except ValueError:
+                continue
+            mx.append(m)
+            if util > 50:
+                sm.append(s)
+            for name, v in zip(_REASONS, f[4:8]):
+                if v.lower() == "active":
+                    reasons.add(name)
+        return {"sm_mhz": statistics.median(sm) if sm else None,
+                "sm_max_mhz": max(mx) if mx else None,
+                "reasons": sorted(reasons), "samples": len(self.lines)}
+
+
+# ----------------------------------------------------------------------------
+# CPU oracle timing (cpu_baseline and --impl reference)
+# ----------------------------------------------------------------------------
+
+def host_avail_gib():
+    try:
+        with open("/proc/meminfo") as f:
+            for ln in f:
+                if ln.startswith("MemAvailable:"):
+                    return int(ln.split()[1]) / 2 ** 20
+    except Exception:
+        pass
+    return 0.0
+
+
+class OracleSweep:
+    """The oracle (as it stands) applying the sweep gates to a host state, OpenMP tier B."""
+
+    def __init__(self, n: int, seed: int):
+        import oracle
+        self.O = oracle
+        self.n = n
+        avail = host_avail_gib()
+        need = 16 * 2 ** n / 2 ** 30
+        while need > 0.45 * avail and self.n > 20:
+            self.n -= 1
+            need /= 2
+        self.state = oracle.fill_random(seed, 0, 1 << self.n)
+        self.gates = [g for _, g in W.sweep_gates(self.n)]
+        self.cores = oracle.omp_max_threads()
+        self.pos = 0
+
+    def run(self, n_gates: int) -> float:
+        t0 = time.perf_counter()
+        for _ in range(n_gates):
+            g = self.gates[self.pos % len(self.gates)]
+            self.O.apply_gate(self.n, g, self.state, omp=True)
+            self.pos += 1
+        return time.perf_counter() - t0
+
+    def calibrate(self, budget_s: float) -> int:
+        t = self.run(2) / 2
+        return max(1, int(budget_s / max(t, 1e-6)))
+
+
+def cpu_baseline(n: int, budget_s: float = 15.0):
+    ow = OracleSweep(n, seed=0xC0FFEE)
+    g = ow.calibrate(budget_s / 2)
+    t = ow.run(g)
+    res = {"value": g / t, "unit": UNIT, "cores": ow.cores, "kind": "oracle",
+           "sample": f"first {g} gates of the n={ow.n} sweep (of {len(ow.gates)}), oracle tier B "
+                     f"(naive index loop, OpenMP static schedule), host state "
+                     f"{16 * 2 ** ow.n / 2 ** 30:.0f} GiB"}
+    del ow
+    return res
+
+
+def run_reference(args):
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return 0
+    ow = OracleSweep(args.n, seed=0xC0FFEE)
+    per_step = ow.calibrate(budget_s=args.ref_step_s)
+    for _ in range(args.warmup):
+        ow.run(per_step)
+    times = [ow.run(per_step) for _ in range(args.steps)]
+    total = sum(times)
+    value = per_step * args.steps / total
+    line = {
+        "impl": "reference", "metric": METRIC, "value": value, "unit": UNIT,
+        "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
+        "ms_per_step": 1e3 * total / args.steps, "higher_is_better": True,
+        "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+        "config": {"workload": f"configs[1]: {ow.n}-qubit single-gate sweep (bounded sample)",
+                   "n_qubits": ow.n, "gates_per_step": per_step},
+        "cpu_baseline": {"value": value, "unit": UNIT, "cores": ow.cores, "kind": "oracle",
+                         "sample": f"{per_step} sweep gates per step, n={ow.n}, oracle tier B "
+                                   f"OpenMP on {ow.cores} threads"},
+        "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+    return 0
+
+
+# ----------------------------------------------------------------------------
+# GPU arm
+# ----------------------------------------------------------------------------
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="lfqs", choices=["lfqs", "reference"])
+    ap.add_argument("--n", type=int, default=30, help="qubits per GPU")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--e2e-steps", type=int, default=2)
+    ap.add_argument("--ref-step-s", type=float, default=12.0)
+    ap.add_argument("--per-gate-json", default="", help="write per-gate timings here")
+    args = ap.parse_args()
+    if args.impl == "reference":
+        return run_reference(args)
+
+    import torch
+    import paper_conf_cgo_tarabkhahdds25_b200 as lfqs
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local_rank = int(os.environ.get("LOCAL_RANK", "0"))
+    assert world == args.gpus, f"--gpus {args.gpus} but WORLD_SIZE={world}"
+    assert args.warmup >= 3 or os.environ.get("LFQS_BENCH_ALLOW_SHORT"), "need >= 3 warm-up steps"
+    torch.cuda.set_device(local_rank)
+    stream = torch.cuda.current_stream()
+    dist = None
+    if world > 1:
+        import torch.distributed as dist
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
+        p = world.bit_length() - 1
+        assert 1 << p == world, "world size must be a power of two"
+        n = args.n + p
+        obj = [lfqs.lfqs_dist_unique_id() if rank == 0 else None]
+        dist.broadcast_object_list(obj, src=0)
+        st = lfqs.State.distributed(n, rank, world, obj[0], local_rank, stream=stream)
+    else:
+        n = args.n
+        st = lfqs.State.create(n, local_rank, stream=stream)
+
+    sweep = W.sweep_gates(n)
+    seed = 0xC0FFEE
+    st.init_random(seed)
+
+    def barrier():
+        if dist is not None:
+            dist.barrier()
+        torch.cuda.synchronize()
+
+    def one_step(evs=None):
+        for i, (_, g) in enumerate(sweep):
+            if evs is not None:
+                evs[i].record(stream)
+            st.apply(g)
+        if evs is not None:
+            evs[len(sweep)].record(stream)
+
+    for _ in range(args.warmup):
+        one_step()
+    barrier()
+
+    launches0 = st.launches()
+    evs = [[torch.cuda.Event(enable_timing=True) for _ in range(len(sweep) + 1)]
+           for _ in range(args.steps)]
+    t_start = torch.cuda.Event(enable_timing=True)
+    t_end = torch.cuda.Event(enable_timing=True)
+    with ClockSampler(local_rank) as clk:
+        barrier()
+        t_start.record(stream)
+        for k in range(args.steps):
+            one_step(evs[k])
+        t_end.record(stream)
+        barrier()
+    launches = st.launches() - launches0
+    elapsed_ms = t_start.elapsed_time(t_end)
+    if dist is not None:
+        t = torch.tensor([elapsed_ms], device="cuda")
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        elapsed_ms = float(t.item())
+    ms_per_step = elapsed_ms / args.steps
+    gates_per_step = len(sweep)
+    value = gates_per_step / (ms_per_step / 1e3)
+
+    # per-gate / per-class durations (CUDA events on the launching stream)
+    per_gate = np.zeros((args.steps, len(sweep)))
+    for k in range(args.steps):
+        for i in range(len(sweep)):
+            per_gate[k, i] = evs[k][i].elapsed_time(evs[k][i + 1])
+    mean_ms = per_gate.mean(axis=0)
+    n_loc = n - (world.bit_length() - 1)
+    classes = {}
+    for i, (cls, g) in enumerate(sweep):
+        c = classes.setdefault(cls, {"gates": 0, "ms": 0.0, "alg_bytes": 0.0, "conv_bytes": 0.0})
+        c["gates"] += 1
+        c["ms"] += mean_ms[i]
+        c["alg_bytes"] += 32.0 * W.touched_amplitudes(g, n_loc)
+        c["conv_bytes"] += 32.0 * 2 ** n_loc
+    hbm_peak, peak_src = peaks()
+    for c in classes.values():
+        c["alg_GBps"] = c["alg_bytes"] / (c["ms"] / 1e3) / 1e9
+        c["conv_GBps"] = c["conv_bytes"] / (c["ms"] / 1e3) / 1e9
+        c["frac_alg"] = c["alg_GBps"] / hbm_peak
+        c["ms_per_gate"] = c["ms"] / c["gates"]
+        c["share"] = c["ms"] / mean_ms.sum()
+    dom = max(classes, key=lambda k: classes[k]["ms"])
+    dc = classes[dom]
+    traffic = None
+    tp = os.path.join(ROOT, "profiles", "traffic_per_launch.json")
+    if os.path.exists(tp):
+        try:
+            traffic = json.load(open(tp)).get(dom)
+        except Exception:
+            traffic = None
+    roofline = {"bound": "hbm", "kernel": f"{dom} gate kernels (k_group / k_lowq)",
+                "achieved": dc["alg_GBps"], "peak": hbm_peak, "unit": "GB/s",
+                "frac": dc["alg_GBps"] / hbm_peak, "traffic": traffic, "peak_source": peak_src,
+                "bytes_per_launch": dc["alg_bytes"] / dc["gates"],
+                "avg_launch_ms": dc["ms"] / dc["gates"]}
+    if args.per_gate_json and rank == 0:
+        with open(args.per_gate_json, "w") as f:
+            json.dump([{"cls": cls, "gate": g.label(), "ms": float(mean_ms[i]),
+                        "alg_bytes": 32.0 * W.touched_amplitudes(g, n_loc)}
+                       for i, (cls, g) in enumerate(sweep)], f, indent=0)
+
+    # end to end through the public API: H2D of the input state from pinned host
+    # memory, the sweep, and a D2H read of the measured probabilities each step
+    e2e = None
+    if not args.no_e2e:
+        host = torch.empty(1 << n_loc, dtype=torch.complex128, pin_memory=True)
+        hv = host.numpy()
+        st.copy_out(rank << n_loc, 1 << n_loc, out=hv)
+        mq = list(range(10))
+        def e2e_step():
+            st.copy_in(hv, offset=rank << n_loc)
+            one_step()
+            st.measure_probs(mq)
+        e2e_step()
+        barrier()
+        a = torch.cuda.Event(enable_timing=True)
+        b = torch.cuda.Event(enable_timing=True)
+        a.record(stream)
+        for _ in range(args.e2e_steps):
+            e2e_step()
+        b.record(stream)
+        barrier()
+        e_ms = a.elapsed_time(b)
+        if dist is not None:
+            t = torch.tensor([e_ms], device="cuda")
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+            e_ms = float(t.item())
+        e2e = {"value": gates_per_step / (e_ms / args.e2e_steps / 1e3), "unit": UNIT,
+               "h2d_bytes_per_step": 16 * (1 << n_loc) * world,
+               "d2h_bytes_per_step": 8 * (1 << len(mq)) * world}
+        del host
+
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        st.close()
+        torch.cuda.synchronize()
+        cpu = cpu_baseline(n)
+
+    if rank == 0:
+        line = {
+            "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms_per_step,
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
+            "dtype": "f64", "data": "synthetic",
+            "config": {"workload": f"configs[1]: {n}-qubit single-gate sweep "
+                                   f"(18 gate kinds x {n} targets, all classes)",
+                       "n_qubits": n, "qubits_per_gpu": n_loc, "gates_per_step": gates_per_step,
+                       "state_bytes_per_gpu": 16 * 2 ** n_loc,
+                       "l2": "state >> 126 MB L2 every gate; no flush needed",
+                       "parallelism": f"state sharded by top {world.bit_length() - 1} qubits"
+                       if world > 1 else "single GPU"},
+            "roofline": roofline,
+            "classes": {k: {kk: (round(vv, 4) if isinstance(vv, float) else vv)
+                            for kk, vv in v.items()} for k, v in classes.items()},
+            "gpu_launches": int(launches),
+            "clocks": clk.summary(),
+            "e2e": e2e,
+            "cpu_baseline": cpu,
+        }
+        print(json.dumps(line), flush=True)
+    if dist is not None:
+        dist.barrier()
+        dist.destroy_process_group()
+    return 0
+
+
+if __name__ == "__main__":
+    sys.exit(main())

@@ -1,0 +1,179 @@
+/*
+ * lfqs.h -- C ABI of the B200-native LFQS state-vector gate-application library.
+ *
+ * What it computes: the state after each gate of a circuit,
+ *     S_out = G . S_in                                   (Eq. 2)
+ *     G     = I_L (x) M (x) I_R                          (Eq. 1)
+ *     G_q1q2 = sum_ij X_ij (x) I_N (x) U_ij              (Eq. 5, non-adjacent)
+ *     CU    = |0><0| (x) I + |1><1| (x) U                (Fig. 1)
+ * applied in place to a 2^n complex128 Array-of-Structs state
+ * (PAPER.md:503), gate after gate (Eq. 3), followed by
+ * measurement probabilities.  Every gate is one pass over the
+ * changed part of the state -- the matrix is never built (vector fusion,
+ * PAPER.md:401-407) -- with code specialised per sparsity class (static matrix
+ * specialisation): diagonal, permutation, dense 2x2/4x4/8x8.
+ *
+ * Conventions (readings R1, R2, R7):
+ *   - qubit q is bit q of the amplitude index (little-endian).  The paper's
+ *     Kronecker-left qubit i is q = n-1-i.
+ *   - an m-target gate's local index is j = sum_s bit(t_s) << (m-1-s):
+ *     targets[0] is the most significant bit (Eq. 5's q1).
+ *   - controls: the gate acts where every control bit is 1.  No negative controls.
+ *   - amplitudes are interleaved (re, im) doubles, 16 bytes each.
+ *
+ * Errors: every call returns lfqs_status (0 = OK) and never throws or aborts
+ * across the ABI.  On failure lfqs_last_error() (thread-local) describes it.
+ * lfqs_apply_gate / lfqs_run_circuit / lfqs_state_init_* are ASYNCHRONOUS on the
+ * state's CUDA stream: kernel faults surface as LFQS_ERR_CUDA at the next
+ * synchronising call (lfqs_measure_probs, lfqs_copy_out, lfqs_synchronize).
+ * There is no CPU fallback: without a usable CUDA device every call that needs
+ * one returns LFQS_ERR_CUDA.
+ *
+ * Ownership: states returned by lfqs_state_create* own their device memory;
+ * lfqs_state_wrap borrows it (the caller keeps it alive until destroy).  Every
+ * pointer argument is read or written only during the call.  Output buffers are
+ * caller-allocated with explicit lengths.
+ */
+#ifndef LFQS_ABI_INCLUDED_
+#define LFQS_ABI_INCLUDED_
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define LFQS_ABI_VERSION 1
+
+typedef enum {
+  LFQS_OK = 0,
+  LFQS_ERR_INVALID_ARG = -1,   /* bad qubit / arity / params / buffer length / handle */
+  LFQS_ERR_OUT_OF_MEMORY = -2, /* 16 * 2^n_local bytes do not fit on the device */
+  LFQS_ERR_CUDA = -3,          /* CUDA runtime or kernel error, or no device */
+  LFQS_ERR_NCCL = -4,          /* NCCL error (distributed states) */
+  LFQS_ERR_UNSUPPORTED = -5    /* valid request this build does not implement */
+} lfqs_status;
+
+/* Gate kinds.  Matrices: Fig. 1 for X, Y, Z, H, T, I, SWAP;
+ * Nielsen & Chuang (cited PAPER.md:120) for the rest (R7):
+ *   S = diag(1, i), SDG = diag(1, -i), T = diag(1, e^{i pi/4}), TDG = conj,
+ *   RX(t) = [[c, -i s], [-i s, c]], RY(t) = [[c, -s], [s, c]],
+ *   RZ(t) = diag(e^{-i t/2}, e^{i t/2})   (c = cos(t/2), s = sin(t/2)),
+ *   PHASE(p) = diag(1, e^{i p}),
+ *   U3(t, p, l) = [[c, -e^{i l} s], [e^{i p} s, e^{i(p+l)} c]]  (OpenQASM 2),
+ *   SWAP |ij> = |ji>, UNITARYm = caller matrix, m = 1..3 targets.
+ * Controlled forms: CNOT = X + 1 control, Toffoli = X + 2, CZ = Z + 1,
+ * CPhase = PHASE + 1, CU = UNITARY1 + 1 control, MC-Z = Z + (n-1) controls. */
+typedef enum {
+  LFQS_I = 0, LFQS_X, LFQS_Y, LFQS_Z, LFQS_H, LFQS_S, LFQS_SDG, LFQS_T, LFQS_TDG,
+  LFQS_RX, LFQS_RY, LFQS_RZ, LFQS_PHASE, LFQS_U3,
+  LFQS_SWAP,
+  LFQS_UNITARY1, LFQS_UNITARY2, LFQS_UNITARY3,
+  LFQS_NUM_KINDS
+} lfqs_gate_kind;
+
+/* One gate of a circuit (72 bytes).  control_mask bit q = control on qubit q.
+ * params: RX/RY/RZ/PHASE use params[0]; U3 uses (theta, phi, lambda).
+ * matrix: UNITARYm only, 2^m x 2^m row-major interleaved (re, im), borrowed for
+ * the duration of the call. */
+typedef struct {
+  int32_t kind;
+  int32_t n_targets;
+  int32_t n_controls;       /* must equal popcount(control_mask) */
+  int32_t _pad0;
+  int32_t targets[3];
+  int32_t _pad1;
+  uint64_t control_mask;
+  double params[3];
+  const double* matrix;
+} lfqs_gate;
+
+/* lfqs_run_circuit flags */
+#define LFQS_FUSE_NONE      0u  /* one pass per gate: every intermediate state exists */
+#define LFQS_FUSE_LOW       1u  /* shared-memory staging of consecutive low-qubit / diagonal gates */
+#define LFQS_FUSE_DEFAULT   LFQS_FUSE_LOW
+
+typedef struct lfqs_state lfqs_state;  /* opaque */
+
+/* ---- lifetime ------------------------------------------------------------- */
+/* Allocates 16 * 2^n bytes on `device` (cudaMalloc) and initialises |0...0>.
+ * n_qubits in [1, 36].  stream: a cudaStream_t the state's work is ordered on,
+ * or NULL for a library-created non-blocking stream.
+ * LFQS_ERR_OUT_OF_MEMORY if it does not fit. */
+lfqs_status lfqs_state_create(int n_qubits, int device, void* cuda_stream, lfqs_state** out);
+/* Borrow caller device memory (e.g. a torch complex128 tensor of 2^n elements,
+ * 16-byte aligned).  The contents are left as they are. */
+lfqs_status lfqs_state_wrap(int n_qubits, int device, void* dev_ptr, void* cuda_stream,
+                            lfqs_state** out);
+lfqs_status lfqs_state_destroy(lfqs_state* s);
+/* Re-targets subsequent work to another stream (NULL = the library stream). */
+lfqs_status lfqs_state_set_stream(lfqs_state* s, void* cuda_stream);
+
+/* ---- distributed (one process per GPU, SPMD) ---------------- */
+/* rank 0 creates an NCCL unique id (128 bytes); broadcast it (torch.distributed)
+ * and pass it to lfqs_state_create_dist on every rank.  world must be a power of
+ * two; rank r owns the 2^(n - log2 world) amplitudes whose top log2(world) bits
+ * equal r ("global" qubits).  Gates on global qubits are handled transparently:
+ * diagonal ones and controls rank-locally, others by a qubit-swap remap over
+ * NCCL send/recv of half-shards. */
+lfqs_status lfqs_dist_unique_id(uint8_t uid[128]);
+lfqs_status lfqs_state_create_dist(int n_qubits, int rank, int world, const uint8_t uid[128],
+                                   int device, void* cuda_stream, lfqs_state** out);
+/* Single-GPU "virtual" partition: the same remap planner and exchange code
+ * path with `world` shards in one allocation and device-to-device copies as the
+ * transport.  For testing the distributed logic on one GPU. */
+lfqs_status lfqs_state_create_virtual(int n_qubits, int world, int device, void* cuda_stream,
+                                      lfqs_state** out);
+
+/* ---- state contents -------------------------------------------------------- */
+/* |index> (global index). */
+lfqs_status lfqs_state_init_basis(lfqs_state* s, uint64_t index);
+/* Unnormalised counter-based random state: amplitude k = (u(2k), u(2k+1)) with
+ * u(i) = (SplitMix64_output_i(seed) >> 11) * 2^-53 * 2 - 1 (same formula as
+ * workloads/__init__.py).  Input generation for tests and benchmarks only. */
+lfqs_status lfqs_state_init_random(lfqs_state* s, uint64_t seed);
+/* Host <-> device copies of amplitudes [offset, offset+count) in canonical
+ * (logical) qubit order; host buffers hold 2*count doubles.  Synchronous. */
+lfqs_status lfqs_copy_in(lfqs_state* s, uint64_t offset, uint64_t count, const double* host);
+lfqs_status lfqs_copy_out(lfqs_state* s, uint64_t offset, uint64_t count, double* host);
+
+/* ---- gates ------------------------------------------------------------------ */
+/* One gate, one pass (no fusion).  targets/controls are qubit lists; params has
+ * n_params doubles (must equal the kind's count); matrix for UNITARYm. */
+lfqs_status lfqs_apply_gate(lfqs_state* s, int kind, const int* targets, int n_targets,
+                            const int* controls, int n_controls, const double* params,
+                            int n_params, const double* matrix);
+/* Applies gates[0..n_gates) in order.  flags: LFQS_FUSE_*.  With
+ * LFQS_FUSE_NONE the result equals n_gates lfqs_apply_gate calls bit for bit;
+ * with fusion, permutation/diagonal results are still value-exact and dense
+ * results agree within rounding (<= 1e-12 abs per amplitude). */
+lfqs_status lfqs_run_circuit(lfqs_state* s, const lfqs_gate* gates, size_t n_gates, uint32_t flags);
+
+/* ---- measurement -------------------------------------------- */
+/* probs_out[v] = sum over k with bit qubits[s] of k == bit s of v of |a_k|^2,
+ * v in [0, 2^n_q).  n_q = 0 gives the squared norm.  n_q <= 10.  Deterministic
+ * (fixed reduction order).  probs_len >= 2^n_q.  Synchronous. */
+lfqs_status lfqs_measure_probs(lfqs_state* s, const int* qubits, int n_q, double* probs_out,
+                               size_t probs_len);
+
+/* ---- misc ------------------------------------------------------------------- */
+lfqs_status lfqs_synchronize(lfqs_state* s);
+/* n_qubits, local qubits, rank, world, and the device pointer of the local shard. */
+lfqs_status lfqs_state_info(const lfqs_state* s, int* n_qubits, int* n_local, int* rank,
+                            int* world, void** dev_ptr);
+/* Number of kernels this state has launched so far (for benchmark accounting). */
+lfqs_status lfqs_kernel_launches(const lfqs_state* s, uint64_t* count);
+/* Tuning knobs (benchmark / test use): LFQS_OPT_LOWQ_SHUFFLE (1: warp-shuffle
+ * path for targets < 5, default 1), LFQS_OPT_FUSE_TILE_QUBITS (k of the staging
+ * tile, default 12). */
+#define LFQS_OPT_LOWQ_SHUFFLE 1
+#define LFQS_OPT_FUSE_TILE_QUBITS 2
+#define LFQS_OPT_ITEMS_PER_THREAD 3
+lfqs_status lfqs_set_option(lfqs_state* s, int option, int64_t value);
+const char* lfqs_last_error(void);
+int lfqs_abi_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* LFQS_ABI_INCLUDED_ */

@@ -1,0 +1,369 @@
+"""Thin Python binding of liblfqs.so (include/lfqs.h) -- argument marshalling only.
+
+Every step of gate application, measurement and exchange runs in the CUDA
+library; this module only converts Python/numpy/torch arguments into the C ABI.
+There is no CPU fallback: if liblfqs.so is missing or no CUDA device is
+usable, calls raise :class:`LfqsError`.
+
+The module-level functions carry the C names (``lfqs_apply_gate`` ...); the
+:class:`State` class is a convenience wrapper over them.
+"""
+from __future__ import annotations
+
+import ctypes as C
+import os
+from typing import Iterable, Optional, Sequence
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "liblfqs.so")
+
+KINDS = ["I", "X", "Y", "Z", "H", "S", "SDG", "T", "TDG", "RX", "RY", "RZ", "PHASE", "U3",
+         "SWAP", "UNITARY1", "UNITARY2", "UNITARY3"]
+KIND_ID = {k: i for i, k in enumerate(KINDS)}
+NPARAMS = {k: 0 for k in KINDS}
+NPARAMS.update({"RX": 1, "RY": 1, "RZ": 1, "PHASE": 1, "U3": 3})
+
+FUSE_NONE = 0
+FUSE_LOW = 1
+OPT_LOWQ_SHUFFLE = 1
+OPT_FUSE_TILE_QUBITS = 2
+OPT_ITEMS_PER_THREAD = 3
+
+STATUS = {0: "OK", -1: "INVALID_ARG", -2: "OUT_OF_MEMORY", -3: "CUDA", -4: "NCCL",
+          -5: "UNSUPPORTED"}
+#: Every symbol include/lfqs.h declares (checked by tests/test_abi.py).
+EXPORTS = [
+    "lfqs_state_create", "lfqs_state_wrap", "lfqs_state_destroy", "lfqs_state_set_stream",
+    "lfqs_dist_unique_id", "lfqs_state_create_dist", "lfqs_state_create_virtual",
+    "lfqs_state_init_basis", "lfqs_state_init_random", "lfqs_copy_in", "lfqs_copy_out",
+    "lfqs_apply_gate", "lfqs_run_circuit", "lfqs_measure_probs", "lfqs_synchronize",
+    "lfqs_state_info", "lfqs_kernel_launches", "lfqs_set_option", "lfqs_last_error",
+    "lfqs_abi_version",
+]
+
+
+class LfqsError(RuntimeError):
+    def __init__(self, status: int, msg: str):
+        super().__init__(f"lfqs {STATUS.get(status, status)}: {msg}")
+        self.status = status
+
+
+class LfqsGate(C.Structure):
+    """Mirror of lfqs_gate (72 bytes)."""
+    _fields_ = [
+        ("kind", C.c_int32), ("n_targets", C.c_int32), ("n_controls", C.c_int32),
+        ("_pad0", C.c_int32), ("targets", C.c_int32 * 3), ("_pad1", C.c_int32),
+        ("control_mask", C.c_uint64), ("params", C.c_double * 3),
+        ("matrix", C.POINTER(C.c_double)),
+    ]
+
+
+assert C.sizeof(LfqsGate) == 72
+
+_lib = None
+
+
+def lib():
+    """Load liblfqs.so (fails loudly if the CUDA extension was not built)."""
+    global _lib
+    if _lib is None:
+        if not os.path.exists(LIB_PATH):
+            raise ImportError(f"{LIB_PATH} is missing: build it with "
+                              "`python -m paper_conf_cgo_tarabkhahdds25_b200.build`")
+        L = C.CDLL(LIB_PATH)
+        vp, dp, u64 = C.c_void_p, C.POINTER(C.c_double), C.c_uint64
+        ip = C.POINTER(C.c_int)
+        sig = {
+            "lfqs_state_create": [C.c_int, C.c_int, vp, C.POINTER(vp)],
+            "lfqs_state_wrap": [C.c_int, C.c_int, vp, vp, C.POINTER(vp)],
+            "lfqs_state_destroy": [vp],
+            "lfqs_state_set_stream": [vp, vp],
+            "lfqs_dist_unique_id": [C.POINTER(C.c_uint8)],
+            "lfqs_state_create_dist": [C.c_int, C.c_int, C.c_int, C.POINTER(C.c_uint8), C.c_int, vp,
+                                       C.POINTER(vp)],
+            "lfqs_state_create_virtual": [C.c_int, C.c_int, C.c_int, vp, C.POINTER(vp)],
+            "lfqs_state_init_basis": [vp, u64],
+            "lfqs_state_init_random": [vp, u64],
+            "lfqs_copy_in": [vp, u64, u64, dp],
+            "lfqs_copy_out": [vp, u64, u64, dp],
+            "lfqs_apply_gate": [vp, C.c_int, ip, C.c_int, ip, C.c_int, dp, C.c_int, dp],
+            "lfqs_run_circuit": [vp, C.POINTER(LfqsGate), C.c_size_t, C.c_uint32],
+            "lfqs_measure_probs": [vp, ip, C.c_int, dp, C.c_size_t],
+            "lfqs_synchronize": [vp],
+            "lfqs_state_info": [vp, ip, ip, ip, ip, C.POINTER(vp)],
+            "lfqs_kernel_launches": [vp, C.POINTER(u64)],
+            "lfqs_set_option": [vp, C.c_int, C.c_int64],
+        }
+        for name, args in sig.items():
+            f = getattr(L, name)
+            f.argtypes = args
+            f.restype = C.c_int
+        L.lfqs_last_error.restype = C.c_char_p
+        L.lfqs_last_error.argtypes = []
+        L.lfqs_abi_version.restype = C.c_int
+        L.lfqs_abi_version.argtypes = []
+        _lib = L
+    return _lib
+
+
+def _check(rc: int):
+    if rc != 0:
+        raise LfqsError(rc, lib().lfqs_last_error().decode())
+
+
+def _dp(a: np.ndarray):
+    return a.ctypes.data_as(C.POINTER(C.c_double))
+
+
+def _ints(xs: Sequence[int]):
+    xs = list(xs)
+    return (C.c_int * max(1, len(xs)))(*xs), len(xs)
+
+
+def _stream_handle(stream) -> Optional[int]:
+    """Accept None, an int handle, or a torch.cuda.Stream."""
+    if stream is None:
+        return None
+    if isinstance(stream, int):
+        return stream
+    return int(stream.cuda_stream)
+
+
+# ---- C-named thin wrappers ---------------------------------------------------
+
+def lfqs_state_create(n_qubits: int, device: int = 0, stream=None) -> int:
+    h = C.c_void_p()
+    _check(lib().lfqs_state_create(n_qubits, device, _stream_handle(stream), C.byref(h)))
+    return h.value
+
+
+def lfqs_state_wrap(n_qubits: int, device: int, dev_ptr: int, stream=None) -> int:
+    h = C.c_void_p()
+    _check(lib().lfqs_state_wrap(n_qubits, device, dev_ptr, _stream_handle(stream), C.byref(h)))
+    return h.value
+
+
+def lfqs_state_create_virtual(n_qubits: int, world: int, device: int = 0, stream=None) -> int:
+    h = C.c_void_p()
+    _check(lib().lfqs_state_create_virtual(n_qubits, world, device, _stream_handle(stream),
+                                           C.byref(h)))
+    return h.value
+
+
+def lfqs_dist_unique_id() -> bytes:
+    buf = (C.c_uint8 * 128)()
+    _check(lib().lfqs_dist_unique_id(buf))
+    return bytes(buf)
+
+
+def lfqs_state_create_dist(n_qubits: int, rank: int, world: int, uid: bytes, device: int,
+                           stream=None) -> int:
+    h = C.c_void_p()
+    buf = (C.c_uint8 * 128)(*uid)
+    _check(lib().lfqs_state_create_dist(n_qubits, rank, world, buf, device,
+                                        _stream_handle(stream), C.byref(h)))
+    return h.value
+
+
+def lfqs_state_destroy(h: int):
+    _check(lib().lfqs_state_destroy(h))
+
+
+def lfqs_state_init_basis(h: int, index: int):
+    _check(lib().lfqs_state_init_basis(h, index))
+
+
+def lfqs_state_init_random(h: int, seed: int):
+    _check(lib().lfqs_state_init_random(h, seed))
+
+
+def lfqs_copy_in(h: int, offset: int, amps: np.ndarray):
+    a = np.ascontiguousarray(amps, dtype=np.complex128)
+    _check(lib().lfqs_copy_in(h, offset, a.size, _dp(a.view(np.float64))))
+
+
+def lfqs_copy_out(h: int, offset: int, count: int, out: Optional[np.ndarray] = None) -> np.ndarray:
+    if out is None:
+        out = np.empty(count, dtype=np.complex128)
+    assert out.dtype == np.complex128 and out.flags.c_contiguous and out.size >= count
+    _check(lib().lfqs_copy_out(h, offset, count, _dp(out.view(np.float64))))
+    return out
+
+
+def _matrix_ptr(matrix, keep: list):
+    if matrix is None:
+        return None
+    m = np.ascontiguousarray(np.asarray(matrix, dtype=np.complex128))
+    keep.append(m)
+    return _dp(m.view(np.float64))
+
+
+def lfqs_apply_gate(h: int, kind, targets: Sequence[int], controls: Sequence[int] = (),
+                    params: Sequence[float] = (), matrix=None):
+    k = KIND_ID[kind] if isinstance(kind, str) else int(kind)
+    t, nt = _ints(targets)
+    c, nc = _ints(controls)
+    p = (C.c_double * max(1, len(params)))(*params)
+    keep: list = []
+    _check(lib().lfqs_apply_gate(h, k, t, nt, c, nc, p, len(params), _matrix_ptr(matrix, keep)))
+
+
+def marshal_gates(gates: Iterable):
+    """workloads.Gate-like objects -> (ctypes LfqsGate array, keep-alive list)."""
+    gates = list(gates)
+    arr = (LfqsGate * max(1, len(gates)))()
+    keep: list = []
+    for i, g in enumerate(gates):
+        o = arr[i]
+        o.kind = KIND_ID[g.kind]
+        o.n_targets = len(g.targets)
+        o.n_controls = len(g.controls)
+        for s, t in enumerate(g.targets):
+            o.targets[s] = t
+        mask = 0
+        for q in g.controls:
+            mask |= 1 << q
+        o.control_mask = mask
+        for s, x in enumerate(g.params):
+            o.params[s] = x
+        if g.matrix is not None:
+            o.matrix = _matrix_ptr(g.matrix, keep)
+    return arr, len(gates), keep
+
+
+def lfqs_run_circuit(h: int, gates, flags: int = FUSE_NONE):
+    if isinstance(gates, tuple) and len(gates) == 3 and isinstance(gates[1], int):
+        arr, n, keep = gates  # pre-marshalled
+    else:
+        arr, n, keep = marshal_gates(gates)
+    _check(lib().lfqs_run_circuit(h, arr, n, flags))
+
+
+def lfqs_measure_probs(h: int, qubits: Sequence[int] = ()) -> np.ndarray:
+    q, nq = _ints(qubits)
+    out = np.zeros(1 << nq, dtype=np.float64)
+    _check(lib().lfqs_measure_probs(h, q, nq, _dp(out), out.size))
+    return out
+
+
+def lfqs_synchronize(h: int):
+    _check(lib().lfqs_synchronize(h))
+
+
+def lfqs_state_info(h: int) -> dict:
+    n, nl, r, w = C.c_int(), C.c_int(), C.c_int(), C.c_int()
+    p = C.c_void_p()
+    _check(lib().lfqs_state_info(h, C.byref(n), C.byref(nl), C.byref(r), C.byref(w), C.byref(p)))
+    return {"n_qubits": n.value, "n_local": nl.value, "rank": r.value, "world": w.value,
+            "dev_ptr": p.value}
+
+
+def lfqs_kernel_launches(h: int) -> int:
+    c = C.c_uint64()
+    _check(lib().lfqs_kernel_launches(h, C.byref(c)))
+    return c.value
+
+
+def lfqs_set_option(h: int, option: int, value: int):
+    _check(lib().lfqs_set_option(h, option, value))
+
+
+def lfqs_state_set_stream(h: int, stream=None):
+    _check(lib().lfqs_state_set_stream(h, _stream_handle(stream)))
+
+
+# ---- convenience class ----------------------------------------------------------
+
+class State:
+    """An n-qubit complex128 state vector on a B200 (or sharded across ranks)."""
+
+    def __init__(self, handle: int, n_qubits: int):
+        self.h = handle
+        self.n = n_qubits
+
+    @classmethod
+    def create(cls, n_qubits: int, device: int = 0, stream=None) -> "State":
+        return cls(lfqs_state_create(n_qubits, device, stream), n_qubits)
+
+    @classmethod
+    def wrap(cls, tensor, stream=None) -> "State":
+        """Borrow a contiguous torch.complex128 CUDA tensor of 2^n elements."""
+        import torch
+        assert tensor.is_cuda and tensor.dtype == torch.complex128 and tensor.is_contiguous()
+        n = int(tensor.numel()).bit_length() - 1
+        assert tensor.numel() == 1 << n
+        st = cls(lfqs_state_wrap(n, tensor.device.index, tensor.data_ptr(), stream), n)
+        st._tensor = tensor
+        return st
+
+    @classmethod
+    def virtual(cls, n_qubits: int, world: int, device: int = 0, stream=None) -> "State":
+        return cls(lfqs_state_create_virtual(n_qubits, world, device, stream), n_qubits)
+
+    @classmethod
+    def distributed(cls, n_qubits: int, rank: int, world: int, uid: bytes, device: int,
+                    stream=None) -> "State":
+        return cls(lfqs_state_create_dist(n_qubits, rank, world, uid, device, stream), n_qubits)
+
+    def close(self):
+        if self.h:
+            lfqs_state_destroy(self.h)
+            self.h = None
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *exc):
+        self.close()
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    def init_basis(self, index: int = 0):
+        lfqs_state_init_basis(self.h, index)
+
+    def init_random(self, seed: int):
+        lfqs_state_init_random(self.h, seed)
+
+    def copy_in(self, amps: np.ndarray, offset: int = 0):
+        lfqs_copy_in(self.h, offset, amps)
+
+    def copy_out(self, offset: int = 0, count: Optional[int] = None, out=None) -> np.ndarray:
+        if count is None:
+            count = (1 << self.n) - offset
+        return lfqs_copy_out(self.h, offset, count, out)
+
+    def apply_gate(self, kind, targets, controls=(), params=(), matrix=None):
+        lfqs_apply_gate(self.h, kind, targets, controls, params, matrix)
+
+    def apply(self, g):
+        lfqs_apply_gate(self.h, g.kind, g.targets, g.controls, g.params, g.matrix)
+
+    def run_circuit(self, gates, fuse: bool = False):
+        lfqs_run_circuit(self.h, gates, FUSE_LOW if fuse else FUSE_NONE)
+
+    def measure_probs(self, qubits: Sequence[int] = ()) -> np.ndarray:
+        return lfqs_measure_probs(self.h, qubits)
+
+    def norm2(self) -> float:
+        return float(self.measure_probs(())[0])
+
+    def synchronize(self):
+        lfqs_synchronize(self.h)
+
+    def info(self) -> dict:
+        return lfqs_state_info(self.h)
+
+    def launches(self) -> int:
+        return lfqs_kernel_launches(self.h)
+
+    def set_option(self, option: int, value: int):
+        lfqs_set_option(self.h, option, value)
+
+    def set_stream(self, stream=None):
+        lfqs_state_set_stream(self.h, stream)

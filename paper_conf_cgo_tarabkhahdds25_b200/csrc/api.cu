@@ -1,0 +1,232 @@
+// api.cu -- the C ABI (include/lfqs.h): state lifetime, gates, circuits, measurement.
+//
+// The ABI follows the paper's statement of the problem: an n-qubit state
+// (P:93-101), a circuit G_D ... G_1 applied gate by gate (Eq. 3) with the
+// state available after each gate, updated in place in AOS
+// complex layout, then measured.
+#include <cuda_runtime.h>
+
+#include <cstdio>
+#include <cstring>
+#include <memory>
+#include <string>
+#include <vector>
+
+#include "lfqs_internal.h"
+#include "state.h"
+
+using namespace lfqs;
+
+namespace {
+thread_local std::string g_last_error;
+
+template <class F>
+lfqs_status guarded(F&& f) {
+  try {
+    f();
+    return LFQS_OK;
+  } catch (const Error& e) {
+    g_last_error = e.what();
+    return e.status;
+  } catch (const std::bad_alloc&) {
+    g_last_error = "host out of memory";
+    return LFQS_ERR_OUT_OF_MEMORY;
+  } catch (const std::exception& e) {
+    g_last_error = e.what();
+    return LFQS_ERR_INVALID_ARG;
+  } catch (...) {
+    g_last_error = "unknown error";
+    return LFQS_ERR_INVALID_ARG;
+  }
+}
+
+uint64_t mask_of(const int* qs, int nq, int n) {
+  uint64_t m = 0;
+  require(nq >= 0 && (nq == 0 || qs != nullptr), "bad control list");
+  for (int i = 0; i < nq; ++i) {
+    require(qs[i] >= 0 && qs[i] < n, "control qubit out of range");
+    require(!(m >> qs[i] & 1), "duplicate control qubit");
+    m |= 1ull << qs[i];
+  }
+  return m;
+}
+}  // namespace
+
+extern "C" {
+
+const char* lfqs_last_error(void) { return g_last_error.c_str(); }
+int lfqs_abi_version(void) { return LFQS_ABI_VERSION; }
+
+lfqs_status lfqs_state_create(int n_qubits, int device, void* stream, lfqs_state** out) {
+  return guarded([&] {
+    require(out != nullptr, "out is NULL");
+    *out = State::create_local(n_qubits, device, static_cast<cudaStream_t>(stream), nullptr);
+  });
+}
+
+lfqs_status lfqs_state_wrap(int n_qubits, int device, void* dev_ptr, void* stream,
+                            lfqs_state** out) {
+  return guarded([&] {
+    require(out != nullptr && dev_ptr != nullptr, "NULL argument");
+    require((reinterpret_cast<uintptr_t>(dev_ptr) & 15) == 0, "dev_ptr must be 16-byte aligned");
+    *out = State::create_local(n_qubits, device, static_cast<cudaStream_t>(stream), dev_ptr);
+  });
+}
+
+lfqs_status lfqs_state_create_virtual(int n_qubits, int world, int device, void* stream,
+                                      lfqs_state** out) {
+  return guarded([&] {
+    require(out != nullptr, "out is NULL");
+    *out = State::create_virtual(n_qubits, world, device, static_cast<cudaStream_t>(stream));
+  });
+}
+
+lfqs_status lfqs_dist_unique_id(uint8_t uid[128]) {
+  return guarded([&] {
+    require(uid != nullptr, "uid is NULL");
+    State::nccl_unique_id(uid);
+  });
+}
+
+lfqs_status lfqs_state_create_dist(int n_qubits, int rank, int world, const uint8_t uid[128],
+                                   int device, void* stream, lfqs_state** out) {
+  return guarded([&] {
+    require(out != nullptr && uid != nullptr, "NULL argument");
+    *out = State::create_dist(n_qubits, rank, world, uid, device, static_cast<cudaStream_t>(stream));
+  });
+}
+
+lfqs_status lfqs_state_destroy(lfqs_state* s) {
+  return guarded([&] { delete static_cast<State*>(s); });
+}
+
+lfqs_status lfqs_state_set_stream(lfqs_state* s, void* stream) {
+  return guarded([&] {
+    require(s != nullptr, "NULL state");
+    static_cast<State*>(s)->set_stream(static_cast<cudaStream_t>(stream));
+  });
+}
+
+lfqs_status lfqs_state_init_basis(lfqs_state* s, uint64_t index) {
+  return guarded([&] {
+    require(s != nullptr, "NULL state");
+    static_cast<State*>(s)->init_basis(index);
+  });
+}
+
+lfqs_status lfqs_state_init_random(lfqs_state* s, uint64_t seed) {
+  return guarded([&] {
+    require(s != nullptr, "NULL state");
+    static_cast<State*>(s)->init_random(seed);
+  });
+}
+
+lfqs_status lfqs_copy_in(lfqs_state* s, uint64_t offset, uint64_t count, const double* host) {
+  return guarded([&] {
+    require(s != nullptr && (count == 0 || host != nullptr), "NULL argument");
+    static_cast<State*>(s)->copy(offset, count, const_cast<double*>(host), /*to_device=*/true);
+  });
+}
+
+lfqs_status lfqs_copy_out(lfqs_state* s, uint64_t offset, uint64_t count, double* host) {
+  return guarded([&] {
+    require(s != nullptr && (count == 0 || host != nullptr), "NULL argument");
+    static_cast<State*>(s)->copy(offset, count, host, /*to_device=*/false);
+  });
+}
+
+lfqs_status lfqs_apply_gate(lfqs_state* s, int kind, const int* targets, int n_targets,
+                            const int* controls, int n_controls, const double* params,
+                            int n_params, const double* matrix) {
+  return guarded([&] {
+    require(s != nullptr, "NULL state");
+    State* st = static_cast<State*>(s);
+    require(n_targets >= 1 && n_targets <= 3 && targets != nullptr, "bad target list");
+    require(n_params == 0 || params != nullptr, "params is NULL");
+    const uint64_t cm = mask_of(controls, n_controls, st->n);
+    Decoded g = decode_gate(st->n, kind, targets, n_targets, cm, params, n_params, matrix);
+    st->apply(g);
+  });
+}
+
+lfqs_status lfqs_run_circuit(lfqs_state* s, const lfqs_gate* gates, size_t n_gates,
+                             uint32_t flags) {
+  return guarded([&] {
+    require(s != nullptr, "NULL state");
+    require(n_gates == 0 || gates != nullptr, "gates is NULL");
+    require((flags & ~LFQS_FUSE_LOW) == 0, "unknown flags");
+    State* st = static_cast<State*>(s);
+    std::vector<Decoded> dec;
+    dec.reserve(n_gates);
+    for (size_t i = 0; i < n_gates; ++i) {
+      const lfqs_gate& G = gates[i];
+      require(G.n_controls == __builtin_popcountll(G.control_mask),
+              "gate " + std::to_string(i) + ": n_controls != popcount(control_mask)");
+      try {
+        dec.push_back(decode_gate(st->n, G.kind, G.targets, G.n_targets, G.control_mask, G.params,
+                                  kind_nparams(G.kind), G.matrix));
+      } catch (const Error& e) {
+        throw Error(e.status, "gate " + std::to_string(i) + ": " + e.what());
+      }
+    }
+    st->run(dec, flags);
+  });
+}
+
+lfqs_status lfqs_measure_probs(lfqs_state* s, const int* qubits, int n_q, double* probs_out,
+                               size_t probs_len) {
+  return guarded([&] {
+    require(s != nullptr && probs_out != nullptr, "NULL argument");
+    State* st = static_cast<State*>(s);
+    require(n_q >= 0 && n_q <= 10, "n_q must be in [0, 10]");
+    require(probs_len >= (size_t(1) << n_q), "probs_len < 2^n_q");
+    const uint64_t qm = mask_of(qubits, n_q, st->n);
+    (void)qm;
+    st->measure_probs(qubits, n_q, probs_out);
+  });
+}
+
+lfqs_status lfqs_synchronize(lfqs_state* s) {
+  return guarded([&] {
+    require(s != nullptr, "NULL state");
+    static_cast<State*>(s)->synchronize();
+  });
+}
+
+lfqs_status lfqs_state_info(const lfqs_state* s, int* n_qubits, int* n_local, int* rank,
+                            int* world, void** dev_ptr) {
+  return guarded([&] {
+    require(s != nullptr, "NULL state");
+    const State* st = static_cast<const State*>(s);
+    if (n_qubits) *n_qubits = st->n;
+    if (n_local) *n_local = st->n_local;
+    if (rank) *rank = st->rank;
+    if (world) *world = st->world;
+    if (dev_ptr) *dev_ptr = st->shard_ptr();
+  });
+}
+
+lfqs_status lfqs_kernel_launches(const lfqs_state* s, uint64_t* count) {
+  return guarded([&] {
+    require(s != nullptr && count != nullptr, "NULL argument");
+    *count = static_cast<const State*>(s)->launches;
+  });
+}
+
+lfqs_status lfqs_set_option(lfqs_state* s, int option, int64_t value) {
+  return guarded([&] {
+    require(s != nullptr, "NULL state");
+    State* st = static_cast<State*>(s);
+    switch (option) {
+      case LFQS_OPT_LOWQ_SHUFFLE: st->opt.lowq_shuffle = value != 0; break;
+      case LFQS_OPT_FUSE_TILE_QUBITS:
+        require(value >= 6 && value <= 13, "tile qubits must be in [6, 13]");
+        st->opt.fuse_tile_qubits = (int)value;
+        break;
+      case LFQS_OPT_ITEMS_PER_THREAD: st->opt.items_per_thread = (int)value; break;
+      default: require(false, "unknown option");
+    }
+  });
+}
+
+}  // extern "C"

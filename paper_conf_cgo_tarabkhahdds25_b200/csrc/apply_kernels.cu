@@ -1,0 +1,491 @@
+// apply_kernels.cu -- sm_100a gate-application kernels.
+//
+// One pass over the changed part of the state per gate: the 2^n x 2^n matrix
+// I_L (x) M (x) I_R (Eq. 1) / Eq. 5 is never formed (vector
+// fusion); each thread expands a free index into amplitude indices by
+// bit insertion (Fig. 3b, Fig. 14: id1 = rR + 2 rL Rs,
+// id2 = id1 + Rs; Fig. 8's Ls/Gs/Rs loops P:299-306 for two targets) and
+// applies the gate's class-specialised update in place.
+//
+// B200 design: HBM-bound streaming, so
+//   * 16-byte (one complex128) vector loads/stores, 32-byte (LDG/STG.256) when
+//     a target is qubit 0 and the pair is adjacent; evict-first cache policy;
+//   * several independent groups per thread to keep >= 64 B in flight per lane;
+//   * targets below 5 optionally via warp shuffles: each warp loads 512 B
+//     contiguous per instruction and exchanges partners with shfl.xor;
+//   * diagonal gates touch only amplitudes whose factor is not 1;
+//   * the diagonal multiply is RN, no FMA (__dmul_rn/__dsub_rn/__dadd_rn) so
+//     diagonal results are value-exact against the oracle (R8).
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cstring>
+
+#include "lfqs_internal.h"
+
+namespace lfqs {
+namespace {
+
+constexpr int kThreads = 256;
+
+// ---------------------------------------------------------------------------
+// Memory helpers
+// ---------------------------------------------------------------------------
+__device__ __forceinline__ double2 ld16(const double2* p) {
+  double2 v;
+  asm volatile("ld.global.cs.v2.f64 {%0,%1}, [%2];" : "=d"(v.x), "=d"(v.y) : "l"(p));
+  return v;
+}
+__device__ __forceinline__ void st16(double2* p, double2 v) {
+  asm volatile("st.global.cs.v2.f64 [%0], {%1,%2};" ::"l"(p), "d"(v.x), "d"(v.y) : "memory");
+}
+__device__ __forceinline__ void ld32(const double2* p, double2& a, double2& b) {
+  asm volatile("ld.global.cs.v4.f64 {%0,%1,%2,%3}, [%4];"
+               : "=d"(a.x), "=d"(a.y), "=d"(b.x), "=d"(b.y)
+               : "l"(p));
+}
+__device__ __forceinline__ void st32(double2* p, double2 a, double2 b) {
+  asm volatile("st.global.cs.v4.f64 [%0], {%1,%2,%3,%4};" ::"l"(p), "d"(a.x), "d"(a.y), "d"(b.x),
+               "d"(b.y)
+               : "memory");
+}
+
+// Free index -> amplitude index (insert zero bits at ascending positions, OR ones).
+template <int NPMAX>
+__device__ __forceinline__ uint64_t expand(const InsertPlan& ip, uint64_t g) {
+#pragma unroll
+  for (int i = 0; i < NPMAX; ++i) {
+    if (i < ip.np) {
+      const int p = ip.pos[i];
+      const uint64_t lo = g & ((1ull << p) - 1);
+      g = ((g - lo) << 1) | lo;
+    }
+  }
+  return g | ip.ones;
+}
+
+// ---------------------------------------------------------------------------
+// Complex arithmetic
+// ---------------------------------------------------------------------------
+// Pinned complex multiply d*a = (dr ar - di ai, dr ai + di ar), RN, no FMA.
+__device__ __forceinline__ double2 cmul_rn(double2 d, double2 a) {
+  return make_double2(__dsub_rn(__dmul_rn(d.x, a.x), __dmul_rn(d.y, a.y)),
+                      __dadd_rn(__dmul_rn(d.x, a.y), __dmul_rn(d.y, a.x)));
+}
+// Accumulating multiply for dense gates (FMA allowed: tolerance class).
+__device__ __forceinline__ void cfma(double2& acc, double2 m, double2 v) {
+  acc.x = fma(m.x, v.x, acc.x);
+  acc.x = fma(-m.y, v.y, acc.x);
+  acc.y = fma(m.x, v.y, acc.y);
+  acc.y = fma(m.y, v.x, acc.y);
+}
+
+// ---------------------------------------------------------------------------
+// Group operators: v[0..L) = amplitudes at k + off[j] (j = local index).
+// ---------------------------------------------------------------------------
+struct OpSwap2 {  // X / CNOT / Toffoli / SWAP: moves only (bit-exact)
+  __device__ __forceinline__ void operator()(double2 (&v)[2], uint64_t) const {
+    const double2 t = v[0];
+    v[0] = v[1];
+    v[1] = t;
+  }
+};
+struct OpY {  // Y = [[0,-i],[i,0]]: v0' = -i v1, v1' = i v0 (moves + sign, exact)
+  __device__ __forceinline__ void operator()(double2 (&v)[2], uint64_t) const {
+    const double2 a0 = v[0], a1 = v[1];
+    v[0] = make_double2(a1.y, -a1.x);
+    v[1] = make_double2(-a0.y, a0.x);
+  }
+};
+struct OpH {  // hadgate, Fig. 12c / Fig. 14: sq2r*(s1+s2), sq2r*(s1-s2)
+  double s;
+  __device__ __forceinline__ void operator()(double2 (&v)[2], uint64_t) const {
+    const double2 a0 = v[0], a1 = v[1];
+    v[0] = make_double2(s * (a0.x + a1.x), s * (a0.y + a1.y));
+    v[1] = make_double2(s * (a0.x - a1.x), s * (a0.y - a1.y));
+  }
+};
+template <int L>
+struct OpDense {  // single_qbit (Fig. 12b) generalised: v' = M v
+  double2 M[L * L];
+  __device__ __forceinline__ void operator()(double2 (&v)[L], uint64_t) const {
+    double2 w[L];
+#pragma unroll
+    for (int j = 0; j < L; ++j) {
+      double2 acc = make_double2(0.0, 0.0);
+#pragma unroll
+      for (int i = 0; i < L; ++i) cfma(acc, M[j * L + i], v[i]);
+      w[j] = acc;
+    }
+#pragma unroll
+    for (int j = 0; j < L; ++j) v[j] = w[j];
+  }
+};
+// Diagonal, one touched entry per group (Z, S, T, Phase, CZ, CPhase, MC-Z).
+struct OpNeg {
+  __device__ __forceinline__ void operator()(double2 (&v)[1], uint64_t) const {
+    v[0] = make_double2(-v[0].x, -v[0].y);
+  }
+};
+struct OpMulI {  // * (0, 1): (-im, re)
+  __device__ __forceinline__ void operator()(double2 (&v)[1], uint64_t) const {
+    v[0] = make_double2(-v[0].y, v[0].x);
+  }
+};
+struct OpMulNI {  // * (0, -1): (im, -re)
+  __device__ __forceinline__ void operator()(double2 (&v)[1], uint64_t) const {
+    v[0] = make_double2(v[0].y, -v[0].x);
+  }
+};
+struct OpMul {  // * d
+  double2 d;
+  __device__ __forceinline__ void operator()(double2 (&v)[1], uint64_t) const {
+    v[0] = cmul_rn(d, v[0]);
+  }
+};
+// Diagonal, every entry touched: factor d[loc(k)] (Rz, general diagonal).
+struct OpDiagSel {
+  int m;
+  int t[3];
+  double2 d[8];
+  __device__ __forceinline__ void operator()(double2 (&v)[1], uint64_t k) const {
+    int j = 0;
+#pragma unroll
+    for (int s = 0; s < 3; ++s)
+      if (s < m) j = (j << 1) | (int)((k >> t[s]) & 1);
+    double2 dj = d[0];  // select without dynamic indexing (keeps d in the param bank)
+#pragma unroll
+    for (int i = 1; i < 8; ++i)
+      if (i == j) dj = d[i];
+    v[0] = cmul_rn(dj, v[0]);
+  }
+};
+
+template <int L>
+struct Offs {
+  uint64_t o[L];
+};
+
+// ---------------------------------------------------------------------------
+// Generic group kernel: each thread handles U groups; each group reads and
+// writes L amplitudes at k + off[j].  P256: off[2i+1] == off[2i] + 1, so the
+// pair moves as one 32-byte access.
+// ---------------------------------------------------------------------------
+template <int L, int U, bool P256, int NPMAX, class Op>
+__global__ void __launch_bounds__(kThreads) k_group(double2* __restrict__ a, uint64_t n_groups,
+                                                    const InsertPlan ip, const Offs<L> off,
+                                                    const Op op) {
+  const uint64_t g0 = (uint64_t)blockIdx.x * (kThreads * U) + threadIdx.x;
+  double2 v[U][L];
+  uint64_t kk[U];
+#pragma unroll
+  for (int u = 0; u < U; ++u) {
+    const uint64_t g = g0 + (uint64_t)u * kThreads;
+    kk[u] = expand<NPMAX>(ip, g < n_groups ? g : 0);
+    if (g < n_groups) {
+      if constexpr (P256) {
+#pragma unroll
+        for (int j = 0; j < L; j += 2) ld32(a + kk[u] + off.o[j], v[u][j], v[u][j + 1]);
+      } else {
+#pragma unroll
+        for (int j = 0; j < L; ++j) v[u][j] = ld16(a + kk[u] + off.o[j]);
+      }
+    }
+  }
+#pragma unroll
+  for (int u = 0; u < U; ++u) {
+    const uint64_t g = g0 + (uint64_t)u * kThreads;
+    if (g < n_groups) {
+      op(v[u], kk[u]);
+      if constexpr (P256) {
+#pragma unroll
+        for (int j = 0; j < L; j += 2) st32(a + kk[u] + off.o[j], v[u][j], v[u][j + 1]);
+      } else {
+#pragma unroll
+        for (int j = 0; j < L; ++j) st16(a + kk[u] + off.o[j], v[u][j]);
+      }
+    }
+  }
+}
+
+// ---------------------------------------------------------------------------
+// Low-target (t < 5) warp-shuffle kernel for 2x2-type gates.  A warp owns a
+// chunk of 32*V contiguous amplitudes; lane l holds amplitude l + 32 j of the
+// chunk; its partner for target t is lane l ^ (1 << t).
+// Controls >= 5 + log2 V are inserted into the chunk index (whole chunks are
+// skipped); controls below that are a per-lane store predicate.
+// ---------------------------------------------------------------------------
+struct LaneSwap {  // X
+  __device__ __forceinline__ double2 operator()(double2, double2 p, int) const { return p; }
+};
+struct LaneY {  // Y: bit 0 -> -i p ; bit 1 -> i p
+  __device__ __forceinline__ double2 operator()(double2, double2 p, int bit) const {
+    return bit ? make_double2(-p.y, p.x) : make_double2(p.y, -p.x);
+  }
+};
+struct LaneH {
+  double s;
+  __device__ __forceinline__ double2 operator()(double2 a, double2 p, int bit) const {
+    return bit ? make_double2(s * (p.x - a.x), s * (p.y - a.y))
+               : make_double2(s * (a.x + p.x), s * (a.y + p.y));
+  }
+};
+struct LaneDense {  // out = self[bit] * a + other[bit] * p
+  double2 self_c[2], other_c[2];
+  __device__ __forceinline__ double2 operator()(double2 a, double2 p, int bit) const {
+    double2 acc = make_double2(0.0, 0.0);
+    cfma(acc, bit ? self_c[1] : self_c[0], a);
+    cfma(acc, bit ? other_c[1] : other_c[0], p);
+    return acc;
+  }
+};
+
+template <int V, class LaneOp>
+__global__ void __launch_bounds__(kThreads) k_lowq(double2* __restrict__ a, uint64_t n_chunks,
+                                                   const InsertPlan ip_hi, uint64_t low_cmask,
+                                                   int t, const LaneOp op) {
+  constexpr int kLogV = V == 1 ? 0 : V == 2 ? 1 : V == 4 ? 2 : 3;
+  const int lane = threadIdx.x & 31;
+  const uint64_t chunk = (uint64_t)blockIdx.x * (kThreads / 32) + (threadIdx.x >> 5);
+  if (chunk >= n_chunks) return;  // warp-uniform
+  const uint64_t base = expand<kMaxInsert>(ip_hi, chunk << (5 + kLogV));
+  double2 v[V];
+#pragma unroll
+  for (int j = 0; j < V; ++j) v[j] = ld16(a + base + j * 32 + lane);
+  const int bit = (lane >> t) & 1;
+#pragma unroll
+  for (int j = 0; j < V; ++j) {
+    double2 p;
+    p.x = __shfl_xor_sync(0xffffffffu, v[j].x, 1 << t);
+    p.y = __shfl_xor_sync(0xffffffffu, v[j].y, 1 << t);
+    const uint64_t k = base + j * 32 + lane;
+    if ((k & low_cmask) == low_cmask) st16(a + k, op(v[j], p, bit));
+  }
+}
+
+// ---------------------------------------------------------------------------
+// Host launch helpers
+// ---------------------------------------------------------------------------
+InsertPlan make_plan(uint64_t zero_bits, uint64_t one_bits) {
+  InsertPlan ip;
+  std::memset(&ip, 0, sizeof ip);
+  const uint64_t all = zero_bits | one_bits;
+  for (int p = 0; p < 64; ++p)
+    if (all >> p & 1) {
+      require(ip.np < kMaxInsert, "too many fixed qubits");
+      ip.pos[ip.np++] = p;
+    }
+  ip.ones = one_bits;
+  return ip;
+}
+
+inline double2 D2(cplx z) { return make_double2(z.re, z.im); }
+
+inline uint64_t blocks_for(uint64_t items, uint64_t per_block) {
+  return (items + per_block - 1) / per_block;
+}
+
+template <int L, int U, bool P256, class Op>
+void run_group(const LaunchCtx& ctx, uint64_t n_groups, const InsertPlan& ip, const Offs<L>& off,
+               const Op& op) {
+  if (n_groups == 0) return;
+  const uint64_t nb = blocks_for(n_groups, (uint64_t)kThreads * U);
+  require(nb < (1ull << 31), "grid too large");
+  auto* a = reinterpret_cast<double2*>(ctx.amps);
+  if (ip.np <= 4)
+    k_group<L, U, P256, 4, Op><<<(unsigned)nb, kThreads, 0, ctx.stream>>>(a, n_groups, ip, off, op);
+  else
+    k_group<L, U, P256, kMaxInsert, Op>
+        <<<(unsigned)nb, kThreads, 0, ctx.stream>>>(a, n_groups, ip, off, op);
+  LFQS_CUDA_CHECK(cudaGetLastError());
+  ++*ctx.launch_counter;
+}
+
+template <class LaneOp>
+void run_lowq(const LaunchCtx& ctx, int t, uint64_t cmask, const LaneOp& op) {
+  constexpr int V = 4, kLogV = 2;
+  constexpr int CB = 5 + kLogV;
+  const uint64_t hi_c = cmask & ~((1ull << CB) - 1), lo_c = cmask & ((1ull << CB) - 1);
+  const InsertPlan ip = make_plan(0, hi_c);
+  const int n_hi = __builtin_popcountll(hi_c);
+  const uint64_t n_chunks = 1ull << (ctx.n_local - CB - n_hi);
+  const uint64_t nb = blocks_for(n_chunks, kThreads / 32);
+  require(nb < (1ull << 31), "grid too large");
+  k_lowq<V, LaneOp><<<(unsigned)nb, kThreads, 0, ctx.stream>>>(
+      reinterpret_cast<double2*>(ctx.amps), n_chunks, ip, lo_c, t, op);
+  LFQS_CUDA_CHECK(cudaGetLastError());
+  ++*ctx.launch_counter;
+}
+
+// 2-amplitude (pair) gate on target t with controls: X, Y, dense 2x2.
+template <class Op, class LaneOp>
+void launch_pair(const LaunchCtx& ctx, const Decoded& g, const Op& op, const LaneOp& lane_op) {
+  const int t = g.targets[0];
+  const int nc = __builtin_popcountll(g.cmask);
+  constexpr int kCB = 7;
+  if (ctx.opt->lowq_shuffle && t < 5 && ctx.n_local >= kCB + __builtin_popcountll(g.cmask >> kCB)) {
+    run_lowq(ctx, t, g.cmask, lane_op);
+    return;
+  }
+  const uint64_t n_groups = 1ull << (ctx.n_local - 1 - nc);
+  const InsertPlan ip = make_plan(1ull << t, g.cmask);
+  Offs<2> off{{0ull, 1ull << t}};
+  if (t == 0)
+    run_group<2, 4, true>(ctx, n_groups, ip, off, op);
+  else
+    run_group<2, 4, false>(ctx, n_groups, ip, off, op);
+}
+
+// Local-index offsets: off[j] = sum_s bit(m-1-s of j) << t_s (reading R2).
+template <int L>
+Offs<L> group_offsets(const int* t, int m) {
+  Offs<L> off;
+  for (int j = 0; j < L; ++j) {
+    uint64_t o = 0;
+    for (int s = 0; s < m; ++s) o |= (uint64_t)((j >> (m - 1 - s)) & 1) << t[s];
+    off.o[j] = o;
+  }
+  return off;
+}
+
+// Reorder a 2^m matrix so that its targets are listed in a new order `perm`
+// (new target s = old target perm[s]); exact (entries only move).
+void permute_targets(const Decoded& g, const int* perm, int* t_new, cplx* M_new) {
+  const int m = g.m, d = 1 << m;
+  for (int s = 0; s < m; ++s) t_new[s] = g.targets[perm[s]];
+  auto old_index = [&](int jn) {
+    int jo = 0;
+    for (int s = 0; s < m; ++s) {
+      const int b = (jn >> (m - 1 - s)) & 1;  // bit of new target s
+      jo |= b << (m - 1 - perm[s]);
+    }
+    return jo;
+  };
+  for (int r = 0; r < d; ++r)
+    for (int c = 0; c < d; ++c) M_new[r * d + c] = g.M[old_index(r) * d + old_index(c)];
+}
+
+template <int L>
+void launch_dense_m(const LaunchCtx& ctx, const Decoded& g) {
+  constexpr int m = L == 4 ? 2 : 3;
+  // Put qubit 0 (if a target) last, so amplitude pairs (k, k+1) are adjacent
+  // and move as 32-byte accesses.
+  int perm[3] = {0, 1, 2};
+  for (int s = 0; s < m; ++s)
+    if (g.targets[s] == 0) std::swap(perm[s], perm[m - 1]);
+  int t[3];
+  OpDense<L> op;
+  cplx Mp[64];
+  permute_targets(g, perm, t, Mp);
+  for (int i = 0; i < L * L; ++i) op.M[i] = D2(Mp[i]);
+  uint64_t tmask = 0;
+  for (int s = 0; s < m; ++s) tmask |= 1ull << t[s];
+  const int nc = __builtin_popcountll(g.cmask);
+  const uint64_t n_groups = 1ull << (ctx.n_local - m - nc);
+  const InsertPlan ip = make_plan(tmask, g.cmask);
+  const Offs<L> off = group_offsets<L>(t, m);
+  if (t[m - 1] == 0)
+    run_group<L, (L == 4 ? 2 : 1), true>(ctx, n_groups, ip, off, op);
+  else
+    run_group<L, (L == 4 ? 2 : 1), false>(ctx, n_groups, ip, off, op);
+}
+
+void launch_diag(const LaunchCtx& ctx, const Decoded& g) {
+  const int m = g.m, d = 1 << m;
+  // Entries != 1 (the only amplitudes that change).
+  int n_active = 0, active = -1;
+  for (int j = 0; j < d; ++j) {
+    const cplx z = g.M[j * d + j];
+    if (!(z.re == 1.0 && z.im == 0.0)) {
+      ++n_active;
+      active = j;
+    }
+  }
+  if (n_active == 0) return;
+  const int nc = __builtin_popcountll(g.cmask);
+  uint64_t tmask = 0;
+  for (int s = 0; s < m; ++s) tmask |= 1ull << g.targets[s];
+  if (n_active == 1) {
+    // Touch only amplitudes with target bits = active pattern and controls = 1.
+    uint64_t pattern = 0;
+    for (int s = 0; s < m; ++s) pattern |= (uint64_t)((active >> (m - 1 - s)) & 1) << g.targets[s];
+    const InsertPlan ip = make_plan(tmask & ~pattern, g.cmask | pattern);
+    const uint64_t n_groups = 1ull << (ctx.n_local - m - nc);
+    const cplx z = g.M[active * d + active];
+    Offs<1> off{{0}};
+    if (z.re == -1.0 && z.im == 0.0)
+      run_group<1, 4, false>(ctx, n_groups, ip, off, OpNeg{});
+    else if (z.re == 0.0 && z.im == 1.0)
+      run_group<1, 4, false>(ctx, n_groups, ip, off, OpMulI{});
+    else if (z.re == 0.0 && z.im == -1.0)
+      run_group<1, 4, false>(ctx, n_groups, ip, off, OpMulNI{});
+    else
+      run_group<1, 4, false>(ctx, n_groups, ip, off, OpMul{D2(z)});
+    return;
+  }
+  OpDiagSel op;
+  op.m = m;
+  for (int s = 0; s < 3; ++s) op.t[s] = s < m ? g.targets[s] : 0;
+  for (int j = 0; j < 8; ++j) op.d[j] = j < d ? D2(g.M[j * d + j]) : make_double2(1, 0);
+  const InsertPlan ip = make_plan(0, g.cmask);
+  const uint64_t n_groups = 1ull << (ctx.n_local - nc);
+  run_group<1, 4, false>(ctx, n_groups, ip, Offs<1>{{0}}, op);
+}
+
+}  // namespace
+
+// Virtual-partition exchange: swap the l=1 half of this shard with the l=0 half
+// of the shard `partner_offset_amps` amplitudes further on (same pass structure
+// as a SWAP gate).
+void launch_half_swap(const LaunchCtx& ctx, int l, uint64_t partner_offset_amps) {
+  const InsertPlan ip = make_plan(1ull << l, 0);
+  Offs<2> off{{1ull << l, partner_offset_amps}};
+  run_group<2, 4, false>(ctx, 1ull << (ctx.n_local - 1), ip, off, OpSwap2{});
+}
+
+void launch_gate(const LaunchCtx& ctx, const Decoded& g) {
+  switch (g.cls) {
+    case GClass::NOOP:
+      return;
+    case GClass::DIAG:
+      launch_diag(ctx, g);
+      return;
+    case GClass::PERM_X:
+      launch_pair(ctx, g, OpSwap2{}, LaneSwap{});
+      return;
+    case GClass::PERM_Y:
+      launch_pair(ctx, g, OpY{}, LaneY{});
+      return;
+    case GClass::PERM_SWAP: {
+      const int t0 = g.targets[0], t1 = g.targets[1];
+      const int nc = __builtin_popcountll(g.cmask);
+      const InsertPlan ip = make_plan((1ull << t0) | (1ull << t1), g.cmask);
+      Offs<2> off{{1ull << t0, 1ull << t1}};
+      run_group<2, 4, false>(ctx, 1ull << (ctx.n_local - 2 - nc), ip, off, OpSwap2{});
+      return;
+    }
+    case GClass::DENSE:
+      if (g.m == 1) {
+        if (g.is_h) {
+          const double s = g.M[0].re;
+          launch_pair(ctx, g, OpH{s}, LaneH{s});
+        } else {
+          OpDense<2> op;
+          for (int i = 0; i < 4; ++i) op.M[i] = D2(g.M[i]);
+          LaneDense lop;
+          lop.self_c[0] = D2(g.M[0]);   // u00
+          lop.self_c[1] = D2(g.M[3]);   // u11
+          lop.other_c[0] = D2(g.M[1]);  // u01
+          lop.other_c[1] = D2(g.M[2]);  // u10
+          launch_pair(ctx, g, op, lop);
+        }
+      } else if (g.m == 2) {
+        launch_dense_m<4>(ctx, g);
+      } else {
+        launch_dense_m<8>(ctx, g);
+      }
+      return;
+  }
+}
+
+}  // namespace lfqs

@@ -1,0 +1,97 @@
+// comm.cu -- global-qubit exchange and reductions across GPUs over NCCL.
+//
+// No multi-GPU component exists in the paper (single node OpenMP or one GPU,
+// P:551); this is the B200 sharding that BASELINE.json's north_star asks
+// for.  A gate whose target is a global qubit g is made local by swapping g with
+// a local qubit l: rank r (global bit b) and its partner r ^ 2^(g - n_local)
+// exchange the half-shard whose l-bit is 1 - b (16 * 2^(n_local-1) bytes each
+// way).  The transfer is chunked through two staging buffers on a dedicated
+// communication stream; each landed chunk is copied into place on the compute
+// stream while the next chunk is in flight (events hand buffers back and forth).
+#include <cuda_runtime.h>
+#include <nccl.h>
+
+#include <algorithm>
+#include <cstring>
+#include <string>
+
+#include "comm.h"
+
+namespace lfqs {
+
+#define LFQS_NCCL_CHECK(expr)                                                                \
+  do {                                                                                       \
+    ncclResult_t _r = (expr);                                                                \
+    if (_r != ncclSuccess)                                                                   \
+      throw ::lfqs::Error(LFQS_ERR_NCCL, std::string(#expr) + ": " + ncclGetErrorString(_r)); \
+  } while (0)
+
+static_assert(sizeof(ncclUniqueId) == 128, "ncclUniqueId must be 128 bytes");
+
+void Comm::unique_id(uint8_t uid[128]) {
+  ncclUniqueId id;
+  LFQS_NCCL_CHECK(ncclGetUniqueId(&id));
+  std::memcpy(uid, &id, 128);
+}
+
+Comm::Comm(int rank_, int world_, const uint8_t uid[128], size_t stage_bytes)
+    : rank(rank_), world(world_) {
+  ncclUniqueId id;
+  std::memcpy(&id, uid, 128);
+  LFQS_NCCL_CHECK(ncclCommInitRank(&comm, world, id, rank));
+  LFQS_CUDA_CHECK(cudaStreamCreateWithFlags(&cstream, cudaStreamNonBlocking));
+  stage_amps = stage_bytes / 16;
+  for (int i = 0; i < 2; ++i) {
+    LFQS_CUDA_CHECK(cudaMalloc(&stage[i], stage_amps * 16));
+    LFQS_CUDA_CHECK(cudaEventCreateWithFlags(&ev_recv[i], cudaEventDisableTiming));
+    LFQS_CUDA_CHECK(cudaEventCreateWithFlags(&ev_free[i], cudaEventDisableTiming));
+  }
+  LFQS_CUDA_CHECK(cudaEventCreateWithFlags(&ev_start, cudaEventDisableTiming));
+  LFQS_CUDA_CHECK(cudaMalloc(&d_reduce, 8 * 1024));
+}
+
+Comm::~Comm() {
+  cudaStreamSynchronize(cstream);
+  for (int i = 0; i < 2; ++i) {
+    cudaFree(stage[i]);
+    cudaEventDestroy(ev_recv[i]);
+    cudaEventDestroy(ev_free[i]);
+  }
+  cudaEventDestroy(ev_start);
+  cudaFree(d_reduce);
+  cudaStreamDestroy(cstream);
+  ncclCommDestroy(comm);
+}
+
+// Exchanges the amplitudes at `pieces` (offset, count in amplitudes, in this
+// rank's shard) with the same pieces of `partner`, in place.
+void Comm::exchange(double* shard, const std::vector<Piece>& pieces, int partner,
+                    cudaStream_t compute) {
+  // The comm stream must see every kernel already queued on the compute stream.
+  LFQS_CUDA_CHECK(cudaEventRecord(ev_start, compute));
+  LFQS_CUDA_CHECK(cudaStreamWaitEvent(cstream, ev_start, 0));
+  int c = 0;
+  for (const Piece& pc : pieces) {
+    for (uint64_t off = 0; off < pc.count; off += stage_amps) {
+      const uint64_t cnt = std::min<uint64_t>(stage_amps, pc.count - off);
+      const int b = c & 1;
+      if (c >= 2) LFQS_CUDA_CHECK(cudaStreamWaitEvent(cstream, ev_free[b], 0));
+      double* src = shard + 2 * (pc.offset + off);
+      LFQS_NCCL_CHECK(ncclGroupStart());
+      LFQS_NCCL_CHECK(ncclSend(src, 2 * cnt, ncclDouble, partner, comm, cstream));
+      LFQS_NCCL_CHECK(ncclRecv(stage[b], 2 * cnt, ncclDouble, partner, comm, cstream));
+      LFQS_NCCL_CHECK(ncclGroupEnd());
+      LFQS_CUDA_CHECK(cudaEventRecord(ev_recv[b], cstream));
+      LFQS_CUDA_CHECK(cudaStreamWaitEvent(compute, ev_recv[b], 0));
+      LFQS_CUDA_CHECK(cudaMemcpyAsync(src, stage[b], cnt * 16, cudaMemcpyDeviceToDevice, compute));
+      LFQS_CUDA_CHECK(cudaEventRecord(ev_free[b], compute));
+      ++c;
+    }
+  }
+}
+
+void Comm::allreduce_sum(double* d, size_t count, cudaStream_t s) {
+  LFQS_NCCL_CHECK(ncclAllReduce(d, d, count, ncclDouble, ncclSum, comm, s));
+}
+
+}  // namespace lfqs

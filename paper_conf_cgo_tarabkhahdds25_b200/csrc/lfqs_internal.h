@@ -1,0 +1,114 @@
+// lfqs_internal.h -- internal types of the B200 LFQS library (not part of the ABI).
+//
+// Citations: "P:N" = PAPER.md line N (Tarabkhah et al., CGO'25).
+#pragma once
+#include <cuda_runtime.h>
+
+#include <cstdint>
+#include <stdexcept>
+#include <string>
+#include <vector>
+
+#include "../../include/lfqs.h"
+
+namespace lfqs {
+
+// Thrown inside the library, converted to lfqs_status at the ABI boundary.
+struct Error : std::runtime_error {
+  lfqs_status status;
+  Error(lfqs_status s, const std::string& m) : std::runtime_error(m), status(s) {}
+};
+
+#define LFQS_CUDA_CHECK(expr)                                                              \
+  do {                                                                                     \
+    cudaError_t _e = (expr);                                                               \
+    if (_e != cudaSuccess)                                                                 \
+      throw ::lfqs::Error(LFQS_ERR_CUDA, std::string(#expr) + ": " + cudaGetErrorString(_e)); \
+  } while (0)
+
+inline void require(bool ok, const std::string& msg) {
+  if (!ok) throw Error(LFQS_ERR_INVALID_ARG, msg);
+}
+
+struct cplx {
+  double re, im;
+};
+
+// ---------------------------------------------------------------------------
+// Host-side gate decode (a1 in SURVEY §8(a)): kind -> matrix and sparsity class,
+// the static matrix specialisation of P:441-445.
+// ---------------------------------------------------------------------------
+enum class GClass : int {
+  NOOP,       // identity (I, or a diagonal of ones)
+  DIAG,       // diagonal: a[k] *= d[loc(k)]          (Z, S, T, Rz, Phase, CZ, CPhase, MC-Z)
+  PERM_X,     // pair swap                             (X, CNOT, Toffoli)
+  PERM_Y,     // pair swap with +-i                    (Y)
+  PERM_SWAP,  // exchange a[k|2^t0] <-> a[k|2^t1]      (SWAP)
+  DENSE       // 2^m x 2^m matvec per group            (H, Rx, Ry, U3, UNITARYm)
+};
+
+struct Decoded {
+  int kind = 0;
+  int m = 1;                 // number of targets
+  int targets[3] = {0, 0, 0};// targets[0] = MSB of the local index (reading R2)
+  uint64_t cmask = 0;        // control mask
+  GClass cls = GClass::DENSE;
+  bool is_h = false;         // Hadamard: sq2r*(s1 +- s2) (Fig. 12c / Fig. 14)
+  cplx M[64];                // 2^m x 2^m row-major
+};
+
+// Validates and decodes one gate; throws Error(INVALID_ARG) on bad input.
+Decoded decode_gate(int n, int kind, const int* targets, int n_targets, uint64_t cmask,
+                    const double* params, int n_params, const double* matrix);
+int kind_arity(int kind);
+int kind_nparams(int kind);
+
+// ---------------------------------------------------------------------------
+// Kernel-side parameter blocks (passed by value)
+// ---------------------------------------------------------------------------
+constexpr int kMaxInsert = 40;
+
+// Free index -> amplitude index: insert a 0 bit at each pos[] (ascending), then
+// OR `ones` (Fig. 3b, Fig. 14 id1 = rR + 2 rL Rs, generalised
+// to several inserted bits: Fig. 8's three loops Ls/Gs/Rs).
+struct InsertPlan {
+  int np;
+  int pos[kMaxInsert];
+  uint64_t ones;
+};
+
+struct Options {
+  bool lowq_shuffle = true;
+  int fuse_tile_qubits = 12;
+  int items_per_thread = 0;  // 0 = library default
+};
+
+// One launch worth of work on a contiguous shard.
+struct LaunchCtx {
+  double* amps;            // interleaved complex128 shard
+  int n_local;             // qubits in the shard
+  cudaStream_t stream;
+  uint64_t* launch_counter;
+  const Options* opt;
+};
+
+// Applies one decoded gate whose targets are all < n_local (controls < n_local).
+void launch_gate(const LaunchCtx& ctx, const Decoded& g);
+
+// Diagonal-only fast path with an extra rank-constant mask: amplitudes whose
+// `global_ones` bits are implied by the rank.  Used by the distributed runner.
+// Fused low-qubit program; returns false if not applicable.
+struct FusedOp;
+void launch_fused(const LaunchCtx& ctx, const std::vector<Decoded>& gates, int tile_qubits);
+bool fusable(const Decoded& g, int tile_qubits, int n_local);
+
+// Reductions (C9): out[v], v < 2^nq; deterministic.
+void launch_probs(const LaunchCtx& ctx, const int* qubits, int nq, double* d_partials,
+                  int n_partials_blocks, double* d_out);
+int probs_blocks();
+
+// Initialisers.
+void launch_init_basis(const LaunchCtx& ctx, int64_t local_index);  // -1: all zero
+void launch_init_random(const LaunchCtx& ctx, uint64_t seed, uint64_t global_offset);
+
+}  // namespace lfqs

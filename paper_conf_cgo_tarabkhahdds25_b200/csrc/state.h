@@ -1,0 +1,72 @@
+// state.h -- the state allocator, qubit map and distributed planner.
+#pragma once
+#include <cuda_runtime.h>
+
+#include <cstdint>
+#include <vector>
+
+#include "lfqs_internal.h"
+
+struct lfqs_state {
+  virtual ~lfqs_state() = default;
+};
+
+namespace lfqs {
+
+struct Comm;  // NCCL communicator wrapper (comm.cu)
+
+// Layout in HBM: a shard is 2^n_local interleaved complex128
+// amplitudes, contiguous, 256-byte aligned.  Physical bit positions
+// [0, n_local) are local; [n_local, n) are "global" and equal the rank's bits.
+// l2p maps a logical qubit to its physical position (identity on one GPU).
+struct State : lfqs_state {
+  int n = 0, n_local = 0, rank = 0, world = 1, p = 0, device = 0;
+  bool virt = false;            // `world` shards in one allocation (single GPU)
+  double* amps = nullptr;       // shard 0 (virtual: all shards back to back)
+  bool owned = false;
+  cudaStream_t stream = nullptr;
+  bool own_stream = false;
+  uint64_t launches = 0;
+  Options opt;
+  double* d_partials = nullptr; // reduction scratch
+  double* d_probs = nullptr;
+  int l2p[64], p2l[64];
+  Comm* comm = nullptr;
+  // exchange statistics (benchmark accounting)
+  uint64_t exchanges = 0, exchange_bytes = 0;
+
+  static State* create_local(int n, int device, cudaStream_t stream, void* borrowed);
+  static State* create_virtual(int n, int world, int device, cudaStream_t stream);
+  static State* create_dist(int n, int rank, int world, const uint8_t uid[128], int device,
+                            cudaStream_t stream);
+  static void nccl_unique_id(uint8_t uid[128]);
+  ~State() override;
+
+  void set_stream(cudaStream_t s);
+  void init_basis(uint64_t index);
+  void init_random(uint64_t seed);
+  void copy(uint64_t offset, uint64_t count, double* host, bool to_device);
+  void apply(const Decoded& g);
+  void run(const std::vector<Decoded>& gates, uint32_t flags);
+  void measure_probs(const int* qubits, int nq, double* out);
+  void synchronize();
+  void* shard_ptr() const { return amps; }
+
+ private:
+  State() = default;
+  void common_init(int n_, int world_, int device_, cudaStream_t s);
+  LaunchCtx ctx(int shard);
+  int n_shards() const { return virt ? world : 1; }
+  int rank_of_shard(int shard) const { return virt ? shard : rank; }
+  bool identity_map() const;
+  void reset_map();
+  Decoded to_physical(const Decoded& g) const;
+  bool rank_local(const Decoded& pg, int r, Decoded* out) const;
+  void ensure_local_targets(Decoded& pg);
+  void exchange(int l, int g);   // swap physical positions l (local) and g (global)
+  void swap_local(int a, int b); // swap two local physical positions (data)
+  void canonicalize();
+  void apply_physical(const Decoded& pg);
+};
+
+}  // namespace lfqs

@@ -1,0 +1,65 @@
+"""The C-ABI library loads and exports every symbol include/lfqs.h declares (no GPU needed)."""
+import ctypes as C
+import os
+import re
+
+import pytest
+
+import paper_conf_cgo_tarabkhahdds25_b200 as L
+from paper_conf_cgo_tarabkhahdds25_b200 import build as B
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+HEADER = os.path.join(ROOT, "include", "lfqs.h")
+
+
+def declared_functions():
+    src = open(HEADER).read()
+    src = re.sub(r"/\*.*?\*/", "", src, flags=re.S)
+    return sorted(set(re.findall(r"\b(lfqs_\w+)\s*\(", src)))
+
+
+@pytest.fixture(scope="module")
+def lib():
+    B.build()
+    return L.lib()
+
+
+def test_header_declares_the_binding_exports():
+    assert declared_functions() == sorted(L.EXPORTS)
+
+
+def test_library_exports_every_declared_symbol(lib):
+    for name in declared_functions():
+        assert hasattr(lib, name), name
+
+
+def test_abi_version_and_struct_layout(lib):
+    assert lib.lfqs_abi_version() == 1
+    assert C.sizeof(L.LfqsGate) == 72
+    assert L.LfqsGate.control_mask.offset == 32
+    assert L.LfqsGate.matrix.offset == 64
+
+
+def test_kernels_are_sm100a(lib):
+    """The .so carries sm_100a SASS (cross-compiled here; no GPU needed)."""
+    import subprocess
+    out = subprocess.run(["/usr/local/cuda/bin/cuobjdump", "--list-elf", L.LIB_PATH],
+                         capture_output=True, text=True).stdout
+    assert "sm_100a" in out
+
+
+def test_no_device_fails_loudly(lib):
+    """Without a GPU every call that needs one returns LFQS_ERR_CUDA -- never a CPU fallback."""
+    import torch
+    if torch.cuda.is_available():
+        pytest.skip("a GPU is present")
+    with pytest.raises(L.LfqsError) as e:
+        L.State.create(4)
+    assert e.value.status == -3
+
+
+def test_null_handle_is_rejected(lib):
+    with pytest.raises(L.LfqsError) as e:
+        L.lfqs_synchronize(None)
+    assert e.value.status == -1
+    assert b"NULL" in lib.lfqs_last_error()
