@@ -223,7 +223,8 @@ def main():
     assert world == args.gpus, f"--gpus {args.gpus} but WORLD_SIZE={world}"
     assert args.warmup >= 3 or os.environ.get("LFQS_BENCH_ALLOW_SHORT"), "need >= 3 warm-up steps"
     torch.cuda.set_device(local_rank)
-    stream = torch.cuda.current_stream()
+    stream = torch.cuda.Stream()      # the library launches on this stream; events too
+    torch.cuda.set_stream(stream)
     dist = None
     if world > 1:
         import torch.distributed as dist

@@ -122,13 +122,19 @@ def _ints(xs: Sequence[int]):
     return (C.c_int * max(1, len(xs)))(*xs), len(xs)
 
 
+CUDA_STREAM_LEGACY = 0x1  # cudaStreamLegacy
+
+
 def _stream_handle(stream) -> Optional[int]:
-    """Accept None, an int handle, or a torch.cuda.Stream."""
+    """Accept None (library-owned stream), an int handle, or a torch.cuda.Stream.
+
+    torch's default stream has handle 0; it is passed as cudaStreamLegacy so that
+    the library's work is ordered with torch's (a NULL handle would mean "make
+    your own stream")."""
     if stream is None:
         return None
-    if isinstance(stream, int):
-        return stream
-    return int(stream.cuda_stream)
+    h = stream if isinstance(stream, int) else int(stream.cuda_stream)
+    return h if h != 0 else CUDA_STREAM_LEGACY
 
 
 # ---- C-named thin wrappers ---------------------------------------------------

@@ -52,7 +52,7 @@ def test_global_qubit_cases(L, world):
     targets (remap), SWAP(global, local) relabel, canonicalisation at copy-out."""
     n = 10
     p = world.bit_length() - 1
-    hi = list(range(n - p, n))
+    hi = list(range(n - p, n)) if p > 1 else [n - 1, n - 2]  # n-2 is local when p = 1
     psi = W.random_state(n, 5)
     gates = [
         W.Gate("H", (hi[-1],)), W.CNOT(hi[0], 2), W.CZ(hi[-1], 3), W.CPHASE(1, hi[0], 0.7),

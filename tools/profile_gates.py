@@ -1,0 +1,81 @@
+"""Launch a few representative gates for ncu / quick per-gate timing.
+
+    python tools/profile_gates.py --n 28 --reps 3 [--time] [--no-shuffle]
+        [--gates H:2,H:20,X:0,Z:15,RZ:3,SWAP:1/20,U2:0/7,CX:1/0,CCX:1/2/5,U3q:0/4/9]
+
+Gate spec: KIND:t (1 target), U2:a/b, U3q:a/b/c, SWAP:a/b, CX:c/t, CCX:c1/c2/t, CZ:c/t.
+With --time, prints per-gate mean ms and algorithmic GB/s from CUDA events.
+"""
+import argparse
+import math
+import os
+import sys
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+
+import workloads as W  # noqa: E402
+
+DEFAULT = "H:2,H:20,X:0,X:3,X:20,Z:15,T:0,RZ:3,SWAP:1/20,U2:0/7,U2:20/25,CX:1/0,CCX:1/2/5,U3q:0/4/9"
+
+
+def parse(spec, n):
+    out = []
+    for tok in spec.split(","):
+        k, a = tok.split(":")
+        q = [int(x) for x in a.split("/")]
+        if k == "U2":
+            out.append(W.Gate("UNITARY2", tuple(q), (), (), W.haar_unitary(2, 1)))
+        elif k == "U3q":
+            out.append(W.Gate("UNITARY3", tuple(q), (), (), W.haar_unitary(3, 2)))
+        elif k == "SWAP":
+            out.append(W.Gate("SWAP", tuple(q)))
+        elif k == "CX":
+            out.append(W.CNOT(q[0], q[1]))
+        elif k == "CZ":
+            out.append(W.CZ(q[0], q[1]))
+        elif k == "CCX":
+            out.append(W.TOFFOLI(q[0], q[1], q[2]))
+        else:
+            out.append(W.Gate(k, (q[0],), (), tuple(0.3 + i for i in range(W.NPARAMS[k]))))
+    return out
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--n", type=int, default=28)
+    ap.add_argument("--reps", type=int, default=3)
+    ap.add_argument("--gates", default=DEFAULT)
+    ap.add_argument("--time", action="store_true")
+    ap.add_argument("--no-shuffle", action="store_true")
+    args = ap.parse_args()
+    import torch
+    import paper_conf_cgo_tarabkhahdds25_b200 as L
+    s = torch.cuda.Stream()
+    torch.cuda.set_stream(s)
+    gates = parse(args.gates, args.n)
+    with L.State.create(args.n, 0, stream=s) as st:
+        st.set_option(L.OPT_LOWQ_SHUFFLE, 0 if args.no_shuffle else 1)
+        st.init_random(7)
+        for g in gates:
+            st.apply(g)  # warm-up
+        torch.cuda.synchronize()
+        for g in gates:
+            ev = [torch.cuda.Event(enable_timing=True) for _ in range(args.reps + 1)]
+            for r in range(args.reps):
+                ev[r].record(s)
+                st.apply(g)
+            ev[-1].record(s)
+            torch.cuda.synchronize()
+            if args.time:
+                ms = [ev[r].elapsed_time(ev[r + 1]) for r in range(args.reps)]
+                alg = 32.0 * W.touched_amplitudes(g, args.n)
+                print(f"{g.label():28s} mean {np.mean(ms):8.3f} ms  min {np.min(ms):8.3f} ms  "
+                      f"alg {alg / np.min(ms) / 1e6:8.1f} GB/s  conv {32 * 2 ** args.n / np.min(ms) / 1e6:8.1f} GB/s",
+                      flush=True)
+
+
+if __name__ == "__main__":
+    main()
