@@ -224,6 +224,7 @@ lfqs_status lfqs_set_option(lfqs_state* s, int option, int64_t value) {
         st->opt.fuse_tile_qubits = (int)value;
         break;
       case LFQS_OPT_ITEMS_PER_THREAD: st->opt.items_per_thread = (int)value; break;
+      case LFQS_OPT_WIDE256: st->opt.wide256 = value != 0; break;
       default: require(false, "unknown option");
     }
   });

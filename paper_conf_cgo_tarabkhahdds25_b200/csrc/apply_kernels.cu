@@ -143,21 +143,47 @@ struct OpMul {  // * d
     v[0] = cmul_rn(d, v[0]);
   }
 };
-// Diagonal, every entry touched: factor d[loc(k)] (Rz, general diagonal).
-struct OpDiagSel {
-  int m;
-  int t[3];
-  double2 d[8];
-  __device__ __forceinline__ void operator()(double2 (&v)[1], uint64_t k) const {
-    int j = 0;
+// Diagonal over a whole group: v[j] *= d[j] (Rz, general diagonals; no selects).
+template <int L>
+struct OpDiagGroup {
+  double2 d[L];
+  uint32_t touch;  // bit j set: d[j] != 1
+  __device__ __forceinline__ void operator()(double2 (&v)[L], uint64_t) const {
 #pragma unroll
-    for (int s = 0; s < 3; ++s)
-      if (s < m) j = (j << 1) | (int)((k >> t[s]) & 1);
-    double2 dj = d[0];  // select without dynamic indexing (keeps d in the param bank)
-#pragma unroll
-    for (int i = 1; i < 8; ++i)
-      if (i == j) dj = d[i];
-    v[0] = cmul_rn(dj, v[0]);
+    for (int j = 0; j < L; ++j)
+      if (touch >> j & 1) v[j] = cmul_rn(d[j], v[j]);
+  }
+};
+// A one-amplitude op applied to element `which` of an adjacent pair (bit 0 fixed by
+// a control or diagonal pattern): the pair moves as one 32-byte sector so no
+// sub-sector (16 B) writes reach L2/DRAM.
+template <class Op1>
+struct OpAtPair {
+  Op1 op;
+  int which;
+  __device__ __forceinline__ void operator()(double2 (&v)[2], uint64_t k) const {
+    double2 t[1];
+    if (which) {
+      t[0] = v[1];
+      op(t, k);
+      v[1] = t[0];
+    } else {
+      t[0] = v[0];
+      op(t, k);
+      v[0] = t[0];
+    }
+  }
+};
+// A pair op with a control on qubit 0: group (k, k+1, k+2^t, k+2^t+1), the op acts
+// on (v1, v3); all four move as two 32-byte sectors.
+template <class Op2>
+struct OpCtrl0 {
+  Op2 op;
+  __device__ __forceinline__ void operator()(double2 (&v)[4], uint64_t k) const {
+    double2 p[2] = {v[1], v[3]};
+    op(p, k | 1);
+    v[1] = p[0];
+    v[3] = p[1];
   }
 };
 
@@ -204,6 +230,37 @@ __global__ void __launch_bounds__(kThreads) k_group(double2* __restrict__ a, uin
 #pragma unroll
         for (int j = 0; j < L; ++j) st16(a + kk[u] + off.o[j], v[u][j]);
       }
+    }
+  }
+}
+
+// Two adjacent groups per item when qubit 0 is free (not a target or control):
+// groups at k and k+1 share every 32-byte sector, so each access is one
+// LDG/STG.256 and the instruction count per byte halves.
+template <int L, int U, int NPMAX, class Op>
+__global__ void __launch_bounds__(kThreads) k_group_x2(double2* __restrict__ a, uint64_t n_items,
+                                                       const InsertPlan ip, const Offs<L> off,
+                                                       const Op op) {
+  const uint64_t i0 = (uint64_t)blockIdx.x * (kThreads * U) + threadIdx.x;
+  double2 v[U][L], w[U][L];
+  uint64_t kk[U];
+#pragma unroll
+  for (int u = 0; u < U; ++u) {
+    const uint64_t i = i0 + (uint64_t)u * kThreads;
+    kk[u] = expand<NPMAX>(ip, (i < n_items ? i : 0) << 1);
+    if (i < n_items) {
+#pragma unroll
+      for (int j = 0; j < L; ++j) ld32(a + kk[u] + off.o[j], v[u][j], w[u][j]);
+    }
+  }
+#pragma unroll
+  for (int u = 0; u < U; ++u) {
+    const uint64_t i = i0 + (uint64_t)u * kThreads;
+    if (i < n_items) {
+      op(v[u], kk[u]);
+      op(w[u], kk[u] | 1);
+#pragma unroll
+      for (int j = 0; j < L; ++j) st32(a + kk[u] + off.o[j], v[u][j], w[u][j]);
     }
   }
 }
@@ -289,9 +346,27 @@ template <int L, int U, bool P256, class Op>
 void run_group(const LaunchCtx& ctx, uint64_t n_groups, const InsertPlan& ip, const Offs<L>& off,
                const Op& op) {
   if (n_groups == 0) return;
+  auto* a = reinterpret_cast<double2*>(ctx.amps);
+  bool even = true;
+  for (int j = 0; j < L; ++j) even &= (off.o[j] & 1) == 0;
+  if constexpr (!P256 && L <= 4) {
+    if (ctx.opt->wide256 && even && n_groups >= 2 && (ip.np == 0 || ip.pos[0] >= 1)) {
+      constexpr int UX = L == 1 ? 4 : (L == 2 ? 2 : 1);
+      const uint64_t n_items = n_groups / 2;
+      const uint64_t nb = blocks_for(n_items, (uint64_t)kThreads * UX);
+      require(nb < (1ull << 31), "grid too large");
+      if (ip.np <= 4)
+        k_group_x2<L, UX, 4, Op><<<(unsigned)nb, kThreads, 0, ctx.stream>>>(a, n_items, ip, off, op);
+      else
+        k_group_x2<L, UX, kMaxInsert, Op>
+            <<<(unsigned)nb, kThreads, 0, ctx.stream>>>(a, n_items, ip, off, op);
+      LFQS_CUDA_CHECK(cudaGetLastError());
+      ++*ctx.launch_counter;
+      return;
+    }
+  }
   const uint64_t nb = blocks_for(n_groups, (uint64_t)kThreads * U);
   require(nb < (1ull << 31), "grid too large");
-  auto* a = reinterpret_cast<double2*>(ctx.amps);
   if (ip.np <= 4)
     k_group<L, U, P256, 4, Op><<<(unsigned)nb, kThreads, 0, ctx.stream>>>(a, n_groups, ip, off, op);
   else
@@ -322,6 +397,14 @@ template <class Op, class LaneOp>
 void launch_pair(const LaunchCtx& ctx, const Decoded& g, const Op& op, const LaneOp& lane_op) {
   const int t = g.targets[0];
   const int nc = __builtin_popcountll(g.cmask);
+  if (g.cmask & 1) {
+    // Control on qubit 0: widen to (k, k+1, k+2^t, k+2^t+1) so the untouched
+    // neighbours are rewritten and no 16-byte (sub-sector) writes occur.
+    const InsertPlan ip = make_plan((1ull << t) | 1ull, g.cmask & ~1ull);
+    Offs<4> off{{0ull, 1ull, 1ull << t, (1ull << t) | 1ull}};
+    run_group<4, 2, true>(ctx, 1ull << (ctx.n_local - 1 - nc), ip, off, OpCtrl0<Op>{op});
+    return;
+  }
   constexpr int kCB = 7;
   if (ctx.opt->lowq_shuffle && t < 5 && ctx.n_local >= kCB + __builtin_popcountll(g.cmask >> kCB)) {
     run_lowq(ctx, t, g.cmask, lane_op);
@@ -390,6 +473,47 @@ void launch_dense_m(const LaunchCtx& ctx, const Decoded& g) {
     run_group<L, (L == 4 ? 2 : 1), false>(ctx, n_groups, ip, off, op);
 }
 
+template <class Op1>
+void run_diag_one(const LaunchCtx& ctx, uint64_t n_groups, uint64_t zeros, uint64_t ones,
+                  const Op1& op) {
+  if ((zeros | ones) & 1) {
+    // Qubit 0 is fixed: widen the group to the adjacent pair so every write is a
+    // whole 32-byte sector (a 16-byte write costs a sector read-modify-write).
+    const InsertPlan ip = make_plan((zeros & ~1ull) | 1ull, ones & ~1ull);
+    run_group<2, 4, true>(ctx, n_groups, ip, Offs<2>{{0, 1}},
+                          OpAtPair<Op1>{op, (int)(ones & 1)});
+  } else {
+    run_group<1, 4, false>(ctx, n_groups, make_plan(zeros, ones), Offs<1>{{0}}, op);
+  }
+}
+
+template <int L>
+void run_diag_group(const LaunchCtx& ctx, const Decoded& g) {
+  constexpr int m = L == 2 ? 1 : (L == 4 ? 2 : 3);
+  int perm[3] = {0, 1, 2};
+  for (int s = 0; s < m; ++s)
+    if (g.targets[s] == 0) std::swap(perm[s], perm[m - 1]);
+  int t[3];
+  cplx Mp[64];
+  permute_targets(g, perm, t, Mp);
+  OpDiagGroup<L> op;
+  op.touch = 0;
+  for (int j = 0; j < L; ++j) {
+    op.d[j] = D2(Mp[j * L + j]);
+    if (!(Mp[j * L + j].re == 1.0 && Mp[j * L + j].im == 0.0)) op.touch |= 1u << j;
+  }
+  uint64_t tmask = 0;
+  for (int s = 0; s < m; ++s) tmask |= 1ull << t[s];
+  const int nc = __builtin_popcountll(g.cmask);
+  const uint64_t n_groups = 1ull << (ctx.n_local - m - nc);
+  const InsertPlan ip = make_plan(tmask, g.cmask);
+  const Offs<L> off = group_offsets<L>(t, m);
+  if (t[m - 1] == 0)
+    run_group<L, (L == 8 ? 1 : 2), true>(ctx, n_groups, ip, off, op);
+  else
+    run_group<L, (L == 8 ? 1 : 2), false>(ctx, n_groups, ip, off, op);
+}
+
 void launch_diag(const LaunchCtx& ctx, const Decoded& g) {
   const int m = g.m, d = 1 << m;
   // Entries != 1 (the only amplitudes that change).
@@ -409,27 +533,25 @@ void launch_diag(const LaunchCtx& ctx, const Decoded& g) {
     // Touch only amplitudes with target bits = active pattern and controls = 1.
     uint64_t pattern = 0;
     for (int s = 0; s < m; ++s) pattern |= (uint64_t)((active >> (m - 1 - s)) & 1) << g.targets[s];
-    const InsertPlan ip = make_plan(tmask & ~pattern, g.cmask | pattern);
+    const uint64_t zeros = tmask & ~pattern, ones = g.cmask | pattern;
     const uint64_t n_groups = 1ull << (ctx.n_local - m - nc);
     const cplx z = g.M[active * d + active];
-    Offs<1> off{{0}};
     if (z.re == -1.0 && z.im == 0.0)
-      run_group<1, 4, false>(ctx, n_groups, ip, off, OpNeg{});
+      run_diag_one(ctx, n_groups, zeros, ones, OpNeg{});
     else if (z.re == 0.0 && z.im == 1.0)
-      run_group<1, 4, false>(ctx, n_groups, ip, off, OpMulI{});
+      run_diag_one(ctx, n_groups, zeros, ones, OpMulI{});
     else if (z.re == 0.0 && z.im == -1.0)
-      run_group<1, 4, false>(ctx, n_groups, ip, off, OpMulNI{});
+      run_diag_one(ctx, n_groups, zeros, ones, OpMulNI{});
     else
-      run_group<1, 4, false>(ctx, n_groups, ip, off, OpMul{D2(z)});
+      run_diag_one(ctx, n_groups, zeros, ones, OpMul{D2(z)});
     return;
   }
-  OpDiagSel op;
-  op.m = m;
-  for (int s = 0; s < 3; ++s) op.t[s] = s < m ? g.targets[s] : 0;
-  for (int j = 0; j < 8; ++j) op.d[j] = j < d ? D2(g.M[j * d + j]) : make_double2(1, 0);
-  const InsertPlan ip = make_plan(0, g.cmask);
-  const uint64_t n_groups = 1ull << (ctx.n_local - nc);
-  run_group<1, 4, false>(ctx, n_groups, ip, Offs<1>{{0}}, op);
+  if (m == 1)
+    run_diag_group<2>(ctx, g);
+  else if (m == 2)
+    run_diag_group<4>(ctx, g);
+  else
+    run_diag_group<8>(ctx, g);
 }
 
 }  // namespace

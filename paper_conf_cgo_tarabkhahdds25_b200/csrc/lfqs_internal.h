@@ -79,6 +79,7 @@ struct InsertPlan {
 
 struct Options {
   bool lowq_shuffle = true;
+  bool wide256 = true;       // two adjacent groups per item, 32-byte accesses
   int fuse_tile_qubits = 12;
   int items_per_thread = 0;  // 0 = library default
 };

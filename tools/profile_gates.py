@@ -18,7 +18,9 @@ import numpy as np  # noqa: E402
 
 import workloads as W  # noqa: E402
 
-DEFAULT = "H:2,H:20,X:0,X:3,X:20,Z:15,T:0,RZ:3,SWAP:1/20,U2:0/7,U2:20/25,CX:1/0,CCX:1/2/5,U3q:0/4/9"
+DEFAULT = ("H:2,H:20,X:0,X:3,X:20,Y:7,RX:12,Z:15,Z:0,T:0,S:1,PHASE:6,RZ:0,RZ:3,RZ:20,CZ:0/9,"
+           "CZ:3/9,SWAP:1/20,SWAP:0/20,SWAP:12/20,U2:0/7,U2:20/25,U2:7/0,CX:1/0,CX:0/29,CX:10/11,"
+           "CCX:1/2/5,CCX:0/1/20,CCX:20/21/5,U3q:0/4/9,U3q:20/25/28")
 
 
 def parse(spec, n):
@@ -50,6 +52,7 @@ def main():
     ap.add_argument("--gates", default=DEFAULT)
     ap.add_argument("--time", action="store_true")
     ap.add_argument("--no-shuffle", action="store_true")
+    ap.add_argument("--no-wide", action="store_true")
     args = ap.parse_args()
     import torch
     import paper_conf_cgo_tarabkhahdds25_b200 as L
@@ -58,6 +61,7 @@ def main():
     gates = parse(args.gates, args.n)
     with L.State.create(args.n, 0, stream=s) as st:
         st.set_option(L.OPT_LOWQ_SHUFFLE, 0 if args.no_shuffle else 1)
+        st.set_option(L.OPT_WIDE256, 0 if args.no_wide else 1)
         st.init_random(7)
         for g in gates:
             st.apply(g)  # warm-up
