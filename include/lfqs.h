@@ -164,7 +164,7 @@ lfqs_status lfqs_state_info(const lfqs_state* s, int* n_qubits, int* n_local, in
 /* Number of kernels this state has launched so far (for benchmark accounting). */
 lfqs_status lfqs_kernel_launches(const lfqs_state* s, uint64_t* count);
 /* Tuning knobs (benchmark / test use): LFQS_OPT_LOWQ_SHUFFLE (1: warp-shuffle
- * path for targets < 5, default 1), LFQS_OPT_FUSE_TILE_QUBITS (k of the staging
+ * path for targets < 5; default 0, measured no faster than the 32-byte path), LFQS_OPT_FUSE_TILE_QUBITS (k of the staging
  * tile, default 12). */
 #define LFQS_OPT_LOWQ_SHUFFLE 1
 #define LFQS_OPT_FUSE_TILE_QUBITS 2

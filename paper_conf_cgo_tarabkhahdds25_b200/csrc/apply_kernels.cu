@@ -90,6 +90,13 @@ struct OpSwap2 {  // X / CNOT / Toffoli / SWAP: moves only (bit-exact)
     v[1] = t;
   }
 };
+struct OpSwapMid {  // SWAP(0, t) on the group (00, 01, 10, 11): exchange 01 <-> 10
+  __device__ __forceinline__ void operator()(double2 (&v)[4], uint64_t) const {
+    const double2 t = v[1];
+    v[1] = v[2];
+    v[2] = t;
+  }
+};
 struct OpY {  // Y = [[0,-i],[i,0]]: v0' = -i v1, v1' = i v0 (moves + sign, exact)
   __device__ __forceinline__ void operator()(double2 (&v)[2], uint64_t) const {
     const double2 a0 = v[0], a1 = v[1];
@@ -582,6 +589,14 @@ void launch_gate(const LaunchCtx& ctx, const Decoded& g) {
       const int t0 = g.targets[0], t1 = g.targets[1];
       const int nc = __builtin_popcountll(g.cmask);
       const InsertPlan ip = make_plan((1ull << t0) | (1ull << t1), g.cmask);
+      if ((t0 == 0 || t1 == 0) && !(g.cmask & 1)) {
+        // SWAP(0, t): move whole sectors (k, k+1), (k+2^t, k+2^t+1) and exchange
+        // the middle two, instead of 16-byte writes into half-used sectors.
+        const uint64_t t = 1ull << (t0 == 0 ? t1 : t0);
+        Offs<4> off{{0ull, 1ull, t, t | 1ull}};
+        run_group<4, 2, true>(ctx, 1ull << (ctx.n_local - 2 - nc), ip, off, OpSwapMid{});
+        return;
+      }
       Offs<2> off{{1ull << t0, 1ull << t1}};
       run_group<2, 4, false>(ctx, 1ull << (ctx.n_local - 2 - nc), ip, off, OpSwap2{});
       return;

@@ -78,7 +78,9 @@ struct InsertPlan {
 };
 
 struct Options {
-  bool lowq_shuffle = true;
+  // Warp-shuffle path for targets < 5.  Measured equal-or-slower than the
+  // generic 32-byte path on B200 (profiles/r01_gate_sweep.md), so off by default.
+  bool lowq_shuffle = false;
   bool wide256 = true;       // two adjacent groups per item, 32-byte accesses
   int fuse_tile_qubits = 12;
   int items_per_thread = 0;  // 0 = library default
@@ -91,7 +93,11 @@ struct LaunchCtx {
   cudaStream_t stream;
   uint64_t* launch_counter;
   const Options* opt;
+  void** fused_prog;       // state-owned device buffer for fused gate programs
 };
+
+// Raises a kernel's dynamic shared memory limit once per device.
+void ensure_smem_attr(const void* kernel, int bytes);
 
 // Applies one decoded gate whose targets are all < n_local (controls < n_local).
 void launch_gate(const LaunchCtx& ctx, const Decoded& g);

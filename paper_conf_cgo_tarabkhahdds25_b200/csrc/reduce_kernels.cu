@@ -12,6 +12,9 @@
 #include <cuda_runtime.h>
 
 #include <cstring>
+#include <mutex>
+#include <set>
+#include <utility>
 
 #include "lfqs_internal.h"
 
@@ -125,6 +128,18 @@ __global__ void __launch_bounds__(kThreads) k_init_random(double2* __restrict__ 
 
 int probs_blocks() { return kBlocks; }
 
+void ensure_smem_attr(const void* kernel, int bytes) {
+  // cudaFuncSetAttribute is per device; remember (kernel, device) pairs done.
+  static std::mutex mu;
+  static std::set<std::pair<const void*, int>> done;
+  int dev = 0;
+  LFQS_CUDA_CHECK(cudaGetDevice(&dev));
+  std::lock_guard<std::mutex> lk(mu);
+  if (done.count({kernel, dev})) return;
+  LFQS_CUDA_CHECK(cudaFuncSetAttribute(kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes));
+  done.insert({kernel, dev});
+}
+
 void launch_probs(const LaunchCtx& ctx, const int* qubits, int nq, double* d_partials,
                   int n_partials_blocks, double* d_out) {
   require(nq >= 0 && nq <= kMaxQ, "measure_probs supports at most 10 qubits");
@@ -148,12 +163,7 @@ void launch_probs(const LaunchCtx& ctx, const int* qubits, int nq, double* d_par
   require(n_partials_blocks >= kBlocks, "partials buffer too small");
   const int nbins = 1 << nq;
   const size_t smem = sizeof(double) * kWarps * nbins;
-  static bool attr_set = false;
-  if (!attr_set) {
-    LFQS_CUDA_CHECK(cudaFuncSetAttribute(k_probs, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                         sizeof(double) * kWarps * (1 << kMaxQ)));
-    attr_set = true;
-  }
+  ensure_smem_attr((const void*)k_probs, sizeof(double) * kWarps * (1 << kMaxQ));
   k_probs<<<kBlocks, kThreads, smem, ctx.stream>>>(a, n_amps / 32, ql, d_partials);
   LFQS_CUDA_CHECK(cudaGetLastError());
   k_probs_final<<<(nbins + 255) / 256, 256, 0, ctx.stream>>>(d_partials, kBlocks, nbins, d_out);

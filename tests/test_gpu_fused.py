@@ -1,0 +1,72 @@
+"""Fused low-qubit staging (LFQS_FUSE_LOW) == unfused per-gate semantics and == oracle.
+
+Permutation/diagonal gates use the same formulas fused or not, so circuits made
+only of them must agree bit-exactly; dense gates within 1e-12."""
+import numpy as np
+import pytest
+
+import oracle as O
+import workloads as W
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def L():
+    import torch
+    if not torch.cuda.is_available():
+        pytest.skip("needs a GPU")
+    import paper_conf_cgo_tarabkhahdds25_b200 as lib
+    lib.lib()
+    return lib
+
+
+def _run(L, n, psi, gates, fuse, tile=None):
+    with L.State.create(n) as st:
+        if tile:
+            st.set_option(L.OPT_FUSE_TILE_QUBITS, tile)
+        st.copy_in(psi)
+        c0 = st.launches()
+        st.run_circuit(gates, fuse=fuse)
+        out = st.copy_out()
+        return out, st.launches() - c0
+
+
+@pytest.mark.parametrize("tile", [6, 9, 12, 13])
+@pytest.mark.parametrize("n", [8, 14, 17])
+def test_fused_random_circuit(L, n, tile):
+    psi = W.random_state(n, n + tile)
+    gates = W.random_gate_list(n, 250, seed=7 * n + tile, max_controls=2)
+    ref = O.run_circuit(n, gates, psi.copy())
+    got, launches = _run(L, n, psi, gates, True, tile)
+    assert np.max(np.abs(got - ref)) <= 1e-12
+    unf, _ = _run(L, n, psi, gates, False)
+    assert np.max(np.abs(got - unf)) <= 1e-12
+    exact = [g for g in gates if g.exact]
+    a, _ = _run(L, n, psi, exact, True, tile)
+    b, _ = _run(L, n, psi, exact, False)
+    assert np.array_equal(a, b)
+
+
+def test_fusion_reduces_passes_qft(L):
+    n, x = 20, 0xBEEF1
+    gates = W.qft(n)
+    with L.State.create(n) as st:
+        st.init_basis(x)
+        c0 = st.launches()
+        st.run_circuit(gates, fuse=True)
+        launches = st.launches() - c0
+        a = st.copy_out()
+    y = np.arange(1 << n, dtype=np.int64)
+    ref = np.exp(2j * np.pi * ((x * y) % (1 << n)) / (1 << n)) / np.sqrt(1 << n)
+    assert np.max(np.abs(a - ref)) <= 1e-12
+    assert launches < len(gates) // 4, (launches, len(gates))
+
+
+def test_fused_layered_and_grover(L):
+    n = 16
+    psi = W.random_state(n, 3)
+    for gates in (W.random_layered(n, 10, seed=5), W.grover(n, 12345, 2), W.ghz(n)):
+        ref = O.run_circuit(n, gates, psi.copy())
+        got, _ = _run(L, n, psi, gates, True)
+        assert np.max(np.abs(got - ref)) <= 1e-12

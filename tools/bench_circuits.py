@@ -1,0 +1,101 @@
+"""Macro benchmarks (BASELINE.json configs[2]-[3] shapes on one GPU): QFT, GHZ, Grover,
+random layered circuits at n qubits, fused and unfused, with closed-form checks on
+sampled amplitudes (n >= 31 does not fit the host oracle).
+
+    python tools/bench_circuits.py --n 30 [--circuits qft,ghz,grover,random] [--reps 2]
+Prints one JSON object per (circuit, mode).
+"""
+import argparse
+import json
+import math
+import os
+import sys
+import time
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+
+import workloads as W  # noqa: E402
+
+
+def sample_idx(n, count, seed):
+    rng = np.random.default_rng(seed)
+    return np.unique(np.concatenate([rng.integers(0, 1 << n, count), [0, (1 << n) - 1]]))
+
+
+def check(name, n, st, meta):
+    idx = sample_idx(n, 64, 1)
+    got = np.array([st.copy_out(int(k), 1)[0] for k in idx])
+    if name == "qft":
+        x = meta["x"]
+        ref = np.exp(2j * np.pi * ((x * idx.astype(object)) % (1 << n)).astype(np.float64) / (1 << n)) \
+            / math.sqrt(2.0 ** n)
+    elif name == "ghz":
+        ref = np.where((idx == 0) | (idx == (1 << n) - 1), math.sqrt(0.5), 0.0).astype(complex)
+    elif name == "grover":
+        k, w = meta["k"], meta["w"]
+        th = math.asin(2.0 ** (-n / 2))
+        ref = np.full(idx.shape, (-1) ** k * math.cos((2 * k + 1) * th) / math.sqrt(2.0 ** n - 1),
+                      dtype=complex)
+        ref[idx == w] = (-1) ** k * math.sin((2 * k + 1) * th)
+    else:
+        return {"norm2": st.norm2()}
+    return {"max_abs_err": float(np.max(np.abs(got - ref)))}
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--n", type=int, default=30)
+    ap.add_argument("--circuits", default="qft,ghz,grover,random")
+    ap.add_argument("--modes", default="fused,unfused")
+    ap.add_argument("--reps", type=int, default=2)
+    ap.add_argument("--tile", type=int, default=0)
+    args = ap.parse_args()
+    import torch
+    import paper_conf_cgo_tarabkhahdds25_b200 as L
+    s = torch.cuda.Stream()
+    torch.cuda.set_stream(s)
+    n = args.n
+    x = int(W.SplitMix64(n).next_u64() & ((1 << n) - 1))
+    w = int(W.SplitMix64(n + 1).next_u64() & ((1 << n) - 1))
+    circuits = {
+        "qft": (W.qft(n), lambda st: st.init_basis(x), {"x": x}),
+        "ghz": (W.ghz(n), lambda st: st.init_basis(0), {}),
+        "grover": (W.grover(n, w, 2), lambda st: st.init_basis(0), {"k": 2, "w": w}),
+        "random": (W.random_layered(n, 20, seed=7), lambda st: st.init_basis(0), {}),
+    }
+    with L.State.create(n, 0, stream=s) as st:
+        if args.tile:
+            st.set_option(L.OPT_FUSE_TILE_QUBITS, args.tile)
+        for name in args.circuits.split(","):
+            gates, init, meta = circuits[name]
+            arr = L.marshal_gates(gates)
+            for mode in args.modes.split(","):
+                flags = L.FUSE_LOW if mode == "fused" else L.FUSE_NONE
+                times, passes = [], 0
+                for r in range(args.reps + 1):
+                    init(st)
+                    torch.cuda.synchronize()
+                    c0 = st.launches()
+                    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                    e0.record(s)
+                    L.lfqs_run_circuit(st.h, arr, flags)
+                    e1.record(s)
+                    torch.cuda.synchronize()
+                    if r > 0:
+                        times.append(e0.elapsed_time(e1))
+                    passes = st.launches() - c0
+                res = check(name, n, st, meta)
+                t = min(times)
+                rec = {"circuit": name, "mode": mode, "n": n, "gates": len(gates), "passes": passes,
+                       "ms": t, "gates_per_s": len(gates) / (t / 1e3),
+                       "conv_GBps": 32.0 * 2 ** n * len(gates) / (t / 1e3) / 1e9,
+                       "pass_GBps": 32.0 * 2 ** n * passes / (t / 1e3) / 1e9}
+                rec.update(res)
+                print(json.dumps(rec), flush=True)
+
+
+if __name__ == "__main__":
+    main()
