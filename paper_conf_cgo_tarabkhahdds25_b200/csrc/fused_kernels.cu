@@ -295,22 +295,22 @@ __global__ void __launch_bounds__(kFThreads, 2) k_fused(double2* __restrict__ a,
     const int type = op.type;
     const uint32_t cl = (uint32_t)op.cl;
     const int t0 = op.t[0];
-    const bool reg_op = type == F_DIAG ||
+    const bool regpath = type == F_DIAG ||
                         (type <= F_U2 && (t0 < 5 || t0 >= 8));
-    if (reg_op && !in_regs) {
+    if (regpath && !in_regs) {
       __syncthreads();
 #pragma unroll
       for (int r = 0; r < R; ++r) v[r] = tile[r * kFThreads + tid];
       in_regs = true;
-    } else if (!reg_op && in_regs) {
+    } else if (!regpath && in_regs) {
 #pragma unroll
       for (int r = 0; r < R; ++r) tile[r * kFThreads + tid] = v[r];
       in_regs = false;
       __syncthreads();
-    } else if (!reg_op) {
+    } else if (!regpath) {
       __syncthreads();
     }
-    if (!reg_op) {
+    if (!regpath) {
       smem_op(tile, op, T);
       continue;
     }
