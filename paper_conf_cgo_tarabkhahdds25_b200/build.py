@@ -54,7 +54,7 @@ def build(force: bool = False, verbose: bool = False) -> str:
         obj = os.path.join(objdir, os.path.basename(src) + ".o")
         cmd = [NVCC] + ARCH + common + ["-Xptxas", "-warn-spills", "-c", src, "-o", obj]
         if src.endswith(".cpp"):
-            cmd = [NVCC] + common + ["-x", "c++", "-c", src, "-o", obj]
+            cmd = [NVCC] + ARCH + common + ["-x", "c++", "-c", src, "-o", obj]
         if verbose:
             print(" ".join(cmd), flush=True)
         subprocess.check_call(cmd)

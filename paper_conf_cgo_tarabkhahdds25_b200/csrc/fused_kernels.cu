@@ -9,11 +9,14 @@
 //   * the tile (2^K contiguous amplitudes, K <= 12 -> 64 KiB) is staged into
 //     shared memory with one TMA bulk copy (cp.async.bulk + mbarrier) and
 //     written back with one bulk store;
-//   * amplitudes then live in registers: thread `tid` of 256 holds tile
-//     elements i = r * 256 + tid, r < 2^(K-8).  Diagonal gates, and 1-target
-//     gates on register bits (8..K-1) or lane bits (0..4, via shfl.xor), are
-//     applied in registers; 1-target gates on warp bits (5..7) and 2/3-target
-//     gates go through the shared-memory tile;
+//   * the gate program is a __grid_constant__ kernel parameter (<= 32 KB:
+//     headers + a coefficient pool), read through the constant cache -- no
+//     global-memory round trips inside the op loop;
+//   * amplitudes live in registers: thread `tid` of 256 holds tile elements
+//     i = r * 256 + tid, r < 2^(K-8).  Diagonal gates, and 1-target gates on
+//     register bits (8..K-1) or lane bits (0..4, via shfl.xor), are applied in
+//     registers; 1-target gates on warp bits (5..7) and 2/3-target gates go
+//     through the shared-memory tile;
 //   * a gate fuses when all its targets are < K (controls anywhere: controls
 //     >= K are a per-tile predicate) or when it is diagonal (any qubits: target
 //     bits >= K come from the tile index).
@@ -31,20 +34,25 @@ namespace lfqs {
 
 namespace {
 
-enum FType : int { F_DIAG = 0, F_X, F_Y, F_H, F_U2, F_SWAP, F_U4, F_U8 };
+enum FType : uint8_t { F_DIAG1 = 0, F_DIAGN, F_X, F_Y, F_H, F_U2, F_SWAP, F_U4, F_U8 };
 
-struct FOp {
-  int type;
-  int m;
-  int t[3];        // targets (DIAG: any position; others: < K)
-  int pad;
-  uint64_t cl;     // controls below K (per amplitude)
-  uint64_t ch;     // controls at or above K (per tile)
-  double2 c[64];   // matrix row-major, or the diagonal d[j] for DIAG
+struct FHdr {       // 32 bytes
+  uint8_t type, m, t0, t1, t2, pad0;
+  uint16_t coef;    // offset into the coefficient pool
+  uint32_t mlo, plo;  // per-amplitude predicate (i & mlo) == plo   (bits < K)
+  uint64_t mhi, phi;  // per-tile predicate     (base & mhi) == phi (bits >= K)
 };
+constexpr int kMaxOps = 192;
+constexpr int kMaxCoef = 1600;
+struct FProg {
+  int nops;
+  int ncoef;
+  FHdr h[kMaxOps];
+  double2 c[kMaxCoef];
+};
+static_assert(sizeof(FProg) + 8 <= 32764, "kernel parameter limit");
 
 constexpr int kFThreads = 256;
-constexpr int kMaxOps = 256;
 constexpr int kMinK = 8, kMaxK = 12;
 
 __device__ __forceinline__ uint32_t smem_u32(const void* p) {
@@ -65,101 +73,8 @@ __device__ __forceinline__ uint32_t ins0(uint32_t p, int t) {
 }
 __device__ __forceinline__ bool is_one(double2 d) { return d.x == 1.0 && d.y == 0.0; }
 
-// The 2x2 update of a pair (a0 = bit 0, a1 = bit 1), same formulas as apply_kernels.cu.
-__device__ __forceinline__ void pair_update(int type, const FOp& op, double2& a0, double2& a1) {
-  const double2 x0 = a0, x1 = a1;
-  if (type == F_X) {
-    a0 = x1;
-    a1 = x0;
-  } else if (type == F_Y) {
-    a0 = make_double2(x1.y, -x1.x);
-    a1 = make_double2(-x0.y, x0.x);
-  } else if (type == F_H) {
-    const double s = op.c[0].x;
-    a0 = make_double2(s * (x0.x + x1.x), s * (x0.y + x1.y));
-    a1 = make_double2(s * (x0.x - x1.x), s * (x0.y - x1.y));
-  } else {
-    double2 b0 = make_double2(0.0, 0.0), b1 = b0;
-    cfma(b0, op.c[0], x0);
-    cfma(b0, op.c[1], x1);
-    cfma(b1, op.c[2], x0);
-    cfma(b1, op.c[3], x1);
-    a0 = b0;
-    a1 = b1;
-  }
-}
-
-template <int L>
-__device__ __forceinline__ void dense_group(double2* tile, const uint32_t (&idx)[L],
-                                            const double2* __restrict__ c) {
-  double2 v[L], w[L];
-#pragma unroll
-  for (int j = 0; j < L; ++j) v[j] = tile[idx[j]];
-#pragma unroll
-  for (int j = 0; j < L; ++j) {
-    double2 acc = make_double2(0.0, 0.0);
-#pragma unroll
-    for (int i = 0; i < L; ++i) cfma(acc, c[j * L + i], v[i]);
-    w[j] = acc;
-  }
-#pragma unroll
-  for (int j = 0; j < L; ++j) tile[idx[j]] = w[j];
-}
-
-// Non-register op on the shared-memory tile (T = 2^K amplitudes).
-__device__ void smem_op(double2* tile, const FOp& op, uint32_t T) {
-  const uint32_t cl = (uint32_t)op.cl;
-  const int type = op.type;
-  if (type <= F_U2) {
-    const int t = op.t[0];
-    for (uint32_t p = threadIdx.x; p < (T >> 1); p += kFThreads) {
-      const uint32_t i0 = ins0(p, t), i1 = i0 | (1u << t);
-      if ((i0 & cl) != cl) continue;
-      double2 a0 = tile[i0], a1 = tile[i1];
-      pair_update(type, op, a0, a1);
-      tile[i0] = a0;
-      tile[i1] = a1;
-    }
-  } else if (type == F_SWAP) {
-    const int lo = op.t[0] < op.t[1] ? op.t[0] : op.t[1];
-    const int hi = op.t[0] < op.t[1] ? op.t[1] : op.t[0];
-    for (uint32_t p = threadIdx.x; p < (T >> 2); p += kFThreads) {
-      const uint32_t i = ins0(ins0(p, lo), hi);
-      if ((i & cl) != cl) continue;
-      const uint32_t x = i | (1u << lo), y = i | (1u << hi);
-      const double2 vx = tile[x];
-      tile[x] = tile[y];
-      tile[y] = vx;
-    }
-  } else if (type == F_U4) {
-    const int t0 = op.t[0], t1 = op.t[1];
-    const int lo = t0 < t1 ? t0 : t1, hi = t0 < t1 ? t1 : t0;
-    for (uint32_t p = threadIdx.x; p < (T >> 2); p += kFThreads) {
-      const uint32_t i = ins0(ins0(p, lo), hi);
-      if ((i & cl) != cl) continue;
-      const uint32_t idx[4] = {i, i | (1u << t1), i | (1u << t0), i | (1u << t0) | (1u << t1)};
-      dense_group<4>(tile, idx, op.c);
-    }
-  } else {  // F_U8
-    const int s0 = op.t[0], s1 = op.t[1], s2 = op.t[2];
-    int a0 = s0 < s1 ? s0 : s1, a1 = s0 < s1 ? s1 : s0, a2 = s2;
-    if (a2 < a1) { const int x = a1; a1 = a2; a2 = x; }
-    if (a1 < a0) { const int x = a0; a0 = a1; a1 = x; }
-    for (uint32_t p = threadIdx.x; p < (T >> 3); p += kFThreads) {
-      const uint32_t i = ins0(ins0(ins0(p, a0), a1), a2);
-      if ((i & cl) != cl) continue;
-      uint32_t idx[8];
-#pragma unroll
-      for (int j = 0; j < 8; ++j)
-        idx[j] = i | (((j >> 2) & 1u) << s0) | (((j >> 1) & 1u) << s1) | ((j & 1u) << s2);
-      dense_group<8>(tile, idx, op.c);
-    }
-  }
-}
-
-// Register-path functors: the gate type is dispatched once per op, outside the
-// unrolled per-register loops (keeps register pressure low).
-struct RX_ {
+// ---- 2x2 functors (type dispatched once per op) ------------------------------
+struct FX_ {
   __device__ __forceinline__ void pair(double2& a0, double2& a1) const {
     const double2 t = a0;
     a0 = a1;
@@ -167,7 +82,7 @@ struct RX_ {
   }
   __device__ __forceinline__ double2 lane(double2, double2 p, int) const { return p; }
 };
-struct RY_ {
+struct FY_ {
   __device__ __forceinline__ void pair(double2& a0, double2& a1) const {
     const double2 x0 = a0, x1 = a1;
     a0 = make_double2(x1.y, -x1.x);
@@ -177,7 +92,7 @@ struct RY_ {
     return bit ? make_double2(-p.y, p.x) : make_double2(p.y, -p.x);
   }
 };
-struct RH_ {
+struct FH_ {
   double s;
   __device__ __forceinline__ void pair(double2& a0, double2& a1) const {
     const double2 x0 = a0, x1 = a1;
@@ -189,7 +104,7 @@ struct RH_ {
                : make_double2(s * (a.x + p.x), s * (a.y + p.y));
   }
 };
-struct RU_ {
+struct FU_ {
   double2 c0, c1, c2, c3;
   __device__ __forceinline__ void pair(double2& a0, double2& a1) const {
     double2 b0 = make_double2(0.0, 0.0), b1 = b0;
@@ -213,28 +128,110 @@ struct RU_ {
   }
 };
 
+// ---- shared-memory path ----------------------------------------------------------
+template <class F>
+__device__ __forceinline__ void smem_pairs(double2* tile, const F& f, int t, uint32_t mlo,
+                                           uint32_t plo, uint32_t T) {
+  for (uint32_t p = threadIdx.x; p < (T >> 1); p += kFThreads) {
+    const uint32_t i0 = ins0(p, t), i1 = i0 | (1u << t);
+    if ((i0 & mlo) != plo) continue;
+    double2 a0 = tile[i0], a1 = tile[i1];
+    f.pair(a0, a1);
+    tile[i0] = a0;
+    tile[i1] = a1;
+  }
+}
+
+template <int L>
+__device__ __forceinline__ void dense_group(double2* tile, const uint32_t (&idx)[L],
+                                            const double2* c) {
+  double2 v[L], w[L];
+#pragma unroll
+  for (int j = 0; j < L; ++j) v[j] = tile[idx[j]];
+#pragma unroll
+  for (int j = 0; j < L; ++j) {
+    double2 acc = make_double2(0.0, 0.0);
+#pragma unroll
+    for (int i = 0; i < L; ++i) cfma(acc, c[j * L + i], v[i]);
+    w[j] = acc;
+  }
+#pragma unroll
+  for (int j = 0; j < L; ++j) tile[idx[j]] = w[j];
+}
+
+__device__ void smem_op(double2* tile, const FHdr& h, const double2* c, uint32_t T) {
+  const uint32_t mlo = h.mlo, plo = h.plo;
+  switch (h.type) {
+    case F_X: smem_pairs(tile, FX_{}, h.t0, mlo, plo, T); return;
+    case F_Y: smem_pairs(tile, FY_{}, h.t0, mlo, plo, T); return;
+    case F_H: smem_pairs(tile, FH_{c[0].x}, h.t0, mlo, plo, T); return;
+    case F_U2: smem_pairs(tile, FU_{c[0], c[1], c[2], c[3]}, h.t0, mlo, plo, T); return;
+    case F_SWAP: {
+      const int lo = h.t0 < h.t1 ? h.t0 : h.t1, hi = h.t0 < h.t1 ? h.t1 : h.t0;
+      for (uint32_t p = threadIdx.x; p < (T >> 2); p += kFThreads) {
+        const uint32_t i = ins0(ins0(p, lo), hi);
+        if ((i & mlo) != plo) continue;
+        const uint32_t x = i | (1u << lo), y = i | (1u << hi);
+        const double2 vx = tile[x];
+        tile[x] = tile[y];
+        tile[y] = vx;
+      }
+      return;
+    }
+    case F_U4: {
+      const int t0 = h.t0, t1 = h.t1;
+      const int lo = t0 < t1 ? t0 : t1, hi = t0 < t1 ? t1 : t0;
+      for (uint32_t p = threadIdx.x; p < (T >> 2); p += kFThreads) {
+        const uint32_t i = ins0(ins0(p, lo), hi);
+        if ((i & mlo) != plo) continue;
+        const uint32_t idx[4] = {i, i | (1u << t1), i | (1u << t0), i | (1u << t0) | (1u << t1)};
+        dense_group<4>(tile, idx, c);
+      }
+      return;
+    }
+    default: {  // F_U8
+      const int s0 = h.t0, s1 = h.t1, s2 = h.t2;
+      int a0 = s0 < s1 ? s0 : s1, a1 = s0 < s1 ? s1 : s0, a2 = s2;
+      if (a2 < a1) { const int x = a1; a1 = a2; a2 = x; }
+      if (a1 < a0) { const int x = a0; a0 = a1; a1 = x; }
+      for (uint32_t p = threadIdx.x; p < (T >> 3); p += kFThreads) {
+        const uint32_t i = ins0(ins0(ins0(p, a0), a1), a2);
+        if ((i & mlo) != plo) continue;
+        uint32_t idx[8];
+#pragma unroll
+        for (int j = 0; j < 8; ++j)
+          idx[j] = i | (((j >> 2) & 1u) << s0) | (((j >> 1) & 1u) << s1) | ((j & 1u) << s2);
+        dense_group<8>(tile, idx, c);
+      }
+      return;
+    }
+  }
+}
+
+// ---- register path ---------------------------------------------------------------
 template <int RB, int R, class F>
-__device__ __forceinline__ void reg_pairs(double2 (&v)[R], const F& f, uint32_t cl, uint32_t tid) {
+__device__ __forceinline__ void reg_pairs(double2 (&v)[R], const F& f, uint32_t mlo, uint32_t plo,
+                                          uint32_t tid) {
   if constexpr ((1 << RB) < R) {
 #pragma unroll
     for (int r = 0; r < R; ++r) {
       if (r >> RB & 1) continue;
       const uint32_t i0 = (uint32_t)r * kFThreads + tid;
-      if ((i0 & cl) != cl) continue;
+      if ((i0 & mlo) != plo) continue;
       f.pair(v[r], v[r | (1 << RB)]);
     }
   }
 }
 
 template <int R, class F>
-__device__ __forceinline__ void reg_op(double2 (&v)[R], const F& f, int t0, uint32_t cl,
-                                       uint32_t tid) {
+__device__ __forceinline__ void reg_1q(double2 (&v)[R], const F& f, int t0, uint32_t mlo,
+                                       uint32_t plo, uint32_t tid) {
   if (t0 >= 8) {
     switch (t0 - 8) {
-      case 0: reg_pairs<0, R>(v, f, cl, tid); break;
-      case 1: reg_pairs<1, R>(v, f, cl, tid); break;
-      case 2: reg_pairs<2, R>(v, f, cl, tid); break;
-      default: reg_pairs<3, R>(v, f, cl, tid); break;
+      case 0: reg_pairs<0, R>(v, f, mlo, plo, tid); break;
+      case 1: reg_pairs<1, R>(v, f, mlo, plo, tid); break;
+      case 2: reg_pairs<2, R>(v, f, mlo, plo, tid); break;
+      default: reg_pairs<3, R>(v, f, mlo, plo, tid); break;
     }
     return;
   }
@@ -246,13 +243,13 @@ __device__ __forceinline__ void reg_op(double2 (&v)[R], const F& f, int t0, uint
     p.x = __shfl_xor_sync(0xffffffffu, v[r].x, 1 << t0);
     p.y = __shfl_xor_sync(0xffffffffu, v[r].y, 1 << t0);
     const uint32_t i = (uint32_t)r * kFThreads + tid;
-    if ((i & cl) == cl) v[r] = f.lane(v[r], p, bit);
+    if ((i & mlo) == plo) v[r] = f.lane(v[r], p, bit);
   }
 }
 
 template <int K>
 __global__ void __launch_bounds__(kFThreads, 2) k_fused(double2* __restrict__ a,
-                                                        const FOp* __restrict__ prog, int nops) {
+                                                        const __grid_constant__ FProg prog) {
   constexpr uint32_t T = 1u << K;
   constexpr int R = T / kFThreads;  // amplitudes per thread
   extern __shared__ __align__(128) double2 tile[];
@@ -288,15 +285,15 @@ __global__ void __launch_bounds__(kFThreads, 2) k_fused(double2* __restrict__ a,
   for (int r = 0; r < R; ++r) v[r] = tile[r * kFThreads + tid];
   bool in_regs = true;  // else the authoritative copy is the smem tile
 
+  const int nops = prog.nops;
   for (int o = 0; o < nops; ++o) {
-    const FOp& op = prog[o];
-    const uint64_t ch = op.ch;
-    if ((base & ch) != ch) continue;  // a high control is 0 on this tile (uniform)
-    const int type = op.type;
-    const uint32_t cl = (uint32_t)op.cl;
-    const int t0 = op.t[0];
-    const bool regpath = type == F_DIAG ||
-                        (type <= F_U2 && (t0 < 5 || t0 >= 8));
+    const FHdr& h = prog.h[o];
+    if ((base & h.mhi) != h.phi) continue;  // tile-level predicate (uniform)
+    const int type = h.type;
+    const int t0 = h.t0;
+    const uint32_t mlo = h.mlo, plo = h.plo;
+    const double2* c = prog.c + h.coef;
+    const bool regpath = type <= F_DIAGN || (type <= F_U2 && (t0 < 5 || t0 >= 8));
     if (regpath && !in_regs) {
       __syncthreads();
 #pragma unroll
@@ -311,55 +308,54 @@ __global__ void __launch_bounds__(kFThreads, 2) k_fused(double2* __restrict__ a,
       __syncthreads();
     }
     if (!regpath) {
-      smem_op(tile, op, T);
+      smem_op(tile, h, c, T);
       continue;
     }
-    if (type == F_DIAG) {
-      // j = local diagonal index; bits of targets >= K come from the tile base.
-      const int m = op.m;
-      uint32_t jh = 0, jmask = 0;  // uniform part of j and which j-bits are per amplitude
-      const int ta = op.t[0], tb = op.t[1], tc = op.t[2];
+    switch (type) {
+      case F_DIAG1: {  // one diagonal entry d != 1 on the amplitudes matching the predicate
+        const double2 d = c[0];
 #pragma unroll
-      for (int s = 0; s < 3; ++s) {
-        const int t = s == 0 ? ta : (s == 1 ? tb : tc);
-        if (s < m) {
-          if (t >= K)
-            jh |= (uint32_t)((base >> t) & 1) << (m - 1 - s);
-          else
-            jmask |= 1u << (m - 1 - s);
+        for (int r = 0; r < R; ++r) {
+          const uint32_t i = (uint32_t)r * kFThreads + tid;
+          if ((i & mlo) == plo) v[r] = cmul_rn(d, v[r]);
         }
+        break;
       }
-      if (jmask == 0) {  // factor uniform over the tile (or over amplitudes passing cl)
-        const double2 d = op.c[jh];
-        if (is_one(d)) continue;
+      case F_DIAGN: {  // factor d[j], j from the target bits (>= K: from the tile base)
+        const int m = h.m;
+        const int ts[3] = {h.t0, h.t1, h.t2};
+        uint32_t jh = 0, jmask = 0;
+#pragma unroll
+        for (int s = 0; s < 3; ++s)
+          if (s < m) {
+            if (ts[s] >= K)
+              jh |= (uint32_t)((base >> ts[s]) & 1) << (m - 1 - s);
+            else
+              jmask |= 1u << (m - 1 - s);
+          }
+        double2 dd[8];
+#pragma unroll
+        for (int j = 0; j < 8; ++j) dd[j] = j < (1 << m) ? c[j] : make_double2(1.0, 0.0);
 #pragma unroll
         for (int r = 0; r < R; ++r) {
           const uint32_t i = (uint32_t)r * kFThreads + tid;
-          if ((i & cl) == cl) v[r] = cmul_rn(d, v[r]);
-        }
-      } else {
-#pragma unroll
-        for (int r = 0; r < R; ++r) {
-          const uint32_t i = (uint32_t)r * kFThreads + tid;
-          if ((i & cl) != cl) continue;
+          if ((i & mlo) != plo) continue;
           uint32_t j = jh;
 #pragma unroll
-          for (int s = 0; s < 3; ++s) {
-            const int t = s == 0 ? ta : (s == 1 ? tb : tc);
-            if (s < m && (jmask >> (m - 1 - s) & 1)) j |= ((i >> t) & 1u) << (m - 1 - s);
-          }
-          const double2 d = op.c[j];
+          for (int s = 0; s < 3; ++s)
+            if (s < m && (jmask >> (m - 1 - s) & 1)) j |= ((i >> ts[s]) & 1u) << (m - 1 - s);
+          double2 d = dd[0];
+#pragma unroll
+          for (int q = 1; q < 8; ++q)
+            if ((uint32_t)q == j) d = dd[q];
           if (!is_one(d)) v[r] = cmul_rn(d, v[r]);
         }
+        break;
       }
-    } else if (type == F_X) {
-      reg_op<R>(v, RX_{}, t0, cl, tid);
-    } else if (type == F_Y) {
-      reg_op<R>(v, RY_{}, t0, cl, tid);
-    } else if (type == F_H) {
-      reg_op<R>(v, RH_{op.c[0].x}, t0, cl, tid);
-    } else {
-      reg_op<R>(v, RU_{op.c[0], op.c[1], op.c[2], op.c[3]}, t0, cl, tid);
+      case F_X: reg_1q<R>(v, FX_{}, t0, mlo, plo, tid); break;
+      case F_Y: reg_1q<R>(v, FY_{}, t0, mlo, plo, tid); break;
+      case F_H: reg_1q<R>(v, FH_{c[0].x}, t0, mlo, plo, tid); break;
+      default: reg_1q<R>(v, FU_{c[0], c[1], c[2], c[3]}, t0, mlo, plo, tid); break;
     }
   }
 
@@ -382,42 +378,84 @@ __global__ void __launch_bounds__(kFThreads, 2) k_fused(double2* __restrict__ a,
 
 inline double2 D2(cplx z) { return make_double2(z.re, z.im); }
 
-void encode(const Decoded& g, int K, FOp* op) {
-  std::memset(op, 0, sizeof(FOp));
-  const uint64_t lowmask = (1ull << K) - 1;
-  op->cl = g.cmask & lowmask;
-  op->ch = g.cmask & ~lowmask;
-  op->m = g.m;
-  for (int s = 0; s < g.m; ++s) op->t[s] = g.targets[s];
+int coef_count(const Decoded& g) {
   const int d = 1 << g.m;
   switch (g.cls) {
-    case GClass::DIAG:
-      op->type = F_DIAG;
-      for (int j = 0; j < d; ++j) op->c[j] = D2(g.M[j * d + j]);
-      return;
-    case GClass::PERM_X: op->type = F_X; return;
-    case GClass::PERM_Y: op->type = F_Y; return;
-    case GClass::PERM_SWAP: op->type = F_SWAP; return;
+    case GClass::DIAG: return d;  // upper bound (DIAG1 uses 1)
+    case GClass::PERM_X: case GClass::PERM_Y: case GClass::PERM_SWAP: return 0;
+    default: return g.is_h ? 1 : d * d;
+  }
+}
+
+// Appends gate g to the program; returns false if it does not fit.
+bool encode(const Decoded& g, int K, FProg& P) {
+  if (g.cls == GClass::NOOP) return true;
+  if (P.nops >= kMaxOps || P.ncoef + coef_count(g) > kMaxCoef) return false;
+  FHdr& h = P.h[P.nops];
+  std::memset(&h, 0, sizeof h);
+  const uint64_t lowmask = (1ull << K) - 1;
+  uint64_t m_all = g.cmask, p_all = g.cmask;
+  h.m = (uint8_t)g.m;
+  h.t0 = (uint8_t)g.targets[0];
+  h.t1 = (uint8_t)(g.m > 1 ? g.targets[1] : 0);
+  h.t2 = (uint8_t)(g.m > 2 ? g.targets[2] : 0);
+  h.coef = (uint16_t)P.ncoef;
+  const int d = 1 << g.m;
+  switch (g.cls) {
+    case GClass::DIAG: {
+      int n_active = 0, active = 0;
+      for (int j = 0; j < d; ++j) {
+        const cplx z = g.M[j * d + j];
+        if (!(z.re == 1.0 && z.im == 0.0)) {
+          ++n_active;
+          active = j;
+        }
+      }
+      if (n_active == 0) return true;
+      if (n_active == 1) {
+        h.type = F_DIAG1;
+        for (int s = 0; s < g.m; ++s) {
+          m_all |= 1ull << g.targets[s];
+          p_all |= (uint64_t)((active >> (g.m - 1 - s)) & 1) << g.targets[s];
+        }
+        P.c[P.ncoef++] = D2(g.M[active * d + active]);
+      } else {
+        h.type = F_DIAGN;
+        for (int j = 0; j < d; ++j) P.c[P.ncoef++] = D2(g.M[j * d + j]);
+      }
+      break;
+    }
+    case GClass::PERM_X: h.type = F_X; break;
+    case GClass::PERM_Y: h.type = F_Y; break;
+    case GClass::PERM_SWAP: h.type = F_SWAP; break;
     default:
+      if (g.m == 1) {
+        h.type = g.is_h ? F_H : F_U2;
+      } else {
+        h.type = g.m == 2 ? F_U4 : F_U8;
+      }
+      if (g.is_h) {
+        P.c[P.ncoef++] = D2(g.M[0]);
+      } else {
+        for (int i = 0; i < d * d; ++i) P.c[P.ncoef++] = D2(g.M[i]);
+      }
       break;
   }
-  if (g.m == 1) {
-    op->type = g.is_h ? F_H : F_U2;
-    if (g.is_h) op->c[0] = D2(g.M[0]);
-  } else {
-    op->type = g.m == 2 ? F_U4 : F_U8;
-  }
-  if (!g.is_h)
-    for (int i = 0; i < d * d; ++i) op->c[i] = D2(g.M[i]);
+  h.mlo = (uint32_t)(m_all & lowmask);
+  h.plo = (uint32_t)(p_all & lowmask);
+  h.mhi = m_all & ~lowmask;
+  h.phi = p_all & ~lowmask;
+  ++P.nops;
+  return true;
 }
 
 template <int K>
-void launch_k(const LaunchCtx& ctx, const FOp* d_prog, int nops) {
+void launch_k(const LaunchCtx& ctx, const FProg& P) {
   const size_t smem = size_t(16) << K;
   ensure_smem_attr((const void*)k_fused<K>, (int)smem);
   const uint64_t tiles = 1ull << (ctx.n_local - K);
-  k_fused<K><<<(unsigned)tiles, kFThreads, smem, ctx.stream>>>(
-      reinterpret_cast<double2*>(ctx.amps), d_prog, nops);
+  k_fused<K><<<(unsigned)tiles, kFThreads, smem, ctx.stream>>>(reinterpret_cast<double2*>(ctx.amps),
+                                                                P);
 }
 
 }  // namespace
@@ -436,31 +474,25 @@ bool run_fused_circuit(const LaunchCtx& ctx, const std::vector<Decoded>& gates, 
   int K = tile_qubits < ctx.n_local ? tile_qubits : ctx.n_local;
   if (K > kMaxK) K = kMaxK;
   if (K < kMinK) return false;
+  // Count the run first: a single gate runs faster in its class kernel.
   size_t i = begin;
-  int nops = 0;
-  while (i < end && nops < kMaxOps && fusable(gates[i], K, ctx.n_local)) {
-    if (gates[i].cls != GClass::NOOP) ++nops;
+  int real = 0;
+  while (i < end && fusable(gates[i], K, ctx.n_local) && real < 2) {
+    if (gates[i].cls != GClass::NOOP) ++real;
     ++i;
   }
-  if (nops < 2) return false;  // a single gate runs faster in its class kernel
-  // Program buffer owned by the state; reuse is stream-ordered (this upload is
-  // queued after the previous fused kernel).  The host vector is pageable, so
-  // cudaMemcpyAsync stages it before returning and no host sync is needed.
-  if (*ctx.fused_prog == nullptr)
-    LFQS_CUDA_CHECK(cudaMalloc(ctx.fused_prog, sizeof(FOp) * kMaxOps));
-  FOp* d_prog = static_cast<FOp*>(*ctx.fused_prog);
-  std::vector<FOp> h(nops);
-  int o = 0;
-  for (size_t q = begin; q < i; ++q)
-    if (gates[q].cls != GClass::NOOP) encode(gates[q], K, &h[o++]);
-  LFQS_CUDA_CHECK(cudaMemcpyAsync(d_prog, h.data(), sizeof(FOp) * o, cudaMemcpyHostToDevice,
-                                  ctx.stream));
+  if (real < 2) return false;
+  static thread_local FProg P;  // ~32 KB, reused (copied into the launch)
+  P.nops = 0;
+  P.ncoef = 0;
+  i = begin;
+  while (i < end && fusable(gates[i], K, ctx.n_local) && encode(gates[i], K, P)) ++i;
   switch (K) {
-    case 8: launch_k<8>(ctx, d_prog, o); break;
-    case 9: launch_k<9>(ctx, d_prog, o); break;
-    case 10: launch_k<10>(ctx, d_prog, o); break;
-    case 11: launch_k<11>(ctx, d_prog, o); break;
-    default: launch_k<12>(ctx, d_prog, o); break;
+    case 8: launch_k<8>(ctx, P); break;
+    case 9: launch_k<9>(ctx, P); break;
+    case 10: launch_k<10>(ctx, P); break;
+    case 11: launch_k<11>(ctx, P); break;
+    default: launch_k<12>(ctx, P); break;
   }
   LFQS_CUDA_CHECK(cudaGetLastError());
   ++*ctx.launch_counter;

@@ -93,7 +93,6 @@ struct LaunchCtx {
   cudaStream_t stream;
   uint64_t* launch_counter;
   const Options* opt;
-  void** fused_prog;       // state-owned device buffer for fused gate programs
 };
 
 // Raises a kernel's dynamic shared memory limit once per device.

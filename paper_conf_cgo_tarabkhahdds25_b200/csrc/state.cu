@@ -138,7 +138,6 @@ State::~State() {
   if (owned && amps) cudaFree(amps);
   if (d_partials) cudaFree(d_partials);
   if (d_probs) cudaFree(d_probs);
-  if (d_fused_prog) cudaFree(d_fused_prog);
   if (own_stream && stream) cudaStreamDestroy(stream);
 }
 
@@ -164,7 +163,6 @@ LaunchCtx State::ctx(int shard) {
   c.stream = stream;
   c.launch_counter = &launches;
   c.opt = &opt;
-  c.fused_prog = &d_fused_prog;
   return c;
 }
 

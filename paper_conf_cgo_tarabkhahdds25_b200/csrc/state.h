@@ -30,7 +30,6 @@ struct State : lfqs_state {
   Options opt;
   double* d_partials = nullptr; // reduction scratch
   double* d_probs = nullptr;
-  void* d_fused_prog = nullptr; // fused gate program buffer (fused_kernels.cu)
   int l2p[64], p2l[64];
   Comm* comm = nullptr;
   // exchange statistics (benchmark accounting)
