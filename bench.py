@@ -294,7 +294,7 @@ def main():
         c = classes.setdefault(cls, {"gates": 0, "ms": 0.0, "alg_bytes": 0.0, "conv_bytes": 0.0})
         c["gates"] += 1
         c["ms"] += mean_ms[i]
-        c["alg_bytes"] += 32.0 * W.touched_amplitudes(g, n_loc)
+        c["alg_bytes"] += W.algorithmic_bytes(g, n_loc)
         c["conv_bytes"] += 32.0 * 2 ** n_loc
     hbm_peak, peak_src = peaks()
     for c in classes.values():
@@ -320,7 +320,7 @@ def main():
     if args.per_gate_json and rank == 0:
         with open(args.per_gate_json, "w") as f:
             json.dump([{"cls": cls, "gate": g.label(), "ms": float(mean_ms[i]),
-                        "alg_bytes": 32.0 * W.touched_amplitudes(g, n_loc)}
+                        "alg_bytes": W.algorithmic_bytes(g, n_loc)}
                        for i, (cls, g) in enumerate(sweep)], f, indent=0)
 
     # end to end through the public API: H2D of the input state from pinned host

@@ -75,7 +75,7 @@ def main():
             torch.cuda.synchronize()
             if args.time:
                 ms = [ev[r].elapsed_time(ev[r + 1]) for r in range(args.reps)]
-                alg = 32.0 * W.touched_amplitudes(g, args.n)
+                alg = W.algorithmic_bytes(g, args.n)
                 print(f"{g.label():28s} mean {np.mean(ms):8.3f} ms  min {np.min(ms):8.3f} ms  "
                       f"alg {alg / np.min(ms) / 1e6:8.1f} GB/s  conv {32 * 2 ** args.n / np.min(ms) / 1e6:8.1f} GB/s",
                       flush=True)

@@ -368,6 +368,22 @@ def sweep_gates(n: int, seed: int = 0x5EED) -> List[Tuple[str, Gate]]:
     return out
 
 
+def algorithmic_bytes(g: Gate, n: int) -> float:
+    """SURVEY.md §8(d) algorithmic bytes of one gate pass (accounting, not arithmetic).
+
+    32 B per touched amplitude (16 read + 16 written).  Exception (§8(d)): when the
+    touched/untouched split falls on bit 0 -- qubit 0 is a control, a one-entry
+    diagonal (Z/S/T/Phase...) targets qubit 0, or a SWAP involves qubit 0 -- every
+    32-byte DRAM sector holds one touched and one untouched amplitude, so the pass
+    reads 32 B and writes 16 B per touched amplitude (24 * 2^n for Z on qubit 0).
+    """
+    t = touched_amplitudes(g, n)
+    one_entry_diag = g.kind in ("Z", "S", "SDG", "T", "TDG", "PHASE")
+    split0 = (0 in g.controls) or (one_entry_diag and 0 in g.targets) or \
+        (g.kind == "SWAP" and 0 in g.targets)
+    return 48.0 * t if split0 else 32.0 * t
+
+
 def touched_amplitudes(g: Gate, n: int) -> int:
     """Amplitudes a gate reads+writes when only the changed subspace is touched
     (PAPER.md:495 in-place update "eliminate unnecessary calculations").  Used for
