@@ -156,6 +156,35 @@ lfqs_status lfqs_run_circuit(lfqs_state* s, const lfqs_gate* gates, size_t n_gat
 lfqs_status lfqs_measure_probs(lfqs_state* s, const int* qubits, int n_q, double* probs_out,
                                size_t probs_len);
 
+/* ---- planning (host only: no GPU needed) ------------------------------------ */
+/* The distributed planner as a query: the physical
+ * operations rank `rank` of `world` performs for gates[0..n_gates), in order.
+ *   kind = LFQS_PLAN_LOCAL: apply `gate` to the rank's shard of n - log2(world)
+ *     local qubits.  The gate is already rank-specialised (global controls
+ *     resolved, diagonals on global qubits folded) and always expressed as
+ *     UNITARYm with gate.matrix pointing at this op's `matrix` (row-major
+ *     interleaved).  Ranks whose global controls are 0 get no op.
+ *   kind = LFQS_PLAN_EXCHANGE: swap local bit position l with global position g:
+ *     this rank exchanges, in place, its amplitudes whose bit l equals
+ *     1 - bit (g - n_local) of `rank` with the same positions of partner rank
+ *     rank ^ 2^(g - n_local).
+ * canonicalize != 0 appends the ops that restore the identity qubit map.
+ * Returns LFQS_ERR_INVALID_ARG with *n_ops = required length if capacity is
+ * too small.  The ops array must outlive any use of gate.matrix. */
+#define LFQS_PLAN_LOCAL 0
+#define LFQS_PLAN_EXCHANGE 1
+typedef struct {
+  int32_t kind;
+  int32_t l;
+  int32_t g;
+  int32_t _pad;
+  lfqs_gate gate;
+  double matrix[128];
+} lfqs_plan_op;
+lfqs_status lfqs_plan_circuit(int n_qubits, int world, int rank, const lfqs_gate* gates,
+                              size_t n_gates, int canonicalize, lfqs_plan_op* ops,
+                              size_t capacity, size_t* n_ops);
+
 /* ---- misc ------------------------------------------------------------------- */
 lfqs_status lfqs_synchronize(lfqs_state* s);
 /* n_qubits, local qubits, rank, world, and the device pointer of the local shard. */

@@ -41,7 +41,7 @@ EXPORTS = [
     "lfqs_state_init_basis", "lfqs_state_init_random", "lfqs_copy_in", "lfqs_copy_out",
     "lfqs_apply_gate", "lfqs_run_circuit", "lfqs_measure_probs", "lfqs_synchronize",
     "lfqs_state_info", "lfqs_kernel_launches", "lfqs_set_option", "lfqs_last_error",
-    "lfqs_abi_version",
+    "lfqs_abi_version", "lfqs_plan_circuit",
 ]
 
 
@@ -62,6 +62,16 @@ class LfqsGate(C.Structure):
 
 
 assert C.sizeof(LfqsGate) == 72
+
+PLAN_LOCAL = 0
+PLAN_EXCHANGE = 1
+
+
+class LfqsPlanOp(C.Structure):
+    """Mirror of lfqs_plan_op."""
+    _fields_ = [("kind", C.c_int32), ("l", C.c_int32), ("g", C.c_int32), ("_pad", C.c_int32),
+                ("gate", LfqsGate), ("matrix", C.c_double * 128)]
+
 
 _lib = None
 
@@ -96,6 +106,9 @@ def lib():
             "lfqs_state_info": [vp, ip, ip, ip, ip, C.POINTER(vp)],
             "lfqs_kernel_launches": [vp, C.POINTER(u64)],
             "lfqs_set_option": [vp, C.c_int, C.c_int64],
+            "lfqs_plan_circuit": [C.c_int, C.c_int, C.c_int, C.POINTER(LfqsGate), C.c_size_t,
+                                  C.c_int, C.POINTER(LfqsPlanOp), C.c_size_t,
+                                  C.POINTER(C.c_size_t)],
         }
         for name, args in sig.items():
             f = getattr(L, name)
@@ -279,6 +292,43 @@ def lfqs_set_option(h: int, option: int, value: int):
 
 def lfqs_state_set_stream(h: int, stream=None):
     _check(lib().lfqs_state_set_stream(h, _stream_handle(stream)))
+
+
+class PlanGate:
+    """A LOCAL plan op's gate (duck-typed like workloads.Gate: kind/targets/controls/params/matrix)."""
+
+    def __init__(self, kind, targets, controls, matrix):
+        self.kind, self.targets, self.controls, self.matrix = kind, targets, controls, matrix
+        self.params = ()
+
+    def label(self):
+        return f"{self.kind}c{list(self.controls)}{list(self.targets)}"
+
+
+def lfqs_plan_circuit(n_qubits: int, world: int, rank: int, gates, canonicalize: bool = True):
+    """Host-only planner query (no GPU).  Returns a list of
+    ("local", PlanGate) and ("exchange", l, g) tuples for `rank` (include/lfqs.h)."""
+    arr, n, keep = marshal_gates(gates)
+    need = C.c_size_t(0)
+    rc = lib().lfqs_plan_circuit(n_qubits, world, rank, arr, n, int(canonicalize), None, 0,
+                                 C.byref(need))
+    if rc != 0 and need.value == 0:
+        _check(rc)
+    ops = (LfqsPlanOp * max(1, need.value))()
+    _check(lib().lfqs_plan_circuit(n_qubits, world, rank, arr, n, int(canonicalize), ops,
+                                   need.value, C.byref(need)))
+    out = []
+    for i in range(need.value):
+        o = ops[i]
+        if o.kind == PLAN_EXCHANGE:
+            out.append(("exchange", o.l, o.g))
+            continue
+        m = o.gate.n_targets
+        d = 1 << m
+        mat = np.array(o.matrix[: 2 * d * d]).view(np.complex128).reshape(d, d).copy()
+        ctrl = tuple(q for q in range(64) if (o.gate.control_mask >> q) & 1)
+        out.append(("local", PlanGate(KINDS[o.gate.kind], tuple(o.gate.targets[:m]), ctrl, mat)))
+    return out
 
 
 # ---- convenience class ----------------------------------------------------------

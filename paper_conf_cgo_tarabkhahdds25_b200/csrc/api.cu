@@ -13,6 +13,7 @@
 #include <vector>
 
 #include "lfqs_internal.h"
+#include "planner.h"
 #include "state.h"
 
 using namespace lfqs;
@@ -170,6 +171,84 @@ lfqs_status lfqs_run_circuit(lfqs_state* s, const lfqs_gate* gates, size_t n_gat
       }
     }
     st->run(dec, flags);
+  });
+}
+
+lfqs_status lfqs_plan_circuit(int n_qubits, int world, int rank, const lfqs_gate* gates,
+                              size_t n_gates, int canonicalize, lfqs_plan_op* ops,
+                              size_t capacity, size_t* n_ops) {
+  return guarded([&] {
+    require(n_ops != nullptr, "n_ops is NULL");
+    require(n_gates == 0 || gates != nullptr, "gates is NULL");
+    require(n_qubits >= 1 && n_qubits <= 40, "n_qubits must be in [1, 40]");
+    require(world >= 1 && rank >= 0 && rank < world, "bad rank / world");
+    Planner plan(n_qubits, world);
+    std::vector<PlanOp> raw;
+    for (size_t i = 0; i < n_gates; ++i) {
+      const lfqs_gate& G = gates[i];
+      require(G.n_controls == __builtin_popcountll(G.control_mask),
+              "gate " + std::to_string(i) + ": n_controls != popcount(control_mask)");
+      Decoded d = decode_gate(n_qubits, G.kind, G.targets, G.n_targets, G.control_mask, G.params,
+                              kind_nparams(G.kind), G.matrix);
+      if (world == 1) {
+        PlanOp op;
+        op.gate = d;
+        raw.push_back(op);
+      } else {
+        plan.plan_gate(d, raw);
+      }
+    }
+    if (canonicalize) plan.plan_canonicalize(raw);
+    // Rank-specialise and convert.
+    std::vector<lfqs_plan_op> out;
+    for (const PlanOp& op : raw) {
+      lfqs_plan_op o;
+      std::memset(&o, 0, sizeof o);
+      if (op.kind == PlanOp::EXCHANGE) {
+        o.kind = LFQS_PLAN_EXCHANGE;
+        o.l = op.l;
+        o.g = op.g;
+        out.push_back(o);
+        continue;
+      }
+      Decoded lg;
+      if (!plan.rank_local(op.gate, rank, &lg) || lg.cls == GClass::NOOP) continue;
+      o.kind = LFQS_PLAN_LOCAL;
+      if (lg.m == 0) {
+        // Scalar on the control-satisfying amplitudes: express as a 1-target gate.
+        const cplx c = lg.M[0];
+        int q = -1;
+        for (int b = 0; b < plan.n_local; ++b)
+          if (!(lg.cmask >> b & 1)) { q = b; break; }
+        lg.m = 1;
+        for (int i = 0; i < 4; ++i) lg.M[i] = cplx{0.0, 0.0};
+        if (q >= 0) {
+          lg.M[0] = c;
+          lg.M[3] = c;
+        } else {  // every local qubit is a control: move one into the target
+          q = 0;
+          lg.cmask &= ~1ull;
+          lg.M[0] = cplx{1.0, 0.0};
+          lg.M[3] = c;
+        }
+        lg.targets[0] = q;
+      }
+      const int d = 1 << lg.m;
+      o.gate.kind = LFQS_UNITARY1 + lg.m - 1;
+      o.gate.n_targets = lg.m;
+      for (int s = 0; s < lg.m; ++s) o.gate.targets[s] = lg.targets[s];
+      o.gate.control_mask = lg.cmask;
+      o.gate.n_controls = __builtin_popcountll(lg.cmask);
+      std::memcpy(o.matrix, lg.M, sizeof(cplx) * d * d);
+      out.push_back(o);
+    }
+    *n_ops = out.size();
+    require(ops != nullptr || out.empty(), "ops is NULL");
+    require(capacity >= out.size(), "capacity < required plan length (see *n_ops)");
+    for (size_t i = 0; i < out.size(); ++i) {
+      ops[i] = out[i];
+      if (ops[i].kind == LFQS_PLAN_LOCAL) ops[i].gate.matrix = ops[i].matrix;
+    }
   });
 }
 

@@ -1,16 +1,12 @@
-// state.cu -- state allocator, logical<->physical qubit map and the distributed
-// gate planner (components C10 and C12).
+// state.cu -- state allocator, shard layout, and executor of the planner's ops
+// (components C10 and C12).
 //
-// One GPU: the map is the identity and every gate is one launch_gate() pass.
-// P = 2^p ranks: rank r owns the amplitudes whose top p physical bits equal r.
-//   (i)  targets local, controls anywhere: global controls are a rank predicate;
-//   (ii) diagonal gate with global targets: the factor of the global bits is
-//        rank-constant -> a smaller diagonal on the local targets, no traffic;
-//   (iii) other gates with a global target g: swap g with the highest local
-//        position l that is not a target (half-shard exchange), then (i);
-//   SWAP(global, local) without controls is a relabel of the map (no traffic).
-// copy_out / copy_in canonicalise the map first; measure_probs translates the
-// measured qubits through the map instead (no data movement).
+// One GPU: the map is the identity and every gate is one launch_gate() pass (or
+// a fused pass, LFQS_FUSE_LOW).  P = 2^p ranks (NCCL) or P virtual shards in one
+// allocation: planner.cpp turns each logical gate into LOCAL ops (specialised per
+// rank) and EXCHANGE ops (half-shard swaps: NCCL send/recv, or a device swap
+// between virtual shards).  copy_out / copy_in canonicalise the map first;
+// measure_probs translates the measured qubits through it (no data movement).
 #include <cuda_runtime.h>
 
 #include <algorithm>
@@ -23,7 +19,7 @@
 
 namespace lfqs {
 
-// Defined in apply_kernels.cu.
+// Defined in apply_kernels.cu / fused_kernels.cu.
 void launch_half_swap(const LaunchCtx& ctx, int l, uint64_t partner_offset_amps);
 bool run_fused_circuit(const LaunchCtx& ctx, const std::vector<Decoded>& gates, size_t begin,
                        size_t end, int tile_qubits, size_t* consumed);
@@ -69,13 +65,13 @@ void State::common_init(int n_, int world_, int device_, cudaStream_t s) {
   }
   require(device_ >= 0 && device_ < ndev, "device index out of range");
   require(world_ >= 1 && log2_exact(world_) >= 0, "world size must be a power of two");
+  require(n_ >= 1 && n_ <= 40, "n_qubits must be in [1, 40]");
+  plan = Planner(n_, world_);
   n = n_;
   world = world_;
   p = log2_exact(world_);
-  n_local = n - p;
+  n_local = plan.n_local;
   device = device_;
-  require(n >= 1 && n <= 40, "n_qubits must be in [1, 40]");
-  require(world == 1 || n_local >= 4, "each shard needs at least 4 local qubits");
   LFQS_CUDA_CHECK(cudaSetDevice(device));
   if (s) {
     stream = s;
@@ -85,7 +81,6 @@ void State::common_init(int n_, int world_, int device_, cudaStream_t s) {
   }
   LFQS_CUDA_CHECK(cudaMalloc(&d_partials, sizeof(double) * probs_blocks() * 1024));
   LFQS_CUDA_CHECK(cudaMalloc(&d_probs, sizeof(double) * 1024));
-  reset_map();
 }
 
 State* State::create_local(int n, int device, cudaStream_t stream, void* borrowed) {
@@ -166,20 +161,10 @@ LaunchCtx State::ctx(int shard) {
   return c;
 }
 
-bool State::identity_map() const {
-  for (int q = 0; q < n; ++q)
-    if (l2p[q] != q) return false;
-  return true;
-}
-
-void State::reset_map() {
-  for (int q = 0; q < 64; ++q) l2p[q] = p2l[q] = q;
-}
-
 void State::init_basis(uint64_t index) {
   DeviceGuard dg(device);
   require(n >= 64 || index < (1ull << n), "basis index out of range");
-  reset_map();
+  plan.reset();
   for (int s = 0; s < n_shards(); ++s) {
     const uint64_t lo = (uint64_t)rank_of_shard(s) << n_local;
     const int64_t li = (index >= lo && index - lo < (1ull << n_local)) ? (int64_t)(index - lo) : -1;
@@ -189,7 +174,7 @@ void State::init_basis(uint64_t index) {
 
 void State::init_random(uint64_t seed) {
   DeviceGuard dg(device);
-  reset_map();
+  plan.reset();
   for (int s = 0; s < n_shards(); ++s)
     launch_init_random(ctx(s), seed, (uint64_t)rank_of_shard(s) << n_local);
 }
@@ -204,7 +189,7 @@ void State::copy(uint64_t offset, uint64_t count, double* host, bool to_device) 
   DeviceGuard dg(device);
   const uint64_t total = 1ull << n;
   require(offset <= total && count <= total - offset, "amplitude range out of bounds");
-  if (!identity_map()) canonicalize();
+  if (!plan.identity()) canonicalize();
   const uint64_t lo = virt ? 0 : (uint64_t)rank << n_local;
   const uint64_t hi = virt ? total : lo + (1ull << n_local);
   const uint64_t a = std::max(offset, lo), b = std::min(offset + count, hi);
@@ -221,68 +206,9 @@ void State::copy(uint64_t offset, uint64_t count, double* host, bool to_device) 
 }
 
 // ---------------------------------------------------------------------------
-// Gates
+// Executing planned ops
 // ---------------------------------------------------------------------------
-Decoded State::to_physical(const Decoded& g) const {
-  Decoded pg = g;
-  for (int s = 0; s < g.m; ++s) pg.targets[s] = l2p[g.targets[s]];
-  uint64_t cm = 0;
-  for (int q = 0; q < n; ++q)
-    if (g.cmask >> q & 1) cm |= 1ull << l2p[q];
-  pg.cmask = cm;
-  return pg;
-}
-
-bool State::rank_local(const Decoded& pg, int r, Decoded* out) const {
-  const uint64_t local_mask = (n_local >= 64) ? ~0ull : ((1ull << n_local) - 1);
-  const uint64_t gctrl = pg.cmask >> n_local;
-  if ((gctrl & (uint64_t)r) != gctrl) return false;  // a global control is 0 on this rank
-  *out = pg;
-  out->cmask = pg.cmask & local_mask;
-  bool all_local = true;
-  for (int s = 0; s < pg.m; ++s) all_local &= pg.targets[s] < n_local;
-  if (all_local) return true;
-  require(pg.cls == GClass::DIAG, "internal: non-diagonal gate with a global target");
-  // Diagonal: fold the rank's global target bits into a smaller diagonal.
-  const int d = 1 << pg.m;
-  int lt[3], ls[3], mp = 0;
-  for (int s = 0; s < pg.m; ++s)
-    if (pg.targets[s] < n_local) {
-      lt[mp] = pg.targets[s];
-      ls[mp] = s;
-      ++mp;
-    }
-  cplx dd[8];
-  for (int jp = 0; jp < (1 << mp); ++jp) {
-    int j = 0;
-    for (int s = 0, u = 0; s < pg.m; ++s) {
-      int bit;
-      if (u < mp && ls[u] == s) {
-        bit = (jp >> (mp - 1 - u)) & 1;
-        ++u;
-      } else {
-        bit = (r >> (pg.targets[s] - n_local)) & 1;
-      }
-      j |= bit << (pg.m - 1 - s);
-    }
-    dd[jp] = pg.M[j * d + j];
-  }
-  out->m = mp;
-  for (int s = 0; s < 3; ++s) out->targets[s] = s < mp ? lt[s] : 0;
-  const int dp = 1 << mp;
-  for (int i = 0; i < dp * dp; ++i) out->M[i] = cplx{0.0, 0.0};
-  bool ones = true;
-  for (int j = 0; j < dp; ++j) {
-    out->M[j * dp + j] = dd[j];
-    ones &= dd[j].re == 1.0 && dd[j].im == 0.0;
-  }
-  out->cls = ones ? GClass::NOOP : GClass::DIAG;
-  out->is_h = false;
-  return true;
-}
-
-void State::exchange(int l, int g) {
-  require(l >= 0 && l < n_local && g >= n_local && g < n, "internal: bad exchange positions");
+void State::exchange_data(int l, int g) {
   const int j = g - n_local;
   if (virt) {
     for (int r = 0; r < world; ++r) {
@@ -303,62 +229,25 @@ void State::exchange(int l, int g) {
   }
   ++exchanges;
   exchange_bytes += 16ull << (n_local - 1);
-  const int qa = p2l[l], qb = p2l[g];
-  l2p[qa] = g;
-  l2p[qb] = l;
-  p2l[l] = qb;
-  p2l[g] = qa;
 }
 
-void State::swap_local(int a, int b) {
-  const int t[2] = {a, b};
-  Decoded sw = decode_gate(n_local, LFQS_SWAP, t, 2, 0, nullptr, 0, nullptr);
-  for (int s = 0; s < n_shards(); ++s) launch_gate(ctx(s), sw);
-  const int qa = p2l[a], qb = p2l[b];
-  l2p[qa] = b;
-  l2p[qb] = a;
-  p2l[a] = qb;
-  p2l[b] = qa;
-}
-
-void State::canonicalize() {
-  for (int q = 0; q < n; ++q) {
-    const int P = l2p[q];
-    if (P == q) continue;
-    const bool pl = P < n_local, ql = q < n_local;
-    if (pl && ql) {
-      swap_local(P, q);
-    } else if (pl != ql) {
-      exchange(pl ? P : q, pl ? q : P);
-    } else {
-      const int L = n_local - 1;  // any local position
-      exchange(L, P);
-      exchange(L, q);
-      exchange(L, P);
+void State::execute(const std::vector<PlanOp>& ops) {
+  for (const PlanOp& op : ops) {
+    if (op.kind == PlanOp::EXCHANGE) {
+      exchange_data(op.l, op.g);
+      continue;
+    }
+    for (int s = 0; s < n_shards(); ++s) {
+      Decoded lg;
+      if (plan.rank_local(op.gate, rank_of_shard(s), &lg)) launch_gate(ctx(s), lg);
     }
   }
 }
 
-void State::ensure_local_targets(Decoded& pg) {
-  for (int s = 0; s < pg.m; ++s) {
-    const int g = pg.targets[s];
-    if (g < n_local) continue;
-    uint64_t tmask = 0;
-    for (int u = 0; u < pg.m; ++u) tmask |= 1ull << pg.targets[u];
-    int l = n_local - 1;
-    while (l >= 0 && (tmask >> l & 1)) --l;
-    require(l >= 0, "internal: no free local qubit");
-    exchange(l, g);
-    pg.targets[s] = l;
-    if (pg.cmask >> l & 1) pg.cmask = (pg.cmask & ~(1ull << l)) | (1ull << g);
-  }
-}
-
-void State::apply_physical(const Decoded& pg) {
-  for (int s = 0; s < n_shards(); ++s) {
-    Decoded lg;
-    if (rank_local(pg, rank_of_shard(s), &lg)) launch_gate(ctx(s), lg);
-  }
+void State::canonicalize() {
+  std::vector<PlanOp> ops;
+  plan.plan_canonicalize(ops);
+  execute(ops);
 }
 
 void State::apply(const Decoded& g) {
@@ -367,19 +256,9 @@ void State::apply(const Decoded& g) {
     launch_gate(ctx(0), g);
     return;
   }
-  Decoded pg = to_physical(g);
-  if (pg.cls == GClass::NOOP) return;
-  if (pg.cls == GClass::PERM_SWAP && pg.cmask == 0 &&
-      (pg.targets[0] >= n_local || pg.targets[1] >= n_local)) {
-    // SWAP of logical qubits = relabel: exchange their physical positions in the map.
-    const int qa = g.targets[0], qb = g.targets[1];
-    std::swap(l2p[qa], l2p[qb]);
-    p2l[l2p[qa]] = qa;
-    p2l[l2p[qb]] = qb;
-    return;
-  }
-  if (pg.cls != GClass::DIAG) ensure_local_targets(pg);
-  apply_physical(pg);
+  std::vector<PlanOp> ops;
+  plan.plan_gate(g, ops);
+  execute(ops);
 }
 
 void State::run(const std::vector<Decoded>& gates, uint32_t flags) {
@@ -411,7 +290,7 @@ void State::measure_probs(const int* qubits, int nq, double* out) {
   }
   int lq[10], ls[10], nl = 0;
   for (int s = 0; s < nq; ++s) {
-    const int P = l2p[qubits[s]];
+    const int P = plan.l2p[qubits[s]];
     if (P < n_local) {
       lq[nl] = P;
       ls[nl] = s;
@@ -427,7 +306,7 @@ void State::measure_probs(const int* qubits, int nq, double* out) {
     LFQS_CUDA_CHECK(cudaStreamSynchronize(stream));
     int gbits = 0;
     for (int s = 0; s < nq; ++s) {
-      const int P = l2p[qubits[s]];
+      const int P = plan.l2p[qubits[s]];
       if (P >= n_local) gbits |= ((r >> (P - n_local)) & 1) << s;
     }
     for (int lb = 0; lb < (1 << nl); ++lb) {

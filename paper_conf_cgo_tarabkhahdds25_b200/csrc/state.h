@@ -1,4 +1,4 @@
-// state.h -- the state allocator, qubit map and distributed planner.
+// state.h -- the state allocator and executor of planned ops.
 #pragma once
 #include <cuda_runtime.h>
 
@@ -6,6 +6,7 @@
 #include <vector>
 
 #include "lfqs_internal.h"
+#include "planner.h"
 
 struct lfqs_state {
   virtual ~lfqs_state() = default;
@@ -15,10 +16,10 @@ namespace lfqs {
 
 struct Comm;  // NCCL communicator wrapper (comm.cu)
 
-// Layout in HBM (DESIGN.md §5): a shard is 2^n_local interleaved complex128
+// Layout in HBM (DESIGN.md §4): a shard is 2^n_local interleaved complex128
 // amplitudes, contiguous, 256-byte aligned.  Physical bit positions
 // [0, n_local) are local; [n_local, n) are "global" and equal the rank's bits.
-// l2p maps a logical qubit to its physical position (identity on one GPU).
+// The planner's l2p maps a logical qubit to its physical position.
 struct State : lfqs_state {
   int n = 0, n_local = 0, rank = 0, world = 1, p = 0, device = 0;
   bool virt = false;            // `world` shards in one allocation (single GPU)
@@ -30,7 +31,7 @@ struct State : lfqs_state {
   Options opt;
   double* d_partials = nullptr; // reduction scratch
   double* d_probs = nullptr;
-  int l2p[64], p2l[64];
+  Planner plan;
   Comm* comm = nullptr;
   // exchange statistics (benchmark accounting)
   uint64_t exchanges = 0, exchange_bytes = 0;
@@ -58,15 +59,9 @@ struct State : lfqs_state {
   LaunchCtx ctx(int shard);
   int n_shards() const { return virt ? world : 1; }
   int rank_of_shard(int shard) const { return virt ? shard : rank; }
-  bool identity_map() const;
-  void reset_map();
-  Decoded to_physical(const Decoded& g) const;
-  bool rank_local(const Decoded& pg, int r, Decoded* out) const;
-  void ensure_local_targets(Decoded& pg);
-  void exchange(int l, int g);   // swap physical positions l (local) and g (global)
-  void swap_local(int a, int b); // swap two local physical positions (data)
+  void execute(const std::vector<PlanOp>& ops);
+  void exchange_data(int l, int g);  // swap physical positions l (local) and g (global)
   void canonicalize();
-  void apply_physical(const Decoded& pg);
 };
 
 }  // namespace lfqs
