@@ -31,6 +31,7 @@ OPT_LOWQ_SHUFFLE = 1
 OPT_FUSE_TILE_QUBITS = 2
 OPT_ITEMS_PER_THREAD = 3
 OPT_WIDE256 = 4
+OPT_FUSE_LOW_QUBITS = 5
 
 STATUS = {0: "OK", -1: "INVALID_ARG", -2: "OUT_OF_MEMORY", -3: "CUDA", -4: "NCCL",
           -5: "UNSUPPORTED"}

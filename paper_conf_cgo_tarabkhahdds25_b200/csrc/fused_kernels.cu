@@ -43,10 +43,20 @@ struct FHdr {       // 32 bytes
   uint64_t mhi, phi;  // per-tile predicate     (base & mhi) == phi (bits >= K)
 };
 constexpr int kMaxOps = 192;
-constexpr int kMaxCoef = 1600;
+constexpr int kMaxCoef = 1580;
+constexpr int kMaxHigh = 8;
+// Tile geometry: tile bits [0, lc) are qubits [0, lc) (one contiguous chunk of
+// 2^lc amplitudes); tile bits lc + i are the "high" qubits hpos[i] (ascending).
+// The tile is 2^(K - lc) chunks, each moved by one TMA bulk copy.
+struct FTile {
+  int lc;
+  int nh;
+  uint8_t hpos[kMaxHigh];
+};
 struct FProg {
   int nops;
   int ncoef;
+  FTile tile;
   FHdr h[kMaxOps];
   double2 c[kMaxCoef];
 };
@@ -255,19 +265,31 @@ __global__ void __launch_bounds__(kFThreads, 2) k_fused(double2* __restrict__ a,
   extern __shared__ __align__(128) double2 tile[];
   __shared__ __align__(8) uint64_t bar;
   const uint32_t tid = threadIdx.x;
-  const uint64_t base = (uint64_t)blockIdx.x << K;
-  const uint32_t bytes = T * 16u;
+  const FTile& tg = prog.tile;
+  const int lc = tg.lc, nh = tg.nh;
+  // Tile base: the tile index with zeros inserted at every tile qubit.
+  uint64_t base = (uint64_t)blockIdx.x << lc;
+  for (int i = 0; i < nh; ++i) {
+    const int p = tg.hpos[i];
+    const uint64_t lo = base & ((1ull << p) - 1);
+    base = ((base - lo) << 1) | lo;
+  }
+  const uint32_t bytes = T * 16u, chunk_bytes = 16u << lc;
   const uint32_t bar_a = smem_u32(&bar), tile_a = smem_u32(tile);
   if (tid == 0) {
     asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(bar_a));
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar_a), "r"(bytes)
                  : "memory");
-    asm volatile(
-        "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::
-            "r"(tile_a),
-        "l"(a + base), "r"(bytes), "r"(bar_a)
-        : "memory");
+    for (uint32_t ch = 0; ch < (1u << nh); ++ch) {
+      uint64_t off = base;
+      for (int i = 0; i < nh; ++i) off |= (uint64_t)((ch >> i) & 1) << tg.hpos[i];
+      asm volatile(
+          "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::
+              "r"(tile_a + ch * chunk_bytes),
+          "l"(a + off), "r"(chunk_bytes), "r"(bar_a)
+          : "memory");
+    }
   }
   __syncthreads();  // barrier initialised before anyone waits on it
   {
@@ -328,8 +350,8 @@ __global__ void __launch_bounds__(kFThreads, 2) k_fused(double2* __restrict__ a,
 #pragma unroll
         for (int s = 0; s < 3; ++s)
           if (s < m) {
-            if (ts[s] >= K)
-              jh |= (uint32_t)((base >> ts[s]) & 1) << (m - 1 - s);
+            if (ts[s] >= 64)  // a qubit outside the tile: its bit comes from the tile base
+              jh |= (uint32_t)((base >> (ts[s] - 64)) & 1) << (m - 1 - s);
             else
               jmask |= 1u << (m - 1 - s);
           }
@@ -368,9 +390,13 @@ __global__ void __launch_bounds__(kFThreads, 2) k_fused(double2* __restrict__ a,
   asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
   __syncthreads();
   if (tid == 0) {
-    asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;" ::"l"(a + base),
-                 "r"(tile_a), "r"(bytes)
-                 : "memory");
+    for (uint32_t ch = 0; ch < (1u << nh); ++ch) {
+      uint64_t off = base;
+      for (int i = 0; i < nh; ++i) off |= (uint64_t)((ch >> i) & 1) << tg.hpos[i];
+      asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;" ::"l"(a + off),
+                   "r"(tile_a + ch * chunk_bytes), "r"(chunk_bytes)
+                   : "memory");
+    }
     asm volatile("cp.async.bulk.commit_group;" ::: "memory");
     asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
   }
@@ -387,18 +413,35 @@ int coef_count(const Decoded& g) {
   }
 }
 
-// Appends gate g to the program; returns false if it does not fit.
-bool encode(const Decoded& g, int K, FProg& P) {
-  if (g.cls == GClass::NOOP) return true;
-  if (P.nops >= kMaxOps || P.ncoef + coef_count(g) > kMaxCoef) return false;
+// tb[q] = tile bit of qubit q, or -1 when q is not a tile qubit.
+struct TileMap {
+  int tb[64];
+};
+
+// Appends gate g to the program (program space was checked by the caller).
+void encode(const Decoded& g, const TileMap& tm, FProg& P) {
+  if (g.cls == GClass::NOOP) return;
   FHdr& h = P.h[P.nops];
   std::memset(&h, 0, sizeof h);
-  const uint64_t lowmask = (1ull << K) - 1;
-  uint64_t m_all = g.cmask, p_all = g.cmask;
+  uint64_t mlo = 0, plo = 0, mhi = 0, phi = 0;
+  // A fixed bit of qubit q with value b: a per-amplitude condition on its tile
+  // bit, or a per-tile condition on the global bit when q is not in the tile.
+  auto fix = [&](int q, int b) {
+    if (tm.tb[q] >= 0) {
+      mlo |= 1ull << tm.tb[q];
+      plo |= (uint64_t)b << tm.tb[q];
+    } else {
+      mhi |= 1ull << q;
+      phi |= (uint64_t)b << q;
+    }
+  };
+  for (int q = 0; q < 64; ++q)
+    if (g.cmask >> q & 1) fix(q, 1);
+  auto tbit = [&](int s) { return tm.tb[g.targets[s]] >= 0 ? tm.tb[g.targets[s]] : 64 + g.targets[s]; };
   h.m = (uint8_t)g.m;
-  h.t0 = (uint8_t)g.targets[0];
-  h.t1 = (uint8_t)(g.m > 1 ? g.targets[1] : 0);
-  h.t2 = (uint8_t)(g.m > 2 ? g.targets[2] : 0);
+  h.t0 = (uint8_t)tbit(0);
+  h.t1 = (uint8_t)(g.m > 1 ? tbit(1) : 0);
+  h.t2 = (uint8_t)(g.m > 2 ? tbit(2) : 0);
   h.coef = (uint16_t)P.ncoef;
   const int d = 1 << g.m;
   switch (g.cls) {
@@ -411,13 +454,10 @@ bool encode(const Decoded& g, int K, FProg& P) {
           active = j;
         }
       }
-      if (n_active == 0) return true;
+      if (n_active == 0) return;
       if (n_active == 1) {
         h.type = F_DIAG1;
-        for (int s = 0; s < g.m; ++s) {
-          m_all |= 1ull << g.targets[s];
-          p_all |= (uint64_t)((active >> (g.m - 1 - s)) & 1) << g.targets[s];
-        }
+        for (int s = 0; s < g.m; ++s) fix(g.targets[s], (active >> (g.m - 1 - s)) & 1);
         P.c[P.ncoef++] = D2(g.M[active * d + active]);
       } else {
         h.type = F_DIAGN;
@@ -441,12 +481,11 @@ bool encode(const Decoded& g, int K, FProg& P) {
       }
       break;
   }
-  h.mlo = (uint32_t)(m_all & lowmask);
-  h.plo = (uint32_t)(p_all & lowmask);
-  h.mhi = m_all & ~lowmask;
-  h.phi = p_all & ~lowmask;
+  h.mlo = (uint32_t)mlo;
+  h.plo = (uint32_t)plo;
+  h.mhi = mhi;
+  h.phi = phi;
   ++P.nops;
-  return true;
 }
 
 template <int K>
@@ -468,25 +507,63 @@ bool fusable(const Decoded& g, int K, int n_local) {
   return true;
 }
 
+// Greedy segmentation (NEXT-1 "general cache-blocked fusion"): the tile holds
+// qubits [0, L) (contiguous, for coalesced 2^L-amplitude chunks) plus up to
+// K - L further qubits claimed, in gate order, by the targets of non-diagonal
+// gates; diagonal gates need no slot.  Free slots are filled with the lowest
+// remaining qubits (larger contiguous chunks).
 bool run_fused_circuit(const LaunchCtx& ctx, const std::vector<Decoded>& gates, size_t begin,
                        size_t end, int tile_qubits, size_t* consumed) {
   *consumed = 0;
   int K = tile_qubits < ctx.n_local ? tile_qubits : ctx.n_local;
   if (K > kMaxK) K = kMaxK;
   if (K < kMinK) return false;
-  // Count the run first: a single gate runs faster in its class kernel.
+  int L = ctx.opt->fuse_low_qubits;
+  if (L > K) L = K;
+  if (L < K - kMaxHigh) L = K - kMaxHigh;
+  const int slots = K - L;
+  uint64_t in_tile = (L >= 64) ? ~0ull : ((1ull << L) - 1);
+  int used = 0, nops = 0, ncoef = 0;
   size_t i = begin;
-  int real = 0;
-  while (i < end && fusable(gates[i], K, ctx.n_local) && real < 2) {
-    if (gates[i].cls != GClass::NOOP) ++real;
-    ++i;
+  for (; i < end; ++i) {
+    const Decoded& g = gates[i];
+    if (g.cls == GClass::NOOP) continue;
+    if (nops >= kMaxOps || ncoef + coef_count(g) > kMaxCoef) break;
+    if (g.cls != GClass::DIAG) {
+      uint64_t need = 0;
+      for (int s = 0; s < g.m; ++s)
+        if (!(in_tile >> g.targets[s] & 1)) need |= 1ull << g.targets[s];
+      const int nn = __builtin_popcountll(need);
+      if (used + nn > slots) break;
+      in_tile |= need;
+      used += nn;
+    }
+    ++nops;
+    ncoef += coef_count(g);
   }
-  if (real < 2) return false;
+  if (nops < 2) return false;  // a single gate runs faster in its class kernel
+  for (int q = 0; q < ctx.n_local && __builtin_popcountll(in_tile) < K; ++q) in_tile |= 1ull << q;
+  TileMap tm;
   static thread_local FProg P;  // ~32 KB, reused (copied into the launch)
   P.nops = 0;
   P.ncoef = 0;
-  i = begin;
-  while (i < end && fusable(gates[i], K, ctx.n_local) && encode(gates[i], K, P)) ++i;
+  int b = 0, lc = 0;
+  P.tile.nh = 0;
+  for (int q = 0; q < 64; ++q) {
+    tm.tb[q] = -1;
+    if (q < ctx.n_local && (in_tile >> q & 1)) {
+      tm.tb[q] = b;
+      if (b == q) {
+        lc = q + 1;
+      } else {
+        P.tile.hpos[P.tile.nh++] = (uint8_t)q;
+      }
+      ++b;
+    }
+  }
+  P.tile.lc = lc;
+  require(b == K && lc + P.tile.nh == K, "internal: bad fused tile");
+  for (size_t q = begin; q < i; ++q) encode(gates[q], tm, P);
   switch (K) {
     case 8: launch_k<8>(ctx, P); break;
     case 9: launch_k<9>(ctx, P); break;

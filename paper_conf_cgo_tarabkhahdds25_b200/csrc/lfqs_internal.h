@@ -83,6 +83,7 @@ struct Options {
   bool lowq_shuffle = false;
   bool wide256 = true;       // two adjacent groups per item, 32-byte accesses
   int fuse_tile_qubits = 12;
+  int fuse_low_qubits = 7;   // contiguous low qubits of a fused tile (chunk = 2^7 amps)
   int items_per_thread = 0;  // 0 = library default
 };
 

@@ -48,6 +48,31 @@ def test_fused_random_circuit(L, n, tile):
     assert np.array_equal(a, b)
 
 
+@pytest.mark.parametrize("low", [3, 5, 7, 12])
+def test_fused_general_tiles(L, low):
+    """Tiles = qubits [0, low) + qubits claimed by the gates (NEXT-1), chunked TMA copies."""
+    n = 18
+    psi = W.random_state(n, low)
+    gates = W.random_gate_list(n, 200, seed=100 + low, max_controls=2) + W.qft(n) + \
+        W.random_layered(n, 4, seed=low)
+    ref = O.run_circuit(n, gates, psi.copy())
+    with L.State.create(n) as st:
+        st.set_option(L.OPT_FUSE_LOW_QUBITS, low)
+        st.copy_in(psi)
+        c0 = st.launches()
+        st.run_circuit(gates, fuse=True)
+        passes = st.launches() - c0
+        got = st.copy_out()
+    assert np.max(np.abs(got - ref)) <= 1e-12
+    assert passes < len(gates) // 3
+    exact = [g for g in gates if g.exact]
+    with L.State.create(n) as st:
+        st.set_option(L.OPT_FUSE_LOW_QUBITS, low)
+        st.copy_in(psi)
+        st.run_circuit(exact, fuse=True)
+        assert np.array_equal(st.copy_out(), O.run_circuit(n, exact, psi.copy()))
+
+
 def test_fusion_reduces_passes_qft(L):
     n, x = 20, 0xBEEF1
     gates = W.qft(n)
