@@ -335,11 +335,14 @@ __global__ void __launch_bounds__(kFThreads, 2) k_fused(double2* __restrict__ a,
     }
     switch (type) {
       case F_DIAG1: {  // one diagonal entry d != 1 on the amplitudes matching the predicate
+        // Split the predicate: register bits (warp-uniform -> branch) and thread bits.
         const double2 d = c[0];
+        const uint32_t mr = mlo >> 8, pr = plo >> 8;
+        const bool bt = (tid & mlo & (kFThreads - 1)) == (plo & (kFThreads - 1));
 #pragma unroll
         for (int r = 0; r < R; ++r) {
-          const uint32_t i = (uint32_t)r * kFThreads + tid;
-          if ((i & mlo) == plo) v[r] = cmul_rn(d, v[r]);
+          if (((uint32_t)r & mr) != pr) continue;  // uniform across the block
+          if (bt) v[r] = cmul_rn(d, v[r]);
         }
         break;
       }
@@ -398,7 +401,9 @@ __global__ void __launch_bounds__(kFThreads, 2) k_fused(double2* __restrict__ a,
                    : "memory");
     }
     asm volatile("cp.async.bulk.commit_group;" ::: "memory");
-    asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
+    // Only the shared-memory source must outlive the copy; completion of the
+    // global writes is ordered by the end of the grid (as in TMA-store epilogues).
+    asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");
   }
 }
 

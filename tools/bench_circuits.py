@@ -65,6 +65,10 @@ def main():
         "ghz": (W.ghz(n), lambda st: st.init_basis(0), {}),
         "grover": (W.grover(n, w, 2), lambda st: st.init_basis(0), {"k": 2, "w": w}),
         "random": (W.random_layered(n, 20, seed=7), lambda st: st.init_basis(0), {}),
+        # light programs: fused-pass memory efficiency (one H per qubit; X pairs)
+        "hlayer": ([W.Gate("H", (q,)) for q in range(n)], lambda st: st.init_basis(0), {}),
+        "xlow": ([W.Gate("X", (0,)), W.Gate("X", (1,))], lambda st: st.init_basis(0), {}),
+        "xhigh": ([W.Gate("X", (n - 1,)), W.Gate("X", (n - 5,))], lambda st: st.init_basis(0), {}),
     }
     with L.State.create(n, 0, stream=s) as st:
         if args.tile:
