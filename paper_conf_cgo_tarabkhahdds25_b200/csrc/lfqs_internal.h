@@ -102,12 +102,10 @@ void ensure_smem_attr(const void* kernel, int bytes);
 // Applies one decoded gate whose targets are all < n_local (controls < n_local).
 void launch_gate(const LaunchCtx& ctx, const Decoded& g);
 
-// Diagonal-only fast path with an extra rank-constant mask: amplitudes whose
-// `global_ones` bits are implied by the rank.  Used by the distributed runner.
-// Fused low-qubit program; returns false if not applicable.
-struct FusedOp;
-void launch_fused(const LaunchCtx& ctx, const std::vector<Decoded>& gates, int tile_qubits);
-bool fusable(const Decoded& g, int tile_qubits, int n_local);
+// Fused staging of gates[begin..): applies the longest prefix that fits one tile
+// program in one HBM pass; false if fewer than two gates fuse (fused_kernels.cu).
+bool run_fused_circuit(const LaunchCtx& ctx, const std::vector<Decoded>& gates, size_t begin,
+                       size_t end, int tile_qubits, size_t* consumed);
 
 // Reductions (C9): out[v], v < 2^nq; deterministic.
 void launch_probs(const LaunchCtx& ctx, const int* qubits, int nq, double* d_partials,

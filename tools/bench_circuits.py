@@ -52,6 +52,7 @@ def main():
     ap.add_argument("--modes", default="fused,unfused")
     ap.add_argument("--reps", type=int, default=2)
     ap.add_argument("--tile", type=int, default=0)
+    ap.add_argument("--low", type=int, default=0)
     args = ap.parse_args()
     import torch
     import paper_conf_cgo_tarabkhahdds25_b200 as L
@@ -73,6 +74,8 @@ def main():
     with L.State.create(n, 0, stream=s) as st:
         if args.tile:
             st.set_option(L.OPT_FUSE_TILE_QUBITS, args.tile)
+        if args.low:
+            st.set_option(L.OPT_FUSE_LOW_QUBITS, args.low)
         for name in args.circuits.split(","):
             gates, init, meta = circuits[name]
             arr = L.marshal_gates(gates)
