@@ -4,30 +4,28 @@
 // state; the optimised kernel of each gate is one pass over S (vector
 // fusion).  On B200 a pass over a 16-128 GiB state costs 5-35 ms of
 // HBM time while the arithmetic of one gate costs far less, so a run of
-// consecutive gates that only mix amplitudes inside a tile of 2^K amplitudes
-// is applied in ONE pass (LFQS_FUSE_LOW):
-//   * a tile is qubits [0, lc) (one contiguous chunk of 2^lc amplitudes) plus
-//     up to 8 further qubits claimed, in gate order, by the targets of the
-//     fused gates (NEXT-1 "general cache-blocked fusion"); diagonal gates need
-//     no tile qubit (bits outside the tile come from the tile index);
-//   * persistent CTAs (one per SM, 512 threads) stream tiles through two
-//     shared-memory buffers: the TMA bulk copies (cp.async.bulk + mbarrier,
-//     one copy per chunk, issued by the 32 lanes of warp 0) of tile j+1 and
-//     the bulk stores of tile j-1 overlap the arithmetic of tile j;
+// consecutive gates that only mix amplitudes inside a 2^K tile is applied in
+// ONE pass (LFQS_FUSE_LOW):
+//   * the tile (2^K contiguous amplitudes, K <= 12 -> 64 KiB) is staged into
+//     shared memory with one TMA bulk copy (cp.async.bulk + mbarrier) and
+//     written back with one bulk store;
 //   * the gate program is a __grid_constant__ kernel parameter (<= 32 KB:
-//     headers + a coefficient pool), read through the constant cache;
-//   * amplitudes live in registers: thread `tid` holds tile elements
-//     i = r * 512 + tid.  Diagonal gates, and 1-target gates on register bits
-//     (9..K-1) or lane bits (0..4, via shfl.xor), are applied in registers;
-//     1-target gates on warp bits (5..8) and 2/3-target gates go through the
-//     shared-memory tile.
+//     headers + a coefficient pool), read through the constant cache -- no
+//     global-memory round trips inside the op loop;
+//   * amplitudes live in registers: thread `tid` of 256 holds tile elements
+//     i = r * 256 + tid, r < 2^(K-8).  Diagonal gates, and 1-target gates on
+//     register bits (8..K-1) or lane bits (0..4, via shfl.xor), are applied in
+//     registers; 1-target gates on warp bits (5..7) and 2/3-target gates go
+//     through the shared-memory tile;
+//   * a gate fuses when all its targets are < K (controls anywhere: controls
+//     >= K are a per-tile predicate) or when it is diagonal (any qubits: target
+//     bits >= K come from the tile index).
 // Permutation and diagonal gates use exactly the unfused formulas (moves;
 // RN complex multiply without FMA, skipped where the factor is exactly 1), so
 // fused == unfused value-exactly for them; dense gates agree within rounding.
 #include <cuda_runtime.h>
 
 #include <cstring>
-#include <mutex>
 #include <vector>
 
 #include "lfqs_internal.h"
@@ -41,14 +39,15 @@ enum FType : uint8_t { F_DIAG1 = 0, F_DIAGN, F_X, F_Y, F_H, F_U2, F_SWAP, F_U4, 
 struct FHdr {       // 32 bytes
   uint8_t type, m, t0, t1, t2, pad0;
   uint16_t coef;    // offset into the coefficient pool
-  uint32_t mlo, plo;  // per-amplitude predicate (i & mlo) == plo   (tile bits)
-  uint64_t mhi, phi;  // per-tile predicate     (base & mhi) == phi (qubits outside the tile)
+  uint32_t mlo, plo;  // per-amplitude predicate (i & mlo) == plo   (bits < K)
+  uint64_t mhi, phi;  // per-tile predicate     (base & mhi) == phi (bits >= K)
 };
 constexpr int kMaxOps = 192;
 constexpr int kMaxCoef = 1580;
 constexpr int kMaxHigh = 8;
-// Tile geometry: tile bits [0, lc) are qubits [0, lc); tile bits lc + i are the
-// qubits hpos[i] (ascending).  A tile is 2^(K - lc) chunks of 2^lc amplitudes.
+// Tile geometry: tile bits [0, lc) are qubits [0, lc) (one contiguous chunk of
+// 2^lc amplitudes); tile bits lc + i are the "high" qubits hpos[i] (ascending).
+// The tile is 2^(K - lc) chunks, each moved by one TMA bulk copy.
 struct FTile {
   int lc;
   int nh;
@@ -61,11 +60,10 @@ struct FProg {
   FHdr h[kMaxOps];
   double2 c[kMaxCoef];
 };
-static_assert(sizeof(FProg) + 16 <= 32764, "kernel parameter limit");
+static_assert(sizeof(FProg) + 8 <= 32764, "kernel parameter limit");
 
-constexpr int kFThreads = 512;
-constexpr int kRS = 9;  // log2(kFThreads): first register bit of the tile index
-constexpr int kMinK = 9, kMaxK = 12;
+constexpr int kFThreads = 256;
+constexpr int kMinK = 8, kMaxK = 12;
 
 __device__ __forceinline__ uint32_t smem_u32(const void* p) {
   return static_cast<uint32_t>(__cvta_generic_to_shared(p));
@@ -238,11 +236,12 @@ __device__ __forceinline__ void reg_pairs(double2 (&v)[R], const F& f, uint32_t 
 template <int R, class F>
 __device__ __forceinline__ void reg_1q(double2 (&v)[R], const F& f, int t0, uint32_t mlo,
                                        uint32_t plo, uint32_t tid) {
-  if (t0 >= kRS) {
-    switch (t0 - kRS) {
+  if (t0 >= 8) {
+    switch (t0 - 8) {
       case 0: reg_pairs<0, R>(v, f, mlo, plo, tid); break;
       case 1: reg_pairs<1, R>(v, f, mlo, plo, tid); break;
-      default: reg_pairs<2, R>(v, f, mlo, plo, tid); break;
+      case 2: reg_pairs<2, R>(v, f, mlo, plo, tid); break;
+      default: reg_pairs<3, R>(v, f, mlo, plo, tid); break;
     }
     return;
   }
@@ -258,16 +257,86 @@ __device__ __forceinline__ void reg_1q(double2 (&v)[R], const F& f, int t0, uint
   }
 }
 
-// Applies the gate program to one tile held in shared memory.
-template <int K>
-__device__ __forceinline__ void run_program(double2* tile, const FProg& prog, uint64_t base,
-                                            uint32_t tid) {
+__device__ __forceinline__ double2 ldcs(const double2* p) {
+  double2 v;
+  asm volatile("ld.global.cs.v2.f64 {%0,%1}, [%2];" : "=d"(v.x), "=d"(v.y) : "l"(p));
+  return v;
+}
+__device__ __forceinline__ void stcs(double2* p, double2 v) {
+  asm volatile("st.global.cs.v2.f64 [%0], {%1,%2};" ::"l"(p), "d"(v.x), "d"(v.y) : "memory");
+}
+// Global amplitude index of tile element i (chunk = i >> lc, offset = low lc bits).
+__device__ __forceinline__ uint64_t tile_addr(const FTile& tg, uint64_t base, uint32_t i) {
+  uint64_t off = base | (i & ((1u << tg.lc) - 1));
+  const uint32_t ch = i >> tg.lc;
+  for (int k = 0; k < tg.nh; ++k) off |= (uint64_t)((ch >> k) & 1) << tg.hpos[k];
+  return off;
+}
+
+template <int K, bool DIRECT>
+__global__ void __launch_bounds__(kFThreads, 2) k_fused(double2* __restrict__ a,
+                                                        const __grid_constant__ FProg prog) {
   constexpr uint32_t T = 1u << K;
   constexpr int R = T / kFThreads;  // amplitudes per thread
+  extern __shared__ __align__(128) double2 tile[];
+  __shared__ __align__(8) uint64_t bar;
+  const uint32_t tid = threadIdx.x;
+  const FTile& tg = prog.tile;
+  const int lc = tg.lc, nh = tg.nh;
+  // Tile base: the tile index with zeros inserted at every tile qubit.
+  uint64_t base = (uint64_t)blockIdx.x << lc;
+  for (int i = 0; i < nh; ++i) {
+    const int p = tg.hpos[i];
+    const uint64_t lo = base & ((1ull << p) - 1);
+    base = ((base - lo) << 1) | lo;
+  }
+  const uint32_t bytes = T * 16u, chunk_bytes = 16u << lc;
+  const uint32_t bar_a = smem_u32(&bar), tile_a = smem_u32(tile);
   double2 v[R];
+  if (DIRECT) {
+    // Many small chunks: a TMA bulk copy costs ~50 SM cycles regardless of size,
+    // so load straight into registers instead (each warp reads 32 consecutive
+    // amplitudes of one chunk per instruction: 512 B, coalesced).
 #pragma unroll
-  for (int r = 0; r < R; ++r) v[r] = tile[r * kFThreads + tid];
+    for (int r = 0; r < R; ++r) v[r] = ldcs(a + tile_addr(tg, base, (uint32_t)r * kFThreads + tid));
+  } else {
+    if (tid < 32) {
+      // Lane 0 arms the barrier with the whole tile; the 32 lanes of warp 0 then
+      // issue the chunk copies in parallel.
+      if (tid == 0) {
+        asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(bar_a));
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+        asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar_a),
+                     "r"(bytes)
+                     : "memory");
+      }
+      __syncwarp();
+      for (uint32_t ch = tid; ch < (1u << nh); ch += 32) {
+        uint64_t off = base;
+        for (int i = 0; i < nh; ++i) off |= (uint64_t)((ch >> i) & 1) << tg.hpos[i];
+        asm volatile(
+            "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::
+                "r"(tile_a + ch * chunk_bytes),
+            "l"(a + off), "r"(chunk_bytes), "r"(bar_a)
+            : "memory");
+      }
+    }
+    __syncthreads();  // barrier initialised before anyone waits on it
+    {
+      uint32_t done = 0;
+      while (!done) {
+        asm volatile(
+            "{ .reg .pred p; mbarrier.try_wait.parity.shared::cta.b64 p, [%1], 0; selp.u32 %0, 1, 0, p; }"
+            : "=r"(done)
+            : "r"(bar_a)
+            : "memory");
+      }
+    }
+#pragma unroll
+    for (int r = 0; r < R; ++r) v[r] = tile[r * kFThreads + tid];
+  }
   bool in_regs = true;  // else the authoritative copy is the smem tile
+
   const int nops = prog.nops;
   for (int o = 0; o < nops; ++o) {
     const FHdr& h = prog.h[o];
@@ -276,7 +345,7 @@ __device__ __forceinline__ void run_program(double2* tile, const FProg& prog, ui
     const int t0 = h.t0;
     const uint32_t mlo = h.mlo, plo = h.plo;
     const double2* c = prog.c + h.coef;
-    const bool regpath = type <= F_DIAGN || (type <= F_U2 && (t0 < 5 || t0 >= kRS));
+    const bool regpath = type <= F_DIAGN || (type <= F_U2 && (t0 < 5 || t0 >= 8));
     if (regpath && !in_regs) {
       __syncthreads();
 #pragma unroll
@@ -296,25 +365,25 @@ __device__ __forceinline__ void run_program(double2* tile, const FProg& prog, ui
     }
     switch (type) {
       case F_DIAG1: {  // one diagonal entry d != 1 on the amplitudes matching the predicate
-        // Split the predicate: register bits (uniform across the block) and thread bits.
+        // Split the predicate: register bits (warp-uniform -> branch) and thread bits.
         const double2 d = c[0];
-        const uint32_t mr = mlo >> kRS, pr = plo >> kRS;
+        const uint32_t mr = mlo >> 8, pr = plo >> 8;
         const bool bt = (tid & mlo & (kFThreads - 1)) == (plo & (kFThreads - 1));
 #pragma unroll
         for (int r = 0; r < R; ++r) {
-          if (((uint32_t)r & mr) != pr) continue;
+          if (((uint32_t)r & mr) != pr) continue;  // uniform across the block
           if (bt) v[r] = cmul_rn(d, v[r]);
         }
         break;
       }
-      case F_DIAGN: {  // factor d[j], j from the target bits (>= 64: outside the tile)
+      case F_DIAGN: {  // factor d[j], j from the target bits (>= K: from the tile base)
         const int m = h.m;
         const int ts[3] = {h.t0, h.t1, h.t2};
         uint32_t jh = 0, jmask = 0;
 #pragma unroll
         for (int s = 0; s < 3; ++s)
           if (s < m) {
-            if (ts[s] >= 64)
+            if (ts[s] >= 64)  // a qubit outside the tile: its bit comes from the tile base
               jh |= (uint32_t)((base >> (ts[s] - 64)) & 1) << (m - 1 - s);
             else
               jmask |= 1u << (m - 1 - s);
@@ -344,102 +413,38 @@ __device__ __forceinline__ void run_program(double2* tile, const FProg& prog, ui
       default: reg_1q<R>(v, FU_{c[0], c[1], c[2], c[3]}, t0, mlo, plo, tid); break;
     }
   }
+
+  if (DIRECT) {
+    if (!in_regs) {
+      __syncthreads();
+#pragma unroll
+      for (int r = 0; r < R; ++r) v[r] = tile[r * kFThreads + tid];
+    }
+#pragma unroll
+    for (int r = 0; r < R; ++r) stcs(a + tile_addr(tg, base, (uint32_t)r * kFThreads + tid), v[r]);
+    return;
+  }
   if (in_regs) {
 #pragma unroll
     for (int r = 0; r < R; ++r) tile[r * kFThreads + tid] = v[r];
   }
-}
-
-__device__ __forceinline__ uint64_t tile_base(const FTile& tg, uint64_t t) {
-  uint64_t base = t << tg.lc;  // zeros at every tile qubit
-  for (int i = 0; i < tg.nh; ++i) {
-    const int p = tg.hpos[i];
-    const uint64_t lo = base & ((1ull << p) - 1);
-    base = ((base - lo) << 1) | lo;
-  }
-  return base;
-}
-__device__ __forceinline__ uint64_t chunk_offset(const FTile& tg, uint64_t base, uint32_t ch) {
-  for (int i = 0; i < tg.nh; ++i) base |= (uint64_t)((ch >> i) & 1) << tg.hpos[i];
-  return base;
-}
-
-// Warp 0: arm the buffer's barrier with the tile size, then lanes issue chunk loads.
-__device__ __forceinline__ void issue_load(const double2* a, const FTile& tg, uint64_t base,
-                                           uint32_t buf_a, uint32_t bar_a, uint32_t lane) {
-  const uint32_t chunk_bytes = 16u << tg.lc;
-  if (lane == 0)
-    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar_a),
-                 "r"(chunk_bytes << tg.nh)
-                 : "memory");
-  __syncwarp();
-  for (uint32_t ch = lane; ch < (1u << tg.nh); ch += 32)
-    asm volatile(
-        "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::
-            "r"(buf_a + ch * chunk_bytes),
-        "l"(a + chunk_offset(tg, base, ch)), "r"(chunk_bytes), "r"(bar_a)
-        : "memory");
-}
-__device__ __forceinline__ void issue_store(double2* a, const FTile& tg, uint64_t base,
-                                            uint32_t buf_a, uint32_t lane) {
-  const uint32_t chunk_bytes = 16u << tg.lc;
-  for (uint32_t ch = lane; ch < (1u << tg.nh); ch += 32)
-    asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;" ::"l"(
-                     a + chunk_offset(tg, base, ch)),
-                 "r"(buf_a + ch * chunk_bytes), "r"(chunk_bytes)
-                 : "memory");
-  asm volatile("cp.async.bulk.commit_group;" ::: "memory");
-}
-
-template <int K>
-__global__ void __launch_bounds__(kFThreads, 1) k_fused(double2* __restrict__ a, uint64_t ntiles,
-                                                        const __grid_constant__ FProg prog) {
-  constexpr uint32_t T = 1u << K;
-  extern __shared__ __align__(128) double2 smem[];  // two tile buffers
-  __shared__ __align__(8) uint64_t bar[2];
-  const uint32_t tid = threadIdx.x;
-  const FTile& tg = prog.tile;
-  // Buffer / barrier b live at buf0 + b * 16T and bar0 + 8b (no indexed arrays).
-  const uint32_t buf0 = smem_u32(smem), bar0 = smem_u32(&bar[0]);
-  if (tid == 0) {
-    asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(bar0));
-    asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(bar0 + 8));
-    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-  }
+  // Make the generic-proxy smem writes visible to the async proxy, then the
+  // lanes of warp 0 issue the bulk stores.
+  asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
   __syncthreads();
-  uint64_t t = blockIdx.x;
-  if (t < ntiles && tid < 32) issue_load(a, tg, tile_base(tg, t), buf0, bar0, tid);
-  for (uint32_t j = 0; t < ntiles; ++j, t += gridDim.x) {
-    const int b = j & 1;
-    const uint64_t tn = t + gridDim.x;
-    if (tn < ntiles && tid < 32) {
-      // Buffer b^1 held tile j-1: its bulk store must have finished reading it.
-      asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");
-      __syncwarp();
-      issue_load(a, tg, tile_base(tg, tn), buf0 + (b ^ 1) * 16u * T, bar0 + 8u * (b ^ 1), tid);
+  if (tid < 32) {
+    for (uint32_t ch = tid; ch < (1u << nh); ch += 32) {
+      uint64_t off = base;
+      for (int i = 0; i < nh; ++i) off |= (uint64_t)((ch >> i) & 1) << tg.hpos[i];
+      asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;" ::"l"(a + off),
+                   "r"(tile_a + ch * chunk_bytes), "r"(chunk_bytes)
+                   : "memory");
     }
-    {  // wait for tile j (phase = number of earlier uses of this buffer, mod 2)
-      const uint32_t parity = (j >> 1) & 1;
-      uint32_t done = 0;
-      while (!done) {
-        asm volatile(
-            "{ .reg .pred p; mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2; selp.u32 %0, 1, 0, p; }"
-            : "=r"(done)
-            : "r"(bar0 + 8u * b), "r"(parity)
-            : "memory");
-      }
-    }
-    const uint64_t base = tile_base(tg, t);
-    double2* buf = smem + (b ? T : 0);
-    run_program<K>(buf, prog, base, tid);
-    // Make the generic-proxy smem writes visible to the async proxy, then store.
-    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-    __syncthreads();
-    if (tid < 32) issue_store(a, tg, base, buf0 + b * 16u * T, tid);
+    asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+    // Only the shared-memory source must outlive the copy; completion of the
+    // global writes is ordered by the end of the grid (as in TMA-store epilogues).
+    asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");
   }
-  // Shared memory must stay valid until the last stores have read it; the
-  // global writes themselves complete with the grid (as in TMA-store epilogues).
-  if (tid < 32) asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");
 }
 
 inline double2 D2(cplx z) { return make_double2(z.re, z.im); }
@@ -528,26 +533,33 @@ void encode(const Decoded& g, const TileMap& tm, FProg& P) {
   ++P.nops;
 }
 
+template <int K, bool DIRECT>
+void launch_kd(const LaunchCtx& ctx, const FProg& P) {
+  const size_t smem = size_t(16) << K;
+  ensure_smem_attr((const void*)k_fused<K, DIRECT>, (int)smem);
+  const uint64_t tiles = 1ull << (ctx.n_local - K);
+  k_fused<K, DIRECT><<<(unsigned)tiles, kFThreads, smem, ctx.stream>>>(
+      reinterpret_cast<double2*>(ctx.amps), P);
+}
+// TMA bulk copies for tiles of few large chunks; direct register loads for many
+// small chunks (the TMA unit's per-copy cost dominates below ~16 KiB chunks).
 template <int K>
 void launch_k(const LaunchCtx& ctx, const FProg& P) {
-  const int smem = 2 * (16 << K);
-  ensure_smem_attr((const void*)k_fused<K>, smem);
-  static std::mutex mu;
-  static int sms[64] = {0};  // SM count per device (persistent grid)
-  int dev = 0;
-  LFQS_CUDA_CHECK(cudaGetDevice(&dev));
-  {
-    std::lock_guard<std::mutex> lk(mu);
-    if (sms[dev & 63] == 0)
-      LFQS_CUDA_CHECK(cudaDeviceGetAttribute(&sms[dev & 63], cudaDevAttrMultiProcessorCount, dev));
-  }
-  const uint64_t tiles = 1ull << (ctx.n_local - K);
-  const uint64_t grid = tiles < (uint64_t)sms[dev & 63] ? tiles : (uint64_t)sms[dev & 63];
-  k_fused<K><<<(unsigned)grid, kFThreads, smem, ctx.stream>>>(reinterpret_cast<double2*>(ctx.amps),
-                                                               tiles, P);
+  if ((1 << P.tile.nh) > ctx.opt->fuse_tma_max_chunks)
+    launch_kd<K, true>(ctx, P);
+  else
+    launch_kd<K, false>(ctx, P);
 }
 
 }  // namespace
+
+bool fusable(const Decoded& g, int K, int n_local) {
+  (void)n_local;
+  if (g.cls == GClass::NOOP || g.cls == GClass::DIAG) return true;
+  for (int s = 0; s < g.m; ++s)
+    if (g.targets[s] >= K) return false;
+  return true;
+}
 
 // Greedy segmentation (NEXT-1 "general cache-blocked fusion"): the tile holds
 // qubits [0, L) (contiguous, for coalesced 2^L-amplitude chunks) plus up to
@@ -607,6 +619,7 @@ bool run_fused_circuit(const LaunchCtx& ctx, const std::vector<Decoded>& gates, 
   require(b == K && lc + P.tile.nh == K, "internal: bad fused tile");
   for (size_t q = begin; q < i; ++q) encode(gates[q], tm, P);
   switch (K) {
+    case 8: launch_k<8>(ctx, P); break;
     case 9: launch_k<9>(ctx, P); break;
     case 10: launch_k<10>(ctx, P); break;
     case 11: launch_k<11>(ctx, P); break;

@@ -84,6 +84,7 @@ struct Options {
   bool wide256 = true;       // two adjacent groups per item, 32-byte accesses
   int fuse_tile_qubits = 12;
   int fuse_low_qubits = 7;   // contiguous low qubits of a fused tile (chunk = 2^7 amps)
+  int fuse_tma_max_chunks = 4;  // tiles with more chunks load/store directly (no TMA)
   int items_per_thread = 0;  // 0 = library default
 };
 

@@ -48,9 +48,11 @@ def test_fused_random_circuit(L, n, tile):
     assert np.array_equal(a, b)
 
 
-@pytest.mark.parametrize("low", [3, 5, 7, 12])
-def test_fused_general_tiles(L, low):
-    """Tiles = qubits [0, low) + qubits claimed by the gates (NEXT-1), chunked TMA copies."""
+@pytest.mark.parametrize("tma", [0, 256])
+@pytest.mark.parametrize("low", [5, 7, 12])
+def test_fused_general_tiles(L, low, tma):
+    """Tiles = qubits [0, low) + qubits claimed by the gates (NEXT-1); chunks moved by
+    TMA bulk copies (tma=256) or by direct register loads/stores (tma=0)."""
     n = 18
     psi = W.random_state(n, low)
     gates = W.random_gate_list(n, 200, seed=100 + low, max_controls=2) + W.qft(n) + \
@@ -58,6 +60,7 @@ def test_fused_general_tiles(L, low):
     ref = O.run_circuit(n, gates, psi.copy())
     with L.State.create(n) as st:
         st.set_option(L.OPT_FUSE_LOW_QUBITS, low)
+        st.set_option(L.OPT_FUSE_TMA_MAX_CHUNKS, tma)
         st.copy_in(psi)
         c0 = st.launches()
         st.run_circuit(gates, fuse=True)
