@@ -202,7 +202,7 @@ lfqs_status lfqs_kernel_launches(const lfqs_state* s, uint64_t* count);
 #define LFQS_OPT_FUSE_LOW_QUBITS 5 /* contiguous low qubits of a fused tile, [3, 12], default 7;
                                       the other tile qubits are claimed by the fused gates */
 #define LFQS_OPT_FUSE_TMA_MAX_CHUNKS 6 /* tiles of at most this many chunks move by TMA bulk
-                                          copies, larger ones by direct loads (default 4) */
+                                          copies, larger ones by direct loads (default 256) */
 lfqs_status lfqs_set_option(lfqs_state* s, int option, int64_t value);
 const char* lfqs_last_error(void);
 int lfqs_abi_version(void);

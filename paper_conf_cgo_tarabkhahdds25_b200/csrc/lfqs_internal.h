@@ -84,7 +84,10 @@ struct Options {
   bool wide256 = true;       // two adjacent groups per item, 32-byte accesses
   int fuse_tile_qubits = 12;
   int fuse_low_qubits = 7;   // contiguous low qubits of a fused tile (chunk = 2^7 amps)
-  int fuse_tma_max_chunks = 4;  // tiles with more chunks load/store directly (no TMA)
+  // Tiles with more chunks load/store directly (no TMA).  Measured on B200 at
+  // n=30 (profiles/r01_fused_variants.md): TMA with parallel issue from warp 0
+  // beats direct loads for every chunk count up to 128, so TMA is the default.
+  int fuse_tma_max_chunks = 256;
   int items_per_thread = 0;  // 0 = library default
 };
 
