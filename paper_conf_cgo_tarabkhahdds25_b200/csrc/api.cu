@@ -184,19 +184,22 @@ lfqs_status lfqs_plan_circuit(int n_qubits, int world, int rank, const lfqs_gate
     require(world >= 1 && rank >= 0 && rank < world, "bad rank / world");
     Planner plan(n_qubits, world);
     std::vector<PlanOp> raw;
+    std::vector<Decoded> dec;
     for (size_t i = 0; i < n_gates; ++i) {
       const lfqs_gate& G = gates[i];
       require(G.n_controls == __builtin_popcountll(G.control_mask),
               "gate " + std::to_string(i) + ": n_controls != popcount(control_mask)");
-      Decoded d = decode_gate(n_qubits, G.kind, G.targets, G.n_targets, G.control_mask, G.params,
-                              kind_nparams(G.kind), G.matrix);
-      if (world == 1) {
+      dec.push_back(decode_gate(n_qubits, G.kind, G.targets, G.n_targets, G.control_mask,
+                                G.params, kind_nparams(G.kind), G.matrix));
+    }
+    if (world == 1) {
+      for (const Decoded& d : dec) {
         PlanOp op;
         op.gate = d;
         raw.push_back(op);
-      } else {
-        plan.plan_gate(d, raw);
       }
+    } else {
+      plan.plan_circuit(dec, raw);  // the same planning State::run uses
     }
     if (canonicalize) plan.plan_canonicalize(raw);
     // Rank-specialise and convert.

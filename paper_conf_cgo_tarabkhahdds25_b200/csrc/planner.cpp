@@ -94,7 +94,26 @@ void Planner::plan_canonicalize(std::vector<PlanOp>& out) {
   }
 }
 
-void Planner::plan_gate(const Decoded& g, std::vector<PlanOp>& out) {
+void Planner::plan_circuit(const std::vector<Decoded>& gates, std::vector<PlanOp>& out) {
+  // uses[q] = ascending gate indices where logical q is a non-diagonal target.
+  std::vector<std::vector<int>> uses(n);
+  for (size_t i = 0; i < gates.size(); ++i) {
+    const Decoded& g = gates[i];
+    if (g.cls == GClass::NOOP || g.cls == GClass::DIAG) continue;
+    for (int s = 0; s < g.m; ++s) uses[g.targets[s]].push_back((int)i);
+  }
+  std::vector<int> next_use(n);
+  for (size_t i = 0; i < gates.size(); ++i) {
+    for (int q = 0; q < n; ++q) {
+      auto it = std::upper_bound(uses[q].begin(), uses[q].end(), (int)i);
+      next_use[q] = it == uses[q].end() ? (1 << 30) : *it;
+    }
+    plan_gate(gates[i], out, &next_use);
+  }
+}
+
+void Planner::plan_gate(const Decoded& g, std::vector<PlanOp>& out,
+                        const std::vector<int>* next_use) {
   if (g.cls == GClass::NOOP) return;
   Decoded pg = to_physical(g);
   if (world > 1 && pg.cls == GClass::PERM_SWAP && pg.cmask == 0 &&
@@ -112,8 +131,18 @@ void Planner::plan_gate(const Decoded& g, std::vector<PlanOp>& out) {
       if (gq < n_local) continue;
       uint64_t tmask = 0;
       for (int u = 0; u < pg.m; ++u) tmask |= 1ull << pg.targets[u];
-      int l = n_local - 1;
-      while (l >= 0 && (tmask >> l & 1)) --l;
+      int l = -1, best = -1;
+      const int lo = std::max(0, n_local - kSwapWindow);
+      for (int p = n_local - 1; p >= lo; --p) {
+        if (tmask >> p & 1) continue;
+        const int score = next_use ? (*next_use)[p2l[p]] : 0;
+        if (score > best) {
+          best = score;
+          l = p;
+        }
+      }
+      for (int p = lo - 1; l < 0 && p >= 0; --p)
+        if (!(tmask >> p & 1)) l = p;
       require(l >= 0, "internal: no free local qubit");
       exchange(l, gq, out);
       pg.targets[s] = l;

@@ -27,7 +27,15 @@ struct Planner {
   void reset();
   bool identity() const;
   // Appends the physical ops for logical gate g and updates the qubit map.
-  void plan_gate(const Decoded& g, std::vector<PlanOp>& out);
+  // next_use(q) (optional) = index of the next gate that has logical qubit q as
+  // a non-diagonal target (a large value if none): the evicted local qubit is
+  // the one used furthest in the future (Belady), among the top kSwapWindow
+  // local positions (so exchanged pieces stay >= 2^(n_local - kSwapWindow) amps).
+  static constexpr int kSwapWindow = 8;
+  void plan_gate(const Decoded& g, std::vector<PlanOp>& out,
+                 const std::vector<int>* next_use = nullptr);
+  // Plans a whole circuit with Belady lookahead.
+  void plan_circuit(const std::vector<Decoded>& gates, std::vector<PlanOp>& out);
   // Appends the ops that restore the identity map.
   void plan_canonicalize(std::vector<PlanOp>& out);
   // Specialises a LOCAL op for rank r: false if a global control is 0 there;

@@ -231,23 +231,51 @@ void State::exchange_data(int l, int g) {
   exchange_bytes += 16ull << (n_local - 1);
 }
 
-void State::execute(const std::vector<PlanOp>& ops) {
-  for (const PlanOp& op : ops) {
-    if (op.kind == PlanOp::EXCHANGE) {
-      exchange_data(op.l, op.g);
+// A run of local gates on one shard: fused passes where possible, else one
+// class kernel per gate.
+void State::run_local(const LaunchCtx& c, const std::vector<Decoded>& gates, bool fuse) {
+  size_t i = 0;
+  while (i < gates.size()) {
+    size_t used = 0;
+    if (fuse && run_fused_circuit(c, gates, i, gates.size(), opt.fuse_tile_qubits, &used)) {
+      i += used;
+    } else {
+      launch_gate(c, gates[i]);
+      ++i;
+    }
+  }
+}
+
+// Executes planned ops: maximal runs of LOCAL ops are rank-specialised per shard
+// and run (fused if requested); EXCHANGE ops move data between shards.
+void State::execute(const std::vector<PlanOp>& ops, bool fuse) {
+  size_t i = 0;
+  while (i < ops.size()) {
+    if (ops[i].kind == PlanOp::EXCHANGE) {
+      exchange_data(ops[i].l, ops[i].g);
+      ++i;
       continue;
     }
+    size_t j = i;
+    while (j < ops.size() && ops[j].kind == PlanOp::LOCAL) ++j;
     for (int s = 0; s < n_shards(); ++s) {
-      Decoded lg;
-      if (plan.rank_local(op.gate, rank_of_shard(s), &lg)) launch_gate(ctx(s), lg);
+      std::vector<Decoded> seg;
+      seg.reserve(j - i);
+      for (size_t k = i; k < j; ++k) {
+        Decoded lg;
+        if (plan.rank_local(ops[k].gate, rank_of_shard(s), &lg) && lg.cls != GClass::NOOP)
+          seg.push_back(lg);
+      }
+      run_local(ctx(s), seg, fuse);
     }
+    i = j;
   }
 }
 
 void State::canonicalize() {
   std::vector<PlanOp> ops;
   plan.plan_canonicalize(ops);
-  execute(ops);
+  execute(ops, false);
 }
 
 void State::apply(const Decoded& g) {
@@ -258,25 +286,19 @@ void State::apply(const Decoded& g) {
   }
   std::vector<PlanOp> ops;
   plan.plan_gate(g, ops);
-  execute(ops);
+  execute(ops, false);
 }
 
 void State::run(const std::vector<Decoded>& gates, uint32_t flags) {
   DeviceGuard dg(device);
-  if ((flags & LFQS_FUSE_LOW) && world == 1) {
-    size_t i = 0;
-    while (i < gates.size()) {
-      size_t used = 0;
-      if (run_fused_circuit(ctx(0), gates, i, gates.size(), opt.fuse_tile_qubits, &used)) {
-        i += used;
-      } else {
-        launch_gate(ctx(0), gates[i]);
-        ++i;
-      }
-    }
+  const bool fuse = (flags & LFQS_FUSE_LOW) != 0;
+  if (world == 1) {
+    run_local(ctx(0), gates, fuse);
     return;
   }
-  for (const Decoded& g : gates) apply(g);
+  std::vector<PlanOp> ops;
+  plan.plan_circuit(gates, ops);  // Belady lookahead over the whole circuit
+  execute(ops, fuse);
 }
 
 void State::measure_probs(const int* qubits, int nq, double* out) {

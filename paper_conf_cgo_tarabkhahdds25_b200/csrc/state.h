@@ -59,7 +59,8 @@ struct State : lfqs_state {
   LaunchCtx ctx(int shard);
   int n_shards() const { return virt ? world : 1; }
   int rank_of_shard(int shard) const { return virt ? shard : rank; }
-  void execute(const std::vector<PlanOp>& ops);
+  void execute(const std::vector<PlanOp>& ops, bool fuse);
+  void run_local(const LaunchCtx& c, const std::vector<Decoded>& gates, bool fuse);
   void exchange_data(int l, int g);  // swap physical positions l (local) and g (global)
   void canonicalize();
 };

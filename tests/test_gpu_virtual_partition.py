@@ -67,6 +67,26 @@ def test_global_qubit_cases(L, world):
     assert np.max(np.abs(got - ref)) <= 1e-12
 
 
+@pytest.mark.parametrize("world", [2, 4, 8])
+def test_virtual_partition_fused(L, world):
+    """Distributed run with Belady remaps and fused local segments == oracle."""
+    n = 16
+    psi = W.random_state(n, 77)
+    gates = W.random_gate_list(n, 150, seed=3 * world, max_controls=2) + W.qft(n) + \
+        W.random_layered(n, 3, seed=world)
+    ref = O.run_circuit(n, gates, psi.copy())
+    with L.State.virtual(n, world) as st:
+        st.copy_in(psi)
+        st.run_circuit(gates, fuse=True)
+        got = st.copy_out()
+    assert np.max(np.abs(got - ref)) <= 1e-12
+    exact = [g for g in gates if g.exact]
+    with L.State.virtual(n, world) as st:
+        st.copy_in(psi)
+        st.run_circuit(exact, fuse=True)
+        assert np.array_equal(st.copy_out(), O.run_circuit(n, exact, psi.copy()))
+
+
 def test_virtual_qft_and_ghz(L):
     n, x = 14, 9001
     with L.State.virtual(n, 4) as st:
