@@ -156,6 +156,20 @@ lfqs_status lfqs_run_circuit(lfqs_state* s, const lfqs_gate* gates, size_t n_gat
 lfqs_status lfqs_measure_probs(lfqs_state* s, const int* qubits, int n_q, double* probs_out,
                                size_t probs_len);
 
+/* Sampling without collapse (reading R15: the paper's "followed by measurement",
+ * P:122).  With p = lfqs_measure_probs(qubits) and c[v] = p[0] + ... + p[v]
+ * (ascending), shot i returns the smallest v with u_i * c[last] < c[v].  The
+ * uniforms u_i in [0, 1) are caller-provided (the random numbers the method draws
+ * are inputs).  outcomes has `shots` entries.  Synchronous. */
+lfqs_status lfqs_measure_sample(lfqs_state* s, const int* qubits, int n_q, const double* uniforms,
+                                size_t shots, uint64_t* outcomes);
+/* Projective measurement with a chosen outcome (mid-circuit measurement):
+ * amplitudes whose measured bits differ from `outcome` become 0, the others are
+ * multiplied by 1/sqrt(P(outcome)).  *probability (optional) receives P(outcome).
+ * LFQS_ERR_INVALID_ARG if P(outcome) == 0.  Synchronous. */
+lfqs_status lfqs_measure_collapse(lfqs_state* s, const int* qubits, int n_q, uint64_t outcome,
+                                  double* probability);
+
 /* ---- planning (host only: no GPU needed) ------------------------------------ */
 /* The distributed planner as a query: the physical
  * operations rank `rank` of `world` performs for gates[0..n_gates), in order.

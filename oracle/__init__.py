@@ -71,6 +71,10 @@ def lib():
         L.oracle_apply_gate_sparse.argtypes = [C.c_int, gp, C.c_size_t,
                                                C.POINTER(C.c_uint64), dp]
         L.oracle_probs.argtypes = [C.c_int, dp, C.POINTER(C.c_int), C.c_int, dp]
+        L.oracle_measure_sample.argtypes = [C.c_int, dp, C.POINTER(C.c_int), C.c_int, dp,
+                                            C.c_size_t, C.POINTER(C.c_uint64)]
+        L.oracle_measure_collapse.argtypes = [C.c_int, dp, C.POINTER(C.c_int), C.c_int,
+                                              C.c_uint64, dp]
         L.oracle_fill_random.argtypes = [C.c_uint64, C.c_uint64, C.c_uint64, dp]
         L.oracle_fill_random.restype = None
         L.oracle_omp_max_threads.restype = C.c_int
@@ -216,6 +220,25 @@ def probs(n: int, state: np.ndarray, qubits: Sequence[int] = ()) -> np.ndarray:
     _check(lib().oracle_probs(n, _dp(np.ascontiguousarray(state).view(np.float64)), q,
                               len(qubits), _dp(out)), "probs")
     return out
+
+
+def measure_sample(n: int, state: np.ndarray, qubits: Sequence[int], u) -> np.ndarray:
+    q = (C.c_int * max(1, len(qubits)))(*qubits)
+    u = np.ascontiguousarray(u, dtype=np.float64)
+    out = np.zeros(u.size, dtype=np.uint64)
+    _check(lib().oracle_measure_sample(n, _dp(np.ascontiguousarray(state).view(np.float64)), q,
+                                       len(qubits), _dp(u), u.size,
+                                       out.ctypes.data_as(C.POINTER(C.c_uint64))), "measure_sample")
+    return out
+
+
+def measure_collapse(n: int, state: np.ndarray, qubits: Sequence[int], outcome: int):
+    """In place on a complex128 array; returns P(outcome)."""
+    q = (C.c_int * max(1, len(qubits)))(*qubits)
+    p = C.c_double(0.0)
+    _check(lib().oracle_measure_collapse(n, _dp(state.view(np.float64)), q, len(qubits), outcome,
+                                         C.byref(p)), "measure_collapse")
+    return p.value
 
 
 def fill_random(seed: int, start: int, count: int) -> np.ndarray:

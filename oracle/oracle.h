@@ -94,6 +94,16 @@ int oracle_omp_max_threads(void);
  * in ascending order per bin; bit s of v = bit qubits[s] of k.  nq = 0 -> norm^2. */
 int oracle_probs(int n, const double* state, const int* qubits, int nq, double* probs);
 
+/* Sampling (reading R15): c[v] = p[0] + ... + p[v] (ascending, p from
+ * oracle_probs); shot i = smallest v with u[i] * c[last] < c[v]. */
+int oracle_measure_sample(int n, const double* state, const int* qubits, int nq,
+                          const double* u, size_t shots, uint64_t* out);
+/* Projective measurement with outcome `outcome`: amplitudes whose measured bits
+ * differ become 0, the rest are multiplied by 1/sqrt(P(outcome)).
+ * *p_out = P(outcome).  -1 if P(outcome) == 0. */
+int oracle_measure_collapse(int n, double* state, const int* qubits, int nq, uint64_t outcome,
+                            double* p_out);
+
 /* ---- Counter-based input generator (same formula as workloads/) ----------- */
 /* amplitudes start..start+count-1 of the SplitMix64 random state, interleaved. */
 void oracle_fill_random(uint64_t seed, uint64_t start, uint64_t count, double* out);

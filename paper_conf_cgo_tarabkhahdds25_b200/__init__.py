@@ -43,7 +43,7 @@ EXPORTS = [
     "lfqs_state_init_basis", "lfqs_state_init_random", "lfqs_copy_in", "lfqs_copy_out",
     "lfqs_apply_gate", "lfqs_run_circuit", "lfqs_measure_probs", "lfqs_synchronize",
     "lfqs_state_info", "lfqs_kernel_launches", "lfqs_set_option", "lfqs_last_error",
-    "lfqs_abi_version", "lfqs_plan_circuit",
+    "lfqs_abi_version", "lfqs_plan_circuit", "lfqs_measure_sample", "lfqs_measure_collapse",
 ]
 
 
@@ -108,6 +108,8 @@ def lib():
             "lfqs_state_info": [vp, ip, ip, ip, ip, C.POINTER(vp)],
             "lfqs_kernel_launches": [vp, C.POINTER(u64)],
             "lfqs_set_option": [vp, C.c_int, C.c_int64],
+            "lfqs_measure_sample": [vp, ip, C.c_int, dp, C.c_size_t, C.POINTER(u64)],
+            "lfqs_measure_collapse": [vp, ip, C.c_int, u64, dp],
             "lfqs_plan_circuit": [C.c_int, C.c_int, C.c_int, C.POINTER(LfqsGate), C.c_size_t,
                                   C.c_int, C.POINTER(LfqsPlanOp), C.c_size_t,
                                   C.POINTER(C.c_size_t)],
@@ -270,6 +272,24 @@ def lfqs_measure_probs(h: int, qubits: Sequence[int] = ()) -> np.ndarray:
     return out
 
 
+def lfqs_measure_sample(h: int, qubits: Sequence[int], uniforms) -> np.ndarray:
+    """Outcomes (uint64) of len(uniforms) shots; uniforms in [0, 1) are the caller's draws."""
+    q, nq = _ints(qubits)
+    u = np.ascontiguousarray(uniforms, dtype=np.float64)
+    out = np.zeros(u.size, dtype=np.uint64)
+    _check(lib().lfqs_measure_sample(h, q, nq, _dp(u), u.size,
+                                     out.ctypes.data_as(C.POINTER(C.c_uint64))))
+    return out
+
+
+def lfqs_measure_collapse(h: int, qubits: Sequence[int], outcome: int) -> float:
+    """Projects onto `outcome` of the measured qubits and renormalises; returns P(outcome)."""
+    q, nq = _ints(qubits)
+    p = C.c_double(0.0)
+    _check(lib().lfqs_measure_collapse(h, q, nq, outcome, C.byref(p)))
+    return p.value
+
+
 def lfqs_synchronize(h: int):
     _check(lib().lfqs_synchronize(h))
 
@@ -408,6 +428,12 @@ class State:
 
     def measure_probs(self, qubits: Sequence[int] = ()) -> np.ndarray:
         return lfqs_measure_probs(self.h, qubits)
+
+    def sample(self, qubits: Sequence[int], uniforms) -> np.ndarray:
+        return lfqs_measure_sample(self.h, qubits, uniforms)
+
+    def collapse(self, qubits: Sequence[int], outcome: int) -> float:
+        return lfqs_measure_collapse(self.h, qubits, outcome)
 
     def norm2(self) -> float:
         return float(self.measure_probs(())[0])

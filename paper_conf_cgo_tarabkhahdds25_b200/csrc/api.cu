@@ -6,6 +6,8 @@
 // complex layout, then measured.
 #include <cuda_runtime.h>
 
+#include <algorithm>
+#include <cmath>
 #include <cstdio>
 #include <cstring>
 #include <memory>
@@ -265,6 +267,44 @@ lfqs_status lfqs_measure_probs(lfqs_state* s, const int* qubits, int n_q, double
     const uint64_t qm = mask_of(qubits, n_q, st->n);
     (void)qm;
     st->measure_probs(qubits, n_q, probs_out);
+  });
+}
+
+lfqs_status lfqs_measure_sample(lfqs_state* s, const int* qubits, int n_q, const double* uniforms,
+                                size_t shots, uint64_t* outcomes) {
+  return guarded([&] {
+    require(s != nullptr && (shots == 0 || (uniforms != nullptr && outcomes != nullptr)),
+            "NULL argument");
+    State* st = static_cast<State*>(s);
+    require(n_q >= 0 && n_q <= 10, "n_q must be in [0, 10]");
+    mask_of(qubits, n_q, st->n);
+    std::vector<double> p(size_t(1) << n_q);
+    st->measure_probs(qubits, n_q, p.data());
+    std::vector<double> c(p.size());
+    double acc = 0.0;
+    for (size_t v = 0; v < p.size(); ++v) c[v] = acc = acc + p[v];
+    for (size_t i = 0; i < shots; ++i) {
+      require(uniforms[i] >= 0.0 && uniforms[i] < 1.0, "uniforms must be in [0, 1)");
+      const double x = uniforms[i] * c.back();
+      outcomes[i] = (uint64_t)(std::upper_bound(c.begin(), c.end(), x) - c.begin());
+      if (outcomes[i] >= c.size()) outcomes[i] = c.size() - 1;
+    }
+  });
+}
+
+lfqs_status lfqs_measure_collapse(lfqs_state* s, const int* qubits, int n_q, uint64_t outcome,
+                                  double* probability) {
+  return guarded([&] {
+    require(s != nullptr, "NULL state");
+    State* st = static_cast<State*>(s);
+    require(n_q >= 0 && n_q <= 10, "n_q must be in [0, 10]");
+    require(outcome < (uint64_t(1) << n_q), "outcome out of range");
+    mask_of(qubits, n_q, st->n);
+    std::vector<double> p(size_t(1) << n_q);
+    st->measure_probs(qubits, n_q, p.data());
+    require(p[outcome] > 0.0, "outcome has probability 0");
+    st->collapse(qubits, n_q, outcome, 1.0 / std::sqrt(p[outcome]));
+    if (probability) *probability = p[outcome];
   });
 }
 

@@ -19,6 +19,7 @@
 #include <cuda_runtime.h>
 
 #include <algorithm>
+#include <type_traits>
 #include <cstring>
 
 #include "lfqs_internal.h"
@@ -358,15 +359,25 @@ void run_group(const LaunchCtx& ctx, uint64_t n_groups, const InsertPlan& ip, co
   for (int j = 0; j < L; ++j) even &= (off.o[j] & 1) == 0;
   if constexpr (!P256 && L <= 4) {
     if (ctx.opt->wide256 && even && n_groups >= 2 && (ip.np == 0 || ip.pos[0] >= 1)) {
-      constexpr int UX = L == 1 ? 4 : (L == 2 ? 2 : 1);
       const uint64_t n_items = n_groups / 2;
-      const uint64_t nb = blocks_for(n_items, (uint64_t)kThreads * UX);
-      require(nb < (1ull << 31), "grid too large");
-      if (ip.np <= 4)
-        k_group_x2<L, UX, 4, Op><<<(unsigned)nb, kThreads, 0, ctx.stream>>>(a, n_items, ip, off, op);
+      auto go = [&](auto ux) {
+        constexpr int UX = decltype(ux)::value;
+        const uint64_t nb = blocks_for(n_items, (uint64_t)kThreads * UX);
+        require(nb < (1ull << 31), "grid too large");
+        if (ip.np <= 4)
+          k_group_x2<L, UX, 4, Op><<<(unsigned)nb, kThreads, 0, ctx.stream>>>(a, n_items, ip, off, op);
+        else
+          k_group_x2<L, UX, kMaxInsert, Op>
+              <<<(unsigned)nb, kThreads, 0, ctx.stream>>>(a, n_items, ip, off, op);
+      };
+      // Groups per thread (tuning knob LFQS_OPT_ITEMS_PER_THREAD for pair gates).
+      const int ipt = ctx.opt->items_per_thread;
+      if (L == 2 && ipt == 1)
+        go(std::integral_constant<int, 1>{});
+      else if (L == 2 && ipt == 4)
+        go(std::integral_constant<int, 4>{});
       else
-        k_group_x2<L, UX, kMaxInsert, Op>
-            <<<(unsigned)nb, kThreads, 0, ctx.stream>>>(a, n_items, ip, off, op);
+        go(std::integral_constant<int, L == 1 ? 4 : (L == 2 ? 2 : 1)>{});
       LFQS_CUDA_CHECK(cudaGetLastError());
       ++*ctx.launch_counter;
       return;

@@ -116,6 +116,10 @@ void launch_probs(const LaunchCtx& ctx, const int* qubits, int nq, double* d_par
                   int n_partials_blocks, double* d_out);
 int probs_blocks();
 
+// Projective collapse: a[k] = (k & mask) == pat ? scale * a[k] : 0 (all zero if
+// zero_all: the rank's global bits do not match the outcome).
+void launch_collapse(const LaunchCtx& ctx, uint64_t mask, uint64_t pat, double scale, bool zero_all);
+
 // Initialisers.
 void launch_init_basis(const LaunchCtx& ctx, int64_t local_index);  // -1: all zero
 void launch_init_random(const LaunchCtx& ctx, uint64_t seed, uint64_t global_offset);

@@ -103,6 +103,24 @@ __global__ void k_probs_tiny(const double2* __restrict__ a, uint64_t n_amps, con
   for (uint64_t k = 0; k < n_amps; ++k) out[bin_of(ql, k)] += a[k].x * a[k].x + a[k].y * a[k].y;
 }
 
+// --- projective collapse (one streaming pass, 32-byte accesses) --------------
+__global__ void __launch_bounds__(kThreads) k_collapse(double2* __restrict__ a, uint64_t n_pairs,
+                                                       uint64_t mask, uint64_t pat, double scale) {
+  const uint64_t stride = (uint64_t)gridDim.x * kThreads;
+  for (uint64_t i = (uint64_t)blockIdx.x * kThreads + threadIdx.x; i < n_pairs; i += stride) {
+    const uint64_t k = 2 * i;
+    double2 x, y;
+    asm volatile("ld.global.cs.v4.f64 {%0,%1,%2,%3}, [%4];"
+                 : "=d"(x.x), "=d"(x.y), "=d"(y.x), "=d"(y.y)
+                 : "l"(a + k));
+    x = ((k & mask) == pat) ? make_double2(scale * x.x, scale * x.y) : make_double2(0.0, 0.0);
+    y = (((k + 1) & mask) == pat) ? make_double2(scale * y.x, scale * y.y) : make_double2(0.0, 0.0);
+    asm volatile("st.global.cs.v4.f64 [%0], {%1,%2,%3,%4};" ::"l"(a + k), "d"(x.x), "d"(x.y),
+                 "d"(y.x), "d"(y.y)
+                 : "memory");
+  }
+}
+
 // --- initialisers -----------------------------------------------------------
 __global__ void k_set_one(double2* a, uint64_t idx) { a[idx] = make_double2(1.0, 0.0); }
 
@@ -169,6 +187,21 @@ void launch_probs(const LaunchCtx& ctx, const int* qubits, int nq, double* d_par
   k_probs_final<<<(nbins + 255) / 256, 256, 0, ctx.stream>>>(d_partials, kBlocks, nbins, d_out);
   LFQS_CUDA_CHECK(cudaGetLastError());
   *ctx.launch_counter += 2;
+}
+
+void launch_collapse(const LaunchCtx& ctx, uint64_t mask, uint64_t pat, double scale,
+                     bool zero_all) {
+  const uint64_t n = 1ull << ctx.n_local;
+  if (zero_all) {
+    LFQS_CUDA_CHECK(cudaMemsetAsync(ctx.amps, 0, n * 16, ctx.stream));
+    return;
+  }
+  uint64_t nb = (n / 2 + kThreads - 1) / kThreads;
+  if (nb > 148ull * 64) nb = 148ull * 64;
+  k_collapse<<<(unsigned)nb, kThreads, 0, ctx.stream>>>(reinterpret_cast<double2*>(ctx.amps),
+                                                        n / 2, mask, pat, scale);
+  LFQS_CUDA_CHECK(cudaGetLastError());
+  ++*ctx.launch_counter;
 }
 
 void launch_init_basis(const LaunchCtx& ctx, int64_t local_index) {

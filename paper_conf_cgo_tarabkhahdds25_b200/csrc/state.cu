@@ -301,6 +301,26 @@ void State::run(const std::vector<Decoded>& gates, uint32_t flags) {
   execute(ops, fuse);
 }
 
+void State::collapse(const int* qubits, int nq, uint64_t outcome, double scale) {
+  DeviceGuard dg(device);
+  for (int sh = 0; sh < n_shards(); ++sh) {
+    const int r = rank_of_shard(sh);
+    uint64_t mask = 0, pat = 0;
+    bool rank_matches = true;
+    for (int s = 0; s < nq; ++s) {
+      const int P = plan.l2p[qubits[s]];
+      const uint64_t bit = (outcome >> s) & 1;
+      if (P < n_local) {
+        mask |= 1ull << P;
+        pat |= bit << P;
+      } else if ((uint64_t)((r >> (P - n_local)) & 1) != bit) {
+        rank_matches = false;
+      }
+    }
+    launch_collapse(ctx(sh), mask, pat, rank_matches ? scale : 0.0, !rank_matches);
+  }
+}
+
 void State::measure_probs(const int* qubits, int nq, double* out) {
   DeviceGuard dg(device);
   const int nb = 1 << nq;

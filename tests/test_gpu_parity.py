@@ -265,3 +265,17 @@ def test_kernel_launch_accounting(L):
         c0 = st.launches()
         st.run_circuit([W.Gate("H", (q,)) for q in range(14)])
         assert st.launches() - c0 == 14
+
+
+@pytest.mark.parametrize("fuse", [False, True])
+def test_table1_workloads_vs_oracle(L, fuse):
+    """QPE (closed form), VQE ansatz and Sycamore-like circuits (Table 1)."""
+    for n, gates in ((13, W.qpe(12, 2901)), (14, W.vqe_ansatz(14, 4, seed=3)),
+                     (15, W.sycamore_like(3, 5, 12, seed=4))):
+        psi = W.basis_state(n, 0)
+        ref = O.run_circuit(n, gates, psi.copy())
+        got = _gpu_apply(L, n, psi, gates, fuse=fuse)
+        assert np.max(np.abs(got - ref)) <= 1e-12
+    with L.State.create(13) as st:
+        st.run_circuit(W.qpe(12, 2901), fuse=fuse)
+        assert abs(st.measure_probs(list(range(12)))[2901] - 1.0) < 1e-12

@@ -397,3 +397,90 @@ def test_oracle_rejects_bad_gates():
     for g in (W.Gate("H", (4,)), W.Gate("X", (1,), (1,)), W.Gate("SWAP", (2, 2))):
         with pytest.raises(ValueError):
             O.apply_gate(n, g, W.random_state(n, 1))
+
+
+# --------------------------------------------------------------------------
+# Remaining Table-1 workloads (NEXT-2): QPE closed form, inverse QFT, inputs
+# --------------------------------------------------------------------------
+
+@pytest.mark.parametrize("t,m", [(3, 5), (6, 37), (9, 300)])
+def test_qpe_exact_phase_closed_form(t, m):
+    """QPE (Table 1; reading R18): with phase m/2^t the counting register is |m>
+    with probability 1 and the eigenstate qubit stays |1>."""
+    n = t + 1
+    psi = W.basis_state(n, 0)
+    O.run_circuit(n, W.qpe(t, m), psi)
+    p = O.probs(n, psi, list(range(t)))
+    assert abs(p[m] - 1.0) < 1e-12
+    assert abs(O.probs(n, psi, [t])[1] - 1.0) < 1e-12
+
+
+def test_qft_inverse_undoes_qft():
+    n = 7
+    psi0 = W.random_state(n, 8)
+    psi = O.run_circuit(n, W.qft(n) + W.qft_inverse(n), psi0.copy())
+    np.testing.assert_allclose(psi, psi0, atol=1e-14)
+
+
+def test_sycamore_inputs_are_the_named_gates():
+    """Input sanity: sqrt(X)^2 = X, sqrt(Y)^2 = Y, sqrt(W)^2 = W; fSim unitary."""
+    gates = W.sycamore_like(2, 3, 8, seed=1)
+    X = np.array([[0, 1], [1, 0]]); Y = np.array([[0, -1j], [1j, 0]])
+    targets = {"X": X, "Y": Y, "W": (X + Y) / np.sqrt(2)}
+    seen = set()
+    for g in gates:
+        if g.kind == "UNITARY1":
+            sq = g.matrix @ g.matrix
+            name = [k for k, v in targets.items() if np.allclose(sq, v, atol=1e-15)]
+            assert len(name) == 1
+            seen.add(name[0])
+        else:
+            np.testing.assert_allclose(g.matrix @ g.matrix.conj().T, np.eye(4), atol=1e-15)
+    assert seen == {"X", "Y", "W"}
+
+
+# --------------------------------------------------------------------------
+# Measurement: sampling and collapse (P:122, P:154; reading R15)
+# --------------------------------------------------------------------------
+
+def test_sampling_inverse_cdf_and_statistics():
+    """Uniform 2-qubit state: u in the v-th quarter -> outcome v exactly; a biased
+    state's sample frequencies follow its probabilities (chi-square)."""
+    n = 2
+    psi = O.run_circuit(n, [W.Gate("H", (0,)), W.Gate("H", (1,))], W.basis_state(n, 0))
+    u = (np.arange(4) + 0.5) / 4
+    assert list(O.measure_sample(n, psi, [0, 1], u)) == [0, 1, 2, 3]
+    assert list(O.measure_sample(n, psi, [1, 0], u)) == [0, 1, 2, 3]
+    n = 6
+    psi = O.run_circuit(n, W.random_layered(n, 3, seed=2), W.basis_state(n, 0))
+    p = O.probs(n, psi, [1, 4])
+    rng = np.random.default_rng(0)
+    shots = 200000
+    counts = np.bincount(O.measure_sample(n, psi, [1, 4], rng.random(shots)).astype(int),
+                         minlength=4)
+    chi2 = float(np.sum((counts - shots * p) ** 2 / (shots * p)))
+    assert chi2 < 16.27  # 3 dof, p = 0.001
+    b = W.basis_state(n, 0b101101)
+    assert set(O.measure_sample(n, b, [0, 2, 5], rng.random(50))) == {7}  # bits 0, 2, 5 all 1
+    assert set(O.measure_sample(n, b, [1, 4, 2], rng.random(50))) == {4}  # bits 1, 4, 2 = 0, 0, 1
+
+
+def test_collapse_closed_forms():
+    """GHZ: measuring qubit 0 as 1 leaves |1..1> exactly (P = 1/2); collapse keeps norm 1
+    and equals the renormalised projection of the state."""
+    n = 5
+    psi = O.run_circuit(n, W.ghz(n), W.basis_state(n, 0))
+    p = O.measure_collapse(n, psi, [0], 1)
+    assert abs(p - 0.5) <= 2.3e-16  # |M_SQRT1_2|^2 = 0.5 + 1 ulp
+    ref = np.zeros(1 << n, dtype=complex)
+    ref[-1] = 1.0
+    np.testing.assert_allclose(psi, ref, atol=2e-16)
+    psi0 = W.random_state(7, 3)
+    psi = psi0.copy()
+    p = O.measure_collapse(7, psi, [2, 5], 0b10)
+    k = np.arange(1 << 7)
+    keep = (((k >> 2) & 1) == 0) & (((k >> 5) & 1) == 1)
+    proj = np.where(keep, psi0, 0)
+    assert abs(p - np.sum(np.abs(proj) ** 2)) < 1e-15
+    np.testing.assert_allclose(psi, proj / np.sqrt(p), atol=1e-15)
+    assert abs(O.probs(7, psi)[0] - 1.0) < 1e-14

@@ -53,6 +53,7 @@ def main():
     ap.add_argument("--time", action="store_true")
     ap.add_argument("--no-shuffle", action="store_true")
     ap.add_argument("--no-wide", action="store_true")
+    ap.add_argument("--ipt", type=int, default=0, help="groups per thread for pair gates (0=default)")
     args = ap.parse_args()
     import torch
     import paper_conf_cgo_tarabkhahdds25_b200 as L
@@ -62,6 +63,7 @@ def main():
     with L.State.create(args.n, 0, stream=s) as st:
         st.set_option(L.OPT_LOWQ_SHUFFLE, 0 if args.no_shuffle else 1)
         st.set_option(L.OPT_WIDE256, 0 if args.no_wide else 1)
+        st.set_option(L.OPT_ITEMS_PER_THREAD, args.ipt)
         st.init_random(7)
         for g in gates:
             st.apply(g)  # warm-up

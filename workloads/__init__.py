@@ -241,6 +241,93 @@ def qft(n: int, with_swaps: bool = True) -> List[Gate]:
     return g
 
 
+def qft_inverse(n: int, with_swaps: bool = True) -> List[Gate]:
+    """QFT^dagger: the QFT gate list reversed with negated phases (H, SWAP self-inverse)."""
+    out = []
+    for g in reversed(qft(n, with_swaps)):
+        out.append(Gate(g.kind, g.targets, g.controls, tuple(-p for p in g.params)))
+    return out
+
+
+def qpe(t: int, m: int) -> List[Gate]:
+    """Quantum phase estimation (Table 1 QPE; reading R18).
+
+    Counting register = qubits 0..t-1, eigenstate qubit = t, prepared in |1>
+    (X), U = Phase(2 pi m / 2^t) with eigenvalue e^{2 pi i m/2^t} on |1>.
+    H on the counting qubits, controlled-U^(2^j) = CPhase(2 pi m 2^j / 2^t)
+    (control j, target t), then QFT^dagger on the counting register.  With the
+    exact phase m/2^t the counting register ends in |m> with probability 1.
+    """
+    g: List[Gate] = [Gate("X", (t,))] + [Gate("H", (q,)) for q in range(t)]
+    for j in range(t):
+        g.append(CPHASE(j, t, 2.0 * math.pi * ((m << j) % (1 << t)) / (1 << t)))
+    g += qft_inverse(t)
+    return g
+
+
+def vqe_ansatz(n: int, layers: int, seed: int) -> List[Gate]:
+    """Hardware-efficient VQE ansatz (Table 1 VQE; reading R19): per layer
+    RY(theta) RZ(theta) on every qubit, then a CNOT ladder q -> q+1; angles seeded."""
+    rng = SplitMix64(seed)
+    g: List[Gate] = []
+    for _ in range(layers):
+        for q in range(n):
+            g.append(Gate("RY", (q,), (), (rng.angle(),)))
+            g.append(Gate("RZ", (q,), (), (rng.angle(),)))
+        g += [CNOT(q, q + 1) for q in range(n - 1)]
+    return g
+
+
+def fsim(theta: float, phi: float) -> np.ndarray:
+    """fSim(theta, phi) two-qubit gate (Sycamore coupler; reading R20)."""
+    c, s = math.cos(theta), math.sin(theta)
+    return np.array([[1, 0, 0, 0], [0, c, -1j * s, 0], [0, -1j * s, c, 0],
+                     [0, 0, 0, complex(math.cos(phi), -math.sin(phi))]], dtype=np.complex128)
+
+
+def sycamore_like(rows: int, cols: int, cycles: int, seed: int) -> List[Gate]:
+    """Sycamore-style random circuit on a rows x cols grid (GSC; reading R20):
+    each cycle a random single-qubit gate from {sqrt X, sqrt Y, sqrt W} per qubit (never
+    repeating on a qubit), then fSim(pi/2, pi/6) on one of four coupler patterns
+    (horizontal even/odd, vertical even/odd) in the order A B C D C D A B.  Qubit
+    (r, c) = bit r*cols + c.  The paper's exact coupler layout is not given: parity of
+    this circuit against the paper's instances is unpinned."""
+    n = rows * cols
+    rng = SplitMix64(seed)
+    # sqrt(P) = e^{i pi/4} (I - i P) / sqrt 2 for P in {X, Y, W = (X + Y)/sqrt 2}
+    X = np.array([[0, 1], [1, 0]], dtype=complex)
+    Y = np.array([[0, -1j], [1j, 0]])
+    sx = np.exp(1j * math.pi / 4) * (np.eye(2) - 1j * X) / math.sqrt(2)
+    sy = np.exp(1j * math.pi / 4) * (np.eye(2) - 1j * Y) / math.sqrt(2)
+    Wm = (X + Y) / math.sqrt(2)
+    sw = np.exp(1j * math.pi / 4) * (np.eye(2) - 1j * Wm) / math.sqrt(2)
+    singles = [sx, sy, sw]
+    patterns = []
+    for kind in ("h0", "h1", "v0", "v1"):
+        pairs = []
+        for r in range(rows):
+            for c in range(cols):
+                if kind[0] == "h" and c + 1 < cols and c % 2 == int(kind[1]):
+                    pairs.append((r * cols + c, r * cols + c + 1))
+                if kind[0] == "v" and r + 1 < rows and r % 2 == int(kind[1]):
+                    pairs.append((r * cols + c, (r + 1) * cols + c))
+        patterns.append(pairs)
+    order = [0, 1, 2, 3, 2, 3, 0, 1]
+    F = fsim(math.pi / 2, math.pi / 6)
+    last = [-1] * n
+    g: List[Gate] = []
+    for cyc in range(cycles):
+        for q in range(n):
+            k = rng.below(3)
+            while k == last[q]:
+                k = rng.below(3)
+            last[q] = k
+            g.append(Gate("UNITARY1", (q,), (), (), singles[k]))
+        for (a, b) in patterns[order[cyc % 8]]:
+            g.append(Gate("UNITARY2", (a, b), (), (), F))
+    return g
+
+
 def mcz(n: int) -> Gate:
     """Z on qubit 0 controlled by qubits 1..n-1 (flips the sign of |1...1>)."""
     return Gate("Z", (0,), tuple(range(1, n)))
