@@ -151,7 +151,8 @@ lfqs_status lfqs_run_circuit(lfqs_state* s, const lfqs_gate* gates, size_t n_gat
 
 /* ---- measurement -------------------------------------------- */
 /* probs_out[v] = sum over k with bit qubits[s] of k == bit s of v of |a_k|^2,
- * v in [0, 2^n_q).  n_q = 0 gives the squared norm.  n_q <= 10.  Deterministic
+ * v in [0, 2^n_q).  n_q = 0 gives the squared norm.  n_q <= 20 (one
+ * streaming pass per 10 measured qubits' worth of bins beyond the first 10).  Deterministic
  * (fixed reduction order).  probs_len >= 2^n_q.  Synchronous. */
 lfqs_status lfqs_measure_probs(lfqs_state* s, const int* qubits, int n_q, double* probs_out,
                                size_t probs_len);

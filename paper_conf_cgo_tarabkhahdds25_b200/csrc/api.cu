@@ -262,7 +262,7 @@ lfqs_status lfqs_measure_probs(lfqs_state* s, const int* qubits, int n_q, double
   return guarded([&] {
     require(s != nullptr && probs_out != nullptr, "NULL argument");
     State* st = static_cast<State*>(s);
-    require(n_q >= 0 && n_q <= 10, "n_q must be in [0, 10]");
+    require(n_q >= 0 && n_q <= 20, "n_q must be in [0, 20]");
     require(probs_len >= (size_t(1) << n_q), "probs_len < 2^n_q");
     const uint64_t qm = mask_of(qubits, n_q, st->n);
     (void)qm;
@@ -276,7 +276,7 @@ lfqs_status lfqs_measure_sample(lfqs_state* s, const int* qubits, int n_q, const
     require(s != nullptr && (shots == 0 || (uniforms != nullptr && outcomes != nullptr)),
             "NULL argument");
     State* st = static_cast<State*>(s);
-    require(n_q >= 0 && n_q <= 10, "n_q must be in [0, 10]");
+    require(n_q >= 0 && n_q <= 20, "n_q must be in [0, 20]");
     mask_of(qubits, n_q, st->n);
     std::vector<double> p(size_t(1) << n_q);
     st->measure_probs(qubits, n_q, p.data());
@@ -297,7 +297,7 @@ lfqs_status lfqs_measure_collapse(lfqs_state* s, const int* qubits, int n_q, uin
   return guarded([&] {
     require(s != nullptr, "NULL state");
     State* st = static_cast<State*>(s);
-    require(n_q >= 0 && n_q <= 10, "n_q must be in [0, 10]");
+    require(n_q >= 0 && n_q <= 20, "n_q must be in [0, 20]");
     require(outcome < (uint64_t(1) << n_q), "outcome out of range");
     mask_of(qubits, n_q, st->n);
     std::vector<double> p(size_t(1) << n_q);

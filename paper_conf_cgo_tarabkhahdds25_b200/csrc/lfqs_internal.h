@@ -112,8 +112,9 @@ bool run_fused_circuit(const LaunchCtx& ctx, const std::vector<Decoded>& gates, 
                        size_t end, int tile_qubits, size_t* consumed);
 
 // Reductions (C9): out[v], v < 2^nq; deterministic.
+// Only amplitudes with (k & fmask) == fpat contribute (used to split > 10 qubits).
 void launch_probs(const LaunchCtx& ctx, const int* qubits, int nq, double* d_partials,
-                  int n_partials_blocks, double* d_out);
+                  int n_partials_blocks, double* d_out, uint64_t fmask = 0, uint64_t fpat = 0);
 int probs_blocks();
 
 // Projective collapse: a[k] = (k & mask) == pat ? scale * a[k] : 0 (all zero if

@@ -31,6 +31,7 @@ struct QList {
   int nq;
   int q[kMaxQ];
   uint32_t lane_free;  // lane bits (0..4) not measured: folded by shuffles
+  uint64_t fmask, fpat;  // only amplitudes with (k & fmask) == fpat contribute
 };
 
 __device__ __forceinline__ double2 ldcs(const double2* p) {
@@ -65,7 +66,7 @@ __global__ void __launch_bounds__(kThreads) k_probs(const double2* __restrict__ 
       const uint64_t r = r0 + u;
       if (r < n_rows) {
         const double2 x = ldcs(a + r * 32 + lane);
-        p[u] = x.x * x.x + x.y * x.y;
+        p[u] = ((r * 32 + lane) & ql.fmask) == ql.fpat ? x.x * x.x + x.y * x.y : 0.0;
       } else {
         p[u] = 0.0;
       }
@@ -100,7 +101,8 @@ __global__ void k_probs_tiny(const double2* __restrict__ a, uint64_t n_amps, con
                              double* __restrict__ out) {
   const int nbins = 1 << ql.nq;
   for (int b = 0; b < nbins; ++b) out[b] = 0.0;
-  for (uint64_t k = 0; k < n_amps; ++k) out[bin_of(ql, k)] += a[k].x * a[k].x + a[k].y * a[k].y;
+  for (uint64_t k = 0; k < n_amps; ++k)
+    if ((k & ql.fmask) == ql.fpat) out[bin_of(ql, k)] += a[k].x * a[k].x + a[k].y * a[k].y;
 }
 
 // --- projective collapse (one streaming pass, 32-byte accesses) --------------
@@ -159,11 +161,13 @@ void ensure_smem_attr(const void* kernel, int bytes) {
 }
 
 void launch_probs(const LaunchCtx& ctx, const int* qubits, int nq, double* d_partials,
-                  int n_partials_blocks, double* d_out) {
-  require(nq >= 0 && nq <= kMaxQ, "measure_probs supports at most 10 qubits");
+                  int n_partials_blocks, double* d_out, uint64_t fmask, uint64_t fpat) {
+  require(nq >= 0 && nq <= kMaxQ, "one probability pass covers at most 10 qubits");
   QList ql;
   std::memset(&ql, 0, sizeof ql);
   ql.nq = nq;
+  ql.fmask = fmask;
+  ql.fpat = fpat;
   uint32_t measured_lane_bits = 0;
   for (int s = 0; s < nq; ++s) {
     ql.q[s] = qubits[s];

@@ -321,16 +321,33 @@ void State::collapse(const int* qubits, int nq, uint64_t outcome, double scale) 
   }
 }
 
+// Probabilities of the local physical qubits lq[0..nl) of one shard into host[2^nl]
+// (bit u of the bin = bit lq[u]).  One reduction pass covers 10 qubits; more are
+// enumerated by filtered passes over the extra qubits' patterns.
+void State::local_probs(int shard, const int* lq, int nl, double* host) {
+  const int lo = nl < 10 ? nl : 10;
+  const int nh = nl - lo;
+  for (uint64_t h = 0; h < (1ull << nh); ++h) {
+    uint64_t fmask = 0, fpat = 0;
+    for (int j = 0; j < nh; ++j) {
+      fmask |= 1ull << lq[lo + j];
+      fpat |= ((h >> j) & 1ull) << lq[lo + j];
+    }
+    launch_probs(ctx(shard), lq, lo, d_partials, probs_blocks(), d_probs, fmask, fpat);
+    LFQS_CUDA_CHECK(cudaMemcpyAsync(host + (h << lo), d_probs, sizeof(double) << lo,
+                                    cudaMemcpyDeviceToHost, stream));
+  }
+  LFQS_CUDA_CHECK(cudaStreamSynchronize(stream));
+}
+
 void State::measure_probs(const int* qubits, int nq, double* out) {
   DeviceGuard dg(device);
-  const int nb = 1 << nq;
+  const size_t nb = size_t(1) << nq;
   if (world == 1) {
-    launch_probs(ctx(0), qubits, nq, d_partials, probs_blocks(), d_probs);
-    LFQS_CUDA_CHECK(cudaMemcpyAsync(out, d_probs, sizeof(double) * nb, cudaMemcpyDeviceToHost, stream));
-    LFQS_CUDA_CHECK(cudaStreamSynchronize(stream));
+    local_probs(0, qubits, nq, out);
     return;
   }
-  int lq[10], ls[10], nl = 0;
+  int lq[64], ls[64], nl = 0;
   for (int s = 0; s < nq; ++s) {
     const int P = plan.l2p[qubits[s]];
     if (P < n_local) {
@@ -339,31 +356,31 @@ void State::measure_probs(const int* qubits, int nq, double* out) {
       ++nl;
     }
   }
-  std::vector<double> full(nb, 0.0), loc(1 << nl);
+  std::vector<double> full(nb, 0.0), loc(size_t(1) << nl);
   for (int sh = 0; sh < n_shards(); ++sh) {
     const int r = rank_of_shard(sh);
-    launch_probs(ctx(sh), lq, nl, d_partials, probs_blocks(), d_probs);
-    LFQS_CUDA_CHECK(cudaMemcpyAsync(loc.data(), d_probs, sizeof(double) * (1 << nl),
-                                    cudaMemcpyDeviceToHost, stream));
-    LFQS_CUDA_CHECK(cudaStreamSynchronize(stream));
-    int gbits = 0;
+    local_probs(sh, lq, nl, loc.data());
+    uint64_t gbits = 0;
     for (int s = 0; s < nq; ++s) {
       const int P = plan.l2p[qubits[s]];
-      if (P >= n_local) gbits |= ((r >> (P - n_local)) & 1) << s;
+      if (P >= n_local) gbits |= (uint64_t)((r >> (P - n_local)) & 1) << s;
     }
-    for (int lb = 0; lb < (1 << nl); ++lb) {
-      int v = gbits;
-      for (int u = 0; u < nl; ++u) v |= ((lb >> u) & 1) << ls[u];
+    for (uint64_t lb = 0; lb < (1ull << nl); ++lb) {
+      uint64_t v = gbits;
+      for (int u = 0; u < nl; ++u) v |= ((lb >> u) & 1ull) << ls[u];
       full[v] += loc[lb];
     }
   }
   if (!virt && world > 1) {
-    LFQS_CUDA_CHECK(cudaMemcpyAsync(comm->d_reduce, full.data(), sizeof(double) * nb,
-                                    cudaMemcpyHostToDevice, stream));
-    comm->allreduce_sum(comm->d_reduce, nb, stream);
-    LFQS_CUDA_CHECK(cudaMemcpyAsync(full.data(), comm->d_reduce, sizeof(double) * nb,
-                                    cudaMemcpyDeviceToHost, stream));
+    double* d = comm->d_reduce;
+    if (nb > 1024) LFQS_CUDA_CHECK(cudaMalloc(&d, sizeof(double) * nb));
+    LFQS_CUDA_CHECK(cudaMemcpyAsync(d, full.data(), sizeof(double) * nb, cudaMemcpyHostToDevice,
+                                    stream));
+    comm->allreduce_sum(d, nb, stream);
+    LFQS_CUDA_CHECK(cudaMemcpyAsync(full.data(), d, sizeof(double) * nb, cudaMemcpyDeviceToHost,
+                                    stream));
     LFQS_CUDA_CHECK(cudaStreamSynchronize(stream));
+    if (d != comm->d_reduce) cudaFree(d);
   }
   std::memcpy(out, full.data(), sizeof(double) * nb);
 }

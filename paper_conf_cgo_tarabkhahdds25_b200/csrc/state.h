@@ -50,6 +50,7 @@ struct State : lfqs_state {
   void apply(const Decoded& g);
   void run(const std::vector<Decoded>& gates, uint32_t flags);
   void measure_probs(const int* qubits, int nq, double* out);
+  void local_probs(int shard, const int* lq, int nl, double* host);
   // Zeroes amplitudes whose measured bits != outcome, scales the rest by `scale`.
   void collapse(const int* qubits, int nq, uint64_t outcome, double scale);
   void synchronize();
