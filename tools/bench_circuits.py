@@ -34,6 +34,10 @@ def check(name, n, st, meta):
             / math.sqrt(2.0 ** n)
     elif name == "ghz":
         ref = np.where((idx == 0) | (idx == (1 << n) - 1), math.sqrt(0.5), 0.0).astype(complex)
+    elif name == "qpe":
+        m = meta["m"]
+        p = st.measure_probs(list(range(min(n - 1, 20))))
+        return {"max_abs_err": float(abs(p[m & ((1 << min(n - 1, 20)) - 1)] - 1.0))}
     elif name == "grover":
         k, w = meta["k"], meta["w"]
         th = math.asin(2.0 ** (-n / 2))
@@ -48,7 +52,7 @@ def check(name, n, st, meta):
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--n", type=int, default=30)
-    ap.add_argument("--circuits", default="qft,ghz,grover,random")
+    ap.add_argument("--circuits", default="qft,ghz,grover,random,qpe,vqe,sycamore")
     ap.add_argument("--modes", default="fused,unfused")
     ap.add_argument("--reps", type=int, default=2)
     ap.add_argument("--tile", type=int, default=0)
@@ -67,6 +71,12 @@ def main():
         "ghz": (W.ghz(n), lambda st: st.init_basis(0), {}),
         "grover": (W.grover(n, w, 2), lambda st: st.init_basis(0), {"k": 2, "w": w}),
         "random": (W.random_layered(n, 20, seed=7), lambda st: st.init_basis(0), {}),
+        "qpe": (W.qpe(n - 1, x >> 1), lambda st: st.init_basis(0), {"m": x >> 1}),
+        "vqe": (W.vqe_ansatz(n, 4, seed=5), lambda st: st.init_basis(0), {}),
+        "sycamore": (W.sycamore_like(5, n // 5, 14, seed=6) if n % 5 == 0 else
+                     W.sycamore_like(n // 6, 6, 14, seed=6) + [W.Gate("H", (q,)) for q in
+                                                            range((n // 6) * 6, n)],
+                     lambda st: st.init_basis(0), {}),
         # light programs: fused-pass memory efficiency (one H per qubit; X pairs)
         "hlayer": ([W.Gate("H", (q,)) for q in range(n)], lambda st: st.init_basis(0), {}),
         "xlow": ([W.Gate("X", (0,)), W.Gate("X", (1,))], lambda st: st.init_basis(0), {}),

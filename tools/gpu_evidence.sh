@@ -18,5 +18,6 @@ timeout 900 ncu --metrics gpu__time_duration.sum,dram__bytes_read.sum,dram__byte
 timeout 900 ncu --set full --clock-control none --import-source on -k regex:k_group_x2 -c 2 \
   -o $O/${TAG}_full_dense1 python tools/profile_gates.py --n 28 --reps 1 --gates RX:12,H:20 \
   > $O/${TAG}_ncu_full.out 2>&1
-timeout 600 python tools/bench_circuits.py --n 30 > $O/${TAG}_circuits_n30.jsonl 2>&1
+timeout 900 python tools/bench_circuits.py --n 30 > $O/${TAG}_circuits_n30.jsonl 2>&1
+timeout 1500 python tools/bench_circuits.py --n 33 --reps 1 --modes fused > $O/${TAG}_circuits_n33.jsonl 2>&1
 echo done
