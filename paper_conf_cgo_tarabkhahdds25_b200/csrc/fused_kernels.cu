@@ -376,8 +376,26 @@ __global__ void __launch_bounds__(kFThreads, 2) k_fused(double2* __restrict__ a,
         }
         break;
       }
-      case F_DIAGN: {  // factor d[j], j from the target bits (>= K: from the tile base)
+      case F_DIAGN: {  // factor d[j], j from the target bits (>= 64: outside the tile)
         const int m = h.m;
+        if (m == 1) {  // Rz-like: two entries selected by one bit
+          const double2 d0 = c[0], d1 = c[1];
+          if (t0 >= 64) {
+            const double2 d = ((base >> (t0 - 64)) & 1) ? d1 : d0;
+#pragma unroll
+            for (int r = 0; r < R; ++r) {
+              const uint32_t i = (uint32_t)r * kFThreads + tid;
+              if ((i & mlo) == plo) v[r] = cmul_rn(d, v[r]);
+            }
+          } else {
+#pragma unroll
+            for (int r = 0; r < R; ++r) {
+              const uint32_t i = (uint32_t)r * kFThreads + tid;
+              if ((i & mlo) == plo) v[r] = cmul_rn(((i >> t0) & 1) ? d1 : d0, v[r]);
+            }
+          }
+          break;
+        }
         const int ts[3] = {h.t0, h.t1, h.t2};
         uint32_t jh = 0, jmask = 0;
 #pragma unroll
