@@ -34,7 +34,12 @@ namespace lfqs {
 
 namespace {
 
-enum FType : uint8_t { F_DIAG1 = 0, F_DIAGN, F_X, F_Y, F_H, F_U2, F_SWAP, F_U4, F_U8 };
+// 1-target dense types are specialised by matrix values (static matrix
+// specialisation): F_UR real matrix (Ry), F_UI real diagonal with
+// imaginary off-diagonal (Rx) -- 4 FP64 ops per amplitude instead of 8.
+enum FType : uint8_t {
+  F_DIAG1 = 0, F_DIAGN, F_X, F_Y, F_H, F_UR, F_UI, F_U2, F_SWAP, F_U4, F_U8
+};
 
 struct FHdr {       // 32 bytes
   uint8_t type, m, t0, t1, t2, pad0;
@@ -138,6 +143,31 @@ struct FU_ {
   }
 };
 
+struct FR_ {  // real 2x2 [[m00, m01], [m10, m11]]
+  double m00, m01, m10, m11;
+  __device__ __forceinline__ void pair(double2& a0, double2& a1) const {
+    const double2 x0 = a0, x1 = a1;
+    a0 = make_double2(fma(m01, x1.x, m00 * x0.x), fma(m01, x1.y, m00 * x0.y));
+    a1 = make_double2(fma(m11, x1.x, m10 * x0.x), fma(m11, x1.y, m10 * x0.y));
+  }
+  __device__ __forceinline__ double2 lane(double2 a, double2 p, int bit) const {
+    return bit ? make_double2(fma(m11, a.x, m10 * p.x), fma(m11, a.y, m10 * p.y))
+               : make_double2(fma(m01, p.x, m00 * a.x), fma(m01, p.y, m00 * a.y));
+  }
+};
+struct FI_ {  // [[d0, i e01], [i e10, d1]] with real d0, d1, e01, e10
+  double d0, e01, e10, d1;
+  __device__ __forceinline__ void pair(double2& a0, double2& a1) const {
+    const double2 x0 = a0, x1 = a1;  // i e x = (-e x.y, e x.x)
+    a0 = make_double2(fma(-e01, x1.y, d0 * x0.x), fma(e01, x1.x, d0 * x0.y));
+    a1 = make_double2(fma(d1, x1.x, -e10 * x0.y), fma(d1, x1.y, e10 * x0.x));
+  }
+  __device__ __forceinline__ double2 lane(double2 a, double2 p, int bit) const {
+    return bit ? make_double2(fma(d1, a.x, -e10 * p.y), fma(d1, a.y, e10 * p.x))
+               : make_double2(fma(-e01, p.y, d0 * a.x), fma(e01, p.x, d0 * a.y));
+  }
+};
+
 // ---- shared-memory path ----------------------------------------------------------
 template <class F>
 __device__ __forceinline__ void smem_pairs(double2* tile, const F& f, int t, uint32_t mlo,
@@ -175,6 +205,8 @@ __device__ void smem_op(double2* tile, const FHdr& h, const double2* c, uint32_t
     case F_X: smem_pairs(tile, FX_{}, h.t0, mlo, plo, T); return;
     case F_Y: smem_pairs(tile, FY_{}, h.t0, mlo, plo, T); return;
     case F_H: smem_pairs(tile, FH_{c[0].x}, h.t0, mlo, plo, T); return;
+    case F_UR: smem_pairs(tile, FR_{c[0].x, c[1].x, c[2].x, c[3].x}, h.t0, mlo, plo, T); return;
+    case F_UI: smem_pairs(tile, FI_{c[0].x, c[1].y, c[2].y, c[3].x}, h.t0, mlo, plo, T); return;
     case F_U2: smem_pairs(tile, FU_{c[0], c[1], c[2], c[3]}, h.t0, mlo, plo, T); return;
     case F_SWAP: {
       const int lo = h.t0 < h.t1 ? h.t0 : h.t1, hi = h.t0 < h.t1 ? h.t1 : h.t0;
@@ -428,6 +460,8 @@ __global__ void __launch_bounds__(kFThreads, 2) k_fused(double2* __restrict__ a,
       case F_X: reg_1q<R>(v, FX_{}, t0, mlo, plo, tid); break;
       case F_Y: reg_1q<R>(v, FY_{}, t0, mlo, plo, tid); break;
       case F_H: reg_1q<R>(v, FH_{c[0].x}, t0, mlo, plo, tid); break;
+      case F_UR: reg_1q<R>(v, FR_{c[0].x, c[1].x, c[2].x, c[3].x}, t0, mlo, plo, tid); break;
+      case F_UI: reg_1q<R>(v, FI_{c[0].x, c[1].y, c[2].y, c[3].x}, t0, mlo, plo, tid); break;
       default: reg_1q<R>(v, FU_{c[0], c[1], c[2], c[3]}, t0, mlo, plo, tid); break;
     }
   }
@@ -534,6 +568,13 @@ void encode(const Decoded& g, const TileMap& tm, FProg& P) {
     default:
       if (g.m == 1) {
         h.type = g.is_h ? F_H : F_U2;
+        if (!g.is_h) {
+          const cplx* M = g.M;
+          if (M[0].im == 0.0 && M[1].im == 0.0 && M[2].im == 0.0 && M[3].im == 0.0)
+            h.type = F_UR;
+          else if (M[0].im == 0.0 && M[3].im == 0.0 && M[1].re == 0.0 && M[2].re == 0.0)
+            h.type = F_UI;
+        }
       } else {
         h.type = g.m == 2 ? F_U4 : F_U8;
       }
