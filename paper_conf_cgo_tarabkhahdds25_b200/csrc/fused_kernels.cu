@@ -255,11 +255,14 @@ template <int RB, int R, class F>
 __device__ __forceinline__ void reg_pairs(double2 (&v)[R], const F& f, uint32_t mlo, uint32_t plo,
                                           uint32_t tid) {
   if constexpr ((1 << RB) < R) {
+    // Predicate split: thread bits once, register bits per r (uniform across the block).
+    const bool bt = (tid & mlo & (kFThreads - 1)) == (plo & (kFThreads - 1));
+    const uint32_t mr = mlo >> 8, pr = plo >> 8;
+    if (!bt) return;
 #pragma unroll
     for (int r = 0; r < R; ++r) {
       if (r >> RB & 1) continue;
-      const uint32_t i0 = (uint32_t)r * kFThreads + tid;
-      if ((i0 & mlo) != plo) continue;
+      if (((uint32_t)r & mr) != pr) continue;
       f.pair(v[r], v[r | (1 << RB)]);
     }
   }
@@ -277,15 +280,18 @@ __device__ __forceinline__ void reg_1q(double2 (&v)[R], const F& f, int t0, uint
     }
     return;
   }
-  // Lane bit (t0 < 5): partner lane tid ^ 2^t0.
+  // Lane bit (t0 < 5): partner lane tid ^ 2^t0.  Register-bit part of the
+  // predicate is uniform (skips whole registers); the thread part selects lanes.
   const int bit = (tid >> t0) & 1;
+  const bool bt = (tid & mlo & (kFThreads - 1)) == (plo & (kFThreads - 1));
+  const uint32_t mr = mlo >> 8, pr = plo >> 8;
 #pragma unroll
   for (int r = 0; r < R; ++r) {
+    if (((uint32_t)r & mr) != pr) continue;
     double2 p;
     p.x = __shfl_xor_sync(0xffffffffu, v[r].x, 1 << t0);
     p.y = __shfl_xor_sync(0xffffffffu, v[r].y, 1 << t0);
-    const uint32_t i = (uint32_t)r * kFThreads + tid;
-    if ((i & mlo) == plo) v[r] = f.lane(v[r], p, bit);
+    if (bt) v[r] = f.lane(v[r], p, bit);
   }
 }
 
@@ -676,7 +682,36 @@ bool run_fused_circuit(const LaunchCtx& ctx, const std::vector<Decoded>& gates, 
   }
   P.tile.lc = lc;
   require(b == K && lc + P.tile.nh == K, "internal: bad fused tile");
-  for (size_t q = begin; q < i; ++q) encode(gates[q], tm, P);
+  // Merge runs of 1-target gates on the same qubit with the same controls when at
+  // least one is dense (matrix product on the host; dense results are compared
+  // within rounding, permutation/diagonal-only runs are never merged).
+  std::vector<Decoded> prog;
+  prog.reserve(i - begin);
+  for (size_t q = begin; q < i; ++q) {
+    const Decoded& g = gates[q];
+    if (g.cls == GClass::NOOP) continue;
+    if (!prog.empty()) {
+      Decoded& a = prog.back();
+      if (a.m == 1 && g.m == 1 && a.targets[0] == g.targets[0] && a.cmask == g.cmask &&
+          (a.cls == GClass::DENSE || g.cls == GClass::DENSE)) {
+        cplx C[4];
+        for (int r = 0; r < 2; ++r)
+          for (int c = 0; c < 2; ++c) {
+            const cplx x = g.M[r * 2 + 0], y = a.M[0 * 2 + c], u = g.M[r * 2 + 1],
+                       w = a.M[1 * 2 + c];
+            C[r * 2 + c] = cplx{x.re * y.re - x.im * y.im + (u.re * w.re - u.im * w.im),
+                                x.re * y.im + x.im * y.re + (u.re * w.im + u.im * w.re)};
+          }
+        for (int k = 0; k < 4; ++k) a.M[k] = C[k];
+        a.cls = GClass::DENSE;
+        a.is_h = false;
+        a.kind = LFQS_UNITARY1;
+        continue;
+      }
+    }
+    prog.push_back(g);
+  }
+  for (const Decoded& g : prog) encode(g, tm, P);
   switch (K) {
     case 8: launch_k<8>(ctx, P); break;
     case 9: launch_k<9>(ctx, P); break;
