@@ -1,0 +1,44 @@
+"""Small-n workload for compute-sanitizer (memcheck / racecheck / synccheck):
+every kernel family once -- class kernels, shuffle path, fused TMA and direct
+tiles (incl. smem ops), virtual-partition exchange, probabilities, collapse.
+
+    compute-sanitizer --tool racecheck python tools/sanitize_run.py
+"""
+import os
+import sys
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+
+import workloads as W  # noqa: E402
+
+
+def main():
+    import paper_conf_cgo_tarabkhahdds25_b200 as L
+    n = 14
+    gates = W.random_gate_list(n, 120, seed=1, max_controls=2) + W.qft(n) + \
+        W.random_layered(n, 3, seed=2) + W.sycamore_like(2, 7, 4, seed=3)
+    with L.State.create(n) as st:
+        st.init_random(1)
+        st.set_option(L.OPT_LOWQ_SHUFFLE, 1)
+        st.run_circuit(gates[:120])
+        st.set_option(L.OPT_LOWQ_SHUFFLE, 0)
+        for tma in (256, 0):
+            st.set_option(L.OPT_FUSE_TMA_MAX_CHUNKS, tma)
+            st.run_circuit(gates, fuse=True)
+        st.measure_probs([0, 3, 13])
+        st.measure_probs(list(range(12)))
+        st.sample([1, 2], np.linspace(0, 0.99, 7))
+        st.collapse([5], 1)
+        st.synchronize()
+    with L.State.virtual(n, 4) as st:
+        st.init_random(2)
+        st.run_circuit(gates, fuse=True)
+        st.copy_out(0, 16)
+    print("sanitize workload done")
+
+
+if __name__ == "__main__":
+    main()
