@@ -218,6 +218,8 @@ lfqs_status lfqs_kernel_launches(const lfqs_state* s, uint64_t* count);
                                       the other tile qubits are claimed by the fused gates */
 #define LFQS_OPT_FUSE_TMA_MAX_CHUNKS 6 /* tiles of at most this many chunks move by TMA bulk
                                           copies, larger ones by direct loads (default 256) */
+#define LFQS_OPT_FUSE_REORDER 7 /* 1: fused passes may take later gates that commute exactly
+                                   with the skipped ones (default 1); 0: prefixes only */
 lfqs_status lfqs_set_option(lfqs_state* s, int option, int64_t value);
 const char* lfqs_last_error(void);
 int lfqs_abi_version(void);

@@ -351,6 +351,7 @@ lfqs_status lfqs_set_option(lfqs_state* s, int option, int64_t value) {
         require(value >= 3 && value <= 12, "fused low qubits must be in [3, 12]");
         st->opt.fuse_low_qubits = (int)value;
         break;
+      case LFQS_OPT_FUSE_REORDER: st->opt.fuse_reorder = value != 0; break;
       case LFQS_OPT_FUSE_TMA_MAX_CHUNKS:
         require(value >= 0 && value <= 256, "TMA max chunks must be in [0, 256]");
         st->opt.fuse_tma_max_chunks = (int)value;

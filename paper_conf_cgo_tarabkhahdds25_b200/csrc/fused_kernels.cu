@@ -626,41 +626,45 @@ bool fusable(const Decoded& g, int K, int n_local) {
   return true;
 }
 
-// Greedy segmentation (NEXT-1 "general cache-blocked fusion"): the tile holds
-// qubits [0, L) (contiguous, for coalesced 2^L-amplitude chunks) plus up to
-// K - L further qubits claimed, in gate order, by the targets of non-diagonal
-// gates; diagonal gates need no slot.  Free slots are filled with the lowest
-// remaining qubits (larger contiguous chunks).
-bool run_fused_circuit(const LaunchCtx& ctx, const std::vector<Decoded>& gates, size_t begin,
-                       size_t end, int tile_qubits, size_t* consumed) {
-  *consumed = 0;
+namespace {
+
+struct TileCfg {
+  int K, L, slots;
+};
+
+bool tile_cfg(const LaunchCtx& ctx, int tile_qubits, TileCfg* c) {
   int K = tile_qubits < ctx.n_local ? tile_qubits : ctx.n_local;
   if (K > kMaxK) K = kMaxK;
   if (K < kMinK) return false;
   int L = ctx.opt->fuse_low_qubits;
   if (L > K) L = K;
   if (L < K - kMaxHigh) L = K - kMaxHigh;
-  const int slots = K - L;
-  uint64_t in_tile = (L >= 64) ? ~0ull : ((1ull << L) - 1);
-  int used = 0, nops = 0, ncoef = 0;
-  size_t i = begin;
-  for (; i < end; ++i) {
-    const Decoded& g = gates[i];
-    if (g.cls == GClass::NOOP) continue;
-    if (nops >= kMaxOps || ncoef + coef_count(g) > kMaxCoef) break;
-    if (g.cls != GClass::DIAG) {
-      uint64_t need = 0;
-      for (int s = 0; s < g.m; ++s)
-        if (!(in_tile >> g.targets[s] & 1)) need |= 1ull << g.targets[s];
-      const int nn = __builtin_popcountll(need);
-      if (used + nn > slots) break;
-      in_tile |= need;
-      used += nn;
-    }
-    ++nops;
-    ncoef += coef_count(g);
-  }
-  if (nops < 2) return false;  // a single gate runs faster in its class kernel
+  c->K = K;
+  c->L = L;
+  c->slots = K - L;
+  return true;
+}
+
+// Qubits a non-diagonal gate needs in the tile that it does not have yet.
+uint64_t tile_need(const Decoded& g, uint64_t in_tile) {
+  if (g.cls == GClass::DIAG) return 0;
+  uint64_t need = 0;
+  for (int s = 0; s < g.m; ++s)
+    if (!(in_tile >> g.targets[s] & 1)) need |= 1ull << g.targets[s];
+  return need;
+}
+
+uint64_t qubit_mask(const Decoded& g) {
+  uint64_t m = g.cmask;
+  for (int s = 0; s < g.m; ++s) m |= 1ull << g.targets[s];
+  return m;
+}
+
+// Builds the tile geometry for qubit set in_tile (filled up to K qubits), merges
+// same-qubit 1-target runs containing a dense gate, encodes and launches.
+void launch_program(const LaunchCtx& ctx, const TileCfg& cfg, uint64_t in_tile,
+                    const std::vector<const Decoded*>& list) {
+  const int K = cfg.K;
   for (int q = 0; q < ctx.n_local && __builtin_popcountll(in_tile) < K; ++q) in_tile |= 1ull << q;
   TileMap tm;
   static thread_local FProg P;  // ~32 KB, reused (copied into the launch)
@@ -686,9 +690,9 @@ bool run_fused_circuit(const LaunchCtx& ctx, const std::vector<Decoded>& gates, 
   // least one is dense (matrix product on the host; dense results are compared
   // within rounding, permutation/diagonal-only runs are never merged).
   std::vector<Decoded> prog;
-  prog.reserve(i - begin);
-  for (size_t q = begin; q < i; ++q) {
-    const Decoded& g = gates[q];
+  prog.reserve(list.size());
+  for (const Decoded* gp : list) {
+    const Decoded& g = *gp;
     if (g.cls == GClass::NOOP) continue;
     if (!prog.empty()) {
       Decoded& a = prog.back();
@@ -721,8 +725,104 @@ bool run_fused_circuit(const LaunchCtx& ctx, const std::vector<Decoded>& gates, 
   }
   LFQS_CUDA_CHECK(cudaGetLastError());
   ++*ctx.launch_counter;
+}
+
+}  // namespace
+
+// Greedy segmentation of a gate prefix (NEXT-1 "general cache-blocked fusion"):
+// the tile holds qubits [0, L) (contiguous, for coalesced 2^L-amplitude chunks)
+// plus up to K - L further qubits claimed, in gate order, by the targets of
+// non-diagonal gates; diagonal gates need no slot.  Free slots are filled with
+// the lowest remaining qubits (larger contiguous chunks).
+bool run_fused_circuit(const LaunchCtx& ctx, const std::vector<Decoded>& gates, size_t begin,
+                       size_t end, int tile_qubits, size_t* consumed) {
+  *consumed = 0;
+  TileCfg cfg;
+  if (!tile_cfg(ctx, tile_qubits, &cfg)) return false;
+  uint64_t in_tile = (1ull << cfg.L) - 1;
+  int used = 0, nops = 0, ncoef = 0;
+  std::vector<const Decoded*> list;
+  size_t i = begin;
+  for (; i < end; ++i) {
+    const Decoded& g = gates[i];
+    if (g.cls == GClass::NOOP) continue;
+    if (nops >= kMaxOps || ncoef + coef_count(g) > kMaxCoef) break;
+    const uint64_t need = tile_need(g, in_tile);
+    const int nn = __builtin_popcountll(need);
+    if (used + nn > cfg.slots) break;
+    in_tile |= need;
+    used += nn;
+    ++nops;
+    ncoef += coef_count(g);
+    list.push_back(&g);
+  }
+  if (nops < 2) return false;  // a single gate runs faster in its class kernel
+  launch_program(ctx, cfg, in_tile, list);
   *consumed = i - begin;
   return true;
+}
+
+// Commutation-aware scheduling: each pass walks the remaining gates in order and
+// takes every gate that fits the tile and commutes *exactly* with all gates it
+// skips: disjoint qubits, and never two diagonal gates (whose multiplications on
+// a shared amplitude would round differently in the other order).  Permutation /
+// diagonal results therefore stay bit-identical to gate-by-gate application;
+// dense gates reorder only across disjoint qubits (rounding-level differences).
+void run_fused_schedule(const LaunchCtx& ctx, const std::vector<Decoded>& gates,
+                        int tile_qubits) {
+  TileCfg cfg;
+  std::vector<int> rest;
+  for (size_t i = 0; i < gates.size(); ++i)
+    if (gates[i].cls != GClass::NOOP) rest.push_back((int)i);
+  if (!tile_cfg(ctx, tile_qubits, &cfg)) {
+    for (int i : rest) launch_gate(ctx, gates[i]);
+    return;
+  }
+  constexpr size_t kWindow = 4096;  // gates scanned per pass
+  std::vector<char> taken(gates.size(), 0);
+  size_t head = 0;  // rest[0, head) are done
+  while (head < rest.size()) {
+    uint64_t in_tile = (1ull << cfg.L) - 1, blocked_q = 0;
+    bool blocked_diag = false;
+    int used = 0, nops = 0, ncoef = 0;
+    std::vector<const Decoded*> list;
+    std::vector<int> picked;
+    size_t scanned = 0;
+    for (size_t p = head; p < rest.size() && scanned < kWindow; ++p) {
+      const int gi = rest[p];
+      if (taken[gi]) continue;
+      ++scanned;
+      const Decoded& g = gates[gi];
+      const bool diag = g.cls == GClass::DIAG;
+      const uint64_t qm = qubit_mask(g);
+      bool ok = (qm & blocked_q) == 0 && !(diag && blocked_diag);
+      if (ok && nops < kMaxOps && ncoef + coef_count(g) <= kMaxCoef) {
+        const uint64_t need = tile_need(g, in_tile);
+        const int nn = __builtin_popcountll(need);
+        if (used + nn <= cfg.slots) {
+          in_tile |= need;
+          used += nn;
+          ++nops;
+          ncoef += coef_count(g);
+          list.push_back(&g);
+          picked.push_back(gi);
+          continue;
+        }
+      }
+      blocked_q |= qm;  // later gates touching these qubits must wait
+      blocked_diag |= diag;
+    }
+    if (nops < 2) {
+      // Nothing to fuse with the first remaining gate: its class kernel.
+      while (taken[rest[head]]) ++head;
+      launch_gate(ctx, gates[rest[head]]);
+      taken[rest[head]] = 1;
+    } else {
+      launch_program(ctx, cfg, in_tile, list);
+      for (int gi : picked) taken[gi] = 1;
+    }
+    while (head < rest.size() && taken[rest[head]]) ++head;
+  }
 }
 
 }  // namespace lfqs

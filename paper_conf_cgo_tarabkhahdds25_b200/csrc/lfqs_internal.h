@@ -84,6 +84,7 @@ struct Options {
   bool wide256 = true;       // two adjacent groups per item, 32-byte accesses
   int fuse_tile_qubits = 12;
   int fuse_low_qubits = 7;   // contiguous low qubits of a fused tile (chunk = 2^7 amps)
+  bool fuse_reorder = true;  // commutation-aware scheduling of fused passes
   // Tiles with more chunks load/store directly (no TMA).  Measured on B200 at
   // n=30 (profiles/r01_fused_variants.md): TMA with parallel issue from warp 0
   // beats direct loads for every chunk count up to 128, so TMA is the default.
@@ -110,6 +111,8 @@ void launch_gate(const LaunchCtx& ctx, const Decoded& g);
 // program in one HBM pass; false if fewer than two gates fuse (fused_kernels.cu).
 bool run_fused_circuit(const LaunchCtx& ctx, const std::vector<Decoded>& gates, size_t begin,
                        size_t end, int tile_qubits, size_t* consumed);
+// Whole-list fused execution with exact-commutation reordering (fused_kernels.cu).
+void run_fused_schedule(const LaunchCtx& ctx, const std::vector<Decoded>& gates, int tile_qubits);
 
 // Reductions (C9): out[v], v < 2^nq; deterministic.
 // Only amplitudes with (k & fmask) == fpat contribute (used to split > 10 qubits).

@@ -234,6 +234,10 @@ void State::exchange_data(int l, int g) {
 // A run of local gates on one shard: fused passes where possible, else one
 // class kernel per gate.
 void State::run_local(const LaunchCtx& c, const std::vector<Decoded>& gates, bool fuse) {
+  if (fuse && opt.fuse_reorder) {
+    run_fused_schedule(c, gates, opt.fuse_tile_qubits);
+    return;
+  }
   size_t i = 0;
   while (i < gates.size()) {
     size_t used = 0;

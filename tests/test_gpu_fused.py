@@ -21,8 +21,9 @@ def L():
     return lib
 
 
-def _run(L, n, psi, gates, fuse, tile=None):
+def _run(L, n, psi, gates, fuse, tile=None, reorder=1):
     with L.State.create(n) as st:
+        st.set_option(L.OPT_FUSE_REORDER, reorder)
         if tile:
             st.set_option(L.OPT_FUSE_TILE_QUBITS, tile)
         st.copy_in(psi)
@@ -32,20 +33,27 @@ def _run(L, n, psi, gates, fuse, tile=None):
         return out, st.launches() - c0
 
 
+@pytest.mark.parametrize("reorder", [0, 1])
 @pytest.mark.parametrize("tile", [6, 9, 12, 13])
 @pytest.mark.parametrize("n", [8, 14, 17])
-def test_fused_random_circuit(L, n, tile):
+def test_fused_random_circuit(L, n, tile, reorder):
     psi = W.random_state(n, n + tile)
     gates = W.random_gate_list(n, 250, seed=7 * n + tile, max_controls=2)
     ref = O.run_circuit(n, gates, psi.copy())
-    got, launches = _run(L, n, psi, gates, True, tile)
+    got, launches = _run(L, n, psi, gates, True, tile, reorder)
     assert np.max(np.abs(got - ref)) <= 1e-12
     unf, _ = _run(L, n, psi, gates, False)
     assert np.max(np.abs(got - unf)) <= 1e-12
     exact = [g for g in gates if g.exact]
-    a, _ = _run(L, n, psi, exact, True, tile)
+    a, _ = _run(L, n, psi, exact, True, tile, reorder)
     b, _ = _run(L, n, psi, exact, False)
     assert np.array_equal(a, b)
+    # diagonal gates are never reordered among themselves: a diagonal-only circuit
+    # (QFT's controlled phases included) stays bit-identical to the oracle
+    diag = [g for g in gates if W.KIND_CLASS[g.kind] == "diag"] + \
+        [g for g in W.qft(n) if g.kind == "PHASE"]
+    a, _ = _run(L, n, psi, diag, True, tile, reorder)
+    assert np.array_equal(a, O.run_circuit(n, diag, psi.copy()))
 
 
 @pytest.mark.parametrize("tma", [0, 256])

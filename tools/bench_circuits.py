@@ -57,6 +57,7 @@ def main():
     ap.add_argument("--reps", type=int, default=2)
     ap.add_argument("--tile", type=int, default=0)
     ap.add_argument("--low", type=int, default=0)
+    ap.add_argument("--reorder", type=int, default=1)
     ap.add_argument("--tma", type=int, default=-1, help="max chunks moved by TMA (-1: default)")
     args = ap.parse_args()
     import torch
@@ -89,6 +90,7 @@ def main():
             st.set_option(L.OPT_FUSE_LOW_QUBITS, args.low)
         if args.tma >= 0:
             st.set_option(L.OPT_FUSE_TMA_MAX_CHUNKS, args.tma)
+        st.set_option(L.OPT_FUSE_REORDER, args.reorder)
         for name in args.circuits.split(","):
             gates, init, meta = circuits[name]
             arr = L.marshal_gates(gates)
