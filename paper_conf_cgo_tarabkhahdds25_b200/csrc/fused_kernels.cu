@@ -43,13 +43,10 @@ enum FType : uint8_t {
 
 struct FHdr {       // 32 bytes
   uint8_t type, m, t0, t1, t2, pad0;
-  uint16_t coef;      // offset into the coefficient pool
-  uint16_t mlo, plo;  // per-amplitude predicate (i & mlo) == plo   (tile bits)
-  uint16_t nz;        // U4: bit 4j+i set = entry (j, i) nonzero (sparse fSim-like gates)
-  uint16_t pad1;
-  uint64_t mhi, phi;  // per-tile predicate     (base & mhi) == phi (qubits outside the tile)
+  uint16_t coef;    // offset into the coefficient pool
+  uint32_t mlo, plo;  // per-amplitude predicate (i & mlo) == plo   (bits < K)
+  uint64_t mhi, phi;  // per-tile predicate     (base & mhi) == phi (bits >= K)
 };
-static_assert(sizeof(FHdr) == 32, "FHdr layout");
 constexpr int kMaxOps = 192;
 constexpr int kMaxCoef = 1580;
 constexpr int kMaxHigh = 8;
@@ -187,7 +184,7 @@ __device__ __forceinline__ void smem_pairs(double2* tile, const F& f, int t, uin
 
 template <int L>
 __device__ __forceinline__ void dense_group(double2* tile, const uint32_t (&idx)[L],
-                                            const double2* c, uint32_t nz = 0xffffffffu) {
+                                            const double2* c) {
   double2 v[L], w[L];
 #pragma unroll
   for (int j = 0; j < L; ++j) v[j] = tile[idx[j]];
@@ -195,8 +192,7 @@ __device__ __forceinline__ void dense_group(double2* tile, const uint32_t (&idx)
   for (int j = 0; j < L; ++j) {
     double2 acc = make_double2(0.0, 0.0);
 #pragma unroll
-    for (int i = 0; i < L; ++i)  // zero entries skipped (nz is uniform: a branch, not a predicate)
-      if (L > 4 || (nz >> (j * L + i) & 1)) cfma(acc, c[j * L + i], v[i]);
+    for (int i = 0; i < L; ++i) cfma(acc, c[j * L + i], v[i]);
     w[j] = acc;
   }
 #pragma unroll
@@ -231,7 +227,7 @@ __device__ void smem_op(double2* tile, const FHdr& h, const double2* c, uint32_t
         const uint32_t i = ins0(ins0(p, lo), hi);
         if ((i & mlo) != plo) continue;
         const uint32_t idx[4] = {i, i | (1u << t1), i | (1u << t0), i | (1u << t0) | (1u << t1)};
-        dense_group<4>(tile, idx, c, h.nz);
+        dense_group<4>(tile, idx, c);
       }
       return;
     }
@@ -595,14 +591,8 @@ void encode(const Decoded& g, const TileMap& tm, FProg& P) {
       }
       break;
   }
-  h.mlo = (uint16_t)mlo;
-  h.plo = (uint16_t)plo;
-  h.nz = 0xffff;
-  if (h.type == F_U4) {
-    h.nz = 0;
-    for (int k = 0; k < 16; ++k)
-      if (!(g.M[k].re == 0.0 && g.M[k].im == 0.0)) h.nz |= (uint16_t)(1u << k);
-  }
+  h.mlo = (uint32_t)mlo;
+  h.plo = (uint32_t)plo;
   h.mhi = mhi;
   h.phi = phi;
   ++P.nops;
