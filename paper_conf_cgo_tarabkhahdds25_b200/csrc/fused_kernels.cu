@@ -407,6 +407,7 @@ __global__ void __launch_bounds__(kFThreads, 2) k_fused(double2* __restrict__ a,
         const double2 d = c[0];
         const uint32_t mr = mlo >> 8, pr = plo >> 8;
         const bool bt = (tid & mlo & (kFThreads - 1)) == (plo & (kFThreads - 1));
+        if (!__any_sync(0xffffffffu, bt)) break;  // whole warp inactive (warp-bit predicate)
 #pragma unroll
         for (int r = 0; r < R; ++r) {
           if (((uint32_t)r & mr) != pr) continue;  // uniform across the block
