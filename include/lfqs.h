@@ -105,6 +105,19 @@ lfqs_status lfqs_state_create(int n_qubits, int device, void* cuda_stream, lfqs_
  * 16-byte aligned).  The contents are left as they are. */
 lfqs_status lfqs_state_wrap(int n_qubits, int device, void* dev_ptr, void* cuda_stream,
                             lfqs_state** out);
+/* Precision / partition variants (NEXT-4).  flags: LFQS_STATE_C64 stores
+ * complex64 amplitudes (8 bytes: float re, im) instead of complex128 -- half
+ * the HBM traffic per gate and one more qubit per GPU; arithmetic is fp32 (the
+ * diagonal multiply RN without FMA, as in complex128).  world >= 2 creates a
+ * single-GPU virtual partition (see lfqs_state_create_virtual).  The paper does
+ * not state its precision (R5); complex128 stays the default. */
+#define LFQS_STATE_C64 1u
+lfqs_status lfqs_state_create_ex(int n_qubits, int world, int device, void* cuda_stream,
+                                 uint32_t flags, lfqs_state** out);
+/* Borrow caller memory with the precision given by flags (LFQS_STATE_C64: a
+ * torch complex64 tensor of 2^n elements). */
+lfqs_status lfqs_state_wrap_ex(int n_qubits, int device, void* dev_ptr, void* cuda_stream,
+                               uint32_t flags, lfqs_state** out);
 lfqs_status lfqs_state_destroy(lfqs_state* s);
 /* Re-targets subsequent work to another stream (NULL = the library stream). */
 lfqs_status lfqs_state_set_stream(lfqs_state* s, void* cuda_stream);
@@ -136,6 +149,11 @@ lfqs_status lfqs_state_init_random(lfqs_state* s, uint64_t seed);
  * (logical) qubit order; host buffers hold 2*count doubles.  Synchronous. */
 lfqs_status lfqs_copy_in(lfqs_state* s, uint64_t offset, uint64_t count, const double* host);
 lfqs_status lfqs_copy_out(lfqs_state* s, uint64_t offset, uint64_t count, double* host);
+/* Same for complex64 states without conversion: 2*count floats (re, im).
+ * LFQS_ERR_INVALID_ARG on a complex128 state.  (lfqs_copy_in/out also work on
+ * complex64 states, converting on the host.) */
+lfqs_status lfqs_copy_in_c64(lfqs_state* s, uint64_t offset, uint64_t count, const float* host);
+lfqs_status lfqs_copy_out_c64(lfqs_state* s, uint64_t offset, uint64_t count, float* host);
 
 /* ---- gates ------------------------------------------------------------------ */
 /* One gate, one pass (no fusion).  targets/controls are qubit lists; params has

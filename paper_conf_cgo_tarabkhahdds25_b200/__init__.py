@@ -45,7 +45,9 @@ EXPORTS = [
     "lfqs_apply_gate", "lfqs_run_circuit", "lfqs_measure_probs", "lfqs_synchronize",
     "lfqs_state_info", "lfqs_kernel_launches", "lfqs_set_option", "lfqs_last_error",
     "lfqs_abi_version", "lfqs_plan_circuit", "lfqs_measure_sample", "lfqs_measure_collapse",
+    "lfqs_state_create_ex", "lfqs_state_wrap_ex", "lfqs_copy_in_c64", "lfqs_copy_out_c64",
 ]
+STATE_C64 = 1
 
 
 class LfqsError(RuntimeError):
@@ -109,6 +111,10 @@ def lib():
             "lfqs_state_info": [vp, ip, ip, ip, ip, C.POINTER(vp)],
             "lfqs_kernel_launches": [vp, C.POINTER(u64)],
             "lfqs_set_option": [vp, C.c_int, C.c_int64],
+            "lfqs_state_create_ex": [C.c_int, C.c_int, C.c_int, vp, C.c_uint32, C.POINTER(vp)],
+            "lfqs_state_wrap_ex": [C.c_int, C.c_int, vp, vp, C.c_uint32, C.POINTER(vp)],
+            "lfqs_copy_in_c64": [vp, u64, u64, C.POINTER(C.c_float)],
+            "lfqs_copy_out_c64": [vp, u64, u64, C.POINTER(C.c_float)],
             "lfqs_measure_sample": [vp, ip, C.c_int, dp, C.c_size_t, C.POINTER(u64)],
             "lfqs_measure_collapse": [vp, ip, C.c_int, u64, dp],
             "lfqs_plan_circuit": [C.c_int, C.c_int, C.c_int, C.POINTER(LfqsGate), C.c_size_t,
@@ -168,6 +174,36 @@ def lfqs_state_wrap(n_qubits: int, device: int, dev_ptr: int, stream=None) -> in
     h = C.c_void_p()
     _check(lib().lfqs_state_wrap(n_qubits, device, dev_ptr, _stream_handle(stream), C.byref(h)))
     return h.value
+
+
+def lfqs_state_create_ex(n_qubits: int, world: int = 1, device: int = 0, stream=None,
+                         flags: int = 0) -> int:
+    h = C.c_void_p()
+    _check(lib().lfqs_state_create_ex(n_qubits, world, device, _stream_handle(stream), flags,
+                                      C.byref(h)))
+    return h.value
+
+
+def lfqs_state_wrap_ex(n_qubits: int, device: int, dev_ptr: int, stream=None, flags: int = 0) -> int:
+    h = C.c_void_p()
+    _check(lib().lfqs_state_wrap_ex(n_qubits, device, dev_ptr, _stream_handle(stream), flags,
+                                    C.byref(h)))
+    return h.value
+
+
+def lfqs_copy_in_c64(h: int, offset: int, amps: np.ndarray):
+    a = np.ascontiguousarray(amps, dtype=np.complex64)
+    _check(lib().lfqs_copy_in_c64(h, offset, a.size, a.view(np.float32).ctypes.data_as(
+        C.POINTER(C.c_float))))
+
+
+def lfqs_copy_out_c64(h: int, offset: int, count: int, out: Optional[np.ndarray] = None):
+    if out is None:
+        out = np.empty(count, dtype=np.complex64)
+    assert out.dtype == np.complex64 and out.flags.c_contiguous and out.size >= count
+    _check(lib().lfqs_copy_out_c64(h, offset, count, out.view(np.float32).ctypes.data_as(
+        C.POINTER(C.c_float))))
+    return out
 
 
 def lfqs_state_create_virtual(n_qubits: int, world: int, device: int = 0, stream=None) -> int:
@@ -357,29 +393,40 @@ def lfqs_plan_circuit(n_qubits: int, world: int, rank: int, gates, canonicalize:
 # ---- convenience class ----------------------------------------------------------
 
 class State:
-    """An n-qubit complex128 state vector on a B200 (or sharded across ranks)."""
+    """An n-qubit state vector on a B200 (complex128 by default, complex64 with c64=True),
+    on one GPU, a virtual partition of one GPU, or sharded across ranks."""
 
-    def __init__(self, handle: int, n_qubits: int):
+    def __init__(self, handle: int, n_qubits: int, c64: bool = False):
         self.h = handle
         self.n = n_qubits
+        self.c64 = c64
 
     @classmethod
-    def create(cls, n_qubits: int, device: int = 0, stream=None) -> "State":
+    def create(cls, n_qubits: int, device: int = 0, stream=None, c64: bool = False) -> "State":
+        if c64:
+            return cls(lfqs_state_create_ex(n_qubits, 1, device, stream, STATE_C64), n_qubits, True)
         return cls(lfqs_state_create(n_qubits, device, stream), n_qubits)
 
     @classmethod
     def wrap(cls, tensor, stream=None) -> "State":
-        """Borrow a contiguous torch.complex128 CUDA tensor of 2^n elements."""
+        """Borrow a contiguous torch.complex128 (or complex64) CUDA tensor of 2^n elements."""
         import torch
-        assert tensor.is_cuda and tensor.dtype == torch.complex128 and tensor.is_contiguous()
+        assert tensor.is_cuda and tensor.is_contiguous()
+        assert tensor.dtype in (torch.complex128, torch.complex64)
         n = int(tensor.numel()).bit_length() - 1
         assert tensor.numel() == 1 << n
-        st = cls(lfqs_state_wrap(n, tensor.device.index, tensor.data_ptr(), stream), n)
+        c64 = tensor.dtype == torch.complex64
+        st = cls(lfqs_state_wrap_ex(n, tensor.device.index, tensor.data_ptr(), stream,
+                                    STATE_C64 if c64 else 0), n, c64)
         st._tensor = tensor
         return st
 
     @classmethod
-    def virtual(cls, n_qubits: int, world: int, device: int = 0, stream=None) -> "State":
+    def virtual(cls, n_qubits: int, world: int, device: int = 0, stream=None,
+                c64: bool = False) -> "State":
+        if c64:
+            return cls(lfqs_state_create_ex(n_qubits, world, device, stream, STATE_C64),
+                       n_qubits, True)
         return cls(lfqs_state_create_virtual(n_qubits, world, device, stream), n_qubits)
 
     @classmethod
@@ -411,12 +458,22 @@ class State:
         lfqs_state_init_random(self.h, seed)
 
     def copy_in(self, amps: np.ndarray, offset: int = 0):
-        lfqs_copy_in(self.h, offset, amps)
+        """complex128 input (converted for complex64 states) or complex64 input (raw)."""
+        if self.c64 and getattr(amps, "dtype", None) == np.complex64:
+            lfqs_copy_in_c64(self.h, offset, amps)
+        else:
+            lfqs_copy_in(self.h, offset, amps)
 
     def copy_out(self, offset: int = 0, count: Optional[int] = None, out=None) -> np.ndarray:
+        """complex128 array (complex64 states are widened); see copy_out_c64 for raw."""
         if count is None:
             count = (1 << self.n) - offset
         return lfqs_copy_out(self.h, offset, count, out)
+
+    def copy_out_c64(self, offset: int = 0, count: Optional[int] = None, out=None) -> np.ndarray:
+        if count is None:
+            count = (1 << self.n) - offset
+        return lfqs_copy_out_c64(self.h, offset, count, out)
 
     def apply_gate(self, kind, targets, controls=(), params=(), matrix=None):
         lfqs_apply_gate(self.h, kind, targets, controls, params, matrix)

@@ -76,6 +76,49 @@ lfqs_status lfqs_state_wrap(int n_qubits, int device, void* dev_ptr, void* strea
   });
 }
 
+lfqs_status lfqs_state_create_ex(int n_qubits, int world, int device, void* stream,
+                                 uint32_t flags, lfqs_state** out) {
+  return guarded([&] {
+    require(out != nullptr, "out is NULL");
+    require((flags & ~LFQS_STATE_C64) == 0, "unknown state flags");
+    const bool c64 = (flags & LFQS_STATE_C64) != 0;
+    if (world <= 1)
+      *out = State::create_local(n_qubits, device, static_cast<cudaStream_t>(stream), nullptr, c64);
+    else
+      *out = State::create_virtual(n_qubits, world, device, static_cast<cudaStream_t>(stream), c64);
+  });
+}
+
+lfqs_status lfqs_state_wrap_ex(int n_qubits, int device, void* dev_ptr, void* stream,
+                               uint32_t flags, lfqs_state** out) {
+  return guarded([&] {
+    require(out != nullptr && dev_ptr != nullptr, "NULL argument");
+    require((flags & ~LFQS_STATE_C64) == 0, "unknown state flags");
+    const bool c64 = (flags & LFQS_STATE_C64) != 0;
+    require((reinterpret_cast<uintptr_t>(dev_ptr) & (c64 ? 7 : 15)) == 0,
+            "dev_ptr is not aligned to one amplitude");
+    *out = State::create_local(n_qubits, device, static_cast<cudaStream_t>(stream), dev_ptr, c64);
+  });
+}
+
+lfqs_status lfqs_copy_in_c64(lfqs_state* s, uint64_t offset, uint64_t count, const float* host) {
+  return guarded([&] {
+    require(s != nullptr && (count == 0 || host != nullptr), "NULL argument");
+    State* st = static_cast<State*>(s);
+    require(st->c64, "not a complex64 state");
+    st->copy_raw(offset, count, const_cast<float*>(host), true);
+  });
+}
+
+lfqs_status lfqs_copy_out_c64(lfqs_state* s, uint64_t offset, uint64_t count, float* host) {
+  return guarded([&] {
+    require(s != nullptr && (count == 0 || host != nullptr), "NULL argument");
+    State* st = static_cast<State*>(s);
+    require(st->c64, "not a complex64 state");
+    st->copy_raw(offset, count, host, false);
+  });
+}
+
 lfqs_status lfqs_state_create_virtual(int n_qubits, int world, int device, void* stream,
                                       lfqs_state** out) {
   return guarded([&] {

@@ -8,48 +8,31 @@
 // applies the gate's class-specialised update in place.
 //
 // B200 design: HBM-bound streaming, so
-//   * 16-byte (one complex128) vector loads/stores, 32-byte (LDG/STG.256) when
-//     a target is qubit 0 and the pair is adjacent; evict-first cache policy;
-//   * several independent groups per thread to keep >= 64 B in flight per lane;
-//   * targets below 5 optionally via warp shuffles: each warp loads 512 B
-//     contiguous per instruction and exchanges partners with shfl.xor;
+//   * one-amplitude (16 B) or two-adjacent-amplitude (32 B, LDG/STG.256) vector
+//     accesses with evict-first policy; two adjacent groups per thread when
+//     qubit 0 is free (k_group_x2);
+//   * several independent groups per thread (>= 64 B in flight per lane);
+//   * whole 32-B sectors whenever qubit 0 is a control / fixed diagonal bit /
+//     SWAP target (a 16-B write costs a sector read-modify-write);
+//   * targets below 5 optionally via warp shuffles (k_lowq);
 //   * diagonal gates touch only amplitudes whose factor is not 1;
-//   * the diagonal multiply is RN, no FMA (__dmul_rn/__dsub_rn/__dadd_rn) so
-//     diagonal results are value-exact against the oracle (R8).
+//   * the diagonal multiply is RN, no FMA, so diagonal results are value-exact
+//     against the oracle (R8).
+// Every kernel is templated on the scalar S: double (complex128, default) or
+// float (complex64, NEXT-4).
 #include <cuda_runtime.h>
 
 #include <algorithm>
-#include <type_traits>
 #include <cstring>
+#include <type_traits>
 
+#include "cx.cuh"
 #include "lfqs_internal.h"
 
 namespace lfqs {
 namespace {
 
 constexpr int kThreads = 256;
-
-// ---------------------------------------------------------------------------
-// Memory helpers
-// ---------------------------------------------------------------------------
-__device__ __forceinline__ double2 ld16(const double2* p) {
-  double2 v;
-  asm volatile("ld.global.cs.v2.f64 {%0,%1}, [%2];" : "=d"(v.x), "=d"(v.y) : "l"(p));
-  return v;
-}
-__device__ __forceinline__ void st16(double2* p, double2 v) {
-  asm volatile("st.global.cs.v2.f64 [%0], {%1,%2};" ::"l"(p), "d"(v.x), "d"(v.y) : "memory");
-}
-__device__ __forceinline__ void ld32(const double2* p, double2& a, double2& b) {
-  asm volatile("ld.global.cs.v4.f64 {%0,%1,%2,%3}, [%4];"
-               : "=d"(a.x), "=d"(a.y), "=d"(b.x), "=d"(b.y)
-               : "l"(p));
-}
-__device__ __forceinline__ void st32(double2* p, double2 a, double2 b) {
-  asm volatile("st.global.cs.v4.f64 [%0], {%1,%2,%3,%4};" ::"l"(p), "d"(a.x), "d"(a.y), "d"(b.x),
-               "d"(b.y)
-               : "memory");
-}
 
 // Free index -> amplitude index (insert zero bits at ascending positions, OR ones).
 template <int NPMAX>
@@ -66,61 +49,49 @@ __device__ __forceinline__ uint64_t expand(const InsertPlan& ip, uint64_t g) {
 }
 
 // ---------------------------------------------------------------------------
-// Complex arithmetic
-// ---------------------------------------------------------------------------
-// Pinned complex multiply d*a = (dr ar - di ai, dr ai + di ar), RN, no FMA.
-__device__ __forceinline__ double2 cmul_rn(double2 d, double2 a) {
-  return make_double2(__dsub_rn(__dmul_rn(d.x, a.x), __dmul_rn(d.y, a.y)),
-                      __dadd_rn(__dmul_rn(d.x, a.y), __dmul_rn(d.y, a.x)));
-}
-// Accumulating multiply for dense gates (FMA allowed: tolerance class).
-__device__ __forceinline__ void cfma(double2& acc, double2 m, double2 v) {
-  acc.x = fma(m.x, v.x, acc.x);
-  acc.x = fma(-m.y, v.y, acc.x);
-  acc.y = fma(m.x, v.y, acc.y);
-  acc.y = fma(m.y, v.x, acc.y);
-}
-
-// ---------------------------------------------------------------------------
 // Group operators: v[0..L) = amplitudes at k + off[j] (j = local index).
 // ---------------------------------------------------------------------------
+template <class S>
 struct OpSwap2 {  // X / CNOT / Toffoli / SWAP: moves only (bit-exact)
-  __device__ __forceinline__ void operator()(double2 (&v)[2], uint64_t) const {
-    const double2 t = v[0];
+  __device__ __forceinline__ void operator()(cx<S> (&v)[2], uint64_t) const {
+    const cx<S> t = v[0];
     v[0] = v[1];
     v[1] = t;
   }
 };
+template <class S>
 struct OpSwapMid {  // SWAP(0, t) on the group (00, 01, 10, 11): exchange 01 <-> 10
-  __device__ __forceinline__ void operator()(double2 (&v)[4], uint64_t) const {
-    const double2 t = v[1];
+  __device__ __forceinline__ void operator()(cx<S> (&v)[4], uint64_t) const {
+    const cx<S> t = v[1];
     v[1] = v[2];
     v[2] = t;
   }
 };
+template <class S>
 struct OpY {  // Y = [[0,-i],[i,0]]: v0' = -i v1, v1' = i v0 (moves + sign, exact)
-  __device__ __forceinline__ void operator()(double2 (&v)[2], uint64_t) const {
-    const double2 a0 = v[0], a1 = v[1];
-    v[0] = make_double2(a1.y, -a1.x);
-    v[1] = make_double2(-a0.y, a0.x);
+  __device__ __forceinline__ void operator()(cx<S> (&v)[2], uint64_t) const {
+    const cx<S> a0 = v[0], a1 = v[1];
+    v[0] = mk<S>(a1.y, -a1.x);
+    v[1] = mk<S>(-a0.y, a0.x);
   }
 };
+template <class S>
 struct OpH {  // hadgate, Fig. 12c / Fig. 14: sq2r*(s1+s2), sq2r*(s1-s2)
-  double s;
-  __device__ __forceinline__ void operator()(double2 (&v)[2], uint64_t) const {
-    const double2 a0 = v[0], a1 = v[1];
-    v[0] = make_double2(s * (a0.x + a1.x), s * (a0.y + a1.y));
-    v[1] = make_double2(s * (a0.x - a1.x), s * (a0.y - a1.y));
+  S s;
+  __device__ __forceinline__ void operator()(cx<S> (&v)[2], uint64_t) const {
+    const cx<S> a0 = v[0], a1 = v[1];
+    v[0] = mk<S>(s * (a0.x + a1.x), s * (a0.y + a1.y));
+    v[1] = mk<S>(s * (a0.x - a1.x), s * (a0.y - a1.y));
   }
 };
-template <int L>
+template <class S, int L>
 struct OpDense {  // single_qbit (Fig. 12b) generalised: v' = M v
-  double2 M[L * L];
-  __device__ __forceinline__ void operator()(double2 (&v)[L], uint64_t) const {
-    double2 w[L];
+  cx<S> M[L * L];
+  __device__ __forceinline__ void operator()(cx<S> (&v)[L], uint64_t) const {
+    cx<S> w[L];
 #pragma unroll
     for (int j = 0; j < L; ++j) {
-      double2 acc = make_double2(0.0, 0.0);
+      cx<S> acc = mk<S>(0, 0);
 #pragma unroll
       for (int i = 0; i < L; ++i) cfma(acc, M[j * L + i], v[i]);
       w[j] = acc;
@@ -130,33 +101,37 @@ struct OpDense {  // single_qbit (Fig. 12b) generalised: v' = M v
   }
 };
 // Diagonal, one touched entry per group (Z, S, T, Phase, CZ, CPhase, MC-Z).
+template <class S>
 struct OpNeg {
-  __device__ __forceinline__ void operator()(double2 (&v)[1], uint64_t) const {
-    v[0] = make_double2(-v[0].x, -v[0].y);
+  __device__ __forceinline__ void operator()(cx<S> (&v)[1], uint64_t) const {
+    v[0] = mk<S>(-v[0].x, -v[0].y);
   }
 };
+template <class S>
 struct OpMulI {  // * (0, 1): (-im, re)
-  __device__ __forceinline__ void operator()(double2 (&v)[1], uint64_t) const {
-    v[0] = make_double2(-v[0].y, v[0].x);
+  __device__ __forceinline__ void operator()(cx<S> (&v)[1], uint64_t) const {
+    v[0] = mk<S>(-v[0].y, v[0].x);
   }
 };
+template <class S>
 struct OpMulNI {  // * (0, -1): (im, -re)
-  __device__ __forceinline__ void operator()(double2 (&v)[1], uint64_t) const {
-    v[0] = make_double2(v[0].y, -v[0].x);
+  __device__ __forceinline__ void operator()(cx<S> (&v)[1], uint64_t) const {
+    v[0] = mk<S>(v[0].y, -v[0].x);
   }
 };
+template <class S>
 struct OpMul {  // * d
-  double2 d;
-  __device__ __forceinline__ void operator()(double2 (&v)[1], uint64_t) const {
+  cx<S> d;
+  __device__ __forceinline__ void operator()(cx<S> (&v)[1], uint64_t) const {
     v[0] = cmul_rn(d, v[0]);
   }
 };
 // Diagonal over a whole group: v[j] *= d[j] (Rz, general diagonals; no selects).
-template <int L>
+template <class S, int L>
 struct OpDiagGroup {
-  double2 d[L];
+  cx<S> d[L];
   uint32_t touch;  // bit j set: d[j] != 1
-  __device__ __forceinline__ void operator()(double2 (&v)[L], uint64_t) const {
+  __device__ __forceinline__ void operator()(cx<S> (&v)[L], uint64_t) const {
 #pragma unroll
     for (int j = 0; j < L; ++j)
       if (touch >> j & 1) v[j] = cmul_rn(d[j], v[j]);
@@ -165,12 +140,12 @@ struct OpDiagGroup {
 // A one-amplitude op applied to element `which` of an adjacent pair (bit 0 fixed by
 // a control or diagonal pattern): the pair moves as one 32-byte sector so no
 // sub-sector (16 B) writes reach L2/DRAM.
-template <class Op1>
+template <class S, class Op1>
 struct OpAtPair {
   Op1 op;
   int which;
-  __device__ __forceinline__ void operator()(double2 (&v)[2], uint64_t k) const {
-    double2 t[1];
+  __device__ __forceinline__ void operator()(cx<S> (&v)[2], uint64_t k) const {
+    cx<S> t[1];
     if (which) {
       t[0] = v[1];
       op(t, k);
@@ -184,11 +159,11 @@ struct OpAtPair {
 };
 // A pair op with a control on qubit 0: group (k, k+1, k+2^t, k+2^t+1), the op acts
 // on (v1, v3); all four move as two 32-byte sectors.
-template <class Op2>
+template <class S, class Op2>
 struct OpCtrl0 {
   Op2 op;
-  __device__ __forceinline__ void operator()(double2 (&v)[4], uint64_t k) const {
-    double2 p[2] = {v[1], v[3]};
+  __device__ __forceinline__ void operator()(cx<S> (&v)[4], uint64_t k) const {
+    cx<S> p[2] = {v[1], v[3]};
     op(p, k | 1);
     v[1] = p[0];
     v[3] = p[1];
@@ -203,14 +178,14 @@ struct Offs {
 // ---------------------------------------------------------------------------
 // Generic group kernel: each thread handles U groups; each group reads and
 // writes L amplitudes at k + off[j].  P256: off[2i+1] == off[2i] + 1, so the
-// pair moves as one 32-byte access.
+// pair moves as one access.
 // ---------------------------------------------------------------------------
-template <int L, int U, bool P256, int NPMAX, class Op>
-__global__ void __launch_bounds__(kThreads) k_group(double2* __restrict__ a, uint64_t n_groups,
+template <class S, int L, int U, bool P256, int NPMAX, class Op>
+__global__ void __launch_bounds__(kThreads) k_group(cx<S>* __restrict__ a, uint64_t n_groups,
                                                     const InsertPlan ip, const Offs<L> off,
                                                     const Op op) {
   const uint64_t g0 = (uint64_t)blockIdx.x * (kThreads * U) + threadIdx.x;
-  double2 v[U][L];
+  cx<S> v[U][L];
   uint64_t kk[U];
 #pragma unroll
   for (int u = 0; u < U; ++u) {
@@ -219,10 +194,10 @@ __global__ void __launch_bounds__(kThreads) k_group(double2* __restrict__ a, uin
     if (g < n_groups) {
       if constexpr (P256) {
 #pragma unroll
-        for (int j = 0; j < L; j += 2) ld32(a + kk[u] + off.o[j], v[u][j], v[u][j + 1]);
+        for (int j = 0; j < L; j += 2) ld2(a + kk[u] + off.o[j], v[u][j], v[u][j + 1]);
       } else {
 #pragma unroll
-        for (int j = 0; j < L; ++j) v[u][j] = ld16(a + kk[u] + off.o[j]);
+        for (int j = 0; j < L; ++j) v[u][j] = ld1(a + kk[u] + off.o[j]);
       }
     }
   }
@@ -233,24 +208,24 @@ __global__ void __launch_bounds__(kThreads) k_group(double2* __restrict__ a, uin
       op(v[u], kk[u]);
       if constexpr (P256) {
 #pragma unroll
-        for (int j = 0; j < L; j += 2) st32(a + kk[u] + off.o[j], v[u][j], v[u][j + 1]);
+        for (int j = 0; j < L; j += 2) st2(a + kk[u] + off.o[j], v[u][j], v[u][j + 1]);
       } else {
 #pragma unroll
-        for (int j = 0; j < L; ++j) st16(a + kk[u] + off.o[j], v[u][j]);
+        for (int j = 0; j < L; ++j) st1(a + kk[u] + off.o[j], v[u][j]);
       }
     }
   }
 }
 
 // Two adjacent groups per item when qubit 0 is free (not a target or control):
-// groups at k and k+1 share every 32-byte sector, so each access is one
-// LDG/STG.256 and the instruction count per byte halves.
-template <int L, int U, int NPMAX, class Op>
-__global__ void __launch_bounds__(kThreads) k_group_x2(double2* __restrict__ a, uint64_t n_items,
+// groups at k and k+1 share every sector, so each access is one two-amplitude
+// LDG/STG and the instruction count per byte halves.
+template <class S, int L, int U, int NPMAX, class Op>
+__global__ void __launch_bounds__(kThreads) k_group_x2(cx<S>* __restrict__ a, uint64_t n_items,
                                                        const InsertPlan ip, const Offs<L> off,
                                                        const Op op) {
   const uint64_t i0 = (uint64_t)blockIdx.x * (kThreads * U) + threadIdx.x;
-  double2 v[U][L], w[U][L];
+  cx<S> v[U][L], w[U][L];
   uint64_t kk[U];
 #pragma unroll
   for (int u = 0; u < U; ++u) {
@@ -258,7 +233,7 @@ __global__ void __launch_bounds__(kThreads) k_group_x2(double2* __restrict__ a, 
     kk[u] = expand<NPMAX>(ip, (i < n_items ? i : 0) << 1);
     if (i < n_items) {
 #pragma unroll
-      for (int j = 0; j < L; ++j) ld32(a + kk[u] + off.o[j], v[u][j], w[u][j]);
+      for (int j = 0; j < L; ++j) ld2(a + kk[u] + off.o[j], v[u][j], w[u][j]);
     }
   }
 #pragma unroll
@@ -268,7 +243,7 @@ __global__ void __launch_bounds__(kThreads) k_group_x2(double2* __restrict__ a, 
       op(v[u], kk[u]);
       op(w[u], kk[u] | 1);
 #pragma unroll
-      for (int j = 0; j < L; ++j) st32(a + kk[u] + off.o[j], v[u][j], w[u][j]);
+      for (int j = 0; j < L; ++j) st2(a + kk[u] + off.o[j], v[u][j], w[u][j]);
     }
   }
 }
@@ -280,33 +255,36 @@ __global__ void __launch_bounds__(kThreads) k_group_x2(double2* __restrict__ a, 
 // Controls >= 5 + log2 V are inserted into the chunk index (whole chunks are
 // skipped); controls below that are a per-lane store predicate.
 // ---------------------------------------------------------------------------
+template <class S>
 struct LaneSwap {  // X
-  __device__ __forceinline__ double2 operator()(double2, double2 p, int) const { return p; }
+  __device__ __forceinline__ cx<S> operator()(cx<S>, cx<S> p, int) const { return p; }
 };
+template <class S>
 struct LaneY {  // Y: bit 0 -> -i p ; bit 1 -> i p
-  __device__ __forceinline__ double2 operator()(double2, double2 p, int bit) const {
-    return bit ? make_double2(-p.y, p.x) : make_double2(p.y, -p.x);
+  __device__ __forceinline__ cx<S> operator()(cx<S>, cx<S> p, int bit) const {
+    return bit ? mk<S>(-p.y, p.x) : mk<S>(p.y, -p.x);
   }
 };
+template <class S>
 struct LaneH {
-  double s;
-  __device__ __forceinline__ double2 operator()(double2 a, double2 p, int bit) const {
-    return bit ? make_double2(s * (p.x - a.x), s * (p.y - a.y))
-               : make_double2(s * (a.x + p.x), s * (a.y + p.y));
+  S s;
+  __device__ __forceinline__ cx<S> operator()(cx<S> a, cx<S> p, int bit) const {
+    return bit ? mk<S>(s * (p.x - a.x), s * (p.y - a.y)) : mk<S>(s * (a.x + p.x), s * (a.y + p.y));
   }
 };
+template <class S>
 struct LaneDense {  // out = self[bit] * a + other[bit] * p
-  double2 self_c[2], other_c[2];
-  __device__ __forceinline__ double2 operator()(double2 a, double2 p, int bit) const {
-    double2 acc = make_double2(0.0, 0.0);
+  cx<S> self_c[2], other_c[2];
+  __device__ __forceinline__ cx<S> operator()(cx<S> a, cx<S> p, int bit) const {
+    cx<S> acc = mk<S>(0, 0);
     cfma(acc, bit ? self_c[1] : self_c[0], a);
     cfma(acc, bit ? other_c[1] : other_c[0], p);
     return acc;
   }
 };
 
-template <int V, class LaneOp>
-__global__ void __launch_bounds__(kThreads) k_lowq(double2* __restrict__ a, uint64_t n_chunks,
+template <class S, int V, class LaneOp>
+__global__ void __launch_bounds__(kThreads) k_lowq(cx<S>* __restrict__ a, uint64_t n_chunks,
                                                    const InsertPlan ip_hi, uint64_t low_cmask,
                                                    int t, const LaneOp op) {
   constexpr int kLogV = V == 1 ? 0 : V == 2 ? 1 : V == 4 ? 2 : 3;
@@ -314,17 +292,17 @@ __global__ void __launch_bounds__(kThreads) k_lowq(double2* __restrict__ a, uint
   const uint64_t chunk = (uint64_t)blockIdx.x * (kThreads / 32) + (threadIdx.x >> 5);
   if (chunk >= n_chunks) return;  // warp-uniform
   const uint64_t base = expand<kMaxInsert>(ip_hi, chunk << (5 + kLogV));
-  double2 v[V];
+  cx<S> v[V];
 #pragma unroll
-  for (int j = 0; j < V; ++j) v[j] = ld16(a + base + j * 32 + lane);
+  for (int j = 0; j < V; ++j) v[j] = ld1(a + base + j * 32 + lane);
   const int bit = (lane >> t) & 1;
 #pragma unroll
   for (int j = 0; j < V; ++j) {
-    double2 p;
+    cx<S> p;
     p.x = __shfl_xor_sync(0xffffffffu, v[j].x, 1 << t);
     p.y = __shfl_xor_sync(0xffffffffu, v[j].y, 1 << t);
     const uint64_t k = base + j * 32 + lane;
-    if ((k & low_cmask) == low_cmask) st16(a + k, op(v[j], p, bit));
+    if ((k & low_cmask) == low_cmask) st1(a + k, op(v[j], p, bit));
   }
 }
 
@@ -344,17 +322,20 @@ InsertPlan make_plan(uint64_t zero_bits, uint64_t one_bits) {
   return ip;
 }
 
-inline double2 D2(cplx z) { return make_double2(z.re, z.im); }
+template <class S>
+inline cx<S> CV(cplx z) {
+  return mk<S>((S)z.re, (S)z.im);
+}
 
 inline uint64_t blocks_for(uint64_t items, uint64_t per_block) {
   return (items + per_block - 1) / per_block;
 }
 
-template <int L, int U, bool P256, class Op>
+template <class S, int L, int U, bool P256, class Op>
 void run_group(const LaunchCtx& ctx, uint64_t n_groups, const InsertPlan& ip, const Offs<L>& off,
                const Op& op) {
   if (n_groups == 0) return;
-  auto* a = reinterpret_cast<double2*>(ctx.amps);
+  auto* a = reinterpret_cast<cx<S>*>(ctx.amps);
   bool even = true;
   for (int j = 0; j < L; ++j) even &= (off.o[j] & 1) == 0;
   if constexpr (!P256 && L <= 4) {
@@ -365,9 +346,10 @@ void run_group(const LaunchCtx& ctx, uint64_t n_groups, const InsertPlan& ip, co
         const uint64_t nb = blocks_for(n_items, (uint64_t)kThreads * UX);
         require(nb < (1ull << 31), "grid too large");
         if (ip.np <= 4)
-          k_group_x2<L, UX, 4, Op><<<(unsigned)nb, kThreads, 0, ctx.stream>>>(a, n_items, ip, off, op);
+          k_group_x2<S, L, UX, 4, Op>
+              <<<(unsigned)nb, kThreads, 0, ctx.stream>>>(a, n_items, ip, off, op);
         else
-          k_group_x2<L, UX, kMaxInsert, Op>
+          k_group_x2<S, L, UX, kMaxInsert, Op>
               <<<(unsigned)nb, kThreads, 0, ctx.stream>>>(a, n_items, ip, off, op);
       };
       // Groups per thread (tuning knob LFQS_OPT_ITEMS_PER_THREAD for pair gates).
@@ -386,15 +368,15 @@ void run_group(const LaunchCtx& ctx, uint64_t n_groups, const InsertPlan& ip, co
   const uint64_t nb = blocks_for(n_groups, (uint64_t)kThreads * U);
   require(nb < (1ull << 31), "grid too large");
   if (ip.np <= 4)
-    k_group<L, U, P256, 4, Op><<<(unsigned)nb, kThreads, 0, ctx.stream>>>(a, n_groups, ip, off, op);
+    k_group<S, L, U, P256, 4, Op><<<(unsigned)nb, kThreads, 0, ctx.stream>>>(a, n_groups, ip, off, op);
   else
-    k_group<L, U, P256, kMaxInsert, Op>
+    k_group<S, L, U, P256, kMaxInsert, Op>
         <<<(unsigned)nb, kThreads, 0, ctx.stream>>>(a, n_groups, ip, off, op);
   LFQS_CUDA_CHECK(cudaGetLastError());
   ++*ctx.launch_counter;
 }
 
-template <class LaneOp>
+template <class S, class LaneOp>
 void run_lowq(const LaunchCtx& ctx, int t, uint64_t cmask, const LaneOp& op) {
   constexpr int V = 4, kLogV = 2;
   constexpr int CB = 5 + kLogV;
@@ -404,14 +386,14 @@ void run_lowq(const LaunchCtx& ctx, int t, uint64_t cmask, const LaneOp& op) {
   const uint64_t n_chunks = 1ull << (ctx.n_local - CB - n_hi);
   const uint64_t nb = blocks_for(n_chunks, kThreads / 32);
   require(nb < (1ull << 31), "grid too large");
-  k_lowq<V, LaneOp><<<(unsigned)nb, kThreads, 0, ctx.stream>>>(
-      reinterpret_cast<double2*>(ctx.amps), n_chunks, ip, lo_c, t, op);
+  k_lowq<S, V, LaneOp><<<(unsigned)nb, kThreads, 0, ctx.stream>>>(
+      reinterpret_cast<cx<S>*>(ctx.amps), n_chunks, ip, lo_c, t, op);
   LFQS_CUDA_CHECK(cudaGetLastError());
   ++*ctx.launch_counter;
 }
 
 // 2-amplitude (pair) gate on target t with controls: X, Y, dense 2x2.
-template <class Op, class LaneOp>
+template <class S, class Op, class LaneOp>
 void launch_pair(const LaunchCtx& ctx, const Decoded& g, const Op& op, const LaneOp& lane_op) {
   const int t = g.targets[0];
   const int nc = __builtin_popcountll(g.cmask);
@@ -420,21 +402,21 @@ void launch_pair(const LaunchCtx& ctx, const Decoded& g, const Op& op, const Lan
     // neighbours are rewritten and no 16-byte (sub-sector) writes occur.
     const InsertPlan ip = make_plan((1ull << t) | 1ull, g.cmask & ~1ull);
     Offs<4> off{{0ull, 1ull, 1ull << t, (1ull << t) | 1ull}};
-    run_group<4, 2, true>(ctx, 1ull << (ctx.n_local - 1 - nc), ip, off, OpCtrl0<Op>{op});
+    run_group<S, 4, 2, true>(ctx, 1ull << (ctx.n_local - 1 - nc), ip, off, OpCtrl0<S, Op>{op});
     return;
   }
   constexpr int kCB = 7;
   if (ctx.opt->lowq_shuffle && t < 5 && ctx.n_local >= kCB + __builtin_popcountll(g.cmask >> kCB)) {
-    run_lowq(ctx, t, g.cmask, lane_op);
+    run_lowq<S>(ctx, t, g.cmask, lane_op);
     return;
   }
   const uint64_t n_groups = 1ull << (ctx.n_local - 1 - nc);
   const InsertPlan ip = make_plan(1ull << t, g.cmask);
   Offs<2> off{{0ull, 1ull << t}};
   if (t == 0)
-    run_group<2, 4, true>(ctx, n_groups, ip, off, op);
+    run_group<S, 2, 4, true>(ctx, n_groups, ip, off, op);
   else
-    run_group<2, 4, false>(ctx, n_groups, ip, off, op);
+    run_group<S, 2, 4, false>(ctx, n_groups, ip, off, op);
 }
 
 // Local-index offsets: off[j] = sum_s bit(m-1-s of j) << t_s (reading R2).
@@ -466,19 +448,19 @@ void permute_targets(const Decoded& g, const int* perm, int* t_new, cplx* M_new)
     for (int c = 0; c < d; ++c) M_new[r * d + c] = g.M[old_index(r) * d + old_index(c)];
 }
 
-template <int L>
+template <class S, int L>
 void launch_dense_m(const LaunchCtx& ctx, const Decoded& g) {
   constexpr int m = L == 4 ? 2 : 3;
   // Put qubit 0 (if a target) last, so amplitude pairs (k, k+1) are adjacent
-  // and move as 32-byte accesses.
+  // and move as one access.
   int perm[3] = {0, 1, 2};
   for (int s = 0; s < m; ++s)
     if (g.targets[s] == 0) std::swap(perm[s], perm[m - 1]);
   int t[3];
-  OpDense<L> op;
+  OpDense<S, L> op;
   cplx Mp[64];
   permute_targets(g, perm, t, Mp);
-  for (int i = 0; i < L * L; ++i) op.M[i] = D2(Mp[i]);
+  for (int i = 0; i < L * L; ++i) op.M[i] = CV<S>(Mp[i]);
   uint64_t tmask = 0;
   for (int s = 0; s < m; ++s) tmask |= 1ull << t[s];
   const int nc = __builtin_popcountll(g.cmask);
@@ -486,26 +468,26 @@ void launch_dense_m(const LaunchCtx& ctx, const Decoded& g) {
   const InsertPlan ip = make_plan(tmask, g.cmask);
   const Offs<L> off = group_offsets<L>(t, m);
   if (t[m - 1] == 0)
-    run_group<L, (L == 4 ? 2 : 1), true>(ctx, n_groups, ip, off, op);
+    run_group<S, L, (L == 4 ? 2 : 1), true>(ctx, n_groups, ip, off, op);
   else
-    run_group<L, (L == 4 ? 2 : 1), false>(ctx, n_groups, ip, off, op);
+    run_group<S, L, (L == 4 ? 2 : 1), false>(ctx, n_groups, ip, off, op);
 }
 
-template <class Op1>
+template <class S, class Op1>
 void run_diag_one(const LaunchCtx& ctx, uint64_t n_groups, uint64_t zeros, uint64_t ones,
                   const Op1& op) {
   if ((zeros | ones) & 1) {
     // Qubit 0 is fixed: widen the group to the adjacent pair so every write is a
-    // whole 32-byte sector (a 16-byte write costs a sector read-modify-write).
+    // whole sector (a 16-byte write costs a sector read-modify-write).
     const InsertPlan ip = make_plan((zeros & ~1ull) | 1ull, ones & ~1ull);
-    run_group<2, 4, true>(ctx, n_groups, ip, Offs<2>{{0, 1}},
-                          OpAtPair<Op1>{op, (int)(ones & 1)});
+    run_group<S, 2, 4, true>(ctx, n_groups, ip, Offs<2>{{0, 1}},
+                             OpAtPair<S, Op1>{op, (int)(ones & 1)});
   } else {
-    run_group<1, 4, false>(ctx, n_groups, make_plan(zeros, ones), Offs<1>{{0}}, op);
+    run_group<S, 1, 4, false>(ctx, n_groups, make_plan(zeros, ones), Offs<1>{{0}}, op);
   }
 }
 
-template <int L>
+template <class S, int L>
 void run_diag_group(const LaunchCtx& ctx, const Decoded& g) {
   constexpr int m = L == 2 ? 1 : (L == 4 ? 2 : 3);
   int perm[3] = {0, 1, 2};
@@ -514,10 +496,10 @@ void run_diag_group(const LaunchCtx& ctx, const Decoded& g) {
   int t[3];
   cplx Mp[64];
   permute_targets(g, perm, t, Mp);
-  OpDiagGroup<L> op;
+  OpDiagGroup<S, L> op;
   op.touch = 0;
   for (int j = 0; j < L; ++j) {
-    op.d[j] = D2(Mp[j * L + j]);
+    op.d[j] = CV<S>(Mp[j * L + j]);
     if (!(Mp[j * L + j].re == 1.0 && Mp[j * L + j].im == 0.0)) op.touch |= 1u << j;
   }
   uint64_t tmask = 0;
@@ -527,11 +509,12 @@ void run_diag_group(const LaunchCtx& ctx, const Decoded& g) {
   const InsertPlan ip = make_plan(tmask, g.cmask);
   const Offs<L> off = group_offsets<L>(t, m);
   if (t[m - 1] == 0)
-    run_group<L, (L == 8 ? 1 : 2), true>(ctx, n_groups, ip, off, op);
+    run_group<S, L, (L == 8 ? 1 : 2), true>(ctx, n_groups, ip, off, op);
   else
-    run_group<L, (L == 8 ? 1 : 2), false>(ctx, n_groups, ip, off, op);
+    run_group<S, L, (L == 8 ? 1 : 2), false>(ctx, n_groups, ip, off, op);
 }
 
+template <class S>
 void launch_diag(const LaunchCtx& ctx, const Decoded& g) {
   const int m = g.m, d = 1 << m;
   // Entries != 1 (the only amplitudes that change).
@@ -555,46 +538,36 @@ void launch_diag(const LaunchCtx& ctx, const Decoded& g) {
     const uint64_t n_groups = 1ull << (ctx.n_local - m - nc);
     const cplx z = g.M[active * d + active];
     if (z.re == -1.0 && z.im == 0.0)
-      run_diag_one(ctx, n_groups, zeros, ones, OpNeg{});
+      run_diag_one<S>(ctx, n_groups, zeros, ones, OpNeg<S>{});
     else if (z.re == 0.0 && z.im == 1.0)
-      run_diag_one(ctx, n_groups, zeros, ones, OpMulI{});
+      run_diag_one<S>(ctx, n_groups, zeros, ones, OpMulI<S>{});
     else if (z.re == 0.0 && z.im == -1.0)
-      run_diag_one(ctx, n_groups, zeros, ones, OpMulNI{});
+      run_diag_one<S>(ctx, n_groups, zeros, ones, OpMulNI<S>{});
     else
-      run_diag_one(ctx, n_groups, zeros, ones, OpMul{D2(z)});
+      run_diag_one<S>(ctx, n_groups, zeros, ones, OpMul<S>{CV<S>(z)});
     return;
   }
   if (m == 1)
-    run_diag_group<2>(ctx, g);
+    run_diag_group<S, 2>(ctx, g);
   else if (m == 2)
-    run_diag_group<4>(ctx, g);
+    run_diag_group<S, 4>(ctx, g);
   else
-    run_diag_group<8>(ctx, g);
+    run_diag_group<S, 8>(ctx, g);
 }
 
-}  // namespace
-
-// Virtual-partition exchange: swap the l=1 half of this shard with the l=0 half
-// of the shard `partner_offset_amps` amplitudes further on (same pass structure
-// as a SWAP gate, SURVEY a9).
-void launch_half_swap(const LaunchCtx& ctx, int l, uint64_t partner_offset_amps) {
-  const InsertPlan ip = make_plan(1ull << l, 0);
-  Offs<2> off{{1ull << l, partner_offset_amps}};
-  run_group<2, 4, false>(ctx, 1ull << (ctx.n_local - 1), ip, off, OpSwap2{});
-}
-
-void launch_gate(const LaunchCtx& ctx, const Decoded& g) {
+template <class S>
+void launch_gate_t(const LaunchCtx& ctx, const Decoded& g) {
   switch (g.cls) {
     case GClass::NOOP:
       return;
     case GClass::DIAG:
-      launch_diag(ctx, g);
+      launch_diag<S>(ctx, g);
       return;
     case GClass::PERM_X:
-      launch_pair(ctx, g, OpSwap2{}, LaneSwap{});
+      launch_pair<S>(ctx, g, OpSwap2<S>{}, LaneSwap<S>{});
       return;
     case GClass::PERM_Y:
-      launch_pair(ctx, g, OpY{}, LaneY{});
+      launch_pair<S>(ctx, g, OpY<S>{}, LaneY<S>{});
       return;
     case GClass::PERM_SWAP: {
       const int t0 = g.targets[0], t1 = g.targets[1];
@@ -605,35 +578,56 @@ void launch_gate(const LaunchCtx& ctx, const Decoded& g) {
         // the middle two, instead of 16-byte writes into half-used sectors.
         const uint64_t t = 1ull << (t0 == 0 ? t1 : t0);
         Offs<4> off{{0ull, 1ull, t, t | 1ull}};
-        run_group<4, 2, true>(ctx, 1ull << (ctx.n_local - 2 - nc), ip, off, OpSwapMid{});
+        run_group<S, 4, 2, true>(ctx, 1ull << (ctx.n_local - 2 - nc), ip, off, OpSwapMid<S>{});
         return;
       }
       Offs<2> off{{1ull << t0, 1ull << t1}};
-      run_group<2, 4, false>(ctx, 1ull << (ctx.n_local - 2 - nc), ip, off, OpSwap2{});
+      run_group<S, 2, 4, false>(ctx, 1ull << (ctx.n_local - 2 - nc), ip, off, OpSwap2<S>{});
       return;
     }
     case GClass::DENSE:
       if (g.m == 1) {
         if (g.is_h) {
-          const double s = g.M[0].re;
-          launch_pair(ctx, g, OpH{s}, LaneH{s});
+          const S s = (S)g.M[0].re;
+          launch_pair<S>(ctx, g, OpH<S>{s}, LaneH<S>{s});
         } else {
-          OpDense<2> op;
-          for (int i = 0; i < 4; ++i) op.M[i] = D2(g.M[i]);
-          LaneDense lop;
-          lop.self_c[0] = D2(g.M[0]);   // u00
-          lop.self_c[1] = D2(g.M[3]);   // u11
-          lop.other_c[0] = D2(g.M[1]);  // u01
-          lop.other_c[1] = D2(g.M[2]);  // u10
-          launch_pair(ctx, g, op, lop);
+          OpDense<S, 2> op;
+          for (int i = 0; i < 4; ++i) op.M[i] = CV<S>(g.M[i]);
+          LaneDense<S> lop;
+          lop.self_c[0] = CV<S>(g.M[0]);   // u00
+          lop.self_c[1] = CV<S>(g.M[3]);   // u11
+          lop.other_c[0] = CV<S>(g.M[1]);  // u01
+          lop.other_c[1] = CV<S>(g.M[2]);  // u10
+          launch_pair<S>(ctx, g, op, lop);
         }
       } else if (g.m == 2) {
-        launch_dense_m<4>(ctx, g);
+        launch_dense_m<S, 4>(ctx, g);
       } else {
-        launch_dense_m<8>(ctx, g);
+        launch_dense_m<S, 8>(ctx, g);
       }
       return;
   }
+}
+
+}  // namespace
+
+// Virtual-partition exchange: swap the l=1 half of this shard with the l=0 half
+// of the shard `partner_offset_amps` amplitudes further on (same pass structure
+// as a SWAP gate, SURVEY a9).
+void launch_half_swap(const LaunchCtx& ctx, int l, uint64_t partner_offset_amps) {
+  const InsertPlan ip = make_plan(1ull << l, 0);
+  Offs<2> off{{1ull << l, partner_offset_amps}};
+  if (ctx.c64)
+    run_group<float, 2, 4, false>(ctx, 1ull << (ctx.n_local - 1), ip, off, OpSwap2<float>{});
+  else
+    run_group<double, 2, 4, false>(ctx, 1ull << (ctx.n_local - 1), ip, off, OpSwap2<double>{});
+}
+
+void launch_gate(const LaunchCtx& ctx, const Decoded& g) {
+  if (ctx.c64)
+    launch_gate_t<float>(ctx, g);
+  else
+    launch_gate_t<double>(ctx, g);
 }
 
 }  // namespace lfqs

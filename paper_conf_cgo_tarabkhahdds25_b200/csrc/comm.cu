@@ -40,9 +40,9 @@ Comm::Comm(int rank_, int world_, const uint8_t uid[128], size_t stage_bytes)
   std::memcpy(&id, uid, 128);
   LFQS_NCCL_CHECK(ncclCommInitRank(&comm, world, id, rank));
   LFQS_CUDA_CHECK(cudaStreamCreateWithFlags(&cstream, cudaStreamNonBlocking));
-  stage_amps = stage_bytes / 16;
+  this->stage_bytes = stage_bytes;
   for (int i = 0; i < 2; ++i) {
-    LFQS_CUDA_CHECK(cudaMalloc(&stage[i], stage_amps * 16));
+    LFQS_CUDA_CHECK(cudaMalloc(&stage[i], stage_bytes));
     LFQS_CUDA_CHECK(cudaEventCreateWithFlags(&ev_recv[i], cudaEventDisableTiming));
     LFQS_CUDA_CHECK(cudaEventCreateWithFlags(&ev_free[i], cudaEventDisableTiming));
   }
@@ -65,25 +65,28 @@ Comm::~Comm() {
 
 // Exchanges the amplitudes at `pieces` (offset, count in amplitudes, in this
 // rank's shard) with the same pieces of `partner`, in place.
-void Comm::exchange(double* shard, const std::vector<Piece>& pieces, int partner,
+void Comm::exchange(void* shard, int amp_bytes, const std::vector<Piece>& pieces, int partner,
                     cudaStream_t compute) {
   // The comm stream must see every kernel already queued on the compute stream.
   LFQS_CUDA_CHECK(cudaEventRecord(ev_start, compute));
   LFQS_CUDA_CHECK(cudaStreamWaitEvent(cstream, ev_start, 0));
+  const uint64_t stage_amps = stage_bytes / amp_bytes;
+  unsigned char* base = static_cast<unsigned char*>(shard);
   int c = 0;
   for (const Piece& pc : pieces) {
     for (uint64_t off = 0; off < pc.count; off += stage_amps) {
       const uint64_t cnt = std::min<uint64_t>(stage_amps, pc.count - off);
+      const size_t bytes = cnt * amp_bytes;
       const int b = c & 1;
       if (c >= 2) LFQS_CUDA_CHECK(cudaStreamWaitEvent(cstream, ev_free[b], 0));
-      double* src = shard + 2 * (pc.offset + off);
+      unsigned char* src = base + (pc.offset + off) * amp_bytes;
       LFQS_NCCL_CHECK(ncclGroupStart());
-      LFQS_NCCL_CHECK(ncclSend(src, 2 * cnt, ncclDouble, partner, comm, cstream));
-      LFQS_NCCL_CHECK(ncclRecv(stage[b], 2 * cnt, ncclDouble, partner, comm, cstream));
+      LFQS_NCCL_CHECK(ncclSend(src, bytes, ncclUint8, partner, comm, cstream));
+      LFQS_NCCL_CHECK(ncclRecv(stage[b], bytes, ncclUint8, partner, comm, cstream));
       LFQS_NCCL_CHECK(ncclGroupEnd());
       LFQS_CUDA_CHECK(cudaEventRecord(ev_recv[b], cstream));
       LFQS_CUDA_CHECK(cudaStreamWaitEvent(compute, ev_recv[b], 0));
-      LFQS_CUDA_CHECK(cudaMemcpyAsync(src, stage[b], cnt * 16, cudaMemcpyDeviceToDevice, compute));
+      LFQS_CUDA_CHECK(cudaMemcpyAsync(src, stage[b], bytes, cudaMemcpyDeviceToDevice, compute));
       LFQS_CUDA_CHECK(cudaEventRecord(ev_free[b], compute));
       ++c;
     }

@@ -20,15 +20,17 @@ struct Comm {
   int rank = 0, world = 1;
   ncclComm_t comm = nullptr;
   cudaStream_t cstream = nullptr;
-  double* stage[2] = {nullptr, nullptr};
-  uint64_t stage_amps = 0;
+  unsigned char* stage[2] = {nullptr, nullptr};
+  uint64_t stage_bytes = 0;
   cudaEvent_t ev_recv[2], ev_free[2], ev_start;
   double* d_reduce = nullptr;
 
   static void unique_id(uint8_t uid[128]);
   Comm(int rank, int world, const uint8_t uid[128], size_t stage_bytes);
   ~Comm();
-  void exchange(double* shard, const std::vector<Piece>& pieces, int partner, cudaStream_t compute);
+  // pieces are in amplitudes of `amp_bytes` bytes each.
+  void exchange(void* shard, int amp_bytes, const std::vector<Piece>& pieces, int partner,
+                cudaStream_t compute);
   void allreduce_sum(double* d, size_t count, cudaStream_t s);
 };
 

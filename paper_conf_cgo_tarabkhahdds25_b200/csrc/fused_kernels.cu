@@ -1,33 +1,39 @@
-// fused_kernels.cu -- staging of consecutive gates in one HBM pass.
+// fused_kernels.cu -- staging of several gates in one HBM pass.
 //
 // The paper applies every gate as its own pass and exposes every intermediate
 // state; the optimised kernel of each gate is one pass over S (vector
 // fusion).  On B200 a pass over a 16-128 GiB state costs 5-35 ms of
-// HBM time while the arithmetic of one gate costs far less, so a run of
-// consecutive gates that only mix amplitudes inside a 2^K tile is applied in
-// ONE pass (LFQS_FUSE_LOW):
-//   * the tile (2^K contiguous amplitudes, K <= 12 -> 64 KiB) is staged into
-//     shared memory with one TMA bulk copy (cp.async.bulk + mbarrier) and
-//     written back with one bulk store;
+// HBM time while the arithmetic of one gate costs far less, so gates that only
+// mix amplitudes inside a tile of 2^K amplitudes are applied in ONE pass
+// (LFQS_FUSE_LOW):
+//   * a tile is qubits [0, lc) (one contiguous chunk of 2^lc amplitudes) plus
+//     up to 8 further qubits claimed by the fused gates' targets (NEXT-1
+//     "general cache-blocked fusion"); diagonal gates need no tile qubit (bits
+//     outside the tile come from the tile index); controls outside the tile are
+//     per-tile predicates;
+//   * tiles move by TMA bulk copies (cp.async.bulk + mbarrier; one copy per
+//     chunk, issued in parallel by the 32 lanes of warp 0), or by direct
+//     coalesced loads/stores (LFQS_OPT_FUSE_TMA_MAX_CHUNKS);
 //   * the gate program is a __grid_constant__ kernel parameter (<= 32 KB:
-//     headers + a coefficient pool), read through the constant cache -- no
-//     global-memory round trips inside the op loop;
+//     headers + a coefficient pool), read through the constant cache;
 //   * amplitudes live in registers: thread `tid` of 256 holds tile elements
 //     i = r * 256 + tid, r < 2^(K-8).  Diagonal gates, and 1-target gates on
 //     register bits (8..K-1) or lane bits (0..4, via shfl.xor), are applied in
 //     registers; 1-target gates on warp bits (5..7) and 2/3-target gates go
 //     through the shared-memory tile;
-//   * a gate fuses when all its targets are < K (controls anywhere: controls
-//     >= K are a per-tile predicate) or when it is diagonal (any qubits: target
-//     bits >= K come from the tile index).
+//   * scheduling (run_fused_schedule) takes later gates into a pass when they
+//     commute *exactly* with the gates they skip.
 // Permutation and diagonal gates use exactly the unfused formulas (moves;
 // RN complex multiply without FMA, skipped where the factor is exactly 1), so
 // fused == unfused value-exactly for them; dense gates agree within rounding.
+// Kernels are templated on the amplitude scalar S (double: complex128; float:
+// complex64, NEXT-4); the program's coefficients are stored in double.
 #include <cuda_runtime.h>
 
 #include <cstring>
 #include <vector>
 
+#include "cx.cuh"
 #include "lfqs_internal.h"
 
 namespace lfqs {
@@ -36,7 +42,7 @@ namespace {
 
 // 1-target dense types are specialised by matrix values (static matrix
 // specialisation): F_UR real matrix (Ry), F_UI real diagonal with
-// imaginary off-diagonal (Rx) -- 4 FP64 ops per amplitude instead of 8.
+// imaginary off-diagonal (Rx) -- 4 FP ops per amplitude instead of 8.
 enum FType : uint8_t {
   F_DIAG1 = 0, F_DIAGN, F_X, F_Y, F_H, F_UR, F_UI, F_U2, F_SWAP, F_U4, F_U8
 };
@@ -44,8 +50,8 @@ enum FType : uint8_t {
 struct FHdr {       // 32 bytes
   uint8_t type, m, t0, t1, t2, pad0;
   uint16_t coef;    // offset into the coefficient pool
-  uint32_t mlo, plo;  // per-amplitude predicate (i & mlo) == plo   (bits < K)
-  uint64_t mhi, phi;  // per-tile predicate     (base & mhi) == phi (bits >= K)
+  uint32_t mlo, plo;  // per-amplitude predicate (i & mlo) == plo   (tile bits)
+  uint64_t mhi, phi;  // per-tile predicate     (base & mhi) == phi (qubits outside the tile)
 };
 constexpr int kMaxOps = 192;
 constexpr int kMaxCoef = 1580;
@@ -73,56 +79,56 @@ constexpr int kMinK = 8, kMaxK = 12;
 __device__ __forceinline__ uint32_t smem_u32(const void* p) {
   return static_cast<uint32_t>(__cvta_generic_to_shared(p));
 }
-__device__ __forceinline__ double2 cmul_rn(double2 d, double2 a) {
-  return make_double2(__dsub_rn(__dmul_rn(d.x, a.x), __dmul_rn(d.y, a.y)),
-                      __dadd_rn(__dmul_rn(d.x, a.y), __dmul_rn(d.y, a.x)));
-}
-__device__ __forceinline__ void cfma(double2& acc, double2 m, double2 v) {
-  acc.x = fma(m.x, v.x, acc.x);
-  acc.x = fma(-m.y, v.y, acc.x);
-  acc.y = fma(m.x, v.y, acc.y);
-  acc.y = fma(m.y, v.x, acc.y);
-}
 __device__ __forceinline__ uint32_t ins0(uint32_t p, int t) {
   return ((p >> t) << (t + 1)) | (p & ((1u << t) - 1));
 }
-__device__ __forceinline__ bool is_one(double2 d) { return d.x == 1.0 && d.y == 0.0; }
+template <class C>
+__device__ __forceinline__ bool is_one(C d) {
+  return d.x == 1 && d.y == 0;
+}
+template <class S>
+__device__ __forceinline__ cx<S> cvs(double2 z) {  // program coefficient -> amplitude type
+  return mk<S>((S)z.x, (S)z.y);
+}
 
 // ---- 2x2 functors (type dispatched once per op) ------------------------------
+template <class S>
 struct FX_ {
-  __device__ __forceinline__ void pair(double2& a0, double2& a1) const {
-    const double2 t = a0;
+  __device__ __forceinline__ void pair(cx<S>& a0, cx<S>& a1) const {
+    const cx<S> t = a0;
     a0 = a1;
     a1 = t;
   }
-  __device__ __forceinline__ double2 lane(double2, double2 p, int) const { return p; }
+  __device__ __forceinline__ cx<S> lane(cx<S>, cx<S> p, int) const { return p; }
 };
+template <class S>
 struct FY_ {
-  __device__ __forceinline__ void pair(double2& a0, double2& a1) const {
-    const double2 x0 = a0, x1 = a1;
-    a0 = make_double2(x1.y, -x1.x);
-    a1 = make_double2(-x0.y, x0.x);
+  __device__ __forceinline__ void pair(cx<S>& a0, cx<S>& a1) const {
+    const cx<S> x0 = a0, x1 = a1;
+    a0 = mk<S>(x1.y, -x1.x);
+    a1 = mk<S>(-x0.y, x0.x);
   }
-  __device__ __forceinline__ double2 lane(double2, double2 p, int bit) const {
-    return bit ? make_double2(-p.y, p.x) : make_double2(p.y, -p.x);
+  __device__ __forceinline__ cx<S> lane(cx<S>, cx<S> p, int bit) const {
+    return bit ? mk<S>(-p.y, p.x) : mk<S>(p.y, -p.x);
   }
 };
+template <class S>
 struct FH_ {
-  double s;
-  __device__ __forceinline__ void pair(double2& a0, double2& a1) const {
-    const double2 x0 = a0, x1 = a1;
-    a0 = make_double2(s * (x0.x + x1.x), s * (x0.y + x1.y));
-    a1 = make_double2(s * (x0.x - x1.x), s * (x0.y - x1.y));
+  S s;
+  __device__ __forceinline__ void pair(cx<S>& a0, cx<S>& a1) const {
+    const cx<S> x0 = a0, x1 = a1;
+    a0 = mk<S>(s * (x0.x + x1.x), s * (x0.y + x1.y));
+    a1 = mk<S>(s * (x0.x - x1.x), s * (x0.y - x1.y));
   }
-  __device__ __forceinline__ double2 lane(double2 a, double2 p, int bit) const {
-    return bit ? make_double2(s * (p.x - a.x), s * (p.y - a.y))
-               : make_double2(s * (a.x + p.x), s * (a.y + p.y));
+  __device__ __forceinline__ cx<S> lane(cx<S> a, cx<S> p, int bit) const {
+    return bit ? mk<S>(s * (p.x - a.x), s * (p.y - a.y)) : mk<S>(s * (a.x + p.x), s * (a.y + p.y));
   }
 };
+template <class S>
 struct FU_ {
-  double2 c0, c1, c2, c3;
-  __device__ __forceinline__ void pair(double2& a0, double2& a1) const {
-    double2 b0 = make_double2(0.0, 0.0), b1 = b0;
+  cx<S> c0, c1, c2, c3;
+  __device__ __forceinline__ void pair(cx<S>& a0, cx<S>& a1) const {
+    cx<S> b0 = mk<S>(0, 0), b1 = b0;
     cfma(b0, c0, a0);
     cfma(b0, c1, a1);
     cfma(b1, c2, a0);
@@ -130,8 +136,8 @@ struct FU_ {
     a0 = b0;
     a1 = b1;
   }
-  __device__ __forceinline__ double2 lane(double2 a, double2 p, int bit) const {
-    double2 acc = make_double2(0.0, 0.0);
+  __device__ __forceinline__ cx<S> lane(cx<S> a, cx<S> p, int bit) const {
+    cx<S> acc = mk<S>(0, 0);
     if (bit) {
       cfma(acc, c2, p);
       cfma(acc, c3, a);
@@ -142,79 +148,88 @@ struct FU_ {
     return acc;
   }
 };
-
+template <class S>
 struct FR_ {  // real 2x2 [[m00, m01], [m10, m11]]
-  double m00, m01, m10, m11;
-  __device__ __forceinline__ void pair(double2& a0, double2& a1) const {
-    const double2 x0 = a0, x1 = a1;
-    a0 = make_double2(fma(m01, x1.x, m00 * x0.x), fma(m01, x1.y, m00 * x0.y));
-    a1 = make_double2(fma(m11, x1.x, m10 * x0.x), fma(m11, x1.y, m10 * x0.y));
+  S m00, m01, m10, m11;
+  __device__ __forceinline__ void pair(cx<S>& a0, cx<S>& a1) const {
+    const cx<S> x0 = a0, x1 = a1;
+    a0 = mk<S>(fma_(m01, x1.x, m00 * x0.x), fma_(m01, x1.y, m00 * x0.y));
+    a1 = mk<S>(fma_(m11, x1.x, m10 * x0.x), fma_(m11, x1.y, m10 * x0.y));
   }
-  __device__ __forceinline__ double2 lane(double2 a, double2 p, int bit) const {
-    return bit ? make_double2(fma(m11, a.x, m10 * p.x), fma(m11, a.y, m10 * p.y))
-               : make_double2(fma(m01, p.x, m00 * a.x), fma(m01, p.y, m00 * a.y));
+  __device__ __forceinline__ cx<S> lane(cx<S> a, cx<S> p, int bit) const {
+    return bit ? mk<S>(fma_(m11, a.x, m10 * p.x), fma_(m11, a.y, m10 * p.y))
+               : mk<S>(fma_(m01, p.x, m00 * a.x), fma_(m01, p.y, m00 * a.y));
   }
 };
+template <class S>
 struct FI_ {  // [[d0, i e01], [i e10, d1]] with real d0, d1, e01, e10
-  double d0, e01, e10, d1;
-  __device__ __forceinline__ void pair(double2& a0, double2& a1) const {
-    const double2 x0 = a0, x1 = a1;  // i e x = (-e x.y, e x.x)
-    a0 = make_double2(fma(-e01, x1.y, d0 * x0.x), fma(e01, x1.x, d0 * x0.y));
-    a1 = make_double2(fma(d1, x1.x, -e10 * x0.y), fma(d1, x1.y, e10 * x0.x));
+  S d0, e01, e10, d1;
+  __device__ __forceinline__ void pair(cx<S>& a0, cx<S>& a1) const {
+    const cx<S> x0 = a0, x1 = a1;  // i e x = (-e x.y, e x.x)
+    a0 = mk<S>(fma_(-e01, x1.y, d0 * x0.x), fma_(e01, x1.x, d0 * x0.y));
+    a1 = mk<S>(fma_(d1, x1.x, -e10 * x0.y), fma_(d1, x1.y, e10 * x0.x));
   }
-  __device__ __forceinline__ double2 lane(double2 a, double2 p, int bit) const {
-    return bit ? make_double2(fma(d1, a.x, -e10 * p.y), fma(d1, a.y, e10 * p.x))
-               : make_double2(fma(-e01, p.y, d0 * a.x), fma(e01, p.x, d0 * a.y));
+  __device__ __forceinline__ cx<S> lane(cx<S> a, cx<S> p, int bit) const {
+    return bit ? mk<S>(fma_(d1, a.x, -e10 * p.y), fma_(d1, a.y, e10 * p.x))
+               : mk<S>(fma_(-e01, p.y, d0 * a.x), fma_(e01, p.x, d0 * a.y));
   }
 };
 
 // ---- shared-memory path ----------------------------------------------------------
-template <class F>
-__device__ __forceinline__ void smem_pairs(double2* tile, const F& f, int t, uint32_t mlo,
+template <class S, class F>
+__device__ __forceinline__ void smem_pairs(cx<S>* tile, const F& f, int t, uint32_t mlo,
                                            uint32_t plo, uint32_t T) {
   for (uint32_t p = threadIdx.x; p < (T >> 1); p += kFThreads) {
     const uint32_t i0 = ins0(p, t), i1 = i0 | (1u << t);
     if ((i0 & mlo) != plo) continue;
-    double2 a0 = tile[i0], a1 = tile[i1];
+    cx<S> a0 = tile[i0], a1 = tile[i1];
     f.pair(a0, a1);
     tile[i0] = a0;
     tile[i1] = a1;
   }
 }
 
-template <int L>
-__device__ __forceinline__ void dense_group(double2* tile, const uint32_t (&idx)[L],
+template <class S, int L>
+__device__ __forceinline__ void dense_group(cx<S>* tile, const uint32_t (&idx)[L],
                                             const double2* c) {
-  double2 v[L], w[L];
+  cx<S> v[L], w[L];
 #pragma unroll
   for (int j = 0; j < L; ++j) v[j] = tile[idx[j]];
 #pragma unroll
   for (int j = 0; j < L; ++j) {
-    double2 acc = make_double2(0.0, 0.0);
+    cx<S> acc = mk<S>(0, 0);
 #pragma unroll
-    for (int i = 0; i < L; ++i) cfma(acc, c[j * L + i], v[i]);
+    for (int i = 0; i < L; ++i) cfma(acc, cvs<S>(c[j * L + i]), v[i]);
     w[j] = acc;
   }
 #pragma unroll
   for (int j = 0; j < L; ++j) tile[idx[j]] = w[j];
 }
 
-__device__ void smem_op(double2* tile, const FHdr& h, const double2* c, uint32_t T) {
+template <class S>
+__device__ void smem_op(cx<S>* tile, const FHdr& h, const double2* c, uint32_t T) {
   const uint32_t mlo = h.mlo, plo = h.plo;
   switch (h.type) {
-    case F_X: smem_pairs(tile, FX_{}, h.t0, mlo, plo, T); return;
-    case F_Y: smem_pairs(tile, FY_{}, h.t0, mlo, plo, T); return;
-    case F_H: smem_pairs(tile, FH_{c[0].x}, h.t0, mlo, plo, T); return;
-    case F_UR: smem_pairs(tile, FR_{c[0].x, c[1].x, c[2].x, c[3].x}, h.t0, mlo, plo, T); return;
-    case F_UI: smem_pairs(tile, FI_{c[0].x, c[1].y, c[2].y, c[3].x}, h.t0, mlo, plo, T); return;
-    case F_U2: smem_pairs(tile, FU_{c[0], c[1], c[2], c[3]}, h.t0, mlo, plo, T); return;
+    case F_X: smem_pairs<S>(tile, FX_<S>{}, h.t0, mlo, plo, T); return;
+    case F_Y: smem_pairs<S>(tile, FY_<S>{}, h.t0, mlo, plo, T); return;
+    case F_H: smem_pairs<S>(tile, FH_<S>{(S)c[0].x}, h.t0, mlo, plo, T); return;
+    case F_UR:
+      smem_pairs<S>(tile, FR_<S>{(S)c[0].x, (S)c[1].x, (S)c[2].x, (S)c[3].x}, h.t0, mlo, plo, T);
+      return;
+    case F_UI:
+      smem_pairs<S>(tile, FI_<S>{(S)c[0].x, (S)c[1].y, (S)c[2].y, (S)c[3].x}, h.t0, mlo, plo, T);
+      return;
+    case F_U2:
+      smem_pairs<S>(tile, FU_<S>{cvs<S>(c[0]), cvs<S>(c[1]), cvs<S>(c[2]), cvs<S>(c[3])}, h.t0, mlo,
+                    plo, T);
+      return;
     case F_SWAP: {
       const int lo = h.t0 < h.t1 ? h.t0 : h.t1, hi = h.t0 < h.t1 ? h.t1 : h.t0;
       for (uint32_t p = threadIdx.x; p < (T >> 2); p += kFThreads) {
         const uint32_t i = ins0(ins0(p, lo), hi);
         if ((i & mlo) != plo) continue;
         const uint32_t x = i | (1u << lo), y = i | (1u << hi);
-        const double2 vx = tile[x];
+        const cx<S> vx = tile[x];
         tile[x] = tile[y];
         tile[y] = vx;
       }
@@ -227,7 +242,7 @@ __device__ void smem_op(double2* tile, const FHdr& h, const double2* c, uint32_t
         const uint32_t i = ins0(ins0(p, lo), hi);
         if ((i & mlo) != plo) continue;
         const uint32_t idx[4] = {i, i | (1u << t1), i | (1u << t0), i | (1u << t0) | (1u << t1)};
-        dense_group<4>(tile, idx, c);
+        dense_group<S, 4>(tile, idx, c);
       }
       return;
     }
@@ -243,7 +258,7 @@ __device__ void smem_op(double2* tile, const FHdr& h, const double2* c, uint32_t
 #pragma unroll
         for (int j = 0; j < 8; ++j)
           idx[j] = i | (((j >> 2) & 1u) << s0) | (((j >> 1) & 1u) << s1) | ((j & 1u) << s2);
-        dense_group<8>(tile, idx, c);
+        dense_group<S, 8>(tile, idx, c);
       }
       return;
     }
@@ -251,8 +266,8 @@ __device__ void smem_op(double2* tile, const FHdr& h, const double2* c, uint32_t
 }
 
 // ---- register path ---------------------------------------------------------------
-template <int RB, int R, class F>
-__device__ __forceinline__ void reg_pairs(double2 (&v)[R], const F& f, uint32_t mlo, uint32_t plo,
+template <int RB, int R, class C, class F>
+__device__ __forceinline__ void reg_pairs(C (&v)[R], const F& f, uint32_t mlo, uint32_t plo,
                                           uint32_t tid) {
   if constexpr ((1 << RB) < R) {
     // Predicate split: thread bits once, register bits per r (uniform across the block).
@@ -268,9 +283,9 @@ __device__ __forceinline__ void reg_pairs(double2 (&v)[R], const F& f, uint32_t 
   }
 }
 
-template <int R, class F>
-__device__ __forceinline__ void reg_1q(double2 (&v)[R], const F& f, int t0, uint32_t mlo,
-                                       uint32_t plo, uint32_t tid) {
+template <int R, class C, class F>
+__device__ __forceinline__ void reg_1q(C (&v)[R], const F& f, int t0, uint32_t mlo, uint32_t plo,
+                                       uint32_t tid) {
   if (t0 >= 8) {
     switch (t0 - 8) {
       case 0: reg_pairs<0, R>(v, f, mlo, plo, tid); break;
@@ -288,21 +303,13 @@ __device__ __forceinline__ void reg_1q(double2 (&v)[R], const F& f, int t0, uint
 #pragma unroll
   for (int r = 0; r < R; ++r) {
     if (((uint32_t)r & mr) != pr) continue;
-    double2 p;
+    C p;
     p.x = __shfl_xor_sync(0xffffffffu, v[r].x, 1 << t0);
     p.y = __shfl_xor_sync(0xffffffffu, v[r].y, 1 << t0);
     if (bt) v[r] = f.lane(v[r], p, bit);
   }
 }
 
-__device__ __forceinline__ double2 ldcs(const double2* p) {
-  double2 v;
-  asm volatile("ld.global.cs.v2.f64 {%0,%1}, [%2];" : "=d"(v.x), "=d"(v.y) : "l"(p));
-  return v;
-}
-__device__ __forceinline__ void stcs(double2* p, double2 v) {
-  asm volatile("st.global.cs.v2.f64 [%0], {%1,%2};" ::"l"(p), "d"(v.x), "d"(v.y) : "memory");
-}
 // Global amplitude index of tile element i (chunk = i >> lc, offset = low lc bits).
 __device__ __forceinline__ uint64_t tile_addr(const FTile& tg, uint64_t base, uint32_t i) {
   uint64_t off = base | (i & ((1u << tg.lc) - 1));
@@ -311,12 +318,14 @@ __device__ __forceinline__ uint64_t tile_addr(const FTile& tg, uint64_t base, ui
   return off;
 }
 
-template <int K, bool DIRECT>
-__global__ void __launch_bounds__(kFThreads, 2) k_fused(double2* __restrict__ a,
+template <int K, bool DIRECT, class S>
+__global__ void __launch_bounds__(kFThreads, 2) k_fused(cx<S>* __restrict__ a,
                                                         const __grid_constant__ FProg prog) {
+  using C = cx<S>;
   constexpr uint32_t T = 1u << K;
   constexpr int R = T / kFThreads;  // amplitudes per thread
-  extern __shared__ __align__(128) double2 tile[];
+  extern __shared__ __align__(128) unsigned char smem_raw[];
+  C* tile = reinterpret_cast<C*>(smem_raw);
   __shared__ __align__(8) uint64_t bar;
   const uint32_t tid = threadIdx.x;
   const FTile& tg = prog.tile;
@@ -328,19 +337,19 @@ __global__ void __launch_bounds__(kFThreads, 2) k_fused(double2* __restrict__ a,
     const uint64_t lo = base & ((1ull << p) - 1);
     base = ((base - lo) << 1) | lo;
   }
-  const uint32_t bytes = T * 16u, chunk_bytes = 16u << lc;
+  const uint32_t bytes = T * (uint32_t)sizeof(C), chunk_bytes = (uint32_t)sizeof(C) << lc;
   const uint32_t bar_a = smem_u32(&bar), tile_a = smem_u32(tile);
-  double2 v[R];
+  C v[R];
   if (DIRECT) {
-    // Many small chunks: a TMA bulk copy costs ~50 SM cycles regardless of size,
-    // so load straight into registers instead (each warp reads 32 consecutive
-    // amplitudes of one chunk per instruction: 512 B, coalesced).
+    // Direct register loads (each warp reads 32 consecutive amplitudes of one
+    // chunk per instruction, coalesced).
 #pragma unroll
-    for (int r = 0; r < R; ++r) v[r] = ldcs(a + tile_addr(tg, base, (uint32_t)r * kFThreads + tid));
+    for (int r = 0; r < R; ++r) v[r] = ld1(a + tile_addr(tg, base, (uint32_t)r * kFThreads + tid));
   } else {
     if (tid < 32) {
       // Lane 0 arms the barrier with the whole tile; the 32 lanes of warp 0 then
-      // issue the chunk copies in parallel.
+      // issue the chunk copies in parallel (a bulk copy costs ~50 SM cycles of
+      // TMA service time whatever its size).
       if (tid == 0) {
         asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(bar_a));
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
@@ -398,13 +407,13 @@ __global__ void __launch_bounds__(kFThreads, 2) k_fused(double2* __restrict__ a,
       __syncthreads();
     }
     if (!regpath) {
-      smem_op(tile, h, c, T);
+      smem_op<S>(tile, h, c, T);
       continue;
     }
     switch (type) {
       case F_DIAG1: {  // one diagonal entry d != 1 on the amplitudes matching the predicate
-        // Split the predicate: register bits (warp-uniform -> branch) and thread bits.
-        const double2 d = c[0];
+        // Split the predicate: register bits (uniform -> branch) and thread bits.
+        const C d = cvs<S>(c[0]);
         const uint32_t mr = mlo >> 8, pr = plo >> 8;
         const bool bt = (tid & mlo & (kFThreads - 1)) == (plo & (kFThreads - 1));
         if (!__any_sync(0xffffffffu, bt)) break;  // whole warp inactive (warp-bit predicate)
@@ -418,9 +427,9 @@ __global__ void __launch_bounds__(kFThreads, 2) k_fused(double2* __restrict__ a,
       case F_DIAGN: {  // factor d[j], j from the target bits (>= 64: outside the tile)
         const int m = h.m;
         if (m == 1) {  // Rz-like: two entries selected by one bit
-          const double2 d0 = c[0], d1 = c[1];
+          const C d0 = cvs<S>(c[0]), d1 = cvs<S>(c[1]);
           if (t0 >= 64) {
-            const double2 d = ((base >> (t0 - 64)) & 1) ? d1 : d0;
+            const C d = ((base >> (t0 - 64)) & 1) ? d1 : d0;
 #pragma unroll
             for (int r = 0; r < R; ++r) {
               const uint32_t i = (uint32_t)r * kFThreads + tid;
@@ -445,9 +454,9 @@ __global__ void __launch_bounds__(kFThreads, 2) k_fused(double2* __restrict__ a,
             else
               jmask |= 1u << (m - 1 - s);
           }
-        double2 dd[8];
+        C dd[8];
 #pragma unroll
-        for (int j = 0; j < 8; ++j) dd[j] = j < (1 << m) ? c[j] : make_double2(1.0, 0.0);
+        for (int j = 0; j < 8; ++j) dd[j] = j < (1 << m) ? cvs<S>(c[j]) : mk<S>(1, 0);
 #pragma unroll
         for (int r = 0; r < R; ++r) {
           const uint32_t i = (uint32_t)r * kFThreads + tid;
@@ -456,7 +465,7 @@ __global__ void __launch_bounds__(kFThreads, 2) k_fused(double2* __restrict__ a,
 #pragma unroll
           for (int s = 0; s < 3; ++s)
             if (s < m && (jmask >> (m - 1 - s) & 1)) j |= ((i >> ts[s]) & 1u) << (m - 1 - s);
-          double2 d = dd[0];
+          C d = dd[0];
 #pragma unroll
           for (int q = 1; q < 8; ++q)
             if ((uint32_t)q == j) d = dd[q];
@@ -464,12 +473,19 @@ __global__ void __launch_bounds__(kFThreads, 2) k_fused(double2* __restrict__ a,
         }
         break;
       }
-      case F_X: reg_1q<R>(v, FX_{}, t0, mlo, plo, tid); break;
-      case F_Y: reg_1q<R>(v, FY_{}, t0, mlo, plo, tid); break;
-      case F_H: reg_1q<R>(v, FH_{c[0].x}, t0, mlo, plo, tid); break;
-      case F_UR: reg_1q<R>(v, FR_{c[0].x, c[1].x, c[2].x, c[3].x}, t0, mlo, plo, tid); break;
-      case F_UI: reg_1q<R>(v, FI_{c[0].x, c[1].y, c[2].y, c[3].x}, t0, mlo, plo, tid); break;
-      default: reg_1q<R>(v, FU_{c[0], c[1], c[2], c[3]}, t0, mlo, plo, tid); break;
+      case F_X: reg_1q<R>(v, FX_<S>{}, t0, mlo, plo, tid); break;
+      case F_Y: reg_1q<R>(v, FY_<S>{}, t0, mlo, plo, tid); break;
+      case F_H: reg_1q<R>(v, FH_<S>{(S)c[0].x}, t0, mlo, plo, tid); break;
+      case F_UR:
+        reg_1q<R>(v, FR_<S>{(S)c[0].x, (S)c[1].x, (S)c[2].x, (S)c[3].x}, t0, mlo, plo, tid);
+        break;
+      case F_UI:
+        reg_1q<R>(v, FI_<S>{(S)c[0].x, (S)c[1].y, (S)c[2].y, (S)c[3].x}, t0, mlo, plo, tid);
+        break;
+      default:
+        reg_1q<R>(v, FU_<S>{cvs<S>(c[0]), cvs<S>(c[1]), cvs<S>(c[2]), cvs<S>(c[3])}, t0, mlo, plo,
+                  tid);
+        break;
     }
   }
 
@@ -480,7 +496,7 @@ __global__ void __launch_bounds__(kFThreads, 2) k_fused(double2* __restrict__ a,
       for (int r = 0; r < R; ++r) v[r] = tile[r * kFThreads + tid];
     }
 #pragma unroll
-    for (int r = 0; r < R; ++r) stcs(a + tile_addr(tg, base, (uint32_t)r * kFThreads + tid), v[r]);
+    for (int r = 0; r < R; ++r) st1(a + tile_addr(tg, base, (uint32_t)r * kFThreads + tid), v[r]);
     return;
   }
   if (in_regs) {
@@ -599,35 +615,31 @@ void encode(const Decoded& g, const TileMap& tm, FProg& P) {
   ++P.nops;
 }
 
-template <int K, bool DIRECT>
+template <int K, bool DIRECT, class S>
 void launch_kd(const LaunchCtx& ctx, const FProg& P) {
-  const size_t smem = size_t(16) << K;
-  ensure_smem_attr((const void*)k_fused<K, DIRECT>, (int)smem);
+  const size_t smem = sizeof(cx<S>) << K;
+  ensure_smem_attr((const void*)k_fused<K, DIRECT, S>, (int)smem);
   const uint64_t tiles = 1ull << (ctx.n_local - K);
-  k_fused<K, DIRECT><<<(unsigned)tiles, kFThreads, smem, ctx.stream>>>(
-      reinterpret_cast<double2*>(ctx.amps), P);
+  k_fused<K, DIRECT, S><<<(unsigned)tiles, kFThreads, smem, ctx.stream>>>(
+      reinterpret_cast<cx<S>*>(ctx.amps), P);
 }
-// TMA bulk copies for tiles of few large chunks; direct register loads for many
-// small chunks (the TMA unit's per-copy cost dominates below ~16 KiB chunks).
+// TMA bulk copies for tiles of at most fuse_tma_max_chunks chunks (default: all),
+// direct register loads otherwise.
 template <int K>
 void launch_k(const LaunchCtx& ctx, const FProg& P) {
-  if ((1 << P.tile.nh) > ctx.opt->fuse_tma_max_chunks)
-    launch_kd<K, true>(ctx, P);
-  else
-    launch_kd<K, false>(ctx, P);
+  const bool direct = (1 << P.tile.nh) > ctx.opt->fuse_tma_max_chunks;
+  if (ctx.c64) {
+    if (direct)
+      launch_kd<K, true, float>(ctx, P);
+    else
+      launch_kd<K, false, float>(ctx, P);
+  } else {
+    if (direct)
+      launch_kd<K, true, double>(ctx, P);
+    else
+      launch_kd<K, false, double>(ctx, P);
+  }
 }
-
-}  // namespace
-
-bool fusable(const Decoded& g, int K, int n_local) {
-  (void)n_local;
-  if (g.cls == GClass::NOOP || g.cls == GClass::DIAG) return true;
-  for (int s = 0; s < g.m; ++s)
-    if (g.targets[s] >= K) return false;
-  return true;
-}
-
-namespace {
 
 struct TileCfg {
   int K, L, slots;
@@ -699,15 +711,15 @@ void launch_program(const LaunchCtx& ctx, const TileCfg& cfg, uint64_t in_tile,
       Decoded& a = prog.back();
       if (a.m == 1 && g.m == 1 && a.targets[0] == g.targets[0] && a.cmask == g.cmask &&
           (a.cls == GClass::DENSE || g.cls == GClass::DENSE)) {
-        cplx C[4];
+        cplx Cm[4];
         for (int r = 0; r < 2; ++r)
           for (int c = 0; c < 2; ++c) {
             const cplx x = g.M[r * 2 + 0], y = a.M[0 * 2 + c], u = g.M[r * 2 + 1],
                        w = a.M[1 * 2 + c];
-            C[r * 2 + c] = cplx{x.re * y.re - x.im * y.im + (u.re * w.re - u.im * w.im),
-                                x.re * y.im + x.im * y.re + (u.re * w.im + u.im * w.re)};
+            Cm[r * 2 + c] = cplx{x.re * y.re - x.im * y.im + (u.re * w.re - u.im * w.im),
+                                 x.re * y.im + x.im * y.re + (u.re * w.im + u.im * w.re)};
           }
-        for (int k = 0; k < 4; ++k) a.M[k] = C[k];
+        for (int k = 0; k < 4; ++k) a.M[k] = Cm[k];
         a.cls = GClass::DENSE;
         a.is_h = false;
         a.kind = LFQS_UNITARY1;

@@ -94,11 +94,12 @@ struct Options {
 
 // One launch worth of work on a contiguous shard.
 struct LaunchCtx {
-  double* amps;            // interleaved complex128 shard
+  void* amps;              // interleaved shard: complex128 (double2) or complex64 (float2)
   int n_local;             // qubits in the shard
   cudaStream_t stream;
   uint64_t* launch_counter;
   const Options* opt;
+  bool c64;                // amplitudes are complex64 (NEXT-4 precision variant)
 };
 
 // Raises a kernel's dynamic shared memory limit once per device.

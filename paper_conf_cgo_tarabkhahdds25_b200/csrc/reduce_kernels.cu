@@ -1,14 +1,14 @@
-// reduce_kernels.cu -- norm / marginal-probability reduction and state initialisers.
+// reduce_kernels.cu -- norm / marginal-probability reduction, collapse and state initialisers.
 //
 // Measurement at the end of a circuit: P(Q = v) = sum_{k: bits_Q(k) = v} |a_k|^2.
 // B200 design: one read-only streaming pass.  Each
-// warp reads 32 contiguous amplitudes per instruction (16 B per lane, evict-
-// first), folds |a|^2 across the lane bits that are NOT measured with xor-
-// shuffles, and the lanes that represent a distinct low-bit outcome add into a
-// per-warp shared-memory histogram (no atomics: each bin has exactly one
-// writer lane).  Warps are then summed in fixed order per block, and blocks in
-// fixed order by a second tiny kernel: the result is deterministic for a given
-// shard size, independent of scheduling.
+// warp reads 32 contiguous amplitudes per instruction (evict-first), folds
+// |a|^2 across the lane bits that are NOT measured with xor-shuffles, and the
+// lanes that represent a distinct low-bit outcome add into a per-warp shared-
+// memory histogram (no atomics: each bin has exactly one writer lane).  Warps
+// are then summed in fixed order per block, and blocks in fixed order by a
+// second tiny kernel: the result is deterministic for a given shard size.
+// Probabilities are accumulated in double for both amplitude precisions.
 #include <cuda_runtime.h>
 
 #include <cstring>
@@ -16,6 +16,7 @@
 #include <set>
 #include <utility>
 
+#include "cx.cuh"
 #include "lfqs_internal.h"
 
 namespace lfqs {
@@ -30,15 +31,9 @@ constexpr int kMaxQ = 10;
 struct QList {
   int nq;
   int q[kMaxQ];
-  uint32_t lane_free;  // lane bits (0..4) not measured: folded by shuffles
+  uint32_t lane_free;    // lane bits (0..4) not measured: folded by shuffles
   uint64_t fmask, fpat;  // only amplitudes with (k & fmask) == fpat contribute
 };
-
-__device__ __forceinline__ double2 ldcs(const double2* p) {
-  double2 v;
-  asm volatile("ld.global.cs.v2.f64 {%0,%1}, [%2];" : "=d"(v.x), "=d"(v.y) : "l"(p));
-  return v;
-}
 
 __device__ __forceinline__ int bin_of(const QList& ql, uint64_t k) {
   int v = 0;
@@ -48,7 +43,14 @@ __device__ __forceinline__ int bin_of(const QList& ql, uint64_t k) {
   return v;
 }
 
-__global__ void __launch_bounds__(kThreads) k_probs(const double2* __restrict__ a, uint64_t n_rows,
+template <class S>
+__device__ __forceinline__ double norm2(cx<S> x) {
+  const double re = (double)x.x, im = (double)x.y;
+  return re * re + im * im;
+}
+
+template <class S>
+__global__ void __launch_bounds__(kThreads) k_probs(const cx<S>* __restrict__ a, uint64_t n_rows,
                                                     const QList ql, double* __restrict__ partials) {
   extern __shared__ double hist[];  // [kWarps][nbins]
   const int nbins = 1 << ql.nq;
@@ -65,8 +67,8 @@ __global__ void __launch_bounds__(kThreads) k_probs(const double2* __restrict__ 
     for (int u = 0; u < kU; ++u) {
       const uint64_t r = r0 + u;
       if (r < n_rows) {
-        const double2 x = ldcs(a + r * 32 + lane);
-        p[u] = ((r * 32 + lane) & ql.fmask) == ql.fpat ? x.x * x.x + x.y * x.y : 0.0;
+        const cx<S> x = ld1(a + r * 32 + lane);
+        p[u] = ((r * 32 + lane) & ql.fmask) == ql.fpat ? norm2<S>(x) : 0.0;
       } else {
         p[u] = 0.0;
       }
@@ -97,34 +99,35 @@ __global__ void k_probs_final(const double* __restrict__ partials, int nblocks, 
 }
 
 // Small-state path (< 32 amplitudes): one thread, ascending order.
-__global__ void k_probs_tiny(const double2* __restrict__ a, uint64_t n_amps, const QList ql,
+template <class S>
+__global__ void k_probs_tiny(const cx<S>* __restrict__ a, uint64_t n_amps, const QList ql,
                              double* __restrict__ out) {
   const int nbins = 1 << ql.nq;
   for (int b = 0; b < nbins; ++b) out[b] = 0.0;
   for (uint64_t k = 0; k < n_amps; ++k)
-    if ((k & ql.fmask) == ql.fpat) out[bin_of(ql, k)] += a[k].x * a[k].x + a[k].y * a[k].y;
+    if ((k & ql.fmask) == ql.fpat) out[bin_of(ql, k)] += norm2<S>(a[k]);
 }
 
-// --- projective collapse (one streaming pass, 32-byte accesses) --------------
-__global__ void __launch_bounds__(kThreads) k_collapse(double2* __restrict__ a, uint64_t n_pairs,
-                                                       uint64_t mask, uint64_t pat, double scale) {
+// --- projective collapse (one streaming pass, two-amplitude accesses) --------
+template <class S>
+__global__ void __launch_bounds__(kThreads) k_collapse(cx<S>* __restrict__ a, uint64_t n_pairs,
+                                                       uint64_t mask, uint64_t pat, S scale) {
   const uint64_t stride = (uint64_t)gridDim.x * kThreads;
   for (uint64_t i = (uint64_t)blockIdx.x * kThreads + threadIdx.x; i < n_pairs; i += stride) {
     const uint64_t k = 2 * i;
-    double2 x, y;
-    asm volatile("ld.global.cs.v4.f64 {%0,%1,%2,%3}, [%4];"
-                 : "=d"(x.x), "=d"(x.y), "=d"(y.x), "=d"(y.y)
-                 : "l"(a + k));
-    x = ((k & mask) == pat) ? make_double2(scale * x.x, scale * x.y) : make_double2(0.0, 0.0);
-    y = (((k + 1) & mask) == pat) ? make_double2(scale * y.x, scale * y.y) : make_double2(0.0, 0.0);
-    asm volatile("st.global.cs.v4.f64 [%0], {%1,%2,%3,%4};" ::"l"(a + k), "d"(x.x), "d"(x.y),
-                 "d"(y.x), "d"(y.y)
-                 : "memory");
+    cx<S> x, y;
+    ld2(a + k, x, y);
+    x = ((k & mask) == pat) ? mk<S>(scale * x.x, scale * x.y) : mk<S>(0, 0);
+    y = (((k + 1) & mask) == pat) ? mk<S>(scale * y.x, scale * y.y) : mk<S>(0, 0);
+    st2(a + k, x, y);
   }
 }
 
 // --- initialisers -----------------------------------------------------------
-__global__ void k_set_one(double2* a, uint64_t idx) { a[idx] = make_double2(1.0, 0.0); }
+template <class S>
+__global__ void k_set_one(cx<S>* a, uint64_t idx) {
+  a[idx] = mk<S>(1, 0);
+}
 
 __device__ __forceinline__ uint64_t sm64(uint64_t seed, uint64_t i) {  // SplitMix64 output #i
   uint64_t z = seed + (i + 1) * 0x9E3779B97F4A7C15ull;
@@ -133,16 +136,39 @@ __device__ __forceinline__ uint64_t sm64(uint64_t seed, uint64_t i) {  // SplitM
   return z ^ (z >> 31);
 }
 
-__global__ void __launch_bounds__(kThreads) k_init_random(double2* __restrict__ a, uint64_t n_amps,
+template <class S>
+__global__ void __launch_bounds__(kThreads) k_init_random(cx<S>* __restrict__ a, uint64_t n_amps,
                                                           uint64_t seed, uint64_t offset) {
   const uint64_t stride = (uint64_t)gridDim.x * kThreads;
   for (uint64_t k = (uint64_t)blockIdx.x * kThreads + threadIdx.x; k < n_amps; k += stride) {
     const uint64_t gk = offset + k;
     const double re = (double)(sm64(seed, 2 * gk) >> 11) * 0x1.0p-53 * 2.0 - 1.0;
     const double im = (double)(sm64(seed, 2 * gk + 1) >> 11) * 0x1.0p-53 * 2.0 - 1.0;
-    a[k] = make_double2(re, im);
+    a[k] = mk<S>((S)re, (S)im);
   }
 }
+
+template <class S>
+void probs_t(const LaunchCtx& ctx, const QList& ql, double* d_partials, double* d_out) {
+  const uint64_t n_amps = 1ull << ctx.n_local;
+  const auto* a = reinterpret_cast<const cx<S>*>(ctx.amps);
+  if (n_amps < 32) {
+    k_probs_tiny<S><<<1, 1, 0, ctx.stream>>>(a, n_amps, ql, d_out);
+    LFQS_CUDA_CHECK(cudaGetLastError());
+    ++*ctx.launch_counter;
+    return;
+  }
+  const int nbins = 1 << ql.nq;
+  const size_t smem = sizeof(double) * kWarps * nbins;
+  ensure_smem_attr((const void*)k_probs<S>, sizeof(double) * kWarps * (1 << kMaxQ));
+  k_probs<S><<<kBlocks, kThreads, smem, ctx.stream>>>(a, n_amps / 32, ql, d_partials);
+  LFQS_CUDA_CHECK(cudaGetLastError());
+  k_probs_final<<<(nbins + 255) / 256, 256, 0, ctx.stream>>>(d_partials, kBlocks, nbins, d_out);
+  LFQS_CUDA_CHECK(cudaGetLastError());
+  *ctx.launch_counter += 2;
+}
+
+inline size_t amp_bytes(const LaunchCtx& ctx) { return ctx.c64 ? 8 : 16; }
 
 }  // namespace
 
@@ -163,6 +189,7 @@ void ensure_smem_attr(const void* kernel, int bytes) {
 void launch_probs(const LaunchCtx& ctx, const int* qubits, int nq, double* d_partials,
                   int n_partials_blocks, double* d_out, uint64_t fmask, uint64_t fpat) {
   require(nq >= 0 && nq <= kMaxQ, "one probability pass covers at most 10 qubits");
+  require(n_partials_blocks >= kBlocks, "partials buffer too small");
   QList ql;
   std::memset(&ql, 0, sizeof ql);
   ql.nq = nq;
@@ -174,44 +201,41 @@ void launch_probs(const LaunchCtx& ctx, const int* qubits, int nq, double* d_par
     if (qubits[s] < 5) measured_lane_bits |= 1u << qubits[s];
   }
   ql.lane_free = 0x1fu & ~measured_lane_bits;
-  const uint64_t n_amps = 1ull << ctx.n_local;
-  const auto* a = reinterpret_cast<const double2*>(ctx.amps);
-  if (n_amps < 32) {
-    k_probs_tiny<<<1, 1, 0, ctx.stream>>>(a, n_amps, ql, d_out);
-    LFQS_CUDA_CHECK(cudaGetLastError());
-    ++*ctx.launch_counter;
-    return;
-  }
-  require(n_partials_blocks >= kBlocks, "partials buffer too small");
-  const int nbins = 1 << nq;
-  const size_t smem = sizeof(double) * kWarps * nbins;
-  ensure_smem_attr((const void*)k_probs, sizeof(double) * kWarps * (1 << kMaxQ));
-  k_probs<<<kBlocks, kThreads, smem, ctx.stream>>>(a, n_amps / 32, ql, d_partials);
-  LFQS_CUDA_CHECK(cudaGetLastError());
-  k_probs_final<<<(nbins + 255) / 256, 256, 0, ctx.stream>>>(d_partials, kBlocks, nbins, d_out);
-  LFQS_CUDA_CHECK(cudaGetLastError());
-  *ctx.launch_counter += 2;
+  if (ctx.c64)
+    probs_t<float>(ctx, ql, d_partials, d_out);
+  else
+    probs_t<double>(ctx, ql, d_partials, d_out);
 }
 
 void launch_collapse(const LaunchCtx& ctx, uint64_t mask, uint64_t pat, double scale,
                      bool zero_all) {
   const uint64_t n = 1ull << ctx.n_local;
   if (zero_all) {
-    LFQS_CUDA_CHECK(cudaMemsetAsync(ctx.amps, 0, n * 16, ctx.stream));
+    LFQS_CUDA_CHECK(cudaMemsetAsync(ctx.amps, 0, n * amp_bytes(ctx), ctx.stream));
     return;
   }
   uint64_t nb = (n / 2 + kThreads - 1) / kThreads;
   if (nb > 148ull * 64) nb = 148ull * 64;
-  k_collapse<<<(unsigned)nb, kThreads, 0, ctx.stream>>>(reinterpret_cast<double2*>(ctx.amps),
-                                                        n / 2, mask, pat, scale);
+  if (ctx.c64)
+    k_collapse<float><<<(unsigned)nb, kThreads, 0, ctx.stream>>>(
+        reinterpret_cast<float2*>(ctx.amps), n / 2, mask, pat, (float)scale);
+  else
+    k_collapse<double><<<(unsigned)nb, kThreads, 0, ctx.stream>>>(
+        reinterpret_cast<double2*>(ctx.amps), n / 2, mask, pat, scale);
   LFQS_CUDA_CHECK(cudaGetLastError());
   ++*ctx.launch_counter;
 }
 
 void launch_init_basis(const LaunchCtx& ctx, int64_t local_index) {
-  LFQS_CUDA_CHECK(cudaMemsetAsync(ctx.amps, 0, sizeof(double) * 2 * (1ull << ctx.n_local), ctx.stream));
+  LFQS_CUDA_CHECK(
+      cudaMemsetAsync(ctx.amps, 0, amp_bytes(ctx) * (1ull << ctx.n_local), ctx.stream));
   if (local_index >= 0) {
-    k_set_one<<<1, 1, 0, ctx.stream>>>(reinterpret_cast<double2*>(ctx.amps), (uint64_t)local_index);
+    if (ctx.c64)
+      k_set_one<float><<<1, 1, 0, ctx.stream>>>(reinterpret_cast<float2*>(ctx.amps),
+                                                 (uint64_t)local_index);
+    else
+      k_set_one<double><<<1, 1, 0, ctx.stream>>>(reinterpret_cast<double2*>(ctx.amps),
+                                                  (uint64_t)local_index);
     LFQS_CUDA_CHECK(cudaGetLastError());
     ++*ctx.launch_counter;
   }
@@ -221,8 +245,12 @@ void launch_init_random(const LaunchCtx& ctx, uint64_t seed, uint64_t global_off
   const uint64_t n = 1ull << ctx.n_local;
   uint64_t nb = (n + kThreads - 1) / kThreads;
   if (nb > 148ull * 64) nb = 148ull * 64;
-  k_init_random<<<(unsigned)nb, kThreads, 0, ctx.stream>>>(reinterpret_cast<double2*>(ctx.amps), n,
-                                                           seed, global_offset);
+  if (ctx.c64)
+    k_init_random<float><<<(unsigned)nb, kThreads, 0, ctx.stream>>>(
+        reinterpret_cast<float2*>(ctx.amps), n, seed, global_offset);
+  else
+    k_init_random<double><<<(unsigned)nb, kThreads, 0, ctx.stream>>>(
+        reinterpret_cast<double2*>(ctx.amps), n, seed, global_offset);
   LFQS_CUDA_CHECK(cudaGetLastError());
   ++*ctx.launch_counter;
 }

@@ -44,20 +44,22 @@ int log2_exact(int x) {
   return (1 << p) == x ? p : -1;
 }
 
-double* alloc_amps(uint64_t n_amps) {
+unsigned char* alloc_amps(uint64_t n_amps, int ab) {
   void* p = nullptr;
-  cudaError_t e = cudaMalloc(&p, n_amps * 16);
+  cudaError_t e = cudaMalloc(&p, n_amps * ab);
   if (e == cudaErrorMemoryAllocation) {
     cudaGetLastError();
     throw Error(LFQS_ERR_OUT_OF_MEMORY,
-                "cannot allocate " + std::to_string(n_amps * 16) + " bytes of device memory");
+                "cannot allocate " + std::to_string(n_amps * ab) + " bytes of device memory");
   }
   LFQS_CUDA_CHECK(e);
-  return static_cast<double*>(p);
+  return static_cast<unsigned char*>(p);
 }
 }  // namespace
 
-void State::common_init(int n_, int world_, int device_, cudaStream_t s) {
+void State::common_init(int n_, int world_, int device_, cudaStream_t s, bool c64_) {
+  c64 = c64_;
+  ab = c64 ? 8 : 16;
   int ndev = 0;
   if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev == 0) {
     cudaGetLastError();
@@ -83,26 +85,26 @@ void State::common_init(int n_, int world_, int device_, cudaStream_t s) {
   LFQS_CUDA_CHECK(cudaMalloc(&d_probs, sizeof(double) * 1024));
 }
 
-State* State::create_local(int n, int device, cudaStream_t stream, void* borrowed) {
+State* State::create_local(int n, int device, cudaStream_t stream, void* borrowed, bool c64) {
   require(n >= 1 && n <= 36, "n_qubits must be in [1, 36] on one GPU");
   std::unique_ptr<State> st(new State());
-  st->common_init(n, 1, device, stream);
+  st->common_init(n, 1, device, stream, c64);
   if (borrowed) {
-    st->amps = static_cast<double*>(borrowed);
+    st->amps = static_cast<unsigned char*>(borrowed);
   } else {
-    st->amps = alloc_amps(1ull << n);
+    st->amps = alloc_amps(1ull << n, st->ab);
     st->owned = true;
     st->init_basis(0);
   }
   return st.release();
 }
 
-State* State::create_virtual(int n, int world, int device, cudaStream_t stream) {
+State* State::create_virtual(int n, int world, int device, cudaStream_t stream, bool c64) {
   require(world >= 2, "virtual partition needs world >= 2");
   std::unique_ptr<State> st(new State());
   st->virt = true;
-  st->common_init(n, world, device, stream);
-  st->amps = alloc_amps(1ull << n);
+  st->common_init(n, world, device, stream, c64);
+  st->amps = alloc_amps(1ull << n, st->ab);
   st->owned = true;
   st->init_basis(0);
   return st.release();
@@ -116,10 +118,10 @@ State* State::create_dist(int n, int rank, int world, const uint8_t uid[128], in
   std::unique_ptr<State> st(new State());
   st->common_init(n, world, device, stream);
   st->rank = rank;
-  st->amps = alloc_amps(1ull << st->n_local);
+  st->amps = alloc_amps(1ull << st->n_local, st->ab);
   st->owned = true;
   if (world > 1) {
-    const uint64_t half = 16ull << (st->n_local - 1);
+    const uint64_t half = (uint64_t)st->ab << (st->n_local - 1);
     st->comm = new Comm(rank, world, uid, std::min<uint64_t>(256ull << 20, half));
   }
   st->init_basis(0);
@@ -153,11 +155,12 @@ void State::set_stream(cudaStream_t s) {
 
 LaunchCtx State::ctx(int shard) {
   LaunchCtx c;
-  c.amps = amps + 2 * ((uint64_t)shard << n_local);
+  c.amps = amps + ((uint64_t)shard << n_local) * ab;
   c.n_local = n_local;
   c.stream = stream;
   c.launch_counter = &launches;
   c.opt = &opt;
+  c.c64 = c64;
   return c;
 }
 
@@ -185,7 +188,7 @@ void State::synchronize() {
   LFQS_CUDA_CHECK(cudaGetLastError());
 }
 
-void State::copy(uint64_t offset, uint64_t count, double* host, bool to_device) {
+void State::copy_raw(uint64_t offset, uint64_t count, void* host, bool to_device) {
   DeviceGuard dg(device);
   const uint64_t total = 1ull << n;
   require(offset <= total && count <= total - offset, "amplitude range out of bounds");
@@ -194,15 +197,32 @@ void State::copy(uint64_t offset, uint64_t count, double* host, bool to_device) 
   const uint64_t hi = virt ? total : lo + (1ull << n_local);
   const uint64_t a = std::max(offset, lo), b = std::min(offset + count, hi);
   if (a < b) {
-    double* dev = amps + 2 * (a - lo);
-    double* h = host + 2 * (a - offset);
-    const size_t bytes = (b - a) * 16;
+    unsigned char* dev = amps + (a - lo) * ab;
+    unsigned char* h = static_cast<unsigned char*>(host) + (a - offset) * ab;
+    const size_t bytes = (b - a) * ab;
     if (to_device)
       LFQS_CUDA_CHECK(cudaMemcpyAsync(dev, h, bytes, cudaMemcpyHostToDevice, stream));
     else
       LFQS_CUDA_CHECK(cudaMemcpyAsync(h, dev, bytes, cudaMemcpyDeviceToHost, stream));
   }
   LFQS_CUDA_CHECK(cudaStreamSynchronize(stream));
+}
+
+void State::copy(uint64_t offset, uint64_t count, double* host, bool to_device) {
+  if (!c64) {
+    copy_raw(offset, count, host, to_device);
+    return;
+  }
+  // complex64 state, complex128 host buffer: convert on the host.
+  std::vector<float> tmp(2 * count);
+  if (to_device) {
+    for (uint64_t i = 0; i < 2 * count; ++i) tmp[i] = (float)host[i];
+    copy_raw(offset, count, tmp.data(), true);
+  } else {
+    for (uint64_t i = 0; i < 2 * count; ++i) tmp[i] = (float)host[i];  // keep untouched ranges
+    copy_raw(offset, count, tmp.data(), false);
+    for (uint64_t i = 0; i < 2 * count; ++i) host[i] = (double)tmp[i];
+  }
 }
 
 // ---------------------------------------------------------------------------
@@ -225,10 +245,10 @@ void State::exchange_data(int l, int g) {
       for (uint64_t hi = 0; hi < (1ull << (n_local - 1 - l)); ++hi)
         pieces.push_back(Piece{(hi << (l + 1)) | ((uint64_t)(1 - b) << l), 1ull << l});
     }
-    comm->exchange(amps, pieces, rank ^ (1 << j), stream);
+    comm->exchange(amps, ab, pieces, rank ^ (1 << j), stream);
   }
   ++exchanges;
-  exchange_bytes += 16ull << (n_local - 1);
+  exchange_bytes += (uint64_t)ab << (n_local - 1);
 }
 
 // A run of local gates on one shard: fused passes where possible, else one

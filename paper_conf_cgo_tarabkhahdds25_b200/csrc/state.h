@@ -23,7 +23,9 @@ struct Comm;  // NCCL communicator wrapper (comm.cu)
 struct State : lfqs_state {
   int n = 0, n_local = 0, rank = 0, world = 1, p = 0, device = 0;
   bool virt = false;            // `world` shards in one allocation (single GPU)
-  double* amps = nullptr;       // shard 0 (virtual: all shards back to back)
+  unsigned char* amps = nullptr;  // shard 0 (virtual: all shards back to back)
+  bool c64 = false;             // complex64 amplitudes (NEXT-4); default complex128
+  int ab = 16;                  // bytes per amplitude
   bool owned = false;
   cudaStream_t stream = nullptr;
   bool own_stream = false;
@@ -36,8 +38,10 @@ struct State : lfqs_state {
   // exchange statistics (benchmark accounting)
   uint64_t exchanges = 0, exchange_bytes = 0;
 
-  static State* create_local(int n, int device, cudaStream_t stream, void* borrowed);
-  static State* create_virtual(int n, int world, int device, cudaStream_t stream);
+  static State* create_local(int n, int device, cudaStream_t stream, void* borrowed,
+                             bool c64 = false);
+  static State* create_virtual(int n, int world, int device, cudaStream_t stream,
+                               bool c64 = false);
   static State* create_dist(int n, int rank, int world, const uint8_t uid[128], int device,
                             cudaStream_t stream);
   static void nccl_unique_id(uint8_t uid[128]);
@@ -46,7 +50,10 @@ struct State : lfqs_state {
   void set_stream(cudaStream_t s);
   void init_basis(uint64_t index);
   void init_random(uint64_t seed);
+  // Host buffers: interleaved doubles (converted for complex64 states) ...
   void copy(uint64_t offset, uint64_t count, double* host, bool to_device);
+  // ... or raw amplitudes of the state's own type (no conversion).
+  void copy_raw(uint64_t offset, uint64_t count, void* host, bool to_device);
   void apply(const Decoded& g);
   void run(const std::vector<Decoded>& gates, uint32_t flags);
   void measure_probs(const int* qubits, int nq, double* out);
@@ -58,7 +65,7 @@ struct State : lfqs_state {
 
  private:
   State() = default;
-  void common_init(int n_, int world_, int device_, cudaStream_t s);
+  void common_init(int n_, int world_, int device_, cudaStream_t s, bool c64_ = false);
   LaunchCtx ctx(int shard);
   int n_shards() const { return virt ? world : 1; }
   int rank_of_shard(int shard) const { return virt ? shard : rank; }
