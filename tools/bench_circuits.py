@@ -58,6 +58,7 @@ def main():
     ap.add_argument("--tile", type=int, default=0)
     ap.add_argument("--low", type=int, default=0)
     ap.add_argument("--reorder", type=int, default=1)
+    ap.add_argument("--c64", action="store_true", help="complex64 state (NEXT-4)")
     ap.add_argument("--tma", type=int, default=-1, help="max chunks moved by TMA (-1: default)")
     args = ap.parse_args()
     import torch
@@ -83,7 +84,8 @@ def main():
         "xlow": ([W.Gate("X", (0,)), W.Gate("X", (1,))], lambda st: st.init_basis(0), {}),
         "xhigh": ([W.Gate("X", (n - 1,)), W.Gate("X", (n - 5,))], lambda st: st.init_basis(0), {}),
     }
-    with L.State.create(n, 0, stream=s) as st:
+    ab = 8 if args.c64 else 16
+    with L.State.create(n, 0, stream=s, c64=args.c64) as st:
         if args.tile:
             st.set_option(L.OPT_FUSE_TILE_QUBITS, args.tile)
         if args.low:
@@ -113,8 +115,9 @@ def main():
                 t = min(times)
                 rec = {"circuit": name, "mode": mode, "n": n, "gates": len(gates), "passes": passes,
                        "ms": t, "gates_per_s": len(gates) / (t / 1e3),
-                       "conv_GBps": 32.0 * 2 ** n * len(gates) / (t / 1e3) / 1e9,
-                       "pass_GBps": 32.0 * 2 ** n * passes / (t / 1e3) / 1e9}
+                       "conv_GBps": 2.0 * ab * 2 ** n * len(gates) / (t / 1e3) / 1e9,
+                       "pass_GBps": 2.0 * ab * 2 ** n * passes / (t / 1e3) / 1e9,
+                       "dtype": "c64" if args.c64 else "c128"}
                 rec.update(res)
                 print(json.dumps(rec), flush=True)
 

@@ -53,6 +53,7 @@ def main():
     ap.add_argument("--time", action="store_true")
     ap.add_argument("--no-shuffle", action="store_true")
     ap.add_argument("--no-wide", action="store_true")
+    ap.add_argument("--c64", action="store_true", help="complex64 state")
     ap.add_argument("--ipt", type=int, default=0, help="groups per thread for pair gates (0=default)")
     args = ap.parse_args()
     import torch
@@ -60,7 +61,8 @@ def main():
     s = torch.cuda.Stream()
     torch.cuda.set_stream(s)
     gates = parse(args.gates, args.n)
-    with L.State.create(args.n, 0, stream=s) as st:
+    ab = 8 if args.c64 else 16
+    with L.State.create(args.n, 0, stream=s, c64=args.c64) as st:
         st.set_option(L.OPT_LOWQ_SHUFFLE, 0 if args.no_shuffle else 1)
         st.set_option(L.OPT_WIDE256, 0 if args.no_wide else 1)
         st.set_option(L.OPT_ITEMS_PER_THREAD, args.ipt)
@@ -77,9 +79,9 @@ def main():
             torch.cuda.synchronize()
             if args.time:
                 ms = [ev[r].elapsed_time(ev[r + 1]) for r in range(args.reps)]
-                alg = W.algorithmic_bytes(g, args.n)
+                alg = W.algorithmic_bytes(g, args.n) * ab / 16
                 print(f"{g.label():28s} mean {np.mean(ms):8.3f} ms  min {np.min(ms):8.3f} ms  "
-                      f"alg {alg / np.min(ms) / 1e6:8.1f} GB/s  conv {32 * 2 ** args.n / np.min(ms) / 1e6:8.1f} GB/s",
+                      f"alg {alg / np.min(ms) / 1e6:8.1f} GB/s  conv {2 * ab * 2 ** args.n / np.min(ms) / 1e6:8.1f} GB/s",
                       flush=True)
 
 
