@@ -76,22 +76,26 @@ void Planner::swap_local(int a, int b, std::vector<PlanOp>& out) {
 }
 
 void Planner::plan_canonicalize(std::vector<PlanOp>& out) {
-  for (int q = 0; q < n; ++q) {
-    const int P = l2p[q];
-    if (P == q) continue;
-    const bool pl = P < n_local, ql = q < n_local;
-    if (pl && ql) {
-      swap_local(P, q, out);
-    } else if (pl != ql) {
-      exchange(pl ? P : q, pl ? q : P, out);
+  // Phase 1: bring each global home position G its logical qubit G -- one exchange
+  // when that qubit sits at a local position, two (through a local staging position
+  // L) when it sits at another global one.  L is chosen as the home of the qubit that
+  // leaves G, so that qubit lands where phase 2 wants it.
+  for (int G = n - 1; G >= n_local; --G) {
+    const int P = l2p[G];
+    if (P == G) continue;
+    if (P < n_local) {
+      exchange(P, G, out);
     } else {
-      // (P q) = (L P)(L q)(L P) with any local position L.
-      const int L = n_local - 1;
+      const int x = p2l[G];
+      const int L = x < n_local ? x : n_local - 1;
       exchange(L, P, out);
-      exchange(L, q, out);
-      exchange(L, P, out);
+      exchange(L, G, out);
     }
   }
+  // Phase 2: the local positions now hold a permutation of the local qubits; fix it
+  // with local SWAP passes (no communication).
+  for (int q = 0; q < n_local; ++q)
+    if (l2p[q] != q) swap_local(l2p[q], q, out);
 }
 
 void Planner::plan_circuit(const std::vector<Decoded>& gates, std::vector<PlanOp>& out) {

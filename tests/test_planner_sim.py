@@ -1,0 +1,87 @@
+"""Property test of the distributed planner (lfqs_plan_circuit, host-only C++) without
+processes: every rank's plan is executed in lockstep in one process -- LOCAL ops with
+the oracle on that rank's shard, EXCHANGE ops as the half-shard swap between rank
+pairs -- and the gathered state must equal the oracle applied to the whole state.
+Covers global controls, diagonal folding on global qubits, Belady remaps, SWAP
+relabels and canonicalisation for many seeded circuits."""
+import numpy as np
+import pytest
+
+import oracle as O
+import paper_conf_cgo_tarabkhahdds25_b200 as L
+import workloads as W
+
+
+@pytest.fixture(scope="module", autouse=True)
+def _lib():
+    from paper_conf_cgo_tarabkhahdds25_b200 import build as B
+    B.build()
+    L.lib()
+
+
+def simulate(n, world, gates, psi):
+    p = world.bit_length() - 1
+    nl = n - p
+    plans = [L.lfqs_plan_circuit(n, world, r, gates, canonicalize=True) for r in range(world)]
+    # split every plan at its EXCHANGE ops; all ranks must agree on them
+    segs = []
+    for ops in plans:
+        cur, parts, exch = [], [], []
+        for op in ops:
+            if op[0] == "exchange":
+                parts.append(cur)
+                exch.append(op[1:])
+                cur = []
+            else:
+                cur.append(op[1])
+        parts.append(cur)
+        segs.append((parts, exch))
+    ex0 = segs[0][1]
+    assert all(s[1] == ex0 for s in segs), "ranks disagree on the exchange sequence"
+    shards = [psi[r << nl:(r + 1) << nl].copy() for r in range(world)]
+    k = np.arange(1 << nl)
+    for si in range(len(ex0) + 1):
+        for r in range(world):
+            for g in segs[r][0][si]:
+                O.apply_gate(nl, g, shards[r])
+        if si == len(ex0):
+            break
+        l, gpos = ex0[si]
+        j = gpos - nl
+        for r in range(world):
+            if r >> j & 1:
+                continue
+            r2 = r | (1 << j)
+            ia = np.flatnonzero(((k >> l) & 1) == 1)  # rank r (bit 0) sends l = 1
+            ib = np.flatnonzero(((k >> l) & 1) == 0)  # rank r2 (bit 1) sends l = 0
+            tmp = shards[r][ia].copy()
+            shards[r][ia] = shards[r2][ib]
+            shards[r2][ib] = tmp
+    return np.concatenate(shards), len(ex0)
+
+
+@pytest.mark.parametrize("world", [2, 4, 8])
+@pytest.mark.parametrize("seed", range(6))
+def test_planner_matches_oracle(world, seed):
+    n = 9
+    psi = W.random_state(n, seed)
+    gates = W.random_gate_list(n, 80, seed=1000 * world + seed, max_controls=3)
+    if seed % 2:
+        gates += W.qft(n) + W.ghz(n)
+    got, _ = simulate(n, world, gates, psi)
+    ref = O.run_circuit(n, gates, psi.copy())
+    assert np.max(np.abs(got - ref)) <= 1e-12
+    exact = [g for g in gates if g.exact]
+    got, _ = simulate(n, world, exact, psi)
+    assert np.array_equal(got, O.run_circuit(n, exact, psi.copy()))
+
+
+def test_qft_needs_few_exchanges():
+    """Every QFT CPhase is communication-free (rank-folded diagonal); exchanges come
+    only from the H gates on global qubits, the final SWAPs (relabels) and
+    canonicalisation: p + 1 for the H gates (Belady lookahead), p to restore the map."""
+    n = 10
+    for world in (2, 4, 8):
+        p = world.bit_length() - 1
+        _, n_ex = simulate(n, world, W.qft(n), W.basis_state(n, 77))
+        assert n_ex <= 2 * p + 1, (world, n_ex)
