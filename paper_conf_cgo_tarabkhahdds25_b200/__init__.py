@@ -17,7 +17,8 @@ from typing import Iterable, Optional, Sequence
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "liblfqs.so")
+# LFQS_LIBRARY: load another build of the same library (A/B timing in tools/).
+LIB_PATH = os.environ.get("LFQS_LIBRARY") or os.path.join(_HERE, "liblfqs.so")
 
 KINDS = ["I", "X", "Y", "Z", "H", "S", "SDG", "T", "TDG", "RX", "RY", "RZ", "PHASE", "U3",
          "SWAP", "UNITARY1", "UNITARY2", "UNITARY3"]

@@ -300,6 +300,16 @@ __device__ __forceinline__ void reg_1q(C (&v)[R], const F& f, int t0, uint32_t m
   const int bit = (tid >> t0) & 1;
   const bool bt = (tid & mlo & (kFThreads - 1)) == (plo & (kFThreads - 1));
   const uint32_t mr = mlo >> 8, pr = plo >> 8;
+  if (mlo == 0) {  // uncontrolled: every lane, every register
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+      C p;
+      p.x = __shfl_xor_sync(0xffffffffu, v[r].x, 1 << t0);
+      p.y = __shfl_xor_sync(0xffffffffu, v[r].y, 1 << t0);
+      v[r] = f.lane(v[r], p, bit);
+    }
+    return;
+  }
 #pragma unroll
   for (int r = 0; r < R; ++r) {
     if (((uint32_t)r & mr) != pr) continue;
@@ -308,6 +318,39 @@ __device__ __forceinline__ void reg_1q(C (&v)[R], const F& f, int t0, uint32_t m
     p.y = __shfl_xor_sync(0xffffffffu, v[r].y, 1 << t0);
     if (bt) v[r] = f.lane(v[r], p, bit);
   }
+}
+
+// F_DIAG1 on the registers r with (r & MR) == PR (MR, PR: register bits 8..11 of
+// the predicate).  One instantiation per pattern with at most two register bits
+// (all QFT / CPhase / CZ / T shapes); more bits take the generic loop.
+template <int MR, int PR, int R, class C>
+__device__ __forceinline__ void diag1_regs(C (&v)[R], const C d) {
+#pragma unroll
+  for (int r = 0; r < R; ++r)
+    if ((r & MR) == PR) v[r] = cmul_rn(d, v[r]);
+}
+
+template <int R, class C>
+__device__ __forceinline__ void diag1_dispatch(C (&v)[R], const C d, uint32_t code) {
+#define LFQS_D1(MR, PR) \
+  case ((MR) << 4) | (PR): diag1_regs<MR, PR, R>(v, d); return;
+  switch (code) {
+    LFQS_D1(0, 0)
+    LFQS_D1(1, 0) LFQS_D1(1, 1) LFQS_D1(2, 0) LFQS_D1(2, 2)
+    LFQS_D1(4, 0) LFQS_D1(4, 4) LFQS_D1(8, 0) LFQS_D1(8, 8)
+    LFQS_D1(3, 0) LFQS_D1(3, 1) LFQS_D1(3, 2) LFQS_D1(3, 3)
+    LFQS_D1(5, 0) LFQS_D1(5, 1) LFQS_D1(5, 4) LFQS_D1(5, 5)
+    LFQS_D1(6, 0) LFQS_D1(6, 2) LFQS_D1(6, 4) LFQS_D1(6, 6)
+    LFQS_D1(9, 0) LFQS_D1(9, 1) LFQS_D1(9, 8) LFQS_D1(9, 9)
+    LFQS_D1(10, 0) LFQS_D1(10, 2) LFQS_D1(10, 8) LFQS_D1(10, 10)
+    LFQS_D1(12, 0) LFQS_D1(12, 4) LFQS_D1(12, 8) LFQS_D1(12, 12)
+    default: break;
+  }
+#undef LFQS_D1
+  const uint32_t mr = code >> 4, pr = code & 15;
+#pragma unroll
+  for (int r = 0; r < R; ++r)
+    if (((uint32_t)r & mr) == pr) v[r] = cmul_rn(d, v[r]);
 }
 
 // Global amplitude index of tile element i (chunk = i >> lc, offset = low lc bits).
@@ -340,6 +383,7 @@ __global__ void __launch_bounds__(kFThreads, 2) k_fused(cx<S>* __restrict__ a,
   const uint32_t bytes = T * (uint32_t)sizeof(C), chunk_bytes = (uint32_t)sizeof(C) << lc;
   const uint32_t bar_a = smem_u32(&bar), tile_a = smem_u32(tile);
   C v[R];
+  const int nops = prog.nops;
   if (DIRECT) {
     // Direct register loads (each warp reads 32 consecutive amplitudes of one
     // chunk per instruction, coalesced).
@@ -384,13 +428,26 @@ __global__ void __launch_bounds__(kFThreads, 2) k_fused(cx<S>* __restrict__ a,
   }
   bool in_regs = true;  // else the authoritative copy is the smem tile
 
-  const int nops = prog.nops;
   for (int o = 0; o < nops; ++o) {
     const FHdr& h = prog.h[o];
     if ((base & h.mhi) != h.phi) continue;  // tile-level predicate (uniform)
     const int type = h.type;
-    const int t0 = h.t0;
     const uint32_t mlo = h.mlo, plo = h.plo;
+    if (type == F_DIAG1) {  // one diagonal entry d != 1 (the dominant op of phase-heavy programs)
+      if (!in_regs) {
+        __syncthreads();
+#pragma unroll
+        for (int r = 0; r < R; ++r) v[r] = tile[r * kFThreads + tid];
+        in_regs = true;
+      }
+      // Split the predicate: thread bits (lanes that fail skip) and register
+      // bits, dispatched to a compile-time register set so that no DP
+      // instruction is issued for a register the predicate excludes.
+      if ((tid & mlo & (kFThreads - 1)) == (plo & (kFThreads - 1)))
+        diag1_dispatch<R>(v, cvs<S>(prog.c[h.coef]), ((mlo >> 8) << 4) | (plo >> 8));
+      continue;
+    }
+    const int t0 = h.t0;
     const double2* c = prog.c + h.coef;
     const bool regpath = type <= F_DIAGN || (type <= F_U2 && (t0 < 5 || t0 >= 8));
     if (regpath && !in_regs) {
@@ -411,19 +468,6 @@ __global__ void __launch_bounds__(kFThreads, 2) k_fused(cx<S>* __restrict__ a,
       continue;
     }
     switch (type) {
-      case F_DIAG1: {  // one diagonal entry d != 1 on the amplitudes matching the predicate
-        // Split the predicate: register bits (uniform -> branch) and thread bits.
-        const C d = cvs<S>(c[0]);
-        const uint32_t mr = mlo >> 8, pr = plo >> 8;
-        const bool bt = (tid & mlo & (kFThreads - 1)) == (plo & (kFThreads - 1));
-        if (!__any_sync(0xffffffffu, bt)) break;  // whole warp inactive (warp-bit predicate)
-#pragma unroll
-        for (int r = 0; r < R; ++r) {
-          if (((uint32_t)r & mr) != pr) continue;  // uniform across the block
-          if (bt) v[r] = cmul_rn(d, v[r]);
-        }
-        break;
-      }
       case F_DIAGN: {  // factor d[j], j from the target bits (>= 64: outside the tile)
         const int m = h.m;
         if (m == 1) {  // Rz-like: two entries selected by one bit
