@@ -167,6 +167,24 @@ lfqs_status lfqs_apply_gate(lfqs_state* s, int kind, const int* targets, int n_t
  * results agree within rounding (<= 1e-12 abs per amplitude). */
 lfqs_status lfqs_run_circuit(lfqs_state* s, const lfqs_gate* gates, size_t n_gates, uint32_t flags);
 
+/* ---- captured circuits (CUDA graphs) ----------------------------------------- */
+/* The circuit runner of Eq. 3 replayed without host work: the
+ * launches lfqs_run_circuit(s, gates, n_gates, flags) would issue are captured
+ * once into a CUDA graph; each lfqs_circuit_launch applies the whole circuit
+ * again (same kernels, same arguments, so bit-identical to lfqs_run_circuit)
+ * on the state's current stream, asynchronously.  For launch-bound sizes
+ * (n <= ~20) this removes the per-gate host and launch cost.
+ *   - compile issues no GPU work (the state is unchanged); a virtual partition
+ *     is canonicalised first and the graph ends canonical, so replays compose;
+ *   - distributed (NCCL) states: LFQS_ERR_UNSUPPORTED;
+ *   - the circuit borrows the state: destroy it before lfqs_state_destroy;
+ *   - *kernels_out (may be NULL) = kernels one launch replays. */
+typedef struct lfqs_circuit lfqs_circuit;  /* opaque */
+lfqs_status lfqs_circuit_compile(lfqs_state* s, const lfqs_gate* gates, size_t n_gates,
+                                 uint32_t flags, lfqs_circuit** out, uint64_t* kernels_out);
+lfqs_status lfqs_circuit_launch(lfqs_circuit* c);
+lfqs_status lfqs_circuit_destroy(lfqs_circuit* c);
+
 /* ---- measurement -------------------------------------------- */
 /* probs_out[v] = sum over k with bit qubits[s] of k == bit s of v of |a_k|^2,
  * v in [0, 2^n_q).  n_q = 0 gives the squared norm.  n_q <= 20 (one

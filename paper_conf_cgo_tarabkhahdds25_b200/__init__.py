@@ -47,6 +47,7 @@ EXPORTS = [
     "lfqs_state_info", "lfqs_kernel_launches", "lfqs_set_option", "lfqs_last_error",
     "lfqs_abi_version", "lfqs_plan_circuit", "lfqs_measure_sample", "lfqs_measure_collapse",
     "lfqs_state_create_ex", "lfqs_state_wrap_ex", "lfqs_copy_in_c64", "lfqs_copy_out_c64",
+    "lfqs_circuit_compile", "lfqs_circuit_launch", "lfqs_circuit_destroy",
 ]
 STATE_C64 = 1
 
@@ -107,6 +108,10 @@ def lib():
             "lfqs_copy_out": [vp, u64, u64, dp],
             "lfqs_apply_gate": [vp, C.c_int, ip, C.c_int, ip, C.c_int, dp, C.c_int, dp],
             "lfqs_run_circuit": [vp, C.POINTER(LfqsGate), C.c_size_t, C.c_uint32],
+            "lfqs_circuit_compile": [vp, C.POINTER(LfqsGate), C.c_size_t, C.c_uint32,
+                                     C.POINTER(vp), C.POINTER(u64)],
+            "lfqs_circuit_launch": [vp],
+            "lfqs_circuit_destroy": [vp],
             "lfqs_measure_probs": [vp, ip, C.c_int, dp, C.c_size_t],
             "lfqs_synchronize": [vp],
             "lfqs_state_info": [vp, ip, ip, ip, ip, C.POINTER(vp)],
@@ -303,6 +308,53 @@ def lfqs_run_circuit(h: int, gates, flags: int = FUSE_NONE):
     _check(lib().lfqs_run_circuit(h, arr, n, flags))
 
 
+def lfqs_circuit_compile(h: int, gates, flags: int = FUSE_NONE):
+    """Captures the circuit into a CUDA graph; returns (circuit handle, kernels per launch)."""
+    if isinstance(gates, tuple) and len(gates) == 3 and isinstance(gates[1], int):
+        arr, n, keep = gates
+    else:
+        arr, n, keep = marshal_gates(gates)
+    out, k = C.c_void_p(), C.c_uint64()
+    _check(lib().lfqs_circuit_compile(h, arr, n, flags, C.byref(out), C.byref(k)))
+    return out.value, k.value
+
+
+def lfqs_circuit_launch(c: int):
+    _check(lib().lfqs_circuit_launch(c))
+
+
+def lfqs_circuit_destroy(c: int):
+    _check(lib().lfqs_circuit_destroy(c))
+
+
+class Circuit:
+    """A circuit captured once (CUDA graph) and replayed by launch()."""
+
+    def __init__(self, state: "State", gates, fuse: bool = False):
+        self.state = state  # keeps the state alive
+        self.h, self.kernels = lfqs_circuit_compile(state.h, gates, FUSE_LOW if fuse else FUSE_NONE)
+
+    def launch(self):
+        lfqs_circuit_launch(self.h)
+
+    def close(self):
+        if self.h:
+            lfqs_circuit_destroy(self.h)
+            self.h = None
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *exc):
+        self.close()
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
 def lfqs_measure_probs(h: int, qubits: Sequence[int] = ()) -> np.ndarray:
     q, nq = _ints(qubits)
     out = np.zeros(1 << nq, dtype=np.float64)
@@ -484,6 +536,9 @@ class State:
 
     def run_circuit(self, gates, fuse: bool = False):
         lfqs_run_circuit(self.h, gates, FUSE_LOW if fuse else FUSE_NONE)
+
+    def compile(self, gates, fuse: bool = False) -> Circuit:
+        return Circuit(self, gates, fuse)
 
     def measure_probs(self, qubits: Sequence[int] = ()) -> np.ndarray:
         return lfqs_measure_probs(self.h, qubits)

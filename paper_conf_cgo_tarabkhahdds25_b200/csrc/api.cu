@@ -195,28 +195,58 @@ lfqs_status lfqs_apply_gate(lfqs_state* s, int kind, const int* targets, int n_t
   });
 }
 
+namespace {
+std::vector<Decoded> decode_circuit(const State* st, const lfqs_gate* gates, size_t n_gates,
+                                    uint32_t flags) {
+  require(n_gates == 0 || gates != nullptr, "gates is NULL");
+  require((flags & ~LFQS_FUSE_LOW) == 0, "unknown flags");
+  std::vector<Decoded> dec;
+  dec.reserve(n_gates);
+  for (size_t i = 0; i < n_gates; ++i) {
+    const lfqs_gate& G = gates[i];
+    require(G.n_controls == __builtin_popcountll(G.control_mask),
+            "gate " + std::to_string(i) + ": n_controls != popcount(control_mask)");
+    try {
+      dec.push_back(decode_gate(st->n, G.kind, G.targets, G.n_targets, G.control_mask, G.params,
+                                kind_nparams(G.kind), G.matrix));
+    } catch (const Error& e) {
+      throw Error(e.status, "gate " + std::to_string(i) + ": " + e.what());
+    }
+  }
+  return dec;
+}
+}  // namespace
+
 lfqs_status lfqs_run_circuit(lfqs_state* s, const lfqs_gate* gates, size_t n_gates,
                              uint32_t flags) {
   return guarded([&] {
     require(s != nullptr, "NULL state");
-    require(n_gates == 0 || gates != nullptr, "gates is NULL");
-    require((flags & ~LFQS_FUSE_LOW) == 0, "unknown flags");
     State* st = static_cast<State*>(s);
-    std::vector<Decoded> dec;
-    dec.reserve(n_gates);
-    for (size_t i = 0; i < n_gates; ++i) {
-      const lfqs_gate& G = gates[i];
-      require(G.n_controls == __builtin_popcountll(G.control_mask),
-              "gate " + std::to_string(i) + ": n_controls != popcount(control_mask)");
-      try {
-        dec.push_back(decode_gate(st->n, G.kind, G.targets, G.n_targets, G.control_mask, G.params,
-                                  kind_nparams(G.kind), G.matrix));
-      } catch (const Error& e) {
-        throw Error(e.status, "gate " + std::to_string(i) + ": " + e.what());
-      }
-    }
-    st->run(dec, flags);
+    st->run(decode_circuit(st, gates, n_gates, flags), flags);
   });
+}
+
+lfqs_status lfqs_circuit_compile(lfqs_state* s, const lfqs_gate* gates, size_t n_gates,
+                                 uint32_t flags, lfqs_circuit** out, uint64_t* kernels_out) {
+  return guarded([&] {
+    require(s != nullptr && out != nullptr, "NULL argument");
+    *out = nullptr;
+    State* st = static_cast<State*>(s);
+    Graph* g = st->compile(decode_circuit(st, gates, n_gates, flags), flags);
+    *out = g;
+    if (kernels_out) *kernels_out = g->kernels;
+  });
+}
+
+lfqs_status lfqs_circuit_launch(lfqs_circuit* c) {
+  return guarded([&] {
+    require(c != nullptr, "NULL circuit");
+    static_cast<Graph*>(c)->launch();
+  });
+}
+
+lfqs_status lfqs_circuit_destroy(lfqs_circuit* c) {
+  return guarded([&] { delete static_cast<Graph*>(c); });
 }
 
 lfqs_status lfqs_plan_circuit(int n_qubits, int world, int rank, const lfqs_gate* gates,

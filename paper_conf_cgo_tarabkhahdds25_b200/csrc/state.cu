@@ -325,6 +325,56 @@ void State::run(const std::vector<Decoded>& gates, uint32_t flags) {
   execute(ops, fuse);
 }
 
+Graph* State::compile(const std::vector<Decoded>& gates, uint32_t flags) {
+  DeviceGuard dg(device);
+  if (comm != nullptr)
+    throw Error(LFQS_ERR_UNSUPPORTED, "circuit capture of a distributed (NCCL) state");
+  if (!plan.identity()) canonicalize();  // eager: the graph starts from the canonical map
+  cudaStream_t cs = nullptr;
+  LFQS_CUDA_CHECK(cudaStreamCreateWithFlags(&cs, cudaStreamNonBlocking));
+  const cudaStream_t saved = stream;
+  const uint64_t launches0 = launches, ex0 = exchanges, exb0 = exchange_bytes;
+  stream = cs;
+  cudaGraph_t graph = nullptr;
+  LFQS_CUDA_CHECK(cudaStreamBeginCapture(cs, cudaStreamCaptureModeThreadLocal));
+  try {
+    run(gates, flags);
+    if (!plan.identity()) canonicalize();  // the graph ends canonical: replays compose
+  } catch (...) {
+    cudaStreamEndCapture(cs, &graph);
+    if (graph) cudaGraphDestroy(graph);
+    stream = saved;
+    plan.reset();
+    launches = launches0;
+    cudaStreamDestroy(cs);
+    throw;
+  }
+  stream = saved;
+  const cudaError_t e = cudaStreamEndCapture(cs, &graph);
+  cudaStreamDestroy(cs);
+  LFQS_CUDA_CHECK(e);
+  std::unique_ptr<Graph> g(new Graph);
+  g->st = this;
+  g->kernels = launches - launches0;
+  launches = launches0;  // nothing ran yet
+  exchanges = ex0;
+  exchange_bytes = exb0;
+  const cudaError_t ei = cudaGraphInstantiate(&g->exec, graph, 0);
+  cudaGraphDestroy(graph);
+  LFQS_CUDA_CHECK(ei);
+  return g.release();
+}
+
+void Graph::launch() {
+  DeviceGuard dg(st->device);
+  LFQS_CUDA_CHECK(cudaGraphLaunch(exec, st->stream));
+  st->launches += kernels;
+}
+
+Graph::~Graph() {
+  if (exec) cudaGraphExecDestroy(exec);
+}
+
 void State::collapse(const int* qubits, int nq, uint64_t outcome, double scale) {
   DeviceGuard dg(device);
   for (int sh = 0; sh < n_shards(); ++sh) {

@@ -11,6 +11,9 @@
 struct lfqs_state {
   virtual ~lfqs_state() = default;
 };
+struct lfqs_circuit {
+  virtual ~lfqs_circuit() = default;
+};
 
 namespace lfqs {
 
@@ -56,6 +59,8 @@ struct State : lfqs_state {
   void copy_raw(uint64_t offset, uint64_t count, void* host, bool to_device);
   void apply(const Decoded& g);
   void run(const std::vector<Decoded>& gates, uint32_t flags);
+  // Captures the launches of run(gates, flags) into a CUDA graph (no GPU work).
+  struct Graph* compile(const std::vector<Decoded>& gates, uint32_t flags);
   void measure_probs(const int* qubits, int nq, double* out);
   void local_probs(int shard, const int* lq, int nl, double* host);
   // Zeroes amplitudes whose measured bits != outcome, scales the rest by `scale`.
@@ -73,6 +78,15 @@ struct State : lfqs_state {
   void run_local(const LaunchCtx& c, const std::vector<Decoded>& gates, bool fuse);
   void exchange_data(int l, int g);  // swap physical positions l (local) and g (global)
   void canonicalize();
+};
+
+// A circuit captured by State::compile; launch() replays it on the state's stream.
+struct Graph : lfqs_circuit {
+  State* st = nullptr;
+  cudaGraphExec_t exec = nullptr;
+  uint64_t kernels = 0;  // kernels per replay
+  void launch();
+  ~Graph() override;
 };
 
 }  // namespace lfqs
