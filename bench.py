@@ -12,7 +12,9 @@ The state (16 GiB) is >> the 126 MB L2, so no L2 flush is needed.
 
 N > 1 (torchrun, one rank per GPU): weak scaling, 2^30 amplitudes per GPU,
 n = 30 + log2 N, the same sweep over all n qubits (gates on the top log2 N
-"global" qubits go through the NCCL half-shard exchange).
+"global" qubits go through the half-shard exchange: by default the in-place
+peer-memory swap kernel over NVLink (CUDA IPC, --transport p2p), or staged NCCL
+send/recv (--transport nccl)).
 
 --impl reference: the CPU oracle (oracle/, tier B index loop with OpenMP on
 all host cores) on a bounded sample of the same sweep, rank 0 only.
@@ -210,6 +212,9 @@ def main():
     ap.add_argument("--e2e-steps", type=int, default=2)
     ap.add_argument("--ref-step-s", type=float, default=12.0)
     ap.add_argument("--per-gate-json", default="", help="write per-gate timings here")
+    ap.add_argument("--transport", default="p2p", choices=["p2p", "nccl"],
+                    help="N>1 global-qubit exchange: in-place peer-memory swap kernel (CUDA IPC "
+                         "over NVLink) or staged NCCL send/recv")
     args = ap.parse_args()
     if args.impl == "reference":
         return run_reference(args)
@@ -232,9 +237,12 @@ def main():
         p = world.bit_length() - 1
         assert 1 << p == world, "world size must be a power of two"
         n = args.n + p
-        obj = [lfqs.lfqs_dist_unique_id() if rank == 0 else None]
-        dist.broadcast_object_list(obj, src=0)
-        st = lfqs.State.distributed(n, rank, world, obj[0], local_rank, stream=stream)
+        if args.transport == "p2p":
+            st = lfqs.State.p2p(n, rank, world, local_rank, stream=stream)
+        else:
+            obj = [lfqs.lfqs_dist_unique_id() if rank == 0 else None]
+            dist.broadcast_object_list(obj, src=0)
+            st = lfqs.State.distributed(n, rank, world, obj[0], local_rank, stream=stream)
     else:
         n = args.n
         st = lfqs.State.create(n, local_rank, stream=stream)
@@ -371,7 +379,8 @@ def main():
                        "n_qubits": n, "qubits_per_gpu": n_loc, "gates_per_step": gates_per_step,
                        "state_bytes_per_gpu": 16 * 2 ** n_loc,
                        "l2": "state >> 126 MB L2 every gate; no flush needed",
-                       "parallelism": f"state sharded by top {world.bit_length() - 1} qubits"
+                       "parallelism": f"state sharded by top {world.bit_length() - 1} qubits, "
+                                      f"{args.transport} exchange"
                        if world > 1 else "single GPU"},
             "roofline": roofline,
             "classes": {k: {kk: (round(vv, 4) if isinstance(vv, float) else vv)

@@ -132,6 +132,27 @@ lfqs_status lfqs_state_set_stream(lfqs_state* s, void* cuda_stream);
 lfqs_status lfqs_dist_unique_id(uint8_t uid[128]);
 lfqs_status lfqs_state_create_dist(int n_qubits, int rank, int world, const uint8_t uid[128],
                                    int device, void* cuda_stream, lfqs_state** out);
+/* Peer-memory (CUDA IPC) sharding, NEXT-3: the same planner, with every global-
+ * qubit exchange done by ONE in-place swap kernel that loads and stores the
+ * partner's shard directly over NVLink / NVSwitch (no staging buffer, no NCCL),
+ * each partner swapping half of the pairs, ordered by device-side flags.
+ * Measurement histograms are summed across ranks in rank order (deterministic).
+ * Setup, on every rank (SPMD):
+ *   1. lfqs_state_create_p2p(n, rank, world, device, stream, flags, &s)
+ *      (flags: 0 or LFQS_STATE_C64; the shard is |0..0>'s part, synchronised);
+ *   2. lfqs_state_p2p_handle(s, blob) -> LFQS_P2P_HANDLE_BYTES opaque bytes;
+ *   3. all-gather the blobs in rank order (e.g. torch.distributed) and pass the
+ *      world * LFQS_P2P_HANDLE_BYTES bytes to lfqs_state_p2p_attach(s, all).
+ * Ranks may share a GPU (tests) or not; with different GPUs they must be
+ * peer-capable (NVLink).  A rank that stops participating makes its partners'
+ * barrier kernels time out after 30 s: the next synchronising call returns
+ * LFQS_ERR_CUDA.  lfqs_state_destroy is collective (a barrier precedes the
+ * unmapping).  Not capturable by lfqs_circuit_compile. */
+#define LFQS_P2P_HANDLE_BYTES 256
+lfqs_status lfqs_state_create_p2p(int n_qubits, int rank, int world, int device,
+                                  void* cuda_stream, uint32_t flags, lfqs_state** out);
+lfqs_status lfqs_state_p2p_handle(lfqs_state* s, uint8_t* blob);
+lfqs_status lfqs_state_p2p_attach(lfqs_state* s, const uint8_t* all_blobs);
 /* Single-GPU "virtual" partition: the same remap planner and exchange code
  * path with `world` shards in one allocation and device-to-device copies as the
  * transport.  For testing the distributed logic on one GPU. */

@@ -48,7 +48,9 @@ EXPORTS = [
     "lfqs_abi_version", "lfqs_plan_circuit", "lfqs_measure_sample", "lfqs_measure_collapse",
     "lfqs_state_create_ex", "lfqs_state_wrap_ex", "lfqs_copy_in_c64", "lfqs_copy_out_c64",
     "lfqs_circuit_compile", "lfqs_circuit_launch", "lfqs_circuit_destroy",
+    "lfqs_state_create_p2p", "lfqs_state_p2p_handle", "lfqs_state_p2p_attach",
 ]
+P2P_HANDLE_BYTES = 256
 STATE_C64 = 1
 
 
@@ -111,6 +113,10 @@ def lib():
             "lfqs_circuit_compile": [vp, C.POINTER(LfqsGate), C.c_size_t, C.c_uint32,
                                      C.POINTER(vp), C.POINTER(u64)],
             "lfqs_circuit_launch": [vp],
+            "lfqs_state_create_p2p": [C.c_int, C.c_int, C.c_int, C.c_int, vp, C.c_uint32,
+                                      C.POINTER(vp)],
+            "lfqs_state_p2p_handle": [vp, C.POINTER(C.c_uint8)],
+            "lfqs_state_p2p_attach": [vp, C.POINTER(C.c_uint8)],
             "lfqs_circuit_destroy": [vp],
             "lfqs_measure_probs": [vp, ip, C.c_int, dp, C.c_size_t],
             "lfqs_synchronize": [vp],
@@ -223,6 +229,25 @@ def lfqs_dist_unique_id() -> bytes:
     buf = (C.c_uint8 * 128)()
     _check(lib().lfqs_dist_unique_id(buf))
     return bytes(buf)
+
+
+def lfqs_state_create_p2p(n_qubits: int, rank: int, world: int, device: int, stream=None,
+                          flags: int = 0) -> int:
+    h = C.c_void_p()
+    _check(lib().lfqs_state_create_p2p(n_qubits, rank, world, device, _stream_handle(stream),
+                                       flags, C.byref(h)))
+    return h.value
+
+
+def lfqs_state_p2p_handle(h: int) -> bytes:
+    buf = (C.c_uint8 * P2P_HANDLE_BYTES)()
+    _check(lib().lfqs_state_p2p_handle(h, buf))
+    return bytes(buf)
+
+
+def lfqs_state_p2p_attach(h: int, blobs: bytes):
+    buf = (C.c_uint8 * len(blobs)).from_buffer_copy(blobs)
+    _check(lib().lfqs_state_p2p_attach(h, buf))
 
 
 def lfqs_state_create_dist(n_qubits: int, rank: int, world: int, uid: bytes, device: int,
@@ -486,6 +511,19 @@ class State:
     def distributed(cls, n_qubits: int, rank: int, world: int, uid: bytes, device: int,
                     stream=None) -> "State":
         return cls(lfqs_state_create_dist(n_qubits, rank, world, uid, device, stream), n_qubits)
+
+    @classmethod
+    def p2p(cls, n_qubits: int, rank: int, world: int, device: int = 0, stream=None,
+            c64: bool = False, group=None) -> "State":
+        """One rank of a peer-memory (CUDA IPC) sharded state; collective over the
+        torch.distributed group (any backend), which carries the 256-byte handles."""
+        import torch.distributed as dist
+        h = lfqs_state_create_p2p(n_qubits, rank, world, device, stream, STATE_C64 if c64 else 0)
+        st = cls(h, n_qubits, c64)
+        blobs = [None] * world
+        dist.all_gather_object(blobs, lfqs_state_p2p_handle(h), group=group)
+        lfqs_state_p2p_attach(h, b"".join(blobs))
+        return st
 
     def close(self):
         if self.h:

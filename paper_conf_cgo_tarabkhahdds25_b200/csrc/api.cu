@@ -142,6 +142,30 @@ lfqs_status lfqs_state_create_dist(int n_qubits, int rank, int world, const uint
   });
 }
 
+lfqs_status lfqs_state_create_p2p(int n_qubits, int rank, int world, int device, void* stream,
+                                  uint32_t flags, lfqs_state** out) {
+  return guarded([&] {
+    require(out != nullptr, "out is NULL");
+    require((flags & ~(uint32_t)LFQS_STATE_C64) == 0, "unknown flags");
+    *out = State::create_p2p(n_qubits, rank, world, device, static_cast<cudaStream_t>(stream),
+                             (flags & LFQS_STATE_C64) != 0);
+  });
+}
+
+lfqs_status lfqs_state_p2p_handle(lfqs_state* s, uint8_t* blob) {
+  return guarded([&] {
+    require(s != nullptr && blob != nullptr, "NULL argument");
+    static_cast<State*>(s)->p2p_handle(blob);
+  });
+}
+
+lfqs_status lfqs_state_p2p_attach(lfqs_state* s, const uint8_t* all_blobs) {
+  return guarded([&] {
+    require(s != nullptr && all_blobs != nullptr, "NULL argument");
+    static_cast<State*>(s)->p2p_attach(all_blobs);
+  });
+}
+
 lfqs_status lfqs_state_destroy(lfqs_state* s) {
   return guarded([&] { delete static_cast<State*>(s); });
 }

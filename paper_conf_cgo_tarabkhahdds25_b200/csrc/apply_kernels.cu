@@ -614,13 +614,17 @@ void launch_gate_t(const LaunchCtx& ctx, const Decoded& g) {
 // Virtual-partition exchange: swap the l=1 half of this shard with the l=0 half
 // of the shard `partner_offset_amps` amplitudes further on (same pass structure
 // as a SWAP gate).
-void launch_half_swap(const LaunchCtx& ctx, int l, uint64_t partner_offset_amps) {
+// n_pairs = 0: all 2^(n_local-1) pairs; otherwise the first n_pairs (the P2P
+// exchange splits the pairs between the two ranks, p2p.cu).  The partner may be
+// any address (a peer GPU's shard mapped by CUDA IPC): the offset wraps mod 2^64.
+void launch_half_swap(const LaunchCtx& ctx, int l, uint64_t partner_offset_amps, uint64_t n_pairs) {
   const InsertPlan ip = make_plan(1ull << l, 0);
   Offs<2> off{{1ull << l, partner_offset_amps}};
+  if (n_pairs == 0) n_pairs = 1ull << (ctx.n_local - 1);
   if (ctx.c64)
-    run_group<float, 2, 4, false>(ctx, 1ull << (ctx.n_local - 1), ip, off, OpSwap2<float>{});
+    run_group<float, 2, 4, false>(ctx, n_pairs, ip, off, OpSwap2<float>{});
   else
-    run_group<double, 2, 4, false>(ctx, 1ull << (ctx.n_local - 1), ip, off, OpSwap2<double>{});
+    run_group<double, 2, 4, false>(ctx, n_pairs, ip, off, OpSwap2<double>{});
 }
 
 void launch_gate(const LaunchCtx& ctx, const Decoded& g) {

@@ -107,6 +107,11 @@ void ensure_smem_attr(const void* kernel, int bytes);
 
 // Applies one decoded gate whose targets are all < n_local (controls < n_local).
 void launch_gate(const LaunchCtx& ctx, const Decoded& g);
+// Half-shard swap for the global-qubit exchange: the l=1 half of the shard at
+// ctx.amps with the l=0 half of the shard partner_offset_amps further on (first
+// n_pairs pairs; 0 = all).
+void launch_half_swap(const LaunchCtx& ctx, int l, uint64_t partner_offset_amps,
+                      uint64_t n_pairs = 0);
 
 // Fused staging of gates[begin..): applies the longest prefix that fits one tile
 // program in one HBM pass; false if fewer than two gates fuse (fused_kernels.cu).

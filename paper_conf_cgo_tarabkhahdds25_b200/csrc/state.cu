@@ -15,12 +15,12 @@
 #include <string>
 
 #include "comm.h"
+#include "p2p.h"
 #include "state.h"
 
 namespace lfqs {
 
 // Defined in apply_kernels.cu / fused_kernels.cu.
-void launch_half_swap(const LaunchCtx& ctx, int l, uint64_t partner_offset_amps);
 bool run_fused_circuit(const LaunchCtx& ctx, const std::vector<Decoded>& gates, size_t begin,
                        size_t end, int tile_qubits, size_t* consumed);
 
@@ -128,10 +128,37 @@ State* State::create_dist(int n, int rank, int world, const uint8_t uid[128], in
   return st.release();
 }
 
+State* State::create_p2p(int n, int rank, int world, int device, cudaStream_t stream, bool c64) {
+  require(world >= 2, "a p2p state needs world >= 2");
+  require(rank >= 0 && rank < world, "rank out of range");
+  std::unique_ptr<State> st(new State());
+  st->common_init(n, world, device, stream, c64);
+  st->rank = rank;
+  st->amps = alloc_amps(1ull << st->n_local, st->ab);
+  st->owned = true;
+  st->p2p = new P2P(rank, world, device);
+  st->init_basis(0);
+  st->synchronize();
+  return st.release();
+}
+
+void State::p2p_handle(uint8_t* out) {
+  require(p2p != nullptr, "not a p2p state");
+  DeviceGuard dg(device);
+  p2p->handle(amps, n_local, ab, out);
+}
+
+void State::p2p_attach(const uint8_t* all) {
+  require(p2p != nullptr, "not a p2p state");
+  DeviceGuard dg(device);
+  p2p->attach(amps, n_local, ab, all);
+}
+
 State::~State() {
   if (device >= 0) cudaSetDevice(device);
   if (stream) cudaStreamSynchronize(stream);
   delete comm;
+  delete p2p;  // barrier: no peer touches this shard any more
   if (owned && amps) cudaFree(amps);
   if (d_partials) cudaFree(d_partials);
   if (d_probs) cudaFree(d_probs);
@@ -186,6 +213,7 @@ void State::synchronize() {
   DeviceGuard dg(device);
   LFQS_CUDA_CHECK(cudaStreamSynchronize(stream));
   LFQS_CUDA_CHECK(cudaGetLastError());
+  if (p2p) p2p->check();
 }
 
 void State::copy_raw(uint64_t offset, uint64_t count, void* host, bool to_device) {
@@ -236,6 +264,8 @@ void State::exchange_data(int l, int g) {
       const int r2 = r | (1 << j);
       launch_half_swap(ctx(r), l, ((uint64_t)(r2 - r)) << n_local);
     }
+  } else if (p2p) {
+    p2p->exchange(ctx(0), l, j, n_local);
   } else {
     const int b = (rank >> j) & 1;
     std::vector<Piece> pieces;
@@ -327,8 +357,8 @@ void State::run(const std::vector<Decoded>& gates, uint32_t flags) {
 
 Graph* State::compile(const std::vector<Decoded>& gates, uint32_t flags) {
   DeviceGuard dg(device);
-  if (comm != nullptr)
-    throw Error(LFQS_ERR_UNSUPPORTED, "circuit capture of a distributed (NCCL) state");
+  if (comm != nullptr || p2p != nullptr)
+    throw Error(LFQS_ERR_UNSUPPORTED, "circuit capture of a multi-process (NCCL / p2p) state");
   if (!plan.identity()) canonicalize();  // eager: the graph starts from the canonical map
   cudaStream_t cs = nullptr;
   LFQS_CUDA_CHECK(cudaStreamCreateWithFlags(&cs, cudaStreamNonBlocking));
@@ -445,7 +475,9 @@ void State::measure_probs(const int* qubits, int nq, double* out) {
       full[v] += loc[lb];
     }
   }
-  if (!virt && world > 1) {
+  if (p2p) {
+    p2p->allreduce_sum(full.data(), nb, stream);
+  } else if (!virt && world > 1) {
     double* d = comm->d_reduce;
     if (nb > 1024) LFQS_CUDA_CHECK(cudaMalloc(&d, sizeof(double) * nb));
     LFQS_CUDA_CHECK(cudaMemcpyAsync(d, full.data(), sizeof(double) * nb, cudaMemcpyHostToDevice,

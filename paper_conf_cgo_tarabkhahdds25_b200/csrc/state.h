@@ -18,6 +18,7 @@ struct lfqs_circuit {
 namespace lfqs {
 
 struct Comm;  // NCCL communicator wrapper (comm.cu)
+struct P2P;   // peer-memory transport (p2p.cu)
 
 // Layout in HBM: a shard is 2^n_local interleaved complex128
 // amplitudes, contiguous, 256-byte aligned.  Physical bit positions
@@ -38,6 +39,7 @@ struct State : lfqs_state {
   double* d_probs = nullptr;
   Planner plan;
   Comm* comm = nullptr;
+  P2P* p2p = nullptr;           // CUDA-IPC peer transport (instead of comm)
   // exchange statistics (benchmark accounting)
   uint64_t exchanges = 0, exchange_bytes = 0;
 
@@ -47,6 +49,11 @@ struct State : lfqs_state {
                                bool c64 = false);
   static State* create_dist(int n, int rank, int world, const uint8_t uid[128], int device,
                             cudaStream_t stream);
+  // One rank of a P2P-sharded state: peers are attached later (p2p_attach).
+  static State* create_p2p(int n, int rank, int world, int device, cudaStream_t stream,
+                           bool c64 = false);
+  void p2p_handle(uint8_t* out);
+  void p2p_attach(const uint8_t* all);
   static void nccl_unique_id(uint8_t uid[128]);
   ~State() override;
 

@@ -1,0 +1,58 @@
+"""Worker of tests/test_gpu_p2p.py: one rank of a peer-memory (CUDA IPC) sharded
+state.  All ranks share cuda:0 (IPC works between processes on one device), so the
+NVLink P2P exchange kernel, the device-side flag barriers and the rank-ordered
+probability reduction run for real on the single test GPU."""
+import os
+import traceback
+
+import numpy as np
+
+
+def worker(rank, world, port, n, seed, out_q):
+    try:
+        import torch
+        import torch.distributed as dist
+
+        os.environ["MASTER_ADDR"] = "127.0.0.1"
+        os.environ["MASTER_PORT"] = str(port)
+        dist.init_process_group("gloo", rank=rank, world_size=world)
+        torch.cuda.set_device(0)
+        import oracle as O
+        import paper_conf_cgo_tarabkhahdds25_b200 as L
+        import workloads as W
+
+        nl = n - (world.bit_length() - 1)
+        lo, hi = rank << nl, (rank + 1) << nl
+        report = {}
+        psi = W.random_state(n, seed)
+        gates = W.random_gate_list(n, 160, seed=seed + 11, max_controls=2) + W.qft(n)
+        exact = [g for g in W.random_gate_list(n, 200, seed=seed + 12, max_controls=2) if g.exact]
+        ref = O.run_circuit(n, gates, psi.copy())
+        ref_exact = O.run_circuit(n, exact, psi.copy())
+        qs = [0, n // 2, n - 1]
+        for fuse in (False, True):
+            with L.State.p2p(n, rank, world) as st:
+                st.copy_in(psi)
+                st.run_circuit(gates, fuse=fuse)
+                got = st.copy_out()[lo:hi]
+                err = float(np.max(np.abs(got - ref[lo:hi])))
+                p = st.measure_probs(qs)
+                perr = float(np.max(np.abs(p - O.probs(n, ref, qs))))
+                report[f"fuse{int(fuse)}"] = (err, perr)
+                st.copy_in(psi)
+                st.run_circuit(exact, fuse=fuse)
+                report[f"exact{int(fuse)}"] = bool(np.array_equal(st.copy_out()[lo:hi],
+                                                                   ref_exact[lo:hi]))
+                st.synchronize()
+        # one gate at a time through lfqs_apply_gate (planner per gate, exchanges included)
+        with L.State.p2p(n, rank, world) as st:
+            st.copy_in(psi)
+            for g in gates[:60]:
+                st.apply(g)
+            want = O.run_circuit(n, gates[:60], psi.copy())
+            report["apply"] = float(np.max(np.abs(st.copy_out()[lo:hi] - want[lo:hi])))
+        dist.barrier()
+        dist.destroy_process_group()
+        out_q.put((rank, "ok", report))
+    except Exception:
+        out_q.put((rank, "error", traceback.format_exc()))
