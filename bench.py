@@ -206,12 +206,14 @@ def main():
     ap.add_argument("--steps", type=int, default=5)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="lfqs", choices=["lfqs", "reference"])
-    ap.add_argument("--n", type=int, default=30, help="qubits per GPU")
+    ap.add_argument("--n", "--qubits-per-gpu", dest="n", type=int, default=30, help="qubits per GPU")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--e2e-steps", type=int, default=2)
     ap.add_argument("--ref-step-s", type=float, default=12.0)
     ap.add_argument("--per-gate-json", default="", help="write per-gate timings here")
+    ap.add_argument("--same-device", action="store_true",
+                    help="test only: every rank on cuda:0 (exercises the N>1 path on one GPU)")
     ap.add_argument("--transport", default="p2p", choices=["p2p", "nccl"],
                     help="N>1 global-qubit exchange: in-place peer-memory swap kernel (CUDA IPC "
                          "over NVLink) or staged NCCL send/recv")
@@ -227,13 +229,17 @@ def main():
     local_rank = int(os.environ.get("LOCAL_RANK", "0"))
     assert world == args.gpus, f"--gpus {args.gpus} but WORLD_SIZE={world}"
     assert args.warmup >= 3 or os.environ.get("LFQS_BENCH_ALLOW_SHORT"), "need >= 3 warm-up steps"
+    if args.same_device:
+        local_rank = 0
     torch.cuda.set_device(local_rank)
     stream = torch.cuda.Stream()      # the library launches on this stream; events too
     torch.cuda.set_stream(stream)
     dist = None
     if world > 1:
         import torch.distributed as dist
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
+        dist.init_process_group("gloo" if args.same_device else "nccl",
+                                device_id=None if args.same_device
+                                else torch.device("cuda", local_rank))
         p = world.bit_length() - 1
         assert 1 << p == world, "world size must be a power of two"
         n = args.n + p
@@ -256,11 +262,18 @@ def main():
             dist.barrier()
         torch.cuda.synchronize()
 
-    def one_step(evs=None):
+    ex_marks = np.zeros((max(args.steps, 1), len(sweep)), dtype=np.int64)  # exchanges (N > 1)
+
+    def one_step(evs=None, k=0):
         for i, (_, g) in enumerate(sweep):
             if evs is not None:
                 evs[i].record(stream)
-            st.apply(g)
+            if world > 1:
+                e0 = st.exchange_stats()[0]
+                st.apply(g)
+                ex_marks[k, i] = st.exchange_stats()[0] - e0
+            else:
+                st.apply(g)
         if evs is not None:
             evs[len(sweep)].record(stream)
 
@@ -269,6 +282,7 @@ def main():
     barrier()
 
     launches0 = st.launches()
+    ex0 = st.exchange_stats()
     evs = [[torch.cuda.Event(enable_timing=True) for _ in range(len(sweep) + 1)]
            for _ in range(args.steps)]
     t_start = torch.cuda.Event(enable_timing=True)
@@ -277,13 +291,14 @@ def main():
         barrier()
         t_start.record(stream)
         for k in range(args.steps):
-            one_step(evs[k])
+            one_step(evs[k], k)
         t_end.record(stream)
         barrier()
     launches = st.launches() - launches0
+    ex1 = st.exchange_stats()
     elapsed_ms = t_start.elapsed_time(t_end)
     if dist is not None:
-        t = torch.tensor([elapsed_ms], device="cuda")
+        t = torch.tensor([elapsed_ms], device="cpu" if args.same_device else "cuda")
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         elapsed_ms = float(t.item())
     ms_per_step = elapsed_ms / args.steps
@@ -315,7 +330,7 @@ def main():
     dc = classes[dom]
     traffic = None
     tp = os.path.join(ROOT, "profiles", "traffic_per_launch.json")
-    if os.path.exists(tp):
+    if world == 1 and os.path.exists(tp):  # ncu capture of the N = 1 workload
         try:
             traffic = json.load(open(tp)).get(dom)
         except Exception:
@@ -325,6 +340,30 @@ def main():
                 "frac": dc["alg_GBps"] / hbm_peak, "traffic": traffic, "peak_source": peak_src,
                 "bytes_per_launch": dc["alg_bytes"] / dc["gates"],
                 "avg_launch_ms": dc["ms"] / dc["gates"]}
+    # N > 1: the global-qubit exchanges (half-shard swaps over NVLink).  A gate that
+    # issued exchanges costs its local pass plus the exchanges; the local part is
+    # estimated by the median of the same class's exchange-free gates.
+    nvlink = None
+    if world > 1:
+        n_ex = (ex1[0] - ex0[0]) / args.steps
+        ex_bytes = (ex1[1] - ex0[1]) / args.steps
+        t_ex = 0.0
+        for k in range(args.steps):
+            for i, (cls, g) in enumerate(sweep):
+                if ex_marks[k, i] > 0:
+                    local = [per_gate[k2, i2] for k2 in range(args.steps)
+                             for i2, (c2, _) in enumerate(sweep)
+                             if c2 == cls and ex_marks[k2, i2] == 0]
+                    t_ex += max(per_gate[k, i] - (float(np.median(local)) if local else 0.0),
+                                1e-6)
+        t_ex /= args.steps
+        link_gbps = ex_bytes / (t_ex / 1e3) / 1e9 if t_ex > 0 else None
+        nvlink = {"exchanges_per_step": n_ex, "bytes_per_rank_per_direction_per_step": ex_bytes,
+                  "exchange_ms_per_step": t_ex, "achieved": link_gbps, "unit": "GB/s",
+                  "peak": 900.0, "peak_source": "nominal NVLink 5, per GPU per direction",
+                  "frac": link_gbps / 900.0 if link_gbps else None,
+                  "transport": args.transport}
+
     if args.per_gate_json and rank == 0:
         with open(args.per_gate_json, "w") as f:
             json.dump([{"cls": cls, "gate": g.label(), "ms": float(mean_ms[i]),
@@ -354,7 +393,7 @@ def main():
         barrier()
         e_ms = a.elapsed_time(b)
         if dist is not None:
-            t = torch.tensor([e_ms], device="cuda")
+            t = torch.tensor([e_ms], device="cpu" if args.same_device else "cuda")
             dist.all_reduce(t, op=dist.ReduceOp.MAX)
             e_ms = float(t.item())
         e2e = {"value": gates_per_step / (e_ms / args.e2e_steps / 1e3), "unit": UNIT,
@@ -381,8 +420,11 @@ def main():
                        "l2": "state >> 126 MB L2 every gate; no flush needed",
                        "parallelism": f"state sharded by top {world.bit_length() - 1} qubits, "
                                       f"{args.transport} exchange"
-                       if world > 1 else "single GPU"},
+                       if world > 1 else "single GPU",
+                       **({"test_same_device": "all ranks share cuda:0 -- not a scaling number"}
+                          if args.same_device else {})},
             "roofline": roofline,
+            "nvlink": nvlink,
             "classes": {k: {kk: (round(vv, 4) if isinstance(vv, float) else vv)
                             for kk, vv in v.items()} for k, v in classes.items()},
             "gpu_launches": int(launches),

@@ -262,6 +262,11 @@ lfqs_status lfqs_synchronize(lfqs_state* s);
 /* n_qubits, local qubits, rank, world, and the device pointer of the local shard. */
 lfqs_status lfqs_state_info(const lfqs_state* s, int* n_qubits, int* n_local, int* rank,
                             int* world, void** dev_ptr);
+/* Global-qubit exchanges this state has issued so far (sharded states; 0 on one
+ * GPU) and the bytes each one sends per rank and direction (16 or 8 * 2^(n_local-1)),
+ * summed.  Counted when the exchange is enqueued (host side, no synchronisation). */
+lfqs_status lfqs_state_exchange_stats(const lfqs_state* s, uint64_t* exchanges,
+                                      uint64_t* bytes_per_rank);
 /* Number of kernels this state has launched so far (for benchmark accounting). */
 lfqs_status lfqs_kernel_launches(const lfqs_state* s, uint64_t* count);
 /* Tuning knobs (benchmark / test use): LFQS_OPT_LOWQ_SHUFFLE (1: warp-shuffle

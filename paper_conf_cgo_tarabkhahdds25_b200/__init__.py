@@ -49,6 +49,7 @@ EXPORTS = [
     "lfqs_state_create_ex", "lfqs_state_wrap_ex", "lfqs_copy_in_c64", "lfqs_copy_out_c64",
     "lfqs_circuit_compile", "lfqs_circuit_launch", "lfqs_circuit_destroy",
     "lfqs_state_create_p2p", "lfqs_state_p2p_handle", "lfqs_state_p2p_attach",
+    "lfqs_state_exchange_stats",
 ]
 P2P_HANDLE_BYTES = 256
 STATE_C64 = 1
@@ -117,6 +118,7 @@ def lib():
                                       C.POINTER(vp)],
             "lfqs_state_p2p_handle": [vp, C.POINTER(C.c_uint8)],
             "lfqs_state_p2p_attach": [vp, C.POINTER(C.c_uint8)],
+            "lfqs_state_exchange_stats": [vp, C.POINTER(u64), C.POINTER(u64)],
             "lfqs_circuit_destroy": [vp],
             "lfqs_measure_probs": [vp, ip, C.c_int, dp, C.c_size_t],
             "lfqs_synchronize": [vp],
@@ -595,6 +597,12 @@ class State:
 
     def info(self) -> dict:
         return lfqs_state_info(self.h)
+
+    def exchange_stats(self):
+        """(exchanges issued, bytes sent per rank and direction), cumulative."""
+        a, b = C.c_uint64(), C.c_uint64()
+        _check(lib().lfqs_state_exchange_stats(self.h, C.byref(a), C.byref(b)))
+        return a.value, b.value
 
     def launches(self) -> int:
         return lfqs_kernel_launches(self.h)

@@ -412,6 +412,16 @@ lfqs_status lfqs_synchronize(lfqs_state* s) {
   });
 }
 
+lfqs_status lfqs_state_exchange_stats(const lfqs_state* s, uint64_t* exchanges,
+                                      uint64_t* bytes_per_rank) {
+  return guarded([&] {
+    require(s != nullptr, "NULL state");
+    const State* st = static_cast<const State*>(s);
+    if (exchanges) *exchanges = st->exchanges;
+    if (bytes_per_rank) *bytes_per_rank = st->exchange_bytes;
+  });
+}
+
 lfqs_status lfqs_state_info(const lfqs_state* s, int* n_qubits, int* n_local, int* rank,
                             int* world, void** dev_ptr) {
   return guarded([&] {
