@@ -314,7 +314,7 @@ lfqs_status lfqs_plan_circuit(int n_qubits, int world, int rank, const lfqs_gate
         continue;
       }
       Decoded lg;
-      if (!plan.rank_local(op.gate, rank, &lg) || lg.cls == GClass::NOOP) continue;
+      if (!plan.rank_local(op.gate, rank, op.gflip, &lg) || lg.cls == GClass::NOOP) continue;
       o.kind = LFQS_PLAN_LOCAL;
       if (lg.m == 0) {
         // Scalar on the control-satisfying amplitudes: express as a 1-target gate.

@@ -30,9 +30,11 @@ Planner::Planner(int n_, int world_) : n(n_), world(world_) {
 
 void Planner::reset() {
   for (int q = 0; q < 64; ++q) l2p[q] = p2l[q] = q;
+  gflip = 0;
 }
 
 bool Planner::identity() const {
+  if (gflip != 0) return false;
   for (int q = 0; q < n; ++q)
     if (l2p[q] != q) return false;
   return true;
@@ -60,6 +62,17 @@ void Planner::exchange(int l, int g, std::vector<PlanOp>& out) {
   l2p[qb] = l;
   p2l[l] = qb;
   p2l[g] = qa;
+  if (gflip >> g & 1) {
+    // The incoming qubit was relabelled by global X gates: materialise the flip
+    // on its new local position (the qubit now at g carries no flip).
+    gflip &= ~(1ull << g);
+    const int t[1] = {l};
+    PlanOp x;
+    x.kind = PlanOp::LOCAL;
+    x.gate = decode_gate(n, LFQS_X, t, 1, 0, nullptr, 0, nullptr);
+    x.gflip = gflip;
+    out.push_back(x);
+  }
 }
 
 void Planner::swap_local(int a, int b, std::vector<PlanOp>& out) {
@@ -67,6 +80,7 @@ void Planner::swap_local(int a, int b, std::vector<PlanOp>& out) {
   PlanOp op;
   op.kind = PlanOp::LOCAL;
   op.gate = decode_gate(n, LFQS_SWAP, t, 2, 0, nullptr, 0, nullptr);
+  op.gflip = gflip;
   out.push_back(op);
   const int qa = p2l[a], qb = p2l[b];
   l2p[qa] = b;
@@ -76,6 +90,10 @@ void Planner::swap_local(int a, int b, std::vector<PlanOp>& out) {
 }
 
 void Planner::plan_canonicalize(std::vector<PlanOp>& out) {
+  // Phase 0: materialise global flips (each costs one exchange and an X pass;
+  // the phases below then move every qubit home).
+  for (int G = n_local; G < n; ++G)
+    if (gflip >> G & 1) exchange(n_local - 1, G, out);
   // Phase 1: bring each global home position G its logical qubit G -- one exchange
   // when that qubit sits at a local position, two (through a local staging position
   // L) when it sits at another global one.  L is chosen as the home of the qubit that
@@ -104,6 +122,7 @@ void Planner::plan_circuit(const std::vector<Decoded>& gates, std::vector<PlanOp
   for (size_t i = 0; i < gates.size(); ++i) {
     const Decoded& g = gates[i];
     if (g.cls == GClass::NOOP || g.cls == GClass::DIAG) continue;
+    if (g.cls == GClass::PERM_X && g.cmask == 0) continue;  // relabel when global
     for (int s = 0; s < g.m; ++s) uses[g.targets[s]].push_back((int)i);
   }
   std::vector<int> next_use(n);
@@ -120,6 +139,10 @@ void Planner::plan_gate(const Decoded& g, std::vector<PlanOp>& out,
                         const std::vector<int>* next_use) {
   if (g.cls == GClass::NOOP) return;
   Decoded pg = to_physical(g);
+  if (world > 1 && pg.cls == GClass::PERM_X && pg.cmask == 0 && pg.targets[0] >= n_local) {
+    gflip ^= 1ull << pg.targets[0];  // global X: relabel, no data movement
+    return;
+  }
   if (world > 1 && pg.cls == GClass::PERM_SWAP && pg.cmask == 0 &&
       (pg.targets[0] >= n_local || pg.targets[1] >= n_local)) {
     // SWAP of logical qubits = exchange their physical positions in the map.
@@ -156,11 +179,14 @@ void Planner::plan_gate(const Decoded& g, std::vector<PlanOp>& out,
   PlanOp op;
   op.kind = PlanOp::LOCAL;
   op.gate = pg;
+  op.gflip = gflip;
   out.push_back(op);
 }
 
-bool Planner::rank_local(const Decoded& pg, int r, Decoded* out) const {
+bool Planner::rank_local(const Decoded& pg, int r_phys, uint64_t f, Decoded* out) const {
   const uint64_t local_mask = (n_local >= 64) ? ~0ull : ((1ull << n_local) - 1);
+  // The logical values of the global positions on this rank (flips applied).
+  const int r = r_phys ^ (int)(f >> n_local);
   const uint64_t gctrl = pg.cmask >> n_local;
   if ((gctrl & (uint64_t)r) != gctrl) return false;  // a global control is 0 on this rank
   *out = pg;

@@ -16,11 +16,18 @@ struct PlanOp {
   Decoded gate;   // LOCAL: gate on physical positions (controls may be global)
   int l = 0;      // EXCHANGE: local physical position
   int g = 0;      // EXCHANGE: global physical position (rank bit g - n_local)
+  uint64_t gflip = 0;  // LOCAL: the global-position flips in force for this op
 };
 
 struct Planner {
   int n = 0, n_local = 0, world = 1;
   int l2p[64], p2l[64];
+  // Global-X relabeling (NEXT-1): bit P set = the data at global position P holds
+  // the complement of its logical qubit (rank bit = logical value ^ 1).  An
+  // uncontrolled X on a global qubit toggles it instead of moving data; the flip
+  // is materialised (an X pass on the local position) when the qubit is
+  // exchanged back into the shard.
+  uint64_t gflip = 0;
 
   Planner() { reset(); }
   Planner(int n_, int world_);
@@ -41,7 +48,12 @@ struct Planner {
   // Specialises a LOCAL op for rank r: false if a global control is 0 there;
   // otherwise *out has only local targets/controls (diagonals on global targets
   // folded into a smaller diagonal; cls NOOP if nothing is left to do).
-  bool rank_local(const Decoded& pg, int r, Decoded* out) const;
+  // gflip: the op's flips (PlanOp::gflip); r is read through them.
+  bool rank_local(const Decoded& pg, int r, uint64_t gflip, Decoded* out) const;
+  // The logical value of global position P on rank r under flips f.
+  int global_bit(int r, int P, uint64_t f) const {
+    return ((r >> (P - n_local)) & 1) ^ (int)((f >> P) & 1);
+  }
 
  private:
   Decoded to_physical(const Decoded& g) const;

@@ -317,7 +317,7 @@ void State::execute(const std::vector<PlanOp>& ops, bool fuse) {
       seg.reserve(j - i);
       for (size_t k = i; k < j; ++k) {
         Decoded lg;
-        if (plan.rank_local(ops[k].gate, rank_of_shard(s), &lg) && lg.cls != GClass::NOOP)
+        if (plan.rank_local(ops[k].gate, rank_of_shard(s), ops[k].gflip, &lg) && lg.cls != GClass::NOOP)
           seg.push_back(lg);
       }
       run_local(ctx(s), seg, fuse);
@@ -417,7 +417,7 @@ void State::collapse(const int* qubits, int nq, uint64_t outcome, double scale) 
       if (P < n_local) {
         mask |= 1ull << P;
         pat |= bit << P;
-      } else if ((uint64_t)((r >> (P - n_local)) & 1) != bit) {
+      } else if ((uint64_t)plan.global_bit(r, P, plan.gflip) != bit) {
         rank_matches = false;
       }
     }
@@ -467,7 +467,7 @@ void State::measure_probs(const int* qubits, int nq, double* out) {
     uint64_t gbits = 0;
     for (int s = 0; s < nq; ++s) {
       const int P = plan.l2p[qubits[s]];
-      if (P >= n_local) gbits |= (uint64_t)((r >> (P - n_local)) & 1) << s;
+      if (P >= n_local) gbits |= (uint64_t)plan.global_bit(r, P, plan.gflip) << s;
     }
     for (uint64_t lb = 0; lb < (1ull << nl); ++lb) {
       uint64_t v = gbits;

@@ -100,3 +100,30 @@ def test_virtual_qft_and_ghz(L):
         st.run_circuit(W.ghz(n))
         a = st.copy_out()
         assert a[0] == np.sqrt(0.5) and a[-1] == np.sqrt(0.5) and np.count_nonzero(a) == 2
+
+
+@pytest.mark.parametrize("world", [2, 4])
+def test_global_x_relabel_measure(L, world):
+    """X on global qubits is a relabel (no exchange); probabilities, sampling and
+    collapse read the flips, and copy_out materialises them."""
+    n = 12
+    psi = W.random_state(n, 33)
+    gates = [W.Gate("X", (n - 1,)), W.Gate("X", (n - 2,)), W.CNOT(n - 1, 0),
+             W.Gate("T", (n - 2,)), W.Gate("X", (n - 1,)), W.Gate("X", (n - 1,))]
+    ref = O.run_circuit(n, gates, psi.copy())
+    qs = [n - 1, 0, n - 2]
+    with L.State.virtual(n, world) as st:
+        st.copy_in(psi)
+        e0 = st.exchange_stats()[0]
+        st.run_circuit(gates)
+        assert st.exchange_stats()[0] == e0  # relabels only
+        p = st.measure_probs(qs)
+        np.testing.assert_allclose(p, O.probs(n, ref, qs), rtol=0, atol=1e-14)
+        u = np.array([0.05, 0.3, 0.61, 0.97])
+        np.testing.assert_array_equal(st.sample(qs, u), O.measure_sample(n, ref, qs, u))
+        pr = st.collapse(qs, 5)
+        want = ref.copy()
+        wp = O.measure_collapse(n, want, qs, 5)
+        assert abs(pr - wp) <= 1e-14
+        got = st.copy_out()
+    assert np.max(np.abs(got - want)) <= 1e-13

@@ -85,3 +85,35 @@ def test_qft_needs_few_exchanges():
         p = world.bit_length() - 1
         _, n_ex = simulate(n, world, W.qft(n), W.basis_state(n, 77))
         assert n_ex <= 2 * p + 1, (world, n_ex)
+
+
+@pytest.mark.parametrize("world", [2, 4, 8])
+def test_global_x_relabel(world):
+    """Uncontrolled X on a global qubit is a relabel (no exchange, no op); the flip is
+    materialised when the qubit comes back into the shard, and read through by
+    global controls and folded diagonals in between (NEXT-1 global-X relabeling)."""
+    n = 9
+    top = n - 1
+    psi = W.random_state(n, 21)
+    only_x = [W.Gate("X", (top,)), W.Gate("X", (top - 1 if world > 2 else top,))]
+    ops = L.lfqs_plan_circuit(n, world, 0, only_x, canonicalize=False)
+    assert ops == [], ops
+    # flips read by controls / diagonals on the flipped qubit, then materialised by H
+    gates = [W.Gate("X", (top,)), W.CNOT(top, 0), W.CZ(top, 3), W.Gate("T", (top,)),
+             W.Gate("X", (top,)), W.Gate("X", (top,)), W.TOFFOLI(top, 2, 5),
+             W.Gate("H", (top,)), W.Gate("X", (top,)), W.CNOT(1, top)]
+    got, _ = simulate(n, world, gates, psi)
+    assert np.array_equal(got, O.run_circuit(n, gates, psi.copy()))
+
+
+@pytest.mark.parametrize("world", [2, 4, 8])
+def test_grover_sharded(world):
+    n = 9
+    w = 0b101100111
+    gates = W.grover(n, w, 2)
+    got, n_ex = simulate(n, world, gates, W.basis_state(n, 0))
+    ref = O.run_circuit(n, gates, W.basis_state(n, 0))
+    assert np.max(np.abs(got - ref)) <= 1e-12
+    # H layers need the global qubits local; X layers are relabels
+    p = world.bit_length() - 1
+    assert n_ex <= 12 * p + 2 * p + 2, n_ex
