@@ -59,6 +59,9 @@ def main():
     ap.add_argument("--low", type=int, default=0)
     ap.add_argument("--reorder", type=int, default=1)
     ap.add_argument("--c64", action="store_true", help="complex64 state (NEXT-4)")
+    ap.add_argument("--world", type=int, default=1,
+                    help="virtual partition into this many shards (the sharded planner and "
+                         "exchange kernels on one GPU)")
     ap.add_argument("--tma", type=int, default=-1, help="max chunks moved by TMA (-1: default)")
     args = ap.parse_args()
     import torch
@@ -85,7 +88,9 @@ def main():
         "xhigh": ([W.Gate("X", (n - 1,)), W.Gate("X", (n - 5,))], lambda st: st.init_basis(0), {}),
     }
     ab = 8 if args.c64 else 16
-    with L.State.create(n, 0, stream=s, c64=args.c64) as st:
+    st_ = (L.State.create(n, 0, stream=s, c64=args.c64) if args.world == 1 else
+           L.State.virtual(n, args.world, 0, stream=s, c64=args.c64))
+    with st_ as st:
         if args.tile:
             st.set_option(L.OPT_FUSE_TILE_QUBITS, args.tile)
         if args.low:
@@ -101,6 +106,7 @@ def main():
                 times, passes = [], 0
                 for r in range(args.reps + 1):
                     init(st)
+                    x0 = st.exchange_stats()[0]
                     torch.cuda.synchronize()
                     c0 = st.launches()
                     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
@@ -111,13 +117,15 @@ def main():
                     if r > 0:
                         times.append(e0.elapsed_time(e1))
                     passes = st.launches() - c0
+                    x1 = st.exchange_stats()[0]
                 res = check(name, n, st, meta)
                 t = min(times)
                 rec = {"circuit": name, "mode": mode, "n": n, "gates": len(gates), "passes": passes,
                        "ms": t, "gates_per_s": len(gates) / (t / 1e3),
                        "conv_GBps": 2.0 * ab * 2 ** n * len(gates) / (t / 1e3) / 1e9,
                        "pass_GBps": 2.0 * ab * 2 ** n * passes / (t / 1e3) / 1e9,
-                       "dtype": "c64" if args.c64 else "c128"}
+                       "dtype": "c64" if args.c64 else "c128", "world": args.world,
+                       "exchanges": x1 - x0}
                 rec.update(res)
                 print(json.dumps(rec), flush=True)
 
