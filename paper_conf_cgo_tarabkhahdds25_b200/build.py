@@ -49,7 +49,7 @@ def build(force: bool = False, verbose: bool = False) -> str:
     os.makedirs(objdir, exist_ok=True)
     common = ["-O3", "-std=c++17", "-lineinfo", "-Xcompiler", "-fPIC", "-Xcompiler", "-Wall",
               "-I", os.path.join(ROOT, "include"), "-I", os.path.join(nd, "include")]
-    objs = []
+    objs, cmds = [], []
     for src in sources():
         obj = os.path.join(objdir, os.path.basename(src) + ".o")
         cmd = [NVCC] + ARCH + common + ["-Xptxas", "-warn-spills", "-c", src, "-o", obj]
@@ -57,8 +57,13 @@ def build(force: bool = False, verbose: bool = False) -> str:
             cmd = [NVCC] + ARCH + common + ["-x", "c++", "-c", src, "-o", obj]
         if verbose:
             print(" ".join(cmd), flush=True)
-        subprocess.check_call(cmd)
+        cmds.append(cmd)
         objs.append(obj)
+    # one nvcc per translation unit, in parallel (the kernel files dominate)
+    from concurrent.futures import ThreadPoolExecutor
+    with ThreadPoolExecutor(max_workers=min(len(cmds), os.cpu_count() or 1)) as ex:
+        for f in [ex.submit(subprocess.check_call, c) for c in cmds]:
+            f.result()
     tmp = LIB + f".tmp{os.getpid()}"
     link = [NVCC] + ARCH + ["-shared", "-cudart", "static", "-o", tmp] + objs + [
         "-L", os.path.join(nd, "lib"), "-l:libnccl.so.2",
