@@ -91,6 +91,14 @@ typedef struct {
 /* lfqs_run_circuit flags */
 #define LFQS_FUSE_NONE      0u  /* one pass per gate: every intermediate state exists */
 #define LFQS_FUSE_LOW       1u  /* shared-memory staging of consecutive low-qubit / diagonal gates */
+/* With LFQS_FUSE_LOW: inside a fused pass, runs of diagonal gates (which
+ * commute, P:441-445 classes) are merged into per-tile phase tables -- each
+ * table entry is the product of the run's factors for one pattern of <= 8 tile
+ * bits, built once per tile; every amplitude then takes one lookup and one
+ * complex multiply per table instead of one per gate.  The product is the same
+ * diagonal (Eq. 3), rounded in a different order, so diagonal
+ * results are then within rounding (<= 1e-12 abs), not value-exact. */
+#define LFQS_FUSE_PHASE     2u
 #define LFQS_FUSE_DEFAULT   LFQS_FUSE_LOW
 
 typedef struct lfqs_state lfqs_state;  /* opaque */
@@ -185,7 +193,9 @@ lfqs_status lfqs_apply_gate(lfqs_state* s, int kind, const int* targets, int n_t
 /* Applies gates[0..n_gates) in order.  flags: LFQS_FUSE_*.  With
  * LFQS_FUSE_NONE the result equals n_gates lfqs_apply_gate calls bit for bit;
  * with fusion, permutation/diagonal results are still value-exact and dense
- * results agree within rounding (<= 1e-12 abs per amplitude). */
+ * results agree within rounding (<= 1e-12 abs per amplitude); adding
+ * LFQS_FUSE_PHASE moves diagonal results into the rounding class too.
+ * Unknown flag bits: LFQS_ERR_INVALID_ARG. */
 lfqs_status lfqs_run_circuit(lfqs_state* s, const lfqs_gate* gates, size_t n_gates, uint32_t flags);
 
 /* ---- captured circuits (CUDA graphs) ----------------------------------------- */

@@ -28,6 +28,7 @@ NPARAMS.update({"RX": 1, "RY": 1, "RZ": 1, "PHASE": 1, "U3": 3})
 
 FUSE_NONE = 0
 FUSE_LOW = 1
+FUSE_PHASE = 2  # with FUSE_LOW: diagonal runs merged into per-tile phase tables (include/lfqs.h)
 OPT_LOWQ_SHUFFLE = 1
 OPT_FUSE_TILE_QUBITS = 2
 OPT_ITEMS_PER_THREAD = 3
@@ -346,6 +347,15 @@ def lfqs_circuit_compile(h: int, gates, flags: int = FUSE_NONE):
     return out.value, k.value
 
 
+def fuse_flags(fuse) -> int:
+    """fuse: False -> FUSE_NONE, True -> FUSE_LOW, "phase" -> FUSE_LOW | FUSE_PHASE, or an int."""
+    if fuse == "phase":
+        return FUSE_LOW | FUSE_PHASE
+    if isinstance(fuse, bool):
+        return FUSE_LOW if fuse else FUSE_NONE
+    return int(fuse)
+
+
 def lfqs_circuit_launch(c: int):
     _check(lib().lfqs_circuit_launch(c))
 
@@ -359,7 +369,7 @@ class Circuit:
 
     def __init__(self, state: "State", gates, fuse: bool = False):
         self.state = state  # keeps the state alive
-        self.h, self.kernels = lfqs_circuit_compile(state.h, gates, FUSE_LOW if fuse else FUSE_NONE)
+        self.h, self.kernels = lfqs_circuit_compile(state.h, gates, fuse_flags(fuse))
 
     def launch(self):
         lfqs_circuit_launch(self.h)
@@ -574,8 +584,10 @@ class State:
     def apply(self, g):
         lfqs_apply_gate(self.h, g.kind, g.targets, g.controls, g.params, g.matrix)
 
-    def run_circuit(self, gates, fuse: bool = False):
-        lfqs_run_circuit(self.h, gates, FUSE_LOW if fuse else FUSE_NONE)
+    def run_circuit(self, gates, fuse=False):
+        """fuse: False (one pass per gate), True (FUSE_LOW, exact for permutation/diagonal
+        gates) or "phase" (FUSE_LOW | FUSE_PHASE)."""
+        lfqs_run_circuit(self.h, gates, fuse_flags(fuse))
 
     def compile(self, gates, fuse: bool = False) -> Circuit:
         return Circuit(self, gates, fuse)

@@ -223,7 +223,7 @@ namespace {
 std::vector<Decoded> decode_circuit(const State* st, const lfqs_gate* gates, size_t n_gates,
                                     uint32_t flags) {
   require(n_gates == 0 || gates != nullptr, "gates is NULL");
-  require((flags & ~LFQS_FUSE_LOW) == 0, "unknown flags");
+  require((flags & ~(LFQS_FUSE_LOW | LFQS_FUSE_PHASE)) == 0, "unknown flags");
   std::vector<Decoded> dec;
   dec.reserve(n_gates);
   for (size_t i = 0; i < n_gates; ++i) {

@@ -43,8 +43,10 @@ namespace {
 // 1-target dense types are specialised by matrix values (static matrix
 // specialisation): F_UR real matrix (Ry), F_UI real diagonal with
 // imaginary off-diagonal (Rx) -- 4 FP ops per amplitude instead of 8.
+// F_DTAB (LFQS_FUSE_PHASE): a phase table over <= 8 tile bits standing for the
+// m diagonal ops that follow it (its members).
 enum FType : uint8_t {
-  F_DIAG1 = 0, F_DIAGN, F_X, F_Y, F_H, F_UR, F_UI, F_U2, F_SWAP, F_U4, F_U8
+  F_DIAG1 = 0, F_DIAGN, F_X, F_Y, F_H, F_UR, F_UI, F_U2, F_SWAP, F_U4, F_U8, F_DTAB
 };
 
 struct FHdr {       // 32 bytes
@@ -52,6 +54,8 @@ struct FHdr {       // 32 bytes
   uint16_t coef;    // offset into the coefficient pool
   uint32_t mlo, plo;  // per-amplitude predicate (i & mlo) == plo   (tile bits)
   uint64_t mhi, phi;  // per-tile predicate     (base & mhi) == phi (qubits outside the tile)
+  // F_DTAB: m = member count, mlo = table bits U (tile bits), plo = common
+  // predicate cm | cp << 16 (every member requires (i & cm) == cp); mhi = phi = 0.
 };
 constexpr int kMaxOps = 192;
 constexpr int kMaxCoef = 1580;
@@ -353,6 +357,26 @@ __device__ __forceinline__ void diag1_dispatch(C (&v)[R], const C d, uint32_t co
     if (((uint32_t)r & mr) == pr) v[r] = cmul_rn(d, v[r]);
 }
 
+// Factor of a DIAG1 / DIAGN op at tile element i of the tile at `base` (1 when
+// its predicate fails).  Used to build phase tables.
+template <class S>
+__device__ __forceinline__ cx<S> diag_factor(const FHdr& g, const double2* pc, uint64_t base,
+                                             uint32_t i) {
+  if ((base & g.mhi) != g.phi || (i & g.mlo) != g.plo) return mk<S>(1, 0);
+  const double2* c = pc + g.coef;
+  if (g.type == F_DIAG1) return cvs<S>(c[0]);
+  const int m = g.m;
+  const int ts[3] = {g.t0, g.t1, g.t2};
+  uint32_t j = 0;
+#pragma unroll
+  for (int s = 0; s < 3; ++s)
+    if (s < m) {
+      const uint32_t b = ts[s] >= 64 ? (uint32_t)((base >> (ts[s] - 64)) & 1) : (i >> ts[s]) & 1u;
+      j |= b << (m - 1 - s);
+    }
+  return cvs<S>(c[j]);
+}
+
 // Global amplitude index of tile element i (chunk = i >> lc, offset = low lc bits).
 __device__ __forceinline__ uint64_t tile_addr(const FTile& tg, uint64_t base, uint32_t i) {
   uint64_t off = base | (i & ((1u << tg.lc) - 1));
@@ -370,6 +394,7 @@ __global__ void __launch_bounds__(kFThreads, 2) k_fused(cx<S>* __restrict__ a,
   extern __shared__ __align__(128) unsigned char smem_raw[];
   C* tile = reinterpret_cast<C*>(smem_raw);
   __shared__ __align__(8) uint64_t bar;
+  __shared__ C dtab[256];  // phase table of the current F_DTAB op
   const uint32_t tid = threadIdx.x;
   const FTile& tg = prog.tile;
   const int lc = tg.lc, nh = tg.nh;
@@ -433,6 +458,61 @@ __global__ void __launch_bounds__(kFThreads, 2) k_fused(cx<S>* __restrict__ a,
     if ((base & h.mhi) != h.phi) continue;  // tile-level predicate (uniform)
     const int type = h.type;
     const uint32_t mlo = h.mlo, plo = h.plo;
+    if (type == F_DTAB) {  // LFQS_FUSE_PHASE: one lookup + multiply for the m member ops
+      const int nm = h.m;
+      const uint32_t U = mlo, cm = plo & 0xffffu, cp = plo >> 16;
+      const int nb = __popc(U);
+      __syncthreads();  // the previous table's readers (and tile writers) are done
+      if (tid < (1u << nb)) {
+        // Entry tid: tile pattern with tid's bits deposited at U's positions.
+        uint32_t ie = cp, u = U;
+        for (int b = 0; b < nb; ++b) {
+          const int pos = __ffs(u) - 1;
+          u &= u - 1;
+          ie |= ((tid >> b) & 1u) << pos;
+        }
+        C t = mk<S>(1, 0);
+        for (int j = 1; j <= nm; ++j) {
+          const C d = diag_factor<S>(prog.h[o + j], prog.c, base, ie);
+          if (!is_one(d)) t = cmul_rn(d, t);
+        }
+        dtab[tid] = t;
+      }
+      if (!in_regs) {
+#pragma unroll
+        for (int r = 0; r < R; ++r) v[r] = tile[r * kFThreads + tid];
+        in_regs = true;
+      }
+      __syncthreads();
+      if ((tid & cm & (kFThreads - 1)) == (cp & (kFThreads - 1))) {
+        // e(i) = pext(i, U): thread bits once, register bits as per-bit weights.
+        uint32_t et = 0, u = U & (kFThreads - 1);
+        for (int k = 0; u; ++k) {
+          const int pos = __ffs(u) - 1;
+          u &= u - 1;
+          et |= ((tid >> pos) & 1u) << k;
+        }
+        uint32_t w[4];
+        int k = __popc(U & (kFThreads - 1));
+#pragma unroll
+        for (int b = 0; b < 4; ++b) {
+          w[b] = (U >> (8 + b) & 1) ? 1u << k : 0u;
+          k += (U >> (8 + b)) & 1;
+        }
+        const uint32_t crm = cm >> 8, crp = cp >> 8;
+#pragma unroll
+        for (int r = 0; r < R; ++r) {
+          if (((uint32_t)r & crm) != crp) continue;
+          uint32_t e = et;
+#pragma unroll
+          for (int b = 0; b < 4; ++b)
+            if ((r >> b) & 1) e += w[b];
+          v[r] = cmul_rn(dtab[e], v[r]);
+        }
+      }
+      o += nm;
+      continue;
+    }
     if (type == F_DIAG1) {  // one diagonal entry d != 1 (the dominant op of phase-heavy programs)
       if (!in_regs) {
         __syncthreads();
@@ -717,6 +797,71 @@ uint64_t qubit_mask(const Decoded& g) {
   return m;
 }
 
+bool is_diag_op(const FHdr& h) { return h.type == F_DIAG1 || h.type == F_DIAGN; }
+
+// Tile bits an encoded diagonal op reads: its predicate bits and, for DIAGN,
+// its in-tile target bits.
+uint32_t diag_support(const FHdr& h) {
+  uint32_t u = h.mlo;
+  if (h.type == F_DIAGN) {
+    const int ts[3] = {h.t0, h.t1, h.t2};
+    for (int s = 0; s < h.m; ++s)
+      if (ts[s] < 64) u |= 1u << ts[s];
+  }
+  return u;
+}
+
+// LFQS_FUSE_PHASE: every maximal run of consecutive diagonal ops in the program
+// (diagonal matrices commute, so their product is order-free up to rounding) is
+// cut greedily, in program order, into groups whose table bits -- the union of
+// the members' tile bits minus the bits every member fixes to the same value
+// (the common predicate) -- number <= 8; a group of >= kMinTable members is
+// preceded by an F_DTAB header and evaluated as one table per tile.
+constexpr int kMinTable = 3;
+constexpr int kTableBits = 8;
+void merge_phase_runs(FProg& P) {
+  static thread_local FHdr out[kMaxOps];
+  int no = 0, o = 0;
+  const int n = P.nops;
+  int spare = kMaxOps - n;  // room for F_DTAB headers
+  while (o < n) {
+    if (!is_diag_op(P.h[o])) {
+      out[no++] = P.h[o++];
+      continue;
+    }
+    int e = o;
+    while (e < n && is_diag_op(P.h[e])) ++e;
+    for (int i = o; i < e;) {
+      uint32_t cm = P.h[i].mlo, cp = P.h[i].plo & cm, sup = diag_support(P.h[i]);
+      int j = i + 1;
+      for (; j < e && j - i < 255; ++j) {
+        const FHdr& g = P.h[j];
+        const uint32_t cm2 = cm & g.mlo & ~(cp ^ g.plo);
+        const uint32_t sup2 = sup | diag_support(g);
+        if (__builtin_popcount(sup2 & ~cm2) > kTableBits) break;
+        cm = cm2;
+        cp &= cm2;
+        sup = sup2;
+      }
+      if (j - i >= kMinTable && spare > 0) {
+        FHdr t;
+        std::memset(&t, 0, sizeof t);
+        t.type = F_DTAB;
+        t.m = (uint8_t)(j - i);
+        t.mlo = sup & ~cm;
+        t.plo = cm | (cp << 16);
+        out[no++] = t;
+        --spare;
+      }
+      for (int k = i; k < j; ++k) out[no++] = P.h[k];
+      i = j;
+    }
+    o = e;
+  }
+  std::memcpy(P.h, out, sizeof(FHdr) * no);
+  P.nops = no;
+}
+
 // Builds the tile geometry for qubit set in_tile (filled up to K qubits), merges
 // same-qubit 1-target runs containing a dense gate, encodes and launches.
 void launch_program(const LaunchCtx& ctx, const TileCfg& cfg, uint64_t in_tile,
@@ -773,6 +918,7 @@ void launch_program(const LaunchCtx& ctx, const TileCfg& cfg, uint64_t in_tile,
     prog.push_back(g);
   }
   for (const Decoded& g : prog) encode(g, tm, P);
+  if (ctx.phase_tables) merge_phase_runs(P);
   switch (K) {
     case 8: launch_k<8>(ctx, P); break;
     case 9: launch_k<9>(ctx, P); break;
@@ -798,12 +944,13 @@ bool run_fused_circuit(const LaunchCtx& ctx, const std::vector<Decoded>& gates, 
   if (!tile_cfg(ctx, tile_qubits, &cfg)) return false;
   uint64_t in_tile = (1ull << cfg.L) - 1;
   int used = 0, nops = 0, ncoef = 0;
+  const int max_ops = ctx.phase_tables ? kMaxOps - 16 : kMaxOps;  // room for F_DTAB headers
   std::vector<const Decoded*> list;
   size_t i = begin;
   for (; i < end; ++i) {
     const Decoded& g = gates[i];
     if (g.cls == GClass::NOOP) continue;
-    if (nops >= kMaxOps || ncoef + coef_count(g) > kMaxCoef) break;
+    if (nops >= max_ops || ncoef + coef_count(g) > kMaxCoef) break;
     const uint64_t need = tile_need(g, in_tile);
     const int nn = __builtin_popcountll(need);
     if (used + nn > cfg.slots) break;
@@ -836,10 +983,11 @@ void run_fused_schedule(const LaunchCtx& ctx, const std::vector<Decoded>& gates,
     return;
   }
   constexpr size_t kWindow = 4096;  // gates scanned per pass
+  const int max_ops = ctx.phase_tables ? kMaxOps - 16 : kMaxOps;  // room for F_DTAB headers
   std::vector<char> taken(gates.size(), 0);
   size_t head = 0;  // rest[0, head) are done
   while (head < rest.size()) {
-    uint64_t in_tile = (1ull << cfg.L) - 1, blocked_q = 0;
+    uint64_t in_tile = (1ull << cfg.L) - 1, blocked_q = 0, blocked_nd = 0;
     bool blocked_diag = false;
     int used = 0, nops = 0, ncoef = 0;
     std::vector<const Decoded*> list;
@@ -852,8 +1000,12 @@ void run_fused_schedule(const LaunchCtx& ctx, const std::vector<Decoded>& gates,
       const Decoded& g = gates[gi];
       const bool diag = g.cls == GClass::DIAG;
       const uint64_t qm = qubit_mask(g);
-      bool ok = (qm & blocked_q) == 0 && !(diag && blocked_diag);
-      if (ok && nops < kMaxOps && ncoef + coef_count(g) <= kMaxCoef) {
+      // Exact mode: a diagonal may not pass a skipped diagonal (rounding order of
+      // the phase products); LFQS_FUSE_PHASE: it may (tables round anyway), so
+      // only skipped non-diagonal gates block it.
+      bool ok = ctx.phase_tables && diag ? (qm & blocked_nd) == 0
+                                         : (qm & blocked_q) == 0 && !(diag && blocked_diag);
+      if (ok && nops < max_ops && ncoef + coef_count(g) <= kMaxCoef) {
         const uint64_t need = tile_need(g, in_tile);
         const int nn = __builtin_popcountll(need);
         if (used + nn <= cfg.slots) {
@@ -867,6 +1019,7 @@ void run_fused_schedule(const LaunchCtx& ctx, const std::vector<Decoded>& gates,
         }
       }
       blocked_q |= qm;  // later gates touching these qubits must wait
+      if (!diag) blocked_nd |= qm;
       blocked_diag |= diag;
     }
     if (nops < 2) {

@@ -100,6 +100,9 @@ struct LaunchCtx {
   uint64_t* launch_counter;
   const Options* opt;
   bool c64;                // amplitudes are complex64 (NEXT-4 precision variant)
+  // LFQS_FUSE_PHASE: runs of diagonal gates in a fused pass are merged into
+  // per-tile phase tables (one lookup + one multiply per amplitude per table).
+  bool phase_tables = false;
 };
 
 // Raises a kernel's dynamic shared memory limit once per device.

@@ -188,6 +188,7 @@ LaunchCtx State::ctx(int shard) {
   c.launch_counter = &launches;
   c.opt = &opt;
   c.c64 = c64;
+  c.phase_tables = phase_tables;
   return c;
 }
 
@@ -346,6 +347,11 @@ void State::apply(const Decoded& g) {
 void State::run(const std::vector<Decoded>& gates, uint32_t flags) {
   DeviceGuard dg(device);
   const bool fuse = (flags & LFQS_FUSE_LOW) != 0;
+  phase_tables = fuse && (flags & LFQS_FUSE_PHASE) != 0;
+  struct Reset {
+    bool& f;
+    ~Reset() { f = false; }
+  } reset{phase_tables};
   if (world == 1) {
     run_local(ctx(0), gates, fuse);
     return;

@@ -53,7 +53,8 @@ def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--n", type=int, default=30)
     ap.add_argument("--circuits", default="qft,ghz,grover,random,qpe,vqe,sycamore")
-    ap.add_argument("--modes", default="fused,unfused")
+    ap.add_argument("--modes", default="fused,phase,unfused",
+                    help="fused = FUSE_LOW (exact), phase = FUSE_LOW|FUSE_PHASE, unfused")
     ap.add_argument("--reps", type=int, default=2)
     ap.add_argument("--tile", type=int, default=0)
     ap.add_argument("--low", type=int, default=0)
@@ -102,7 +103,8 @@ def main():
             gates, init, meta = circuits[name]
             arr = L.marshal_gates(gates)
             for mode in args.modes.split(","):
-                flags = L.FUSE_LOW if mode == "fused" else L.FUSE_NONE
+                flags = {"fused": L.FUSE_LOW, "phase": L.FUSE_LOW | L.FUSE_PHASE,
+                         "unfused": L.FUSE_NONE}[mode]
                 times, passes = [], 0
                 for r in range(args.reps + 1):
                     init(st)
@@ -114,7 +116,7 @@ def main():
                     L.lfqs_run_circuit(st.h, arr, flags)
                     e1.record(s)
                     torch.cuda.synchronize()
-                    if r > 0:
+                    if r > 0 or args.reps == 0:
                         times.append(e0.elapsed_time(e1))
                     passes = st.launches() - c0
                     x1 = st.exchange_stats()[0]
