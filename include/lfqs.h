@@ -99,6 +99,15 @@ typedef struct {
  * diagonal (Eq. 3), rounded in a different order, so diagonal
  * results are then within rounding (<= 1e-12 abs), not value-exact. */
 #define LFQS_FUSE_PHASE     2u
+/* With LFQS_FUSE_LOW: every fused pass is compiled into its own kernel (the
+ * pass's gate program emitted as PTX with indices, predicates and op types
+ * resolved, coefficients left as a kernel parameter; compiled in-process,
+ * in parallel, and cached by structure) instead of being interpreted per tile
+ * -- the paper's compile-the-circuit approach applied to
+ * fused passes.  Results are bit-identical to the interpreted passes; the
+ * first run of a new circuit structure pays the compile time (~0.1-1 s per
+ * pass, on all host cores).  Compile failure: LFQS_ERR_CUDA. */
+#define LFQS_FUSE_JIT       4u
 #define LFQS_FUSE_DEFAULT   LFQS_FUSE_LOW
 
 typedef struct lfqs_state lfqs_state;  /* opaque */
@@ -266,6 +275,15 @@ typedef struct {
 lfqs_status lfqs_plan_circuit(int n_qubits, int world, int rank, const lfqs_gate* gates,
                               size_t n_gates, int canonicalize, lfqs_plan_op* ops,
                               size_t capacity, size_t* n_ops);
+
+/* Ahead-of-time compile for LFQS_FUSE_JIT (host only, no device needed): plans the
+ * fused passes lfqs_run_circuit(s, gates, n_gates, flags) would run on a
+ * single-GPU n_qubits state (complex64 if c64 != 0, default tile options) and
+ * compiles every pass not yet in the process-wide cache, in parallel.
+ * *n_passes (may be NULL) receives the number of passes of the plan.
+ * flags must contain LFQS_FUSE_LOW | LFQS_FUSE_JIT. */
+lfqs_status lfqs_jit_precompile(int n_qubits, int c64, const lfqs_gate* gates, size_t n_gates,
+                                uint32_t flags, uint64_t* n_passes);
 
 /* ---- misc ------------------------------------------------------------------- */
 lfqs_status lfqs_synchronize(lfqs_state* s);

@@ -29,6 +29,7 @@ NPARAMS.update({"RX": 1, "RY": 1, "RZ": 1, "PHASE": 1, "U3": 3})
 FUSE_NONE = 0
 FUSE_LOW = 1
 FUSE_PHASE = 2  # with FUSE_LOW: diagonal runs merged into per-tile phase tables (include/lfqs.h)
+FUSE_JIT = 4  # with FUSE_LOW: each fused pass compiled into its own kernel (include/lfqs.h)
 OPT_LOWQ_SHUFFLE = 1
 OPT_FUSE_TILE_QUBITS = 2
 OPT_ITEMS_PER_THREAD = 3
@@ -50,7 +51,7 @@ EXPORTS = [
     "lfqs_state_create_ex", "lfqs_state_wrap_ex", "lfqs_copy_in_c64", "lfqs_copy_out_c64",
     "lfqs_circuit_compile", "lfqs_circuit_launch", "lfqs_circuit_destroy",
     "lfqs_state_create_p2p", "lfqs_state_p2p_handle", "lfqs_state_p2p_attach",
-    "lfqs_state_exchange_stats",
+    "lfqs_state_exchange_stats", "lfqs_jit_precompile",
 ]
 P2P_HANDLE_BYTES = 256
 STATE_C64 = 1
@@ -135,6 +136,8 @@ def lib():
             "lfqs_plan_circuit": [C.c_int, C.c_int, C.c_int, C.POINTER(LfqsGate), C.c_size_t,
                                   C.c_int, C.POINTER(LfqsPlanOp), C.c_size_t,
                                   C.POINTER(C.c_size_t)],
+            "lfqs_jit_precompile": [C.c_int, C.c_int, C.POINTER(LfqsGate), C.c_size_t, C.c_uint32,
+                                    C.POINTER(u64)],
         }
         for name, args in sig.items():
             f = getattr(L, name)
@@ -348,12 +351,23 @@ def lfqs_circuit_compile(h: int, gates, flags: int = FUSE_NONE):
 
 
 def fuse_flags(fuse) -> int:
-    """fuse: False -> FUSE_NONE, True -> FUSE_LOW, "phase" -> FUSE_LOW | FUSE_PHASE, or an int."""
-    if fuse == "phase":
-        return FUSE_LOW | FUSE_PHASE
+    """fuse: False -> FUSE_NONE, True -> FUSE_LOW, "phase" -> FUSE_LOW | FUSE_PHASE,
+    "jit" -> FUSE_LOW | FUSE_JIT, "jit+phase" -> all three, or an int."""
+    if isinstance(fuse, str):
+        return {"phase": FUSE_LOW | FUSE_PHASE, "jit": FUSE_LOW | FUSE_JIT,
+                "jit+phase": FUSE_LOW | FUSE_JIT | FUSE_PHASE}[fuse]
     if isinstance(fuse, bool):
         return FUSE_LOW if fuse else FUSE_NONE
     return int(fuse)
+
+
+def lfqs_jit_precompile(n_qubits: int, gates, fuse="jit", c64: bool = False) -> int:
+    """Compiles the fused passes of `gates` for LFQS_FUSE_JIT ahead of time (host only,
+    no device needed); returns the number of passes of the plan."""
+    arr, n, keep = gates if (isinstance(gates, tuple) and len(gates) == 3) else marshal_gates(gates)
+    k = C.c_uint64()
+    _check(lib().lfqs_jit_precompile(n_qubits, int(c64), arr, n, fuse_flags(fuse), C.byref(k)))
+    return k.value
 
 
 def lfqs_circuit_launch(c: int):

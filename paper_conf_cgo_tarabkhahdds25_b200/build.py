@@ -18,6 +18,7 @@ ROOT = os.path.dirname(HERE)
 CSRC = os.path.join(HERE, "csrc")
 LIB = os.path.join(HERE, "liblfqs.so")
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
+CUDA = os.path.dirname(os.path.dirname(NVCC))
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 
 
@@ -67,6 +68,8 @@ def build(force: bool = False, verbose: bool = False) -> str:
     tmp = LIB + f".tmp{os.getpid()}"
     link = [NVCC] + ARCH + ["-shared", "-cudart", "static", "-o", tmp] + objs + [
         "-L", os.path.join(nd, "lib"), "-l:libnccl.so.2",
+        # in-process PTX compiler for the pass JIT (jit.cpp), linked statically
+        "-L", os.path.join(CUDA, "lib64"), "-lnvptxcompiler_static", "-lpthread",
         "-Xlinker", "-rpath=" + os.path.join(nd, "lib")]
     if verbose:
         print(" ".join(link), flush=True)

@@ -223,7 +223,7 @@ namespace {
 std::vector<Decoded> decode_circuit(const State* st, const lfqs_gate* gates, size_t n_gates,
                                     uint32_t flags) {
   require(n_gates == 0 || gates != nullptr, "gates is NULL");
-  require((flags & ~(LFQS_FUSE_LOW | LFQS_FUSE_PHASE)) == 0, "unknown flags");
+  require((flags & ~(LFQS_FUSE_LOW | LFQS_FUSE_PHASE | LFQS_FUSE_JIT)) == 0, "unknown flags");
   std::vector<Decoded> dec;
   dec.reserve(n_gates);
   for (size_t i = 0; i < n_gates; ++i) {
@@ -271,6 +271,39 @@ lfqs_status lfqs_circuit_launch(lfqs_circuit* c) {
 
 lfqs_status lfqs_circuit_destroy(lfqs_circuit* c) {
   return guarded([&] { delete static_cast<Graph*>(c); });
+}
+
+lfqs_status lfqs_jit_precompile(int n_qubits, int c64, const lfqs_gate* gates, size_t n_gates,
+                                uint32_t flags, uint64_t* n_passes) {
+  return guarded([&] {
+    require(n_gates == 0 || gates != nullptr, "gates is NULL");
+    require(n_qubits >= 1 && n_qubits <= 36, "n_qubits must be in [1, 36]");
+    require((flags & (LFQS_FUSE_LOW | LFQS_FUSE_JIT)) == (LFQS_FUSE_LOW | LFQS_FUSE_JIT) &&
+                (flags & ~(LFQS_FUSE_LOW | LFQS_FUSE_PHASE | LFQS_FUSE_JIT)) == 0,
+            "flags must be LFQS_FUSE_LOW | LFQS_FUSE_JIT [| LFQS_FUSE_PHASE]");
+    std::vector<Decoded> dec;
+    for (size_t i = 0; i < n_gates; ++i) {
+      const lfqs_gate& G = gates[i];
+      require(G.n_controls == __builtin_popcountll(G.control_mask),
+              "gate " + std::to_string(i) + ": n_controls != popcount(control_mask)");
+      dec.push_back(decode_gate(n_qubits, G.kind, G.targets, G.n_targets, G.control_mask,
+                                G.params, kind_nparams(G.kind), G.matrix));
+    }
+    Options opt;
+    uint64_t count = 0;
+    LaunchCtx c;
+    c.amps = nullptr;
+    c.n_local = n_qubits;
+    c.stream = nullptr;
+    c.launch_counter = &count;
+    c.opt = &opt;
+    c.c64 = c64 != 0;
+    c.phase_tables = (flags & LFQS_FUSE_PHASE) != 0;
+    c.jit = true;
+    c.dry_run = true;
+    run_fused_schedule(c, dec, opt.fuse_tile_qubits);
+    if (n_passes) *n_passes = count;
+  });
 }
 
 lfqs_status lfqs_plan_circuit(int n_qubits, int world, int rank, const lfqs_gate* gates,

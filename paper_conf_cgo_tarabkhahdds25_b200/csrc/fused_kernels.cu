@@ -31,54 +31,19 @@
 #include <cuda_runtime.h>
 
 #include <cstring>
+#include <memory>
+#include <string>
 #include <vector>
 
 #include "cx.cuh"
+#include "fused_prog.h"
+#include "jit.h"
 #include "lfqs_internal.h"
 
 namespace lfqs {
 
 namespace {
 
-// 1-target dense types are specialised by matrix values (static matrix
-// specialisation): F_UR real matrix (Ry), F_UI real diagonal with
-// imaginary off-diagonal (Rx) -- 4 FP ops per amplitude instead of 8.
-// F_DTAB (LFQS_FUSE_PHASE): a phase table over <= 8 tile bits standing for the
-// m diagonal ops that follow it (its members).
-enum FType : uint8_t {
-  F_DIAG1 = 0, F_DIAGN, F_X, F_Y, F_H, F_UR, F_UI, F_U2, F_SWAP, F_U4, F_U8, F_DTAB
-};
-
-struct FHdr {       // 32 bytes
-  uint8_t type, m, t0, t1, t2, pad0;
-  uint16_t coef;    // offset into the coefficient pool
-  uint32_t mlo, plo;  // per-amplitude predicate (i & mlo) == plo   (tile bits)
-  uint64_t mhi, phi;  // per-tile predicate     (base & mhi) == phi (qubits outside the tile)
-  // F_DTAB: m = member count, mlo = table bits U (tile bits), plo = common
-  // predicate cm | cp << 16 (every member requires (i & cm) == cp); mhi = phi = 0.
-};
-constexpr int kMaxOps = 192;
-constexpr int kMaxCoef = 1580;
-constexpr int kMaxHigh = 8;
-// Tile geometry: tile bits [0, lc) are qubits [0, lc) (one contiguous chunk of
-// 2^lc amplitudes); tile bits lc + i are the "high" qubits hpos[i] (ascending).
-// The tile is 2^(K - lc) chunks, each moved by one TMA bulk copy.
-struct FTile {
-  int lc;
-  int nh;
-  uint8_t hpos[kMaxHigh];
-};
-struct FProg {
-  int nops;
-  int ncoef;
-  FTile tile;
-  FHdr h[kMaxOps];
-  double2 c[kMaxCoef];
-};
-static_assert(sizeof(FProg) + 8 <= 32764, "kernel parameter limit");
-
-constexpr int kFThreads = 256;
-constexpr int kMinK = 8, kMaxK = 12;
 
 __device__ __forceinline__ uint32_t smem_u32(const void* p) {
   return static_cast<uint32_t>(__cvta_generic_to_shared(p));
@@ -863,13 +828,12 @@ void merge_phase_runs(FProg& P) {
 }
 
 // Builds the tile geometry for qubit set in_tile (filled up to K qubits), merges
-// same-qubit 1-target runs containing a dense gate, encodes and launches.
-void launch_program(const LaunchCtx& ctx, const TileCfg& cfg, uint64_t in_tile,
-                    const std::vector<const Decoded*>& list) {
+// same-qubit 1-target runs containing a dense gate, and encodes the program.
+void build_program(const LaunchCtx& ctx, const TileCfg& cfg, uint64_t in_tile,
+                   const std::vector<const Decoded*>& list, FProg& P) {
   const int K = cfg.K;
   for (int q = 0; q < ctx.n_local && __builtin_popcountll(in_tile) < K; ++q) in_tile |= 1ull << q;
   TileMap tm;
-  static thread_local FProg P;  // ~32 KB, reused (copied into the launch)
   P.nops = 0;
   P.ncoef = 0;
   int b = 0, lc = 0;
@@ -919,6 +883,16 @@ void launch_program(const LaunchCtx& ctx, const TileCfg& cfg, uint64_t in_tile,
   }
   for (const Decoded& g : prog) encode(g, tm, P);
   if (ctx.phase_tables) merge_phase_runs(P);
+}
+
+// Launches an encoded pass: the compiled kernel of its program (LFQS_FUSE_JIT)
+// or the interpreting kernel k_fused<K>.
+void launch_built(const LaunchCtx& ctx, int K, const FProg& P, const std::string* ptx = nullptr) {
+  if (ctx.jit && (1 << P.tile.nh) <= ctx.opt->fuse_tma_max_chunks) {
+    jit_launch(ctx, P, K, ptx ? *ptx : jit_ptx(P, K, ctx.c64));
+    ++*ctx.launch_counter;
+    return;
+  }
   switch (K) {
     case 8: launch_k<8>(ctx, P); break;
     case 9: launch_k<9>(ctx, P); break;
@@ -928,6 +902,13 @@ void launch_program(const LaunchCtx& ctx, const TileCfg& cfg, uint64_t in_tile,
   }
   LFQS_CUDA_CHECK(cudaGetLastError());
   ++*ctx.launch_counter;
+}
+
+void launch_program(const LaunchCtx& ctx, const TileCfg& cfg, uint64_t in_tile,
+                    const std::vector<const Decoded*>& list) {
+  static thread_local FProg P;  // ~32 KB, reused (copied into the launch)
+  build_program(ctx, cfg, in_tile, list, P);
+  launch_built(ctx, cfg.K, P);
 }
 
 }  // namespace
@@ -982,6 +963,14 @@ void run_fused_schedule(const LaunchCtx& ctx, const std::vector<Decoded>& gates,
     for (int i : rest) launch_gate(ctx, gates[i]);
     return;
   }
+  // LFQS_FUSE_JIT: passes are planned first, compiled in parallel, then launched.
+  struct Pass {
+    int gate = -1;                 // single-gate pass (class kernel)
+    std::unique_ptr<FProg> prog;   // fused pass
+    std::string ptx;
+  };
+  std::vector<Pass> passes;
+  const bool collect = ctx.jit && (1 << (cfg.K - cfg.L)) <= ctx.opt->fuse_tma_max_chunks;
   constexpr size_t kWindow = 4096;  // gates scanned per pass
   const int max_ops = ctx.phase_tables ? kMaxOps - 16 : kMaxOps;  // room for F_DTAB headers
   std::vector<char> taken(gates.size(), 0);
@@ -1025,13 +1014,40 @@ void run_fused_schedule(const LaunchCtx& ctx, const std::vector<Decoded>& gates,
     if (nops < 2) {
       // Nothing to fuse with the first remaining gate: its class kernel.
       while (taken[rest[head]]) ++head;
-      launch_gate(ctx, gates[rest[head]]);
+      if (collect) {
+        passes.emplace_back();
+        passes.back().gate = rest[head];
+      } else {
+        launch_gate(ctx, gates[rest[head]]);
+      }
       taken[rest[head]] = 1;
     } else {
-      launch_program(ctx, cfg, in_tile, list);
+      if (collect) {
+        passes.emplace_back();
+        passes.back().prog.reset(new FProg);
+        build_program(ctx, cfg, in_tile, list, *passes.back().prog);
+        passes.back().ptx = jit_ptx(*passes.back().prog, cfg.K, ctx.c64);
+      } else {
+        launch_program(ctx, cfg, in_tile, list);
+      }
       for (int gi : picked) taken[gi] = 1;
     }
     while (head < rest.size() && taken[rest[head]]) ++head;
+  }
+  if (!collect) return;
+  std::vector<std::string> srcs;
+  for (const Pass& ps : passes)
+    if (ps.prog) srcs.push_back(ps.ptx);
+  jit_compile(srcs);
+  if (ctx.dry_run) {
+    *ctx.launch_counter += passes.size();
+    return;
+  }
+  for (const Pass& ps : passes) {
+    if (ps.prog)
+      launch_built(ctx, cfg.K, *ps.prog, &ps.ptx);
+    else
+      launch_gate(ctx, gates[ps.gate]);
   }
 }
 

@@ -1,0 +1,990 @@
+// jit.cpp -- pass compiler: each fused pass's gate program (fused_prog.h) is
+// compiled into its own straight-line sm_100a kernel (LFQS_FUSE_JIT).
+//
+// The paper synthesises a simulator by compiling the circuit: vector fusion,
+// loop unrolling and static matrix specialisation turn
+// every gate into code with its structure baked in.  The interpreting kernel
+// k_fused (fused_kernels.cu) re-decodes each op of a pass for every tile; on
+// B200 that decode (constant-bank header loads, predicate arithmetic, branch
+// trees) costs more issue slots than the FP64 math of phase-heavy passes
+// (ncu: ~65% of stall samples, profiles/r01_fused_jit.md).  Here the program
+// of a pass is emitted as PTX with every index, predicate, register selection
+// and op type resolved at generation time; only the coefficients stay a kernel
+// parameter (constant bank), so one compiled pass serves every angle set of
+// the same circuit structure.  PTX is compiled in-process by nvPTXCompiler
+// (no NVVM: compiling generated CUDA C++ through NVRTC took seconds per pass),
+// passes are compiled in parallel and cached by their PTX text, and loaded
+// with cudaLibraryLoadData.
+//
+// The emitted arithmetic replicates k_fused op by op (same formulas, same FMA
+// and rounding order, same tile/register transitions), so a JIT pass is
+// bit-identical to the interpreted pass (tests/test_gpu_jit.py).
+#include "jit.h"
+
+#include <nvPTXCompiler.h>
+
+#include <atomic>
+#include <cstdarg>
+#include <cstdio>
+#include <cstdlib>
+#include <cstring>
+#include <functional>
+#include <map>
+#include <memory>
+#include <mutex>
+#include <string>
+#include <thread>
+#include <unordered_map>
+#include <vector>
+
+namespace lfqs {
+
+namespace {
+
+// ---------------------------------------------------------------------------
+// PTX emitter
+// ---------------------------------------------------------------------------
+struct Gen {
+  const FProg& P;
+  const int K;
+  const bool c64;
+  const char* FT;       // "f64" | "f32"
+  int ES;               // bytes per amplitude
+  int R;                // amplitudes per thread
+  std::string body;
+  int nr = 0, nrd = 0, nf = 0, np = 0, nl = 0;
+  bool in_regs = true;
+
+  Gen(const FProg& p, int k, bool c) : P(p), K(k), c64(c) {
+    FT = c64 ? "f32" : "f64";
+    ES = c64 ? 8 : 16;
+    R = (1 << K) / kFThreads;
+  }
+
+  void e(const char* fmt, ...) {
+    char buf[512];
+    va_list ap;
+    va_start(ap, fmt);
+    vsnprintf(buf, sizeof buf, fmt, ap);
+    va_end(ap);
+    body += "  ";
+    body += buf;
+    body += "\n";
+  }
+  std::string r() { return "%r" + std::to_string(nr++); }
+  std::string rd() { return "%rd" + std::to_string(nrd++); }
+  std::string f() { return "%f" + std::to_string(nf++); }
+  std::string p() { return "%p" + std::to_string(np++); }
+  std::string L() { return "L" + std::to_string(nl++); }
+  void label(const std::string& l) { body += l + ":\n"; }
+
+  // Amplitude registers of slot r.
+  static std::string vx(int r) { return "%vx" + std::to_string(r); }
+  static std::string vy(int r) { return "%vy" + std::to_string(r); }
+
+  struct Cx {
+    std::string x, y;
+  };
+
+  // Coefficient j of the pool as amplitude-type registers (cvs<S>).
+  Cx coef(int j) {
+    Cx c{f(), f()};
+    if (!c64) {
+      e("ld.param.v2.f64 {%s, %s}, [pc+%d];", c.x.c_str(), c.y.c_str(), j * 16);
+    } else {
+      const std::string a = "%dd" + std::to_string(nrd), b = "%dd" + std::to_string(nrd + 1);
+      nrd += 2;
+      e("ld.param.v2.f64 {%s, %s}, [pc+%d];", a.c_str(), b.c_str(), j * 16);
+      e("cvt.rn.f32.f64 %s, %s;", c.x.c_str(), a.c_str());
+      e("cvt.rn.f32.f64 %s, %s;", c.y.c_str(), b.c_str());
+    }
+    return c;
+  }
+  std::string coef_re(int j) { return coef(j).x; }
+  std::string coef_im(int j) { return coef(j).y; }
+
+  std::string neg(const std::string& a) {
+    std::string t = f();
+    e("neg.%s %s, %s;", FT, t.c_str(), a.c_str());
+    return t;
+  }
+  std::string mul(const std::string& a, const std::string& b) {
+    std::string t = f();
+    e("mul.rn.%s %s, %s, %s;", FT, t.c_str(), a.c_str(), b.c_str());
+    return t;
+  }
+  std::string add(const std::string& a, const std::string& b) {
+    std::string t = f();
+    e("add.rn.%s %s, %s, %s;", FT, t.c_str(), a.c_str(), b.c_str());
+    return t;
+  }
+  std::string sub(const std::string& a, const std::string& b) {
+    std::string t = f();
+    e("sub.rn.%s %s, %s, %s;", FT, t.c_str(), a.c_str(), b.c_str());
+    return t;
+  }
+  std::string fma(const std::string& a, const std::string& b, const std::string& c) {
+    std::string t = f();
+    e("fma.rn.%s %s, %s, %s, %s;", FT, t.c_str(), a.c_str(), b.c_str(), c.c_str());
+    return t;
+  }
+  std::string zero() { return c64 ? "0f00000000" : "0d0000000000000000"; }
+  std::string sel(const std::string& a, const std::string& b, const std::string& pr) {
+    std::string t = f();
+    e("selp.%s %s, %s, %s, %s;", FT, t.c_str(), a.c_str(), b.c_str(), pr.c_str());
+    return t;
+  }
+  // cmul_rn(d, a) (cx.cuh): (dx ax - dy ay, dx ay + dy ax), RN, no FMA.
+  Cx cmul(const Cx& d, const Cx& a) {
+    const std::string t1 = mul(d.x, a.x), t2 = mul(d.y, a.y);
+    const std::string nx = sub(t1, t2);
+    const std::string t3 = mul(d.x, a.y), t4 = mul(d.y, a.x);
+    const std::string ny = add(t3, t4);
+    return {nx, ny};
+  }
+  // cfma(acc, m, v) with acc == (0, 0) when first.
+  void cfma(Cx& acc, const Cx& m, const Cx& nmy, const Cx& v, bool first) {
+    // nmy.x holds -m.y (precomputed)
+    acc.x = fma(m.x, v.x, first ? zero() : acc.x);
+    acc.x = fma(nmy.x, v.y, acc.x);
+    acc.y = fma(m.x, v.y, first ? zero() : acc.y);
+    acc.y = fma(m.y, v.x, acc.y);
+  }
+  void set(int r, const Cx& z) {
+    e("mov.%s %s, %s;", FT, vx(r).c_str(), z.x.c_str());
+    e("mov.%s %s, %s;", FT, vy(r).c_str(), z.y.c_str());
+  }
+
+  // ---- integer helpers -----------------------------------------------------
+  // Branch to `skip` unless (base & mhi) == phi.
+  void tile_pred(uint64_t mhi, uint64_t phi, const std::string& skip) {
+    if (mhi == 0) return;
+    const std::string t = rd(), q = p();
+    e("and.b64 %s, %%base, %llu;", t.c_str(), (unsigned long long)mhi);
+    e("setp.ne.b64 %s, %s, %llu;", q.c_str(), t.c_str(), (unsigned long long)phi);
+    e("@%s bra %s;", q.c_str(), skip.c_str());
+  }
+  // Predicate register: (tid & m) == pv  (m == 0: none -> "")
+  std::string thread_pred(uint32_t m, uint32_t pv) {
+    m &= kFThreads - 1;
+    pv &= kFThreads - 1;
+    if (m == 0) return "";
+    const std::string t = r(), q = p();
+    e("and.b32 %s, %%ltid, %u;", t.c_str(), m);
+    e("setp.eq.b32 %s, %s, %u;", q.c_str(), t.c_str(), pv);
+    return q;
+  }
+  void skip_unless(const std::string& q, const std::string& skip) {
+    if (!q.empty()) e("@!%s bra %s;", q.c_str(), skip.c_str());
+  }
+
+  // ---- tile <-> registers ----------------------------------------------------
+  void regs_to_tile() {
+    for (int r = 0; r < R; ++r)
+      e("st.shared.v2.%s [%%taddr+%d], {%s, %s};", FT, r * kFThreads * ES, vx(r).c_str(),
+        vy(r).c_str());
+  }
+  void tile_to_regs() {
+    for (int r = 0; r < R; ++r)
+      e("ld.shared.v2.%s {%s, %s}, [%%taddr+%d];", FT, vx(r).c_str(), vy(r).c_str(),
+        r * kFThreads * ES);
+  }
+  void sync() { e("bar.sync 0;"); }
+
+  // ---- 2x2 functor semantics (fused_kernels.cu FX_/FY_/FH_/FR_/FI_/FU_) -----
+  struct Op2 {
+    int type;
+    std::string s;                  // F_H
+    std::string m00, m01, m10, m11; // F_UR
+    std::string d0, e01, e10, d1;   // F_UI
+    Cx c0, c1, c2, c3, n0, n1, n2, n3;  // F_U2 (n*.x = -c*.y)
+  };
+  Op2 load_op2(const FHdr& h) {
+    Op2 o;
+    o.type = h.type;
+    const int c = h.coef;
+    switch (h.type) {
+      case F_H: o.s = coef_re(c); break;
+      case F_UR:
+        o.m00 = coef_re(c); o.m01 = coef_re(c + 1); o.m10 = coef_re(c + 2); o.m11 = coef_re(c + 3);
+        break;
+      case F_UI:
+        o.d0 = coef_re(c); o.e01 = coef_im(c + 1); o.e10 = coef_im(c + 2); o.d1 = coef_re(c + 3);
+        break;
+      case F_U2:
+        o.c0 = coef(c); o.c1 = coef(c + 1); o.c2 = coef(c + 2); o.c3 = coef(c + 3);
+        o.n0 = {neg(o.c0.y), ""}; o.n1 = {neg(o.c1.y), ""};
+        o.n2 = {neg(o.c2.y), ""}; o.n3 = {neg(o.c3.y), ""};
+        break;
+      default: break;
+    }
+    return o;
+  }
+  void pair(const Op2& o, Cx& a0, Cx& a1) {
+    const Cx x0 = a0, x1 = a1;
+    switch (o.type) {
+      case F_X: a0 = x1; a1 = x0; return;
+      case F_Y:
+        a0 = {x1.y, neg(x1.x)};
+        a1 = {neg(x0.y), x0.x};
+        return;
+      case F_H:
+        a0 = {mul(o.s, add(x0.x, x1.x)), mul(o.s, add(x0.y, x1.y))};
+        a1 = {mul(o.s, sub(x0.x, x1.x)), mul(o.s, sub(x0.y, x1.y))};
+        return;
+      case F_UR:
+        a0 = {fma(o.m01, x1.x, mul(o.m00, x0.x)), fma(o.m01, x1.y, mul(o.m00, x0.y))};
+        a1 = {fma(o.m11, x1.x, mul(o.m10, x0.x)), fma(o.m11, x1.y, mul(o.m10, x0.y))};
+        return;
+      case F_UI: {
+        const std::string ne01 = neg(o.e01), ne10 = neg(o.e10);
+        a0 = {fma(ne01, x1.y, mul(o.d0, x0.x)), fma(o.e01, x1.x, mul(o.d0, x0.y))};
+        a1 = {fma(o.d1, x1.x, mul(ne10, x0.y)), fma(o.d1, x1.y, mul(o.e10, x0.x))};
+        return;
+      }
+      default: {  // F_U2
+        Cx b0, b1;
+        cfma(b0, o.c0, o.n0, x0, true);
+        cfma(b0, o.c1, o.n1, x1, false);
+        cfma(b1, o.c2, o.n2, x0, true);
+        cfma(b1, o.c3, o.n3, x1, false);
+        a0 = b0;
+        a1 = b1;
+        return;
+      }
+    }
+  }
+  // Lane form: amplitude a, partner p, runtime bit predicate `bit` (bit == 1).
+  Cx lane(const Op2& o, const Cx& a, const Cx& pp, const std::string& bit) {
+    switch (o.type) {
+      case F_X: return pp;
+      case F_Y: {
+        // bit ? (-p.y, p.x) : (p.y, -p.x)
+        const std::string npy = neg(pp.y), npx = neg(pp.x);
+        return {sel(npy, pp.y, bit), sel(pp.x, npx, bit)};
+      }
+      case F_H: {
+        // bit ? s (p - a) : s (a + p)
+        const std::string sx = sel(sub(pp.x, a.x), add(a.x, pp.x), bit);
+        const std::string sy = sel(sub(pp.y, a.y), add(a.y, pp.y), bit);
+        return {mul(o.s, sx), mul(o.s, sy)};
+      }
+      case F_UR: {
+        // bit ? (fma(m11, a, m10 p)) : (fma(m01, p, m00 a))
+        const std::string k1 = sel(o.m11, o.m01, bit), k2 = sel(o.m10, o.m00, bit);
+        const std::string y1x = sel(a.x, pp.x, bit), y1y = sel(a.y, pp.y, bit);
+        const std::string y2x = sel(pp.x, a.x, bit), y2y = sel(pp.y, a.y, bit);
+        return {fma(k1, y1x, mul(k2, y2x)), fma(k1, y1y, mul(k2, y2y))};
+      }
+      case F_UI: {
+        // bit ? (fma(d1, a.x, -e10 p.y), fma(d1, a.y, e10 p.x))
+        //     : (fma(-e01, p.y, d0 a.x), fma(e01, p.x, d0 a.y))
+        const std::string ne01 = neg(o.e01), ne10 = neg(o.e10);
+        const std::string rk1 = sel(o.d1, ne01, bit), rk2 = sel(ne10, o.d0, bit);
+        const std::string ry1 = sel(a.x, pp.y, bit), ry2 = sel(pp.y, a.x, bit);
+        const std::string ik1 = sel(o.d1, o.e01, bit), ik2 = sel(o.e10, o.d0, bit);
+        const std::string iy1 = sel(a.y, pp.x, bit), iy2 = sel(pp.x, a.y, bit);
+        return {fma(rk1, ry1, mul(rk2, ry2)), fma(ik1, iy1, mul(ik2, iy2))};
+      }
+      default: {  // F_U2: bit ? c2 p + c3 a : c0 a + c1 p (accumulation order kept)
+        Cx m1{sel(o.c2.x, o.c0.x, bit), sel(o.c2.y, o.c0.y, bit)};
+        Cx n1{sel(o.n2.x, o.n0.x, bit), ""};
+        Cx m2{sel(o.c3.x, o.c1.x, bit), sel(o.c3.y, o.c1.y, bit)};
+        Cx n2{sel(o.n3.x, o.n1.x, bit), ""};
+        Cx v1{sel(pp.x, a.x, bit), sel(pp.y, a.y, bit)};
+        Cx v2{sel(a.x, pp.x, bit), sel(a.y, pp.y, bit)};
+        Cx acc;
+        cfma(acc, m1, n1, v1, true);
+        cfma(acc, m2, n2, v2, false);
+        return acc;
+      }
+    }
+  }
+
+  Cx shfl(const Cx& v, int t0) {
+    Cx o{f(), f()};
+    for (int c = 0; c < 2; ++c) {
+      const std::string& src = c ? v.y : v.x;
+      const std::string& dst = c ? o.y : o.x;
+      if (!c64) {
+        const std::string lo = r(), hi = r(), lo2 = r(), hi2 = r();
+        e("mov.b64 {%s, %s}, %s;", lo.c_str(), hi.c_str(), src.c_str());
+        e("shfl.sync.bfly.b32 %s, %s, %d, 31, -1;", lo2.c_str(), lo.c_str(), 1 << t0);
+        e("shfl.sync.bfly.b32 %s, %s, %d, 31, -1;", hi2.c_str(), hi.c_str(), 1 << t0);
+        e("mov.b64 %s, {%s, %s};", dst.c_str(), lo2.c_str(), hi2.c_str());
+      } else {
+        const std::string a = r(), b = r();
+        e("mov.b32 %s, %s;", a.c_str(), src.c_str());
+        e("shfl.sync.bfly.b32 %s, %s, %d, 31, -1;", b.c_str(), a.c_str(), 1 << t0);
+        e("mov.b32 %s, %s;", dst.c_str(), b.c_str());
+      }
+    }
+    return o;
+  }
+
+  // ---- ops -------------------------------------------------------------------
+  void op_diag1(const FHdr& h) {
+    const std::string end = L();
+    tile_pred(h.mhi, h.phi, end);
+    skip_unless(thread_pred(h.mlo, h.plo), end);
+    const uint32_t mr = h.mlo >> 8, pr = h.plo >> 8;
+    bool any = false;
+    for (int r = 0; r < R; ++r) any |= ((uint32_t)r & mr) == pr;
+    if (any) {
+      const Cx d = coef(h.coef);
+      for (int r = 0; r < R; ++r)
+        if (((uint32_t)r & mr) == pr) set(r, cmul(d, {vx(r), vy(r)}));
+    }
+    label(end);
+  }
+
+  void op_diagn(const FHdr& h) {
+    const std::string end = L();
+    tile_pred(h.mhi, h.phi, end);
+    skip_unless(thread_pred(h.mlo, h.plo), end);
+    const uint32_t mr = h.mlo >> 8, pr = h.plo >> 8;
+    const int m = h.m;
+    const int ts[3] = {h.t0, h.t1, h.t2};
+    std::vector<Cx> dd;
+    for (int j = 0; j < (1 << m); ++j) dd.push_back(coef(h.coef + j));
+    // Runtime bits of the entry index (thread bits, tile-base bits) as predicates;
+    // register bits are compile-time per slot.
+    std::vector<std::string> bitp(3);
+    for (int s = 0; s < m; ++s) {
+      const int t = ts[s];
+      if (t >= 64) {
+        const std::string a = rd();
+        bitp[s] = p();
+        e("and.b64 %s, %%base, %llu;", a.c_str(), 1ull << (t - 64));
+        e("setp.ne.b64 %s, %s, 0;", bitp[s].c_str(), a.c_str());
+      } else if (t < 8) {
+        const std::string a = r();
+        bitp[s] = p();
+        e("and.b32 %s, %%ltid, %u;", a.c_str(), 1u << t);
+        e("setp.ne.b32 %s, %s, 0;", bitp[s].c_str(), a.c_str());
+      }
+    }
+    // Per slot: entry j = runtime bits + compile-time register bits.
+    std::map<uint32_t, Cx> cache;  // compile-time part -> selected d
+    for (int r = 0; r < R; ++r) {
+      if (((uint32_t)r & mr) != pr) continue;
+      uint32_t jc = 0;
+      for (int s = 0; s < m; ++s)
+        if (ts[s] >= 8 && ts[s] < 64) jc |= (((uint32_t)r >> (ts[s] - 8)) & 1u) << (m - 1 - s);
+      auto it = cache.find(jc);
+      if (it == cache.end()) {
+        // Select among the entries consistent with jc by the runtime bits.
+        std::vector<Cx> cand;
+        std::vector<int> idx;
+        for (int j = 0; j < (1 << m); ++j) {
+          bool ok = true;
+          for (int s = 0; s < m; ++s)
+            if (ts[s] >= 8 && ts[s] < 64 && (((j >> (m - 1 - s)) & 1u) != ((jc >> (m - 1 - s)) & 1u)))
+              ok = false;
+          if (ok) idx.push_back(j);
+        }
+        // Reduce by runtime bits from the least significant index bit upward.
+        std::vector<Cx> lvl;
+        for (int j : idx) lvl.push_back(dd[j]);
+        std::vector<int> lj = idx;
+        for (int s = m - 1; s >= 0; --s) {
+          if (bitp[s].empty()) continue;
+          std::vector<Cx> nx;
+          std::vector<int> nj;
+          for (size_t a = 0; a < lvl.size(); ++a) {
+            if ((lj[a] >> (m - 1 - s)) & 1) continue;
+            size_t b = a + 1;
+            for (; b < lvl.size(); ++b)
+              if (lj[b] == (lj[a] | (1 << (m - 1 - s)))) break;
+            nx.push_back({sel(lvl[b].x, lvl[a].x, bitp[s]), sel(lvl[b].y, lvl[a].y, bitp[s])});
+            nj.push_back(lj[a]);
+          }
+          lvl = nx;
+          lj = nj;
+        }
+        it = cache.emplace(jc, lvl[0]).first;
+      }
+      const Cx d = it->second;
+      const Cx z = cmul(d, {vx(r), vy(r)});
+      if (m == 1) {
+        set(r, z);
+      } else {
+        // if (!is_one(d)) v = d v
+        const std::string q1 = p(), q2 = p();
+        e("setp.eq.%s %s, %s, %s;", FT, q1.c_str(), d.x.c_str(), c64 ? "0f3F800000" : "0d3FF0000000000000");
+        e("setp.eq.and.%s %s, %s, %s, %s;", FT, q2.c_str(), d.y.c_str(), zero().c_str(), q1.c_str());
+        e("selp.%s %s, %s, %s, %s;", FT, vx(r).c_str(), vx(r).c_str(), z.x.c_str(), q2.c_str());
+        e("selp.%s %s, %s, %s, %s;", FT, vy(r).c_str(), vy(r).c_str(), z.y.c_str(), q2.c_str());
+      }
+    }
+    label(end);
+  }
+
+  void op_reg1q(const FHdr& h) {
+    const std::string end = L();
+    tile_pred(h.mhi, h.phi, end);
+    const Op2 o = load_op2(h);
+    const int t0 = h.t0;
+    const uint32_t mr = h.mlo >> 8, pr = h.plo >> 8;
+    const std::string bt = thread_pred(h.mlo, h.plo);
+    if (t0 >= 8) {
+      const int rb = t0 - 8;
+      skip_unless(bt, end);
+      for (int r = 0; r < R; ++r) {
+        if ((r >> rb) & 1) continue;
+        if (((uint32_t)r & mr) != pr) continue;
+        Cx a0{vx(r), vy(r)}, a1{vx(r | (1 << rb)), vy(r | (1 << rb))};
+        pair(o, a0, a1);
+        set(r, a0);
+        set(r | (1 << rb), a1);
+      }
+    } else {
+      const std::string bit = p(), a = r();
+      e("and.b32 %s, %%ltid, %u;", a.c_str(), 1u << t0);
+      e("setp.ne.b32 %s, %s, 0;", bit.c_str(), a.c_str());
+      for (int r = 0; r < R; ++r) {
+        if (((uint32_t)r & mr) != pr) continue;
+        const Cx pp = shfl({vx(r), vy(r)}, t0);
+        const Cx z = lane(o, {vx(r), vy(r)}, pp, bit);
+        if (bt.empty()) {
+          set(r, z);
+        } else {
+          e("selp.%s %s, %s, %s, %s;", FT, vx(r).c_str(), z.x.c_str(), vx(r).c_str(), bt.c_str());
+          e("selp.%s %s, %s, %s, %s;", FT, vy(r).c_str(), z.y.c_str(), vy(r).c_str(), bt.c_str());
+        }
+      }
+    }
+    label(end);
+  }
+
+  // Index helpers for the shared-memory ops: ins0(p, t) on a runtime u32.
+  std::string ins0(const std::string& pv, int t) {
+    const std::string hi = r(), lo = r(), o = r();
+    e("shr.b32 %s, %s, %d;", hi.c_str(), pv.c_str(), t);
+    e("shl.b32 %s, %s, %d;", hi.c_str(), hi.c_str(), t + 1);
+    e("and.b32 %s, %s, %u;", lo.c_str(), pv.c_str(), (1u << t) - 1);
+    e("or.b32 %s, %s, %s;", o.c_str(), hi.c_str(), lo.c_str());
+    return o;
+  }
+  // Shared address of tile element i (runtime u32).
+  std::string saddr(const std::string& i) {
+    const std::string a = r();
+    e("mad.lo.u32 %s, %s, %d, %%tile;", a.c_str(), i.c_str(), ES);
+    return a;
+  }
+  Cx lds(const std::string& addr, int off = 0) {
+    Cx v{f(), f()};
+    e("ld.shared.v2.%s {%s, %s}, [%s+%d];", FT, v.x.c_str(), v.y.c_str(), addr.c_str(), off);
+    return v;
+  }
+  void sts(const std::string& addr, const Cx& v, int off = 0) {
+    e("st.shared.v2.%s [%s+%d], {%s, %s};", FT, addr.c_str(), off, v.x.c_str(), v.y.c_str());
+  }
+  // Loop body over p = pp * 256 + tid, pp < n; `fn(pvreg)` emits one item.
+  template <class F>
+  void for_items(int n, F fn) {
+    for (int pp = 0; pp < n; ++pp) {
+      const std::string pv = r();
+      e("add.u32 %s, %%ltid, %d;", pv.c_str(), pp * kFThreads);
+      fn(pv);
+    }
+  }
+  void pred_skip_i(const std::string& i, uint32_t mlo, uint32_t plo, const std::string& skip) {
+    if (mlo == 0) return;
+    const std::string t = r(), q = p();
+    e("and.b32 %s, %s, %u;", t.c_str(), i.c_str(), mlo);
+    e("setp.ne.b32 %s, %s, %u;", q.c_str(), t.c_str(), plo);
+    e("@%s bra %s;", q.c_str(), skip.c_str());
+  }
+
+  void op_smem(const FHdr& h) {
+    const std::string end = L();
+    tile_pred(h.mhi, h.phi, end);
+    const uint32_t T = 1u << K, mlo = h.mlo, plo = h.plo;
+    switch (h.type) {
+      case F_X: case F_Y: case F_H: case F_UR: case F_UI: case F_U2: {
+        const Op2 o = load_op2(h);
+        const int t = h.t0;
+        for_items((int)(T >> 1) / kFThreads, [&](const std::string& pv) {
+          const std::string nx = L();
+          const std::string i0 = ins0(pv, t);
+          pred_skip_i(i0, mlo, plo, nx);
+          const std::string a0a = saddr(i0);
+          Cx a0 = lds(a0a), a1 = lds(a0a, (1 << t) * ES);
+          pair(o, a0, a1);
+          sts(a0a, a0);
+          sts(a0a, a1, (1 << t) * ES);
+          label(nx);
+        });
+        break;
+      }
+      case F_SWAP: {
+        const int lo = h.t0 < h.t1 ? h.t0 : h.t1, hi = h.t0 < h.t1 ? h.t1 : h.t0;
+        for_items((int)(T >> 2) / kFThreads, [&](const std::string& pv) {
+          const std::string nx = L();
+          const std::string i = ins0(ins0(pv, lo), hi);
+          pred_skip_i(i, mlo, plo, nx);
+          const std::string ia = saddr(i);
+          const Cx x = lds(ia, (1 << lo) * ES), y = lds(ia, (1 << hi) * ES);
+          sts(ia, y, (1 << lo) * ES);
+          sts(ia, x, (1 << hi) * ES);
+          label(nx);
+        });
+        break;
+      }
+      case F_U4: case F_U8: {
+        const int Lm = h.type == F_U4 ? 4 : 8;
+        std::vector<Cx> c, nc;
+        for (int j = 0; j < Lm * Lm; ++j) {
+          c.push_back(coef(h.coef + j));
+          nc.push_back({neg(c.back().y), ""});
+        }
+        int offs[8];
+        int sorted[3];
+        if (Lm == 4) {
+          const int t0 = h.t0, t1 = h.t1;
+          sorted[0] = t0 < t1 ? t0 : t1;
+          sorted[1] = t0 < t1 ? t1 : t0;
+          offs[0] = 0; offs[1] = 1 << t1; offs[2] = 1 << t0; offs[3] = (1 << t0) | (1 << t1);
+        } else {
+          const int s0 = h.t0, s1 = h.t1, s2 = h.t2;
+          int a0 = s0 < s1 ? s0 : s1, a1 = s0 < s1 ? s1 : s0, a2 = s2;
+          if (a2 < a1) { const int x = a1; a1 = a2; a2 = x; }
+          if (a1 < a0) { const int x = a0; a0 = a1; a1 = x; }
+          sorted[0] = a0; sorted[1] = a1; sorted[2] = a2;
+          for (int j = 0; j < 8; ++j)
+            offs[j] = (((j >> 2) & 1) << s0) | (((j >> 1) & 1) << s1) | ((j & 1) << s2);
+        }
+        const int nb = Lm == 4 ? 2 : 3;
+        for_items((int)(T / Lm) / kFThreads, [&](const std::string& pv) {
+          const std::string nx = L();
+          std::string i = pv;
+          for (int b = 0; b < nb; ++b) i = ins0(i, sorted[b]);
+          pred_skip_i(i, mlo, plo, nx);
+          const std::string ia = saddr(i);
+          std::vector<Cx> v;
+          for (int j = 0; j < Lm; ++j) v.push_back(lds(ia, offs[j] * ES));
+          std::vector<Cx> w(Lm);
+          for (int j = 0; j < Lm; ++j)
+            for (int q = 0; q < Lm; ++q) cfma(w[j], c[j * Lm + q], nc[j * Lm + q], v[q], q == 0);
+          for (int j = 0; j < Lm; ++j) sts(ia, w[j], offs[j] * ES);
+          label(nx);
+        });
+        break;
+      }
+      default: break;
+    }
+    label(end);
+  }
+
+  // Factor of diagonal member g at entry pattern ie (u32 reg), multiplied into t
+  // when its predicate holds and it is not exactly one (k_fused F_DTAB build).
+  void dtab_member(const FHdr& g, const std::string& ie, Cx& t) {
+    const std::string skip = L();
+    tile_pred(g.mhi, g.phi, skip);
+    pred_skip_i(ie, g.mlo, g.plo, skip);
+    Cx d;
+    if (g.type == F_DIAG1) {
+      d = coef(g.coef);
+    } else {
+      const int m = g.m;
+      const int ts[3] = {g.t0, g.t1, g.t2};
+      // j from the bits of ie / base (all runtime here)
+      const std::string j = r();
+      e("mov.u32 %s, 0;", j.c_str());
+      for (int s = 0; s < m; ++s) {
+        const std::string b = r();
+        if (ts[s] >= 64) {
+          const std::string a = rd();
+          e("shr.b64 %s, %%base, %d;", a.c_str(), ts[s] - 64);
+          e("cvt.u32.u64 %s, %s;", b.c_str(), a.c_str());
+          e("and.b32 %s, %s, 1;", b.c_str(), b.c_str());
+        } else {
+          e("bfe.u32 %s, %s, %d, 1;", b.c_str(), ie.c_str(), ts[s]);
+        }
+        e("bfi.b32 %s, %s, %s, %d, 1;", j.c_str(), b.c_str(), j.c_str(), m - 1 - s);
+      }
+      // select entry j among 2^m
+      d = coef(g.coef);
+      for (int k = 1; k < (1 << m); ++k) {
+        const Cx ck = coef(g.coef + k);
+        const std::string q = p();
+        e("setp.eq.u32 %s, %s, %d;", q.c_str(), j.c_str(), k);
+        d = {sel(ck.x, d.x, q), sel(ck.y, d.y, q)};
+      }
+    }
+    const std::string q1 = p(), q2 = p();
+    e("setp.eq.%s %s, %s, %s;", FT, q1.c_str(), d.x.c_str(), c64 ? "0f3F800000" : "0d3FF0000000000000");
+    e("setp.eq.and.%s %s, %s, %s, %s;", FT, q2.c_str(), d.y.c_str(), zero().c_str(), q1.c_str());
+    e("@%s bra %s;", q2.c_str(), skip.c_str());
+    const Cx z = cmul(d, t);
+    e("mov.%s %s, %s;", FT, t.x.c_str(), z.x.c_str());
+    e("mov.%s %s, %s;", FT, t.y.c_str(), z.y.c_str());
+    label(skip);
+  }
+
+  void op_dtab(int o) {
+    const FHdr& h = P.h[o];
+    const int nm = h.m;
+    const uint32_t U = h.mlo, cm = h.plo & 0xffffu, cp = h.plo >> 16;
+    const int nb = __builtin_popcount(U);
+    sync();
+    {
+      const std::string skip = L(), q = p();
+      e("setp.ge.u32 %s, %%ltid, %u;", q.c_str(), 1u << nb);
+      e("@%s bra %s;", q.c_str(), skip.c_str());
+      const std::string ie = r();
+      e("mov.u32 %s, %u;", ie.c_str(), cp);
+      uint32_t u = U;
+      for (int b = 0; b < nb; ++b) {
+        const int pos = __builtin_ctz(u);
+        u &= u - 1;
+        const std::string t = r();
+        e("bfe.u32 %s, %%ltid, %d, 1;", t.c_str(), b);
+        e("bfi.b32 %s, %s, %s, %d, 1;", ie.c_str(), t.c_str(), ie.c_str(), pos);
+      }
+      Cx t{f(), f()};
+      e("mov.%s %s, %s;", FT, t.x.c_str(), c64 ? "0f3F800000" : "0d3FF0000000000000");
+      e("mov.%s %s, %s;", FT, t.y.c_str(), zero().c_str());
+      for (int j = 1; j <= nm; ++j) dtab_member(P.h[o + j], ie, t);
+      const std::string a = r();
+      e("mad.lo.u32 %s, %%ltid, %d, %%dtab;", a.c_str(), ES);
+      sts(a, t);
+      label(skip);
+    }
+    if (!in_regs) {
+      tile_to_regs();
+      in_regs = true;
+    }
+    sync();
+    const std::string end = L();
+    skip_unless(thread_pred(cm, cp), end);
+    // et = pext(tid, U & 255)
+    const std::string et = r();
+    e("mov.u32 %s, 0;", et.c_str());
+    uint32_t u = U & (kFThreads - 1);
+    for (int k = 0; u; ++k) {
+      const int pos = __builtin_ctz(u);
+      u &= u - 1;
+      const std::string t = r();
+      e("bfe.u32 %s, %%ltid, %d, 1;", t.c_str(), pos);
+      e("bfi.b32 %s, %s, %s, %d, 1;", et.c_str(), t.c_str(), et.c_str(), k);
+    }
+    uint32_t w[4];
+    int k = __builtin_popcount(U & (kFThreads - 1));
+    for (int b = 0; b < 4; ++b) {
+      w[b] = ((U >> (8 + b)) & 1) ? 1u << k : 0u;
+      k += (U >> (8 + b)) & 1;
+    }
+    const std::string ebase = r();
+    e("mad.lo.u32 %s, %s, %d, %%dtab;", ebase.c_str(), et.c_str(), ES);
+    const uint32_t crm = cm >> 8, crp = cp >> 8;
+    for (int r_ = 0; r_ < R; ++r_) {
+      if (((uint32_t)r_ & crm) != crp) continue;
+      uint32_t off = 0;
+      for (int b = 0; b < 4; ++b)
+        if ((r_ >> b) & 1) off += w[b];
+      const Cx d = lds(ebase, (int)off * ES);
+      set(r_, cmul(d, {vx(r_), vy(r_)}));
+    }
+    label(end);
+  }
+
+  // ---- whole kernel -------------------------------------------------------------
+  std::string build() {
+    const FTile& tg = P.tile;
+    const uint32_t T = 1u << K;
+    const uint32_t bytes = T * ES, chunk_bytes = (uint32_t)ES << tg.lc;
+    const int nch = 1 << tg.nh;
+    // prologue: base, TMA load
+    e("ld.param.u64 %%ga, [pa];");
+    e("cvta.to.global.u64 %%ga, %%ga;");
+    e("mov.u32 %%ltid, %%tid.x;");
+    e("mov.u32 %%bid, %%ctaid.x;");
+    e("cvt.u64.u32 %%base, %%bid;");
+    e("shl.b64 %%base, %%base, %d;", tg.lc);
+    for (int i = 0; i < tg.nh; ++i) {
+      const int pp = tg.hpos[i];
+      const std::string lo = rd();
+      e("and.b64 %s, %%base, %llu;", lo.c_str(), (unsigned long long)((1ull << pp) - 1));
+      e("sub.u64 %%base, %%base, %s;", lo.c_str());
+      e("shl.b64 %%base, %%base, 1;");
+      e("or.b64 %%base, %%base, %s;", lo.c_str());
+    }
+    e("mov.u32 %%tile, lfqs_tile;");
+    e("mov.u32 %%dtab, lfqs_dtab;");
+    e("mov.u32 %%bar, lfqs_bar;");
+    e("mad.lo.u32 %%taddr, %%ltid, %d, %%tile;", ES);
+    {
+      const std::string w0 = L(), q = p(), q0 = p();
+      e("setp.ge.u32 %s, %%ltid, 32;", q.c_str());
+      e("@%s bra %s;", q.c_str(), w0.c_str());
+      e("setp.eq.u32 %s, %%ltid, 0;", q0.c_str());
+      const std::string s0 = L();
+      e("@!%s bra %s;", q0.c_str(), s0.c_str());
+      e("mbarrier.init.shared::cta.b64 [%%bar], 1;");
+      e("fence.mbarrier_init.release.cluster;");
+      e("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%%bar], %u;", bytes);
+      label(s0);
+      e("bar.warp.sync -1;");
+      chunk_loop(nch, chunk_bytes, true);
+      label(w0);
+    }
+    sync();
+    {
+      const std::string wt = L(), q = p();
+      label(wt);
+      e("mbarrier.try_wait.parity.shared::cta.b64 %s, [%%bar], 0;", q.c_str());
+      e("@!%s bra %s;", q.c_str(), wt.c_str());
+    }
+    tile_to_regs();
+    in_regs = true;
+    for (int o = 0; o < P.nops; ++o) {
+      const FHdr& h = P.h[o];
+      const int type = h.type;
+      if (type == F_DTAB) {
+        op_dtab(o);
+        o += h.m;
+        continue;
+      }
+      if (type == F_DIAG1) {
+        if (!in_regs) {
+          sync();
+          tile_to_regs();
+          in_regs = true;
+        }
+        op_diag1(h);
+        continue;
+      }
+      const int t0 = h.t0;
+      const bool regpath = type <= F_DIAGN || (type <= F_U2 && (t0 < 5 || t0 >= 8));
+      if (regpath && !in_regs) {
+        sync();
+        tile_to_regs();
+        in_regs = true;
+      } else if (!regpath && in_regs) {
+        regs_to_tile();
+        in_regs = false;
+        sync();
+      } else if (!regpath) {
+        sync();
+      }
+      if (!regpath) {
+        op_smem(h);
+      } else if (type == F_DIAGN) {
+        op_diagn(h);
+      } else {
+        op_reg1q(h);
+      }
+    }
+    if (in_regs) regs_to_tile();
+    e("fence.proxy.async.shared::cta;");
+    sync();
+    {
+      const std::string w0 = L(), q = p();
+      e("setp.ge.u32 %s, %%ltid, 32;", q.c_str());
+      e("@%s bra %s;", q.c_str(), w0.c_str());
+      chunk_loop(nch, chunk_bytes, false);
+      e("cp.async.bulk.commit_group;");
+      e("cp.async.bulk.wait_group.read 0;");
+      label(w0);
+    }
+    e("ret;");
+
+    std::string out;
+    out += ".version 8.7\n.target sm_100a\n.address_size 64\n\n";
+    out += ".extern .shared .align 128 .b8 lfqs_tile[];\n";
+    out += ".shared .align 8 .b64 lfqs_bar;\n";
+    out += ".shared .align 16 .b8 lfqs_dtab[" + std::to_string(256 * ES) + "];\n\n";
+    const int nc = P.ncoef > 0 ? P.ncoef : 1;
+    out += ".visible .entry lfqs_jit(.param .u64 pa, .param .align 16 .b8 pc[" +
+           std::to_string(nc * 16) + "])\n";
+    out += ".maxntid 256, 1, 1\n.minnctapersm 2\n{\n";
+    out += "  .reg .pred %p<" + std::to_string(np + 1) + ">;\n";
+    out += "  .reg .b32 %r<" + std::to_string(nr + 1) + ">;\n";
+    out += "  .reg .b64 %rd<" + std::to_string(nrd + 1) + ">;\n";
+    out += "  .reg .f64 %dd<" + std::to_string(nrd + 1) + ">;\n";
+    out += std::string("  .reg .") + FT + " %f<" + std::to_string(nf + 1) + ">;\n";
+    out += std::string("  .reg .") + FT + " %vx<" + std::to_string(R) + ">;\n";
+    out += std::string("  .reg .") + FT + " %vy<" + std::to_string(R) + ">;\n";
+    out += "  .reg .b64 %ga, %base;\n  .reg .b32 %ltid, %bid, %tile, %dtab, %bar, %taddr;\n";
+    out += body;
+    out += "}\n";
+    return out;
+  }
+
+  // Chunk copies by the lanes of warp 0: chunk ch = lane + 32 k.
+  void chunk_loop(int nch, uint32_t chunk_bytes, bool load) {
+    const FTile& tg = P.tile;
+    for (int k = 0; k * 32 < nch; ++k) {
+      const std::string skip = L();
+      const std::string ch = r();
+      e("add.u32 %s, %%ltid, %d;", ch.c_str(), 32 * k);
+      if (nch < 32 * (k + 1)) {
+        const std::string q = p();
+        e("setp.ge.u32 %s, %s, %d;", q.c_str(), ch.c_str(), nch);
+        e("@%s bra %s;", q.c_str(), skip.c_str());
+      }
+      // off = base | deposit(ch) at hpos
+      const std::string off = rd();
+      e("mov.b64 %s, %%base;", off.c_str());
+      for (int i = 0; i < tg.nh; ++i) {
+        const std::string b = r(), b64 = rd();
+        e("bfe.u32 %s, %s, %d, 1;", b.c_str(), ch.c_str(), i);
+        e("cvt.u64.u32 %s, %s;", b64.c_str(), b.c_str());
+        e("shl.b64 %s, %s, %d;", b64.c_str(), b64.c_str(), tg.hpos[i]);
+        e("or.b64 %s, %s, %s;", off.c_str(), off.c_str(), b64.c_str());
+      }
+      const std::string ga = rd(), sa = r();
+      e("mad.lo.u64 %s, %s, %d, %%ga;", ga.c_str(), off.c_str(), ES);
+      e("mad.lo.u32 %s, %s, %u, %%tile;", sa.c_str(), ch.c_str(), chunk_bytes);
+      if (load)
+        e("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%s], [%s], %u, [%%bar];",
+          sa.c_str(), ga.c_str(), chunk_bytes);
+      else
+        e("cp.async.bulk.global.shared::cta.bulk_group [%s], [%s], %u;", ga.c_str(), sa.c_str(),
+          chunk_bytes);
+      label(skip);
+    }
+  }
+};
+
+// ---------------------------------------------------------------------------
+// Compilation cache
+// ---------------------------------------------------------------------------
+struct Entry {
+  std::vector<char> cubin;
+  std::string error;
+  bool compiled = false;
+  cudaLibrary_t lib = nullptr;
+  cudaKernel_t kern = nullptr;
+  int smem_set = 0;
+};
+
+std::mutex g_mu;
+std::unordered_map<std::string, std::shared_ptr<Entry>> g_cache;
+
+void compile_entry(const std::string& ptx, Entry& en) {
+  nvPTXCompilerHandle h = nullptr;
+  if (nvPTXCompilerCreate(&h, ptx.size(), ptx.c_str()) != NVPTXCOMPILE_SUCCESS) {
+    en.error = "nvPTXCompilerCreate failed";
+    return;
+  }
+  const char* opts[] = {"--gpu-name=sm_100a", "-O3"};
+  const nvPTXCompileResult rc = nvPTXCompilerCompile(h, 2, opts);
+  if (rc != NVPTXCOMPILE_SUCCESS) {
+    size_t n = 0;
+    nvPTXCompilerGetErrorLogSize(h, &n);
+    std::string log(n, '\0');
+    if (n) nvPTXCompilerGetErrorLog(h, &log[0]);
+    en.error = "nvPTXCompiler: " + log.substr(0, 600);
+  } else {
+    size_t n = 0;
+    nvPTXCompilerGetCompiledProgramSize(h, &n);
+    en.cubin.resize(n);
+    nvPTXCompilerGetCompiledProgram(h, en.cubin.data());
+  }
+  nvPTXCompilerDestroy(&h);
+}
+
+}  // namespace
+
+std::string jit_ptx(const FProg& P, int K, bool c64) {
+  Gen g(P, K, c64);
+  return g.build();
+}
+
+void jit_compile(const std::vector<std::string>& ptxs) {
+  std::vector<std::pair<const std::string*, std::shared_ptr<Entry>>> todo;
+  {
+    std::lock_guard<std::mutex> lk(g_mu);
+    for (const std::string& s : ptxs) {
+      auto it = g_cache.find(s);
+      if (it != g_cache.end()) continue;
+      auto en = std::make_shared<Entry>();
+      g_cache.emplace(s, en);
+      todo.emplace_back(&s, en);
+    }
+  }
+  if (todo.empty()) return;
+  unsigned nt = std::thread::hardware_concurrency();
+  if (nt == 0) nt = 4;
+  if (nt > todo.size()) nt = (unsigned)todo.size();
+  std::atomic<size_t> next{0};
+  if (const char* dir = std::getenv("LFQS_JIT_DUMP")) {  // debugging aid
+    for (auto& t : todo) {
+      const std::string fn = std::string(dir) + "/pass_" +
+                             std::to_string(std::hash<std::string>()(*t.first)) + ".ptx";
+      if (FILE* fp = std::fopen(fn.c_str(), "w")) {
+        std::fwrite(t.first->data(), 1, t.first->size(), fp);
+        std::fclose(fp);
+      }
+    }
+  }
+  auto work = [&] {
+    for (size_t i; (i = next.fetch_add(1)) < todo.size();) {
+      compile_entry(*todo[i].first, *todo[i].second);
+      todo[i].second->compiled = true;
+    }
+  };
+  std::vector<std::thread> th;
+  for (unsigned t = 1; t < nt; ++t) th.emplace_back(work);
+  work();
+  for (auto& t : th) t.join();
+  for (auto& t : todo)
+    if (!t.second->error.empty()) {
+      const std::string err = t.second->error;
+      std::lock_guard<std::mutex> lk(g_mu);
+      g_cache.erase(*t.first);
+      throw Error(LFQS_ERR_CUDA, "JIT pass compile failed: " + err);
+    }
+}
+
+size_t jit_cache_size() {
+  std::lock_guard<std::mutex> lk(g_mu);
+  return g_cache.size();
+}
+
+void jit_launch(const LaunchCtx& ctx, const FProg& P, int K, const std::string& ptx) {
+  std::shared_ptr<Entry> en;
+  {
+    std::lock_guard<std::mutex> lk(g_mu);
+    auto it = g_cache.find(ptx);
+    if (it != g_cache.end()) en = it->second;
+  }
+  if (!en) {
+    jit_compile({ptx});
+    std::lock_guard<std::mutex> lk(g_mu);
+    en = g_cache.at(ptx);
+  }
+  const int es = ctx.c64 ? 8 : 16;
+  const int smem = es << K;
+  {
+    std::lock_guard<std::mutex> lk(g_mu);
+    if (en->lib == nullptr || en->smem_set < smem) {
+      // Module loading is not a stream operation: allowed while this thread
+      // captures a CUDA graph (lfqs_circuit_compile) under relaxed mode.
+      cudaStreamCaptureMode mode = cudaStreamCaptureModeRelaxed;
+      LFQS_CUDA_CHECK(cudaThreadExchangeStreamCaptureMode(&mode));
+      cudaError_t err = cudaSuccess;
+      if (en->lib == nullptr) {
+        err = cudaLibraryLoadData(&en->lib, en->cubin.data(), nullptr, nullptr, 0, nullptr,
+                                  nullptr, 0);
+        if (err == cudaSuccess) err = cudaLibraryGetKernel(&en->kern, en->lib, "lfqs_jit");
+      }
+      if (err == cudaSuccess)
+        err = cudaFuncSetAttribute((const void*)en->kern,
+                                   cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+      cudaThreadExchangeStreamCaptureMode(&mode);
+      LFQS_CUDA_CHECK(err);
+      en->smem_set = smem;
+    }
+  }
+  void* a = ctx.amps;
+  void* args[2] = {&a, (void*)P.c};
+  const uint64_t tiles = 1ull << (ctx.n_local - K);
+  LFQS_CUDA_CHECK(cudaLaunchKernel((const void*)en->kern, dim3((unsigned)tiles), dim3(kFThreads),
+                                   args, (size_t)smem, ctx.stream));
+}
+
+}  // namespace lfqs

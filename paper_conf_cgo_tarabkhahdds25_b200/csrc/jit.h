@@ -1,0 +1,19 @@
+// jit.h -- pass compiler for fused passes (LFQS_FUSE_JIT, jit.cpp).
+#pragma once
+#include <string>
+#include <vector>
+
+#include "fused_prog.h"
+#include "lfqs_internal.h"
+
+namespace lfqs {
+
+// PTX of one fused pass: structure baked in, coefficients a kernel parameter.
+std::string jit_ptx(const FProg& P, int K, bool c64);
+// Compiles (in parallel, nvPTXCompiler) every source not yet cached.
+void jit_compile(const std::vector<std::string>& ptxs);
+// Launches the pass (compiling it first if needed) on ctx.stream.
+void jit_launch(const LaunchCtx& ctx, const FProg& P, int K, const std::string& ptx);
+size_t jit_cache_size();
+
+}  // namespace lfqs

@@ -103,6 +103,10 @@ struct LaunchCtx {
   // LFQS_FUSE_PHASE: runs of diagonal gates in a fused pass are merged into
   // per-tile phase tables (one lookup + one multiply per amplitude per table).
   bool phase_tables = false;
+  // LFQS_FUSE_JIT: each fused pass runs as its own compiled kernel (jit.cpp).
+  bool jit = false;
+  // Plan and compile only (lfqs_jit_precompile): no kernel is launched.
+  bool dry_run = false;
 };
 
 // Raises a kernel's dynamic shared memory limit once per device.

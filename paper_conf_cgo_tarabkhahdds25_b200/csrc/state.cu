@@ -189,6 +189,7 @@ LaunchCtx State::ctx(int shard) {
   c.opt = &opt;
   c.c64 = c64;
   c.phase_tables = phase_tables;
+  c.jit = jit;
   return c;
 }
 
@@ -348,10 +349,12 @@ void State::run(const std::vector<Decoded>& gates, uint32_t flags) {
   DeviceGuard dg(device);
   const bool fuse = (flags & LFQS_FUSE_LOW) != 0;
   phase_tables = fuse && (flags & LFQS_FUSE_PHASE) != 0;
+  jit = fuse && (flags & LFQS_FUSE_JIT) != 0;
   struct Reset {
     bool& f;
-    ~Reset() { f = false; }
-  } reset{phase_tables};
+    bool& g;
+    ~Reset() { f = g = false; }
+  } reset{phase_tables, jit};
   if (world == 1) {
     run_local(ctx(0), gates, fuse);
     return;

@@ -80,6 +80,7 @@ struct State : lfqs_state {
   void common_init(int n_, int world_, int device_, cudaStream_t s, bool c64_ = false);
   LaunchCtx ctx(int shard);
   bool phase_tables = false;  // LFQS_FUSE_PHASE of the run in progress
+  bool jit = false;           // LFQS_FUSE_JIT of the run in progress
   int n_shards() const { return virt ? world : 1; }
   int rank_of_shard(int shard) const { return virt ? shard : rank; }
   void execute(const std::vector<PlanOp>& ops, bool fuse);

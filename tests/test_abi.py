@@ -63,3 +63,23 @@ def test_null_handle_is_rejected(lib):
         L.lfqs_synchronize(None)
     assert e.value.status == -1
     assert b"NULL" in lib.lfqs_last_error()
+
+
+def test_jit_precompile_host_only(lib):
+    """LFQS_FUSE_JIT: the pass compiler plans and compiles every fused pass on the
+    host (nvPTXCompiler, no device); a second call hits the cache."""
+    import time
+
+    import workloads as W
+    n = 16
+    gates = W.qft(n) + W.random_layered(n, 3, seed=1)
+    t0 = time.time()
+    k = L.lfqs_jit_precompile(n, gates, "jit")
+    t1 = time.time()
+    assert k >= 2
+    assert L.lfqs_jit_precompile(n, gates, "jit") == k
+    assert time.time() - t1 < max(0.5, t1 - t0)
+    assert L.lfqs_jit_precompile(n, gates, "jit+phase") >= 2
+    assert L.lfqs_jit_precompile(n, gates, "jit", c64=True) == k
+    with pytest.raises(L.LfqsError):
+        L.lfqs_jit_precompile(n, gates, True)  # FUSE_JIT missing

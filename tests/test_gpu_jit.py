@@ -1,0 +1,134 @@
+"""LFQS_FUSE_JIT: every fused pass compiled into its own kernel (csrc/jit.cpp).
+
+The pass compiler emits the interpreting kernel's arithmetic op by op (same
+formulas, FMA/rounding order and tile/register transitions), so a compiled pass
+must equal the interpreted pass BIT FOR BIT on every circuit, tile geometry and
+precision; against the oracle the usual bar holds (permutation/diagonal circuits
+exact, otherwise max abs error <= 1e-12, BASELINE.json north_star)."""
+import numpy as np
+import pytest
+
+import oracle as O
+import workloads as W
+from tests.test_gpu_phase import diag_heavy
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def L():
+    import torch
+    if not torch.cuda.is_available():
+        pytest.skip("needs a GPU")
+    import paper_conf_cgo_tarabkhahdds25_b200 as lib
+    lib.lib()
+    return lib
+
+
+def _run(L, n, psi, gates, fuse, tile=None, low=None, c64=False, reorder=1):
+    with L.State.create(n, c64=c64) as st:
+        st.set_option(L.OPT_FUSE_REORDER, reorder)
+        if tile:
+            st.set_option(L.OPT_FUSE_TILE_QUBITS, tile)
+        if low:
+            st.set_option(L.OPT_FUSE_LOW_QUBITS, low)
+        st.copy_in(psi)
+        c0 = st.launches()
+        st.run_circuit(gates, fuse=fuse)
+        return st.copy_out(), st.launches() - c0
+
+
+def _mixed(n, seed):
+    return (W.random_gate_list(n, 220, seed=seed, max_controls=2) + W.qft(n) +
+            W.random_layered(n, 4, seed=seed) + diag_heavy(n, 120, seed + 1))
+
+
+@pytest.mark.parametrize("reorder", [0, 1])
+@pytest.mark.parametrize("low", [5, 7])
+@pytest.mark.parametrize("tile", [8, 10, 12])
+@pytest.mark.parametrize("n", [13, 17])
+def test_jit_equals_interpreter(L, n, tile, low, reorder):
+    psi = W.random_state(n, 7 * n + tile + low)
+    gates = _mixed(n, 1000 + 13 * n + tile + low)
+    a, ka = _run(L, n, psi, gates, True, tile, low, reorder=reorder)
+    b, kb = _run(L, n, psi, gates, "jit", tile, low, reorder=reorder)
+    assert ka == kb
+    assert np.array_equal(a, b)
+    ref = O.run_circuit(n, gates, psi.copy())
+    assert np.max(np.abs(b - ref)) <= 1e-12
+
+
+@pytest.mark.parametrize("tile", [9, 12])
+def test_jit_phase_equals_interpreter_phase(L, tile):
+    n = 16
+    psi = W.random_state(n, 99)
+    gates = _mixed(n, 5) + W.qpe(n - 1, 0x2B3) + diag_heavy(n, 300, 17)
+    a, _ = _run(L, n, psi, gates, "phase", tile)
+    b, _ = _run(L, n, psi, gates, "jit+phase", tile)
+    assert np.array_equal(a, b)
+    assert np.max(np.abs(b - O.run_circuit(n, gates, psi.copy()))) <= 1e-12
+
+
+def test_jit_exact_classes_bit_exact_vs_oracle(L):
+    n = 15
+    psi = W.random_state(n, 3)
+    exact = [g for g in _mixed(n, 44) if g.exact]
+    got, _ = _run(L, n, psi, exact, "jit")
+    assert np.array_equal(got, O.run_circuit(n, exact, psi.copy()))
+
+
+def test_jit_c64(L):
+    n = 14
+    psi = W.random_state(n, 8).astype(np.complex64).astype(np.complex128)
+    gates = _mixed(n, 8)
+    a, _ = _run(L, n, psi, gates, True, c64=True)
+    b, _ = _run(L, n, psi, gates, "jit", c64=True)
+    assert np.array_equal(a, b)
+    assert np.max(np.abs(b - O.run_circuit(n, gates, psi.copy()))) <= 2e-5
+
+
+def test_jit_macro_closed_forms(L):
+    n = 20
+    x = 0xABCDE
+    with L.State.create(n) as st:
+        for fuse in ("jit", "jit+phase"):
+            st.init_basis(x)
+            st.run_circuit(W.qft(n), fuse=fuse)
+            a = st.copy_out()
+            y = np.arange(1 << n, dtype=np.int64)
+            ref = np.exp(2j * np.pi * ((x * y) % (1 << n)) / (1 << n)) / np.sqrt(1 << n)
+            assert np.max(np.abs(a - ref)) <= 1e-12
+            st.init_basis(0)
+            st.run_circuit(W.ghz(n), fuse=fuse)
+            g = st.copy_out()
+            assert g[0] == np.sqrt(0.5) and g[-1] == np.sqrt(0.5)
+            assert np.count_nonzero(g) == 2
+
+
+def test_jit_virtual_partition_and_graph(L):
+    """The sharded planner's fused local segments and captured circuits run the
+    compiled passes too."""
+    n = 14
+    psi = W.random_state(n, 12)
+    gates = _mixed(n, 21)
+    ref = O.run_circuit(n, gates, psi.copy())
+    for world in (2, 4):
+        with L.State.virtual(n, world) as st:
+            st.copy_in(psi)
+            st.run_circuit(gates, fuse="jit")
+            assert np.max(np.abs(st.copy_out() - ref)) <= 1e-12
+    with L.State.create(n) as st:
+        st.copy_in(psi)
+        with st.compile(gates, fuse="jit") as c:
+            c.launch()
+        assert np.max(np.abs(st.copy_out() - ref)) <= 1e-12
+
+
+def test_jit_precompile_then_run(L):
+    n = 18
+    gates = W.random_layered(n, 6, seed=2)
+    k = L.lfqs_jit_precompile(n, gates, "jit")
+    psi = W.random_state(n, 2)
+    got, passes = _run(L, n, psi, gates, "jit")
+    assert passes == k
+    assert np.max(np.abs(got - O.run_circuit(n, gates, psi.copy()))) <= 1e-12

@@ -53,8 +53,9 @@ def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--n", type=int, default=30)
     ap.add_argument("--circuits", default="qft,ghz,grover,random,qpe,vqe,sycamore")
-    ap.add_argument("--modes", default="fused,phase,unfused",
-                    help="fused = FUSE_LOW (exact), phase = FUSE_LOW|FUSE_PHASE, unfused")
+    ap.add_argument("--modes", default="fused,jit,jit+phase,unfused",
+                    help="fused = FUSE_LOW (exact), phase = FUSE_LOW|FUSE_PHASE, jit = "
+                         "FUSE_LOW|FUSE_JIT, jit+phase, unfused")
     ap.add_argument("--reps", type=int, default=2)
     ap.add_argument("--tile", type=int, default=0)
     ap.add_argument("--low", type=int, default=0)
@@ -104,7 +105,14 @@ def main():
             arr = L.marshal_gates(gates)
             for mode in args.modes.split(","):
                 flags = {"fused": L.FUSE_LOW, "phase": L.FUSE_LOW | L.FUSE_PHASE,
+                         "jit": L.FUSE_LOW | L.FUSE_JIT,
+                         "jit+phase": L.FUSE_LOW | L.FUSE_JIT | L.FUSE_PHASE,
                          "unfused": L.FUSE_NONE}[mode]
+                compile_s = None
+                if flags & L.FUSE_JIT:  # compile outside the timed region (reported)
+                    t0 = time.time()
+                    L.lfqs_jit_precompile(n, arr, flags, c64=args.c64)
+                    compile_s = time.time() - t0
                 times, passes = [], 0
                 for r in range(args.reps + 1):
                     init(st)
@@ -128,6 +136,8 @@ def main():
                        "pass_GBps": 2.0 * ab * 2 ** n * passes / (t / 1e3) / 1e9,
                        "dtype": "c64" if args.c64 else "c128", "world": args.world,
                        "exchanges": x1 - x0}
+                if compile_s is not None:
+                    rec["jit_compile_s"] = round(compile_s, 3)
                 rec.update(res)
                 print(json.dumps(rec), flush=True)
 
