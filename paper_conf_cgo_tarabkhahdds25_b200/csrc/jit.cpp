@@ -150,6 +150,12 @@ struct Gen {
     acc.y = fma(m.x, v.y, first ? zero() : acc.y);
     acc.y = fma(m.y, v.x, acc.y);
   }
+  Cx copy(const Cx& z) {
+    Cx c{f(), f()};
+    e("mov.%s %s, %s;", FT, c.x.c_str(), z.x.c_str());
+    e("mov.%s %s, %s;", FT, c.y.c_str(), z.y.c_str());
+    return c;
+  }
   void set(int r, const Cx& z) {
     e("mov.%s %s, %s;", FT, vx(r).c_str(), z.x.c_str());
     e("mov.%s %s, %s;", FT, vy(r).c_str(), z.y.c_str());
@@ -433,7 +439,8 @@ struct Gen {
       for (int r = 0; r < R; ++r) {
         if ((r >> rb) & 1) continue;
         if (((uint32_t)r & mr) != pr) continue;
-        Cx a0{vx(r), vy(r)}, a1{vx(r | (1 << rb)), vy(r | (1 << rb))};
+        // Snapshot the slot registers: pair() may return them swapped (X, Y).
+        Cx a0 = copy({vx(r), vy(r)}), a1 = copy({vx(r | (1 << rb)), vy(r | (1 << rb))});
         pair(o, a0, a1);
         set(r, a0);
         set(r | (1 << rb), a1);
