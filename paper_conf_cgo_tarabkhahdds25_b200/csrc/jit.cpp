@@ -487,13 +487,22 @@ struct Gen {
   void sts(const std::string& addr, const Cx& v, int off = 0) {
     e("st.shared.v2.%s [%s+%d], {%s, %s};", FT, addr.c_str(), off, v.x.c_str(), v.y.c_str());
   }
-  // Loop body over p = pp * 256 + tid, pp < n; `fn(pvreg)` emits one item.
+  // Items p = tid, tid + 256, ... < total (the interpreter's strided loop);
+  // `fn(pvreg)` emits one item.
   template <class F>
-  void for_items(int n, F fn) {
-    for (int pp = 0; pp < n; ++pp) {
+  void for_items(int total, F fn) {
+    for (int pp = 0; pp * kFThreads < total; ++pp) {
       const std::string pv = r();
       e("add.u32 %s, %%ltid, %d;", pv.c_str(), pp * kFThreads);
+      std::string skip;
+      if ((pp + 1) * kFThreads > total) {
+        skip = L();
+        const std::string q = p();
+        e("setp.ge.u32 %s, %s, %d;", q.c_str(), pv.c_str(), total);
+        e("@%s bra %s;", q.c_str(), skip.c_str());
+      }
       fn(pv);
+      if (!skip.empty()) label(skip);
     }
   }
   void pred_skip_i(const std::string& i, uint32_t mlo, uint32_t plo, const std::string& skip) {
@@ -512,7 +521,7 @@ struct Gen {
       case F_X: case F_Y: case F_H: case F_UR: case F_UI: case F_U2: {
         const Op2 o = load_op2(h);
         const int t = h.t0;
-        for_items((int)(T >> 1) / kFThreads, [&](const std::string& pv) {
+        for_items((int)(T >> 1), [&](const std::string& pv) {
           const std::string nx = L();
           const std::string i0 = ins0(pv, t);
           pred_skip_i(i0, mlo, plo, nx);
@@ -527,7 +536,7 @@ struct Gen {
       }
       case F_SWAP: {
         const int lo = h.t0 < h.t1 ? h.t0 : h.t1, hi = h.t0 < h.t1 ? h.t1 : h.t0;
-        for_items((int)(T >> 2) / kFThreads, [&](const std::string& pv) {
+        for_items((int)(T >> 2), [&](const std::string& pv) {
           const std::string nx = L();
           const std::string i = ins0(ins0(pv, lo), hi);
           pred_skip_i(i, mlo, plo, nx);
@@ -563,7 +572,7 @@ struct Gen {
             offs[j] = (((j >> 2) & 1) << s0) | (((j >> 1) & 1) << s1) | ((j & 1) << s2);
         }
         const int nb = Lm == 4 ? 2 : 3;
-        for_items((int)(T / Lm) / kFThreads, [&](const std::string& pv) {
+        for_items((int)(T / Lm), [&](const std::string& pv) {
           const std::string nx = L();
           std::string i = pv;
           for (int b = 0; b < nb; ++b) i = ins0(i, sorted[b]);
