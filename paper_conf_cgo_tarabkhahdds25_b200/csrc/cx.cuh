@@ -83,6 +83,15 @@ __device__ __forceinline__ float2 cmul_rn(float2 d, float2 a) {
 }
 __device__ __forceinline__ double fma_(double a, double b, double c) { return __fma_rn(a, b, c); }
 __device__ __forceinline__ float fma_(float a, float b, float c) { return __fmaf_rn(a, b, c); }
+// Complex multiply with FMA: (fma(dr, ar, -(di ai)), fma(dr, ai, di ar)) -- 4 FP ops.
+// Only for results in the rounding class (LFQS_FUSE_PHASE tables).
+template <class C>
+__device__ __forceinline__ C cmul_fma(C d, C a) {
+  C r;
+  r.x = fma_(d.x, a.x, -(d.y * a.y));
+  r.y = fma_(d.x, a.y, d.y * a.x);
+  return r;
+}
 // Accumulating multiply for dense gates (FMA allowed: tolerance class).
 template <class C>
 __device__ __forceinline__ void cfma(C& acc, C m, C v) {

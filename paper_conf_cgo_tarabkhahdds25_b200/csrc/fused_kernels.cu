@@ -439,7 +439,7 @@ __global__ void __launch_bounds__(kFThreads, 2) k_fused(cx<S>* __restrict__ a,
         C t = mk<S>(1, 0);
         for (int j = 1; j <= nm; ++j) {
           const C d = diag_factor<S>(prog.h[o + j], prog.c, base, ie);
-          if (!is_one(d)) t = cmul_rn(d, t);
+          if (!is_one(d)) t = cmul_fma(d, t);
         }
         dtab[tid] = t;
       }
@@ -472,7 +472,7 @@ __global__ void __launch_bounds__(kFThreads, 2) k_fused(cx<S>* __restrict__ a,
 #pragma unroll
           for (int b = 0; b < 4; ++b)
             if ((r >> b) & 1) e += w[b];
-          v[r] = cmul_rn(dtab[e], v[r]);
+          v[r] = cmul_fma(dtab[e], v[r]);
         }
       }
       o += nm;

@@ -82,13 +82,24 @@ struct Gen {
   static std::string vx(int r) { return "%vx" + std::to_string(r); }
   static std::string vy(int r) { return "%vy" + std::to_string(r); }
 
+  // A complex value in registers.  For program coefficients the value is known at
+  // generation time (kv): exact zeros / ones in it are specialised away (static
+  // matrix specialisation) -- value-identical to the interpreter,
+  // whose products with those exact constants are exact.
   struct Cx {
     std::string x, y;
+    bool kv = false;
+    double vx = 0, vy = 0;
+    bool zx() const { return kv && vx == 0.0; }
+    bool zy() const { return kv && vy == 0.0; }
   };
 
   // Coefficient j of the pool as amplitude-type registers (cvs<S>).
   Cx coef(int j) {
     Cx c{f(), f()};
+    c.kv = true;
+    c.vx = c64 ? (double)(float)P.c[j].x : P.c[j].x;
+    c.vy = c64 ? (double)(float)P.c[j].y : P.c[j].y;
     if (!c64) {
       e("ld.param.v2.f64 {%s, %s}, [pc+%d];", c.x.c_str(), c.y.c_str(), j * 16);
     } else {
@@ -136,6 +147,16 @@ struct Gen {
   }
   // cmul_rn(d, a) (cx.cuh): (dx ax - dy ay, dx ay + dy ax), RN, no FMA.
   Cx cmul(const Cx& d, const Cx& a) {
+    if (d.zy()) {  // real factor: (dx ax, dx ay); dx = +-1: copy / negate
+      if (d.vx == 1.0) return a;
+      if (d.vx == -1.0) return {neg(a.x), neg(a.y)};
+      return {mul(d.x, a.x), mul(d.x, a.y)};
+    }
+    if (d.zx()) {  // imaginary factor: (-(dy ay), dy ax)
+      if (d.vy == 1.0) return {neg(a.y), a.x};
+      if (d.vy == -1.0) return {a.y, neg(a.x)};
+      return {neg(mul(d.y, a.y)), mul(d.y, a.x)};
+    }
     const std::string t1 = mul(d.x, a.x), t2 = mul(d.y, a.y);
     const std::string nx = sub(t1, t2);
     const std::string t3 = mul(d.x, a.y), t4 = mul(d.y, a.x);
@@ -143,12 +164,42 @@ struct Gen {
     return {nx, ny};
   }
   // cfma(acc, m, v) with acc == (0, 0) when first.
+  // cmul_fma(d, a) (cx.cuh): (fma(dx, ax, -(dy ay)), fma(dx, ay, dy ax)) -- phase tables.
+  Cx cmulf(const Cx& d, const Cx& a) {
+    if (d.zy()) {
+      if (d.vx == 1.0) return a;
+      if (d.vx == -1.0) return {neg(a.x), neg(a.y)};
+      return {mul(d.x, a.x), mul(d.x, a.y)};
+    }
+    if (d.zx()) {
+      if (d.vy == 1.0) return {neg(a.y), a.x};
+      if (d.vy == -1.0) return {a.y, neg(a.x)};
+      return {neg(mul(d.y, a.y)), mul(d.y, a.x)};
+    }
+    return {fma(d.x, a.x, neg(mul(d.y, a.y))), fma(d.x, a.y, mul(d.y, a.x))};
+  }
+  // Terms with an exactly-zero coefficient part are skipped (fma(0, v, acc) == acc).
   void cfma(Cx& acc, const Cx& m, const Cx& nmy, const Cx& v, bool first) {
     // nmy.x holds -m.y (precomputed)
-    acc.x = fma(m.x, v.x, first ? zero() : acc.x);
-    acc.x = fma(nmy.x, v.y, acc.x);
-    acc.y = fma(m.x, v.y, first ? zero() : acc.y);
-    acc.y = fma(m.y, v.x, acc.y);
+    if (first) acc = Cx{zero(), zero()};
+    if (!m.zx()) acc.x = fma(m.x, v.x, acc.x);
+    if (!m.zy()) acc.x = fma(nmy.x, v.y, acc.x);
+    if (!m.zx()) acc.y = fma(m.x, v.y, acc.y);
+    if (!m.zy()) acc.y = fma(m.y, v.x, acc.y);
+  }
+  // selp of two known coefficients: known zero parts when both agree.
+  Cx sel_c(const Cx& a, const Cx& b, const std::string& bit) {
+    Cx o{sel(a.x, b.x, bit), sel(a.y, b.y, bit)};
+    if (a.kv && b.kv) {
+      if (a.vx == 0.0 && b.vx == 0.0) { o.kv = true; o.vx = 0.0; o.vy = 1.0; }
+      if (a.vy == 0.0 && b.vy == 0.0) {
+        if (!o.kv) { o.kv = true; o.vx = 1.0; }
+        o.vy = 0.0;
+      }
+      if (o.kv && o.vx != 0.0) o.vx = 2.0;  // nonzero, not a special value
+      if (o.kv && o.vy != 0.0) o.vy = 2.0;
+    }
+    return o;
   }
   Cx copy(const Cx& z) {
     Cx c{f(), f()};
@@ -156,10 +207,13 @@ struct Gen {
     e("mov.%s %s, %s;", FT, c.y.c_str(), z.y.c_str());
     return c;
   }
-  void set(int r, const Cx& z) {
-    e("mov.%s %s, %s;", FT, vx(r).c_str(), z.x.c_str());
-    e("mov.%s %s, %s;", FT, vy(r).c_str(), z.y.c_str());
+  // (dx, dy) = z; safe when z.y names dx (e.g. z = (-a.y, a.x) for a = (dx, dy)).
+  void assign(const std::string& dx, const std::string& dy, Cx z) {
+    if (z.y == dx) z.y = copy({z.y, z.y}).x;
+    if (z.x != dx) e("mov.%s %s, %s;", FT, dx.c_str(), z.x.c_str());
+    if (z.y != dy) e("mov.%s %s, %s;", FT, dy.c_str(), z.y.c_str());
   }
+  void set(int r, const Cx& z) { assign(vx(r), vy(r), z); }
 
   // ---- integer helpers -----------------------------------------------------
   // Branch to `skip` unless (base & mhi) == phi.
@@ -293,9 +347,9 @@ struct Gen {
         return {fma(rk1, ry1, mul(rk2, ry2)), fma(ik1, iy1, mul(ik2, iy2))};
       }
       default: {  // F_U2: bit ? c2 p + c3 a : c0 a + c1 p (accumulation order kept)
-        Cx m1{sel(o.c2.x, o.c0.x, bit), sel(o.c2.y, o.c0.y, bit)};
+        Cx m1 = sel_c(o.c2, o.c0, bit);
         Cx n1{sel(o.n2.x, o.n0.x, bit), ""};
-        Cx m2{sel(o.c3.x, o.c1.x, bit), sel(o.c3.y, o.c1.y, bit)};
+        Cx m2 = sel_c(o.c3, o.c1, bit);
         Cx n2{sel(o.n3.x, o.n1.x, bit), ""};
         Cx v1{sel(pp.x, a.x, bit), sel(pp.y, a.y, bit)};
         Cx v2{sel(a.x, pp.x, bit), sel(a.y, pp.y, bit)};
@@ -602,6 +656,9 @@ struct Gen {
     Cx d;
     if (g.type == F_DIAG1) {
       d = coef(g.coef);
+      if (!(d.vx == 1.0 && d.vy == 0.0)) assign(t.x, t.y, cmulf(d, t));  // is_one: compile time
+      label(skip);
+      return;
     } else {
       const int m = g.m;
       const int ts[3] = {g.t0, g.t1, g.t2};
@@ -633,9 +690,7 @@ struct Gen {
     e("setp.eq.%s %s, %s, %s;", FT, q1.c_str(), d.x.c_str(), c64 ? "0f3F800000" : "0d3FF0000000000000");
     e("setp.eq.and.%s %s, %s, %s, %s;", FT, q2.c_str(), d.y.c_str(), zero().c_str(), q1.c_str());
     e("@%s bra %s;", q2.c_str(), skip.c_str());
-    const Cx z = cmul(d, t);
-    e("mov.%s %s, %s;", FT, t.x.c_str(), z.x.c_str());
-    e("mov.%s %s, %s;", FT, t.y.c_str(), z.y.c_str());
+    assign(t.x, t.y, cmulf(d, t));
     label(skip);
   }
 
@@ -701,7 +756,7 @@ struct Gen {
       for (int b = 0; b < 4; ++b)
         if ((r_ >> b) & 1) off += w[b];
       const Cx d = lds(ebase, (int)off * ES);
-      set(r_, cmul(d, {vx(r_), vy(r_)}));
+      set(r_, cmulf(d, {vx(r_), vy(r_)}));
     }
     label(end);
   }
