@@ -55,10 +55,72 @@ struct Gen {
   int nr = 0, nrd = 0, nf = 0, np = 0, nl = 0;
   bool in_regs = true;
 
+  // Placement of tile bits in (thread, slot): tile bits 0..4 are the lane bits
+  // (fixed: warp accesses stay contiguous); the other K-5 tile bits sit at the 3
+  // warp positions (thread bits 5..7) or at the K-8 register positions (slot bits).
+  // The interpreter's placement is the identity; the compiled pass moves a tile bit
+  // into a register position (a tile round trip, `remap`) when a gate needs it
+  // there, so 1-target gates on warp bits and multi-target gates on register bits
+  // run in registers instead of as shared-memory ops.  Every amplitude still sees
+  // the same arithmetic, so results stay bit-identical to the interpreter.
+  int wpos[3] = {5, 6, 7};
+  int rpos[4] = {8, 9, 10, 11};
+  int nreg = 0;
+
   Gen(const FProg& p, int k, bool c) : P(p), K(k), c64(c) {
     FT = c64 ? "f32" : "f64";
     ES = c64 ? 8 : 16;
     R = (1 << K) / kFThreads;
+    nreg = K - 8;
+  }
+
+  int reg_of(int b) const {
+    for (int j = 0; j < nreg; ++j)
+      if (rpos[j] == b) return j;
+    return -1;
+  }
+  // Thread bit holding tile bit b, or -1 when b is register-held.
+  int tbit(int b) const {
+    if (b < 5) return b;
+    for (int j = 0; j < 3; ++j)
+      if (wpos[j] == b) return 5 + j;
+    return -1;
+  }
+  // (i & m) == v split into a thread part and a slot part.
+  void split(uint32_t m, uint32_t v, uint32_t& tm, uint32_t& tv, uint32_t& rm, uint32_t& rv) const {
+    tm = tv = rm = rv = 0;
+    for (int b = 0; b < K; ++b) {
+      if (!((m >> b) & 1)) continue;
+      const uint32_t bit = (v >> b) & 1;
+      const int t = tbit(b);
+      if (t >= 0) {
+        tm |= 1u << t;
+        tv |= bit << t;
+      } else {
+        const int j = reg_of(b);
+        rm |= 1u << j;
+        rv |= bit << j;
+      }
+    }
+  }
+  // Tile-index offset of slot r.
+  uint32_t roff(int r) const {
+    uint32_t o = 0;
+    for (int j = 0; j < nreg; ++j)
+      if ((r >> j) & 1) o |= 1u << rpos[j];
+    return o;
+  }
+  // %taddr = tile + ES * (thread part of the tile index).
+  void emit_taddr() {
+    const std::string t = r();
+    e("and.b32 %s, %%ltid, 31;", t.c_str());
+    for (int j = 0; j < 3; ++j) {
+      const std::string x = r();
+      e("bfe.u32 %s, %%ltid, %d, 1;", x.c_str(), 5 + j);
+      e("shl.b32 %s, %s, %d;", x.c_str(), x.c_str(), wpos[j]);
+      e("or.b32 %s, %s, %s;", t.c_str(), t.c_str(), x.c_str());
+    }
+    e("mad.lo.u32 %%taddr, %s, %d, %%tile;", t.c_str(), ES);
   }
 
   void e(const char* fmt, ...) {
@@ -226,8 +288,8 @@ struct Gen {
   }
   // Predicate register: (tid & m) == pv  (m == 0: none -> "")
   std::string thread_pred(uint32_t m, uint32_t pv) {
-    m &= kFThreads - 1;
-    pv &= kFThreads - 1;
+    uint32_t rm, rv;
+    split(m, pv, m, pv, rm, rv);
     if (m == 0) return "";
     const std::string t = r(), q = p();
     e("and.b32 %s, %%ltid, %u;", t.c_str(), m);
@@ -241,13 +303,13 @@ struct Gen {
   // ---- tile <-> registers ----------------------------------------------------
   void regs_to_tile() {
     for (int r = 0; r < R; ++r)
-      e("st.shared.v2.%s [%%taddr+%d], {%s, %s};", FT, r * kFThreads * ES, vx(r).c_str(),
+      e("st.shared.v2.%s [%%taddr+%u], {%s, %s};", FT, roff(r) * ES, vx(r).c_str(),
         vy(r).c_str());
   }
   void tile_to_regs() {
     for (int r = 0; r < R; ++r)
-      e("ld.shared.v2.%s {%s, %s}, [%%taddr+%d];", FT, vx(r).c_str(), vy(r).c_str(),
-        r * kFThreads * ES);
+      e("ld.shared.v2.%s {%s, %s}, [%%taddr+%u];", FT, vx(r).c_str(), vy(r).c_str(),
+        roff(r) * ES);
   }
   void sync() { e("bar.sync 0;"); }
 
@@ -387,7 +449,8 @@ struct Gen {
     const std::string end = L();
     tile_pred(h.mhi, h.phi, end);
     skip_unless(thread_pred(h.mlo, h.plo), end);
-    const uint32_t mr = h.mlo >> 8, pr = h.plo >> 8;
+    uint32_t tm_, tv_, mr, pr;
+    split(h.mlo, h.plo, tm_, tv_, mr, pr);
     bool any = false;
     for (int r = 0; r < R; ++r) any |= ((uint32_t)r & mr) == pr;
     if (any) {
@@ -402,7 +465,8 @@ struct Gen {
     const std::string end = L();
     tile_pred(h.mhi, h.phi, end);
     skip_unless(thread_pred(h.mlo, h.plo), end);
-    const uint32_t mr = h.mlo >> 8, pr = h.plo >> 8;
+    uint32_t tm_, tv_, mr, pr;
+    split(h.mlo, h.plo, tm_, tv_, mr, pr);
     const int m = h.m;
     const int ts[3] = {h.t0, h.t1, h.t2};
     std::vector<Cx> dd;
@@ -417,10 +481,10 @@ struct Gen {
         bitp[s] = p();
         e("and.b64 %s, %%base, %llu;", a.c_str(), 1ull << (t - 64));
         e("setp.ne.b64 %s, %s, 0;", bitp[s].c_str(), a.c_str());
-      } else if (t < 8) {
+      } else if (tbit(t) >= 0) {
         const std::string a = r();
         bitp[s] = p();
-        e("and.b32 %s, %%ltid, %u;", a.c_str(), 1u << t);
+        e("and.b32 %s, %%ltid, %u;", a.c_str(), 1u << tbit(t));
         e("setp.ne.b32 %s, %s, 0;", bitp[s].c_str(), a.c_str());
       }
     }
@@ -430,7 +494,8 @@ struct Gen {
       if (((uint32_t)r & mr) != pr) continue;
       uint32_t jc = 0;
       for (int s = 0; s < m; ++s)
-        if (ts[s] >= 8 && ts[s] < 64) jc |= (((uint32_t)r >> (ts[s] - 8)) & 1u) << (m - 1 - s);
+        if (ts[s] < 64 && tbit(ts[s]) < 0)
+          jc |= (((uint32_t)r >> reg_of(ts[s])) & 1u) << (m - 1 - s);
       auto it = cache.find(jc);
       if (it == cache.end()) {
         // Select among the entries consistent with jc by the runtime bits.
@@ -439,7 +504,8 @@ struct Gen {
         for (int j = 0; j < (1 << m); ++j) {
           bool ok = true;
           for (int s = 0; s < m; ++s)
-            if (ts[s] >= 8 && ts[s] < 64 && (((j >> (m - 1 - s)) & 1u) != ((jc >> (m - 1 - s)) & 1u)))
+            if (ts[s] < 64 && tbit(ts[s]) < 0 &&
+                (((j >> (m - 1 - s)) & 1u) != ((jc >> (m - 1 - s)) & 1u)))
               ok = false;
           if (ok) idx.push_back(j);
         }
@@ -485,10 +551,11 @@ struct Gen {
     tile_pred(h.mhi, h.phi, end);
     const Op2 o = load_op2(h);
     const int t0 = h.t0;
-    const uint32_t mr = h.mlo >> 8, pr = h.plo >> 8;
+    uint32_t tm_, tv_, mr, pr;
+    split(h.mlo, h.plo, tm_, tv_, mr, pr);
     const std::string bt = thread_pred(h.mlo, h.plo);
-    if (t0 >= 8) {
-      const int rb = t0 - 8;
+    if (t0 >= 5) {  // register-held (remapped there if it was a warp bit)
+      const int rb = reg_of(t0);
       skip_unless(bt, end);
       for (int r = 0; r < R; ++r) {
         if ((r >> rb) & 1) continue;
@@ -730,33 +797,146 @@ struct Gen {
     sync();
     const std::string end = L();
     skip_unless(thread_pred(cm, cp), end);
-    // et = pext(tid, U & 255)
+    // e(i) = pext(i, U): table-index bit k is tile bit u_k, held by a thread bit
+    // (runtime, et) or a slot bit (compile time, w[j]).
     const std::string et = r();
     e("mov.u32 %s, 0;", et.c_str());
-    uint32_t u = U & (kFThreads - 1);
+    uint32_t w[4] = {0, 0, 0, 0};
+    uint32_t u = U;
     for (int k = 0; u; ++k) {
       const int pos = __builtin_ctz(u);
       u &= u - 1;
-      const std::string t = r();
-      e("bfe.u32 %s, %%ltid, %d, 1;", t.c_str(), pos);
-      e("bfi.b32 %s, %s, %s, %d, 1;", et.c_str(), t.c_str(), et.c_str(), k);
-    }
-    uint32_t w[4];
-    int k = __builtin_popcount(U & (kFThreads - 1));
-    for (int b = 0; b < 4; ++b) {
-      w[b] = ((U >> (8 + b)) & 1) ? 1u << k : 0u;
-      k += (U >> (8 + b)) & 1;
+      if (tbit(pos) >= 0) {
+        const std::string t = r();
+        e("bfe.u32 %s, %%ltid, %d, 1;", t.c_str(), tbit(pos));
+        e("bfi.b32 %s, %s, %s, %d, 1;", et.c_str(), t.c_str(), et.c_str(), k);
+      } else {
+        w[reg_of(pos)] = 1u << k;
+      }
     }
     const std::string ebase = r();
     e("mad.lo.u32 %s, %s, %d, %%dtab;", ebase.c_str(), et.c_str(), ES);
-    const uint32_t crm = cm >> 8, crp = cp >> 8;
+    uint32_t ctm, ctv, crm, crp;
+    split(cm, cp, ctm, ctv, crm, crp);
     for (int r_ = 0; r_ < R; ++r_) {
       if (((uint32_t)r_ & crm) != crp) continue;
       uint32_t off = 0;
-      for (int b = 0; b < 4; ++b)
+      for (int b = 0; b < nreg; ++b)
         if ((r_ >> b) & 1) off += w[b];
       const Cx d = lds(ebase, (int)off * ES);
       set(r_, cmulf(d, {vx(r_), vy(r_)}));
+    }
+    label(end);
+  }
+
+  void ensure_regs() {
+    if (!in_regs) {
+      sync();
+      tile_to_regs();
+      in_regs = true;
+    }
+  }
+  static int op_targets(const FHdr& h, int* ts) {
+    ts[0] = h.t0;
+    ts[1] = h.t1;
+    ts[2] = h.t2;
+    switch (h.type) {
+      case F_SWAP: case F_U4: return 2;
+      case F_U8: return 3;
+      default: return 1;
+    }
+  }
+  // Ops until tile bit b is next a target of a non-diagonal op (Belady distance).
+  int next_use(int b, int from) const {
+    for (int o = from; o < P.nops; ++o) {
+      const FHdr& h = P.h[o];
+      if (h.type == F_DTAB) {
+        o += h.m;
+        continue;
+      }
+      if (h.type == F_DIAG1 || h.type == F_DIAGN) continue;
+      int ts[3];
+      const int m = op_targets(h, ts);
+      for (int s_ = 0; s_ < m; ++s_)
+        if (ts[s_] == b) return o - from;
+    }
+    return 1 << 30;
+  }
+  // Moves the warp-held tile bits `need` into register positions (evicting, by
+  // furthest next use, register-held bits that are not targets of op o) with one
+  // round trip through the shared-memory tile.
+  void remap(const std::vector<int>& need, const int* ts, int m, int o) {
+    if (in_regs) regs_to_tile();  // under the old placement
+    for (int b : need) {
+      int best = -1, bd = -1;
+      for (int j = 0; j < nreg; ++j) {
+        bool tgt = false;
+        for (int s_ = 0; s_ < m; ++s_) tgt |= rpos[j] == ts[s_];
+        if (tgt) continue;
+        const int d = next_use(rpos[j], o + 1);
+        if (d > bd) {
+          bd = d;
+          best = j;
+        }
+      }
+      const int w = tbit(b) - 5;
+      wpos[w] = rpos[best];
+      rpos[best] = b;
+    }
+    sync();
+    emit_taddr();
+    tile_to_regs();
+    in_regs = true;
+  }
+
+  // SWAP / U4 / U8 with every target register-held.
+  void op_regmulti(const FHdr& h) {
+    const std::string end = L();
+    tile_pred(h.mhi, h.phi, end);
+    skip_unless(thread_pred(h.mlo, h.plo), end);
+    uint32_t tm_, tv_, mr, pr;
+    split(h.mlo, h.plo, tm_, tv_, mr, pr);
+    if (h.type == F_SWAP) {
+      const int j0 = reg_of(h.t0), j1 = reg_of(h.t1);
+      for (int r_ = 0; r_ < R; ++r_) {
+        if (((r_ >> j0) & 1) || ((r_ >> j1) & 1)) continue;
+        if (((uint32_t)r_ & mr) != pr) continue;
+        const int x = r_ | (1 << j0), y = r_ | (1 << j1);
+        const Cx a = copy({vx(x), vy(x)}), b = copy({vx(y), vy(y)});
+        set(x, b);
+        set(y, a);
+      }
+      label(end);
+      return;
+    }
+    const int Lm = h.type == F_U4 ? 4 : 8;
+    std::vector<Cx> c, nc;
+    for (int j = 0; j < Lm * Lm; ++j) {
+      c.push_back(coef(h.coef + j));
+      nc.push_back({c.back().zy() ? std::string() : neg(c.back().y), ""});
+    }
+    int sb[3] = {reg_of(h.t0), reg_of(h.t1), Lm == 8 ? reg_of(h.t2) : -1};
+    for (int r_ = 0; r_ < R; ++r_) {
+      bool clear = true;
+      for (int q = 0; q < (Lm == 4 ? 2 : 3); ++q) clear &= !((r_ >> sb[q]) & 1);
+      if (!clear || ((uint32_t)r_ & mr) != pr) continue;
+      int idx[8];
+      for (int j = 0; j < Lm; ++j) {
+        idx[j] = r_;
+        if (Lm == 4) {
+          if ((j >> 1) & 1) idx[j] |= 1 << sb[0];
+          if (j & 1) idx[j] |= 1 << sb[1];
+        } else {
+          if ((j >> 2) & 1) idx[j] |= 1 << sb[0];
+          if ((j >> 1) & 1) idx[j] |= 1 << sb[1];
+          if (j & 1) idx[j] |= 1 << sb[2];
+        }
+      }
+      std::vector<Cx> v, w(Lm);
+      for (int j = 0; j < Lm; ++j) v.push_back({vx(idx[j]), vy(idx[j])});
+      for (int j = 0; j < Lm; ++j)
+        for (int q = 0; q < Lm; ++q) cfma(w[j], c[j * Lm + q], nc[j * Lm + q], v[q], q == 0);
+      for (int j = 0; j < Lm; ++j) set(idx[j], w[j]);
     }
     label(end);
   }
@@ -785,7 +965,7 @@ struct Gen {
     e("mov.u32 %%tile, lfqs_tile;");
     e("mov.u32 %%dtab, lfqs_dtab;");
     e("mov.u32 %%bar, lfqs_bar;");
-    e("mad.lo.u32 %%taddr, %%ltid, %d, %%tile;", ES);
+    emit_taddr();
     {
       const std::string w0 = L(), q = p(), q0 = p();
       e("setp.ge.u32 %s, %%ltid, 32;", q.c_str());
@@ -818,34 +998,39 @@ struct Gen {
         o += h.m;
         continue;
       }
-      if (type == F_DIAG1) {
-        if (!in_regs) {
-          sync();
-          tile_to_regs();
-          in_regs = true;
-        }
-        op_diag1(h);
+      if (type == F_DIAG1 || type == F_DIAGN) {
+        ensure_regs();
+        if (type == F_DIAG1)
+          op_diag1(h);
+        else
+          op_diagn(h);
         continue;
       }
-      const int t0 = h.t0;
-      const bool regpath = type <= F_DIAGN || (type <= F_U2 && (t0 < 5 || t0 >= 8));
-      if (regpath && !in_regs) {
-        sync();
-        tile_to_regs();
-        in_regs = true;
-      } else if (!regpath && in_regs) {
-        regs_to_tile();
-        in_regs = false;
-        sync();
-      } else if (!regpath) {
-        sync();
-      }
-      if (!regpath) {
-        op_smem(h);
-      } else if (type == F_DIAGN) {
-        op_diagn(h);
+      int ts[3];
+      const int m = op_targets(h, ts);
+      bool any_lane = false;
+      for (int s_ = 0; s_ < m; ++s_) any_lane |= ts[s_] < 5;
+      // 1-target gates: lane bits by shuffle, everything else in registers (a warp
+      // bit is first moved into a register position).  Multi-target gates: in
+      // registers when no target is a lane bit and they fit the register positions.
+      const bool in_reg_path = m == 1 ? (ts[0] < 5 || nreg >= 1) : (!any_lane && m <= nreg);
+      if (in_reg_path) {
+        std::vector<int> need;
+        for (int s_ = 0; s_ < m; ++s_)
+          if (ts[s_] >= 5 && reg_of(ts[s_]) < 0) need.push_back(ts[s_]);
+        if (!need.empty()) remap(need, ts, m, o);
+        ensure_regs();
+        if (m == 1)
+          op_reg1q(h);
+        else
+          op_regmulti(h);
       } else {
-        op_reg1q(h);
+        if (in_regs) {
+          regs_to_tile();
+          in_regs = false;
+        }
+        sync();
+        op_smem(h);
       }
     }
     if (in_regs) regs_to_tile();
