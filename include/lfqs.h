@@ -129,6 +129,16 @@ lfqs_status lfqs_state_wrap(int n_qubits, int device, void* dev_ptr, void* cuda_
  * single-GPU virtual partition (see lfqs_state_create_virtual).  The paper does
  * not state its precision (R5); complex128 stays the default. */
 #define LFQS_STATE_C64 1u
+/* LFQS_STATE_SOA: structure-of-arrays layout -- the paper's layout study (§6.6,
+ * PAPER.md:501-505, 605-613): the real plane re[0, 2^n) followed by the
+ * imaginary plane im[0, 2^n) in one allocation (a borrowed buffer holds the
+ * same two planes), instead of interleaved (re, im) pairs.  Single shard only
+ * (world >= 2: LFQS_ERR_UNSUPPORTED); gates run one pass each (lfqs_apply_gate,
+ * lfqs_run_circuit with LFQS_FUSE_NONE; fused runs return
+ * LFQS_ERR_UNSUPPORTED); copy_in/out keep interleaved host buffers;
+ * probabilities, sampling and collapse are layout-independent (bit-identical
+ * probabilities to an AOS state holding the same amplitudes). */
+#define LFQS_STATE_SOA 2u
 lfqs_status lfqs_state_create_ex(int n_qubits, int world, int device, void* cuda_stream,
                                  uint32_t flags, lfqs_state** out);
 /* Borrow caller memory with the precision given by flags (LFQS_STATE_C64: a

@@ -55,6 +55,7 @@ EXPORTS = [
 ]
 P2P_HANDLE_BYTES = 256
 STATE_C64 = 1
+STATE_SOA = 2  # structure-of-arrays planes (include/lfqs.h, NEXT-4 layout study)
 
 
 class LfqsError(RuntimeError):
@@ -506,9 +507,11 @@ class State:
         self.c64 = c64
 
     @classmethod
-    def create(cls, n_qubits: int, device: int = 0, stream=None, c64: bool = False) -> "State":
-        if c64:
-            return cls(lfqs_state_create_ex(n_qubits, 1, device, stream, STATE_C64), n_qubits, True)
+    def create(cls, n_qubits: int, device: int = 0, stream=None, c64: bool = False,
+               soa: bool = False) -> "State":
+        if c64 or soa:
+            flags = (STATE_C64 if c64 else 0) | (STATE_SOA if soa else 0)
+            return cls(lfqs_state_create_ex(n_qubits, 1, device, stream, flags), n_qubits, c64)
         return cls(lfqs_state_create(n_qubits, device, stream), n_qubits)
 
     @classmethod

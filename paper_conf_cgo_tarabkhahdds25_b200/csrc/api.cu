@@ -80,10 +80,13 @@ lfqs_status lfqs_state_create_ex(int n_qubits, int world, int device, void* stre
                                  uint32_t flags, lfqs_state** out) {
   return guarded([&] {
     require(out != nullptr, "out is NULL");
-    require((flags & ~LFQS_STATE_C64) == 0, "unknown state flags");
-    const bool c64 = (flags & LFQS_STATE_C64) != 0;
+    require((flags & ~(LFQS_STATE_C64 | LFQS_STATE_SOA)) == 0, "unknown state flags");
+    const bool c64 = (flags & LFQS_STATE_C64) != 0, soa = (flags & LFQS_STATE_SOA) != 0;
+    if (soa && world > 1)
+      throw Error(LFQS_ERR_UNSUPPORTED, "LFQS_STATE_SOA states are single-shard");
     if (world <= 1)
-      *out = State::create_local(n_qubits, device, static_cast<cudaStream_t>(stream), nullptr, c64);
+      *out = State::create_local(n_qubits, device, static_cast<cudaStream_t>(stream), nullptr, c64,
+                                 soa);
     else
       *out = State::create_virtual(n_qubits, world, device, static_cast<cudaStream_t>(stream), c64);
   });
@@ -93,11 +96,12 @@ lfqs_status lfqs_state_wrap_ex(int n_qubits, int device, void* dev_ptr, void* st
                                uint32_t flags, lfqs_state** out) {
   return guarded([&] {
     require(out != nullptr && dev_ptr != nullptr, "NULL argument");
-    require((flags & ~LFQS_STATE_C64) == 0, "unknown state flags");
-    const bool c64 = (flags & LFQS_STATE_C64) != 0;
+    require((flags & ~(LFQS_STATE_C64 | LFQS_STATE_SOA)) == 0, "unknown state flags");
+    const bool c64 = (flags & LFQS_STATE_C64) != 0, soa = (flags & LFQS_STATE_SOA) != 0;
     require((reinterpret_cast<uintptr_t>(dev_ptr) & (c64 ? 7 : 15)) == 0,
             "dev_ptr is not aligned to one amplitude");
-    *out = State::create_local(n_qubits, device, static_cast<cudaStream_t>(stream), dev_ptr, c64);
+    *out = State::create_local(n_qubits, device, static_cast<cudaStream_t>(stream), dev_ptr, c64,
+                               soa);
   });
 }
 

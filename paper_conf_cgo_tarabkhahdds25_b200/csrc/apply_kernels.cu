@@ -628,6 +628,10 @@ void launch_half_swap(const LaunchCtx& ctx, int l, uint64_t partner_offset_amps,
 }
 
 void launch_gate(const LaunchCtx& ctx, const Decoded& g) {
+  if (ctx.soa) {
+    launch_gate_soa(ctx, g);
+    return;
+  }
   if (ctx.c64)
     launch_gate_t<float>(ctx, g);
   else

@@ -107,6 +107,8 @@ struct LaunchCtx {
   bool jit = false;
   // Plan and compile only (lfqs_jit_precompile): no kernel is launched.
   bool dry_run = false;
+  // Structure-of-arrays shard (LFQS_STATE_SOA): real plane, then imaginary plane.
+  bool soa = false;
 };
 
 // Raises a kernel's dynamic shared memory limit once per device.
@@ -114,6 +116,8 @@ void ensure_smem_attr(const void* kernel, int bytes);
 
 // Applies one decoded gate whose targets are all < n_local (controls < n_local).
 void launch_gate(const LaunchCtx& ctx, const Decoded& g);
+// The same on a structure-of-arrays shard (soa_kernels.cu).
+void launch_gate_soa(const LaunchCtx& ctx, const Decoded& g);
 // Half-shard swap for the global-qubit exchange: the l=1 half of the shard at
 // ctx.amps with the l=0 half of the shard partner_offset_amps further on (first
 // n_pairs pairs; 0 = all).

@@ -85,10 +85,12 @@ void State::common_init(int n_, int world_, int device_, cudaStream_t s, bool c6
   LFQS_CUDA_CHECK(cudaMalloc(&d_probs, sizeof(double) * 1024));
 }
 
-State* State::create_local(int n, int device, cudaStream_t stream, void* borrowed, bool c64) {
+State* State::create_local(int n, int device, cudaStream_t stream, void* borrowed, bool c64,
+                           bool soa) {
   require(n >= 1 && n <= 36, "n_qubits must be in [1, 36] on one GPU");
   std::unique_ptr<State> st(new State());
   st->common_init(n, 1, device, stream, c64);
+  st->soa = soa;
   if (borrowed) {
     st->amps = static_cast<unsigned char*>(borrowed);
   } else {
@@ -188,6 +190,7 @@ LaunchCtx State::ctx(int shard) {
   c.launch_counter = &launches;
   c.opt = &opt;
   c.c64 = c64;
+  c.soa = soa;
   c.phase_tables = phase_tables;
   c.jit = jit;
   return c;
@@ -226,7 +229,20 @@ void State::copy_raw(uint64_t offset, uint64_t count, void* host, bool to_device
   const uint64_t lo = virt ? 0 : (uint64_t)rank << n_local;
   const uint64_t hi = virt ? total : lo + (1ull << n_local);
   const uint64_t a = std::max(offset, lo), b = std::min(offset + count, hi);
-  if (a < b) {
+  if (a < b && soa) {
+    // interleaved host pairs <-> the two planes: strided 2-D copies
+    const size_t es = ab / 2;
+    unsigned char* h = static_cast<unsigned char*>(host) + (a - offset) * ab;
+    for (int part = 0; part < 2; ++part) {
+      unsigned char* dev = amps + ((uint64_t)part << n_local) * es + (a - lo) * es;
+      if (to_device)
+        LFQS_CUDA_CHECK(cudaMemcpy2DAsync(dev, es, h + part * es, ab, es, b - a,
+                                          cudaMemcpyHostToDevice, stream));
+      else
+        LFQS_CUDA_CHECK(cudaMemcpy2DAsync(h + part * es, ab, dev, es, es, b - a,
+                                          cudaMemcpyDeviceToHost, stream));
+    }
+  } else if (a < b) {
     unsigned char* dev = amps + (a - lo) * ab;
     unsigned char* h = static_cast<unsigned char*>(host) + (a - offset) * ab;
     const size_t bytes = (b - a) * ab;
@@ -348,6 +364,8 @@ void State::apply(const Decoded& g) {
 void State::run(const std::vector<Decoded>& gates, uint32_t flags) {
   DeviceGuard dg(device);
   const bool fuse = (flags & LFQS_FUSE_LOW) != 0;
+  if (fuse && soa)
+    throw Error(LFQS_ERR_UNSUPPORTED, "fused passes need an AOS state (LFQS_STATE_SOA is per-gate only)");
   phase_tables = fuse && (flags & LFQS_FUSE_PHASE) != 0;
   jit = fuse && (flags & LFQS_FUSE_JIT) != 0;
   struct Reset {

@@ -29,6 +29,7 @@ struct State : lfqs_state {
   bool virt = false;            // `world` shards in one allocation (single GPU)
   unsigned char* amps = nullptr;  // shard 0 (virtual: all shards back to back)
   bool c64 = false;             // complex64 amplitudes (NEXT-4); default complex128
+  bool soa = false;             // structure-of-arrays planes (NEXT-4); default AOS
   int ab = 16;                  // bytes per amplitude
   bool owned = false;
   cudaStream_t stream = nullptr;
@@ -44,7 +45,7 @@ struct State : lfqs_state {
   uint64_t exchanges = 0, exchange_bytes = 0;
 
   static State* create_local(int n, int device, cudaStream_t stream, void* borrowed,
-                             bool c64 = false);
+                             bool c64 = false, bool soa = false);
   static State* create_virtual(int n, int world, int device, cudaStream_t stream,
                                bool c64 = false);
   static State* create_dist(int n, int rank, int world, const uint8_t uid[128], int device,

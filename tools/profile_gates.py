@@ -54,6 +54,7 @@ def main():
     ap.add_argument("--no-shuffle", action="store_true")
     ap.add_argument("--no-wide", action="store_true")
     ap.add_argument("--c64", action="store_true", help="complex64 state")
+    ap.add_argument("--soa", action="store_true", help="structure-of-arrays state (NEXT-4 layout study)")
     ap.add_argument("--ipt", type=int, default=0, help="groups per thread for pair gates (0=default)")
     args = ap.parse_args()
     import torch
@@ -62,7 +63,7 @@ def main():
     torch.cuda.set_stream(s)
     gates = parse(args.gates, args.n)
     ab = 8 if args.c64 else 16
-    with L.State.create(args.n, 0, stream=s, c64=args.c64) as st:
+    with L.State.create(args.n, 0, stream=s, c64=args.c64, soa=args.soa) as st:
         st.set_option(L.OPT_LOWQ_SHUFFLE, 0 if args.no_shuffle else 1)
         st.set_option(L.OPT_WIDE256, 0 if args.no_wide else 1)
         st.set_option(L.OPT_ITEMS_PER_THREAD, args.ipt)
