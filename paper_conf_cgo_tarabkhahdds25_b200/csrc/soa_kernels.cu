@@ -27,9 +27,10 @@ namespace {
 constexpr int kThreads = 256;
 
 struct SoaGate {
-  InsertPlan ip;       // zeros at targets and controls, ones at controls
-  uint64_t off[8];     // offset of local index j: sum of its target bits
+  InsertPlan ip;       // zeros at group bits and controls, ones at controls
+  uint64_t off[8];     // offset of local index j: sum of its group bits
   double2 m[64];       // DENSE: L x L row-major; DIAG: the L diagonal entries
+  int store_all;       // DIAG: rewrite unchanged entries too (whole 32-B sectors)
 };
 
 template <class S, int L, bool DIAG>
@@ -52,7 +53,13 @@ __global__ void __launch_bounds__(kThreads) k_soa(S* __restrict__ re, S* __restr
 #pragma unroll
       for (int j = 0; j < L; ++j) {
         const double2 d = g.m[j];
-        if (d.x == 1.0 && d.y == 0.0) continue;
+        if (d.x == 1.0 && d.y == 0.0) {
+          if (g.store_all) {
+            __stcs(re + k + g.off[j], v[j].x);
+            __stcs(im + k + g.off[j], v[j].y);
+          }
+          continue;
+        }
         const C z = cmul_rn(mk<S>((S)d.x, (S)d.y), v[j]);
         __stcs(re + k + g.off[j], z.x);
         __stcs(im + k + g.off[j], z.y);
@@ -87,23 +94,72 @@ void launch_soa_t(const LaunchCtx& ctx, const Decoded& d) {
   if (d.cls == GClass::NOOP) return;
   SoaGate g;
   std::memset(&g, 0, sizeof g);
-  uint64_t zmask = d.cmask;
-  for (int s = 0; s < d.m; ++s) zmask |= 1ull << d.targets[s];
+  const bool diag = d.cls == GClass::DIAG;
+  const int m = d.m, Lg = 1 << m;
+  uint64_t tmask = 0;
+  for (int s = 0; s < m; ++s) tmask |= 1ull << d.targets[s];
+  // Sector rules (as in the AOS kernels): the 8-byte planes put 4
+  // consecutive amplitudes in one 32-B sector, so a pass that writes only some
+  // of the indices with bits 0/1 fixed pays read-modify-writes.  Controls on
+  // bits 0/1 therefore join the group (the gate acts where they are 1, identity
+  // elsewhere) and diagonal groups touching bits 0/1 rewrite every entry.
+  uint64_t wctl = d.cmask & 3ull;
+  if (m + __builtin_popcountll(wctl) > 3) wctl = 0;
+  int gbits[3], ng = 0;
+  for (int s = 0; s < m; ++s) gbits[ng++] = d.targets[s];  // local index MSB first
+  for (int q = 0; q < 2; ++q)
+    if ((wctl >> q) & 1) gbits[ng++] = q;
+  const uint64_t ctl = d.cmask & ~wctl;
+  const int L = 1 << ng;
+  // Expanded matrix over the group: gate where the widened controls are 1.
+  auto entry = [&](int row, int col) -> double2 {
+    const int ncw = ng - m;
+    const int rc = row & ((1 << ncw) - 1), cc = col & ((1 << ncw) - 1);
+    const int rt = row >> ncw, ct = col >> ncw;
+    if (rc != cc) return make_double2(0.0, 0.0);
+    if (rc != (1 << ncw) - 1) return make_double2(rt == ct ? 1.0 : 0.0, 0.0);
+    return make_double2(d.M[rt * Lg + ct].re, d.M[rt * Lg + ct].im);
+  };
+  uint64_t zmask = ctl, ones = ctl;
+  const bool low = ((tmask | d.cmask) & 3ull) != 0;
+  if (diag && !low) {
+    // One-entry diagonals (Z, S, T, Phase, CZ, CPhase, MC-Z) touch only the
+    // amplitudes whose factor is not 1: fold the targets into the fixed bits.
+    int active = -1, na = 0;
+    for (int j = 0; j < Lg; ++j)
+      if (!(d.M[j * Lg + j].re == 1.0 && d.M[j * Lg + j].im == 0.0)) {
+        ++na;
+        active = j;
+      }
+    if (na == 1) {
+      for (int s = 0; s < m; ++s)
+        if ((active >> (m - 1 - s)) & 1) ones |= 1ull << d.targets[s];
+      zmask |= tmask;
+      for (int q = 0; q < 64; ++q)
+        if ((zmask >> q) & 1) g.ip.pos[g.ip.np++] = q;
+      g.ip.ones = ones;
+      g.off[0] = 0;
+      g.m[0] = make_double2(d.M[active * Lg + active].re, d.M[active * Lg + active].im);
+      run_soa<S, 1, true>(ctx, 1ull << (ctx.n_local - g.ip.np), g);
+      return;
+    }
+  }
+  for (int s = 0; s < ng; ++s) zmask |= 1ull << gbits[s];
   for (int q = 0; q < 64; ++q)
     if ((zmask >> q) & 1) g.ip.pos[g.ip.np++] = q;
-  g.ip.ones = d.cmask;
-  const int L = 1 << d.m;
+  g.ip.ones = ones;
   for (int j = 0; j < L; ++j) {
     uint64_t o = 0;
-    for (int s = 0; s < d.m; ++s)
-      if ((j >> (d.m - 1 - s)) & 1) o |= 1ull << d.targets[s];
+    for (int s = 0; s < ng; ++s)
+      if ((j >> (ng - 1 - s)) & 1) o |= 1ull << gbits[s];
     g.off[j] = o;
   }
-  const bool diag = d.cls == GClass::DIAG;
+  g.store_all = low ? 1 : 0;
   if (diag) {
-    for (int j = 0; j < L; ++j) g.m[j] = make_double2(d.M[j * L + j].re, d.M[j * L + j].im);
+    for (int j = 0; j < L; ++j) g.m[j] = entry(j, j);
   } else {
-    for (int j = 0; j < L * L; ++j) g.m[j] = make_double2(d.M[j].re, d.M[j].im);
+    for (int r = 0; r < L; ++r)
+      for (int c = 0; c < L; ++c) g.m[r * L + c] = entry(r, c);
   }
   const uint64_t n_groups = 1ull << (ctx.n_local - g.ip.np);
   switch (L) {
