@@ -77,8 +77,77 @@ __global__ void __launch_bounds__(kThreads) k_soa(S* __restrict__ re, S* __restr
   }
 }
 
+// Two adjacent groups per item when bit 0 is neither a group bit nor fixed: the
+// base indices k, k + 1 share every other bit, so each plane access is one
+// 2-element vector (16 B for complex128 planes), contiguous across the warp.
+template <class S> struct V2;
+template <> struct V2<double> { using T = double2; };
+template <> struct V2<float> { using T = float2; };
+
+template <class S, int L, bool DIAG>
+__global__ void __launch_bounds__(kThreads) k_soa2(S* __restrict__ re, S* __restrict__ im,
+                                                   uint64_t n_items, const __grid_constant__ SoaGate g) {
+  using C = cx<S>;
+  using VT = typename V2<S>::T;
+  const uint64_t stride = (uint64_t)gridDim.x * kThreads;
+  for (uint64_t it = (uint64_t)blockIdx.x * kThreads + threadIdx.x; it < n_items; it += stride) {
+    uint64_t k = 2 * it;
+    for (int i = 0; i < g.ip.np; ++i) {
+      const int p = g.ip.pos[i];
+      const uint64_t lo = k & ((1ull << p) - 1);
+      k = ((k - lo) << 1) | lo;
+    }
+    k |= g.ip.ones;
+    C v[2][L];
+#pragma unroll
+    for (int j = 0; j < L; ++j) {
+      const VT r = __ldcs(reinterpret_cast<const VT*>(re + k + g.off[j]));
+      const VT i = __ldcs(reinterpret_cast<const VT*>(im + k + g.off[j]));
+      v[0][j] = mk<S>(r.x, i.x);
+      v[1][j] = mk<S>(r.y, i.y);
+    }
+    C w[2][L];
+#pragma unroll
+    for (int h = 0; h < 2; ++h)
+#pragma unroll
+      for (int j = 0; j < L; ++j) {
+        if (DIAG) {
+          const double2 d = g.m[j];
+          w[h][j] = (d.x == 1.0 && d.y == 0.0) ? v[h][j] : cmul_rn(mk<S>((S)d.x, (S)d.y), v[h][j]);
+        } else {
+          C acc = mk<S>(0, 0);
+#pragma unroll
+          for (int i = 0; i < L; ++i)
+            cfma(acc, mk<S>((S)g.m[j * L + i].x, (S)g.m[j * L + i].y), v[h][i]);
+          w[h][j] = acc;
+        }
+      }
+#pragma unroll
+    for (int j = 0; j < L; ++j) {
+      if (DIAG && g.m[j].x == 1.0 && g.m[j].y == 0.0) continue;
+      VT r, i;
+      r.x = w[0][j].x;
+      r.y = w[1][j].x;
+      i.x = w[0][j].y;
+      i.y = w[1][j].y;
+      __stcs(reinterpret_cast<VT*>(re + k + g.off[j]), r);
+      __stcs(reinterpret_cast<VT*>(im + k + g.off[j]), i);
+    }
+  }
+}
+
 template <class S, int L, bool DIAG>
 void run_soa(const LaunchCtx& ctx, uint64_t n_groups, const SoaGate& g) {
+  if (g.ip.np > 0 && g.ip.pos[0] > 0 && n_groups >= 2) {  // bit 0 free: paired vector accesses
+    S* re = reinterpret_cast<S*>(ctx.amps);
+    S* im = re + (1ull << ctx.n_local);
+    uint64_t nb = (n_groups / 2 + kThreads - 1) / kThreads;
+    if (nb > 148ull * 32) nb = 148ull * 32;
+    k_soa2<S, L, DIAG><<<(unsigned)nb, kThreads, 0, ctx.stream>>>(re, im, n_groups / 2, g);
+    LFQS_CUDA_CHECK(cudaGetLastError());
+    ++*ctx.launch_counter;
+    return;
+  }
   S* re = reinterpret_cast<S*>(ctx.amps);
   S* im = re + (1ull << ctx.n_local);
   uint64_t nb = (n_groups + kThreads - 1) / kThreads;
@@ -98,13 +167,12 @@ void launch_soa_t(const LaunchCtx& ctx, const Decoded& d) {
   const int m = d.m, Lg = 1 << m;
   uint64_t tmask = 0;
   for (int s = 0; s < m; ++s) tmask |= 1ull << d.targets[s];
-  // Sector rules (as in the AOS kernels): the 8-byte planes put 4
-  // consecutive amplitudes in one 32-B sector, so a pass that writes only some
-  // of the indices with bits 0/1 fixed pays read-modify-writes.  Controls on
-  // bits 0/1 therefore join the group (the gate acts where they are 1, identity
-  // elsewhere) and diagonal groups touching bits 0/1 rewrite every entry.
-  uint64_t wctl = d.cmask & 3ull;
-  if (m + __builtin_popcountll(wctl) > 3) wctl = 0;
+  // Sector rule (as in the AOS kernels): the 8-byte planes put 4
+  // consecutive amplitudes in one 32-B sector, so diagonal groups touching bits
+  // 0/1 rewrite every entry instead of leaving holes (read-modify-writes).
+  // (Moving controls on bits 0/1 into the group, as the AOS path does, measured
+  // slower here: the 4 strided 8-byte accesses per plane cost more than the holes.)
+  const uint64_t wctl = 0;
   int gbits[3], ng = 0;
   for (int s = 0; s < m; ++s) gbits[ng++] = d.targets[s];  // local index MSB first
   for (int q = 0; q < 2; ++q)
