@@ -30,7 +30,7 @@ def worker(rank, world, port, n, seed, out_q):
         ref = O.run_circuit(n, gates, psi.copy())
         ref_exact = O.run_circuit(n, exact, psi.copy())
         qs = [0, n // 2, n - 1]
-        for fuse in (False, True):
+        for key, fuse in ((0, False), (1, True), (2, "jit")):
             with L.State.p2p(n, rank, world) as st:
                 st.copy_in(psi)
                 st.run_circuit(gates, fuse=fuse)
@@ -38,10 +38,10 @@ def worker(rank, world, port, n, seed, out_q):
                 err = float(np.max(np.abs(got - ref[lo:hi])))
                 p = st.measure_probs(qs)
                 perr = float(np.max(np.abs(p - O.probs(n, ref, qs))))
-                report[f"fuse{int(fuse)}"] = (err, perr)
+                report[f"fuse{key}"] = (err, perr)
                 st.copy_in(psi)
                 st.run_circuit(exact, fuse=fuse)
-                report[f"exact{int(fuse)}"] = bool(np.array_equal(st.copy_out()[lo:hi],
+                report[f"exact{key}"] = bool(np.array_equal(st.copy_out()[lo:hi],
                                                                    ref_exact[lo:hi]))
                 st.synchronize()
         # one gate at a time through lfqs_apply_gate (planner per gate, exchanges included)

@@ -46,7 +46,7 @@ def test_p2p_sharded_circuits(world):
     for rank in range(world):
         status, payload = results[rank]
         assert status == "ok", f"rank {rank}:\n{payload}"
-        for fuse in (0, 1):
+        for fuse in (0, 1, 2):  # unfused, fused (interpreted), fused (compiled passes)
             err, perr = payload[f"fuse{fuse}"]
             assert err <= 1e-12 and perr <= 1e-12, (rank, fuse, err, perr)
             assert payload[f"exact{fuse}"], (rank, fuse)
