@@ -837,7 +837,7 @@ void build_program(const LaunchCtx& ctx, const TileCfg& cfg, uint64_t in_tile,
   P.nops = 0;
   P.ncoef = 0;
   int b = 0, lc = 0;
-  P.tile.nh = 0;
+  std::memset(&P.tile, 0, sizeof P.tile);  // unused hpos entries too (JIT cache key)
   for (int q = 0; q < 64; ++q) {
     tm.tb[q] = -1;
     if (q < ctx.n_local && (in_tile >> q & 1)) {
@@ -887,9 +887,9 @@ void build_program(const LaunchCtx& ctx, const TileCfg& cfg, uint64_t in_tile,
 
 // Launches an encoded pass: the compiled kernel of its program (LFQS_FUSE_JIT)
 // or the interpreting kernel k_fused<K>.
-void launch_built(const LaunchCtx& ctx, int K, const FProg& P, const std::string* ptx = nullptr) {
+void launch_built(const LaunchCtx& ctx, int K, const FProg& P, const std::string* key = nullptr) {
   if (ctx.jit && (1 << P.tile.nh) <= ctx.opt->fuse_tma_max_chunks) {
-    jit_launch(ctx, P, K, ptx ? *ptx : jit_ptx(P, K, ctx.c64));
+    jit_launch(ctx, P, K, key ? *key : jit_key(P, K, ctx.c64));
     ++*ctx.launch_counter;
     return;
   }
@@ -967,7 +967,7 @@ void run_fused_schedule(const LaunchCtx& ctx, const std::vector<Decoded>& gates,
   struct Pass {
     int gate = -1;                 // single-gate pass (class kernel)
     std::unique_ptr<FProg> prog;   // fused pass
-    std::string ptx;
+    std::string key;
   };
   std::vector<Pass> passes;
   const bool collect = ctx.jit && (1 << (cfg.K - cfg.L)) <= ctx.opt->fuse_tma_max_chunks;
@@ -1026,7 +1026,7 @@ void run_fused_schedule(const LaunchCtx& ctx, const std::vector<Decoded>& gates,
         passes.emplace_back();
         passes.back().prog.reset(new FProg);
         build_program(ctx, cfg, in_tile, list, *passes.back().prog);
-        passes.back().ptx = jit_ptx(*passes.back().prog, cfg.K, ctx.c64);
+        passes.back().key = jit_key(*passes.back().prog, cfg.K, ctx.c64);
       } else {
         launch_program(ctx, cfg, in_tile, list);
       }
@@ -1035,17 +1035,17 @@ void run_fused_schedule(const LaunchCtx& ctx, const std::vector<Decoded>& gates,
     while (head < rest.size() && taken[rest[head]]) ++head;
   }
   if (!collect) return;
-  std::vector<std::string> srcs;
+  std::vector<std::pair<std::string, const FProg*>> items;
   for (const Pass& ps : passes)
-    if (ps.prog) srcs.push_back(ps.ptx);
-  jit_compile(srcs);
+    if (ps.prog) items.emplace_back(ps.key, ps.prog.get());
+  jit_compile(items, cfg.K, ctx.c64);
   if (ctx.dry_run) {
     *ctx.launch_counter += passes.size();
     return;
   }
   for (const Pass& ps : passes) {
     if (ps.prog)
-      launch_built(ctx, cfg.K, *ps.prog, &ps.ptx);
+      launch_built(ctx, cfg.K, *ps.prog, &ps.key);
     else
       launch_gate(ctx, gates[ps.gate]);
   }

@@ -13,7 +13,7 @@
 // parameter (constant bank), so one compiled pass serves every angle set of
 // the same circuit structure.  PTX is compiled in-process by nvPTXCompiler
 // (no NVVM: compiling generated CUDA C++ through NVRTC took seconds per pass),
-// passes are compiled in parallel and cached by their PTX text, and loaded
+// passes are compiled in parallel and cached by their structure, and loaded
 // with cudaLibraryLoadData.
 //
 // The emitted arithmetic replicates k_fused op by op (same formulas, same FMA
@@ -1150,16 +1150,44 @@ std::string jit_ptx(const FProg& P, int K, bool c64) {
   return g.build();
 }
 
-void jit_compile(const std::vector<std::string>& ptxs) {
-  std::vector<std::pair<const std::string*, std::shared_ptr<Entry>>> todo;
+// Cache key: everything the generator reads -- geometry, op headers, and per
+// coefficient component its class (0, +1, -1, other; the generator specialises
+// exact zeros and ones) -- but not the coefficient values, which are a kernel
+// parameter.  Building the key costs O(program), not a PTX generation.
+std::string jit_key(const FProg& P, int K, bool c64) {
+  std::string k;
+  k.reserve(64 + P.nops * sizeof(FHdr) + P.ncoef);
+  const int head[4] = {K, c64 ? 1 : 0, P.nops, P.ncoef};
+  k.append(reinterpret_cast<const char*>(head), sizeof head);
+  k.append(reinterpret_cast<const char*>(&P.tile), sizeof P.tile);
+  k.append(reinterpret_cast<const char*>(P.h), sizeof(FHdr) * P.nops);
+  for (int j = 0; j < P.ncoef; ++j) {
+    char cls = 0;
+    const double v[2] = {P.c[j].x, P.c[j].y};
+    for (int q = 0; q < 2; ++q) {
+      const double x = c64 ? (double)(float)v[q] : v[q];
+      const int c = x == 0.0 ? 0 : x == 1.0 ? 1 : x == -1.0 ? 2 : 3;
+      cls = (char)(cls | (c << (2 * q)));
+    }
+    k.push_back(cls);
+  }
+  return k;
+}
+
+void jit_compile(const std::vector<std::pair<std::string, const FProg*>>& items, int K, bool c64) {
+  struct Todo {
+    const std::string* key;
+    const FProg* prog;
+    std::shared_ptr<Entry> en;
+  };
+  std::vector<Todo> todo;
   {
     std::lock_guard<std::mutex> lk(g_mu);
-    for (const std::string& s : ptxs) {
-      auto it = g_cache.find(s);
-      if (it != g_cache.end()) continue;
+    for (const auto& it : items) {
+      if (g_cache.count(it.first)) continue;
       auto en = std::make_shared<Entry>();
-      g_cache.emplace(s, en);
-      todo.emplace_back(&s, en);
+      g_cache.emplace(it.first, en);
+      todo.push_back({&it.first, it.second, en});
     }
   }
   if (todo.empty()) return;
@@ -1167,20 +1195,20 @@ void jit_compile(const std::vector<std::string>& ptxs) {
   if (nt == 0) nt = 4;
   if (nt > todo.size()) nt = (unsigned)todo.size();
   std::atomic<size_t> next{0};
-  if (const char* dir = std::getenv("LFQS_JIT_DUMP")) {  // debugging aid
-    for (auto& t : todo) {
-      const std::string fn = std::string(dir) + "/pass_" +
-                             std::to_string(std::hash<std::string>()(*t.first)) + ".ptx";
-      if (FILE* fp = std::fopen(fn.c_str(), "w")) {
-        std::fwrite(t.first->data(), 1, t.first->size(), fp);
-        std::fclose(fp);
-      }
-    }
-  }
+  const char* dump = std::getenv("LFQS_JIT_DUMP");  // debugging aid: write the PTX
   auto work = [&] {
     for (size_t i; (i = next.fetch_add(1)) < todo.size();) {
-      compile_entry(*todo[i].first, *todo[i].second);
-      todo[i].second->compiled = true;
+      const std::string ptx = jit_ptx(*todo[i].prog, K, c64);
+      if (dump) {
+        const std::string fn = std::string(dump) + "/pass_" +
+                               std::to_string(std::hash<std::string>()(ptx)) + ".ptx";
+        if (FILE* fp = std::fopen(fn.c_str(), "w")) {
+          std::fwrite(ptx.data(), 1, ptx.size(), fp);
+          std::fclose(fp);
+        }
+      }
+      compile_entry(ptx, *todo[i].en);
+      todo[i].en->compiled = true;
     }
   };
   std::vector<std::thread> th;
@@ -1188,10 +1216,10 @@ void jit_compile(const std::vector<std::string>& ptxs) {
   work();
   for (auto& t : th) t.join();
   for (auto& t : todo)
-    if (!t.second->error.empty()) {
-      const std::string err = t.second->error;
+    if (!t.en->error.empty()) {
+      const std::string err = t.en->error;
       std::lock_guard<std::mutex> lk(g_mu);
-      g_cache.erase(*t.first);
+      g_cache.erase(*t.key);
       throw Error(LFQS_ERR_CUDA, "JIT pass compile failed: " + err);
     }
 }
@@ -1201,17 +1229,17 @@ size_t jit_cache_size() {
   return g_cache.size();
 }
 
-void jit_launch(const LaunchCtx& ctx, const FProg& P, int K, const std::string& ptx) {
+void jit_launch(const LaunchCtx& ctx, const FProg& P, int K, const std::string& key) {
   std::shared_ptr<Entry> en;
   {
     std::lock_guard<std::mutex> lk(g_mu);
-    auto it = g_cache.find(ptx);
+    auto it = g_cache.find(key);
     if (it != g_cache.end()) en = it->second;
   }
   if (!en) {
-    jit_compile({ptx});
+    jit_compile({{key, &P}}, K, ctx.c64);
     std::lock_guard<std::mutex> lk(g_mu);
-    en = g_cache.at(ptx);
+    en = g_cache.at(key);
   }
   const int es = ctx.c64 ? 8 : 16;
   const int smem = es << K;

@@ -1,6 +1,7 @@
 // jit.h -- pass compiler for fused passes (LFQS_FUSE_JIT, jit.cpp).
 #pragma once
 #include <string>
+#include <utility>
 #include <vector>
 
 #include "fused_prog.h"
@@ -10,10 +11,12 @@ namespace lfqs {
 
 // PTX of one fused pass: structure baked in, coefficients a kernel parameter.
 std::string jit_ptx(const FProg& P, int K, bool c64);
-// Compiles (in parallel, nvPTXCompiler) every source not yet cached.
-void jit_compile(const std::vector<std::string>& ptxs);
+// Cache key of a pass (its structure and coefficient classes, not values).
+std::string jit_key(const FProg& P, int K, bool c64);
+// Generates and compiles (in parallel, nvPTXCompiler) every pass not yet cached.
+void jit_compile(const std::vector<std::pair<std::string, const FProg*>>& items, int K, bool c64);
 // Launches the pass (compiling it first if needed) on ctx.stream.
-void jit_launch(const LaunchCtx& ctx, const FProg& P, int K, const std::string& ptx);
+void jit_launch(const LaunchCtx& ctx, const FProg& P, int K, const std::string& key);
 size_t jit_cache_size();
 
 }  // namespace lfqs

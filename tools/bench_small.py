@@ -7,6 +7,9 @@ launch-bound, so it reports the ways of issuing them:
   graph    the same launches captured once in a CUDA graph (lfqs_circuit_launch)
   fused    lfqs_run_circuit with LFQS_FUSE_LOW (the 16 KiB state is one tile)
   fgraph   the fused program captured in a CUDA graph
+  jit      lfqs_run_circuit with LFQS_FUSE_LOW | LFQS_FUSE_JIT (compiled passes; compile
+           done once before timing, reported as jit_compile_s)
+  jgraph   the compiled passes captured in a CUDA graph
   oracle   the oracle, tier B, one host thread
 
     python tools/bench_small.py [--n 10] [--reps 50]
@@ -67,6 +70,12 @@ def main():
         with st.compile(arr, fuse=True) as c:
             res["fgraph"] = timed(c.launch, reps)
             fkern = c.kernels
+        t0 = time.perf_counter()
+        L.lfqs_jit_precompile(n, arr, "jit")
+        jit_s = time.perf_counter() - t0
+        res["jit"] = timed(lambda: L.lfqs_run_circuit(st.h, arr, L.FUSE_LOW | L.FUSE_JIT), reps)
+        with st.compile(arr, fuse="jit") as c:
+            res["jgraph"] = timed(c.launch, reps)
     import oracle as O
     O.build()
     t0 = time.perf_counter()
@@ -76,7 +85,8 @@ def main():
         print(json.dumps({"config": "configs[0]", "n": n, "gates": len(gates), "mode": mode,
                           "s_per_circuit": t, "us_per_gate": t / len(gates) * 1e6,
                           "gates_per_s": len(gates) / t,
-                          "kernels": kern if mode == "graph" else fkern if mode == "fgraph" else None,
+                          "kernels": kern if mode == "graph" else fkern if mode in ("fgraph", "jgraph") else None,
+                          "jit_compile_s": jit_s if mode in ("jit", "jgraph") else None,
                           "host_threads": 1 if mode == "oracle" else None}), flush=True)
 
 
