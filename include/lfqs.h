@@ -320,6 +320,8 @@ lfqs_status lfqs_kernel_launches(const lfqs_state* s, uint64_t* count);
                                           copies, larger ones by direct loads (default 256) */
 #define LFQS_OPT_FUSE_REORDER 7 /* 1: fused passes may take later gates that commute exactly
                                    with the skipped ones (default 1); 0: prefixes only */
+#define LFQS_OPT_JIT_THREADS 8 /* threads per CTA of LFQS_FUSE_JIT passes: 256 (default) or 512
+                                   (twice the warps per SM, half the amplitudes per thread) */
 lfqs_status lfqs_set_option(lfqs_state* s, int option, int64_t value);
 const char* lfqs_last_error(void);
 int lfqs_abi_version(void);

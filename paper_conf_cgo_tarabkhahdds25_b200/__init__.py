@@ -37,6 +37,7 @@ OPT_WIDE256 = 4
 OPT_FUSE_LOW_QUBITS = 5
 OPT_FUSE_TMA_MAX_CHUNKS = 6
 OPT_FUSE_REORDER = 7
+OPT_JIT_THREADS = 8
 
 STATUS = {0: "OK", -1: "INVALID_ARG", -2: "OUT_OF_MEMORY", -3: "CUDA", -4: "NCCL",
           -5: "UNSUPPORTED"}

@@ -63,15 +63,21 @@ struct Gen {
   // there, so 1-target gates on warp bits and multi-target gates on register bits
   // run in registers instead of as shared-memory ops.  Every amplitude still sees
   // the same arithmetic, so results stay bit-identical to the interpreter.
-  int wpos[3] = {5, 6, 7};
+  int NT = 256;   // threads per CTA (256, or 512 for K >= 9: twice the warps per SM)
+  int NWB = 3;    // warp bits of the thread index
+  int wpos[4] = {5, 6, 7, 8};
   int rpos[4] = {8, 9, 10, 11};
   int nreg = 0;
 
-  Gen(const FProg& p, int k, bool c) : P(p), K(k), c64(c) {
+  Gen(const FProg& p, int k, bool c, int nt) : P(p), K(k), c64(c) {
     FT = c64 ? "f32" : "f64";
     ES = c64 ? 8 : 16;
-    R = (1 << K) / kFThreads;
-    nreg = K - 8;
+    NT = nt;
+    NWB = NT == 512 ? 4 : 3;
+    R = (1 << K) / NT;
+    nreg = K - 5 - NWB;
+    for (int j = 0; j < NWB; ++j) wpos[j] = 5 + j;
+    for (int j = 0; j < nreg; ++j) rpos[j] = 5 + NWB + j;
   }
 
   int reg_of(int b) const {
@@ -82,7 +88,7 @@ struct Gen {
   // Thread bit holding tile bit b, or -1 when b is register-held.
   int tbit(int b) const {
     if (b < 5) return b;
-    for (int j = 0; j < 3; ++j)
+    for (int j = 0; j < NWB; ++j)
       if (wpos[j] == b) return 5 + j;
     return -1;
   }
@@ -114,7 +120,7 @@ struct Gen {
   void emit_taddr() {
     const std::string t = r();
     e("and.b32 %s, %%ltid, 31;", t.c_str());
-    for (int j = 0; j < 3; ++j) {
+    for (int j = 0; j < NWB; ++j) {
       const std::string x = r();
       e("bfe.u32 %s, %%ltid, %d, 1;", x.c_str(), 5 + j);
       e("shl.b32 %s, %s, %d;", x.c_str(), x.c_str(), wpos[j]);
@@ -612,11 +618,11 @@ struct Gen {
   // `fn(pvreg)` emits one item.
   template <class F>
   void for_items(int total, F fn) {
-    for (int pp = 0; pp * kFThreads < total; ++pp) {
+    for (int pp = 0; pp * NT < total; ++pp) {
       const std::string pv = r();
-      e("add.u32 %s, %%ltid, %d;", pv.c_str(), pp * kFThreads);
+      e("add.u32 %s, %%ltid, %d;", pv.c_str(), pp * NT);
       std::string skip;
-      if ((pp + 1) * kFThreads > total) {
+      if ((pp + 1) * NT > total) {
         skip = L();
         const std::string q = p();
         e("setp.ge.u32 %s, %s, %d;", q.c_str(), pv.c_str(), total);
@@ -1055,7 +1061,7 @@ struct Gen {
     const int nc = P.ncoef > 0 ? P.ncoef : 1;
     out += ".visible .entry lfqs_jit(.param .u64 pa, .param .align 16 .b8 pc[" +
            std::to_string(nc * 16) + "])\n";
-    out += ".maxntid 256, 1, 1\n.minnctapersm 2\n{\n";
+    out += ".maxntid " + std::to_string(NT) + ", 1, 1\n.minnctapersm 2\n{\n";
     out += "  .reg .pred %p<" + std::to_string(np + 1) + ">;\n";
     out += "  .reg .b32 %r<" + std::to_string(nr + 1) + ">;\n";
     out += "  .reg .b64 %rd<" + std::to_string(nrd + 1) + ">;\n";
@@ -1145,8 +1151,8 @@ void compile_entry(const std::string& ptx, Entry& en) {
 
 }  // namespace
 
-std::string jit_ptx(const FProg& P, int K, bool c64) {
-  Gen g(P, K, c64);
+std::string jit_ptx(const FProg& P, int K, bool c64, int nt) {
+  Gen g(P, K, c64, nt);
   return g.build();
 }
 
@@ -1154,10 +1160,10 @@ std::string jit_ptx(const FProg& P, int K, bool c64) {
 // coefficient component its class (0, +1, -1, other; the generator specialises
 // exact zeros and ones) -- but not the coefficient values, which are a kernel
 // parameter.  Building the key costs O(program), not a PTX generation.
-std::string jit_key(const FProg& P, int K, bool c64) {
+std::string jit_key(const FProg& P, int K, bool c64, int nt) {
   std::string k;
   k.reserve(64 + P.nops * sizeof(FHdr) + P.ncoef);
-  const int head[4] = {K, c64 ? 1 : 0, P.nops, P.ncoef};
+  const int head[5] = {K, c64 ? 1 : 0, P.nops, P.ncoef, nt};
   k.append(reinterpret_cast<const char*>(head), sizeof head);
   k.append(reinterpret_cast<const char*>(&P.tile), sizeof P.tile);
   k.append(reinterpret_cast<const char*>(P.h), sizeof(FHdr) * P.nops);
@@ -1174,7 +1180,8 @@ std::string jit_key(const FProg& P, int K, bool c64) {
   return k;
 }
 
-void jit_compile(const std::vector<std::pair<std::string, const FProg*>>& items, int K, bool c64) {
+void jit_compile(const std::vector<std::pair<std::string, const FProg*>>& items, int K, bool c64,
+                 int nt) {
   struct Todo {
     const std::string* key;
     const FProg* prog;
@@ -1198,7 +1205,7 @@ void jit_compile(const std::vector<std::pair<std::string, const FProg*>>& items,
   const char* dump = std::getenv("LFQS_JIT_DUMP");  // debugging aid: write the PTX
   auto work = [&] {
     for (size_t i; (i = next.fetch_add(1)) < todo.size();) {
-      const std::string ptx = jit_ptx(*todo[i].prog, K, c64);
+      const std::string ptx = jit_ptx(*todo[i].prog, K, c64, nt);
       if (dump) {
         const std::string fn = std::string(dump) + "/pass_" +
                                std::to_string(std::hash<std::string>()(ptx)) + ".ptx";
@@ -1224,12 +1231,16 @@ void jit_compile(const std::vector<std::pair<std::string, const FProg*>>& items,
     }
 }
 
+int jit_threads(const LaunchCtx& ctx, int K) {
+  return (ctx.opt->jit_threads == 512 && K >= 9) ? 512 : 256;
+}
+
 size_t jit_cache_size() {
   std::lock_guard<std::mutex> lk(g_mu);
   return g_cache.size();
 }
 
-void jit_launch(const LaunchCtx& ctx, const FProg& P, int K, const std::string& key) {
+void jit_launch(const LaunchCtx& ctx, const FProg& P, int K, const std::string& key, int nt) {
   std::shared_ptr<Entry> en;
   {
     std::lock_guard<std::mutex> lk(g_mu);
@@ -1237,7 +1248,7 @@ void jit_launch(const LaunchCtx& ctx, const FProg& P, int K, const std::string& 
     if (it != g_cache.end()) en = it->second;
   }
   if (!en) {
-    jit_compile({{key, &P}}, K, ctx.c64);
+    jit_compile({{key, &P}}, K, ctx.c64, nt);
     std::lock_guard<std::mutex> lk(g_mu);
     en = g_cache.at(key);
   }
@@ -1267,7 +1278,7 @@ void jit_launch(const LaunchCtx& ctx, const FProg& P, int K, const std::string& 
   void* a = ctx.amps;
   void* args[2] = {&a, (void*)P.c};
   const uint64_t tiles = 1ull << (ctx.n_local - K);
-  LFQS_CUDA_CHECK(cudaLaunchKernel((const void*)en->kern, dim3((unsigned)tiles), dim3(kFThreads),
+  LFQS_CUDA_CHECK(cudaLaunchKernel((const void*)en->kern, dim3((unsigned)tiles), dim3(nt),
                                    args, (size_t)smem, ctx.stream));
 }
 

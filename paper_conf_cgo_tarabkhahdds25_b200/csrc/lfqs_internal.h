@@ -90,6 +90,7 @@ struct Options {
   // beats direct loads for every chunk count up to 128, so TMA is the default.
   int fuse_tma_max_chunks = 256;
   int items_per_thread = 0;  // 0 = library default
+  int jit_threads = 256;     // threads per CTA of compiled passes (256 or 512)
 };
 
 // One launch worth of work on a contiguous shard.

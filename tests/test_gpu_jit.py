@@ -25,9 +25,10 @@ def L():
     return lib
 
 
-def _run(L, n, psi, gates, fuse, tile=None, low=None, c64=False, reorder=1):
+def _run(L, n, psi, gates, fuse, tile=None, low=None, c64=False, reorder=1, threads=256):
     with L.State.create(n, c64=c64) as st:
         st.set_option(L.OPT_FUSE_REORDER, reorder)
+        st.set_option(L.OPT_JIT_THREADS, threads)
         if tile:
             st.set_option(L.OPT_FUSE_TILE_QUBITS, tile)
         if low:
@@ -56,6 +57,22 @@ def test_jit_equals_interpreter(L, n, tile, low, reorder):
     assert np.array_equal(a, b)
     ref = O.run_circuit(n, gates, psi.copy())
     assert np.max(np.abs(b - ref)) <= 1e-12
+
+
+@pytest.mark.parametrize("threads", [256, 512])
+@pytest.mark.parametrize("tile", [9, 10, 12])
+@pytest.mark.parametrize("n", [13, 16])
+def test_jit_512_threads_equals_interpreter(L, n, tile, threads):
+    """Compiled passes with 512 threads per CTA (LFQS_OPT_JIT_THREADS): a different
+    thread/register placement of the same per-amplitude arithmetic."""
+    psi = W.random_state(n, 3 * n + tile)
+    gates = _mixed(n, 2000 + n + tile)
+    a, _ = _run(L, n, psi, gates, True, tile)
+    b, _ = _run(L, n, psi, gates, "jit", tile, threads=threads)
+    assert np.array_equal(a, b)
+    c, _ = _run(L, n, psi, gates, "phase", tile)
+    d, _ = _run(L, n, psi, gates, "jit+phase", tile, threads=threads)
+    assert np.array_equal(c, d)
 
 
 @pytest.mark.parametrize("tile", [9, 12])

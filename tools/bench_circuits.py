@@ -60,6 +60,7 @@ def main():
     ap.add_argument("--tile", type=int, default=0)
     ap.add_argument("--low", type=int, default=0)
     ap.add_argument("--reorder", type=int, default=1)
+    ap.add_argument("--jit-threads", type=int, default=256, help="LFQS_OPT_JIT_THREADS (256/512)")
     ap.add_argument("--c64", action="store_true", help="complex64 state (NEXT-4)")
     ap.add_argument("--world", type=int, default=1,
                     help="virtual partition into this many shards (the sharded planner and "
@@ -100,6 +101,7 @@ def main():
         if args.tma >= 0:
             st.set_option(L.OPT_FUSE_TMA_MAX_CHUNKS, args.tma)
         st.set_option(L.OPT_FUSE_REORDER, args.reorder)
+        st.set_option(L.OPT_JIT_THREADS, args.jit_threads)
         for name in args.circuits.split(","):
             gates, init, meta = circuits[name]
             arr = L.marshal_gates(gates)
