@@ -1198,9 +1198,9 @@ void jit_compile(const std::vector<std::pair<std::string, const FProg*>>& items,
     }
   }
   if (todo.empty()) return;
-  unsigned nt = std::thread::hardware_concurrency();
-  if (nt == 0) nt = 4;
-  if (nt > todo.size()) nt = (unsigned)todo.size();
+  unsigned nth = std::thread::hardware_concurrency();
+  if (nth == 0) nth = 4;
+  if (nth > todo.size()) nth = (unsigned)todo.size();
   std::atomic<size_t> next{0};
   const char* dump = std::getenv("LFQS_JIT_DUMP");  // debugging aid: write the PTX
   auto work = [&] {
@@ -1219,7 +1219,7 @@ void jit_compile(const std::vector<std::pair<std::string, const FProg*>>& items,
     }
   };
   std::vector<std::thread> th;
-  for (unsigned t = 1; t < nt; ++t) th.emplace_back(work);
+  for (unsigned t = 1; t < nth; ++t) th.emplace_back(work);
   work();
   for (auto& t : th) t.join();
   for (auto& t : todo)
