@@ -89,8 +89,10 @@ struct FH_ {
     a0 = mk<S>(s * (x0.x + x1.x), s * (x0.y + x1.y));
     a1 = mk<S>(s * (x0.x - x1.x), s * (x0.y - x1.y));
   }
+  // bit ? s (p - a) : s (a + p), written as s (p + (+-a)) -- the same values.
   __device__ __forceinline__ cx<S> lane(cx<S> a, cx<S> p, int bit) const {
-    return bit ? mk<S>(s * (p.x - a.x), s * (p.y - a.y)) : mk<S>(s * (a.x + p.x), s * (a.y + p.y));
+    const S ax = bit ? -a.x : a.x, ay = bit ? -a.y : a.y;
+    return mk<S>(s * (p.x + ax), s * (p.y + ay));
   }
 };
 template <class S>
@@ -105,15 +107,12 @@ struct FU_ {
     a0 = b0;
     a1 = b1;
   }
+  // Own amplitude first, partner second, in both lanes: only the coefficients
+  // depend on the lane bit (the compiled passes select them once per op).
   __device__ __forceinline__ cx<S> lane(cx<S> a, cx<S> p, int bit) const {
     cx<S> acc = mk<S>(0, 0);
-    if (bit) {
-      cfma(acc, c2, p);
-      cfma(acc, c3, a);
-    } else {
-      cfma(acc, c0, a);
-      cfma(acc, c1, p);
-    }
+    cfma(acc, bit ? c3 : c0, a);
+    cfma(acc, bit ? c2 : c1, p);
     return acc;
   }
 };
@@ -126,8 +125,8 @@ struct FR_ {  // real 2x2 [[m00, m01], [m10, m11]]
     a1 = mk<S>(fma_(m11, x1.x, m10 * x0.x), fma_(m11, x1.y, m10 * x0.y));
   }
   __device__ __forceinline__ cx<S> lane(cx<S> a, cx<S> p, int bit) const {
-    return bit ? mk<S>(fma_(m11, a.x, m10 * p.x), fma_(m11, a.y, m10 * p.y))
-               : mk<S>(fma_(m01, p.x, m00 * a.x), fma_(m01, p.y, m00 * a.y));
+    const S A = bit ? m11 : m00, B = bit ? m10 : m01;  // own, partner coefficient
+    return mk<S>(fma_(B, p.x, A * a.x), fma_(B, p.y, A * a.y));
   }
 };
 template <class S>
@@ -139,8 +138,8 @@ struct FI_ {  // [[d0, i e01], [i e10, d1]] with real d0, d1, e01, e10
     a1 = mk<S>(fma_(d1, x1.x, -e10 * x0.y), fma_(d1, x1.y, e10 * x0.x));
   }
   __device__ __forceinline__ cx<S> lane(cx<S> a, cx<S> p, int bit) const {
-    return bit ? mk<S>(fma_(d1, a.x, -e10 * p.y), fma_(d1, a.y, e10 * p.x))
-               : mk<S>(fma_(-e01, p.y, d0 * a.x), fma_(e01, p.x, d0 * a.y));
+    const S D = bit ? d1 : d0, E = bit ? e10 : e01;  // own diagonal, partner (imaginary) entry
+    return mk<S>(fma_(-E, p.y, D * a.x), fma_(E, p.x, D * a.y));
   }
 };
 

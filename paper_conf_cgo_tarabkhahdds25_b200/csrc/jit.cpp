@@ -382,8 +382,37 @@ struct Gen {
       }
     }
   }
-  // Lane form: amplitude a, partner p, runtime bit predicate `bit` (bit == 1).
-  Cx lane(const Op2& o, const Cx& a, const Cx& pp, const std::string& bit) {
+  // Lane form: amplitude a, partner p, runtime bit predicate `bit` (bit == 1);
+  // k_fused's FX_/FY_/FH_/FR_/FI_/FU_ lane(): only the coefficients depend on the
+  // lane bit, selected once per op (lane_coefs), so no per-amplitude selects
+  // except the sign of H and the permutation of Y.
+  struct LaneC {
+    std::string A, B, D, E, nE;  // F_UR: own A, partner B; F_UI: own D, partner E
+    Cx m1, n1, m2, n2;           // F_U2: own m1, partner m2 (n*.x = -m*.y)
+  };
+  LaneC lane_coefs(const Op2& o, const std::string& bit) {
+    LaneC l;
+    switch (o.type) {
+      case F_UR:
+        l.A = sel(o.m11, o.m00, bit);
+        l.B = sel(o.m10, o.m01, bit);
+        break;
+      case F_UI:
+        l.D = sel(o.d1, o.d0, bit);
+        l.E = sel(o.e10, o.e01, bit);
+        l.nE = neg(l.E);
+        break;
+      case F_U2:
+        l.m1 = sel_c(o.c3, o.c0, bit);
+        l.n1 = {sel(o.n3.x, o.n0.x, bit), ""};
+        l.m2 = sel_c(o.c2, o.c1, bit);
+        l.n2 = {sel(o.n2.x, o.n1.x, bit), ""};
+        break;
+      default: break;
+    }
+    return l;
+  }
+  Cx lane(const Op2& o, const LaneC& l, const Cx& a, const Cx& pp, const std::string& bit) {
     switch (o.type) {
       case F_X: return pp;
       case F_Y: {
@@ -392,38 +421,18 @@ struct Gen {
         return {sel(npy, pp.y, bit), sel(pp.x, npx, bit)};
       }
       case F_H: {
-        // bit ? s (p - a) : s (a + p)
-        const std::string sx = sel(sub(pp.x, a.x), add(a.x, pp.x), bit);
-        const std::string sy = sel(sub(pp.y, a.y), add(a.y, pp.y), bit);
-        return {mul(o.s, sx), mul(o.s, sy)};
+        // s (p + (bit ? -a : a))
+        const std::string ax = sel(neg(a.x), a.x, bit), ay = sel(neg(a.y), a.y, bit);
+        return {mul(o.s, add(pp.x, ax)), mul(o.s, add(pp.y, ay))};
       }
-      case F_UR: {
-        // bit ? (fma(m11, a, m10 p)) : (fma(m01, p, m00 a))
-        const std::string k1 = sel(o.m11, o.m01, bit), k2 = sel(o.m10, o.m00, bit);
-        const std::string y1x = sel(a.x, pp.x, bit), y1y = sel(a.y, pp.y, bit);
-        const std::string y2x = sel(pp.x, a.x, bit), y2y = sel(pp.y, a.y, bit);
-        return {fma(k1, y1x, mul(k2, y2x)), fma(k1, y1y, mul(k2, y2y))};
-      }
-      case F_UI: {
-        // bit ? (fma(d1, a.x, -e10 p.y), fma(d1, a.y, e10 p.x))
-        //     : (fma(-e01, p.y, d0 a.x), fma(e01, p.x, d0 a.y))
-        const std::string ne01 = neg(o.e01), ne10 = neg(o.e10);
-        const std::string rk1 = sel(o.d1, ne01, bit), rk2 = sel(ne10, o.d0, bit);
-        const std::string ry1 = sel(a.x, pp.y, bit), ry2 = sel(pp.y, a.x, bit);
-        const std::string ik1 = sel(o.d1, o.e01, bit), ik2 = sel(o.e10, o.d0, bit);
-        const std::string iy1 = sel(a.y, pp.x, bit), iy2 = sel(pp.x, a.y, bit);
-        return {fma(rk1, ry1, mul(rk2, ry2)), fma(ik1, iy1, mul(ik2, iy2))};
-      }
-      default: {  // F_U2: bit ? c2 p + c3 a : c0 a + c1 p (accumulation order kept)
-        Cx m1 = sel_c(o.c2, o.c0, bit);
-        Cx n1{sel(o.n2.x, o.n0.x, bit), ""};
-        Cx m2 = sel_c(o.c3, o.c1, bit);
-        Cx n2{sel(o.n3.x, o.n1.x, bit), ""};
-        Cx v1{sel(pp.x, a.x, bit), sel(pp.y, a.y, bit)};
-        Cx v2{sel(a.x, pp.x, bit), sel(a.y, pp.y, bit)};
+      case F_UR:
+        return {fma(l.B, pp.x, mul(l.A, a.x)), fma(l.B, pp.y, mul(l.A, a.y))};
+      case F_UI:
+        return {fma(l.nE, pp.y, mul(l.D, a.x)), fma(l.E, pp.x, mul(l.D, a.y))};
+      default: {  // F_U2: own amplitude first, partner second
         Cx acc;
-        cfma(acc, m1, n1, v1, true);
-        cfma(acc, m2, n2, v2, false);
+        cfma(acc, l.m1, l.n1, a, true);
+        cfma(acc, l.m2, l.n2, pp, false);
         return acc;
       }
     }
@@ -576,10 +585,11 @@ struct Gen {
       const std::string bit = p(), a = r();
       e("and.b32 %s, %%ltid, %u;", a.c_str(), 1u << t0);
       e("setp.ne.b32 %s, %s, 0;", bit.c_str(), a.c_str());
+      const LaneC lc = lane_coefs(o, bit);
       for (int r = 0; r < R; ++r) {
         if (((uint32_t)r & mr) != pr) continue;
         const Cx pp = shfl({vx(r), vy(r)}, t0);
-        const Cx z = lane(o, {vx(r), vy(r)}, pp, bit);
+        const Cx z = lane(o, lc, {vx(r), vy(r)}, pp, bit);
         if (bt.empty()) {
           set(r, z);
         } else {
