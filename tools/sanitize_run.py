@@ -1,6 +1,7 @@
 """Small-n workload for compute-sanitizer (memcheck / racecheck / synccheck):
 every kernel family once -- class kernels, shuffle path, fused TMA and direct
-tiles (incl. smem ops), virtual-partition exchange, probabilities, collapse.
+tiles (incl. smem ops), compiled passes (LFQS_FUSE_JIT, with phase tables, 256 and
+512 threads), SOA kernels, virtual-partition exchange, probabilities, collapse.
 
     compute-sanitizer --tool racecheck python tools/sanitize_run.py
 """
@@ -28,11 +29,20 @@ def main():
         for tma in (256, 0):
             st.set_option(L.OPT_FUSE_TMA_MAX_CHUNKS, tma)
             st.run_circuit(gates, fuse=True)
+        for threads in (256, 512):
+            st.set_option(L.OPT_JIT_THREADS, threads)
+            st.run_circuit(gates, fuse="jit")
+            st.run_circuit(gates, fuse="jit+phase")
         st.measure_probs([0, 3, 13])
         st.measure_probs(list(range(12)))
         st.sample([1, 2], np.linspace(0, 0.99, 7))
         st.collapse([5], 1)
         st.synchronize()
+    with L.State.create(n, soa=True) as st:
+        st.init_random(3)
+        st.run_circuit(gates)
+        st.measure_probs([0, 1])
+        st.collapse([0], 0)
     with L.State.virtual(n, 4) as st:
         st.init_random(2)
         st.run_circuit(gates, fuse=True)
