@@ -322,6 +322,10 @@ lfqs_status lfqs_kernel_launches(const lfqs_state* s, uint64_t* count);
                                    with the skipped ones (default 1); 0: prefixes only */
 #define LFQS_OPT_JIT_THREADS 8 /* threads per CTA of LFQS_FUSE_JIT passes: 256 (default) or 512
                                    (twice the warps per SM, half the amplitudes per thread) */
+#define LFQS_OPT_JIT_LANE_MOVE 9 /* 1: compiled passes may move the lane tile bits >= 3
+                                     (complex64: >= 4) into register positions, so 1-target
+                                     gates on them run in registers instead of by warp
+                                     shuffles; bit-identical results either way */
 lfqs_status lfqs_set_option(lfqs_state* s, int option, int64_t value);
 const char* lfqs_last_error(void);
 int lfqs_abi_version(void);

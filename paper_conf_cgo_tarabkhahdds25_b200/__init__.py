@@ -38,6 +38,7 @@ OPT_FUSE_LOW_QUBITS = 5
 OPT_FUSE_TMA_MAX_CHUNKS = 6
 OPT_FUSE_REORDER = 7
 OPT_JIT_THREADS = 8
+OPT_JIT_LANE_MOVE = 9
 
 STATUS = {0: "OK", -1: "INVALID_ARG", -2: "OUT_OF_MEMORY", -3: "CUDA", -4: "NCCL",
           -5: "UNSUPPORTED"}

@@ -888,8 +888,8 @@ void build_program(const LaunchCtx& ctx, const TileCfg& cfg, uint64_t in_tile,
 // or the interpreting kernel k_fused<K>.
 void launch_built(const LaunchCtx& ctx, int K, const FProg& P, const std::string* key = nullptr) {
   if (ctx.jit && (1 << P.tile.nh) <= ctx.opt->fuse_tma_max_chunks) {
-    const int nt = jit_threads(ctx, K);
-    jit_launch(ctx, P, K, key ? *key : jit_key(P, K, ctx.c64, nt), nt);
+    const int jc = jit_config(ctx, K);
+    jit_launch(ctx, P, K, key ? *key : jit_key(P, K, ctx.c64, jc), jc);
     ++*ctx.launch_counter;
     return;
   }
@@ -1026,7 +1026,7 @@ void run_fused_schedule(const LaunchCtx& ctx, const std::vector<Decoded>& gates,
         passes.emplace_back();
         passes.back().prog.reset(new FProg);
         build_program(ctx, cfg, in_tile, list, *passes.back().prog);
-        passes.back().key = jit_key(*passes.back().prog, cfg.K, ctx.c64, jit_threads(ctx, cfg.K));
+        passes.back().key = jit_key(*passes.back().prog, cfg.K, ctx.c64, jit_config(ctx, cfg.K));
       } else {
         launch_program(ctx, cfg, in_tile, list);
       }
@@ -1038,7 +1038,7 @@ void run_fused_schedule(const LaunchCtx& ctx, const std::vector<Decoded>& gates,
   std::vector<std::pair<std::string, const FProg*>> items;
   for (const Pass& ps : passes)
     if (ps.prog) items.emplace_back(ps.key, ps.prog.get());
-  jit_compile(items, cfg.K, ctx.c64, jit_threads(ctx, cfg.K));
+  jit_compile(items, cfg.K, ctx.c64, jit_config(ctx, cfg.K));
   if (ctx.dry_run) {
     *ctx.launch_counter += passes.size();
     return;

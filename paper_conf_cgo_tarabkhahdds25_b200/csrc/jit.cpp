@@ -55,28 +55,34 @@ struct Gen {
   int nr = 0, nrd = 0, nf = 0, np = 0, nl = 0;
   bool in_regs = true;
 
-  // Placement of tile bits in (thread, slot): tile bits 0..4 are the lane bits
-  // (fixed: warp accesses stay contiguous); the other K-5 tile bits sit at the 3
-  // warp positions (thread bits 5..7) or at the K-8 register positions (slot bits).
+  // Placement of tile bits in (thread, slot): thread bit j holds tile bit tpos[j],
+  // slot bit j holds rpos[j].  The low FL lane bits always hold tile bits 0..FL-1, so
+  // the 16-B (8-B for complex64) shared-memory accesses of a quarter-warp (half-warp)
+  // cover distinct banks; FL = 5 unless lane moves are on (LFQS_OPT_JIT_LANE_MOVE),
+  // then lane bits FL..4 are movable like the 3 warp positions (thread bits 5..7).
   // The interpreter's placement is the identity; the compiled pass moves a tile bit
   // into a register position (a tile round trip, `remap`) when a gate needs it
-  // there, so 1-target gates on warp bits and multi-target gates on register bits
-  // run in registers instead of as shared-memory ops.  Every amplitude still sees
-  // the same arithmetic, so results stay bit-identical to the interpreter.
+  // there, so 1-target gates on warp bits (and, with lane moves, on lane bits >= FL)
+  // and multi-target gates on movable bits run in registers instead of as
+  // shared-memory ops or shuffles.  Every amplitude still sees the same arithmetic
+  // (a moved lane bit keeps the interpreter's lane formulas), so results stay
+  // bit-identical to the interpreter.
   int NT = 256;   // threads per CTA (256, or 512 for K >= 9: twice the warps per SM)
   int NWB = 3;    // warp bits of the thread index
-  int wpos[4] = {5, 6, 7, 8};
+  int FL = 5;     // fixed lane bits
+  int tpos[9] = {0, 1, 2, 3, 4, 5, 6, 7, 8};
   int rpos[4] = {8, 9, 10, 11};
   int nreg = 0;
 
-  Gen(const FProg& p, int k, bool c, int nt) : P(p), K(k), c64(c) {
+  Gen(const FProg& p, int k, bool c, int jc) : P(p), K(k), c64(c) {
     FT = c64 ? "f32" : "f64";
     ES = c64 ? 8 : 16;
-    NT = nt;
+    NT = jc & JIT_THREADS_MASK;
     NWB = NT == 512 ? 4 : 3;
     R = (1 << K) / NT;
     nreg = K - 5 - NWB;
-    for (int j = 0; j < NWB; ++j) wpos[j] = 5 + j;
+    FL = ((jc & JIT_LANE_MOVE) && nreg >= 1) ? (c64 ? 4 : 3) : 5;
+    for (int j = 0; j < 5 + NWB; ++j) tpos[j] = j;
     for (int j = 0; j < nreg; ++j) rpos[j] = 5 + NWB + j;
   }
 
@@ -87,10 +93,14 @@ struct Gen {
   }
   // Thread bit holding tile bit b, or -1 when b is register-held.
   int tbit(int b) const {
-    if (b < 5) return b;
-    for (int j = 0; j < NWB; ++j)
-      if (wpos[j] == b) return 5 + j;
+    for (int j = 0; j < 5 + NWB; ++j)
+      if (tpos[j] == b) return j;
     return -1;
+  }
+  // Tile bit b sits at a fixed lane position (shuffle path only).
+  bool fixed_lane(int b) const {
+    const int t = tbit(b);
+    return t >= 0 && t < FL;
   }
   // (i & m) == v split into a thread part and a slot part.
   void split(uint32_t m, uint32_t v, uint32_t& tm, uint32_t& tv, uint32_t& rm, uint32_t& rv) const {
@@ -119,11 +129,11 @@ struct Gen {
   // %taddr = tile + ES * (thread part of the tile index).
   void emit_taddr() {
     const std::string t = r();
-    e("and.b32 %s, %%ltid, 31;", t.c_str());
-    for (int j = 0; j < NWB; ++j) {
+    e("and.b32 %s, %%ltid, %d;", t.c_str(), (1 << FL) - 1);
+    for (int j = FL; j < 5 + NWB; ++j) {
       const std::string x = r();
-      e("bfe.u32 %s, %%ltid, %d, 1;", x.c_str(), 5 + j);
-      e("shl.b32 %s, %s, %d;", x.c_str(), x.c_str(), wpos[j]);
+      e("bfe.u32 %s, %%ltid, %d, 1;", x.c_str(), j);
+      e("shl.b32 %s, %s, %d;", x.c_str(), x.c_str(), tpos[j]);
       e("or.b32 %s, %s, %s;", t.c_str(), t.c_str(), x.c_str());
     }
     e("mad.lo.u32 %%taddr, %s, %d, %%tile;", t.c_str(), ES);
@@ -438,6 +448,35 @@ struct Gen {
     }
   }
 
+  // lane() with the lane bit known at generation time (a lane tile bit moved into
+  // a register position): the same operations with the selections resolved.
+  Cx lane_const(const Op2& o, const Cx& a, const Cx& pp, int bit) {
+    switch (o.type) {
+      case F_X: return pp;
+      case F_Y: return bit ? Cx{neg(pp.y), pp.x} : Cx{pp.y, neg(pp.x)};
+      case F_H: {
+        const std::string ax = bit ? neg(a.x) : a.x, ay = bit ? neg(a.y) : a.y;
+        return {mul(o.s, add(pp.x, ax)), mul(o.s, add(pp.y, ay))};
+      }
+      case F_UR: {
+        const std::string& A = bit ? o.m11 : o.m00;
+        const std::string& B = bit ? o.m10 : o.m01;
+        return {fma(B, pp.x, mul(A, a.x)), fma(B, pp.y, mul(A, a.y))};
+      }
+      case F_UI: {
+        const std::string& D = bit ? o.d1 : o.d0;
+        const std::string& E = bit ? o.e10 : o.e01;
+        return {fma(neg(E), pp.y, mul(D, a.x)), fma(E, pp.x, mul(D, a.y))};
+      }
+      default: {  // F_U2: own amplitude first, partner second
+        Cx acc;
+        cfma(acc, bit ? o.c3 : o.c0, bit ? o.n3 : o.n0, a, true);
+        cfma(acc, bit ? o.c2 : o.c1, bit ? o.n2 : o.n1, pp, false);
+        return acc;
+      }
+    }
+  }
+
   Cx shfl(const Cx& v, int t0) {
     Cx o{f(), f()};
     for (int c = 0; c < 2; ++c) {
@@ -569,7 +608,7 @@ struct Gen {
     uint32_t tm_, tv_, mr, pr;
     split(h.mlo, h.plo, tm_, tv_, mr, pr);
     const std::string bt = thread_pred(h.mlo, h.plo);
-    if (t0 >= 5) {  // register-held (remapped there if it was a warp bit)
+    if (reg_of(t0) >= 0) {  // register-held (remapped there if it was a warp/lane bit)
       const int rb = reg_of(t0);
       skip_unless(bt, end);
       for (int r = 0; r < R; ++r) {
@@ -577,18 +616,25 @@ struct Gen {
         if (((uint32_t)r & mr) != pr) continue;
         // Snapshot the slot registers: pair() may return them swapped (X, Y).
         Cx a0 = copy({vx(r), vy(r)}), a1 = copy({vx(r | (1 << rb)), vy(r | (1 << rb))});
-        pair(o, a0, a1);
+        if (t0 < 5) {  // a lane bit of the interpreter: its lane formulas
+          const Cx z0 = lane_const(o, a0, a1, 0), z1 = lane_const(o, a1, a0, 1);
+          a0 = z0;
+          a1 = z1;
+        } else {
+          pair(o, a0, a1);
+        }
         set(r, a0);
         set(r | (1 << rb), a1);
       }
     } else {
+      const int tl = tbit(t0);  // a fixed lane position
       const std::string bit = p(), a = r();
-      e("and.b32 %s, %%ltid, %u;", a.c_str(), 1u << t0);
+      e("and.b32 %s, %%ltid, %u;", a.c_str(), 1u << tl);
       e("setp.ne.b32 %s, %s, 0;", bit.c_str(), a.c_str());
       const LaneC lc = lane_coefs(o, bit);
       for (int r = 0; r < R; ++r) {
         if (((uint32_t)r & mr) != pr) continue;
-        const Cx pp = shfl({vx(r), vy(r)}, t0);
+        const Cx pp = shfl({vx(r), vy(r)}, tl);
         const Cx z = lane(o, lc, {vx(r), vy(r)}, pp, bit);
         if (bt.empty()) {
           set(r, z);
@@ -895,8 +941,7 @@ struct Gen {
           best = j;
         }
       }
-      const int w = tbit(b) - 5;
-      wpos[w] = rpos[best];
+      tpos[tbit(b)] = rpos[best];
       rpos[best] = b;
     }
     sync();
@@ -1025,15 +1070,16 @@ struct Gen {
       int ts[3];
       const int m = op_targets(h, ts);
       bool any_lane = false;
-      for (int s_ = 0; s_ < m; ++s_) any_lane |= ts[s_] < 5;
-      // 1-target gates: lane bits by shuffle, everything else in registers (a warp
-      // bit is first moved into a register position).  Multi-target gates: in
-      // registers when no target is a lane bit and they fit the register positions.
-      const bool in_reg_path = m == 1 ? (ts[0] < 5 || nreg >= 1) : (!any_lane && m <= nreg);
+      for (int s_ = 0; s_ < m; ++s_) any_lane |= fixed_lane(ts[s_]);
+      // 1-target gates: fixed lane bits by shuffle, everything else in registers (a
+      // warp or movable lane bit is first moved into a register position).
+      // Multi-target gates: in registers when no target is at a fixed lane position
+      // and they fit the register positions.
+      const bool in_reg_path = m == 1 ? (any_lane || nreg >= 1) : (!any_lane && m <= nreg);
       if (in_reg_path) {
         std::vector<int> need;
         for (int s_ = 0; s_ < m; ++s_)
-          if (ts[s_] >= 5 && reg_of(ts[s_]) < 0) need.push_back(ts[s_]);
+          if (!fixed_lane(ts[s_]) && reg_of(ts[s_]) < 0) need.push_back(ts[s_]);
         if (!need.empty()) remap(need, ts, m, o);
         ensure_regs();
         if (m == 1)
@@ -1161,8 +1207,8 @@ void compile_entry(const std::string& ptx, Entry& en) {
 
 }  // namespace
 
-std::string jit_ptx(const FProg& P, int K, bool c64, int nt) {
-  Gen g(P, K, c64, nt);
+std::string jit_ptx(const FProg& P, int K, bool c64, int jc) {
+  Gen g(P, K, c64, jc);
   return g.build();
 }
 
@@ -1170,10 +1216,10 @@ std::string jit_ptx(const FProg& P, int K, bool c64, int nt) {
 // coefficient component its class (0, +1, -1, other; the generator specialises
 // exact zeros and ones) -- but not the coefficient values, which are a kernel
 // parameter.  Building the key costs O(program), not a PTX generation.
-std::string jit_key(const FProg& P, int K, bool c64, int nt) {
+std::string jit_key(const FProg& P, int K, bool c64, int jc) {
   std::string k;
   k.reserve(64 + P.nops * sizeof(FHdr) + P.ncoef);
-  const int head[5] = {K, c64 ? 1 : 0, P.nops, P.ncoef, nt};
+  const int head[5] = {K, c64 ? 1 : 0, P.nops, P.ncoef, jc};
   k.append(reinterpret_cast<const char*>(head), sizeof head);
   k.append(reinterpret_cast<const char*>(&P.tile), sizeof P.tile);
   k.append(reinterpret_cast<const char*>(P.h), sizeof(FHdr) * P.nops);
@@ -1191,7 +1237,7 @@ std::string jit_key(const FProg& P, int K, bool c64, int nt) {
 }
 
 void jit_compile(const std::vector<std::pair<std::string, const FProg*>>& items, int K, bool c64,
-                 int nt) {
+                 int jc) {
   struct Todo {
     const std::string* key;
     const FProg* prog;
@@ -1215,7 +1261,7 @@ void jit_compile(const std::vector<std::pair<std::string, const FProg*>>& items,
   const char* dump = std::getenv("LFQS_JIT_DUMP");  // debugging aid: write the PTX
   auto work = [&] {
     for (size_t i; (i = next.fetch_add(1)) < todo.size();) {
-      const std::string ptx = jit_ptx(*todo[i].prog, K, c64, nt);
+      const std::string ptx = jit_ptx(*todo[i].prog, K, c64, jc);
       if (dump) {
         const std::string fn = std::string(dump) + "/pass_" +
                                std::to_string(std::hash<std::string>()(ptx)) + ".ptx";
@@ -1241,8 +1287,9 @@ void jit_compile(const std::vector<std::pair<std::string, const FProg*>>& items,
     }
 }
 
-int jit_threads(const LaunchCtx& ctx, int K) {
-  return (ctx.opt->jit_threads == 512 && K >= 9) ? 512 : 256;
+int jit_config(const LaunchCtx& ctx, int K) {
+  return ((ctx.opt->jit_threads == 512 && K >= 9) ? 512 : 256) |
+         (ctx.opt->jit_lane_move ? JIT_LANE_MOVE : 0);
 }
 
 size_t jit_cache_size() {
@@ -1250,7 +1297,8 @@ size_t jit_cache_size() {
   return g_cache.size();
 }
 
-void jit_launch(const LaunchCtx& ctx, const FProg& P, int K, const std::string& key, int nt) {
+void jit_launch(const LaunchCtx& ctx, const FProg& P, int K, const std::string& key, int jc) {
+  const int nt = jc & JIT_THREADS_MASK;
   std::shared_ptr<Entry> en;
   {
     std::lock_guard<std::mutex> lk(g_mu);
@@ -1258,7 +1306,7 @@ void jit_launch(const LaunchCtx& ctx, const FProg& P, int K, const std::string& 
     if (it != g_cache.end()) en = it->second;
   }
   if (!en) {
-    jit_compile({{key, &P}}, K, ctx.c64, nt);
+    jit_compile({{key, &P}}, K, ctx.c64, jc);
     std::lock_guard<std::mutex> lk(g_mu);
     en = g_cache.at(key);
   }

@@ -9,17 +9,22 @@
 
 namespace lfqs {
 
+// Generator configuration `jc` of a compiled pass: threads per CTA (low bits) and
+// variant flags.
+constexpr int JIT_THREADS_MASK = 0xffff;
+constexpr int JIT_LANE_MOVE = 1 << 16;  // lane bits >= 3 (c64: >= 4) movable (LFQS_OPT_JIT_LANE_MOVE)
+
 // PTX of one fused pass: structure baked in, coefficients a kernel parameter.
-std::string jit_ptx(const FProg& P, int K, bool c64, int nt);
+std::string jit_ptx(const FProg& P, int K, bool c64, int jc);
 // Cache key of a pass (its structure and coefficient classes, not values).
-std::string jit_key(const FProg& P, int K, bool c64, int nt);
+std::string jit_key(const FProg& P, int K, bool c64, int jc);
 // Generates and compiles (in parallel, nvPTXCompiler) every pass not yet cached.
 void jit_compile(const std::vector<std::pair<std::string, const FProg*>>& items, int K, bool c64,
-                 int nt);
+                 int jc);
 // Launches the pass (compiling it first if needed) on ctx.stream.
-void jit_launch(const LaunchCtx& ctx, const FProg& P, int K, const std::string& key, int nt);
-// Threads per CTA of a compiled pass for tile size K (LFQS_OPT_JIT_THREADS).
-int jit_threads(const LaunchCtx& ctx, int K);
+void jit_launch(const LaunchCtx& ctx, const FProg& P, int K, const std::string& key, int jc);
+// Generator configuration for tile size K (LFQS_OPT_JIT_THREADS, LFQS_OPT_JIT_LANE_MOVE).
+int jit_config(const LaunchCtx& ctx, int K);
 size_t jit_cache_size();
 
 }  // namespace lfqs
