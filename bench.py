@@ -169,6 +169,38 @@ def cpu_baseline(n: int, budget_s: float = 15.0):
     return res
 
 
+def oracle_circuit_prefix(n: int, gates, budget_s: float) -> dict:
+    """cpu_baseline for the macro circuits (tools/bench_circuits.py --oracle-s): the oracle as
+    it stands (tier B index loop, OpenMP static schedule on every host core) on the first
+    gates of the same circuit at the same n, from a seeded random host state, for about
+    budget_s seconds.  Needs 16 * 2^n B of host memory; beyond 45 % of MemAvailable it
+    reports why it did not run."""
+    import oracle
+    cores = oracle.omp_max_threads()
+    if 16.0 * 2 ** n > 0.45 * host_avail_gib() * 2 ** 30:
+        return {"unavailable": f"16*2^{n} B host state exceeds 45% of MemAvailable "
+                               f"({host_avail_gib():.0f} GiB)", "cores": cores}
+    st = oracle.fill_random(0x0AC1E, 0, 1 << n)
+    done, t0 = 0, time.perf_counter()
+    while done < len(gates) and time.perf_counter() - t0 < budget_s:
+        oracle.apply_gate(n, gates[done], st, omp=True)
+        done += 1
+    t = time.perf_counter() - t0
+    del st
+    return {"gates_per_s": done / t, "gates": done, "of": len(gates), "s": t, "cores": cores,
+            "kind": "oracle tier B (OpenMP), circuit prefix"}
+
+
+def oracle_circuit_time(n: int, gates, psi) -> float:
+    """Seconds the oracle (tier B, one host thread) takes for a whole small circuit
+    (configs[0], tools/bench_small.py)."""
+    import oracle
+    oracle.build()
+    t0 = time.perf_counter()
+    oracle.run_circuit(n, gates, psi.copy())
+    return time.perf_counter() - t0
+
+
 def run_reference(args):
     rank = int(os.environ.get("RANK", "0"))
     if rank != 0:

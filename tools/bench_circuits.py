@@ -18,6 +18,7 @@ sys.path.insert(0, ROOT)
 import numpy as np  # noqa: E402
 
 import workloads as W  # noqa: E402
+from bench import oracle_circuit_prefix, peaks  # noqa: E402  (bench.py's cpu_baseline leg)
 
 
 def sample_idx(n, count, seed):
@@ -68,6 +69,10 @@ def main():
                     help="virtual partition into this many shards (the sharded planner and "
                          "exchange kernels on one GPU)")
     ap.add_argument("--tma", type=int, default=-1, help="max chunks moved by TMA (-1: default)")
+    ap.add_argument("--oracle-s", type=float, default=0.0,
+                    help="time the CPU oracle (tier B, OpenMP on all host cores) on a prefix of "
+                         "each circuit for about this many seconds (SURVEY 8(d): oracle beside "
+                         "the GPU; 0 = off)")
     args = ap.parse_args()
     import torch
     import paper_conf_cgo_tarabkhahdds25_b200 as L
@@ -93,6 +98,7 @@ def main():
         "xhigh": ([W.Gate("X", (n - 1,)), W.Gate("X", (n - 5,))], lambda st: st.init_basis(0), {}),
     }
     ab = 8 if args.c64 else 16
+    peak, peak_src = peaks()
     st_ = (L.State.create(n, 0, stream=s, c64=args.c64) if args.world == 1 else
            L.State.virtual(n, args.world, 0, stream=s, c64=args.c64))
     with st_ as st:
@@ -109,6 +115,7 @@ def main():
         for name in args.circuits.split(","):
             gates, init, meta = circuits[name]
             arr = L.marshal_gates(gates)
+            orc = oracle_circuit_prefix(n, gates, args.oracle_s) if args.oracle_s > 0 else None
             for mode in args.modes.split(","):
                 flags = {"fused": L.FUSE_LOW, "phase": L.FUSE_LOW | L.FUSE_PHASE,
                          "jit": L.FUSE_LOW | L.FUSE_JIT,
@@ -141,10 +148,18 @@ def main():
                        "conv_GBps": 2.0 * ab * 2 ** n * len(gates) / (t / 1e3) / 1e9,
                        "pass_GBps": 2.0 * ab * 2 ** n * passes / (t / 1e3) / 1e9,
                        "dtype": "c64" if args.c64 else "c128", "world": args.world,
-                       "exchanges": x1 - x0, "lane_move": args.lane_move}
+                       "exchanges": x1 - x0, "lane_move": args.lane_move,
+                       "hbm_peak_GBps": peak, "peak_source": peak_src}
+                # fraction of the HBM roofline: per pass actually made, and against the
+                # north-star convention of one 2*16*2^n-byte pass per gate
+                rec["pass_frac"] = rec["pass_GBps"] / peak
+                rec["conv_frac"] = rec["conv_GBps"] / peak
                 if compile_s is not None:
                     rec["jit_compile_s"] = round(compile_s, 3)
                 rec.update(res)
+                if orc is not None:
+                    rec["oracle"] = orc
+                    rec["gpu_over_oracle"] = rec["gates_per_s"] / orc["gates_per_s"]
                 print(json.dumps(rec), flush=True)
 
 

@@ -76,11 +76,8 @@ def main():
         res["jit"] = timed(lambda: L.lfqs_run_circuit(st.h, arr, L.FUSE_LOW | L.FUSE_JIT), reps)
         with st.compile(arr, fuse="jit") as c:
             res["jgraph"] = timed(c.launch, reps)
-    import oracle as O
-    O.build()
-    t0 = time.perf_counter()
-    O.run_circuit(n, gates, psi.copy())
-    res["oracle"] = time.perf_counter() - t0
+    from bench import oracle_circuit_time  # bench.py's cpu_baseline leg
+    res["oracle"] = oracle_circuit_time(n, gates, psi)
     for mode, t in res.items():
         print(json.dumps({"config": "configs[0]", "n": n, "gates": len(gates), "mode": mode,
                           "s_per_circuit": t, "us_per_gate": t / len(gates) * 1e6,
