@@ -326,6 +326,12 @@ lfqs_status lfqs_kernel_launches(const lfqs_state* s, uint64_t* count);
                                      (complex64: >= 4) into register positions, so 1-target
                                      gates on them run in registers instead of by warp
                                      shuffles; bit-identical results either way */
+#define LFQS_OPT_FUSE_MERGE_COMMUTING 10 /* 1 (default): inside a fused pass, a 1-target gate
+                                     merges (host matrix product) into the last earlier gate
+                                     touching any of its qubits when that is a 1-target gate on
+                                     the same target with the same controls and one of the two
+                                     is dense; 0: only directly adjacent runs merge.  Changes
+                                     rounding only (dense tolerance class) */
 lfqs_status lfqs_set_option(lfqs_state* s, int option, int64_t value);
 const char* lfqs_last_error(void);
 int lfqs_abi_version(void);

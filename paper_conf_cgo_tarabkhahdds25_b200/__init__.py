@@ -39,6 +39,7 @@ OPT_FUSE_TMA_MAX_CHUNKS = 6
 OPT_FUSE_REORDER = 7
 OPT_JIT_THREADS = 8
 OPT_JIT_LANE_MOVE = 9
+OPT_FUSE_MERGE_COMMUTING = 10
 
 STATUS = {0: "OK", -1: "INVALID_ARG", -2: "OUT_OF_MEMORY", -3: "CUDA", -4: "NCCL",
           -5: "UNSUPPORTED"}

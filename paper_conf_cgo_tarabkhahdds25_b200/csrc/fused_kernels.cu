@@ -853,14 +853,28 @@ void build_program(const LaunchCtx& ctx, const TileCfg& cfg, uint64_t in_tile,
   require(b == K && lc + P.tile.nh == K, "internal: bad fused tile");
   // Merge runs of 1-target gates on the same qubit with the same controls when at
   // least one is dense (matrix product on the host; dense results are compared
-  // within rounding, permutation/diagonal-only runs are never merged).
+  // within rounding, permutation/diagonal-only runs are never merged).  With
+  // LFQS_OPT_FUSE_MERGE_COMMUTING the run may be interleaved with gates on other
+  // qubits: g merges into the last earlier gate that touches any of its qubits
+  // when that gate is a 1-target gate on the same target with the same controls --
+  // every gate in between acts on disjoint qubits and commutes with g exactly
+  // (Eq. 3), so e.g. the H layer and X layer of a Grover diffusion become
+  // one dense layer.
   std::vector<Decoded> prog;
   prog.reserve(list.size());
   for (const Decoded* gp : list) {
     const Decoded& g = *gp;
     if (g.cls == GClass::NOOP) continue;
     if (!prog.empty()) {
-      Decoded& a = prog.back();
+      size_t ai = prog.size() - 1;
+      if (ctx.opt->fuse_merge_commuting && g.m == 1) {
+        const uint64_t gq = qubit_mask(g);
+        for (size_t k = prog.size(); k-- > 0 && prog.size() - k <= 256;) {
+          ai = k;
+          if (qubit_mask(prog[k]) & gq) break;
+        }
+      }
+      Decoded& a = prog[ai];
       if (a.m == 1 && g.m == 1 && a.targets[0] == g.targets[0] && a.cmask == g.cmask &&
           (a.cls == GClass::DENSE || g.cls == GClass::DENSE)) {
         cplx Cm[4];

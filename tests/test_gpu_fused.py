@@ -21,9 +21,11 @@ def L():
     return lib
 
 
-def _run(L, n, psi, gates, fuse, tile=None, reorder=1):
+def _run(L, n, psi, gates, fuse, tile=None, reorder=1, merge=None):
     with L.State.create(n) as st:
         st.set_option(L.OPT_FUSE_REORDER, reorder)
+        if merge is not None:
+            st.set_option(L.OPT_FUSE_MERGE_COMMUTING, merge)
         if tile:
             st.set_option(L.OPT_FUSE_TILE_QUBITS, tile)
         st.copy_in(psi)
@@ -106,3 +108,25 @@ def test_fused_layered_and_grover(L):
         ref = O.run_circuit(n, gates, psi.copy())
         got, _ = _run(L, n, psi, gates, True)
         assert np.max(np.abs(got - ref)) <= 1e-12
+
+
+@pytest.mark.parametrize("fuse", [True, "phase", "jit", "jit+phase"])
+@pytest.mark.parametrize("tile", [9, 12])
+def test_merge_commuting_1q_runs(L, fuse, tile):
+    """LFQS_OPT_FUSE_MERGE_COMMUTING: same-qubit 1-target gates separated by gates on
+    other qubits merge into one matrix (Grover's H and X layers, VQE's RY and RZ
+    layers); the result changes by rounding only, and exact-class circuits never merge."""
+    n = 14
+    psi = W.random_state(n, 5 + tile)
+    gates = (W.grover(n, 0x2A7D, 1) + W.vqe_ansatz(n, 2, seed=3) +
+             W.random_gate_list(n, 200, seed=tile, max_controls=2))
+    ref = O.run_circuit(n, gates, psi.copy())
+    a, ka = _run(L, n, psi, gates, fuse, tile, merge=1)
+    b, kb = _run(L, n, psi, gates, fuse, tile, merge=0)
+    assert ka == kb
+    assert np.max(np.abs(a - ref)) <= 1e-12
+    assert np.max(np.abs(b - ref)) <= 1e-12
+    exact = [g for g in gates if g.exact]
+    c, _ = _run(L, n, psi, exact, fuse, tile, merge=1)
+    if fuse in (True, "jit"):
+        assert np.array_equal(c, O.run_circuit(n, exact, psi.copy()))
