@@ -332,6 +332,11 @@ lfqs_status lfqs_kernel_launches(const lfqs_state* s, uint64_t* count);
                                      the same target with the same controls and one of the two
                                      is dense; 0: only directly adjacent runs merge.  Changes
                                      rounding only (dense tolerance class) */
+#define LFQS_OPT_JIT_GREEDY_PLACE 11 /* 1 (default): a compiled pass's tile round trip moves
+                                     into register positions the targets of the longest run
+                                     of upcoming gates that fit them (fewest round trips);
+                                     0: only the current gate's targets (furthest-next-use
+                                     eviction).  Bit-identical results either way */
 lfqs_status lfqs_set_option(lfqs_state* s, int option, int64_t value);
 const char* lfqs_last_error(void);
 int lfqs_abi_version(void);

@@ -70,6 +70,7 @@ struct Gen {
   int NT = 256;   // threads per CTA (256, or 512 for K >= 9: twice the warps per SM)
   int NWB = 3;    // warp bits of the thread index
   int FL = 5;     // fixed lane bits
+  bool greedy = false;  // greedy placement (JIT_GREEDY_PLACE)
   int tpos[9] = {0, 1, 2, 3, 4, 5, 6, 7, 8};
   int rpos[4] = {8, 9, 10, 11};
   int nreg = 0;
@@ -82,6 +83,7 @@ struct Gen {
     R = (1 << K) / NT;
     nreg = K - 5 - NWB;
     FL = ((jc & JIT_LANE_MOVE) && nreg >= 1) ? (c64 ? 4 : 3) : 5;
+    greedy = (jc & JIT_GREEDY_PLACE) != 0;
     for (int j = 0; j < 5 + NWB; ++j) tpos[j] = j;
     for (int j = 0; j < nreg; ++j) rpos[j] = 5 + NWB + j;
   }
@@ -853,6 +855,10 @@ struct Gen {
       label(skip);
     }
     if (!in_regs) {
+      if (greedy && nreg >= 1) {
+        place(plan_set(o + nm + 1), o + nm + 1);
+        emit_taddr();
+      }
       tile_to_regs();
       in_regs = true;
     }
@@ -891,11 +897,75 @@ struct Gen {
     label(end);
   }
 
-  void ensure_regs() {
+  // Tile -> registers after the tile was last written in shared memory (smem ops,
+  // phase-table builds): the placement may change for free here, so with greedy
+  // placement the register positions are chosen for the ops from `o` on.
+  void ensure_regs(int o) {
     if (!in_regs) {
       sync();
+      if (greedy && nreg >= 1) {
+        place(plan_set(o), o);
+        emit_taddr();
+      }
       tile_to_regs();
       in_regs = true;
+    }
+  }
+  // Register-position requirement of op o: 0 none (diagonal, fixed-lane shuffle),
+  // 1 its targets in `bits`, 2 it runs as a shared-memory op.
+  int op_need(int o, uint32_t& bits) const {
+    const FHdr& h = P.h[o];
+    bits = 0;
+    if (h.type == F_DTAB || h.type == F_DIAG1 || h.type == F_DIAGN) return 0;
+    int ts[3];
+    const int m = op_targets(h, ts);
+    bool anyl = false;
+    for (int s_ = 0; s_ < m; ++s_) anyl |= fixed_lane(ts[s_]);
+    if (m == 1) {
+      if (anyl) return 0;
+      if (nreg < 1) return 2;
+      bits = 1u << ts[0];
+      return 1;
+    }
+    if (anyl || m > nreg) return 2;
+    for (int s_ = 0; s_ < m; ++s_) bits |= 1u << ts[s_];
+    return 1;
+  }
+  // Greedy placement (LFQS_OPT_JIT_GREEDY_PLACE): one tile round trip costs the same
+  // whatever number of bits it moves, so a remap takes into register positions the
+  // targets of the longest run of upcoming ops whose register requirements fit
+  // nreg positions together (interval covering: the fewest round trips).
+  uint32_t plan_set(int o) const {
+    uint32_t S = 0;
+    for (int q = o; q < P.nops; ++q) {
+      if (P.h[q].type == F_DTAB) {
+        q += P.h[q].m;
+        continue;
+      }
+      uint32_t b;
+      const int k = op_need(q, b);
+      if (k == 0) continue;
+      if (k == 2 || __builtin_popcount(S | b) > nreg) break;
+      S |= b;
+    }
+    return S;
+  }
+  // Placement change (no code): every bit of S not register-held takes the register
+  // position of a bit outside S, the one with the furthest next use first.
+  void place(uint32_t S, int o) {
+    for (int b = 0; b < K; ++b) {
+      if (!((S >> b) & 1) || reg_of(b) >= 0) continue;
+      int best = -1, bd = -1;
+      for (int j = 0; j < nreg; ++j) {
+        if ((S >> rpos[j]) & 1) continue;
+        const int d = next_use(rpos[j], o);
+        if (d > bd) {
+          bd = d;
+          best = j;
+        }
+      }
+      tpos[tbit(b)] = rpos[best];
+      rpos[best] = b;
     }
   }
   static int op_targets(const FHdr& h, int* ts) {
@@ -929,7 +999,9 @@ struct Gen {
   // round trip through the shared-memory tile.
   void remap(const std::vector<int>& need, const int* ts, int m, int o) {
     if (in_regs) regs_to_tile();  // under the old placement
-    for (int b : need) {
+    if (greedy) {
+      place(plan_set(o), o);
+    } else for (int b : need) {
       int best = -1, bd = -1;
       for (int j = 0; j < nreg; ++j) {
         bool tgt = false;
@@ -1060,7 +1132,7 @@ struct Gen {
         continue;
       }
       if (type == F_DIAG1 || type == F_DIAGN) {
-        ensure_regs();
+        ensure_regs(o);
         if (type == F_DIAG1)
           op_diag1(h);
         else
@@ -1081,7 +1153,7 @@ struct Gen {
         for (int s_ = 0; s_ < m; ++s_)
           if (!fixed_lane(ts[s_]) && reg_of(ts[s_]) < 0) need.push_back(ts[s_]);
         if (!need.empty()) remap(need, ts, m, o);
-        ensure_regs();
+        ensure_regs(o);
         if (m == 1)
           op_reg1q(h);
         else
@@ -1289,7 +1361,8 @@ void jit_compile(const std::vector<std::pair<std::string, const FProg*>>& items,
 
 int jit_config(const LaunchCtx& ctx, int K) {
   return ((ctx.opt->jit_threads == 512 && K >= 9) ? 512 : 256) |
-         (ctx.opt->jit_lane_move ? JIT_LANE_MOVE : 0);
+         (ctx.opt->jit_lane_move ? JIT_LANE_MOVE : 0) |
+         (ctx.opt->jit_greedy_place ? JIT_GREEDY_PLACE : 0);
 }
 
 size_t jit_cache_size() {

@@ -26,8 +26,10 @@ def L():
 
 
 def _run(L, n, psi, gates, fuse, tile=None, low=None, c64=False, reorder=1, threads=256,
-         lane_move=None):
+         lane_move=None, greedy=None):
     with L.State.create(n, c64=c64) as st:
+        if greedy is not None:
+            st.set_option(L.OPT_JIT_GREEDY_PLACE, greedy)
         st.set_option(L.OPT_FUSE_REORDER, reorder)
         st.set_option(L.OPT_JIT_THREADS, threads)
         if lane_move is not None:
@@ -80,12 +82,15 @@ def test_jit_512_threads_equals_interpreter(L, n, tile, threads):
 
 @pytest.mark.parametrize("c64", [False, True])
 @pytest.mark.parametrize("threads", [256, 512])
-@pytest.mark.parametrize("tile", [9, 10, 12])
+@pytest.mark.parametrize("tile", [9, 12])
+@pytest.mark.parametrize("greedy", [0, 1])
 @pytest.mark.parametrize("lane_move", [0, 1])
-def test_jit_lane_move_equals_interpreter(L, lane_move, tile, threads, c64):
-    """LFQS_OPT_JIT_LANE_MOVE: lane tile bits 3-4 (complex64: 4) move into register
-    positions and keep the interpreter's lane formulas there -- bit-identical to the
-    interpreted pass on lane-heavy circuits (Grover, layered, Sycamore-like)."""
+def test_jit_placement_variants_equal_interpreter(L, lane_move, greedy, tile, threads, c64):
+    """Tile-bit placement variants of the compiled passes: LFQS_OPT_JIT_LANE_MOVE (lane
+    tile bits 3-4, complex64: 4, move into register positions and keep the interpreter's
+    lane formulas there) and LFQS_OPT_JIT_GREEDY_PLACE (multi-bit remaps) -- all
+    bit-identical to the interpreted pass on lane-heavy and layered circuits (Grover,
+    layered, Sycamore-like)."""
     n = 15
     psi = W.random_state(n, 31 + tile)
     if c64:
@@ -93,10 +98,12 @@ def test_jit_lane_move_equals_interpreter(L, lane_move, tile, threads, c64):
     gates = (W.grover(n, 0x1A5B, 1) + W.random_layered(n, 5, seed=tile) +
              W.sycamore_like(3, 5, 4, seed=threads) + W.random_gate_list(n, 150, seed=9, max_controls=2))
     a, _ = _run(L, n, psi, gates, True, tile, c64=c64)
-    b, _ = _run(L, n, psi, gates, "jit", tile, c64=c64, threads=threads, lane_move=lane_move)
+    b, _ = _run(L, n, psi, gates, "jit", tile, c64=c64, threads=threads, lane_move=lane_move,
+                greedy=greedy)
     assert np.array_equal(a, b)
     c, _ = _run(L, n, psi, gates, "phase", tile, c64=c64)
-    d, _ = _run(L, n, psi, gates, "jit+phase", tile, c64=c64, threads=threads, lane_move=lane_move)
+    d, _ = _run(L, n, psi, gates, "jit+phase", tile, c64=c64, threads=threads,
+                lane_move=lane_move, greedy=greedy)
     assert np.array_equal(c, d)
     tol = 2e-5 if c64 else 1e-12
     assert np.max(np.abs(b - O.run_circuit(n, gates, psi.copy()))) <= tol
