@@ -1098,6 +1098,8 @@ struct Gen {
     e("mov.u32 %%tile, lfqs_tile;");
     e("mov.u32 %%dtab, lfqs_dtab;");
     e("mov.u32 %%bar, lfqs_bar;");
+    // The first tile -> registers transfer is free to choose the placement too.
+    if (greedy && nreg >= 1) place(plan_set(0), 0);
     emit_taddr();
     {
       const std::string w0 = L(), q = p(), q0 = p();
