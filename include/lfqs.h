@@ -337,6 +337,10 @@ lfqs_status lfqs_kernel_launches(const lfqs_state* s, uint64_t* count);
                                      of upcoming gates that fit them (fewest round trips);
                                      0: only the current gate's targets (furthest-next-use
                                      eviction).  Bit-identical results either way */
+#define LFQS_OPT_LANE_GROUP 12 /* 1 (default): per-gate dense 4x4 / 8x8 gates whose targets
+                                  all lie in qubits 1..5 (qubit 0 free) run as coalesced
+                                  warp chunks with shuffle exchange; 0: generic group
+                                  kernel.  Bit-identical results either way */
 lfqs_status lfqs_set_option(lfqs_state* s, int option, int64_t value);
 const char* lfqs_last_error(void);
 int lfqs_abi_version(void);

@@ -279,3 +279,36 @@ def test_table1_workloads_vs_oracle(L, fuse):
     with L.State.create(13) as st:
         st.run_circuit(W.qpe(12, 2901), fuse=fuse)
         assert abs(st.measure_probs(list(range(12)))[2901] - 1.0) < 1e-12
+
+
+# ---------------------------------------------------------------------------
+# Dense 4x4 / 8x8 gates with every target in qubits 1..5 (coalesced lane-group
+# kernel, LFQS_OPT_LANE_GROUP): same terms in the same order as the group kernel
+# ---------------------------------------------------------------------------
+
+@pytest.mark.parametrize("c64", [False, True])
+@pytest.mark.parametrize("n", [8, 9, 13])
+def test_lane_group_dense_low_targets(L, n, c64):
+    psi = W.random_state(n, 77 + n)
+    if c64:
+        psi = psi.astype(np.complex64).astype(np.complex128)
+    cases = []
+    for ts in [(1, 2), (2, 1), (1, 5), (5, 3), (4, 2), (1, 2, 3), (3, 1, 5), (5, 4, 2)]:
+        m = len(ts)
+        U = W.haar_unitary(m, sum(ts) + 7 * m)
+        kind = "UNITARY2" if m == 2 else "UNITARY3"
+        free = [q for q in range(n) if q not in ts]
+        for ctrl in [(), (0,), (free[-1],), (free[1], free[-1]), (6,) if 6 in free else ()]:
+            cases.append(W.Gate(kind, ts, tuple(ctrl), (), U))
+    tol = 4e-6 if c64 else TOL
+    for g in cases:
+        ref = O.apply_gate(n, g, psi.copy())
+        outs = []
+        for lg in (1, 0):
+            with L.State.create(n, c64=c64) as st:
+                st.set_option(L.OPT_LANE_GROUP, lg)
+                st.copy_in(psi)
+                st.apply(g)
+                outs.append(st.copy_out())
+        assert np.array_equal(outs[0], outs[1]), g
+        assert np.max(np.abs(outs[0] - ref)) <= tol, g
