@@ -167,7 +167,8 @@ def main():
                 rec.update(res)
                 if orc is not None:
                     rec["oracle"] = orc
-                    rec["gpu_over_oracle"] = rec["gates_per_s"] / orc["gates_per_s"]
+                    if "gates_per_s" in orc:
+                        rec["gpu_over_oracle"] = rec["gates_per_s"] / orc["gates_per_s"]
                 print(json.dumps(rec), flush=True)
 
 

@@ -19,7 +19,7 @@ def fmt_oracle(d):
     if o is None:
         return "", ""
     if "unavailable" in o:
-        return f"n/a ({o['cores']} cores: host RAM)", ""
+        return f"not run: {o['unavailable']}", ""
     return (f"{o['gates_per_s']:.2f} ({o['gates']}/{o['of']} gates, {o['cores']} cores)",
             f"{d['gpu_over_oracle']:.0f}×")
 
