@@ -1,7 +1,7 @@
 """Small-n workload for compute-sanitizer (memcheck / racecheck / synccheck):
 every kernel family once -- class kernels, shuffle path, fused TMA and direct
 tiles (incl. smem ops), compiled passes (LFQS_FUSE_JIT, with phase tables, 256 and
-512 threads), SOA kernels, virtual-partition exchange, probabilities, collapse.
+512 threads, placement variants), the lane-group kernel, SOA kernels, virtual-partition exchange, probabilities, collapse.
 
     compute-sanitizer --tool racecheck python tools/sanitize_run.py
 """
@@ -33,6 +33,17 @@ def main():
             st.set_option(L.OPT_JIT_THREADS, threads)
             st.run_circuit(gates, fuse="jit")
             st.run_circuit(gates, fuse="jit+phase")
+        st.set_option(L.OPT_JIT_THREADS, 256)
+        for lm, gr in ((1, 1), (0, 0)):  # placement variants of the compiled passes
+            st.set_option(L.OPT_JIT_LANE_MOVE, lm)
+            st.set_option(L.OPT_JIT_GREEDY_PLACE, gr)
+            st.run_circuit(gates, fuse="jit")
+        # lane-group kernel: dense 4x4 / 8x8 with targets in qubits 1..5
+        U2, U3 = W.haar_unitary(2, 5), W.haar_unitary(3, 6)
+        st.run_circuit([W.Gate("UNITARY2", (1, 2), (), (), U2),
+                        W.Gate("UNITARY2", (5, 3), (0, 11), (), U2),
+                        W.Gate("UNITARY3", (1, 2, 3), (), (), U3),
+                        W.Gate("UNITARY3", (4, 1, 5), (7,), (), U3)])
         st.measure_probs([0, 3, 13])
         st.measure_probs(list(range(12)))
         st.sample([1, 2], np.linspace(0, 0.99, 7))
