@@ -67,19 +67,19 @@ struct Gen {
   // shared-memory ops or shuffles.  Every amplitude still sees the same arithmetic
   // (a moved lane bit keeps the interpreter's lane formulas), so results stay
   // bit-identical to the interpreter.
-  int NT = 256;   // threads per CTA (256, or 512 for K >= 9: twice the warps per SM)
+  int NT = 256;   // threads per CTA (128 for K >= 8, 256, or 512 for K >= 9)
   int NWB = 3;    // warp bits of the thread index
   int FL = 5;     // fixed lane bits
   bool greedy = false;  // greedy placement (JIT_GREEDY_PLACE)
   int tpos[9] = {0, 1, 2, 3, 4, 5, 6, 7, 8};
-  int rpos[4] = {8, 9, 10, 11};
+  int rpos[8] = {8, 9, 10, 11, 12, 13, 14, 15};
   int nreg = 0;
 
   Gen(const FProg& p, int k, bool c, int jc) : P(p), K(k), c64(c) {
     FT = c64 ? "f32" : "f64";
     ES = c64 ? 8 : 16;
     NT = jc & JIT_THREADS_MASK;
-    NWB = NT == 512 ? 4 : 3;
+    NWB = NT == 512 ? 4 : NT == 128 ? 2 : 3;
     R = (1 << K) / NT;
     nreg = K - 5 - NWB;
     FL = ((jc & JIT_LANE_MOVE) && nreg >= 1) ? (c64 ? 4 : 3) : 5;
@@ -831,9 +831,11 @@ struct Gen {
     const uint32_t U = h.mlo, cm = h.plo & 0xffffu, cp = h.plo >> 16;
     const int nb = __builtin_popcount(U);
     sync();
-    {
-      const std::string skip = L(), q = p();
-      e("setp.ge.u32 %s, %%ltid, %u;", q.c_str(), 1u << nb);
+    // Entry e of the table is built by thread e mod NT (entries e = ltid + k NT).
+    for (int k = 0; k * NT < (1 << nb); ++k) {
+      const std::string skip = L(), q = p(), eid = r();
+      e("add.u32 %s, %%ltid, %d;", eid.c_str(), k * NT);
+      e("setp.ge.u32 %s, %s, %u;", q.c_str(), eid.c_str(), 1u << nb);
       e("@%s bra %s;", q.c_str(), skip.c_str());
       const std::string ie = r();
       e("mov.u32 %s, %u;", ie.c_str(), cp);
@@ -842,7 +844,7 @@ struct Gen {
         const int pos = __builtin_ctz(u);
         u &= u - 1;
         const std::string t = r();
-        e("bfe.u32 %s, %%ltid, %d, 1;", t.c_str(), b);
+        e("bfe.u32 %s, %s, %d, 1;", t.c_str(), eid.c_str(), b);
         e("bfi.b32 %s, %s, %s, %d, 1;", ie.c_str(), t.c_str(), ie.c_str(), pos);
       }
       Cx t{f(), f()};
@@ -850,7 +852,7 @@ struct Gen {
       e("mov.%s %s, %s;", FT, t.y.c_str(), zero().c_str());
       for (int j = 1; j <= nm; ++j) dtab_member(P.h[o + j], ie, t);
       const std::string a = r();
-      e("mad.lo.u32 %s, %%ltid, %d, %%dtab;", a.c_str(), ES);
+      e("mad.lo.u32 %s, %s, %d, %%dtab;", a.c_str(), eid.c_str(), ES);
       sts(a, t);
       label(skip);
     }
@@ -869,7 +871,7 @@ struct Gen {
     // (runtime, et) or a slot bit (compile time, w[j]).
     const std::string et = r();
     e("mov.u32 %s, 0;", et.c_str());
-    uint32_t w[4] = {0, 0, 0, 0};
+    uint32_t w[8] = {0, 0, 0, 0, 0, 0, 0, 0};
     uint32_t u = U;
     for (int k = 0; u; ++k) {
       const int pos = __builtin_ctz(u);
@@ -1191,7 +1193,8 @@ struct Gen {
     const int nc = P.ncoef > 0 ? P.ncoef : 1;
     out += ".visible .entry lfqs_jit(.param .u64 pa, .param .align 16 .b8 pc[" +
            std::to_string(nc * 16) + "])\n";
-    out += ".maxntid " + std::to_string(NT) + ", 1, 1\n.minnctapersm 2\n{\n";
+    out += ".maxntid " + std::to_string(NT) + ", 1, 1\n.minnctapersm " +
+           std::to_string(NT == 128 ? 3 : 2) + "\n{\n";
     out += "  .reg .pred %p<" + std::to_string(np + 1) + ">;\n";
     out += "  .reg .b32 %r<" + std::to_string(nr + 1) + ">;\n";
     out += "  .reg .b64 %rd<" + std::to_string(nrd + 1) + ">;\n";
@@ -1362,7 +1365,8 @@ void jit_compile(const std::vector<std::pair<std::string, const FProg*>>& items,
 }
 
 int jit_config(const LaunchCtx& ctx, int K) {
-  return ((ctx.opt->jit_threads == 512 && K >= 9) ? 512 : 256) |
+  const int t = ctx.opt->jit_threads;
+  return ((t == 512 && K >= 9) ? 512 : (t == 128 && K >= 8) ? 128 : 256) |
          (ctx.opt->jit_lane_move ? JIT_LANE_MOVE : 0) |
          (ctx.opt->jit_greedy_place ? JIT_GREEDY_PLACE : 0);
 }

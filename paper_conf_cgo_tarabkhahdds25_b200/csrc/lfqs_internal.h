@@ -90,7 +90,7 @@ struct Options {
   // beats direct loads for every chunk count up to 128, so TMA is the default.
   int fuse_tma_max_chunks = 256;
   int items_per_thread = 0;  // 0 = library default
-  int jit_threads = 256;     // threads per CTA of compiled passes (256 or 512)
+  int jit_threads = 256;     // threads per CTA of compiled passes (128, 256 or 512)
   bool lane_group = true;  // dense 4x4/8x8 with targets in [1, 5]: coalesced lane-group kernel
   bool fuse_merge_commuting = true;  // merge same-qubit 1-target gates across commuting gates
   bool jit_lane_move = false;    // compiled passes may move lane bits >= 3 into registers

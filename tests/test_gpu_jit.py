@@ -64,7 +64,7 @@ def test_jit_equals_interpreter(L, n, tile, low, reorder):
     assert np.max(np.abs(b - ref)) <= 1e-12
 
 
-@pytest.mark.parametrize("threads", [256, 512])
+@pytest.mark.parametrize("threads", [128, 256, 512])
 @pytest.mark.parametrize("tile", [9, 10, 12])
 @pytest.mark.parametrize("n", [13, 16])
 def test_jit_512_threads_equals_interpreter(L, n, tile, threads):
@@ -81,7 +81,7 @@ def test_jit_512_threads_equals_interpreter(L, n, tile, threads):
 
 
 @pytest.mark.parametrize("c64", [False, True])
-@pytest.mark.parametrize("threads", [256, 512])
+@pytest.mark.parametrize("threads", [128, 256, 512])
 @pytest.mark.parametrize("tile", [9, 12])
 @pytest.mark.parametrize("greedy", [0, 1])
 @pytest.mark.parametrize("lane_move", [0, 1])

@@ -61,7 +61,7 @@ def main():
     ap.add_argument("--tile", type=int, default=0)
     ap.add_argument("--low", type=int, default=0)
     ap.add_argument("--reorder", type=int, default=1)
-    ap.add_argument("--jit-threads", type=int, default=256, help="LFQS_OPT_JIT_THREADS (256/512)")
+    ap.add_argument("--jit-threads", type=int, default=256, help="LFQS_OPT_JIT_THREADS (128/256/512)")
     ap.add_argument("--lane-move", type=int, default=-1,
                     help="LFQS_OPT_JIT_LANE_MOVE (0/1; -1: library default)")
     ap.add_argument("--greedy", type=int, default=-1,
