@@ -338,10 +338,11 @@ lfqs_status lfqs_kernel_launches(const lfqs_state* s, uint64_t* count);
                                      of upcoming gates that fit them (fewest round trips);
                                      0: only the current gate's targets (furthest-next-use
                                      eviction).  Bit-identical results either way */
-#define LFQS_OPT_LANE_GROUP 12 /* 1 (default): per-gate dense 4x4 / 8x8 gates whose targets
-                                  all lie in qubits 1..5 (qubit 0 free) run as coalesced
-                                  warp chunks with shuffle exchange; 0: generic group
-                                  kernel.  Bit-identical results either way */
+#define LFQS_OPT_LANE_GROUP 12 /* 1 (default): per-gate dense 4x4 gates on qubits {1, 2}
+                                  run as coalesced warp chunks with shuffle exchange (the
+                                  group kernel's accesses are 128-B strided there); 2: also
+                                  every other dense 4x4 / 8x8 gate with targets in 1..5;
+                                  0: never.  Bit-identical results either way */
 lfqs_status lfqs_set_option(lfqs_state* s, int option, int64_t value);
 const char* lfqs_last_error(void);
 int lfqs_abi_version(void);

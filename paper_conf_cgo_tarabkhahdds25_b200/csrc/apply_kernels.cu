@@ -307,7 +307,8 @@ __global__ void __launch_bounds__(kThreads) k_lowq(cx<S>* __restrict__ a, uint64
 }
 
 // ---------------------------------------------------------------------------
-// Dense 4x4 / 8x8 gate whose targets all lie in [1, 5] with qubit 0 free.  The
+// Dense 4x4 / 8x8 gate whose targets all lie in [1, 5] with qubit 0 free (used by
+// default for 4x4 on qubits {1, 2} only; LFQS_OPT_LANE_GROUP = 2 forces it).  The
 // generic group kernels give each thread one group; with targets this low a
 // group (x2: with its bit-0 neighbours) is a single contiguous 128-256 B run, so
 // every warp access touches 32 different lines, one sector each (UNITARY2 on
@@ -527,10 +528,15 @@ void launch_dense_m(const LaunchCtx& ctx, const Decoded& g) {
   const uint64_t n_groups = 1ull << (ctx.n_local - m - nc);
   const InsertPlan ip = make_plan(tmask, g.cmask);
   const Offs<L> off = group_offsets<L>(t, m);
-  // Targets in [1, 5], qubit 0 free: coalesced lane-group kernel (k_lanegroup).
+  // Targets {1, 2} (qubit 0 free): the group kernel's item is one contiguous 128-B
+  // run per thread (32 lines per warp access): coalesced lane-group kernel instead
+  // (k_lanegroup; measured at n = 30: 6.5 -> 4.9 ms).  For other low targets, and
+  // for 8x8 gates, its shuffle volume (8 shuffles per partner and pair) makes it
+  // slower than the group kernel (profiles/r01_lane_group.md), so they stay there.
   constexpr int kLGV = 4, kLGB = 6 + 2;  // 4 pairs per lane: 256-amplitude chunks
   const uint64_t hi_c = g.cmask & ~((1ull << kLGB) - 1);
-  if (ctx.opt->lane_group && !(tmask & 1) && (tmask >> 6) == 0 &&
+  if (ctx.opt->lane_group && (L == 4 ? tmask == 6ull : ctx.opt->lane_group > 1) &&
+      !(tmask & 1) && (tmask >> 6) == 0 &&
       ctx.n_local >= kLGB + __builtin_popcountll(hi_c)) {
     LaneGroupArgs<S, L> la;
     for (int i = 0; i < L * L; ++i) la.M[i] = op.M[i];

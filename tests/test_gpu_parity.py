@@ -304,11 +304,11 @@ def test_lane_group_dense_low_targets(L, n, c64):
     for g in cases:
         ref = O.apply_gate(n, g, psi.copy())
         outs = []
-        for lg in (1, 0):
+        for lg in (2, 0):
             with L.State.create(n, c64=c64) as st:
                 st.set_option(L.OPT_LANE_GROUP, lg)
                 st.copy_in(psi)
                 st.apply(g)
                 outs.append(st.copy_out())
-        assert np.array_equal(outs[0], outs[1]), g
+        assert np.array_equal(outs[0], outs[1]), g  # forced lane-group == group kernel
         assert np.max(np.abs(outs[0] - ref)) <= tol, g
