@@ -343,6 +343,11 @@ lfqs_status lfqs_kernel_launches(const lfqs_state* s, uint64_t* count);
                                   group kernel's accesses are 128-B strided there); 2: also
                                   every other dense 4x4 / 8x8 gate with targets in 1..5;
                                   0: never.  Bit-identical results either way */
+#define LFQS_OPT_JIT_LANE_REG2 13 /* 1 (default): in a compiled pass, a SWAP / 2-target dense
+                                     gate with one target on a lane bit (0-4) and the other
+                                     on a register-held tile bit runs by warp shuffles in
+                                     registers instead of as a shared-memory op; 0: shared
+                                     memory.  Bit-identical results either way */
 lfqs_status lfqs_set_option(lfqs_state* s, int option, int64_t value);
 const char* lfqs_last_error(void);
 int lfqs_abi_version(void);

@@ -71,6 +71,7 @@ struct Gen {
   int NWB = 3;    // warp bits of the thread index
   int FL = 5;     // fixed lane bits
   bool greedy = false;  // greedy placement (JIT_GREEDY_PLACE)
+  bool lane_reg2 = false;  // SWAP / U4 with one fixed-lane target by shuffles (JIT_LANE_REG2)
   int tpos[9] = {0, 1, 2, 3, 4, 5, 6, 7, 8};
   int rpos[8] = {8, 9, 10, 11, 12, 13, 14, 15};
   int nreg = 0;
@@ -84,6 +85,7 @@ struct Gen {
     nreg = K - 5 - NWB;
     FL = ((jc & JIT_LANE_MOVE) && nreg >= 1) ? (c64 ? 4 : 3) : 5;
     greedy = (jc & JIT_GREEDY_PLACE) != 0;
+    lane_reg2 = (jc & JIT_LANE_REG2) != 0;
     for (int j = 0; j < 5 + NWB; ++j) tpos[j] = j;
     for (int j = 0; j < nreg; ++j) rpos[j] = 5 + NWB + j;
   }
@@ -929,6 +931,11 @@ struct Gen {
       bits = 1u << ts[0];
       return 1;
     }
+    if (lane_reg2 && m == 2 && nreg >= 1 && (h.type == F_U4 || h.type == F_SWAP) &&
+        fixed_lane(ts[0]) != fixed_lane(ts[1])) {
+      bits = 1u << (fixed_lane(ts[0]) ? ts[1] : ts[0]);
+      return 1;
+    }
     if (anyl || m > nreg) return 2;
     for (int s_ = 0; s_ < m; ++s_) bits |= 1u << ts[s_];
     return 1;
@@ -1022,6 +1029,81 @@ struct Gen {
     emit_taddr();
     tile_to_regs();
     in_regs = true;
+  }
+
+  // SWAP / U4 with one target at a fixed lane position (a) and the other register-held
+  // (b): the partner lane (lane ^ 2^tbit(a)) holds the other half of every group, fetched
+  // by shuffles, so the gate needs no shared-memory round trip.  The group values are
+  // put in local-index order and each output is the interpreter's sum over q ascending
+  // (F_U4) or its move (F_SWAP): bit-identical.
+  void op_lanereg2(const FHdr& h) {
+    const std::string end = L();
+    tile_pred(h.mhi, h.phi, end);
+    const bool a_is_t0 = fixed_lane(h.t0);
+    const int ta = a_is_t0 ? h.t0 : h.t1, tb = a_is_t0 ? h.t1 : h.t0;
+    const int tl = tbit(ta), rb = reg_of(tb);
+    // local index j = 2 bit(t0) + bit(t1)
+    auto jidx = [&](int av, int bv) { return a_is_t0 ? (av << 1) | bv : (bv << 1) | av; };
+    uint32_t tm_, tv_, mr, pr;
+    split(h.mlo, h.plo, tm_, tv_, mr, pr);
+    const std::string bt = thread_pred(h.mlo, h.plo);
+    const std::string x = p(), xa = r();
+    e("and.b32 %s, %%ltid, %u;", xa.c_str(), 1u << tl);
+    e("setp.ne.b32 %s, %s, 0;", x.c_str(), xa.c_str());
+    // Coefficient rows of this thread's two outputs (a = x, b = 0 / 1), selected once.
+    std::vector<Cx> row[2], nrow[2];
+    if (h.type == F_U4) {
+      std::vector<Cx> c, nc;
+      for (int k = 0; k < 16; ++k) {
+        c.push_back(coef(h.coef + k));
+        nc.push_back({c.back().zy() ? std::string() : neg(c.back().y), ""});
+      }
+      for (int bv = 0; bv < 2; ++bv)
+        for (int q = 0; q < 4; ++q) {
+          const int j1 = jidx(1, bv), j0 = jidx(0, bv);
+          row[bv].push_back(sel_c(c[j1 * 4 + q], c[j0 * 4 + q], x));
+          const Cx& n1 = nc[j1 * 4 + q];
+          const Cx& n0 = nc[j0 * 4 + q];
+          if (row[bv].back().zy())
+            nrow[bv].push_back({std::string(), ""});
+          else
+            nrow[bv].push_back({sel(n1.x.empty() ? zero() : n1.x, n0.x.empty() ? zero() : n0.x, x), ""});
+        }
+    }
+    for (int r_ = 0; r_ < R; ++r_) {
+      if ((r_ >> rb) & 1) continue;
+      if (((uint32_t)r_ & mr) != pr) continue;
+      const int r1 = r_ | (1 << rb);
+      const Cx A0 = copy({vx(r_), vy(r_)}), A1 = copy({vx(r1), vy(r1)});
+      const Cx P0 = shfl(A0, tl), P1 = shfl(A1, tl);
+      Cx o0, o1;
+      if (h.type == F_SWAP) {
+        // new(a, b) = old(b, a): (x, 0) <- old(0, x); (x, 1) <- old(1, x)
+        o0 = {sel(P1.x, A0.x, x), sel(P1.y, A0.y, x)};
+        o1 = {sel(A1.x, P0.x, x), sel(A1.y, P0.y, x)};
+      } else {
+        // group values by local index: (a = x) own, (a = 1 - x) partner
+        Cx v[4];
+        for (int bv = 0; bv < 2; ++bv) {
+          const Cx& own = bv ? A1 : A0;
+          const Cx& par = bv ? P1 : P0;
+          v[jidx(0, bv)] = {sel(par.x, own.x, x), sel(par.y, own.y, x)};
+          v[jidx(1, bv)] = {sel(own.x, par.x, x), sel(own.y, par.y, x)};
+        }
+        for (int q = 0; q < 4; ++q) cfma(o0, row[0][q], nrow[0][q], v[q], q == 0);
+        for (int q = 0; q < 4; ++q) cfma(o1, row[1][q], nrow[1][q], v[q], q == 0);
+      }
+      if (bt.empty()) {
+        set(r_, o0);
+        set(r1, o1);
+      } else {
+        e("selp.%s %s, %s, %s, %s;", FT, vx(r_).c_str(), o0.x.c_str(), vx(r_).c_str(), bt.c_str());
+        e("selp.%s %s, %s, %s, %s;", FT, vy(r_).c_str(), o0.y.c_str(), vy(r_).c_str(), bt.c_str());
+        e("selp.%s %s, %s, %s, %s;", FT, vx(r1).c_str(), o1.x.c_str(), vx(r1).c_str(), bt.c_str());
+        e("selp.%s %s, %s, %s, %s;", FT, vy(r1).c_str(), o1.y.c_str(), vy(r1).c_str(), bt.c_str());
+      }
+    }
+    label(end);
   }
 
   // SWAP / U4 / U8 with every target register-held.
@@ -1152,7 +1234,19 @@ struct Gen {
       // Multi-target gates: in registers when no target is at a fixed lane position
       // and they fit the register positions.
       const bool in_reg_path = m == 1 ? (any_lane || nreg >= 1) : (!any_lane && m <= nreg);
-      if (in_reg_path) {
+      // SWAP / U4 with exactly one fixed-lane target: shuffles + registers.
+      const bool lanereg = lane_reg2 && !in_reg_path && m == 2 && nreg >= 1 &&
+                           (h.type == F_U4 || h.type == F_SWAP) &&
+                           (fixed_lane(ts[0]) != fixed_lane(ts[1]));
+      if (lanereg) {
+        const int tb = fixed_lane(ts[0]) ? ts[1] : ts[0];
+        if (reg_of(tb) < 0) {
+          std::vector<int> need{tb};
+          remap(need, ts, m, o);
+        }
+        ensure_regs(o);
+        op_lanereg2(h);
+      } else if (in_reg_path) {
         std::vector<int> need;
         for (int s_ = 0; s_ < m; ++s_)
           if (!fixed_lane(ts[s_]) && reg_of(ts[s_]) < 0) need.push_back(ts[s_]);
@@ -1368,7 +1462,8 @@ int jit_config(const LaunchCtx& ctx, int K) {
   const int t = ctx.opt->jit_threads;
   return ((t == 512 && K >= 9) ? 512 : (t == 128 && K >= 8) ? 128 : 256) |
          (ctx.opt->jit_lane_move ? JIT_LANE_MOVE : 0) |
-         (ctx.opt->jit_greedy_place ? JIT_GREEDY_PLACE : 0);
+         (ctx.opt->jit_greedy_place ? JIT_GREEDY_PLACE : 0) |
+         (ctx.opt->jit_lane_reg2 ? JIT_LANE_REG2 : 0);
 }
 
 size_t jit_cache_size() {

@@ -26,8 +26,10 @@ def L():
 
 
 def _run(L, n, psi, gates, fuse, tile=None, low=None, c64=False, reorder=1, threads=256,
-         lane_move=None, greedy=None):
+         lane_move=None, greedy=None, lane_reg2=None):
     with L.State.create(n, c64=c64) as st:
+        if lane_reg2 is not None:
+            st.set_option(L.OPT_JIT_LANE_REG2, lane_reg2)
         if greedy is not None:
             st.set_option(L.OPT_JIT_GREEDY_PLACE, greedy)
         st.set_option(L.OPT_FUSE_REORDER, reorder)
@@ -105,6 +107,27 @@ def test_jit_placement_variants_equal_interpreter(L, lane_move, greedy, tile, th
     d, _ = _run(L, n, psi, gates, "jit+phase", tile, c64=c64, threads=threads,
                 lane_move=lane_move, greedy=greedy)
     assert np.array_equal(c, d)
+    tol = 2e-5 if c64 else 1e-12
+    assert np.max(np.abs(b - O.run_circuit(n, gates, psi.copy()))) <= tol
+
+
+@pytest.mark.parametrize("c64", [False, True])
+@pytest.mark.parametrize("tile", [9, 10, 12])
+@pytest.mark.parametrize("lane_reg2", [0, 1])
+def test_jit_lane_register_2q_equals_interpreter(L, lane_reg2, tile, c64):
+    """LFQS_OPT_JIT_LANE_REG2: SWAP / 2-target dense gates with one target on a lane
+    bit and the other register-held run by shuffles in registers -- bit-identical to
+    the interpreter's shared-memory op (2-target gates on every placement, with
+    controls, Sycamore-like fSim layers)."""
+    n = 14
+    psi = W.random_state(n, 5 * tile + 1)
+    if c64:
+        psi = psi.astype(np.complex64).astype(np.complex128)
+    gates = (W.random_gate_list(n, 300, seed=tile, max_targets=2, max_controls=2) +
+             W.sycamore_like(2, 7, 6, seed=tile))
+    a, _ = _run(L, n, psi, gates, True, tile, c64=c64)
+    b, _ = _run(L, n, psi, gates, "jit", tile, c64=c64, lane_reg2=lane_reg2)
+    assert np.array_equal(a, b)
     tol = 2e-5 if c64 else 1e-12
     assert np.max(np.abs(b - O.run_circuit(n, gates, psi.copy()))) <= tol
 
