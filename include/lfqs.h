@@ -323,7 +323,7 @@ lfqs_status lfqs_kernel_launches(const lfqs_state* s, uint64_t* count);
 #define LFQS_OPT_JIT_THREADS 8 /* threads per CTA of LFQS_FUSE_JIT passes: 256 (default), 512
                                    (twice the warps per SM, half the amplitudes per thread) or
                                    128 (one more register-held tile bit, 3 CTAs per SM) */
-#define LFQS_OPT_JIT_LANE_MOVE 9 /* 1: compiled passes may move the lane tile bits >= 3
+#define LFQS_OPT_JIT_LANE_MOVE 9 /* 1 (default): compiled passes may move the lane tile bits >= 3
                                      (complex64: >= 4) into register positions, so 1-target
                                      gates on them run in registers instead of by warp
                                      shuffles; bit-identical results either way */
