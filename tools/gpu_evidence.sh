@@ -25,4 +25,7 @@ timeout 2400 python tools/bench_circuits.py --n 30 --modes fused,phase,jit,jit+p
 timeout 2400 python tools/bench_circuits.py --n 33 --reps 1 --circuits qft,ghz,qpe,grover,random --modes fused,jit,jit+phase --oracle-s 12 > $O/${TAG}_circuits_n33.jsonl 2>&1
 timeout 900 python tools/bench_circuits.py --n 31 --c64 --circuits qft,ghz,random --modes fused,jit,jit+phase > $O/${TAG}_circuits_c64_n31.jsonl 2>&1
 timeout 600 python tools/bench_small.py > $O/${TAG}_small.jsonl 2>&1
+for tool in memcheck racecheck synccheck; do
+  timeout 900 compute-sanitizer --tool $tool --print-limit 20 python tools/sanitize_run.py > $O/${TAG}_sanitize_$tool.txt 2>&1
+done
 echo done
