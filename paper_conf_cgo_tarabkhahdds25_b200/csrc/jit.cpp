@@ -936,6 +936,9 @@ struct Gen {
       bits = 1u << (fixed_lane(ts[0]) ? ts[1] : ts[0]);
       return 1;
     }
+    if (lane_reg2 && m == 2 && (h.type == F_U4 || h.type == F_SWAP) && fixed_lane(ts[0]) &&
+        fixed_lane(ts[1]))
+      return 0;  // op_lanelane2: shuffles only
     if (anyl || m > nreg) return 2;
     for (int s_ = 0; s_ < m; ++s_) bits |= 1u << ts[s_];
     return 1;
@@ -1106,6 +1109,106 @@ struct Gen {
     label(end);
   }
 
+  // Shuffle by source lane (idx mode).
+  Cx shfl_idx(const Cx& v, const std::string& src) {
+    Cx o{f(), f()};
+    for (int c = 0; c < 2; ++c) {
+      const std::string& sv = c ? v.y : v.x;
+      const std::string& dv = c ? o.y : o.x;
+      if (!c64) {
+        const std::string lo = r(), hi = r(), lo2 = r(), hi2 = r();
+        e("mov.b64 {%s, %s}, %s;", lo.c_str(), hi.c_str(), sv.c_str());
+        e("shfl.sync.idx.b32 %s, %s, %s, 31, -1;", lo2.c_str(), lo.c_str(), src.c_str());
+        e("shfl.sync.idx.b32 %s, %s, %s, 31, -1;", hi2.c_str(), hi.c_str(), src.c_str());
+        e("mov.b64 %s, {%s, %s};", dv.c_str(), lo2.c_str(), hi2.c_str());
+      } else {
+        const std::string a = r(), b = r();
+        e("mov.b32 %s, %s;", a.c_str(), sv.c_str());
+        e("shfl.sync.idx.b32 %s, %s, %s, 31, -1;", b.c_str(), a.c_str(), src.c_str());
+        e("mov.b32 %s, %s;", dv.c_str(), b.c_str());
+      }
+    }
+    return o;
+  }
+
+  // SWAP / U4 with both targets at fixed lane positions: the four lanes that differ
+  // only in the two target bits hold a group (one amplitude per slot each); every lane
+  // gathers the group in local-index order by idx shuffles and computes its own output
+  // with the interpreter's sum (F_U4) or move (F_SWAP) -- bit-identical, no tile round
+  // trip and no strided shared-memory items.
+  void op_lanelane2(const FHdr& h) {
+    const std::string end = L();
+    tile_pred(h.mhi, h.phi, end);
+    const int l0 = tbit(h.t0), l1 = tbit(h.t1);  // lane bits of the local index MSB / LSB
+    uint32_t tm_, tv_, mr, pr;
+    split(h.mlo, h.plo, tm_, tv_, mr, pr);
+    const std::string bt = thread_pred(h.mlo, h.plo);
+    const std::string b0 = p(), b1 = p(), a0 = r(), a1 = r();
+    e("and.b32 %s, %%ltid, %u;", a0.c_str(), 1u << l0);
+    e("setp.ne.b32 %s, %s, 0;", b0.c_str(), a0.c_str());
+    e("and.b32 %s, %%ltid, %u;", a1.c_str(), 1u << l1);
+    e("setp.ne.b32 %s, %s, 0;", b1.c_str(), a1.c_str());
+    const std::string base = r();
+    e("and.b32 %s, %%ltid, %u;", base.c_str(), 31u & ~((1u << l0) | (1u << l1)));
+    if (h.type == F_SWAP) {
+      // new(x0, x1) = old(x1, x0): source lane with the two bits exchanged
+      const std::string src = r(), t = r(), u = r();
+      e("shr.u32 %s, %s, %d;", t.c_str(), a0.c_str(), l0);
+      e("shl.b32 %s, %s, %d;", t.c_str(), t.c_str(), l1);
+      e("shr.u32 %s, %s, %d;", u.c_str(), a1.c_str(), l1);
+      e("shl.b32 %s, %s, %d;", u.c_str(), u.c_str(), l0);
+      e("or.b32 %s, %s, %s;", src.c_str(), base.c_str(), t.c_str());
+      e("or.b32 %s, %s, %s;", src.c_str(), src.c_str(), u.c_str());
+      for (int r_ = 0; r_ < R; ++r_) {
+        if (((uint32_t)r_ & mr) != pr) continue;
+        const Cx o = shfl_idx({vx(r_), vy(r_)}, src);
+        if (bt.empty()) {
+          set(r_, o);
+        } else {
+          e("selp.%s %s, %s, %s, %s;", FT, vx(r_).c_str(), o.x.c_str(), vx(r_).c_str(), bt.c_str());
+          e("selp.%s %s, %s, %s, %s;", FT, vy(r_).c_str(), o.y.c_str(), vy(r_).c_str(), bt.c_str());
+        }
+      }
+      label(end);
+      return;
+    }
+    std::string src[4];
+    for (int q = 0; q < 4; ++q) {
+      src[q] = r();
+      e("or.b32 %s, %s, %u;", src[q].c_str(), base.c_str(),
+        (uint32_t)(((q >> 1) & 1) << l0) | (uint32_t)((q & 1) << l1));
+    }
+    // coefficient row of this lane's local index j = 2 b0 + b1, selected once
+    std::vector<Cx> c, nc;
+    for (int k = 0; k < 16; ++k) {
+      c.push_back(coef(h.coef + k));
+      nc.push_back({c.back().zy() ? zero() : neg(c.back().y), ""});
+    }
+    std::vector<Cx> row, nrow;
+    for (int q = 0; q < 4; ++q) {
+      const Cx lo = sel_c(c[1 * 4 + q], c[0 * 4 + q], b1);   // j = 0 / 1
+      const Cx hi = sel_c(c[3 * 4 + q], c[2 * 4 + q], b1);   // j = 2 / 3
+      row.push_back(sel_c(hi, lo, b0));
+      const std::string nlo = sel(nc[1 * 4 + q].x, nc[0 * 4 + q].x, b1);
+      const std::string nhi = sel(nc[3 * 4 + q].x, nc[2 * 4 + q].x, b1);
+      nrow.push_back({sel(nhi, nlo, b0), ""});
+    }
+    for (int r_ = 0; r_ < R; ++r_) {
+      if (((uint32_t)r_ & mr) != pr) continue;
+      Cx v[4];
+      for (int q = 0; q < 4; ++q) v[q] = shfl_idx({vx(r_), vy(r_)}, src[q]);
+      Cx o;
+      for (int q = 0; q < 4; ++q) cfma(o, row[q], nrow[q], v[q], q == 0);
+      if (bt.empty()) {
+        set(r_, o);
+      } else {
+        e("selp.%s %s, %s, %s, %s;", FT, vx(r_).c_str(), o.x.c_str(), vx(r_).c_str(), bt.c_str());
+        e("selp.%s %s, %s, %s, %s;", FT, vy(r_).c_str(), o.y.c_str(), vy(r_).c_str(), bt.c_str());
+      }
+    }
+    label(end);
+  }
+
   // SWAP / U4 / U8 with every target register-held.
   void op_regmulti(const FHdr& h) {
     const std::string end = L();
@@ -1238,7 +1341,13 @@ struct Gen {
       const bool lanereg = lane_reg2 && !in_reg_path && m == 2 && nreg >= 1 &&
                            (h.type == F_U4 || h.type == F_SWAP) &&
                            (fixed_lane(ts[0]) != fixed_lane(ts[1]));
-      if (lanereg) {
+      const bool lanelane = lane_reg2 && !in_reg_path && m == 2 &&
+                            (h.type == F_U4 || h.type == F_SWAP) && fixed_lane(ts[0]) &&
+                            fixed_lane(ts[1]);
+      if (lanelane) {
+        ensure_regs(o);
+        op_lanelane2(h);
+      } else if (lanereg) {
         const int tb = fixed_lane(ts[0]) ? ts[1] : ts[0];
         if (reg_of(tb) < 0) {
           std::vector<int> need{tb};
