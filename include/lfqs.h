@@ -348,6 +348,12 @@ lfqs_status lfqs_kernel_launches(const lfqs_state* s, uint64_t* count);
                                      on a register-held tile bit runs by warp shuffles in
                                      registers instead of as a shared-memory op; 0: shared
                                      memory.  Bit-identical results either way */
+#define LFQS_OPT_JIT_LANE_POOL 14 /* 1: with greedy placement, lane-move and lane/register
+                                     2-target gates on, the movable lane positions serve
+                                     1-target and 2-target gates by shuffles like register
+                                     positions (more tile bits per placement, fewer tile
+                                     round trips); 0 (default): registers only.
+                                     Bit-identical results either way */
 lfqs_status lfqs_set_option(lfqs_state* s, int option, int64_t value);
 const char* lfqs_last_error(void);
 int lfqs_abi_version(void);

@@ -43,6 +43,7 @@ OPT_FUSE_MERGE_COMMUTING = 10
 OPT_JIT_GREEDY_PLACE = 11
 OPT_LANE_GROUP = 12
 OPT_JIT_LANE_REG2 = 13
+OPT_JIT_LANE_POOL = 14
 
 STATUS = {0: "OK", -1: "INVALID_ARG", -2: "OUT_OF_MEMORY", -3: "CUDA", -4: "NCCL",
           -5: "UNSUPPORTED"}

@@ -72,6 +72,7 @@ struct Gen {
   int FL = 5;     // fixed lane bits
   bool greedy = false;  // greedy placement (JIT_GREEDY_PLACE)
   bool lane_reg2 = false;  // SWAP / U4 with one fixed-lane target by shuffles (JIT_LANE_REG2)
+  bool pool = false;       // lane-pool placement (JIT_LANE_POOL)
   int tpos[9] = {0, 1, 2, 3, 4, 5, 6, 7, 8};
   int rpos[8] = {8, 9, 10, 11, 12, 13, 14, 15};
   int nreg = 0;
@@ -86,6 +87,7 @@ struct Gen {
     FL = ((jc & JIT_LANE_MOVE) && nreg >= 1) ? (c64 ? 4 : 3) : 5;
     greedy = (jc & JIT_GREEDY_PLACE) != 0;
     lane_reg2 = (jc & JIT_LANE_REG2) != 0;
+    pool = (jc & JIT_LANE_POOL) && greedy && lane_reg2 && FL < 5 && nreg >= 1;
     for (int j = 0; j < 5 + NWB; ++j) tpos[j] = j;
     for (int j = 0; j < nreg; ++j) rpos[j] = 5 + NWB + j;
   }
@@ -101,6 +103,13 @@ struct Gen {
       if (tpos[j] == b) return j;
     return -1;
   }
+  // Tile bit b sits at a lane position (0..4).
+  bool at_lane(int b) const {
+    const int t = tbit(b);
+    return t >= 0 && t < 5;
+  }
+  // Lane pool: the movable lane positions are "cheap" positions like the registers.
+  bool cheap(int b) const { return reg_of(b) >= 0 || (pool && at_lane(b)); }
   // Tile bit b sits at a fixed lane position (shuffle path only).
   bool fixed_lane(int b) const {
     const int t = tbit(b);
@@ -481,6 +490,63 @@ struct Gen {
     }
   }
 
+  // pair() evaluated by a lane that holds one amplitude of the pair (tile bit >= 5 at
+  // a lane position, lane-pool placement): x0 / x1 put back in pair order by value
+  // selects, coefficients selected once per op (LaneP), then pair()'s exact operation
+  // sequence -- bit-identical to the register / shared-memory pair.
+  struct LaneP {
+    std::string c1, c2, f1, f2, g1, g2;  // F_UR: c1, c2; F_UI: f* (re), g* (im)
+    Cx m1, n1, m2, n2;                   // F_U2
+  };
+  LaneP lanep_coefs(const Op2& o, const std::string& bit) {
+    LaneP l;
+    switch (o.type) {
+      case F_UR:
+        l.c1 = sel(o.m10, o.m00, bit);
+        l.c2 = sel(o.m11, o.m01, bit);
+        break;
+      case F_UI:
+        l.f1 = sel(neg(o.e10), o.d0, bit);
+        l.f2 = sel(o.d1, neg(o.e01), bit);
+        l.g1 = sel(o.e10, o.d0, bit);
+        l.g2 = sel(o.d1, o.e01, bit);
+        break;
+      case F_U2:
+        l.m1 = sel_c(o.c2, o.c0, bit);
+        l.n1 = {sel(o.n2.x, o.n0.x, bit), ""};
+        l.m2 = sel_c(o.c3, o.c1, bit);
+        l.n2 = {sel(o.n3.x, o.n1.x, bit), ""};
+        break;
+      default: break;
+    }
+    return l;
+  }
+  Cx lane_pair(const Op2& o, const LaneP& l, const Cx& a, const Cx& pp, const std::string& bit) {
+    switch (o.type) {
+      case F_X: case F_Y: case F_H:
+        // moves, and s(p +- a) == s(x0 +- x1) bit for bit: the lane formulas
+        return lane(o, LaneC(), a, pp, bit);
+      default: break;
+    }
+    const Cx x0{sel(pp.x, a.x, bit), sel(pp.y, a.y, bit)};
+    const Cx x1{sel(a.x, pp.x, bit), sel(a.y, pp.y, bit)};
+    switch (o.type) {
+      case F_UR:
+        return {fma(l.c2, x1.x, mul(l.c1, x0.x)), fma(l.c2, x1.y, mul(l.c1, x0.y))};
+      case F_UI: {
+        const std::string o1 = sel(x0.y, x0.x, bit), o2 = sel(x1.x, x1.y, bit);
+        const std::string q1 = sel(x0.x, x0.y, bit), q2 = sel(x1.y, x1.x, bit);
+        return {fma(l.f2, o2, mul(l.f1, o1)), fma(l.g2, q2, mul(l.g1, q1))};
+      }
+      default: {  // F_U2: x0 term first, as pair()
+        Cx acc;
+        cfma(acc, l.m1, l.n1, x0, true);
+        cfma(acc, l.m2, l.n2, x1, false);
+        return acc;
+      }
+    }
+  }
+
   Cx shfl(const Cx& v, int t0) {
     Cx o{f(), f()};
     for (int c = 0; c < 2; ++c) {
@@ -631,15 +697,19 @@ struct Gen {
         set(r | (1 << rb), a1);
       }
     } else {
-      const int tl = tbit(t0);  // a fixed lane position
+      const int tl = tbit(t0);  // a lane position
       const std::string bit = p(), a = r();
       e("and.b32 %s, %%ltid, %u;", a.c_str(), 1u << tl);
       e("setp.ne.b32 %s, %s, 0;", bit.c_str(), a.c_str());
-      const LaneC lc = lane_coefs(o, bit);
+      // interpreter lane bit (tile bit < 5): its lane formulas; else pair() order
+      const bool lane_form = t0 < 5;
+      const LaneC lc = lane_form ? lane_coefs(o, bit) : LaneC();
+      const LaneP lp = lane_form ? LaneP() : lanep_coefs(o, bit);
       for (int r = 0; r < R; ++r) {
         if (((uint32_t)r & mr) != pr) continue;
         const Cx pp = shfl({vx(r), vy(r)}, tl);
-        const Cx z = lane(o, lc, {vx(r), vy(r)}, pp, bit);
+        const Cx z = lane_form ? lane(o, lc, {vx(r), vy(r)}, pp, bit)
+                               : lane_pair(o, lp, {vx(r), vy(r)}, pp, bit);
         if (bt.empty()) {
           set(r, z);
         } else {
@@ -948,6 +1018,7 @@ struct Gen {
   // targets of the longest run of upcoming ops whose register requirements fit
   // nreg positions together (interval covering: the fewest round trips).
   uint32_t plan_set(int o) const {
+    if (pool) return plan_pool(o);
     uint32_t S = 0;
     for (int q = o; q < P.nops; ++q) {
       if (P.h[q].type == F_DTAB) {
@@ -964,7 +1035,59 @@ struct Gen {
   }
   // Placement change (no code): every bit of S not register-held takes the register
   // position of a bit outside S, the one with the furthest next use first.
+  // Lane-pool requirement / plan: 1-target gates and SWAP / U4 need their non-fixed-lane
+  // targets at cheap positions (registers or movable lanes); an 8x8 gate ends the run.
+  uint32_t plan_pool(int o) const {
+    const int npool = nreg + (5 - FL);
+    uint32_t S = 0;
+    for (int q = o; q < P.nops; ++q) {
+      const FHdr& h = P.h[q];
+      if (h.type == F_DTAB) {
+        q += h.m;
+        continue;
+      }
+      if (h.type == F_DIAG1 || h.type == F_DIAGN) continue;
+      if (h.type == F_U8) break;
+      int ts[3];
+      const int m = op_targets(h, ts);
+      uint32_t b = 0;
+      for (int s_ = 0; s_ < m; ++s_)
+        if (!fixed_lane(ts[s_])) b |= 1u << ts[s_];
+      if (__builtin_popcount(S | b) > npool) break;
+      S |= b;
+    }
+    return S;
+  }
+  void place_pool(uint32_t S, int o) {
+    for (int b = 0; b < K; ++b) {
+      if (!((S >> b) & 1) || cheap(b)) continue;
+      // victim: a cheap position holding a bit outside S, furthest next use (ties: register)
+      int best_r = -1, best_l = -1, bd = -1;
+      for (int j = 0; j < nreg; ++j) {
+        if ((S >> rpos[j]) & 1) continue;
+        const int d = next_use(rpos[j], o);
+        if (d > bd) { bd = d; best_r = j; best_l = -1; }
+      }
+      for (int j = FL; j < 5; ++j) {
+        if ((S >> tpos[j]) & 1) continue;
+        const int d = next_use(tpos[j], o);
+        if (d > bd) { bd = d; best_l = j; best_r = -1; }
+      }
+      const int tb = tbit(b);
+      if (best_r >= 0) {
+        tpos[tb] = rpos[best_r];
+        rpos[best_r] = b;
+      } else {
+        tpos[tb] = tpos[best_l];
+        tpos[best_l] = b;
+      }
+    }
+  }
   void place(uint32_t S, int o) {
+    if (pool) {
+      place_pool(S, o);
+      return;
+    }
     for (int b = 0; b < K; ++b) {
       if (!((S >> b) & 1) || reg_of(b) >= 0) continue;
       int best = -1, bd = -1;
@@ -1010,6 +1133,7 @@ struct Gen {
   // furthest next use, register-held bits that are not targets of op o) with one
   // round trip through the shared-memory tile.
   void remap(const std::vector<int>& need, const int* ts, int m, int o) {
+    body += "  // remap\n";
     if (in_regs) regs_to_tile();  // under the old placement
     if (greedy) {
       place(plan_set(o), o);
@@ -1042,7 +1166,7 @@ struct Gen {
   void op_lanereg2(const FHdr& h) {
     const std::string end = L();
     tile_pred(h.mhi, h.phi, end);
-    const bool a_is_t0 = fixed_lane(h.t0);
+    const bool a_is_t0 = at_lane(h.t0) && reg_of(h.t1) >= 0;
     const int ta = a_is_t0 ? h.t0 : h.t1, tb = a_is_t0 ? h.t1 : h.t0;
     const int tl = tbit(ta), rb = reg_of(tb);
     // local index j = 2 bit(t0) + bit(t1)
@@ -1261,6 +1385,51 @@ struct Gen {
     label(end);
   }
 
+  // Lane-pool dispatch: every target of a 1-target gate or SWAP / U4 at a cheap
+  // position (register or lane) after at most one greedy round trip; 1-target gates at a
+  // lane run by shuffle, 2-target gates by registers / shuffles (regmulti, lanereg2,
+  // lanelane2); 8x8 gates in registers when all three targets are there, else as a
+  // shared-memory op.
+  void dispatch_pool(int o, const FHdr& h, const int* ts, int m) {
+    if (h.type == F_U8) {
+      if (reg_of(ts[0]) >= 0 && reg_of(ts[1]) >= 0 && reg_of(ts[2]) >= 0) {
+        ensure_regs(o);
+        op_regmulti(h);
+      } else {
+        if (in_regs) {
+          regs_to_tile();
+          in_regs = false;
+        }
+        sync();
+        op_smem(h);
+      }
+      return;
+    }
+    bool ok = true;
+    for (int s_ = 0; s_ < m; ++s_) ok &= fixed_lane(ts[s_]) || cheap(ts[s_]);
+    if (!ok) {
+      body += "  // remap\n";
+      if (in_regs) regs_to_tile();
+      place_pool(plan_pool(o), o);
+      sync();
+      emit_taddr();
+      tile_to_regs();
+      in_regs = true;
+    }
+    ensure_regs(o);
+    if (m == 1) {
+      op_reg1q(h);
+      return;
+    }
+    const bool r0 = reg_of(ts[0]) >= 0, r1 = reg_of(ts[1]) >= 0;
+    if (r0 && r1)
+      op_regmulti(h);
+    else if (!r0 && !r1)
+      op_lanelane2(h);
+    else
+      op_lanereg2(h);
+  }
+
   // ---- whole kernel -------------------------------------------------------------
   std::string build() {
     const FTile& tg = P.tile;
@@ -1315,6 +1484,11 @@ struct Gen {
     for (int o = 0; o < P.nops; ++o) {
       const FHdr& h = P.h[o];
       const int type = h.type;
+      body += "  // op " + std::to_string(o) + " type " + std::to_string(type) + " t " +
+              std::to_string(h.t0) + "," + std::to_string(h.t1) + "," + std::to_string(h.t2) +
+              " m " + std::to_string(h.m) + " regs";
+      for (int j = 0; j < nreg; ++j) body += " " + std::to_string(rpos[j]);
+      body += "\n";
       if (type == F_DTAB) {
         op_dtab(o);
         o += h.m;
@@ -1330,6 +1504,10 @@ struct Gen {
       }
       int ts[3];
       const int m = op_targets(h, ts);
+      if (pool) {
+        dispatch_pool(o, h, ts, m);
+        continue;
+      }
       bool any_lane = false;
       for (int s_ = 0; s_ < m; ++s_) any_lane |= fixed_lane(ts[s_]);
       // 1-target gates: fixed lane bits by shuffle, everything else in registers (a
@@ -1572,7 +1750,8 @@ int jit_config(const LaunchCtx& ctx, int K) {
   return ((t == 512 && K >= 9) ? 512 : (t == 128 && K >= 8) ? 128 : 256) |
          (ctx.opt->jit_lane_move ? JIT_LANE_MOVE : 0) |
          (ctx.opt->jit_greedy_place ? JIT_GREEDY_PLACE : 0) |
-         (ctx.opt->jit_lane_reg2 ? JIT_LANE_REG2 : 0);
+         (ctx.opt->jit_lane_reg2 ? JIT_LANE_REG2 : 0) |
+         (ctx.opt->jit_lane_pool ? JIT_LANE_POOL : 0);
 }
 
 size_t jit_cache_size() {

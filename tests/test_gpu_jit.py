@@ -26,8 +26,10 @@ def L():
 
 
 def _run(L, n, psi, gates, fuse, tile=None, low=None, c64=False, reorder=1, threads=256,
-         lane_move=None, greedy=None, lane_reg2=None):
+         lane_move=None, greedy=None, lane_reg2=None, pool=None):
     with L.State.create(n, c64=c64) as st:
+        if pool is not None:
+            st.set_option(L.OPT_JIT_LANE_POOL, pool)
         if lane_reg2 is not None:
             st.set_option(L.OPT_JIT_LANE_REG2, lane_reg2)
         if greedy is not None:
@@ -85,9 +87,9 @@ def test_jit_512_threads_equals_interpreter(L, n, tile, threads):
 @pytest.mark.parametrize("c64", [False, True])
 @pytest.mark.parametrize("threads", [128, 256, 512])
 @pytest.mark.parametrize("tile", [9, 12])
-@pytest.mark.parametrize("greedy", [0, 1])
+@pytest.mark.parametrize("greedy,pool", [(0, 0), (1, 0), (1, 1)])
 @pytest.mark.parametrize("lane_move", [0, 1])
-def test_jit_placement_variants_equal_interpreter(L, lane_move, greedy, tile, threads, c64):
+def test_jit_placement_variants_equal_interpreter(L, lane_move, greedy, pool, tile, threads, c64):
     """Tile-bit placement variants of the compiled passes: LFQS_OPT_JIT_LANE_MOVE (lane
     tile bits 3-4, complex64: 4, move into register positions and keep the interpreter's
     lane formulas there) and LFQS_OPT_JIT_GREEDY_PLACE (multi-bit remaps) -- all
@@ -101,11 +103,11 @@ def test_jit_placement_variants_equal_interpreter(L, lane_move, greedy, tile, th
              W.sycamore_like(3, 5, 4, seed=threads) + W.random_gate_list(n, 150, seed=9, max_controls=2))
     a, _ = _run(L, n, psi, gates, True, tile, c64=c64)
     b, _ = _run(L, n, psi, gates, "jit", tile, c64=c64, threads=threads, lane_move=lane_move,
-                greedy=greedy)
+                greedy=greedy, pool=pool)
     assert np.array_equal(a, b)
     c, _ = _run(L, n, psi, gates, "phase", tile, c64=c64)
     d, _ = _run(L, n, psi, gates, "jit+phase", tile, c64=c64, threads=threads,
-                lane_move=lane_move, greedy=greedy)
+                lane_move=lane_move, greedy=greedy, pool=pool)
     assert np.array_equal(c, d)
     tol = 2e-5 if c64 else 1e-12
     assert np.max(np.abs(b - O.run_circuit(n, gates, psi.copy()))) <= tol
@@ -113,8 +115,8 @@ def test_jit_placement_variants_equal_interpreter(L, lane_move, greedy, tile, th
 
 @pytest.mark.parametrize("c64", [False, True])
 @pytest.mark.parametrize("tile", [9, 10, 12])
-@pytest.mark.parametrize("lane_reg2", [0, 1])
-def test_jit_lane_register_2q_equals_interpreter(L, lane_reg2, tile, c64):
+@pytest.mark.parametrize("lane_reg2,pool", [(0, 0), (1, 0), (1, 1)])
+def test_jit_lane_register_2q_equals_interpreter(L, lane_reg2, pool, tile, c64):
     """LFQS_OPT_JIT_LANE_REG2: SWAP / 2-target dense gates with one target on a lane
     bit and the other register-held run by shuffles in registers -- bit-identical to
     the interpreter's shared-memory op (2-target gates on every placement, with
@@ -124,9 +126,10 @@ def test_jit_lane_register_2q_equals_interpreter(L, lane_reg2, tile, c64):
     if c64:
         psi = psi.astype(np.complex64).astype(np.complex128)
     gates = (W.random_gate_list(n, 300, seed=tile, max_targets=2, max_controls=2) +
-             W.sycamore_like(2, 7, 6, seed=tile))
+             W.sycamore_like(2, 7, 6, seed=tile) + W.random_layered(n, 4, seed=tile) +
+             W.random_gate_list(n, 100, seed=tile + 1, max_targets=3, max_controls=1))
     a, _ = _run(L, n, psi, gates, True, tile, c64=c64)
-    b, _ = _run(L, n, psi, gates, "jit", tile, c64=c64, lane_reg2=lane_reg2)
+    b, _ = _run(L, n, psi, gates, "jit", tile, c64=c64, lane_reg2=lane_reg2, pool=pool)
     assert np.array_equal(a, b)
     tol = 2e-5 if c64 else 1e-12
     assert np.max(np.abs(b - O.run_circuit(n, gates, psi.copy()))) <= tol
