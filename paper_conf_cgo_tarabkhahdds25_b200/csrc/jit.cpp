@@ -73,6 +73,7 @@ struct Gen {
   bool greedy = false;  // greedy placement (JIT_GREEDY_PLACE)
   bool lane_reg2 = false;  // SWAP / U4 with one fixed-lane target by shuffles (JIT_LANE_REG2)
   bool pool = false;       // lane-pool placement (JIT_LANE_POOL)
+  bool partial_rt = false; // round trips move only re-placed amplitudes (JIT_PARTIAL_RT)
   int tpos[9] = {0, 1, 2, 3, 4, 5, 6, 7, 8};
   int rpos[8] = {8, 9, 10, 11, 12, 13, 14, 15};
   int nreg = 0;
@@ -88,6 +89,7 @@ struct Gen {
     greedy = (jc & JIT_GREEDY_PLACE) != 0;
     lane_reg2 = (jc & JIT_LANE_REG2) != 0;
     pool = (jc & JIT_LANE_POOL) && greedy && lane_reg2 && FL < 5 && nreg >= 1;
+    partial_rt = (jc & JIT_PARTIAL_RT) != 0;
     for (int j = 0; j < 5 + NWB; ++j) tpos[j] = j;
     for (int j = 0; j < nreg; ++j) rpos[j] = 5 + NWB + j;
   }
@@ -341,6 +343,99 @@ struct Gen {
         roff(r) * ES);
   }
   void sync() { e("bar.sync 0;"); }
+
+  // Placement change by a tile round trip that moves only the amplitudes whose (thread,
+  // slot) changes (LFQS_OPT_JIT_PARTIAL_RT): amplitude (t, r) of the old placement (ot,
+  // orp) stays in its register iff every position holds the same tile-index bit value
+  // under the new placement (tpos, rpos); the condition is the same in old and new
+  // coordinates, so one predicate per slot guards both the store and the load.  A swap
+  // of k position pairs moves 1 - 2^-k of the tile instead of all of it.
+  void partial_roundtrip(const int* ot, const int* orp) {
+    const int NTB = 5 + NWB;
+    auto old_thread_pos = [&](int b) {
+      for (int j = 0; j < NTB; ++j)
+        if (ot[j] == b) return j;
+      return -1;
+    };
+    auto old_slot_pos = [&](int b) {
+      for (int j = 0; j < nreg; ++j)
+        if (orp[j] == b) return j;
+      return -1;
+    };
+    // thread-thread equalities (runtime, same for every slot)
+    std::string ptt;
+    for (int j = 0; j < NTB; ++j) {
+      if (tpos[j] == ot[j]) continue;
+      const int jt = old_thread_pos(tpos[j]);
+      if (jt < 0) continue;
+      const std::string a = r(), q = p();
+      e("shr.u32 %s, %%ltid, %d;", a.c_str(), jt - j > 0 ? jt - j : 0);
+      if (j > jt) e("shl.b32 %s, %%ltid, %d;", a.c_str(), j - jt);
+      e("xor.b32 %s, %s, %%ltid;", a.c_str(), a.c_str());
+      e("and.b32 %s, %s, %u;", a.c_str(), a.c_str(), 1u << j);
+      if (ptt.empty()) {
+        e("setp.eq.b32 %s, %s, 0;", q.c_str(), a.c_str());
+      } else {
+        e("setp.eq.and.b32 %s, %s, 0, %s;", q.c_str(), a.c_str(), ptt.c_str());
+      }
+      ptt = q;
+    }
+    // per slot: (t & M) == V from thread-slot equalities; compile-time slot-slot ones
+    std::vector<std::string> pslot(R);
+    std::map<std::pair<uint32_t, uint32_t>, std::string> cache;
+    for (int r_ = 0; r_ < R; ++r_) {
+      bool never = false;
+      uint32_t M = 0, V = 0;
+      for (int j = 0; j < NTB; ++j) {  // new thread bit j holds tile bit tpos[j]
+        if (tpos[j] == ot[j]) continue;
+        const int js = old_slot_pos(tpos[j]);
+        if (js >= 0) {
+          M |= 1u << j;
+          V |= (uint32_t)((r_ >> js) & 1) << j;
+        }
+      }
+      for (int j = 0; j < nreg; ++j) {  // new slot bit j holds tile bit rpos[j]
+        if (rpos[j] == orp[j]) continue;
+        const int jt = old_thread_pos(rpos[j]);
+        if (jt >= 0) {
+          M |= 1u << jt;
+          V |= (uint32_t)((r_ >> j) & 1) << jt;
+        } else {
+          const int js = old_slot_pos(rpos[j]);
+          if (((r_ >> js) & 1) != ((r_ >> j) & 1)) never = true;
+        }
+      }
+      if (never) continue;  // always moves
+      auto it = cache.find({M, V});
+      if (it == cache.end()) {
+        const std::string a = r(), q = p();
+        e("and.b32 %s, %%ltid, %u;", a.c_str(), M);
+        if (ptt.empty())
+          e("setp.eq.b32 %s, %s, %u;", q.c_str(), a.c_str(), V);
+        else
+          e("setp.eq.and.b32 %s, %s, %u, %s;", q.c_str(), a.c_str(), V, ptt.c_str());
+        it = cache.emplace(std::make_pair(M, V), q).first;
+      }
+      pslot[r_] = it->second;
+    }
+    // stores of moving amplitudes under the old placement (old %taddr, old slot offsets)
+    for (int r_ = 0; r_ < R; ++r_) {
+      uint32_t o = 0;
+      for (int j = 0; j < nreg; ++j)
+        if ((r_ >> j) & 1) o |= 1u << orp[j];
+      const std::string g = pslot[r_].empty() ? "" : "@!" + pslot[r_] + " ";
+      e("%sst.shared.v2.%s [%%taddr+%u], {%s, %s};", g.c_str(), FT, o * ES, vx(r_).c_str(),
+        vy(r_).c_str());
+    }
+    sync();
+    emit_taddr();
+    for (int r_ = 0; r_ < R; ++r_) {
+      const std::string g = pslot[r_].empty() ? "" : "@!" + pslot[r_] + " ";
+      e("%sld.shared.v2.%s {%s, %s}, [%%taddr+%u];", g.c_str(), FT, vx(r_).c_str(),
+        vy(r_).c_str(), roff(r_) * ES);
+    }
+    in_regs = true;
+  }
 
   // ---- 2x2 functor semantics (fused_kernels.cu FX_/FY_/FH_/FR_/FI_/FU_) -----
   struct Op2 {
@@ -1134,7 +1229,11 @@ struct Gen {
   // round trip through the shared-memory tile.
   void remap(const std::vector<int>& need, const int* ts, int m, int o) {
     body += "  // remap\n";
-    if (in_regs) regs_to_tile();  // under the old placement
+    int ot[9], orp[8];
+    std::memcpy(ot, tpos, sizeof ot);
+    std::memcpy(orp, rpos, sizeof orp);
+    const bool partial = partial_rt && in_regs;
+    if (in_regs && !partial) regs_to_tile();  // under the old placement
     if (greedy) {
       place(plan_set(o), o);
     } else for (int b : need) {
@@ -1151,6 +1250,10 @@ struct Gen {
       }
       tpos[tbit(b)] = rpos[best];
       rpos[best] = b;
+    }
+    if (partial) {
+      partial_roundtrip(ot, orp);
+      return;
     }
     sync();
     emit_taddr();
@@ -1409,12 +1512,20 @@ struct Gen {
     for (int s_ = 0; s_ < m; ++s_) ok &= fixed_lane(ts[s_]) || cheap(ts[s_]);
     if (!ok) {
       body += "  // remap\n";
-      if (in_regs) regs_to_tile();
+      int ot[9], orp[8];
+      std::memcpy(ot, tpos, sizeof ot);
+      std::memcpy(orp, rpos, sizeof orp);
+      const bool partial = partial_rt && in_regs;
+      if (in_regs && !partial) regs_to_tile();
       place_pool(plan_pool(o), o);
-      sync();
-      emit_taddr();
-      tile_to_regs();
-      in_regs = true;
+      if (partial) {
+        partial_roundtrip(ot, orp);
+      } else {
+        sync();
+        emit_taddr();
+        tile_to_regs();
+        in_regs = true;
+      }
     }
     ensure_regs(o);
     if (m == 1) {
@@ -1751,7 +1862,8 @@ int jit_config(const LaunchCtx& ctx, int K) {
          (ctx.opt->jit_lane_move ? JIT_LANE_MOVE : 0) |
          (ctx.opt->jit_greedy_place ? JIT_GREEDY_PLACE : 0) |
          (ctx.opt->jit_lane_reg2 ? JIT_LANE_REG2 : 0) |
-         (ctx.opt->jit_lane_pool ? JIT_LANE_POOL : 0);
+         (ctx.opt->jit_lane_pool ? JIT_LANE_POOL : 0) |
+         (ctx.opt->jit_partial_rt ? JIT_PARTIAL_RT : 0);
 }
 
 size_t jit_cache_size() {

@@ -16,6 +16,7 @@ constexpr int JIT_LANE_MOVE = 1 << 16;  // lane bits >= 3 (c64: >= 4) movable (L
 constexpr int JIT_GREEDY_PLACE = 1 << 17;  // multi-bit remaps (LFQS_OPT_JIT_GREEDY_PLACE)
 constexpr int JIT_LANE_REG2 = 1 << 18;     // lane/register 2-target gates (LFQS_OPT_JIT_LANE_REG2)
 constexpr int JIT_LANE_POOL = 1 << 19;     // movable lanes as cheap positions (LFQS_OPT_JIT_LANE_POOL)
+constexpr int JIT_PARTIAL_RT = 1 << 20;    // round trips move only re-placed amplitudes
 
 // PTX of one fused pass: structure baked in, coefficients a kernel parameter.
 std::string jit_ptx(const FProg& P, int K, bool c64, int jc);

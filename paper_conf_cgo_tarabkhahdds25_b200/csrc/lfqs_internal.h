@@ -96,6 +96,7 @@ struct Options {
   bool fuse_merge_commuting = true;  // merge same-qubit 1-target gates across commuting gates
   bool jit_lane_move = true;     // compiled passes may move lane bits >= 3 into registers
   bool jit_greedy_place = true;  // compiled passes: remaps fill every register position
+  bool jit_partial_rt = true;    // compiled passes: round trips move only re-placed amplitudes
   bool jit_lane_pool = false;    // compiled passes: movable lanes serve gates like registers
   bool jit_lane_reg2 = true;     // compiled passes: SWAP/U4 on a lane bit + a register bit by shuffles
 };

@@ -26,8 +26,10 @@ def L():
 
 
 def _run(L, n, psi, gates, fuse, tile=None, low=None, c64=False, reorder=1, threads=256,
-         lane_move=None, greedy=None, lane_reg2=None, pool=None):
+         lane_move=None, greedy=None, lane_reg2=None, pool=None, partial=None):
     with L.State.create(n, c64=c64) as st:
+        if partial is not None:
+            st.set_option(L.OPT_JIT_PARTIAL_RT, partial)
         if pool is not None:
             st.set_option(L.OPT_JIT_LANE_POOL, pool)
         if lane_reg2 is not None:
@@ -115,12 +117,14 @@ def test_jit_placement_variants_equal_interpreter(L, lane_move, greedy, pool, ti
 
 @pytest.mark.parametrize("c64", [False, True])
 @pytest.mark.parametrize("tile", [9, 10, 12])
-@pytest.mark.parametrize("lane_reg2,pool", [(0, 0), (1, 0), (1, 1)])
-def test_jit_lane_register_2q_equals_interpreter(L, lane_reg2, pool, tile, c64):
+@pytest.mark.parametrize("lane_reg2,pool,partial", [(0, 0, 1), (1, 0, 1), (1, 1, 1), (1, 0, 0),
+                                                    (1, 1, 0)])
+def test_jit_lane_register_2q_equals_interpreter(L, lane_reg2, pool, partial, tile, c64):
     """LFQS_OPT_JIT_LANE_REG2: SWAP / 2-target dense gates with one target on a lane
     bit and the other register-held run by shuffles in registers -- bit-identical to
     the interpreter's shared-memory op (2-target gates on every placement, with
-    controls, Sycamore-like fSim layers)."""
+    controls, Sycamore-like fSim layers); with and without the lane pool and partial
+    round trips (LFQS_OPT_JIT_PARTIAL_RT)."""
     n = 14
     psi = W.random_state(n, 5 * tile + 1)
     if c64:
@@ -129,7 +133,8 @@ def test_jit_lane_register_2q_equals_interpreter(L, lane_reg2, pool, tile, c64):
              W.sycamore_like(2, 7, 6, seed=tile) + W.random_layered(n, 4, seed=tile) +
              W.random_gate_list(n, 100, seed=tile + 1, max_targets=3, max_controls=1))
     a, _ = _run(L, n, psi, gates, True, tile, c64=c64)
-    b, _ = _run(L, n, psi, gates, "jit", tile, c64=c64, lane_reg2=lane_reg2, pool=pool)
+    b, _ = _run(L, n, psi, gates, "jit", tile, c64=c64, lane_reg2=lane_reg2, pool=pool,
+                partial=partial)
     assert np.array_equal(a, b)
     tol = 2e-5 if c64 else 1e-12
     assert np.max(np.abs(b - O.run_circuit(n, gates, psi.copy()))) <= tol
