@@ -59,7 +59,7 @@ EXPORTS = [
     "lfqs_state_create_ex", "lfqs_state_wrap_ex", "lfqs_copy_in_c64", "lfqs_copy_out_c64",
     "lfqs_circuit_compile", "lfqs_circuit_launch", "lfqs_circuit_destroy",
     "lfqs_state_create_p2p", "lfqs_state_p2p_handle", "lfqs_state_p2p_attach",
-    "lfqs_state_exchange_stats", "lfqs_jit_precompile",
+    "lfqs_state_exchange_stats", "lfqs_jit_precompile", "lfqs_run_circuit_streamed",
 ]
 P2P_HANDLE_BYTES = 256
 STATE_C64 = 1
@@ -122,6 +122,8 @@ def lib():
             "lfqs_copy_out": [vp, u64, u64, dp],
             "lfqs_apply_gate": [vp, C.c_int, ip, C.c_int, ip, C.c_int, dp, C.c_int, dp],
             "lfqs_run_circuit": [vp, C.POINTER(LfqsGate), C.c_size_t, C.c_uint32],
+            "lfqs_run_circuit_streamed": [vp, dp, C.POINTER(LfqsGate), C.c_size_t, C.c_uint32,
+                                          C.c_int],
             "lfqs_circuit_compile": [vp, C.POINTER(LfqsGate), C.c_size_t, C.c_uint32,
                                      C.POINTER(vp), C.POINTER(u64)],
             "lfqs_circuit_launch": [vp],
@@ -346,6 +348,19 @@ def lfqs_run_circuit(h: int, gates, flags: int = FUSE_NONE):
     else:
         arr, n, keep = marshal_gates(gates)
     _check(lib().lfqs_run_circuit(h, arr, n, flags))
+
+
+def lfqs_run_circuit_streamed(h: int, host: np.ndarray, gates, flags: int = FUSE_NONE,
+                              chunk_bits: int = 3):
+    """host: the whole state, a C-contiguous complex128 array (page-locked for overlap);
+    it must stay alive and unchanged until the next synchronising call."""
+    assert host.dtype == np.complex128 and host.flags.c_contiguous
+    if isinstance(gates, tuple) and len(gates) == 3 and isinstance(gates[1], int):
+        arr, n, keep = gates
+    else:
+        arr, n, keep = marshal_gates(gates)
+    _check(lib().lfqs_run_circuit_streamed(h, _dp(host.view(np.float64)), arr, n, flags,
+                                           chunk_bits))
 
 
 def lfqs_circuit_compile(h: int, gates, flags: int = FUSE_NONE):
@@ -613,6 +628,11 @@ class State:
         """fuse: False (one pass per gate), True (FUSE_LOW, exact for permutation/diagonal
         gates) or "phase" (FUSE_LOW | FUSE_PHASE)."""
         lfqs_run_circuit(self.h, gates, fuse_flags(fuse))
+
+    def run_circuit_streamed(self, host: np.ndarray, gates, fuse=False, chunk_bits: int = 3):
+        """Whole-state upload from `host` overlapped with the circuit (lfqs_run_circuit_streamed)."""
+        assert host.size == 1 << self.n
+        lfqs_run_circuit_streamed(self.h, host, gates, fuse_flags(fuse), chunk_bits)
 
     def compile(self, gates, fuse: bool = False) -> Circuit:
         return Circuit(self, gates, fuse)

@@ -254,6 +254,18 @@ lfqs_status lfqs_run_circuit(lfqs_state* s, const lfqs_gate* gates, size_t n_gat
   });
 }
 
+lfqs_status lfqs_run_circuit_streamed(lfqs_state* s, const double* host_interleaved,
+                                      const lfqs_gate* gates, size_t n_gates, uint32_t flags,
+                                      int chunk_bits) {
+  return guarded([&] {
+    require(s != nullptr && host_interleaved != nullptr, "NULL argument");
+    State* st = static_cast<State*>(s);
+    require(!st->c64, "streamed runs take complex128 host data (complex128 states)");
+    st->run_streamed(host_interleaved, decode_circuit(st, gates, n_gates, flags), flags,
+                     chunk_bits);
+  });
+}
+
 lfqs_status lfqs_circuit_compile(lfqs_state* s, const lfqs_gate* gates, size_t n_gates,
                                  uint32_t flags, lfqs_circuit** out, uint64_t* kernels_out) {
   return guarded([&] {

@@ -165,6 +165,7 @@ State::~State() {
   if (d_partials) cudaFree(d_partials);
   if (d_probs) cudaFree(d_probs);
   if (own_stream && stream) cudaStreamDestroy(stream);
+  if (copy_stream) cudaStreamDestroy(copy_stream);
 }
 
 void State::set_stream(cudaStream_t s) {
@@ -380,6 +381,71 @@ void State::run(const std::vector<Decoded>& gates, uint32_t flags) {
   std::vector<PlanOp> ops;
   plan.plan_circuit(gates, ops);  // Belady lookahead over the whole circuit
   execute(ops, fuse);
+}
+
+// Upload overlapped with computation (lfqs_run_circuit_streamed).  The state is split by
+// its top chunk_bits qubits into pieces of 2^(n - chunk_bits) amplitudes.  Every gate of
+// the longest circuit prefix whose targets and controls all lie below n - chunk_bits acts
+// inside each piece independently (G = I (x) G' on the piece index, Eq. 1), so piece c
+// runs that prefix as soon as its copy has landed -- with the same kernels and the same
+// per-amplitude arithmetic as on the whole state -- while later pieces are still in flight;
+// the rest of the circuit then runs on the whole state.  Bit-identical to copy_in + run.
+void State::run_streamed(const void* host, const std::vector<Decoded>& gates, uint32_t flags,
+                         int chunk_bits) {
+  DeviceGuard dg(device);
+  require(world == 1 && !soa, "streamed runs need a single-GPU AOS state");
+  require(chunk_bits >= 0 && chunk_bits <= 8 && chunk_bits < n, "chunk_bits must be in [0, 8]");
+  const bool fuse = (flags & LFQS_FUSE_LOW) != 0;
+  const int nl = n - chunk_bits;
+  size_t pre = 0;
+  for (; pre < gates.size(); ++pre) {
+    uint64_t m = gates[pre].cmask;
+    for (int s = 0; s < gates[pre].m; ++s) m |= 1ull << gates[pre].targets[s];
+    if (m >> nl) break;
+  }
+  if (copy_stream == nullptr)
+    LFQS_CUDA_CHECK(cudaStreamCreateWithFlags(&copy_stream, cudaStreamNonBlocking));
+  const int pieces = 1 << chunk_bits;
+  const size_t piece_bytes = (size_t)ab << nl;
+  std::vector<cudaEvent_t> ev(pieces, nullptr);
+  struct Events {
+    std::vector<cudaEvent_t>& e;
+    ~Events() {
+      for (cudaEvent_t x : e)
+        if (x) cudaEventDestroy(x);
+    }
+  } guard{ev};
+  // the copies must not overtake work already queued on the state's stream
+  cudaEvent_t start = nullptr;
+  LFQS_CUDA_CHECK(cudaEventCreateWithFlags(&start, cudaEventDisableTiming));
+  ev.push_back(start);
+  LFQS_CUDA_CHECK(cudaEventRecord(start, stream));
+  LFQS_CUDA_CHECK(cudaStreamWaitEvent(copy_stream, start, 0));
+  phase_tables = fuse && (flags & LFQS_FUSE_PHASE) != 0;
+  jit = fuse && (flags & LFQS_FUSE_JIT) != 0;
+  struct Reset {
+    bool& f;
+    bool& g;
+    ~Reset() { f = g = false; }
+  } reset{phase_tables, jit};
+  const std::vector<Decoded> prefix(gates.begin(), gates.begin() + pre);
+  for (int c = 0; c < pieces; ++c) {
+    LFQS_CUDA_CHECK(cudaEventCreateWithFlags(&ev[c], cudaEventDisableTiming));
+    LFQS_CUDA_CHECK(cudaMemcpyAsync(amps + (size_t)c * piece_bytes,
+                                    static_cast<const unsigned char*>(host) + (size_t)c * piece_bytes,
+                                    piece_bytes, cudaMemcpyHostToDevice, copy_stream));
+    LFQS_CUDA_CHECK(cudaEventRecord(ev[c], copy_stream));
+  }
+  for (int c = 0; c < pieces; ++c) {
+    LFQS_CUDA_CHECK(cudaStreamWaitEvent(stream, ev[c], 0));
+    if (prefix.empty()) continue;
+    LaunchCtx pc = ctx(0);
+    pc.amps = amps + (size_t)c * piece_bytes;
+    pc.n_local = nl;
+    run_local(pc, prefix, fuse);
+  }
+  const std::vector<Decoded> rest(gates.begin() + pre, gates.end());
+  if (!rest.empty()) run_local(ctx(0), rest, fuse);
 }
 
 Graph* State::compile(const std::vector<Decoded>& gates, uint32_t flags) {

@@ -67,6 +67,10 @@ struct State : lfqs_state {
   void copy_raw(uint64_t offset, uint64_t count, void* host, bool to_device);
   void apply(const Decoded& g);
   void run(const std::vector<Decoded>& gates, uint32_t flags);
+  // Uploads the whole state from `host` in 2^chunk_bits pieces on a copy stream while the
+  // circuit prefix that stays inside pieces runs on each landed piece; then the rest.
+  void run_streamed(const void* host, const std::vector<Decoded>& gates, uint32_t flags,
+                    int chunk_bits);
   // Captures the launches of run(gates, flags) into a CUDA graph (no GPU work).
   struct Graph* compile(const std::vector<Decoded>& gates, uint32_t flags);
   void measure_probs(const int* qubits, int nq, double* out);
@@ -82,6 +86,7 @@ struct State : lfqs_state {
   LaunchCtx ctx(int shard);
   bool phase_tables = false;  // LFQS_FUSE_PHASE of the run in progress
   bool jit = false;           // LFQS_FUSE_JIT of the run in progress
+  cudaStream_t copy_stream = nullptr;  // run_streamed uploads (created on first use)
   int n_shards() const { return virt ? world : 1; }
   int rank_of_shard(int shard) const { return virt ? shard : rank; }
   void execute(const std::vector<PlanOp>& ops, bool fuse);
