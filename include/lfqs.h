@@ -225,9 +225,11 @@ lfqs_status lfqs_run_circuit(lfqs_state* s, const lfqs_gate* gates, size_t n_gat
  * prefix of the circuit whose targets and controls all lie below n - chunk_bits acts inside
  * each piece (Eq. 1: I on the piece index (x) the gate), so every piece runs that prefix as
  * soon as it has landed while later pieces are still being copied; the remaining gates run
- * on the whole state.  Result: bit-identical to lfqs_copy_in of the whole state followed by
- * lfqs_run_circuit(flags).  Asynchronous like lfqs_run_circuit.  Single-GPU complex128 AOS
- * states only (else LFQS_ERR_INVALID_ARG). */
+ * on the whole state.  Result: with LFQS_FUSE_NONE bit-identical to lfqs_copy_in of the
+ * whole state followed by lfqs_run_circuit; with fusion the prefix and the rest are fused
+ * separately, so (as for fusion itself) permutation/diagonal results stay value-exact and
+ * dense ones agree within rounding.  Asynchronous like lfqs_run_circuit.  Single-GPU
+ * complex128 AOS states only (else LFQS_ERR_INVALID_ARG). */
 lfqs_status lfqs_run_circuit_streamed(lfqs_state* s, const double* host_interleaved,
                                       const lfqs_gate* gates, size_t n_gates, uint32_t flags,
                                       int chunk_bits);

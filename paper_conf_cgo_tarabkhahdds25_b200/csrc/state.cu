@@ -389,7 +389,8 @@ void State::run(const std::vector<Decoded>& gates, uint32_t flags) {
 // inside each piece independently (G = I (x) G' on the piece index, Eq. 1), so piece c
 // runs that prefix as soon as its copy has landed -- with the same kernels and the same
 // per-amplitude arithmetic as on the whole state -- while later pieces are still in flight;
-// the rest of the circuit then runs on the whole state.  Bit-identical to copy_in + run.
+// the rest of the circuit then runs on the whole state.  Without fusion bit-identical to
+// copy_in + run; fused, the prefix and the rest form separate passes (rounding only).
 void State::run_streamed(const void* host, const std::vector<Decoded>& gates, uint32_t flags,
                          int chunk_bits) {
   DeviceGuard dg(device);

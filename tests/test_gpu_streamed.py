@@ -1,7 +1,9 @@
 """lfqs_run_circuit_streamed: the whole-state upload overlapped with the circuit prefix
 that stays inside the upload pieces (Eq. 1: a gate below the piece bits acts on every
-piece independently).  Must equal lfqs_copy_in + lfqs_run_circuit bit for bit, for every
-piece count, fusion mode, and prefixes of any length (empty, partial, the whole circuit)."""
+piece independently).  Without fusion it must equal lfqs_copy_in + lfqs_run_circuit bit for
+bit, for every piece count and prefixes of any length (empty, partial, the whole circuit);
+with fusion the prefix and the rest are fused separately (different pass boundaries), so
+dense results agree within rounding and permutation/diagonal circuits stay exact."""
 import numpy as np
 import pytest
 
@@ -44,8 +46,15 @@ def test_streamed_equals_copy_in_then_run(L, cb, fuse):
     gates = low + W.random_gate_list(n, 150, seed=cb + 1, max_controls=2) + W.qft(n)
     a = _plain(L, n, psi, gates, fuse)
     b = _streamed(L, n, psi, gates, fuse, cb)
-    assert np.array_equal(a, b)
+    if fuse is False or cb == 0:
+        assert np.array_equal(a, b)
+    else:
+        assert np.max(np.abs(a - b)) <= 1e-12
     assert np.max(np.abs(b - O.run_circuit(n, gates, psi.copy()))) <= 1e-12
+    if fuse is True:
+        exact = [g for g in gates if g.exact]
+        assert np.array_equal(_streamed(L, n, psi, exact, fuse, cb),
+                              O.run_circuit(n, exact, psi.copy()))
 
 
 def test_streamed_edge_prefixes(L):
