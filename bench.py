@@ -411,12 +411,12 @@ def main():
         st.copy_out(rank << n_loc, 1 << n_loc, out=hv)
         mq = list(range(10))
         if world == 1:
-            # lfqs_run_circuit_streamed: the 16 GiB upload in 8 pieces on a copy stream,
-            # each piece running the sweep prefix that stays below qubit n - 3 as soon as
+            # lfqs_run_circuit_streamed: the 16 GiB upload in 32 pieces on a copy stream,
+            # each piece running the sweep prefix that stays below qubit n - 5 as soon as
             # it has landed (bit-identical to copy_in + the sweep; tests/test_gpu_streamed.py)
             marshalled = lfqs.marshal_gates([g for _, g in sweep])
             def e2e_step():
-                st.run_circuit_streamed(hv, marshalled, fuse=False, chunk_bits=3)
+                st.run_circuit_streamed(hv, marshalled, fuse=False, chunk_bits=5)
                 st.measure_probs(mq)
         else:
             def e2e_step():
