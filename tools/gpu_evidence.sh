@@ -22,7 +22,7 @@ timeout 900 ncu --set full --clock-control none --import-source on -k regex:k_gr
   -o $O/${TAG}_full_dense1 python tools/profile_gates.py --n 28 --reps 1 --gates RX:12,H:20 \
   > $O/${TAG}_ncu_full.out 2>&1
 timeout 2400 python tools/bench_circuits.py --n 30 --modes fused,phase,jit,jit+phase,unfused --oracle-s 12 > $O/${TAG}_circuits_n30.jsonl 2>&1
-timeout 2400 python tools/bench_circuits.py --n 33 --reps 1 --circuits qft,ghz,qpe,grover,random --modes fused,jit,jit+phase --oracle-s 12 > $O/${TAG}_circuits_n33.jsonl 2>&1
+timeout 2400 python tools/bench_circuits.py --n 33 --reps 1 --circuits qft,ghz,qpe,grover,random,sycamore --modes fused,jit,jit+phase --oracle-s 12 > $O/${TAG}_circuits_n33.jsonl 2>&1
 timeout 900 python tools/bench_circuits.py --n 31 --c64 --circuits qft,ghz,random --modes fused,jit,jit+phase > $O/${TAG}_circuits_c64_n31.jsonl 2>&1
 timeout 600 python tools/bench_small.py > $O/${TAG}_small.jsonl 2>&1
 for tool in memcheck racecheck synccheck; do
