@@ -374,7 +374,9 @@ lfqs_status lfqs_kernel_launches(const lfqs_state* s, uint64_t* count);
 #define LFQS_OPT_JIT_PARTIAL_RT 15 /* 1 (default): a compiled pass's tile round trip stores
                                       and reloads only the amplitudes whose (thread, slot)
                                       changes (a swap of k tile-bit positions moves 1 - 2^-k
-                                      of the tile); 0: the whole tile.  Bit-identical */
+                                      of the tile; complex128 states only -- measured
+                                      slower for complex64); 0: the whole tile.
+                                      Bit-identical */
 lfqs_status lfqs_set_option(lfqs_state* s, int option, int64_t value);
 const char* lfqs_last_error(void);
 int lfqs_abi_version(void);

@@ -89,7 +89,8 @@ struct Gen {
     greedy = (jc & JIT_GREEDY_PLACE) != 0;
     lane_reg2 = (jc & JIT_LANE_REG2) != 0;
     pool = (jc & JIT_LANE_POOL) && greedy && lane_reg2 && FL < 5 && nreg >= 1;
-    partial_rt = (jc & JIT_PARTIAL_RT) != 0;
+    // complex64: measured slower with partial round trips (QFT(31) 83 -> 96 ms), off there
+    partial_rt = (jc & JIT_PARTIAL_RT) != 0 && !c64;
     for (int j = 0; j < 5 + NWB; ++j) tpos[j] = j;
     for (int j = 0; j < nreg; ++j) rpos[j] = 5 + NWB + j;
   }
