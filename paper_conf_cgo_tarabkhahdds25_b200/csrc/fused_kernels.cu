@@ -783,8 +783,25 @@ uint32_t diag_support(const FHdr& h) {
 // preceded by an F_DTAB header and evaluated as one table per tile.
 constexpr int kMinTable = 3;
 constexpr int kTableBits = 8;
-void merge_phase_runs(FProg& P) {
+// A diagonal op whose factor depends on the tile (out-of-tile fixed bits or targets).
+bool tile_dependent(const FHdr& h) {
+  if (h.mhi != 0) return true;
+  if (h.type == F_DIAGN) {
+    const int ts[3] = {h.t0, h.t1, h.t2};
+    for (int s = 0; s < h.m; ++s)
+      if (ts[s] >= 64) return true;
+  }
+  return false;
+}
+
+// split: each run is first stable-partitioned into tile-invariant and tile-dependent
+// members (LFQS_OPT_FUSE_PHASE_SPLIT).  A tile-dependent member (e.g. a QFT CPhase whose
+// control lies outside the tile) adds no table bits, but every table entry evaluates it;
+// grouped apart, such members usually share their in-tile bits as a common predicate and
+// form a table of very few entries, so the per-tile build does ~1/256 of the work.
+void merge_phase_runs(FProg& P, bool split) {
   static thread_local FHdr out[kMaxOps];
+  static thread_local FHdr run[kMaxOps];
   int no = 0, o = 0;
   const int n = P.nops;
   int spare = kMaxOps - n;  // room for F_DTAB headers
@@ -795,30 +812,42 @@ void merge_phase_runs(FProg& P) {
     }
     int e = o;
     while (e < n && is_diag_op(P.h[e])) ++e;
-    for (int i = o; i < e;) {
-      uint32_t cm = P.h[i].mlo, cp = P.h[i].plo & cm, sup = diag_support(P.h[i]);
-      int j = i + 1;
-      for (; j < e && j - i < 255; ++j) {
-        const FHdr& g = P.h[j];
-        const uint32_t cm2 = cm & g.mlo & ~(cp ^ g.plo);
-        const uint32_t sup2 = sup | diag_support(g);
-        if (__builtin_popcount(sup2 & ~cm2) > kTableBits) break;
-        cm = cm2;
-        cp &= cm2;
-        sup = sup2;
+    int nr = 0;
+    if (split) {
+      for (int k = o; k < e; ++k)
+        if (!tile_dependent(P.h[k])) run[nr++] = P.h[k];
+    }
+    const int ninv = nr;
+    for (int k = o; k < e; ++k)
+      if (!split || tile_dependent(P.h[k])) run[nr++] = P.h[k];
+    // groups never straddle the invariant / dependent boundary
+    for (int part = 0; part < 2; ++part) {
+      const int b0 = part == 0 ? 0 : ninv, b1 = part == 0 ? ninv : nr;
+      for (int i = b0; i < b1;) {
+        uint32_t cm = run[i].mlo, cp = run[i].plo & cm, sup = diag_support(run[i]);
+        int j = i + 1;
+        for (; j < b1 && j - i < 255; ++j) {
+          const FHdr& g = run[j];
+          const uint32_t cm2 = cm & g.mlo & ~(cp ^ g.plo);
+          const uint32_t sup2 = sup | diag_support(g);
+          if (__builtin_popcount(sup2 & ~cm2) > kTableBits) break;
+          cm = cm2;
+          cp &= cm2;
+          sup = sup2;
+        }
+        if (j - i >= kMinTable && spare > 0) {
+          FHdr t;
+          std::memset(&t, 0, sizeof t);
+          t.type = F_DTAB;
+          t.m = (uint8_t)(j - i);
+          t.mlo = sup & ~cm;
+          t.plo = cm | (cp << 16);
+          out[no++] = t;
+          --spare;
+        }
+        for (int k = i; k < j; ++k) out[no++] = run[k];
+        i = j;
       }
-      if (j - i >= kMinTable && spare > 0) {
-        FHdr t;
-        std::memset(&t, 0, sizeof t);
-        t.type = F_DTAB;
-        t.m = (uint8_t)(j - i);
-        t.mlo = sup & ~cm;
-        t.plo = cm | (cp << 16);
-        out[no++] = t;
-        --spare;
-      }
-      for (int k = i; k < j; ++k) out[no++] = P.h[k];
-      i = j;
     }
     o = e;
   }
@@ -895,7 +924,7 @@ void build_program(const LaunchCtx& ctx, const TileCfg& cfg, uint64_t in_tile,
     prog.push_back(g);
   }
   for (const Decoded& g : prog) encode(g, tm, P);
-  if (ctx.phase_tables) merge_phase_runs(P);
+  if (ctx.phase_tables) merge_phase_runs(P, ctx.opt->fuse_phase_split);
 }
 
 // Launches an encoded pass: the compiled kernel of its program (LFQS_FUSE_JIT)

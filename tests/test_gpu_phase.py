@@ -50,8 +50,10 @@ def diag_heavy(n, count, seed):
     return out
 
 
-def _run(L, n, psi, gates, fuse, tile=None, low=None, c64=False):
+def _run(L, n, psi, gates, fuse, tile=None, low=None, c64=False, split=None):
     with L.State.create(n, c64=c64) as st:
+        if split is not None:
+            st.set_option(L.OPT_FUSE_PHASE_SPLIT, split)
         if tile:
             st.set_option(L.OPT_FUSE_TILE_QUBITS, tile)
         if low:
@@ -63,14 +65,19 @@ def _run(L, n, psi, gates, fuse, tile=None, low=None, c64=False):
         return out, st.launches() - c0
 
 
+@pytest.mark.parametrize("split", [0, 1])
 @pytest.mark.parametrize("low", [5, 7])
 @pytest.mark.parametrize("tile", [8, 10, 12])
 @pytest.mark.parametrize("n", [12, 17])
-def test_phase_tables_diag_heavy(L, n, tile, low):
+def test_phase_tables_diag_heavy(L, n, tile, low, split):
+    """split: LFQS_OPT_FUSE_PHASE_SPLIT (tile-invariant and tile-dependent diagonals in
+    separate tables) -- a different rounding order, the same bar."""
     psi = W.random_state(n, 31 * n + tile)
     gates = diag_heavy(n, 400, seed=n * 100 + tile + low)
     ref = O.run_circuit(n, gates, psi.copy())
-    got, passes = _run(L, n, psi, gates, "phase", tile, low)
+    got, passes = _run(L, n, psi, gates, "phase", tile, low, split=split)
+    jit, _ = _run(L, n, psi, gates, "jit+phase", tile, low, split=split)
+    assert np.array_equal(got, jit)  # compiled == interpreted, bit for bit
     assert np.max(np.abs(got - ref)) <= 1e-12
     exact, passes_exact = _run(L, n, psi, gates, True, tile, low)
     assert np.max(np.abs(got - exact)) <= 1e-12

@@ -64,6 +64,8 @@ def main():
     ap.add_argument("--jit-threads", type=int, default=256, help="LFQS_OPT_JIT_THREADS (128/256/512)")
     ap.add_argument("--lane-move", type=int, default=-1,
                     help="LFQS_OPT_JIT_LANE_MOVE (0/1; -1: library default)")
+    ap.add_argument("--phase-split", type=int, default=-1,
+                    help="LFQS_OPT_FUSE_PHASE_SPLIT (0/1; -1: library default)")
     ap.add_argument("--partial-rt", type=int, default=-1,
                     help="LFQS_OPT_JIT_PARTIAL_RT (0/1; -1: library default)")
     ap.add_argument("--pool", type=int, default=-1,
@@ -120,6 +122,8 @@ def main():
             st.set_option(L.OPT_FUSE_TMA_MAX_CHUNKS, args.tma)
         st.set_option(L.OPT_FUSE_REORDER, args.reorder)
         st.set_option(L.OPT_JIT_THREADS, args.jit_threads)
+        if args.phase_split >= 0:
+            st.set_option(L.OPT_FUSE_PHASE_SPLIT, args.phase_split)
         if args.partial_rt >= 0:
             st.set_option(L.OPT_JIT_PARTIAL_RT, args.partial_rt)
         if args.pool >= 0:
@@ -168,7 +172,7 @@ def main():
                        "conv_GBps": 2.0 * ab * 2 ** n * len(gates) / (t / 1e3) / 1e9,
                        "pass_GBps": 2.0 * ab * 2 ** n * passes / (t / 1e3) / 1e9,
                        "dtype": "c64" if args.c64 else "c128", "world": args.world,
-                       "exchanges": x1 - x0, "lane_move": args.lane_move, "merge": args.merge, "greedy": args.greedy, "lane_reg2": args.lane_reg2, "pool": args.pool, "partial_rt": args.partial_rt,
+                       "exchanges": x1 - x0, "lane_move": args.lane_move, "merge": args.merge, "greedy": args.greedy, "lane_reg2": args.lane_reg2, "pool": args.pool, "partial_rt": args.partial_rt, "phase_split": args.phase_split,
                        "hbm_peak_GBps": peak, "peak_source": peak_src}
                 # fraction of the HBM roofline: per pass actually made, and against the
                 # north-star convention of one 2*16*2^n-byte pass per gate
