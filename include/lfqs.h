@@ -377,12 +377,13 @@ lfqs_status lfqs_kernel_launches(const lfqs_state* s, uint64_t* count);
                                       of the tile; complex128 states only -- measured
                                       slower for complex64); 0: the whole tile.
                                       Bit-identical */
-#define LFQS_OPT_FUSE_PHASE_SPLIT 16 /* 1 (default): LFQS_FUSE_PHASE groups the tile-invariant
+#define LFQS_OPT_FUSE_PHASE_SPLIT 16 /* 1: LFQS_FUSE_PHASE groups the tile-invariant
                                         and the tile-dependent diagonals of a run separately
                                         (the latter -- e.g. QFT CPhases controlled from
                                         outside the tile -- become tables of few entries);
-                                        0: one greedy grouping in program order.  Changes
-                                        the rounding order only (phase-table tolerance) */
+                                        0 (default; measured 1-9 % faster): one greedy
+                                        grouping in program order.  Changes the rounding
+                                        order only (phase-table tolerance) */
 lfqs_status lfqs_set_option(lfqs_state* s, int option, int64_t value);
 const char* lfqs_last_error(void);
 int lfqs_abi_version(void);
