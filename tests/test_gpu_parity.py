@@ -312,3 +312,71 @@ def test_lane_group_dense_low_targets(L, n, c64):
                 outs.append(st.copy_out())
         assert np.array_equal(outs[0], outs[1]), g  # forced lane-group == group kernel
         assert np.max(np.abs(outs[0] - ref)) <= tol, g
+
+
+# ---------------------------------------------------------------------------
+# Maximum sizes on one B200 (180 GB HBM3e): n = 33 complex128 and n = 34 complex64,
+# 128 GiB each (BASELINE configs[2]); sampled outputs against the sparse oracle and
+# closed forms
+# ---------------------------------------------------------------------------
+
+def _free_gib():
+    import torch
+    free, _ = torch.cuda.mem_get_info()
+    return free / 2 ** 30
+
+
+def test_maximum_size_n33_c128(L):
+    if _free_gib() < 132:
+        pytest.skip("needs 128 GiB of free device memory")
+    n, seed = 33, 0x5EED33
+    rng = np.random.default_rng(33)
+    s2 = math.sqrt(0.5)
+    top = (1 << n) - 1
+    with L.State.create(n) as st:
+        # single gates on the top qubit / spanning the whole index range vs the sparse oracle
+        for g in [W.Gate("H", (n - 1,)), W.Gate("UNITARY2", (0, n - 1), (), (), W.haar_unitary(2, 9)),
+                  W.TOFFOLI(n - 2, 1, n - 1), W.CPHASE(n - 1, 0, 0.7), W.Gate("U3", (16,), (n - 1,),
+                                                                            (0.3, 1.1, -0.4))]:
+            st.init_random(seed)
+            st.apply(g)
+            tm = sum(1 << t for t in g.targets)
+            m = len(g.targets)
+            bases = rng.integers(0, 1 << n, 16, dtype=np.uint64) & np.uint64(~tm & top)
+            idx = np.unique(np.array([int(b) | sum(((j >> (m - 1 - s)) & 1) << t
+                                                   for s, t in enumerate(g.targets))
+                                      for b in bases for j in range(1 << m)], dtype=np.uint64))
+            ref = O.apply_gate_sparse(n, g, idx, W.random_amplitudes_at(seed, idx))
+            got = np.array([st.copy_out(int(k), 1)[0] for k in idx])
+            _cmp(got, ref, g.exact, f"n=33 {g.label()}")
+        # GHZ(33), compiled fused passes: two amplitudes of exactly 1/sqrt(2), zeros elsewhere
+        st.init_basis(0)
+        st.run_circuit(W.ghz(n), fuse="jit")
+        assert st.copy_out(0, 1)[0] == s2 and st.copy_out(top, 1)[0] == s2
+        for k in rng.integers(1, top, 32):
+            assert st.copy_out(int(k), 1)[0] == 0
+        assert st.measure_probs([]).sum() == 1.0
+        # QFT(33)|x>, compiled passes with phase tables: closed form on sampled amplitudes
+        x = 0x1F2E3D4C5 & top
+        st.init_basis(x)
+        st.run_circuit(W.qft(n), fuse="jit+phase")
+        ys = [0, 1, top] + [int(v) for v in rng.integers(0, 1 << n, 61)]
+        got = np.array([st.copy_out(y, 1)[0] for y in ys])
+        ref = np.array([np.exp(2j * np.pi * ((x * y) % (1 << n)) / (1 << n)) for y in ys]) \
+            / math.sqrt(2.0 ** n)
+        assert np.max(np.abs(got - ref)) <= 1e-12
+
+
+def test_maximum_size_n34_c64(L):
+    if _free_gib() < 132:
+        pytest.skip("needs 128 GiB of free device memory")
+    n = 34
+    top = (1 << n) - 1
+    with L.State.create(n, c64=True) as st:
+        st.init_basis(0)
+        st.run_circuit(W.ghz(n), fuse="jit")
+        s2 = float(np.float32(math.sqrt(0.5)))
+        assert st.copy_out(0, 1)[0] == s2 and st.copy_out(top, 1)[0] == s2
+        rng = np.random.default_rng(34)
+        for k in rng.integers(1, top, 32):
+            assert st.copy_out(int(k), 1)[0] == 0
