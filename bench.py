@@ -415,6 +415,11 @@ def main():
             # each piece running the sweep prefix that stays below qubit n - 5 as soon as
             # it has landed (bit-identical to copy_in + the sweep; tests/test_gpu_streamed.py)
             marshalled = lfqs.marshal_gates([g for _, g in sweep])
+            # Pieces only need their own launches while later pieces are in flight: piece
+            # c+1 lands (PCIe, ~55 GB/s) after 16*2^25 B / 55 GB/s = 9.8 ms; q gates on a
+            # 1/32 piece take q * 3.65 ms / 32, so q >= 86 keeps the GPU busy.  The other
+            # piece-local gates run on the whole state (fewer, larger launches).
+            st.set_option(lfqs.OPT_STREAM_MAX_PREFIX, 96)
             def e2e_step():
                 st.run_circuit_streamed(hv, marshalled, fuse=False, chunk_bits=5)
                 st.measure_probs(mq)

@@ -384,6 +384,11 @@ lfqs_status lfqs_kernel_launches(const lfqs_state* s, uint64_t* count);
                                         0 (default; measured 1-9 % faster): one greedy
                                         grouping in program order.  Changes the rounding
                                         order only (phase-table tolerance) */
+#define LFQS_OPT_STREAM_MAX_PREFIX 17 /* lfqs_run_circuit_streamed: at most this many prefix
+                                         gates run piece by piece (0, default: the whole
+                                         piece-local prefix); the rest run on the whole
+                                         state.  Enough to cover the upload keeps the GPU
+                                         busy with fewer, larger launches.  Same results */
 lfqs_status lfqs_set_option(lfqs_state* s, int option, int64_t value);
 const char* lfqs_last_error(void);
 int lfqs_abi_version(void);

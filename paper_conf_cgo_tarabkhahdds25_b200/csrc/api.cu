@@ -520,6 +520,10 @@ lfqs_status lfqs_set_option(lfqs_state* s, int option, int64_t value) {
       case LFQS_OPT_JIT_LANE_POOL: st->opt.jit_lane_pool = value != 0; break;
       case LFQS_OPT_JIT_PARTIAL_RT: st->opt.jit_partial_rt = value != 0; break;
       case LFQS_OPT_FUSE_PHASE_SPLIT: st->opt.fuse_phase_split = value != 0; break;
+      case LFQS_OPT_STREAM_MAX_PREFIX:
+        require(value >= 0, "LFQS_OPT_STREAM_MAX_PREFIX must be >= 0");
+        st->opt.stream_max_prefix = (int)value;
+        break;
       case LFQS_OPT_LANE_GROUP:
         require(value >= 0 && value <= 2, "LFQS_OPT_LANE_GROUP must be 0, 1 or 2");
         st->opt.lane_group = (int)value;

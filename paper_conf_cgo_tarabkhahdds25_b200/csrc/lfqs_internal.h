@@ -93,6 +93,7 @@ struct Options {
   int jit_threads = 256;     // threads per CTA of compiled passes (128, 256 or 512)
   int lane_group = 1;  // 1: dense 4x4 on qubits {1, 2} via k_lanegroup; 2: every dense 4x4/8x8
                        // with targets in [1, 5] (test / measurement); 0: never
+  int stream_max_prefix = 0;  // lfqs_run_circuit_streamed: max gates run per piece (0: all)
   bool fuse_phase_split = false;     // phase tables: tile-invariant / tile-dependent groups
   bool fuse_merge_commuting = true;  // merge same-qubit 1-target gates across commuting gates
   bool jit_lane_move = true;     // compiled passes may move lane bits >= 3 into registers

@@ -400,6 +400,7 @@ void State::run_streamed(const void* host, const std::vector<Decoded>& gates, ui
   const int nl = n - chunk_bits;
   size_t pre = 0;
   for (; pre < gates.size(); ++pre) {
+    if (opt.stream_max_prefix > 0 && pre >= (size_t)opt.stream_max_prefix) break;
     uint64_t m = gates[pre].cmask;
     for (int s = 0; s < gates[pre].m; ++s) m |= 1ull << gates[pre].targets[s];
     if (m >> nl) break;

@@ -30,8 +30,9 @@ def _plain(L, n, psi, gates, fuse):
         return st.copy_out()
 
 
-def _streamed(L, n, psi, gates, fuse, cb):
+def _streamed(L, n, psi, gates, fuse, cb, max_prefix=0):
     with L.State.create(n) as st:
+        st.set_option(L.OPT_STREAM_MAX_PREFIX, max_prefix)
         st.init_basis(0)
         st.run_circuit_streamed(psi, gates, fuse=fuse, chunk_bits=cb)
         return st.copy_out()
@@ -64,8 +65,9 @@ def test_streamed_edge_prefixes(L):
     starts_high = [W.Gate("H", (n - 1,))] + only_low
     for gates in (only_low, starts_high, []):
         for cb in (2, 3):
-            assert np.array_equal(_plain(L, n, psi, gates, False),
-                                  _streamed(L, n, psi, gates, False, cb))
+            for mp in (0, 1, 17):  # LFQS_OPT_STREAM_MAX_PREFIX
+                assert np.array_equal(_plain(L, n, psi, gates, False),
+                                      _streamed(L, n, psi, gates, False, cb, mp))
 
 
 def test_streamed_sweep_configs1_shape(L):
