@@ -389,6 +389,9 @@ lfqs_status lfqs_kernel_launches(const lfqs_state* s, uint64_t* count);
                                          piece-local prefix); the rest run on the whole
                                          state.  Enough to cover the upload keeps the GPU
                                          busy with fewer, larger launches.  Same results */
+#define LFQS_OPT_L2_FETCH_GRANULARITY 18 /* device-wide L2 fetch granularity hint in bytes
+                                            (cudaLimitMaxL2FetchGranularity: 0, 32, 64 or
+                                            128) for the state's device; measurement knob */
 lfqs_status lfqs_set_option(lfqs_state* s, int option, int64_t value);
 const char* lfqs_last_error(void);
 int lfqs_abi_version(void);

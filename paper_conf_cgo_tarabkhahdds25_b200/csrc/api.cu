@@ -520,6 +520,17 @@ lfqs_status lfqs_set_option(lfqs_state* s, int option, int64_t value) {
       case LFQS_OPT_JIT_LANE_POOL: st->opt.jit_lane_pool = value != 0; break;
       case LFQS_OPT_JIT_PARTIAL_RT: st->opt.jit_partial_rt = value != 0; break;
       case LFQS_OPT_FUSE_PHASE_SPLIT: st->opt.fuse_phase_split = value != 0; break;
+      case LFQS_OPT_L2_FETCH_GRANULARITY: {
+        require(value == 0 || value == 32 || value == 64 || value == 128,
+                "LFQS_OPT_L2_FETCH_GRANULARITY must be 0, 32, 64 or 128");
+        int prev = -1;
+        cudaGetDevice(&prev);
+        if (prev != st->device) LFQS_CUDA_CHECK(cudaSetDevice(st->device));
+        const cudaError_t err = cudaDeviceSetLimit(cudaLimitMaxL2FetchGranularity, (size_t)value);
+        if (prev >= 0 && prev != st->device) cudaSetDevice(prev);
+        LFQS_CUDA_CHECK(err);
+        break;
+      }
       case LFQS_OPT_STREAM_MAX_PREFIX:
         require(value >= 0, "LFQS_OPT_STREAM_MAX_PREFIX must be >= 0");
         st->opt.stream_max_prefix = (int)value;
