@@ -410,24 +410,19 @@ def main():
         hv = host.numpy()
         st.copy_out(rank << n_loc, 1 << n_loc, out=hv)
         mq = list(range(10))
-        if world == 1:
-            # lfqs_run_circuit_streamed: the 16 GiB upload in 32 pieces on a copy stream,
-            # each piece running the sweep prefix that stays below qubit n - 5 as soon as
-            # it has landed (bit-identical to copy_in + the sweep; tests/test_gpu_streamed.py)
-            marshalled = lfqs.marshal_gates([g for _, g in sweep])
-            # Pieces only need their own launches while later pieces are in flight: piece
-            # c+1 lands (PCIe, ~55 GB/s) after 16*2^25 B / 55 GB/s = 9.8 ms; q gates on a
-            # 1/32 piece take q * 3.65 ms / 32, so q >= 86 keeps the GPU busy.  The other
-            # piece-local gates run on the whole state (fewer, larger launches).
-            st.set_option(lfqs.OPT_STREAM_MAX_PREFIX, 96)
-            def e2e_step():
-                st.run_circuit_streamed(hv, marshalled, fuse=False, chunk_bits=5)
-                st.measure_probs(mq)
-        else:
-            def e2e_step():
-                st.copy_in(hv, offset=rank << n_loc)
-                one_step()
-                st.measure_probs(mq)
+        # lfqs_run_circuit_streamed (every rank: its own shard): the 16 GiB upload in 32
+        # pieces on a copy stream, each piece running the sweep prefix that stays below
+        # local qubit n_loc - 5 as soon as it has landed (bit-identical to copy_in + the
+        # sweep; tests/test_gpu_streamed.py).  Pieces only need their own launches while
+        # later pieces are in flight: piece c+1 lands (PCIe, ~55 GB/s) after
+        # 16*2^25 B / 55 GB/s = 9.8 ms; q gates on a 1/32 piece take q * 3.65 ms / 32, so
+        # q >= 86 keeps the GPU busy; the other gates run on the whole shard.
+        marshalled = lfqs.marshal_gates([g for _, g in sweep])
+        st.set_option(lfqs.OPT_STREAM_MAX_PREFIX, 96)
+
+        def e2e_step():
+            st.run_circuit_streamed(hv, marshalled, fuse=False, chunk_bits=5)
+            st.measure_probs(mq)
         e2e_step()
         barrier()
         a = torch.cuda.Event(enable_timing=True)
@@ -446,8 +441,7 @@ def main():
                "h2d_bytes_per_step": 16 * (1 << n_loc) * world,
                "d2h_bytes_per_step": 8 * (1 << len(mq)) * world,
                "api": "lfqs_run_circuit_streamed (upload overlapped with the sweep prefix) + "
-                      "lfqs_measure_probs" if world == 1 else
-                      "lfqs_copy_in + lfqs_apply_gate per gate + lfqs_measure_probs"}
+                      "lfqs_measure_probs"}
         del host
 
     cpu = None

@@ -217,19 +217,22 @@ lfqs_status lfqs_apply_gate(lfqs_state* s, int kind, const int* targets, int n_t
  * Unknown flag bits: LFQS_ERR_INVALID_ARG. */
 lfqs_status lfqs_run_circuit(lfqs_state* s, const lfqs_gate* gates, size_t n_gates, uint32_t flags);
 /* Loads the whole state from host memory and runs a circuit, overlapping the upload with
- * the computation (the state's input is 2^n interleaved complex128 values, host_interleaved
+ * the computation (the state's input is 2^n interleaved complex128 values -- for a sharded
+ * state (one shard per rank, NCCL or p2p) this rank's 2^n_local amplitudes, every rank
+ * calling with the same circuit -- host_interleaved
  * [2*k] = Re a_k, [2*k+1] = Im a_k, read during the call's asynchronous execution: keep it
  * alive and unchanged until the next synchronising call; page-locked memory for the copies
  * to overlap).  The state is uploaded in 2^chunk_bits pieces (split by its top chunk_bits
- * qubits, chunk_bits in [0, 8], < n) on an internal copy stream; each gate of the longest
- * prefix of the circuit whose targets and controls all lie below n - chunk_bits acts inside
+ * qubits, chunk_bits in [0, 8], < n_local) on an internal copy stream; each gate of the longest
+ * prefix of the circuit whose targets and controls all lie below n_local - chunk_bits acts inside
  * each piece (Eq. 1: I on the piece index (x) the gate), so every piece runs that prefix as
  * soon as it has landed while later pieces are still being copied; the remaining gates run
- * on the whole state.  Result: with LFQS_FUSE_NONE bit-identical to lfqs_copy_in of the
+ * on the whole state (sharded: through the planner's exchanges).  The qubit map is reset to
+ * canonical.  Result: with LFQS_FUSE_NONE bit-identical to lfqs_copy_in of the
  * whole state followed by lfqs_run_circuit; with fusion the prefix and the rest are fused
  * separately, so (as for fusion itself) permutation/diagonal results stay value-exact and
- * dense ones agree within rounding.  Asynchronous like lfqs_run_circuit.  Single-GPU
- * complex128 AOS states only (else LFQS_ERR_INVALID_ARG). */
+ * dense ones agree within rounding.  Asynchronous like lfqs_run_circuit.  complex128 AOS
+ * states, not virtual partitions (else LFQS_ERR_INVALID_ARG). */
 lfqs_status lfqs_run_circuit_streamed(lfqs_state* s, const double* host_interleaved,
                                       const lfqs_gate* gates, size_t n_gates, uint32_t flags,
                                       int chunk_bits);

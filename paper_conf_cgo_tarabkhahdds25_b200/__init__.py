@@ -633,8 +633,9 @@ class State:
         lfqs_run_circuit(self.h, gates, fuse_flags(fuse))
 
     def run_circuit_streamed(self, host: np.ndarray, gates, fuse=False, chunk_bits: int = 3):
-        """Whole-state upload from `host` overlapped with the circuit (lfqs_run_circuit_streamed)."""
-        assert host.size == 1 << self.n
+        """Upload of this process's part of the state from `host` (the whole state on one
+        GPU, this rank's shard when sharded) overlapped with the circuit
+        (lfqs_run_circuit_streamed)."""
         lfqs_run_circuit_streamed(self.h, host, gates, fuse_flags(fuse), chunk_bits)
 
     def compile(self, gates, fuse: bool = False) -> Circuit:

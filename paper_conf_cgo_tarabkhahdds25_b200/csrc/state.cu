@@ -394,10 +394,12 @@ void State::run(const std::vector<Decoded>& gates, uint32_t flags) {
 void State::run_streamed(const void* host, const std::vector<Decoded>& gates, uint32_t flags,
                          int chunk_bits) {
   DeviceGuard dg(device);
-  require(world == 1 && !soa, "streamed runs need a single-GPU AOS state");
-  require(chunk_bits >= 0 && chunk_bits <= 8 && chunk_bits < n, "chunk_bits must be in [0, 8]");
+  require(!virt && !soa, "streamed runs need an AOS state on one GPU or one shard per rank");
+  require(chunk_bits >= 0 && chunk_bits <= 8 && chunk_bits < n_local,
+          "chunk_bits must be in [0, 8] and below the local qubit count");
   const bool fuse = (flags & LFQS_FUSE_LOW) != 0;
-  const int nl = n - chunk_bits;
+  const int nl = n_local - chunk_bits;
+  plan.reset();  // the whole (local) state is overwritten: canonical qubit map
   size_t pre = 0;
   for (; pre < gates.size(); ++pre) {
     if (opt.stream_max_prefix > 0 && pre >= (size_t)opt.stream_max_prefix) break;
@@ -447,7 +449,14 @@ void State::run_streamed(const void* host, const std::vector<Decoded>& gates, ui
     run_local(pc, prefix, fuse);
   }
   const std::vector<Decoded> rest(gates.begin() + pre, gates.end());
-  if (!rest.empty()) run_local(ctx(0), rest, fuse);
+  if (rest.empty()) return;
+  if (world == 1) {
+    run_local(ctx(0), rest, fuse);
+  } else {
+    std::vector<PlanOp> ops;
+    plan.plan_circuit(rest, ops);  // exchanges for the global qubits, as in run()
+    execute(ops, fuse);
+  }
 }
 
 Graph* State::compile(const std::vector<Decoded>& gates, uint32_t flags) {

@@ -51,6 +51,20 @@ def worker(rank, world, port, n, seed, out_q):
                 st.apply(g)
             want = O.run_circuit(n, gates[:60], psi.copy())
             report["apply"] = float(np.max(np.abs(st.copy_out()[lo:hi] - want[lo:hi])))
+        # lfqs_run_circuit_streamed on the sharded state: this rank's shard uploaded in
+        # pieces, the piece-local prefix run per piece, the rest through the planner
+        low = W.random_gate_list(nl - 2, 60, seed=seed + 13, max_controls=1)
+        sg = low + gates
+        want = O.run_circuit(n, sg, psi.copy())
+        with L.State.p2p(n, rank, world) as st:
+            st.copy_in(psi)
+            st.run_circuit(sg)
+            plain = st.copy_out()[lo:hi]
+            st.init_basis(0)
+            st.run_circuit_streamed(np.ascontiguousarray(psi[lo:hi]), sg, chunk_bits=2)
+            streamed = st.copy_out()[lo:hi]
+            report["streamed"] = (bool(np.array_equal(plain, streamed)),
+                                  float(np.max(np.abs(streamed - want[lo:hi]))))
         dist.barrier()
         dist.destroy_process_group()
         out_q.put((rank, "ok", report))
