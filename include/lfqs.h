@@ -334,8 +334,10 @@ lfqs_status lfqs_kernel_launches(const lfqs_state* s, uint64_t* count);
 #define LFQS_OPT_FUSE_TILE_QUBITS 2
 #define LFQS_OPT_ITEMS_PER_THREAD 3
 #define LFQS_OPT_WIDE256 4 /* 1: two adjacent groups per thread, 32-byte accesses (default 1) */
-#define LFQS_OPT_FUSE_LOW_QUBITS 5 /* contiguous low qubits of a fused tile, [3, 12], default 7;
-                                      the other tile qubits are claimed by the fused gates */
+#define LFQS_OPT_FUSE_LOW_QUBITS 5 /* contiguous low qubits of a fused tile, [3, 12], or 0
+                                      (default): 7, or 6 when planning the circuit with 6
+                                      saves >= 20 % of the passes; the other tile qubits
+                                      are claimed by the fused gates */
 #define LFQS_OPT_FUSE_TMA_MAX_CHUNKS 6 /* tiles of at most this many chunks move by TMA bulk
                                           copies, larger ones by direct loads (default 256) */
 #define LFQS_OPT_FUSE_REORDER 7 /* 1: fused passes may take later gates that commute exactly

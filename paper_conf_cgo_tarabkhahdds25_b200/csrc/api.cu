@@ -504,7 +504,8 @@ lfqs_status lfqs_set_option(lfqs_state* s, int option, int64_t value) {
       case LFQS_OPT_ITEMS_PER_THREAD: st->opt.items_per_thread = (int)value; break;
       case LFQS_OPT_WIDE256: st->opt.wide256 = value != 0; break;
       case LFQS_OPT_FUSE_LOW_QUBITS:
-        require(value >= 3 && value <= 12, "fused low qubits must be in [3, 12]");
+        require(value == 0 || (value >= 3 && value <= 12),
+                "fused low qubits must be 0 (auto) or in [3, 12]");
         st->opt.fuse_low_qubits = (int)value;
         break;
       case LFQS_OPT_FUSE_REORDER: st->opt.fuse_reorder = value != 0; break;

@@ -83,7 +83,8 @@ struct Options {
   bool lowq_shuffle = false;
   bool wide256 = true;       // two adjacent groups per item, 32-byte accesses
   int fuse_tile_qubits = 12;
-  int fuse_low_qubits = 7;   // contiguous low qubits of a fused tile (chunk = 2^7 amps)
+  int fuse_low_qubits = 0;   // contiguous low qubits of a fused tile (chunk = 2^L amps);
+                             // 0: auto, 7 or 6 by planned pass count (fused_kernels.cu)
   bool fuse_reorder = true;  // commutation-aware scheduling of fused passes
   // Tiles with more chunks load/store directly (no TMA).  Measured on B200 at
   // n=30 (profiles/r01_fused_variants.md): TMA with parallel issue from warp 0
@@ -118,6 +119,8 @@ struct LaunchCtx {
   bool jit = false;
   // Plan and compile only (lfqs_jit_precompile): no kernel is launched.
   bool dry_run = false;
+  // Count the passes of the fused schedule only (no programs, no launches).
+  bool plan_only = false;
   // Structure-of-arrays shard (LFQS_STATE_SOA): real plane, then imaginary plane.
   bool soa = false;
 };
