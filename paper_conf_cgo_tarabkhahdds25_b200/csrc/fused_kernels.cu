@@ -33,6 +33,7 @@
 #include <cstring>
 #include <memory>
 #include <string>
+#include <type_traits>
 #include <vector>
 
 #include "cx.cuh"
@@ -109,6 +110,12 @@ struct FU_ {
   }
   // Own amplitude first, partner second, in both lanes: only the coefficients
   // depend on the lane bit (the compiled passes select them once per op).
+  // The lane's own coefficients moved to (c0, c1): lane(a, p, 0) of the result
+  // equals lane(a, p, bit) -- selected once per op, so the loop keeps 2 of 4 live.
+  static constexpr bool kSel = true;
+  __device__ __forceinline__ FU_ sel(int bit) const {
+    return bit ? FU_{c3, c2, c3, c2} : FU_{c0, c1, c0, c1};
+  }
   __device__ __forceinline__ cx<S> lane(cx<S> a, cx<S> p, int bit) const {
     cx<S> acc = mk<S>(0, 0);
     cfma(acc, bit ? c3 : c0, a);
@@ -124,6 +131,10 @@ struct FR_ {  // real 2x2 [[m00, m01], [m10, m11]]
     a0 = mk<S>(fma_(m01, x1.x, m00 * x0.x), fma_(m01, x1.y, m00 * x0.y));
     a1 = mk<S>(fma_(m11, x1.x, m10 * x0.x), fma_(m11, x1.y, m10 * x0.y));
   }
+  static constexpr bool kSel = true;
+  __device__ __forceinline__ FR_ sel(int bit) const {
+    return bit ? FR_{m11, m10, m11, m10} : FR_{m00, m01, m00, m01};
+  }
   __device__ __forceinline__ cx<S> lane(cx<S> a, cx<S> p, int bit) const {
     const S A = bit ? m11 : m00, B = bit ? m10 : m01;  // own, partner coefficient
     return mk<S>(fma_(B, p.x, A * a.x), fma_(B, p.y, A * a.y));
@@ -136,6 +147,10 @@ struct FI_ {  // [[d0, i e01], [i e10, d1]] with real d0, d1, e01, e10
     const cx<S> x0 = a0, x1 = a1;  // i e x = (-e x.y, e x.x)
     a0 = mk<S>(fma_(-e01, x1.y, d0 * x0.x), fma_(e01, x1.x, d0 * x0.y));
     a1 = mk<S>(fma_(d1, x1.x, -e10 * x0.y), fma_(d1, x1.y, e10 * x0.x));
+  }
+  static constexpr bool kSel = true;
+  __device__ __forceinline__ FI_ sel(int bit) const {
+    return bit ? FI_{d1, e10, e10, d1} : FI_{d0, e01, e01, d0};
   }
   __device__ __forceinline__ cx<S> lane(cx<S> a, cx<S> p, int bit) const {
     const S D = bit ? d1 : d0, E = bit ? e10 : e01;  // own diagonal, partner (imaginary) entry
@@ -251,21 +266,14 @@ __device__ __forceinline__ void reg_pairs(C (&v)[R], const F& f, uint32_t mlo, u
   }
 }
 
+template <class F, class = void>
+struct lane_sel : std::false_type {};
+template <class F>
+struct lane_sel<F, std::void_t<decltype(F::kSel)>> : std::true_type {};
+
 template <int R, class C, class F>
-__device__ __forceinline__ void reg_1q(C (&v)[R], const F& f, int t0, uint32_t mlo, uint32_t plo,
-                                       uint32_t tid) {
-  if (t0 >= 8) {
-    switch (t0 - 8) {
-      case 0: reg_pairs<0, R>(v, f, mlo, plo, tid); break;
-      case 1: reg_pairs<1, R>(v, f, mlo, plo, tid); break;
-      case 2: reg_pairs<2, R>(v, f, mlo, plo, tid); break;
-      default: reg_pairs<3, R>(v, f, mlo, plo, tid); break;
-    }
-    return;
-  }
-  // Lane bit (t0 < 5): partner lane tid ^ 2^t0.  Register-bit part of the
-  // predicate is uniform (skips whole registers); the thread part selects lanes.
-  const int bit = (tid >> t0) & 1;
+__device__ __forceinline__ void reg_lane(C (&v)[R], const F& f, int bit, int t0, uint32_t mlo,
+                                         uint32_t plo, uint32_t tid) {
   const bool bt = (tid & mlo & (kFThreads - 1)) == (plo & (kFThreads - 1));
   const uint32_t mr = mlo >> 8, pr = plo >> 8;
   if (mlo == 0) {  // uncontrolled: every lane, every register
@@ -286,6 +294,27 @@ __device__ __forceinline__ void reg_1q(C (&v)[R], const F& f, int t0, uint32_t m
     p.y = __shfl_xor_sync(0xffffffffu, v[r].y, 1 << t0);
     if (bt) v[r] = f.lane(v[r], p, bit);
   }
+}
+
+template <int R, class C, class F>
+__device__ __forceinline__ void reg_1q(C (&v)[R], const F& f, int t0, uint32_t mlo, uint32_t plo,
+                                       uint32_t tid) {
+  if (t0 >= 8) {
+    switch (t0 - 8) {
+      case 0: reg_pairs<0, R>(v, f, mlo, plo, tid); break;
+      case 1: reg_pairs<1, R>(v, f, mlo, plo, tid); break;
+      case 2: reg_pairs<2, R>(v, f, mlo, plo, tid); break;
+      default: reg_pairs<3, R>(v, f, mlo, plo, tid); break;
+    }
+    return;
+  }
+  // Lane bit (t0 < 5): partner lane tid ^ 2^t0.  Register-bit part of the
+  // predicate is uniform (skips whole registers); the thread part selects lanes.
+  const int bit = (tid >> t0) & 1;
+  if constexpr (lane_sel<F>::value)
+    reg_lane(v, f.sel(bit), 0, t0, mlo, plo, tid);
+  else
+    reg_lane(v, f, bit, t0, mlo, plo, tid);
 }
 
 // F_DIAG1 on the registers r with (r & MR) == PR (MR, PR: register bits 8..11 of
