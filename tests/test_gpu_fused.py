@@ -130,3 +130,37 @@ def test_merge_commuting_1q_runs(L, fuse, tile):
     c, _ = _run(L, n, psi, exact, fuse, tile, merge=1)
     if fuse in (True, "jit"):
         assert np.array_equal(c, O.run_circuit(n, exact, psi.copy()))
+
+
+@pytest.mark.parametrize("tma", [0, 256])
+@pytest.mark.parametrize("low", [6, 7])
+def test_fused_lane_bit_dense_1q(L, low, tma):
+    """Dense 1-target gates on lane bits (tile bits 0-4: shuffle path) for every
+    register specialisation -- H, Ry (real), Rx (real diagonal, imaginary
+    off-diagonal), U3 / UNITARY1 (general) -- uncontrolled and controlled on lane,
+    register and out-of-tile qubits; commuting merges off so each gate keeps its own
+    kind.  Interpreted fused passes vs the oracle, and vs the compiled passes
+    (identical arithmetic, so bit-identical)."""
+    n = 14
+    rng = np.random.default_rng(1000 + low + tma)
+    u = W.haar_unitary(1, 77)
+    gates = []
+    for t in range(5):
+        for ctl in [(), ((t + 1) % 5,), (9,), (13,), ((t + 2) % 5, 10)]:
+            th = rng.uniform(-np.pi, np.pi, 3)
+            gates += [W.Gate("H", (t,), ctl), W.Gate("RY", (t,), ctl, (th[0],)),
+                      W.Gate("RX", (t,), ctl, (th[1],)), W.Gate("U3", (t,), ctl, tuple(th)),
+                      W.Gate("UNITARY1", (t,), ctl, matrix=u)]
+    psi = W.random_state(n, 31 + low)
+    ref = O.run_circuit(n, gates, psi.copy())
+    out = {}
+    for fuse in (True, "jit"):
+        with L.State.create(n) as st:
+            st.set_option(L.OPT_FUSE_LOW_QUBITS, low)
+            st.set_option(L.OPT_FUSE_TMA_MAX_CHUNKS, tma)
+            st.set_option(L.OPT_FUSE_MERGE_COMMUTING, 0)
+            st.copy_in(psi)
+            st.run_circuit(gates, fuse=fuse)
+            out[fuse] = st.copy_out()
+    assert np.max(np.abs(out[True] - ref)) <= 1e-12
+    assert np.array_equal(out[True], out["jit"])
