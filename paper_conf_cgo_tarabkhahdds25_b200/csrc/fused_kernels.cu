@@ -379,7 +379,7 @@ __device__ __forceinline__ uint64_t tile_addr(const FTile& tg, uint64_t base, ui
 }
 
 template <int K, bool DIRECT, class S>
-__global__ void __launch_bounds__(kFThreads, 2) k_fused(cx<S>* __restrict__ a,
+__global__ void __launch_bounds__(kFThreads, sizeof(S) == 4 ? 4 : 2) k_fused(cx<S>* __restrict__ a,
                                                         const __grid_constant__ FProg prog) {
   using C = cx<S>;
   constexpr uint32_t T = 1u << K;

@@ -95,6 +95,16 @@ struct Gen {
     for (int j = 0; j < nreg; ++j) rpos[j] = 5 + NWB + j;
   }
 
+  // .minnctapersm: complex64 tiles are half the bytes, so more CTAs fit per SM (up
+  // to 1024 threads and the shared memory the tile allows); complex128 keeps 2 (3 at
+  // 128 threads), which its register-resident amplitudes need.
+  int min_ctas() const {
+    const int base = NT == 128 ? 3 : 2;
+    if (!c64) return base;
+    const int by_smem = (200 * 1024) / ((ES << K) + 4096);
+    return std::max(base, std::min(by_smem, 1024 / NT));
+  }
+
   int reg_of(int b) const {
     for (int j = 0; j < nreg; ++j)
       if (rpos[j] == b) return j;
@@ -1687,7 +1697,7 @@ struct Gen {
     out += ".visible .entry lfqs_jit(.param .u64 pa, .param .align 16 .b8 pc[" +
            std::to_string(nc * 16) + "])\n";
     out += ".maxntid " + std::to_string(NT) + ", 1, 1\n.minnctapersm " +
-           std::to_string(NT == 128 ? 3 : 2) + "\n{\n";
+           std::to_string(min_ctas()) + "\n{\n";
     out += "  .reg .pred %p<" + std::to_string(np + 1) + ">;\n";
     out += "  .reg .b32 %r<" + std::to_string(nr + 1) + ">;\n";
     out += "  .reg .b64 %rd<" + std::to_string(nrd + 1) + ">;\n";
