@@ -378,6 +378,8 @@ __device__ __forceinline__ uint64_t tile_addr(const FTile& tg, uint64_t base, ui
   return off;
 }
 
+// complex64 tiles are half the bytes: 4 CTAs per SM (64 registers) instead of 2
+// (profiles/r01_c64_occupancy.md).
 template <int K, bool DIRECT, class S>
 __global__ void __launch_bounds__(kFThreads, sizeof(S) == 4 ? 4 : 2) k_fused(cx<S>* __restrict__ a,
                                                         const __grid_constant__ FProg prog) {
