@@ -78,6 +78,8 @@ def lib():
         L.oracle_fill_random.argtypes = [C.c_uint64, C.c_uint64, C.c_uint64, dp]
         L.oracle_fill_random.restype = None
         L.oracle_omp_max_threads.restype = C.c_int
+        L.oracle_omp_set_threads.argtypes = [C.c_int]
+        L.oracle_omp_set_threads.restype = None
         _lib = L
     return _lib
 
@@ -249,3 +251,7 @@ def fill_random(seed: int, start: int, count: int) -> np.ndarray:
 
 def omp_max_threads() -> int:
     return int(lib().oracle_omp_max_threads())
+
+
+def omp_set_threads(threads: int) -> None:
+    lib().oracle_omp_set_threads(int(threads))

@@ -88,6 +88,7 @@ int oracle_apply_gate_sparse(int n, const oracle_gate* g, size_t cnt,
  * to time the oracle on the host cores. */
 int oracle_apply_gate_omp(int n, const oracle_gate* g, double* state);
 int oracle_omp_max_threads(void);
+void oracle_omp_set_threads(int threads);  /* omp_set_num_threads (tests) */
 
 /* ---- Measurement -------------------------------------------------- */
 /* probs[v] = sum_{k: bits_Q(k) = v} |a_k|^2, pairwise (recursive halving) over k

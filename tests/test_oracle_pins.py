@@ -284,6 +284,84 @@ def test_circuit_is_ordered_product_eq3():
     np.testing.assert_allclose(O.run_circuit(n, gates, psi.copy()), P @ psi, atol=2e-15)
 
 
+def test_dense_matmul_is_eq3_product():
+    """oracle_dense_matmul (the exported C = A.B, Eq. 3): (a) the oracle's product of
+    two gate matrices, applied with the oracle's mvdot, equals applying the two gates one
+    after the other by tier B (G_2 G_1 -- a transposed operand or swapped order fails);
+    (b) it equals numpy's matmul (an independent library routine) on random complex
+    matrices, non-commuting ones included; (c) I.A = A.I = A value-exactly."""
+    rng = np.random.default_rng(31)
+    n = 4
+    psi = W.random_state(n, 8)
+    gates = W.random_gate_list(n, 10, seed=12, max_controls=2)
+    for g1, g2 in zip(gates[:-1], gates[1:]):
+        G = O.dense_matmul(O.dense_kron(n, g2), O.dense_kron(n, g1))
+        seq = O.apply_gate(n, g2, O.apply_gate(n, g1, psi.copy()))
+        np.testing.assert_allclose(O.dense_matvec(G, psi), seq, rtol=0, atol=2e-15,
+                                   err_msg=f"{g1.label()} then {g2.label()}")
+    for dim in (1, 2, 3, 8, 16):
+        A = rng.standard_normal((dim, dim)) + 1j * rng.standard_normal((dim, dim))
+        B = rng.standard_normal((dim, dim)) + 1j * rng.standard_normal((dim, dim))
+        np.testing.assert_allclose(O.dense_matmul(A, B), A @ B, rtol=0, atol=1e-13 * dim)
+        I = np.eye(dim, dtype=complex)
+        assert np.array_equal(O.dense_matmul(I, A), A) and np.array_equal(O.dense_matmul(A, I), A)
+    X, Z = O.gate_matrix(W.Gate("X", (0,))), O.gate_matrix(W.Gate("Z", (0,)))
+    assert np.array_equal(O.dense_matmul(Z, X), np.array([[0, 1], [-1, 0]], dtype=complex))
+    assert np.array_equal(O.dense_matmul(X, Z), np.array([[0, -1], [1, 0]], dtype=complex))
+
+
+def _omp_cases(n, rng):
+    """Every kind, every target placement class (low/high/straddling, both orders) and
+    0-3 controls (low, high, mixed) at size n."""
+    for kind in O.KINDS:
+        m = W.ARITY[kind]
+        if m > n:
+            continue
+        for nc in range(0, min(3, n - m) + 1):
+            for _ in range(3):
+                qs = [int(x) for x in rng.permutation(n)]
+                mat = (W.haar_unitary(m, int(rng.integers(1 << 30)))
+                       if kind.startswith("UNITARY") else None)
+                yield W.Gate(kind, tuple(qs[:m]), tuple(qs[m:m + nc]), _rand_params(kind, rng), mat)
+        # extremes: targets on the lowest / highest bits, controls at the other end
+        lo = tuple(range(m)); hi = tuple(range(n - 1, n - 1 - m, -1))
+        for tg, cq in ((lo, tuple(range(n - 1, n - 1 - min(3, n - m), -1))),
+                       (hi, tuple(range(min(3, n - m))))):
+            mat = W.haar_unitary(m, 5) if kind.startswith("UNITARY") else None
+            yield W.Gate(kind, tg, cq, _rand_params(kind, rng), mat)
+
+
+@pytest.mark.parametrize("threads", [1, 3, "all"])
+def test_omp_tier_b_equals_serial_tier_b(threads):
+    """oracle_apply_gate_omp (the OpenMP parallel-for of the P:465-467 pattern, which times
+    every cpu_baseline and --impl reference number) equals oracle_apply_gate bit for bit:
+    every kind, target/control placement and 0-3 controls, n = 1..12, on 1 thread, an odd
+    thread count (uneven static chunks) and every host core.  A race, a dropped or doubled
+    group, or a chunk-boundary bug changes at least one amplitude."""
+    rng = np.random.default_rng(77)
+    t = O.omp_max_threads() if threads == "all" else threads
+    before = O.omp_max_threads()
+    O.omp_set_threads(t)
+    try:
+        assert O.omp_max_threads() == t
+        for n in (1, 2, 3, 5, 8, 12):
+            psi = W.random_state(n, 1000 + n)
+            for g in _omp_cases(n, rng):
+                a = O.apply_gate(n, g, psi.copy())
+                b = O.apply_gate(n, g, psi.copy(), omp=True)
+                assert np.array_equal(a.view(np.float64), b.view(np.float64)), (n, g.label())
+        # the bench's own sweep at a size where every thread owns many groups
+        n = 16
+        psi = W.random_state(n, 99)
+        a, b = psi.copy(), psi.copy()
+        for _, g in W.sweep_gates(n)[::5]:
+            O.apply_gate(n, g, a)
+            O.apply_gate(n, g, b, omp=True)
+        assert np.array_equal(a.view(np.float64), b.view(np.float64))
+    finally:
+        O.omp_set_threads(before)
+
+
 # --------------------------------------------------------------------------
 # Closed forms (circuits of Table 1, readings R10-R12)
 # --------------------------------------------------------------------------
