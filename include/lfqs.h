@@ -118,8 +118,13 @@ typedef struct lfqs_state lfqs_state;  /* opaque */
  * or NULL for a library-created non-blocking stream.
  * LFQS_ERR_OUT_OF_MEMORY if it does not fit. */
 lfqs_status lfqs_state_create(int n_qubits, int device, void* cuda_stream, lfqs_state** out);
-/* Borrow caller device memory (e.g. a torch complex128 tensor of 2^n elements,
- * 16-byte aligned).  The contents are left as they are. */
+/* Borrow caller device memory (e.g. a torch complex128 tensor of 2^n elements).
+ * dev_ptr must be 32-byte aligned: the kernels read and write two adjacent
+ * amplitudes per 32-B vector access (LDG/STG.256) and move tiles with TMA bulk
+ * copies; a merely element-aligned view (torch t[1:]) returns
+ * LFQS_ERR_INVALID_ARG.  cudaMalloc / torch allocations are 256-B aligned.
+ * The contents are left as they are; the caller keeps ownership and must keep
+ * the buffer alive until lfqs_state_destroy. */
 lfqs_status lfqs_state_wrap(int n_qubits, int device, void* dev_ptr, void* cuda_stream,
                             lfqs_state** out);
 /* Precision / partition variants (NEXT-4).  flags: LFQS_STATE_C64 stores
@@ -142,7 +147,9 @@ lfqs_status lfqs_state_wrap(int n_qubits, int device, void* dev_ptr, void* cuda_
 lfqs_status lfqs_state_create_ex(int n_qubits, int world, int device, void* cuda_stream,
                                  uint32_t flags, lfqs_state** out);
 /* Borrow caller memory with the precision given by flags (LFQS_STATE_C64: a
- * torch complex64 tensor of 2^n elements). */
+ * torch complex64 tensor of 2^n elements).  Alignment: 32 B for complex128,
+ * 16 B for complex64 (two amplitudes per vector access), else
+ * LFQS_ERR_INVALID_ARG. */
 lfqs_status lfqs_state_wrap_ex(int n_qubits, int device, void* dev_ptr, void* cuda_stream,
                                uint32_t flags, lfqs_state** out);
 lfqs_status lfqs_state_destroy(lfqs_state* s);

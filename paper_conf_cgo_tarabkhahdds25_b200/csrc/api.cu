@@ -43,6 +43,17 @@ lfqs_status guarded(F&& f) {
   }
 }
 
+// Borrowed buffers must be aligned for the widest access any kernel issues: two adjacent
+// amplitudes per vector access (ld/st.global.v4: 32 B complex128, 16 B complex64) and TMA
+// bulk copies (cp.async.bulk, 16 B).  A merely element-aligned torch view (e.g. t[1:]) is
+// rejected here instead of faulting with a misaligned address inside a kernel.
+void require_wrap_alignment(const void* p, bool c64) {
+  const uintptr_t need = c64 ? 16 : 32;
+  require((reinterpret_cast<uintptr_t>(p) & (need - 1)) == 0,
+          std::string("dev_ptr must be ") + (c64 ? "16" : "32") +
+              "-byte aligned (two amplitudes per vector access)");
+}
+
 uint64_t mask_of(const int* qs, int nq, int n) {
   uint64_t m = 0;
   require(nq >= 0 && (nq == 0 || qs != nullptr), "bad control list");
@@ -71,7 +82,7 @@ lfqs_status lfqs_state_wrap(int n_qubits, int device, void* dev_ptr, void* strea
                             lfqs_state** out) {
   return guarded([&] {
     require(out != nullptr && dev_ptr != nullptr, "NULL argument");
-    require((reinterpret_cast<uintptr_t>(dev_ptr) & 15) == 0, "dev_ptr must be 16-byte aligned");
+    require_wrap_alignment(dev_ptr, false);
     *out = State::create_local(n_qubits, device, static_cast<cudaStream_t>(stream), dev_ptr);
   });
 }
@@ -98,8 +109,7 @@ lfqs_status lfqs_state_wrap_ex(int n_qubits, int device, void* dev_ptr, void* st
     require(out != nullptr && dev_ptr != nullptr, "NULL argument");
     require((flags & ~(LFQS_STATE_C64 | LFQS_STATE_SOA)) == 0, "unknown state flags");
     const bool c64 = (flags & LFQS_STATE_C64) != 0, soa = (flags & LFQS_STATE_SOA) != 0;
-    require((reinterpret_cast<uintptr_t>(dev_ptr) & (c64 ? 7 : 15)) == 0,
-            "dev_ptr is not aligned to one amplitude");
+    require_wrap_alignment(dev_ptr, c64);
     *out = State::create_local(n_qubits, device, static_cast<cudaStream_t>(stream), dev_ptr, c64,
                                soa);
   });

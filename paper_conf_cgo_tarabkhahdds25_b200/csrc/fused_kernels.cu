@@ -643,12 +643,17 @@ __global__ void __launch_bounds__(kFThreads, sizeof(S) == 4 ? 4 : 2) k_fused(cx<
 
 inline double2 D2(cplx z) { return make_double2(z.re, z.im); }
 
+// Coefficient budget of one gate, an upper bound on what encode() appends for it after
+// build_program's merges: any 1-target gate may end up merged into (or absorb) a dense
+// 1-target neighbour, which is encoded as a full U2 (4 coefficients), so every 1-target
+// gate is budgeted at 4 whatever its class.
 int coef_count(const Decoded& g) {
   const int d = 1 << g.m;
+  if (g.m == 1) return 4;
   switch (g.cls) {
     case GClass::DIAG: return d;  // upper bound (DIAG1 uses 1)
     case GClass::PERM_X: case GClass::PERM_Y: case GClass::PERM_SWAP: return 0;
-    default: return g.is_h ? 1 : d * d;
+    default: return d * d;
   }
 }
 
@@ -660,6 +665,8 @@ struct TileMap {
 // Appends gate g to the program (program space was checked by the caller).
 void encode(const Decoded& g, const TileMap& tm, FProg& P) {
   if (g.cls == GClass::NOOP) return;
+  require(P.nops < kMaxOps && P.ncoef + coef_count(g) <= kMaxCoef,
+          "internal: fused program over its op / coefficient budget");
   FHdr& h = P.h[P.nops];
   std::memset(&h, 0, sizeof h);
   uint64_t mlo = 0, plo = 0, mhi = 0, phi = 0;
@@ -1058,7 +1065,7 @@ void run_fused_schedule(const LaunchCtx& ctx_in, const std::vector<Decoded>& gat
   for (size_t i = 0; i < gates.size(); ++i)
     if (gates[i].cls != GClass::NOOP) rest.push_back((int)i);
   if (!tile_cfg(ctx, tile_qubits, &cfg)) {
-    if (ctx.plan_only) {
+    if (ctx.plan_only || ctx.dry_run) {  // host-only callers (lfqs_jit_precompile): no launch
       *ctx.launch_counter += rest.size();
       return;
     }
@@ -1073,6 +1080,12 @@ void run_fused_schedule(const LaunchCtx& ctx_in, const std::vector<Decoded>& gat
   };
   std::vector<Pass> passes;
   const bool collect = ctx.jit && (1 << (cfg.K - cfg.L)) <= ctx.opt->fuse_tma_max_chunks;
+  if (ctx.dry_run && !collect && !ctx.plan_only) {  // nothing to compile: count passes only
+    LaunchCtx pc = ctx;
+    pc.plan_only = true;
+    run_fused_schedule(pc, gates, tile_qubits);
+    return;
+  }
   constexpr size_t kWindow = 4096;  // gates scanned per pass
   const int max_ops = ctx.phase_tables ? kMaxOps - 16 : kMaxOps;  // room for F_DTAB headers
   std::vector<char> taken(gates.size(), 0);

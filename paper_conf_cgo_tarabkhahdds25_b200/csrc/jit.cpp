@@ -24,6 +24,7 @@
 #include <nvPTXCompiler.h>
 
 #include <atomic>
+#include <condition_variable>
 #include <cstdarg>
 #include <cstdio>
 #include <cstdlib>
@@ -1750,16 +1751,22 @@ struct Gen {
 // ---------------------------------------------------------------------------
 // Compilation cache
 // ---------------------------------------------------------------------------
+// An entry is published in g_cache as soon as one thread starts compiling it; `done`
+// (guarded by g_mu, signalled on g_cv) says its cubin / error are final.  Any other
+// thread that finds the entry waits for `done` before reading the cubin, so a
+// concurrent jit_launch never loads a half-written image.  The dynamic shared-memory
+// attribute is a per-device property of the kernel, so it is tracked per device.
 struct Entry {
   std::vector<char> cubin;
   std::string error;
-  bool compiled = false;
+  bool done = false;
   cudaLibrary_t lib = nullptr;
   cudaKernel_t kern = nullptr;
-  int smem_set = 0;
+  std::map<int, int> smem_set;  // device -> dynamic smem bytes already allowed
 };
 
 std::mutex g_mu;
+std::condition_variable g_cv;
 std::unordered_map<std::string, std::shared_ptr<Entry>> g_cache;
 
 void compile_entry(const std::string& ptx, Entry& en) {
@@ -1824,16 +1831,31 @@ void jit_compile(const std::vector<std::pair<std::string, const FProg*>>& items,
     std::shared_ptr<Entry> en;
   };
   std::vector<Todo> todo;
+  std::vector<std::shared_ptr<Entry>> others;  // being compiled by another thread
   {
     std::lock_guard<std::mutex> lk(g_mu);
     for (const auto& it : items) {
-      if (g_cache.count(it.first)) continue;
+      auto f = g_cache.find(it.first);
+      if (f != g_cache.end()) {
+        if (!f->second->done) others.push_back(f->second);
+        continue;
+      }
       auto en = std::make_shared<Entry>();
       g_cache.emplace(it.first, en);
       todo.push_back({&it.first, it.second, en});
     }
   }
-  if (todo.empty()) return;
+  auto wait_others = [&] {
+    std::unique_lock<std::mutex> lk(g_mu);
+    for (const auto& en : others) {
+      g_cv.wait(lk, [&] { return en->done; });
+      if (!en->error.empty()) throw Error(LFQS_ERR_CUDA, "JIT pass compile failed: " + en->error);
+    }
+  };
+  if (todo.empty()) {
+    wait_others();
+    return;
+  }
   unsigned nth = std::thread::hardware_concurrency();
   if (nth == 0) nth = 4;
   if (nth > todo.size()) nth = (unsigned)todo.size();
@@ -1851,20 +1873,26 @@ void jit_compile(const std::vector<std::pair<std::string, const FProg*>>& items,
         }
       }
       compile_entry(ptx, *todo[i].en);
-      todo[i].en->compiled = true;
     }
   };
   std::vector<std::thread> th;
   for (unsigned t = 1; t < nth; ++t) th.emplace_back(work);
   work();
   for (auto& t : th) t.join();
-  for (auto& t : todo)
-    if (!t.en->error.empty()) {
-      const std::string err = t.en->error;
-      std::lock_guard<std::mutex> lk(g_mu);
-      g_cache.erase(*t.key);
-      throw Error(LFQS_ERR_CUDA, "JIT pass compile failed: " + err);
+  std::string err;
+  {
+    std::lock_guard<std::mutex> lk(g_mu);
+    for (auto& t : todo) {
+      t.en->done = true;  // waiters read cubin / error only after this
+      if (!t.en->error.empty()) {
+        if (err.empty()) err = t.en->error;
+        g_cache.erase(*t.key);  // a later call retries
+      }
     }
+  }
+  g_cv.notify_all();
+  if (!err.empty()) throw Error(LFQS_ERR_CUDA, "JIT pass compile failed: " + err);
+  wait_others();
 }
 
 int jit_config(const LaunchCtx& ctx, int K) {
@@ -1888,18 +1916,23 @@ void jit_launch(const LaunchCtx& ctx, const FProg& P, int K, const std::string& 
   {
     std::lock_guard<std::mutex> lk(g_mu);
     auto it = g_cache.find(key);
-    if (it != g_cache.end()) en = it->second;
+    if (it != g_cache.end() && it->second->done) en = it->second;
   }
   if (!en) {
-    jit_compile({{key, &P}}, K, ctx.c64, jc);
+    jit_compile({{key, &P}}, K, ctx.c64, jc);  // compiles, or waits for another thread's compile
     std::lock_guard<std::mutex> lk(g_mu);
-    en = g_cache.at(key);
+    auto it = g_cache.find(key);
+    require(it != g_cache.end() && it->second->done, "internal: JIT entry missing after compile");
+    en = it->second;
   }
   const int es = ctx.c64 ? 8 : 16;
   const int smem = es << K;
+  int dev = 0;
+  LFQS_CUDA_CHECK(cudaGetDevice(&dev));
   {
     std::lock_guard<std::mutex> lk(g_mu);
-    if (en->lib == nullptr || en->smem_set < smem) {
+    auto ss = en->smem_set.find(dev);
+    if (en->lib == nullptr || ss == en->smem_set.end() || ss->second < smem) {
       // Module loading is not a stream operation: allowed while this thread
       // captures a CUDA graph (lfqs_circuit_compile) under relaxed mode.
       cudaStreamCaptureMode mode = cudaStreamCaptureModeRelaxed;
@@ -1915,7 +1948,7 @@ void jit_launch(const LaunchCtx& ctx, const FProg& P, int K, const std::string& 
                                    cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
       cudaThreadExchangeStreamCaptureMode(&mode);
       LFQS_CUDA_CHECK(err);
-      en->smem_set = smem;
+      en->smem_set[dev] = smem;
     }
   }
   void* a = ctx.amps;

@@ -98,14 +98,23 @@ void Planner::plan_canonicalize(std::vector<PlanOp>& out) {
   // when that qubit sits at a local position, two (through a local staging position
   // L) when it sits at another global one.  L is chosen as the home of the qubit that
   // leaves G, so that qubit lands where phase 2 wants it.
+  // Every exchange stays inside the top kSwapWindow local positions, as in plan_gate: a
+  // low position l would split the exchanged half-shard into 2^(n_local-1-l) pieces of
+  // 2^l amplitudes (the NCCL transport sends one message per piece).  A qubit that sits
+  // lower is first moved to the top local position by one local SWAP pass.
+  const int wlo = std::max(0, n_local - kSwapWindow);
   for (int G = n - 1; G >= n_local; --G) {
-    const int P = l2p[G];
+    int P = l2p[G];
     if (P == G) continue;
     if (P < n_local) {
+      if (P < wlo) {
+        swap_local(P, n_local - 1, out);
+        P = n_local - 1;
+      }
       exchange(P, G, out);
     } else {
       const int x = p2l[G];
-      const int L = x < n_local ? x : n_local - 1;
+      const int L = (x < n_local && x >= wlo) ? x : n_local - 1;
       exchange(L, P, out);
       exchange(L, G, out);
     }

@@ -260,15 +260,28 @@ void State::copy(uint64_t offset, uint64_t count, double* host, bool to_device) 
     copy_raw(offset, count, host, to_device);
     return;
   }
-  // complex64 state, complex128 host buffer: convert on the host.
-  std::vector<float> tmp(2 * count);
+  // complex64 state, complex128 host buffer: convert on the host -- only the sub-range
+  // this rank owns (a sharded rank's copy leaves the rest of the caller's buffer as it was,
+  // in full complex128 precision).  Bounds are checked before anything is allocated.
+  const uint64_t total = 1ull << n;
+  require(offset <= total && count <= total - offset, "amplitude range out of bounds");
+  const uint64_t lo = virt ? 0 : (uint64_t)rank << n_local;
+  const uint64_t hi = virt ? total : lo + (1ull << n_local);
+  const uint64_t a = std::max(offset, lo), b = std::min(offset + count, hi);
+  if (!plan.identity()) {
+    DeviceGuard dg(device);
+    canonicalize();
+  }
+  if (a >= b) return;
+  double* h = host + 2 * (a - offset);
+  const uint64_t cnt = b - a;
+  std::vector<float> tmp(2 * cnt);
   if (to_device) {
-    for (uint64_t i = 0; i < 2 * count; ++i) tmp[i] = (float)host[i];
-    copy_raw(offset, count, tmp.data(), true);
+    for (uint64_t i = 0; i < 2 * cnt; ++i) tmp[i] = (float)h[i];
+    copy_raw(a, cnt, tmp.data(), true);
   } else {
-    for (uint64_t i = 0; i < 2 * count; ++i) tmp[i] = (float)host[i];  // keep untouched ranges
-    copy_raw(offset, count, tmp.data(), false);
-    for (uint64_t i = 0; i < 2 * count; ++i) host[i] = (double)tmp[i];
+    copy_raw(a, cnt, tmp.data(), false);
+    for (uint64_t i = 0; i < 2 * cnt; ++i) h[i] = (double)tmp[i];
   }
 }
 

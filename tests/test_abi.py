@@ -83,3 +83,29 @@ def test_jit_precompile_host_only(lib):
     assert L.lfqs_jit_precompile(n, gates, "jit", c64=True) == k
     with pytest.raises(L.LfqsError):
         L.lfqs_jit_precompile(n, gates, True)  # FUSE_JIT missing
+
+
+def test_jit_precompile_small_n_launches_nothing(lib):
+    """Below the smallest fused tile (n < 8) the schedule falls back to per-gate kernels;
+    lfqs_jit_precompile is host-only, so it must count those passes without launching
+    anything (no device here: a launch would fail the call)."""
+    import workloads as W
+    for n in (1, 3, 7):
+        gates = W.random_gate_list(n, 20, seed=n)
+        k = L.lfqs_jit_precompile(n, gates, "jit")   # one pass per non-identity gate
+        assert len(gates) - 3 <= k <= len(gates), (n, k)
+
+
+def test_fused_coefficient_budget_counts_merged_gates(lib):
+    """A pass of 1-target gates that build_program merges into dense U2 matrices (4
+    coefficients each, e.g. X followed by H on the same qubit) must stay inside the
+    program's coefficient budget: the planner budgets every 1-target gate at 4
+    (ADVICE r1).  Host-only: plan + compile, no launch."""
+    import workloads as W
+    n = 14
+    gates = []
+    for rep in range(24):   # 24 x 64 = 1536 coefficients
+        gates.append(W.Gate("UNITARY3", (3, 4, 5), (), (), W.haar_unitary(3, rep)))
+    for rep in range(14):   # X(0) H(0) merge into one U2: 4 coefficients (budgeted 0 + 1 before)
+        gates += [W.CNOT(1, 0), W.Gate("X", (0,)), W.Gate("H", (0,))]
+    assert L.lfqs_jit_precompile(n, gates, "jit") >= 2

@@ -243,6 +243,37 @@ def test_wrap_torch_tensor_and_stream(L):
     _cmp(t.cpu().numpy(), O.apply_gate(n, g, psi.copy()), False, "wrap")
 
 
+@pytest.mark.parametrize("dtype,bad,good", [("complex128", 1, 2), ("complex64", 1, 2),
+                                             ("complex64", 3, 4)])
+def test_wrap_rejects_underaligned_views(L, dtype, bad, good):
+    """The wrap contract is as wide as the narrowest kernel access (two amplitudes per
+    vector access: 32 B complex128, 16 B complex64): a torch view offset by an odd
+    number of amplitudes is LFQS_ERR_INVALID_ARG, not a misaligned-address fault; a view
+    at the next aligned offset works and matches the oracle."""
+    import torch
+    n = 9
+    dt = getattr(torch, dtype)
+    base = torch.zeros((1 << n) + 8, dtype=dt, device="cuda")
+    with pytest.raises(L.LfqsError) as e:
+        L.State.wrap(base[bad:bad + (1 << n)])
+    assert e.value.status == -1 and "aligned" in str(e.value)
+    psi = W.random_state(n, 12)
+    if dtype == "complex64":
+        psi = psi.astype(np.complex64)
+    view = base[good:good + (1 << n)]
+    view.copy_(torch.from_numpy(psi))
+    g = W.Gate("U3", (0,), (4,), (0.3, -0.2, 0.9))
+    with L.State.wrap(view) as st:
+        st.apply(g)
+        st.apply(W.Gate("T", (0,)))
+        st.synchronize()
+    ref = O.apply_gate(n, W.Gate("T", (0,)), O.apply_gate(n, g, psi.astype(np.complex128)))
+    tol = 1e-12 if dtype == "complex128" else 2e-6
+    assert np.max(np.abs(view.cpu().numpy().astype(np.complex128) - ref)) <= tol
+    assert torch.count_nonzero(base[:good]) == 0     # nothing written outside the view
+    assert torch.count_nonzero(base[good + (1 << n):]) == 0
+
+
 def test_invalid_arguments_raise(L):
     with L.State.create(5) as st:
         for bad in [dict(kind="H", targets=(5,)), dict(kind="X", targets=(1,), controls=(1,)),

@@ -117,3 +117,25 @@ def test_grover_sharded(world):
     # H layers need the global qubits local; X layers are relabels
     p = world.bit_length() - 1
     assert n_ex <= 12 * p + 2 * p + 2, n_ex
+
+
+@pytest.mark.parametrize("world", [2, 4])
+def test_exchanges_stay_in_the_top_window(world):
+    """Every EXCHANGE -- from gates and from canonicalisation after SWAP relabels that
+    leave a global qubit's logical home at a low local position -- uses a local position
+    in the top 8 (planner.h kSwapWindow), so a transport that moves the strided half-shard
+    as 2^(n_local-1-l) contiguous pieces sends at most 128 of them (a low l would mean
+    ~2^n_local tiny messages).  The plan still equals the oracle."""
+    n = 16
+    p = world.bit_length() - 1
+    nl = n - p
+    psi = W.random_state(n, 5)
+    # SWAP(top, 0) relabels: logical qubit 0 goes global, logical top lands at position 0
+    gates = [W.Gate("SWAP", (n - 1, 0)), W.Gate("H", (3,)), W.Gate("SWAP", (n - 2, 1)),
+             W.CNOT(2, n - 1)] + W.qft(n)
+    for r in range(world):
+        for op in L.lfqs_plan_circuit(n, world, r, gates, canonicalize=True):
+            if op[0] == "exchange":
+                assert op[1] >= nl - 8, op
+    got, _ = simulate(n, world, gates, psi)
+    assert np.max(np.abs(got - O.run_circuit(n, gates, psi.copy()))) <= 1e-12
