@@ -229,6 +229,78 @@ def run_reference(args):
 
 
 # ----------------------------------------------------------------------------
+# configs[2]: 33-qubit QFT and GHZ on one B200 (macro leg of the N = 1 line)
+# ----------------------------------------------------------------------------
+
+def _closed_form_err(name, n, st, meta):
+    """Max abs error against the closed form (readings R10/R11) on 64 sampled
+    indices plus both ends; GHZ also reports bit-exactness (amplitude M_SQRT1_2 exactly)."""
+    rng = np.random.default_rng(1)
+    idx = np.unique(np.concatenate([rng.integers(0, 1 << n, 64), [0, (1 << n) - 1]]))
+    got = np.array([st.copy_out(int(k), 1)[0] for k in idx])
+    if name == "qft":
+        x = meta["x"]
+        ph = ((x * idx.astype(object)) % (1 << n)).astype(np.float64) / (1 << n)
+        ref = np.exp(2j * np.pi * ph) / math.sqrt(2.0 ** n)
+        return {"closed_form_max_abs_err": float(np.max(np.abs(got - ref))),
+                "samples": int(idx.size)}
+    ref = np.where((idx == 0) | (idx == (1 << n) - 1), math.sqrt(0.5), 0.0).astype(complex)
+    return {"closed_form_max_abs_err": float(np.max(np.abs(got - ref))),
+            "bit_exact": bool(np.array_equal(got, ref)), "samples": int(idx.size)}
+
+
+def run_macro(lfqs, stream, n: int, reps: int, unfused: bool, hbm_peak: float):
+    """configs[2]: QFT(n)|x> and GHZ(n) from |0> on one GPU (n = 33: a 128 GiB state), as
+    compiled fused passes (LFQS_FUSE_JIT, compile outside the timed region) and, strict,
+    one class-kernel pass per gate (LFQS_FUSE_NONE).  CUDA events on the launching stream;
+    min and mean over `reps` after one warm-up; closed-form checks on sampled amplitudes."""
+    import torch
+    x = int(W.SplitMix64(n).next_u64() & ((1 << n) - 1))
+    circuits = [("qft", W.qft(n), x, {"x": x}), ("ghz", W.ghz(n), 0, {})]
+    modes = [("jit+phase", lfqs.FUSE_LOW | lfqs.FUSE_JIT | lfqs.FUSE_PHASE)]
+    if unfused:
+        modes.append(("unfused", lfqs.FUSE_NONE))
+    out = {}
+    with lfqs.State.create(n, 0, stream=stream) as st:
+        for name, gates, init, meta in circuits:
+            arr = lfqs.marshal_gates(gates)
+            for mode, flags in modes:
+                compile_s = None
+                if flags & lfqs.FUSE_JIT:
+                    t0 = time.time()
+                    lfqs.lfqs_jit_precompile(n, arr, flags)
+                    compile_s = time.time() - t0
+                times, passes = [], 0
+                nrep = reps if mode != "unfused" or name == "ghz" else 1
+                for r in range(nrep + (1 if mode != "unfused" else 0)):
+                    st.init_basis(init)
+                    torch.cuda.synchronize()
+                    c0 = st.launches()
+                    e0 = torch.cuda.Event(enable_timing=True)
+                    e1 = torch.cuda.Event(enable_timing=True)
+                    e0.record(stream)
+                    lfqs.lfqs_run_circuit(st.h, arr, flags)
+                    e1.record(stream)
+                    torch.cuda.synchronize()
+                    passes = st.launches() - c0
+                    if mode == "unfused" or r > 0:
+                        times.append(e0.elapsed_time(e1))
+                t = min(times)
+                pass_bytes = 2.0 * 16 * 2 ** n
+                rec = {"mode": mode, "gates": len(gates), "passes": int(passes),
+                       "ms": round(t, 3), "ms_mean": round(float(np.mean(times)), 3),
+                       "reps": len(times), "gates_per_s": len(gates) / (t / 1e3),
+                       "hbm_frac_per_pass": pass_bytes * passes / (t / 1e3) / 1e9 / hbm_peak,
+                       "conv_frac": pass_bytes * len(gates) / (t / 1e3) / 1e9 / hbm_peak}
+                if compile_s is not None:
+                    rec["jit_compile_s_untimed"] = round(compile_s, 3)
+                rec.update(_closed_form_err(name, n, st, meta))
+                out[f"{name}{n}_{mode}"] = rec
+    torch.cuda.synchronize()
+    return out
+
+
+# ----------------------------------------------------------------------------
 # GPU arm
 # ----------------------------------------------------------------------------
 
@@ -244,6 +316,12 @@ def main():
     ap.add_argument("--e2e-steps", type=int, default=2)
     ap.add_argument("--ref-step-s", type=float, default=12.0)
     ap.add_argument("--per-gate-json", default="", help="write per-gate timings here")
+    ap.add_argument("--macro-n", type=int, default=33,
+                    help="configs[2] leg at N = 1: QFT and GHZ at this many qubits after the "
+                         "sweep (0: skip)")
+    ap.add_argument("--macro-reps", type=int, default=3)
+    ap.add_argument("--no-macro-unfused", action="store_true",
+                    help="skip the strict one-pass-per-gate QFT/GHZ runs of the macro leg")
     ap.add_argument("--same-device", action="store_true",
                     help="test only: every rank on cuda:0 (exercises the N>1 path on one GPU)")
     ap.add_argument("--transport", default="p2p", choices=["p2p", "nccl"],
@@ -360,6 +438,14 @@ def main():
         c["share"] = c["ms"] / mean_ms.sum()
     dom = max(classes, key=lambda k: classes[k]["ms"])
     dc = classes[dom]
+    # the gate furthest below its own roofline (SURVEY §8(d) touched bytes / mean time)
+    fr = [(W.algorithmic_bytes(g, n_loc) / (mean_ms[i] / 1e3) / 1e9 / hbm_peak, i)
+          for i, (_, g) in enumerate(sweep)]
+    wf, wi = min(fr)
+    worst_gate = {"label": sweep[wi][1].label(), "class": sweep[wi][0],
+                  "ms": round(float(mean_ms[wi]), 4),
+                  "alg_bytes": W.algorithmic_bytes(sweep[wi][1], n_loc), "alg_frac": round(wf, 4),
+                  "conv_frac": round(32.0 * 2 ** n_loc / (mean_ms[wi] / 1e3) / 1e9 / hbm_peak, 4)}
     traffic = None
     tp = os.path.join(ROOT, "profiles", "traffic_per_launch.json")
     if world == 1 and os.path.exists(tp):  # ncu capture of the N = 1 workload
@@ -367,7 +453,8 @@ def main():
             traffic = json.load(open(tp)).get(dom)
         except Exception:
             traffic = None
-    roofline = {"bound": "hbm", "kernel": f"{dom} gate kernels (k_group / k_lowq)",
+    roofline = {"bound": "hbm",
+                "kernel": f"{dom} class per-gate kernels (apply_kernels.cu k_group_x2 / k_group)",
                 "achieved": dc["alg_GBps"], "peak": hbm_peak, "unit": "GB/s",
                 "frac": dc["alg_GBps"] / hbm_peak, "traffic": traffic, "peak_source": peak_src,
                 "bytes_per_launch": dc["alg_bytes"] / dc["gates"],
@@ -444,6 +531,13 @@ def main():
                       "lfqs_measure_probs"}
         del host
 
+    macro = None
+    if world == 1 and args.macro_n > 0:
+        st.close()
+        torch.cuda.synchronize()
+        macro = run_macro(lfqs, stream, args.macro_n, args.macro_reps,
+                          not args.no_macro_unfused, hbm_peak)
+
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         st.close()
@@ -467,6 +561,8 @@ def main():
                        **({"test_same_device": "all ranks share cuda:0 -- not a scaling number"}
                           if args.same_device else {})},
             "roofline": roofline,
+            "worst_gate": worst_gate,
+            "macro": macro,
             "nvlink": nvlink,
             "classes": {k: {kk: (round(vv, 4) if isinstance(vv, float) else vv)
                             for kk, vv in v.items()} for k, v in classes.items()},

@@ -145,11 +145,12 @@ bool run_fused_circuit(const LaunchCtx& ctx, const std::vector<Decoded>& gates, 
 // Whole-list fused execution with exact-commutation reordering (fused_kernels.cu).
 void run_fused_schedule(const LaunchCtx& ctx, const std::vector<Decoded>& gates, int tile_qubits);
 
-// Reductions (C9): out[v], v < 2^nq; deterministic.
-// Only amplitudes with (k & fmask) == fpat contribute (used to split > 10 qubits).
+// Reductions (C9): d_out[v], v < 2^nq (nq <= 20, bit s of v = bit qubits[s]); one read
+// pass over the shard whatever nq is; deterministic (fixed grid and summation order).
+// d_partials must hold probs_partials_doubles(ctx.n_local, qubits, nq) doubles.
 void launch_probs(const LaunchCtx& ctx, const int* qubits, int nq, double* d_partials,
-                  int n_partials_blocks, double* d_out, uint64_t fmask = 0, uint64_t fpat = 0);
-int probs_blocks();
+                  size_t partials_doubles, double* d_out);
+size_t probs_partials_doubles(int n_local, const int* qubits, int nq);
 
 // Projective collapse: a[k] = (k & mask) == pat ? scale * a[k] : 0 (all zero if
 // zero_all: the rank's global bits do not match the outcome).

@@ -11,6 +11,7 @@
 // Probabilities are accumulated in double for both amplitude precisions.
 #include <cuda_runtime.h>
 
+#include <algorithm>
 #include <cstring>
 #include <mutex>
 #include <set>
@@ -26,21 +27,43 @@ constexpr int kThreads = 256;
 constexpr int kWarps = kThreads / 32;
 constexpr int kBlocks = 148 * 4;  // fixed grid => fixed summation order
 constexpr int kU = 4;             // 32-amplitude rows per warp iteration
-constexpr int kMaxQ = 10;
+constexpr int kMaxLo = 10;        // qubits binned in the shared-memory histogram
+constexpr int kMaxQ = 20;         // qubits per measurement (lfqs_measure_probs)
 
+// Two-level binning (one read pass for up to 20 measured qubits): the measured qubits
+// at the kMaxLo lowest positions ("lo") are histogrammed per warp in shared memory as
+// before; the others ("hi", all at positions >= 10, so never a lane bit) select a
+// subspace: work unit u = h * slices + s reads slice s of the amplitudes whose hi bits
+// equal h -- their indices are the subspace index with h's bits inserted at the hi
+// positions -- and writes its lo-histogram to partials[u].  A final kernel sums the
+// slices of each (h, lo) bin in fixed order, so the result is deterministic.
 struct QList {
-  int nq;
-  int q[kMaxQ];
+  int nq;                // lo qubits (<= kMaxLo)
+  int q[kMaxLo];         // their positions; bin bit u = bit q[u]
   uint32_t lane_free;    // lane bits (0..4) not measured: folded by shuffles
-  uint64_t fmask, fpat;  // only amplitudes with (k & fmask) == fpat contribute
+  int nh;                // hi qubits (<= kMaxQ - kMaxLo), ascending positions
+  int hpos[kMaxQ - kMaxLo];
+  uint64_t slices;       // slices per hi pattern
+  uint64_t rows;         // 32-amplitude rows in one hi subspace
 };
 
 __device__ __forceinline__ int bin_of(const QList& ql, uint64_t k) {
   int v = 0;
 #pragma unroll
-  for (int s = 0; s < kMaxQ; ++s)
+  for (int s = 0; s < kMaxLo; ++s)
     if (s < ql.nq) v |= (int)((k >> ql.q[s]) & 1) << s;
   return v;
+}
+
+// subspace index j -> amplitude index: insert the bits of h at the hi positions
+__device__ __forceinline__ uint64_t insert_hi(const QList& ql, uint64_t j, uint64_t h) {
+#pragma unroll
+  for (int u = 0; u < kMaxQ - kMaxLo; ++u)
+    if (u < ql.nh) {
+      const int p = ql.hpos[u];
+      j = ((j >> p) << (p + 1)) | (j & ((1ull << p) - 1)) | (((h >> u) & 1ull) << p);
+    }
+  return j;
 }
 
 // Amplitude accessors: interleaved pairs (AOS) or two planes (SOA, LFQS_STATE_SOA).
@@ -82,8 +105,8 @@ __device__ __forceinline__ double norm2(cx<S> x) {
 }
 
 template <class S, class A>
-__global__ void __launch_bounds__(kThreads) k_probs(const A a, uint64_t n_rows,
-                                                    const QList ql, double* __restrict__ partials) {
+__global__ void __launch_bounds__(kThreads) k_probs(const A a, const QList ql, uint64_t units,
+                                                    double* __restrict__ partials) {
   extern __shared__ double hist[];  // [kWarps][nbins]
   const int nbins = 1 << ql.nq;
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
@@ -91,53 +114,80 @@ __global__ void __launch_bounds__(kThreads) k_probs(const A a, uint64_t n_rows,
   __syncthreads();
   double* my = hist + warp * nbins;
   const bool rep = (lane & ql.lane_free) == 0;
-  // rows of 32 amplitudes; warp w of block b handles row groups in a fixed stride
-  const uint64_t stride = (uint64_t)gridDim.x * kWarps * kU;
-  for (uint64_t r0 = ((uint64_t)blockIdx.x * kWarps + warp) * kU; r0 < n_rows; r0 += stride) {
-    double p[kU];
+  const uint64_t per = (ql.rows + ql.slices - 1) / ql.slices;
+  for (uint64_t unit = blockIdx.x; unit < units; unit += gridDim.x) {
+    const uint64_t h = unit / ql.slices, sl = unit % ql.slices;
+    const uint64_t rb = sl * per, re = min(ql.rows, rb + per);
+    // rows of 32 amplitudes; warp w handles row groups in a fixed stride
+    for (uint64_t r0 = rb + (uint64_t)warp * kU; r0 < re; r0 += (uint64_t)kWarps * kU) {
+      double p[kU];
+      uint64_t k[kU];
 #pragma unroll
-    for (int u = 0; u < kU; ++u) {
-      const uint64_t r = r0 + u;
-      if (r < n_rows) {
-        const cx<S> x = a.get(r * 32 + lane);
-        p[u] = ((r * 32 + lane) & ql.fmask) == ql.fpat ? norm2<S>(x) : 0.0;
-      } else {
-        p[u] = 0.0;
+      for (int u = 0; u < kU; ++u) {
+        k[u] = insert_hi(ql, (r0 + u) * 32, h) + lane;
+        p[u] = (r0 + u < re) ? norm2<S>(a.get(k[u])) : 0.0;
+      }
+#pragma unroll
+      for (int u = 0; u < kU; ++u) {
+#pragma unroll
+        for (int b = 0; b < 5; ++b)
+          if (ql.lane_free >> b & 1) p[u] += __shfl_xor_sync(0xffffffffu, p[u], 1 << b);
+        if (rep && r0 + u < re) my[bin_of(ql, k[u])] += p[u];
       }
     }
-#pragma unroll
-    for (int u = 0; u < kU; ++u) {
-#pragma unroll
-      for (int b = 0; b < 5; ++b)
-        if (ql.lane_free >> b & 1) p[u] += __shfl_xor_sync(0xffffffffu, p[u], 1 << b);
-      if (rep && r0 + u < n_rows) my[bin_of(ql, (r0 + u) * 32 + lane)] += p[u];
+    __syncthreads();
+    for (int bin = threadIdx.x; bin < nbins; bin += kThreads) {
+      double s = 0.0;
+      for (int w = 0; w < kWarps; ++w) {
+        s += hist[w * nbins + bin];
+        hist[w * nbins + bin] = 0.0;
+      }
+      partials[unit * nbins + bin] = s;
     }
-  }
-  __syncthreads();
-  for (int bin = threadIdx.x; bin < nbins; bin += kThreads) {
-    double s = 0.0;
-    for (int w = 0; w < kWarps; ++w) s += hist[w * nbins + bin];
-    partials[(uint64_t)blockIdx.x * nbins + bin] = s;
+    __syncthreads();
   }
 }
 
-__global__ void k_probs_final(const double* __restrict__ partials, int nblocks, int nbins,
-                              double* __restrict__ out) {
-  const int bin = blockIdx.x * blockDim.x + threadIdx.x;
-  if (bin >= nbins) return;
-  double s = 0.0;
-  for (int b = 0; b < nblocks; ++b) s += partials[(uint64_t)b * nbins + bin];
-  out[bin] = s;
+// out[v], v < 2^(nlo + nh): bit u of v's lo part = lo qubit u, of its hi part = hi qubit u
+// (the caller's order is restored on the host side of launch_probs through lo_of / hi_of).
+struct FinalMap {
+  int nq;                 // caller's qubit count
+  int lo_of[kMaxQ];       // caller index s -> lo bit (or -1)
+  int hi_of[kMaxQ];       // caller index s -> hi bit (or -1)
+};
+
+__global__ void k_probs_final(const double* __restrict__ partials, uint64_t slices, int nlo,
+                              const FinalMap fm, double* __restrict__ out) {
+  const uint64_t v = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (v >= (1ull << fm.nq)) return;
+  uint64_t lo = 0, h = 0;
+  for (int s = 0; s < fm.nq; ++s) {
+    const uint64_t b = (v >> s) & 1;
+    if (fm.lo_of[s] >= 0) lo |= b << fm.lo_of[s];
+    else h |= b << fm.hi_of[s];
+  }
+  double acc = 0.0;
+  const uint64_t base = h * slices;
+  for (uint64_t s = 0; s < slices; ++s) acc += partials[((base + s) << nlo) + lo];
+  out[v] = acc;
 }
 
-// Small-state path (< 32 amplitudes): one thread, ascending order.
+// Small-state path (< 32 amplitudes): one thread, ascending order, the caller's bins.
+struct CallerQ {
+  int nq;
+  int q[kMaxQ];
+};
+
 template <class S, class A>
-__global__ void k_probs_tiny(const A a, uint64_t n_amps, const QList ql,
+__global__ void k_probs_tiny(const A a, uint64_t n_amps, const CallerQ cq,
                              double* __restrict__ out) {
-  const int nbins = 1 << ql.nq;
+  const int nbins = 1 << cq.nq;
   for (int b = 0; b < nbins; ++b) out[b] = 0.0;
-  for (uint64_t k = 0; k < n_amps; ++k)
-    if ((k & ql.fmask) == ql.fpat) out[bin_of(ql, k)] += norm2<S>(a.get_plain(k));
+  for (uint64_t k = 0; k < n_amps; ++k) {
+    int v = 0;
+    for (int s = 0; s < cq.nq; ++s) v |= (int)((k >> cq.q[s]) & 1) << s;
+    out[v] += norm2<S>(a.get_plain(k));
+  }
 }
 
 // --- projective collapse (one streaming pass, two-amplitude accesses) --------
@@ -190,21 +240,71 @@ Soa<S> soa_acc(const LaunchCtx& ctx) {
   return Soa<S>{re, re + (1ull << ctx.n_local)};
 }
 
+// Splits the caller's qubits into lo (the kMaxLo lowest positions) and hi (ascending).
+struct ProbsPlan {
+  QList ql;
+  FinalMap fm;
+  CallerQ cq;
+  uint64_t units;
+};
+
+ProbsPlan make_probs_plan(int n_local, const int* qubits, int nq) {
+  ProbsPlan pp;
+  std::memset(&pp, 0, sizeof pp);
+  pp.fm.nq = nq;
+  pp.cq.nq = nq;
+  int order[kMaxQ];
+  for (int s = 0; s < nq; ++s) {
+    order[s] = s;
+    pp.cq.q[s] = qubits[s];
+  }
+  std::sort(order, order + nq, [&](int x, int y) { return qubits[x] < qubits[y]; });
+  const int nlo = nq < kMaxLo ? nq : kMaxLo;
+  uint32_t measured_lane_bits = 0;
+  for (int u = 0; u < nq; ++u) {
+    const int s = order[u];
+    pp.fm.lo_of[s] = pp.fm.hi_of[s] = -1;
+    if (u < nlo) {
+      pp.ql.q[u] = qubits[s];
+      pp.fm.lo_of[s] = u;
+      if (qubits[s] < 5) measured_lane_bits |= 1u << qubits[s];
+    } else {
+      pp.ql.hpos[u - nlo] = qubits[s];  // ascending: insert_hi's order
+      pp.fm.hi_of[s] = u - nlo;
+    }
+  }
+  pp.ql.nq = nlo;
+  pp.ql.nh = nq - nlo;
+  pp.ql.lane_free = 0x1fu & ~measured_lane_bits;
+  pp.ql.rows = n_local >= 5 ? (1ull << (n_local - pp.ql.nh)) / 32 : 0;
+  // enough units for every block to see several (balance), each slice >= kU rows per warp
+  const uint64_t hs = 1ull << pp.ql.nh;
+  uint64_t sl = pp.ql.nh == 0 ? (uint64_t)kBlocks : std::max<uint64_t>(1, 4ull * kBlocks / hs);
+  sl = std::min<uint64_t>(sl, std::max<uint64_t>(1, pp.ql.rows / (kWarps * kU)));
+  pp.ql.slices = sl;
+  pp.units = hs * sl;
+  return pp;
+}
+
 template <class S, class A>
-void probs_t(const LaunchCtx& ctx, const A a, const QList& ql, double* d_partials, double* d_out) {
+void probs_t(const LaunchCtx& ctx, const A a, const ProbsPlan& pp, double* d_partials,
+             double* d_out) {
   const uint64_t n_amps = 1ull << ctx.n_local;
   if (n_amps < 32) {
-    k_probs_tiny<S, A><<<1, 1, 0, ctx.stream>>>(a, n_amps, ql, d_out);
+    k_probs_tiny<S, A><<<1, 1, 0, ctx.stream>>>(a, n_amps, pp.cq, d_out);
     LFQS_CUDA_CHECK(cudaGetLastError());
     ++*ctx.launch_counter;
     return;
   }
-  const int nbins = 1 << ql.nq;
+  const int nbins = 1 << pp.ql.nq;
   const size_t smem = sizeof(double) * kWarps * nbins;
-  ensure_smem_attr((const void*)k_probs<S, A>, sizeof(double) * kWarps * (1 << kMaxQ));
-  k_probs<S, A><<<kBlocks, kThreads, smem, ctx.stream>>>(a, n_amps / 32, ql, d_partials);
+  ensure_smem_attr((const void*)k_probs<S, A>, sizeof(double) * kWarps * (1 << kMaxLo));
+  const unsigned grid = (unsigned)std::min<uint64_t>(pp.units, kBlocks);
+  k_probs<S, A><<<grid, kThreads, smem, ctx.stream>>>(a, pp.ql, pp.units, d_partials);
   LFQS_CUDA_CHECK(cudaGetLastError());
-  k_probs_final<<<(nbins + 255) / 256, 256, 0, ctx.stream>>>(d_partials, kBlocks, nbins, d_out);
+  const uint64_t nout = 1ull << pp.fm.nq;
+  k_probs_final<<<(unsigned)((nout + 255) / 256), 256, 0, ctx.stream>>>(
+      d_partials, pp.ql.slices, pp.ql.nq, pp.fm, d_out);
   LFQS_CUDA_CHECK(cudaGetLastError());
   *ctx.launch_counter += 2;
 }
@@ -213,7 +313,10 @@ inline size_t amp_bytes(const LaunchCtx& ctx) { return ctx.c64 ? 8 : 16; }
 
 }  // namespace
 
-int probs_blocks() { return kBlocks; }
+size_t probs_partials_doubles(int n_local, const int* qubits, int nq) {
+  const ProbsPlan pp = make_probs_plan(n_local, qubits, nq);
+  return std::max<size_t>(1, pp.units << pp.ql.nq);
+}
 
 void ensure_smem_attr(const void* kernel, int bytes) {
   // cudaFuncSetAttribute is per device; remember (kernel, device) pairs done.
@@ -228,28 +331,18 @@ void ensure_smem_attr(const void* kernel, int bytes) {
 }
 
 void launch_probs(const LaunchCtx& ctx, const int* qubits, int nq, double* d_partials,
-                  int n_partials_blocks, double* d_out, uint64_t fmask, uint64_t fpat) {
-  require(nq >= 0 && nq <= kMaxQ, "one probability pass covers at most 10 qubits");
-  require(n_partials_blocks >= kBlocks, "partials buffer too small");
-  QList ql;
-  std::memset(&ql, 0, sizeof ql);
-  ql.nq = nq;
-  ql.fmask = fmask;
-  ql.fpat = fpat;
-  uint32_t measured_lane_bits = 0;
-  for (int s = 0; s < nq; ++s) {
-    ql.q[s] = qubits[s];
-    if (qubits[s] < 5) measured_lane_bits |= 1u << qubits[s];
-  }
-  ql.lane_free = 0x1fu & ~measured_lane_bits;
+                  size_t partials_doubles, double* d_out) {
+  require(nq >= 0 && nq <= kMaxQ, "one probability pass covers at most 20 qubits");
+  const ProbsPlan pp = make_probs_plan(ctx.n_local, qubits, nq);
+  require(partials_doubles >= (pp.units << pp.ql.nq), "internal: partials buffer too small");
   if (ctx.c64 && ctx.soa)
-    probs_t<float>(ctx, soa_acc<float>(ctx), ql, d_partials, d_out);
+    probs_t<float>(ctx, soa_acc<float>(ctx), pp, d_partials, d_out);
   else if (ctx.c64)
-    probs_t<float>(ctx, aos<float>(ctx), ql, d_partials, d_out);
+    probs_t<float>(ctx, aos<float>(ctx), pp, d_partials, d_out);
   else if (ctx.soa)
-    probs_t<double>(ctx, soa_acc<double>(ctx), ql, d_partials, d_out);
+    probs_t<double>(ctx, soa_acc<double>(ctx), pp, d_partials, d_out);
   else
-    probs_t<double>(ctx, aos<double>(ctx), ql, d_partials, d_out);
+    probs_t<double>(ctx, aos<double>(ctx), pp, d_partials, d_out);
 }
 
 void launch_collapse(const LaunchCtx& ctx, uint64_t mask, uint64_t pat, double scale,

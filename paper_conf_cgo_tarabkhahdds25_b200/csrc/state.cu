@@ -81,8 +81,10 @@ void State::common_init(int n_, int world_, int device_, cudaStream_t s, bool c6
     LFQS_CUDA_CHECK(cudaStreamCreateWithFlags(&stream, cudaStreamNonBlocking));
     own_stream = true;
   }
-  LFQS_CUDA_CHECK(cudaMalloc(&d_partials, sizeof(double) * probs_blocks() * 1024));
-  LFQS_CUDA_CHECK(cudaMalloc(&d_probs, sizeof(double) * 1024));
+  partials_cap = size_t(148) * 4 * 1024;  // nq <= 10: one 1024-bin histogram per block
+  probs_cap = 1024;
+  LFQS_CUDA_CHECK(cudaMalloc(&d_partials, sizeof(double) * partials_cap));
+  LFQS_CUDA_CHECK(cudaMalloc(&d_probs, sizeof(double) * probs_cap));
 }
 
 State* State::create_local(int n, int device, cudaStream_t stream, void* borrowed, bool c64,
@@ -543,21 +545,23 @@ void State::collapse(const int* qubits, int nq, uint64_t outcome, double scale) 
 }
 
 // Probabilities of the local physical qubits lq[0..nl) of one shard into host[2^nl]
-// (bit u of the bin = bit lq[u]).  One reduction pass covers 10 qubits; more are
-// enumerated by filtered passes over the extra qubits' patterns.
+// (bit u of the bin = bit lq[u]): one read pass (two-level binning, reduce_kernels.cu).
 void State::local_probs(int shard, const int* lq, int nl, double* host) {
-  const int lo = nl < 10 ? nl : 10;
-  const int nh = nl - lo;
-  for (uint64_t h = 0; h < (1ull << nh); ++h) {
-    uint64_t fmask = 0, fpat = 0;
-    for (int j = 0; j < nh; ++j) {
-      fmask |= 1ull << lq[lo + j];
-      fpat |= ((h >> j) & 1ull) << lq[lo + j];
-    }
-    launch_probs(ctx(shard), lq, lo, d_partials, probs_blocks(), d_probs, fmask, fpat);
-    LFQS_CUDA_CHECK(cudaMemcpyAsync(host + (h << lo), d_probs, sizeof(double) << lo,
-                                    cudaMemcpyDeviceToHost, stream));
-  }
+  const size_t need = probs_partials_doubles(n_local, lq, nl);
+  auto grow = [&](double*& p, size_t& cap, size_t want) {
+    if (cap >= want) return;
+    LFQS_CUDA_CHECK(cudaStreamSynchronize(stream));
+    if (p) cudaFree(p);
+    p = nullptr;
+    cap = 0;
+    LFQS_CUDA_CHECK(cudaMalloc(&p, sizeof(double) * want));
+    cap = want;
+  };
+  grow(d_partials, partials_cap, need);
+  grow(d_probs, probs_cap, size_t(1) << nl);
+  launch_probs(ctx(shard), lq, nl, d_partials, partials_cap, d_probs);
+  LFQS_CUDA_CHECK(cudaMemcpyAsync(host, d_probs, sizeof(double) << nl, cudaMemcpyDeviceToHost,
+                                  stream));
   LFQS_CUDA_CHECK(cudaStreamSynchronize(stream));
 }
 

@@ -36,8 +36,9 @@ struct State : lfqs_state {
   bool own_stream = false;
   uint64_t launches = 0;
   Options opt;
-  double* d_partials = nullptr; // reduction scratch
-  double* d_probs = nullptr;
+  double* d_partials = nullptr; // reduction scratch (grown on demand)
+  double* d_probs = nullptr;    // 2^nq result bins (grown on demand)
+  size_t partials_cap = 0, probs_cap = 0;  // doubles
   Planner plan;
   Comm* comm = nullptr;
   P2P* p2p = nullptr;           // CUDA-IPC peer transport (instead of comm)

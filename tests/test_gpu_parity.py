@@ -181,6 +181,46 @@ def test_measure_probs_vs_oracle(L, n):
             assert np.array_equal(got, st.measure_probs(qs))  # deterministic
 
 
+@pytest.mark.parametrize("n,world", [(11, 1), (16, 1), (21, 1), (16, 4)])
+def test_measure_probs_many_qubits_one_pass(L, n, world):
+    """11..20 measured qubits (two-level binning: the 10 lowest positions in the shared
+    histogram, the rest select subspaces), in caller order, including lane bits, vs the
+    oracle's pairwise sums; deterministic; also through a virtual partition."""
+    psi = W.random_state(n, 3 * n)
+    rng = np.random.default_rng(n)
+    cases = [list(range(min(n, 20))), list(range(n - 1, max(-1, n - 21), -1)),
+             [int(x) for x in rng.permutation(n)[:min(n, 20)]],
+             [int(x) for x in rng.permutation(n)[:11]]]
+    st = L.State.create(n) if world == 1 else L.State.virtual(n, world)
+    with st:
+        st.copy_in(psi)
+        if world > 1:
+            st.run_circuit([W.Gate("X", (n - 1,)), W.Gate("X", (n - 1,))])  # flip + unflip
+        for qs in cases:
+            got = st.measure_probs(qs)
+            ref = O.probs(n, psi, qs)
+            np.testing.assert_allclose(got, ref, rtol=1e-13, atol=1e-17, err_msg=str(qs))
+            assert np.array_equal(got, st.measure_probs(qs))
+
+
+def test_measure_probs_20_qubits_costs_one_pass(L):
+    """n = 28, 20 measured qubits: one read pass (not 2^10 filtered passes):
+    the 20-qubit measurement costs at most ~2x the 1-qubit one (same bytes read)."""
+    import time
+    n = 28
+    with L.State.create(n) as st:
+        st.init_random(5)
+        for qs in ([3], list(range(4, 24))):
+            st.measure_probs(qs)  # warm-up (scratch allocation)
+        t = {}
+        for key, qs in (("one", [3]), ("twenty", list(range(4, 24)))):
+            t0 = time.perf_counter()
+            for _ in range(5):
+                st.measure_probs(qs)
+            t[key] = (time.perf_counter() - t0) / 5
+        assert t["twenty"] <= 2.5 * t["one"] + 2e-3, t
+
+
 @pytest.mark.parametrize("n", [8, 20, 26])
 def test_ghz_and_uniform_closed_forms(L, n):
     with L.State.create(n) as st:
