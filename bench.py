@@ -242,7 +242,9 @@ def _closed_form_err(name, n, st, meta):
         x = meta["x"]
         ph = ((x * idx.astype(object)) % (1 << n)).astype(np.float64) / (1 << n)
         ref = np.exp(2j * np.pi * ph) / math.sqrt(2.0 ** n)
-        return {"closed_form_max_abs_err": float(np.max(np.abs(got - ref))),
+        err = float(np.max(np.abs(got - ref)))
+        return {"closed_form_max_abs_err": err,
+                "closed_form_rel_err": err * math.sqrt(2.0 ** n),  # amplitudes are 2^(-n/2)
                 "samples": int(idx.size)}
     ref = np.where((idx == 0) | (idx == (1 << n) - 1), math.sqrt(0.5), 0.0).astype(complex)
     return {"closed_form_max_abs_err": float(np.max(np.abs(got - ref))),
@@ -287,10 +289,18 @@ def run_macro(lfqs, stream, n: int, reps: int, unfused: bool, hbm_peak: float):
                         times.append(e0.elapsed_time(e1))
                 t = min(times)
                 pass_bytes = 2.0 * 16 * 2 ** n
+                # bytes the passes must move: a fused pass reads and writes the whole state;
+                # a per-gate pass its touched part / its DRAM lines
+                if mode == "unfused":
+                    need = sum(W.algorithmic_bytes(g, n) for g in gates)
+                    need_dram = sum(W.dram_line_bytes(g, n) for g in gates)
+                else:
+                    need = need_dram = pass_bytes * passes
                 rec = {"mode": mode, "gates": len(gates), "passes": int(passes),
                        "ms": round(t, 3), "ms_mean": round(float(np.mean(times)), 3),
                        "reps": len(times), "gates_per_s": len(gates) / (t / 1e3),
-                       "hbm_frac_per_pass": pass_bytes * passes / (t / 1e3) / 1e9 / hbm_peak,
+                       "hbm_frac": need / (t / 1e3) / 1e9 / hbm_peak,
+                       "hbm_frac_dram_model": need_dram / (t / 1e3) / 1e9 / hbm_peak,
                        "conv_frac": pass_bytes * len(gates) / (t / 1e3) / 1e9 / hbm_peak}
                 if compile_s is not None:
                     rec["jit_compile_s_untimed"] = round(compile_s, 3)
@@ -442,10 +452,21 @@ def main():
     fr = [(W.algorithmic_bytes(g, n_loc) / (mean_ms[i] / 1e3) / 1e9 / hbm_peak, i)
           for i, (_, g) in enumerate(sweep)]
     wf, wi = min(fr)
-    worst_gate = {"label": sweep[wi][1].label(), "class": sweep[wi][0],
-                  "ms": round(float(mean_ms[wi]), 4),
-                  "alg_bytes": W.algorithmic_bytes(sweep[wi][1], n_loc), "alg_frac": round(wf, 4),
-                  "conv_frac": round(32.0 * 2 ** n_loc / (mean_ms[wi] / 1e3) / 1e9 / hbm_peak, 4)}
+
+    def gate_rec(i):
+        g = sweep[i][1]
+        t = mean_ms[i] / 1e3
+        return {"label": g.label(), "class": sweep[i][0], "ms": round(float(mean_ms[i]), 4),
+                "alg_bytes": W.algorithmic_bytes(g, n_loc),
+                "alg_frac": round(W.algorithmic_bytes(g, n_loc) / t / 1e9 / hbm_peak, 4),
+                "dram_model_bytes": W.dram_line_bytes(g, n_loc),
+                "dram_model_frac": round(W.dram_line_bytes(g, n_loc) / t / 1e9 / hbm_peak, 4),
+                "conv_frac": round(32.0 * 2 ** n_loc / t / 1e9 / hbm_peak, 4)}
+    # worst by SURVEY §8(d) touched bytes, and by the DRAM line-granularity model
+    # (workloads.dram_line_bytes, from tools/probe_sparse.cu)
+    worst_gate = gate_rec(wi)
+    dm = min(range(len(sweep)), key=lambda i: W.dram_line_bytes(sweep[i][1], n_loc) / mean_ms[i])
+    worst_gate["worst_by_dram_model"] = gate_rec(dm)
     traffic = None
     tp = os.path.join(ROOT, "profiles", "traffic_per_launch.json")
     if world == 1 and os.path.exists(tp):  # ncu capture of the N = 1 workload

@@ -404,6 +404,12 @@ lfqs_status lfqs_kernel_launches(const lfqs_state* s, uint64_t* count);
 #define LFQS_OPT_L2_FETCH_GRANULARITY 18 /* device-wide L2 fetch granularity hint in bytes
                                             (cudaLimitMaxL2FetchGranularity: 0, 32, 64 or
                                             128) for the state's device; measurement knob */
+#define LFQS_OPT_LINE_READS 19 /* 1 (default): per-gate kernels whose gate fixes qubit 1 or 2
+                                  (a control, or the pattern of a one-entry diagonal) read
+                                  whole 128-B lines coalesced and store only the touched
+                                  groups (DRAM reads whole lines anyway:
+                                  tools/probe_sparse.cu); 0: read only the touched groups.
+                                  Bit-identical results either way */
 lfqs_status lfqs_set_option(lfqs_state* s, int option, int64_t value);
 const char* lfqs_last_error(void);
 int lfqs_abi_version(void);

@@ -513,6 +513,7 @@ lfqs_status lfqs_set_option(lfqs_state* s, int option, int64_t value) {
         break;
       case LFQS_OPT_ITEMS_PER_THREAD: st->opt.items_per_thread = (int)value; break;
       case LFQS_OPT_WIDE256: st->opt.wide256 = value != 0; break;
+      case LFQS_OPT_LINE_READS: st->opt.line_reads = value != 0; break;
       case LFQS_OPT_FUSE_LOW_QUBITS:
         require(value == 0 || (value >= 3 && value <= 12),
                 "fused low qubits must be 0 (auto) or in [3, 12]");

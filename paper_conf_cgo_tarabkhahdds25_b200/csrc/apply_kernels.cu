@@ -180,10 +180,14 @@ struct Offs {
 // writes L amplitudes at k + off[j].  P256: off[2i+1] == off[2i] + 1, so the
 // pair moves as one access.
 // ---------------------------------------------------------------------------
+//
+// pmask / ppat (line-shaped reads): fixed bits at positions 1-2 that run_group took out of
+// the insertion plan; every group is loaded (whole 128-B lines, coalesced) but only groups
+// with (k & pmask) == ppat are updated and stored (probe: tools/probe_sparse.cu).
 template <class S, int L, int U, bool P256, int NPMAX, class Op>
 __global__ void __launch_bounds__(kThreads) k_group(cx<S>* __restrict__ a, uint64_t n_groups,
                                                     const InsertPlan ip, const Offs<L> off,
-                                                    const Op op) {
+                                                    const Op op, uint64_t pmask, uint64_t ppat) {
   const uint64_t g0 = (uint64_t)blockIdx.x * (kThreads * U) + threadIdx.x;
   cx<S> v[U][L];
   uint64_t kk[U];
@@ -204,7 +208,7 @@ __global__ void __launch_bounds__(kThreads) k_group(cx<S>* __restrict__ a, uint6
 #pragma unroll
   for (int u = 0; u < U; ++u) {
     const uint64_t g = g0 + (uint64_t)u * kThreads;
-    if (g < n_groups) {
+    if (g < n_groups && (kk[u] & pmask) == ppat) {
       op(v[u], kk[u]);
       if constexpr (P256) {
 #pragma unroll
@@ -223,7 +227,7 @@ __global__ void __launch_bounds__(kThreads) k_group(cx<S>* __restrict__ a, uint6
 template <class S, int L, int U, int NPMAX, class Op>
 __global__ void __launch_bounds__(kThreads) k_group_x2(cx<S>* __restrict__ a, uint64_t n_items,
                                                        const InsertPlan ip, const Offs<L> off,
-                                                       const Op op) {
+                                                       const Op op, uint64_t pmask, uint64_t ppat) {
   const uint64_t i0 = (uint64_t)blockIdx.x * (kThreads * U) + threadIdx.x;
   cx<S> v[U][L], w[U][L];
   uint64_t kk[U];
@@ -239,7 +243,7 @@ __global__ void __launch_bounds__(kThreads) k_group_x2(cx<S>* __restrict__ a, ui
 #pragma unroll
   for (int u = 0; u < U; ++u) {
     const uint64_t i = i0 + (uint64_t)u * kThreads;
-    if (i < n_items) {
+    if (i < n_items && (kk[u] & pmask) == ppat) {
       op(v[u], kk[u]);
       op(w[u], kk[u] | 1);
 #pragma unroll
@@ -393,10 +397,30 @@ inline uint64_t blocks_for(uint64_t items, uint64_t per_block) {
 }
 
 template <class S, int L, int U, bool P256, class Op>
-void run_group(const LaunchCtx& ctx, uint64_t n_groups, const InsertPlan& ip, const Offs<L>& off,
-               const Op& op) {
+void run_group(const LaunchCtx& ctx, uint64_t n_groups, const InsertPlan& ip_in,
+               const Offs<L>& off, const Op& op) {
   if (n_groups == 0) return;
   auto* a = reinterpret_cast<cx<S>*>(ctx.amps);
+  // Line-shaped reads (LFQS_OPT_LINE_READS): a fixed bit (control or one-entry diagonal
+  // pattern) at position 1 or 2 leaves 1 of every 2 or 4 sectors of each 128-B line
+  // touched, yet DRAM reads whole lines whatever is requested (tools/probe_sparse.cu:
+  // reading 1 sector in 4 takes as long as reading all).  Such bits are taken out of the
+  // insertion plan and become a store predicate: the warps stream whole lines, coalesced,
+  // and write back only the touched groups.  Same per-amplitude arithmetic.
+  InsertPlan ip = ip_in;
+  uint64_t pmask = 0, ppat = 0;
+  if (ctx.opt->line_reads) {
+    uint64_t tb = 0, all = 0;
+    for (int j = 0; j < L; ++j) tb |= off.o[j];
+    for (int i = 0; i < ip_in.np; ++i) all |= 1ull << ip_in.pos[i];
+    const uint64_t F = all & 6ull & ~tb;
+    if (F) {
+      ip = make_plan(all & ~F, ip_in.ones & ~F);
+      pmask = F;
+      ppat = ip_in.ones & F;
+      n_groups <<= __builtin_popcountll(F);
+    }
+  }
   bool even = true;
   for (int j = 0; j < L; ++j) even &= (off.o[j] & 1) == 0;
   if constexpr (!P256 && L <= 4) {
@@ -408,10 +432,10 @@ void run_group(const LaunchCtx& ctx, uint64_t n_groups, const InsertPlan& ip, co
         require(nb < (1ull << 31), "grid too large");
         if (ip.np <= 4)
           k_group_x2<S, L, UX, 4, Op>
-              <<<(unsigned)nb, kThreads, 0, ctx.stream>>>(a, n_items, ip, off, op);
+              <<<(unsigned)nb, kThreads, 0, ctx.stream>>>(a, n_items, ip, off, op, pmask, ppat);
         else
           k_group_x2<S, L, UX, kMaxInsert, Op>
-              <<<(unsigned)nb, kThreads, 0, ctx.stream>>>(a, n_items, ip, off, op);
+              <<<(unsigned)nb, kThreads, 0, ctx.stream>>>(a, n_items, ip, off, op, pmask, ppat);
       };
       // Groups per thread (tuning knob LFQS_OPT_ITEMS_PER_THREAD for pair gates).
       const int ipt = ctx.opt->items_per_thread;
@@ -429,10 +453,11 @@ void run_group(const LaunchCtx& ctx, uint64_t n_groups, const InsertPlan& ip, co
   const uint64_t nb = blocks_for(n_groups, (uint64_t)kThreads * U);
   require(nb < (1ull << 31), "grid too large");
   if (ip.np <= 4)
-    k_group<S, L, U, P256, 4, Op><<<(unsigned)nb, kThreads, 0, ctx.stream>>>(a, n_groups, ip, off, op);
+    k_group<S, L, U, P256, 4, Op>
+        <<<(unsigned)nb, kThreads, 0, ctx.stream>>>(a, n_groups, ip, off, op, pmask, ppat);
   else
     k_group<S, L, U, P256, kMaxInsert, Op>
-        <<<(unsigned)nb, kThreads, 0, ctx.stream>>>(a, n_groups, ip, off, op);
+        <<<(unsigned)nb, kThreads, 0, ctx.stream>>>(a, n_groups, ip, off, op, pmask, ppat);
   LFQS_CUDA_CHECK(cudaGetLastError());
   ++*ctx.launch_counter;
 }

@@ -82,6 +82,7 @@ struct Options {
   // generic 32-byte path on B200 (profiles/r01_gate_sweep.md), so off by default.
   bool lowq_shuffle = false;
   bool wide256 = true;       // two adjacent groups per item, 32-byte accesses
+  bool line_reads = true;    // fixed bits 1-2 -> store predicate, whole-line reads (apply_kernels.cu)
   int fuse_tile_qubits = 12;
   int fuse_low_qubits = 0;   // contiguous low qubits of a fused tile (chunk = 2^L amps);
                              // 0: auto, 7 or 6 by planned pass count (fused_kernels.cu)

@@ -58,6 +58,8 @@ def main():
     ap.add_argument("--l2-fetch", type=int, default=-1,
                     help="LFQS_OPT_L2_FETCH_GRANULARITY in bytes (-1: leave the device default)")
     ap.add_argument("--c64", action="store_true", help="complex64 state")
+    ap.add_argument("--line-reads", type=int, default=-1,
+                    help="LFQS_OPT_LINE_READS (0/1; -1: library default)")
     ap.add_argument("--soa", action="store_true", help="structure-of-arrays state (NEXT-4 layout study)")
     ap.add_argument("--ipt", type=int, default=0, help="groups per thread for pair gates (0=default)")
     args = ap.parse_args()
@@ -72,6 +74,8 @@ def main():
         st.set_option(L.OPT_WIDE256, 0 if args.no_wide else 1)
         st.set_option(L.OPT_ITEMS_PER_THREAD, args.ipt)
         st.set_option(L.OPT_LANE_GROUP, args.lane_group)
+        if args.line_reads >= 0:
+            st.set_option(L.OPT_LINE_READS, args.line_reads)
         if args.l2_fetch >= 0:
             st.set_option(L.OPT_L2_FETCH_GRANULARITY, args.l2_fetch)
         st.init_random(7)

@@ -481,3 +481,44 @@ def touched_amplitudes(g: Gate, n: int) -> int:
     if g.kind == "SWAP":
         return 1 << (n - c - 1)
     return 1 << (n - c)
+
+
+def dram_line_bytes(g: Gate, n: int) -> float:
+    """DRAM cost of one per-gate pass at the memory's access granularity (accounting only).
+
+    Measured with tools/probe_sparse.cu on B200 (profiles/r02_probe_sparse.md): DRAM reads
+    whole 128-B lines whatever part of a line is requested (reading 1 sector in 4 takes as
+    long as reading them all), and a line whose writes cover fewer than two 32-B sectors
+    costs as much as writing two (1-sector-in-4 writes run at half the rate of
+    1-sector-in-2 writes).  So a line holding any touched amplitude costs 128 B of reads
+    plus max(64, 32 * touched sectors) B of writes; the kernels widen touched amplitudes to
+    whole 32-B sectors (bit-0 neighbours).  This is the floor for gates whose touched set
+    is sparser than a line (controls / one-entry diagonals on qubits 0-2), where SURVEY
+    §8(d)'s touched bytes undercount; for line-dense gates it equals algorithmic_bytes.
+    """
+    if g.kind == "I":
+        return 0.0
+    one_entry = g.kind in ("Z", "S", "SDG", "T", "TDG", "PHASE")
+    fixed = {c: 1 for c in g.controls}
+    if one_entry:
+        fixed[g.targets[0]] = 1
+    high_fixed = [b for b in fixed if b >= 3]
+    swap_hi = [t for t in g.targets if t >= 3] if g.kind == "SWAP" else []
+    line_types = 1 << len(swap_hi)
+    rd = wr = 0.0
+    for lt in range(line_types):
+        hib = {t: (lt >> i) & 1 for i, t in enumerate(swap_hi)}
+        sectors = set()
+        for low in range(8):
+            def bit(q):
+                return (low >> q) & 1 if q < 3 else hib.get(q, 1)
+            ok = all(bit(b) == v for b, v in fixed.items() if b < 3)
+            if g.kind == "SWAP":
+                ok = ok and bit(g.targets[0]) != bit(g.targets[1])
+            if ok:
+                sectors.add(low >> 1)
+        if sectors:
+            rd += 128.0
+            wr += max(64.0, 32.0 * len(sectors))
+    lines = 2.0 ** (n - 3) / line_types / 2.0 ** len(high_fixed)
+    return lines * (rd + wr)
