@@ -410,6 +410,24 @@ lfqs_status lfqs_kernel_launches(const lfqs_state* s, uint64_t* count);
                                   groups (DRAM reads whole lines anyway:
                                   tools/probe_sparse.cu); 0: read only the touched groups.
                                   Bit-identical results either way */
+#define LFQS_OPT_EXCHANGE_CHUNK_BITS 20 /* sharded states: each global-qubit exchange is
+                                  split into 2^value parts by the top `value` local qubits
+                                  (the planner never uses the top 2 as exchange positions,
+                                  whatever the value, so the plan does not depend on it;
+                                  an exchange at a position among the top `value` runs
+                                  serially);
+                                  the local ops right before it and right after it that do
+                                  not touch those qubits run part by part on the state's
+                                  stream while the parts move on an exchange stream (NCCL:
+                                  the communicator's stream) -- exchange overlapped with
+                                  local work.  Default 2; 0: serial exchanges.  Same
+                                  per-amplitude arithmetic; pass boundaries of fused runs
+                                  follow the split (rounding-level differences for dense
+                                  gates only) */
+#define LFQS_OPT_EXCHANGE_CTAS 21 /* grid of the device / P2P exchange swap kernels (a
+                                     persistent grid-stride kernel); 0 (default): one
+                                     thread per pair.  A small grid saturates NVLink and
+                                     leaves the SMs to the overlapped local passes */
 lfqs_status lfqs_set_option(lfqs_state* s, int option, int64_t value);
 const char* lfqs_last_error(void);
 int lfqs_abi_version(void);

@@ -49,6 +49,8 @@ OPT_FUSE_PHASE_SPLIT = 16
 OPT_STREAM_MAX_PREFIX = 17
 OPT_L2_FETCH_GRANULARITY = 18
 OPT_LINE_READS = 19
+OPT_EXCHANGE_CHUNK_BITS = 20
+OPT_EXCHANGE_CTAS = 21
 
 STATUS = {0: "OK", -1: "INVALID_ARG", -2: "OUT_OF_MEMORY", -3: "CUDA", -4: "NCCL",
           -5: "UNSUPPORTED"}

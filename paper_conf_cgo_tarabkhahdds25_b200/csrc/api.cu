@@ -514,6 +514,14 @@ lfqs_status lfqs_set_option(lfqs_state* s, int option, int64_t value) {
       case LFQS_OPT_ITEMS_PER_THREAD: st->opt.items_per_thread = (int)value; break;
       case LFQS_OPT_WIDE256: st->opt.wide256 = value != 0; break;
       case LFQS_OPT_LINE_READS: st->opt.line_reads = value != 0; break;
+      case LFQS_OPT_EXCHANGE_CHUNK_BITS:
+        require(value >= 0 && value <= 4, "LFQS_OPT_EXCHANGE_CHUNK_BITS must be in [0, 4]");
+        st->opt.exchange_chunk_bits = (int)value;  // the plan is the same for every value
+        break;
+      case LFQS_OPT_EXCHANGE_CTAS:
+        require(value >= 0 && value <= 65535, "LFQS_OPT_EXCHANGE_CTAS must be in [0, 65535]");
+        st->opt.exchange_ctas = (int)value;
+        break;
       case LFQS_OPT_FUSE_LOW_QUBITS:
         require(value == 0 || (value >= 3 && value <= 12),
                 "fused low qubits must be 0 (auto) or in [3, 12]");

@@ -66,10 +66,14 @@ Comm::~Comm() {
 // Exchanges the amplitudes at `pieces` (offset, count in amplitudes, in this
 // rank's shard) with the same pieces of `partner`, in place.
 void Comm::exchange(void* shard, int amp_bytes, const std::vector<Piece>& pieces, int partner,
-                    cudaStream_t compute) {
-  // The comm stream must see every kernel already queued on the compute stream.
-  LFQS_CUDA_CHECK(cudaEventRecord(ev_start, compute));
-  LFQS_CUDA_CHECK(cudaStreamWaitEvent(cstream, ev_start, 0));
+                    cudaStream_t compute, cudaEvent_t ready) {
+  // The comm stream must see every kernel the exchanged data depends on: `ready`, or
+  // everything already queued on the compute stream.
+  if (ready == nullptr) {
+    LFQS_CUDA_CHECK(cudaEventRecord(ev_start, compute));
+    ready = ev_start;
+  }
+  LFQS_CUDA_CHECK(cudaStreamWaitEvent(cstream, ready, 0));
   const uint64_t stage_amps = stage_bytes / amp_bytes;
   unsigned char* base = static_cast<unsigned char*>(shard);
   int c = 0;

@@ -29,8 +29,10 @@ struct Comm {
   Comm(int rank, int world, const uint8_t uid[128], size_t stage_bytes);
   ~Comm();
   // pieces are in amplitudes of `amp_bytes` bytes each.
+  // ready: the transfers wait for this event (NULL: for all work queued on `compute`);
+  // landed chunks are copied into place on `compute`.
   void exchange(void* shard, int amp_bytes, const std::vector<Piece>& pieces, int partner,
-                cudaStream_t compute);
+                cudaStream_t compute, cudaEvent_t ready = nullptr);
   void allreduce_sum(double* d, size_t count, cudaStream_t s);
 };
 

@@ -83,6 +83,12 @@ struct Options {
   bool lowq_shuffle = false;
   bool wide256 = true;       // two adjacent groups per item, 32-byte accesses
   bool line_reads = true;    // fixed bits 1-2 -> store predicate, whole-line reads (apply_kernels.cu)
+  // Global-qubit exchanges overlapped with local work (state.cu execute): the
+  // exchange is split into 2^exchange_chunk_bits parts by the top local qubits; the last
+  // local ops before it and the first after it run part by part on the compute stream
+  // while the parts move on the exchange stream.  0 bits: serial exchanges.
+  int exchange_chunk_bits = 2;
+  int exchange_ctas = 0;     // grid of the (device / P2P) exchange swap kernels; 0: full grid
   int fuse_tile_qubits = 12;
   int fuse_low_qubits = 0;   // contiguous low qubits of a fused tile (chunk = 2^L amps);
                              // 0: auto, 7 or 6 by planned pass count (fused_kernels.cu)
@@ -136,8 +142,10 @@ void launch_gate_soa(const LaunchCtx& ctx, const Decoded& g);
 // Half-shard swap for the global-qubit exchange: the l=1 half of the shard at
 // ctx.amps with the l=0 half of the shard partner_offset_amps further on (first
 // n_pairs pairs; 0 = all).
+// ctas > 0: a grid of at most that many CTAs (persistent grid-stride kernel) -- for
+// exchanges overlapped with local passes on another stream.
 void launch_half_swap(const LaunchCtx& ctx, int l, uint64_t partner_offset_amps,
-                      uint64_t n_pairs = 0);
+                      uint64_t n_pairs = 0, int ctas = 0);
 
 // Fused staging of gates[begin..): applies the longest prefix that fits one tile
 // program in one HBM pass; false if fewer than two gates fuse (fused_kernels.cu).

@@ -180,21 +180,23 @@ void P2P::barrier_all(cudaStream_t s) {
   LFQS_CUDA_CHECK(cudaGetLastError());
 }
 
-void P2P::exchange(const LaunchCtx& ctx, int l, int j, int n_local) {
+void P2P::exchange(const LaunchCtx& ctx, int l, int j, int n_sub, uint64_t offset, int ctas) {
   const int partner = rank ^ (1 << j);
   const int b = (rank >> j) & 1;
   const int low = b ? partner : rank, high = b ? rank : partner;
   const int ab = ctx.c64 ? 8 : 16;
+  require(l < n_sub && n_sub >= 2, "internal: exchange position outside the block");
   // Pairs (low[k | 2^l], high[k]) for k with bit l = 0.  The index bit hb splits
   // them: rank b swaps the pairs whose bit hb equals b.
-  const int hb = (l == n_local - 1) ? n_local - 2 : n_local - 1;
+  const int hb = (l == n_sub - 1) ? n_sub - 2 : n_sub - 1;
   const int64_t d = reinterpret_cast<intptr_t>(peer_amps[high]) -
                     reinterpret_cast<intptr_t>(peer_amps[low]);
   require(d % (2 * ab) == 0, "internal: peer shards are not 32-byte aligned");
-  barrier_pair(partner, ctx.stream);  // both shards are final up to here
+  barrier_pair(partner, ctx.stream);  // both blocks are final up to here
   LaunchCtx c = ctx;
-  c.amps = peer_amps[low] + ((uint64_t)b << hb) * ab;
-  launch_half_swap(c, l, (uint64_t)(d / ab), 1ull << (n_local - 2));
+  c.amps = peer_amps[low] + (offset + ((uint64_t)b << hb)) * ab;
+  c.n_local = n_sub;
+  launch_half_swap(c, l, (uint64_t)(d / ab), 1ull << (n_sub - 2), ctas);
   barrier_pair(partner, ctx.stream);  // both halves swapped before either moves on
 }
 

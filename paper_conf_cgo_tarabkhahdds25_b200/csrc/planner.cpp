@@ -168,8 +168,10 @@ void Planner::plan_gate(const Decoded& g, std::vector<PlanOp>& out,
       uint64_t tmask = 0;
       for (int u = 0; u < pg.m; ++u) tmask |= 1ull << pg.targets[u];
       int l = -1, best = -1;
-      const int lo = std::max(0, n_local - kSwapWindow);
-      for (int p = n_local - 1; p >= lo; --p) {
+      const int rsv = std::max(0, std::min(reserve_top, n_local - 4));
+      const int top = n_local - 1 - rsv;
+      const int lo = std::max(0, top + 1 - kSwapWindow);
+      for (int p = top; p >= lo; --p) {
         if (tmask >> p & 1) continue;
         const int score = next_use ? (*next_use)[p2l[p]] : 0;
         if (score > best) {
@@ -178,6 +180,8 @@ void Planner::plan_gate(const Decoded& g, std::vector<PlanOp>& out,
         }
       }
       for (int p = lo - 1; l < 0 && p >= 0; --p)
+        if (!(tmask >> p & 1)) l = p;
+      for (int p = n_local - 1; l < 0 && p > top; --p)  // only the reserved ones are left
         if (!(tmask >> p & 1)) l = p;
       require(l >= 0, "internal: no free local qubit");
       exchange(l, gq, out);

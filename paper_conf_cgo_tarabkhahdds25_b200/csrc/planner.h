@@ -39,6 +39,13 @@ struct Planner {
   // the one used furthest in the future (Belady), among the top kSwapWindow
   // local positions (so exchanged pieces stay >= 2^(n_local - kSwapWindow) amps).
   static constexpr int kSwapWindow = 8;
+  // The top reserve_top local positions are never chosen as the exchange position l by
+  // plan_gate: they are the chunk bits of overlapped exchanges (state.cu execute), which
+  // split an exchange into parts by them while the neighbouring local ops run part by part.
+  // kOverlapBits (Options::exchange_chunk_bits' default) whatever that option is, so serial
+  // and overlapped executions run the same plan; fewer for tiny shards.
+  static constexpr int kOverlapBits = 2;
+  int reserve_top = kOverlapBits;
   void plan_gate(const Decoded& g, std::vector<PlanOp>& out,
                  const std::vector<int>* next_use = nullptr);
   // Plans a whole circuit with Belady lookahead.

@@ -168,6 +168,9 @@ State::~State() {
   if (d_probs) cudaFree(d_probs);
   if (own_stream && stream) cudaStreamDestroy(stream);
   if (copy_stream) cudaStreamDestroy(copy_stream);
+  if (xstream) cudaStreamDestroy(xstream);
+  for (cudaEvent_t e : ev_tail) cudaEventDestroy(e);
+  for (cudaEvent_t e : ev_done) cudaEventDestroy(e);
 }
 
 void State::set_stream(cudaStream_t s) {
@@ -299,7 +302,7 @@ void State::exchange_data(int l, int g) {
       launch_half_swap(ctx(r), l, ((uint64_t)(r2 - r)) << n_local);
     }
   } else if (p2p) {
-    p2p->exchange(ctx(0), l, j, n_local);
+    p2p->exchange(ctx(0), l, j, n_local, 0, opt.exchange_ctas);
   } else {
     const int b = (rank >> j) & 1;
     std::vector<Piece> pieces;
@@ -334,29 +337,154 @@ void State::run_local(const LaunchCtx& c, const std::vector<Decoded>& gates, boo
   }
 }
 
+std::vector<Decoded> State::segment(const std::vector<PlanOp>& ops, size_t b, size_t e,
+                                    int shard) {
+  std::vector<Decoded> seg;
+  seg.reserve(e - b);
+  for (size_t k = b; k < e; ++k) {
+    Decoded lg;
+    if (plan.rank_local(ops[k].gate, rank_of_shard(shard), ops[k].gflip, &lg) &&
+        lg.cls != GClass::NOOP)
+      seg.push_back(lg);
+  }
+  return seg;
+}
+
+void State::run_range(const std::vector<PlanOp>& ops, size_t b, size_t e, bool fuse, int c,
+                      int v) {
+  if (b >= e) return;
+  for (int s = 0; s < n_shards(); ++s) {
+    LaunchCtx x = ctx(s);
+    if (c > 0) {
+      x.amps = static_cast<unsigned char*>(x.amps) + ((uint64_t)v << (n_local - c)) * ab;
+      x.n_local = n_local - c;
+    }
+    run_local(x, segment(ops, b, e, s), fuse);
+  }
+}
+
+int State::overlap_bits() const {
+  const int c = opt.exchange_chunk_bits;
+  if (world <= 1 || c <= 0 || n_local - c < 4) return 0;
+  return c;
+}
+
+cudaEvent_t State::part_event(std::vector<cudaEvent_t>& pool, int v) {
+  while ((int)pool.size() <= v) {
+    cudaEvent_t e = nullptr;
+    LFQS_CUDA_CHECK(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+    pool.push_back(e);
+  }
+  return pool[v];
+}
+
+cudaEvent_t State::exchange_part(int l, int g, int c, int v, cudaEvent_t ready) {
+  const int j = g - n_local, ns = n_local - c;
+  const uint64_t off = (uint64_t)v << ns;
+  if (virt || p2p) {
+    if (xstream == nullptr)
+      LFQS_CUDA_CHECK(cudaStreamCreateWithFlags(&xstream, cudaStreamNonBlocking));
+    LFQS_CUDA_CHECK(cudaStreamWaitEvent(xstream, ready, 0));
+    if (virt) {
+      for (int r = 0; r < world; ++r) {
+        if (r >> j & 1) continue;
+        const int r2 = r | (1 << j);
+        LaunchCtx x = ctx(r);
+        x.stream = xstream;
+        x.amps = static_cast<unsigned char*>(x.amps) + off * ab;
+        x.n_local = ns;
+        launch_half_swap(x, l, ((uint64_t)(r2 - r)) << n_local, 0, opt.exchange_ctas);
+      }
+    } else {
+      LaunchCtx x = ctx(0);
+      x.stream = xstream;
+      p2p->exchange(x, l, j, ns, off, opt.exchange_ctas);
+    }
+    cudaEvent_t done = part_event(ev_done, v);
+    LFQS_CUDA_CHECK(cudaEventRecord(done, xstream));
+    return done;
+  }
+  // NCCL: this part's half (local bit l = 1 - own global bit) as contiguous pieces.
+  const int b = (rank >> j) & 1;
+  std::vector<Piece> pieces;
+  if (l == ns - 1) {
+    pieces.push_back(Piece{off + ((uint64_t)(1 - b) << (ns - 1)), 1ull << (ns - 1)});
+  } else {
+    for (uint64_t hi = 0; hi < (1ull << (ns - 1 - l)); ++hi)
+      pieces.push_back(Piece{off + ((hi << (l + 1)) | ((uint64_t)(1 - b) << l)), 1ull << l});
+  }
+  comm->exchange(amps, ab, pieces, rank ^ (1 << j), stream, ready);
+  return nullptr;
+}
+
+// Global-qubit exchange overlapped with local work (BASELINE north_star
+// "overlapped with local work on separate streams").  The exchange moves data only inside
+// each block whose top c local bits are fixed (its position l is below them; the planner
+// reserves those bits, planner.h), so it splits into 2^c independent parts.  The last local
+// ops before it that do not touch the top c bits (tail [tb, te)) run part by part on the
+// compute stream; part v moves as soon as its tail is done, while the compute stream works
+// on the next part; the first local ops after the exchange that do not touch those bits
+// (head [hb, he)) run on part v as soon as it has landed.  Every op sees exactly the data
+// it would see in the serial order (Eq. 3: ops on disjoint blocks commute), and each
+// part runs the same kernels as the whole shard, so results equal the serial path's for the
+// same segmentation (tests/test_gpu_overlap.py).
+void State::overlapped_exchange(const std::vector<PlanOp>& ops, size_t tb, size_t te,
+                                const PlanOp& x, size_t hb, size_t he, bool fuse, int c) {
+  const int parts = 1 << c;
+  for (int v = 0; v < parts; ++v) {
+    run_range(ops, tb, te, fuse, c, v);
+    LFQS_CUDA_CHECK(cudaEventRecord(part_event(ev_tail, v), stream));
+  }
+  for (int v = 0; v < parts; ++v) {
+    cudaEvent_t done = exchange_part(x.l, x.g, c, v, part_event(ev_tail, v));
+    if (done) LFQS_CUDA_CHECK(cudaStreamWaitEvent(stream, done, 0));
+    run_range(ops, hb, he, fuse, c, v);
+  }
+  ++exchanges;
+  exchange_bytes += (uint64_t)ab << (n_local - 1);
+}
+
+namespace {
+// Does a physical op touch one of the top c local positions?
+bool touches_top(const Decoded& pg, int n_local, int c) {
+  const uint64_t H = ((1ull << c) - 1) << (n_local - c);
+  uint64_t m = pg.cmask;
+  for (int s = 0; s < pg.m; ++s) m |= 1ull << pg.targets[s];
+  return (m & H) != 0;
+}
+}  // namespace
+
 // Executes planned ops: maximal runs of LOCAL ops are rank-specialised per shard
-// and run (fused if requested); EXCHANGE ops move data between shards.
+// and run (fused if requested); EXCHANGE ops move data between shards -- overlapped with
+// the neighbouring local ops when Options::exchange_chunk_bits > 0 and the exchange
+// position lies below the chunk bits, serially otherwise.
 void State::execute(const std::vector<PlanOp>& ops, bool fuse) {
-  size_t i = 0;
-  while (i < ops.size()) {
-    if (ops[i].kind == PlanOp::EXCHANGE) {
-      exchange_data(ops[i].l, ops[i].g);
-      ++i;
+  std::vector<size_t> ex;
+  for (size_t i = 0; i < ops.size(); ++i)
+    if (ops[i].kind == PlanOp::EXCHANGE) ex.push_back(i);
+  const int c = overlap_bits();
+  size_t pos = 0;  // first op of the current run not yet executed (a head may be done)
+  for (size_t k = 0; k <= ex.size(); ++k) {
+    const size_t re = k < ex.size() ? ex[k] : ops.size();
+    if (k == ex.size()) {
+      run_range(ops, pos, re, fuse, 0, 0);
+      break;
+    }
+    const PlanOp& X = ops[ex[k]];
+    if (c == 0 || X.l >= n_local - c) {
+      run_range(ops, pos, re, fuse, 0, 0);
+      exchange_data(X.l, X.g);
+      pos = ex[k] + 1;
       continue;
     }
-    size_t j = i;
-    while (j < ops.size() && ops[j].kind == PlanOp::LOCAL) ++j;
-    for (int s = 0; s < n_shards(); ++s) {
-      std::vector<Decoded> seg;
-      seg.reserve(j - i);
-      for (size_t k = i; k < j; ++k) {
-        Decoded lg;
-        if (plan.rank_local(ops[k].gate, rank_of_shard(s), ops[k].gflip, &lg) && lg.cls != GClass::NOOP)
-          seg.push_back(lg);
-      }
-      run_local(ctx(s), seg, fuse);
-    }
-    i = j;
+    size_t ts = re;
+    while (ts > pos && !touches_top(ops[ts - 1].gate, n_local, c)) --ts;
+    run_range(ops, pos, ts, fuse, 0, 0);  // the body of the run
+    const size_t hb = ex[k] + 1, ne = k + 1 < ex.size() ? ex[k + 1] : ops.size();
+    size_t he = hb;
+    while (he < ne && !touches_top(ops[he].gate, n_local, c)) ++he;
+    overlapped_exchange(ops, ts, re, X, hb, he, fuse, c);
+    pos = he;
   }
 }
 

@@ -44,6 +44,19 @@ def worker(rank, world, port, n, seed, out_q):
                 report[f"exact{key}"] = bool(np.array_equal(st.copy_out()[lo:hi],
                                                                    ref_exact[lo:hi]))
                 st.synchronize()
+        # exchanges overlapped with local work (chunk bits 2, the default; also with a
+        # grid-limited swap kernel) vs serial exchanges (chunk bits 0): the same plan and
+        # the same kernels per amplitude, so the same bits
+        outs = []
+        for bits, ctas in ((0, 0), (2, 0), (2, 8)):
+            with L.State.p2p(n, rank, world) as st:
+                st.set_option(L.OPT_EXCHANGE_CHUNK_BITS, bits)
+                st.set_option(L.OPT_EXCHANGE_CTAS, ctas)
+                st.copy_in(psi)
+                st.run_circuit(gates)
+                outs.append(st.copy_out()[lo:hi])
+        report["overlap"] = (all(np.array_equal(outs[0], o) for o in outs[1:]),
+                             float(np.max(np.abs(outs[1] - ref[lo:hi]))))
         # one gate at a time through lfqs_apply_gate (planner per gate, exchanges included)
         with L.State.p2p(n, rank, world) as st:
             st.copy_in(psi)

@@ -1,0 +1,97 @@
+"""Global-qubit exchanges overlapped with local work (BASELINE
+north_star "overlapped with local work on separate streams"), on the single-GPU virtual
+partition: the exchange is split into 2^c parts by the top c local qubits, moved on an
+exchange stream while the neighbouring local ops run part by part (state.cu
+overlapped_exchange).  Unfused runs apply exactly the same kernels per amplitude as the
+serial path, so they are bit-identical to it; fused runs may cut passes differently
+(rounding only) and are held to the oracle (<= 1e-12; permutation/diagonal circuits
+bit-exact)."""
+import numpy as np
+import pytest
+
+import oracle as O
+import workloads as W
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def L():
+    import torch
+    if not torch.cuda.is_available():
+        pytest.skip("needs a GPU")
+    import paper_conf_cgo_tarabkhahdds25_b200 as lib
+    lib.lib()
+    return lib
+
+
+def _run(L, n, world, psi, gates, fuse, bits, ctas=0):
+    with L.State.virtual(n, world) as st:
+        st.set_option(L.OPT_EXCHANGE_CHUNK_BITS, bits)
+        st.set_option(L.OPT_EXCHANGE_CTAS, ctas)
+        st.copy_in(psi)
+        x0 = st.exchange_stats()[0]
+        st.run_circuit(gates, fuse=fuse)
+        nx = st.exchange_stats()[0] - x0
+        out = st.copy_out()
+        probs = st.measure_probs([n - 1, 1])
+    return out, probs, nx
+
+
+@pytest.mark.parametrize("world", [2, 4, 8])
+def test_overlap_unfused_bit_identical_to_serial(L, world):
+    """The plan does not depend on the chunk bits (the planner always keeps the top two
+    local positions free), so chunk bits 0 (serial exchanges), 1, 2 (default), 3 (an
+    exchange at position n_local - 3 falls back to serial) and a grid-limited swap kernel
+    all run the same plan; unfused they apply the same kernels per amplitude: bit-identical."""
+    n = 14
+    psi = W.random_state(n, 31 + world)
+    gates = (W.random_gate_list(n, 160, seed=70 + world, max_controls=2) + W.qft(n) +
+             W.random_layered(n, 3, seed=world))
+    ref = O.run_circuit(n, gates, psi.copy())
+    serial, ps, nx0 = _run(L, n, world, psi, gates, False, 0)
+    assert nx0 > 0
+    assert np.max(np.abs(serial - ref)) <= 1e-12
+    for bits, ctas in ((2, 0), (2, 8), (1, 0), (3, 3)):
+        out, probs, nx = _run(L, n, world, psi, gates, False, bits, ctas)
+        assert nx == nx0
+        assert np.array_equal(out, serial), (bits, ctas)
+        assert np.array_equal(probs, ps), (bits, ctas)
+
+
+@pytest.mark.parametrize("fuse", [True, "jit", "jit+phase"])
+@pytest.mark.parametrize("world", [2, 8])
+def test_overlap_fused_vs_oracle(L, world, fuse):
+    n = 16
+    psi = W.random_state(n, 9)
+    gates = W.random_gate_list(n, 200, seed=world, max_controls=2) + W.qft(n)
+    ref = O.run_circuit(n, gates, psi.copy())
+    exact = [g for g in W.random_gate_list(n, 300, seed=world + 1, max_controls=2) if g.exact]
+    ref_exact = O.run_circuit(n, exact, psi.copy())
+    for bits in (0, 2, 3):
+        out, probs, _ = _run(L, n, world, psi, gates, fuse, bits)
+        assert np.max(np.abs(out - ref)) <= 1e-12, bits
+        np.testing.assert_allclose(probs, O.probs(n, ref, [n - 1, 1]), rtol=1e-12, atol=1e-15)
+        if fuse != "jit+phase":
+            out, _, _ = _run(L, n, world, psi, exact, fuse, bits)
+            assert np.array_equal(out, ref_exact), bits
+
+
+def test_overlap_graph_capture_and_per_gate_apply(L):
+    """The exchange stream forks from and joins the capturing stream (lfqs_circuit_compile
+    on a virtual partition), and per-gate lfqs_apply_gate overlaps its own exchange."""
+    n, world = 14, 4
+    psi = W.random_state(n, 77)
+    gates = W.qft(n) + W.random_gate_list(n, 60, seed=2, max_controls=1)
+    ref = O.run_circuit(n, gates, psi.copy())
+    with L.State.virtual(n, world) as st:
+        st.set_option(L.OPT_EXCHANGE_CTAS, 16)
+        st.copy_in(psi)
+        with st.compile(gates) as c:
+            c.launch()
+            got = st.copy_out()
+        assert np.max(np.abs(got - ref)) <= 1e-12
+        st.copy_in(psi)
+        for g in gates:
+            st.apply(g)
+        assert np.max(np.abs(st.copy_out() - ref)) <= 1e-12

@@ -51,5 +51,7 @@ def test_p2p_sharded_circuits(world):
             assert err <= 1e-12 and perr <= 1e-12, (rank, fuse, err, perr)
             assert payload[f"exact{fuse}"], (rank, fuse)
         assert payload["apply"] <= 1e-12
+        same, err = payload["overlap"]
+        assert same and err <= 1e-12, (rank, same, err)
         same, err = payload["streamed"]
         assert same and err <= 1e-12, (rank, same, err)

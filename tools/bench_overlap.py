@@ -1,0 +1,95 @@
+"""Exchange/compute overlap on one GPU: a virtual partition into `world` shards
+runs a circuit with serial exchanges (LFQS_OPT_EXCHANGE_CHUNK_BITS = 0) and overlapped
+ones (2^c parts on an exchange stream while the neighbouring local passes run part by part),
+with the exchange swap kernel's grid limited to `ctas` CTAs -- a small grid moves the
+exchange at a link-like rate (NVLink 5: ~0.9 TB/s per direction, an eighth of HBM) and
+leaves the SMs to the local passes, which is what an exchange over NVLink looks like to
+the GPU.  The same circuit on an unsharded state (world = 1) gives the local work alone.
+
+    python tools/bench_overlap.py --n 32 --world 4 --circuit qft --ctas 0,16,8
+
+Prints one JSON object per (ctas, chunk bits): ms, exchanges, exposed exchange time
+(ms - unsharded ms) and the fraction of the serial exchange time hidden by overlapping.
+"""
+import argparse
+import json
+import os
+import sys
+import time
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+
+import workloads as W  # noqa: E402
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--n", type=int, default=32)
+    ap.add_argument("--world", type=int, default=4)
+    ap.add_argument("--circuit", default="qft")
+    ap.add_argument("--mode", default="jit+phase")
+    ap.add_argument("--ctas", default="0,32,16,8")
+    ap.add_argument("--bits", default="0,1,2,3")
+    ap.add_argument("--reps", type=int, default=3)
+    args = ap.parse_args()
+    import torch
+    import paper_conf_cgo_tarabkhahdds25_b200 as L
+    s = torch.cuda.Stream()
+    torch.cuda.set_stream(s)
+    n = args.n
+    x = int(W.SplitMix64(n).next_u64() & ((1 << n) - 1))
+    gates = {"qft": W.qft(n), "random": W.random_layered(n, 20, seed=7),
+             "grover": W.grover(n, x, 1), "ghz": W.ghz(n)}[args.circuit]
+    flags = {"unfused": L.FUSE_NONE, "fused": L.FUSE_LOW, "jit": L.FUSE_LOW | L.FUSE_JIT,
+             "jit+phase": L.FUSE_LOW | L.FUSE_JIT | L.FUSE_PHASE}[args.mode]
+    arr = L.marshal_gates(gates)
+
+    def timed(st):
+        best = 1e30
+        for r in range(args.reps + 1):
+            st.init_basis(x if args.circuit == "qft" else 0)
+            torch.cuda.synchronize()
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record(s)
+            L.lfqs_run_circuit(st.h, arr, flags)
+            e1.record(s)
+            torch.cuda.synchronize()
+            if r > 0:
+                best = min(best, e0.elapsed_time(e1))
+        return best
+
+    with L.State.create(n, 0, stream=s) as st:
+        if flags & L.FUSE_JIT:
+            L.lfqs_jit_precompile(n, arr, flags)
+        t1 = timed(st)
+    print(json.dumps({"circuit": args.circuit, "mode": args.mode, "n": n, "world": 1,
+                      "ms": round(t1, 3)}), flush=True)
+    with L.State.virtual(n, args.world, 0, stream=s) as st:
+        if flags & L.FUSE_JIT:  # compile every pass shape outside the timed region
+            for b in [int(v) for v in args.bits.split(",")]:
+                st.set_option(L.OPT_EXCHANGE_CHUNK_BITS, b)
+                st.init_basis(0)
+                L.lfqs_run_circuit(st.h, arr, flags)
+            torch.cuda.synchronize()
+        for ctas in [int(v) for v in args.ctas.split(",")]:
+            st.set_option(L.OPT_EXCHANGE_CTAS, ctas)
+            serial = None
+            for b in [int(v) for v in args.bits.split(",")]:
+                st.set_option(L.OPT_EXCHANGE_CHUNK_BITS, b)
+                x0 = st.exchange_stats()[0]
+                t = timed(st)
+                nx = (st.exchange_stats()[0] - x0) // (args.reps + 1)
+                rec = {"circuit": args.circuit, "mode": args.mode, "n": n, "world": args.world,
+                       "exchange_ctas": ctas, "chunk_bits": b, "ms": round(t, 3),
+                       "exchanges": int(nx), "unsharded_ms": round(t1, 3),
+                       "exposed_exchange_ms": round(t - t1, 3)}
+                if b == 0:
+                    serial = t
+                elif serial is not None and serial > t1:
+                    rec["hidden_frac"] = round((serial - t) / (serial - t1), 3)
+                print(json.dumps(rec), flush=True)
+
+
+if __name__ == "__main__":
+    main()
