@@ -1034,8 +1034,14 @@ bool run_fused_circuit(const LaunchCtx& ctx, const std::vector<Decoded>& gates, 
 // a shared amplitude would round differently in the other order).  Permutation /
 // diagonal results therefore stay bit-identical to gate-by-gate application;
 // dense gates reorder only across disjoint qubits (rounding-level differences).
-void run_fused_schedule(const LaunchCtx& ctx_in, const std::vector<Decoded>& gates,
-                        int tile_qubits) {
+//
+// plan_fused_schedule builds the passes (and, for LFQS_FUSE_JIT, compiles them) without
+// launching anything; launch_fused_pass runs one of them on any block of the state whose
+// qubits include every qubit the pass touches (the executor runs boundary passes of an
+// overlapped exchange part by part, state.cu).
+void plan_fused_schedule(const LaunchCtx& ctx_in, const std::vector<Decoded>& gates,
+                         int tile_qubits, std::vector<FusedPass>& out) {
+  out.clear();
   // LFQS_OPT_FUSE_LOW_QUBITS = 0 (auto): plan the passes (host only) with 7 and with 6
   // contiguous low qubits per tile and take 6 only when it saves >= 20 % of the passes --
   // a 1-KiB-chunk tile costs ~10 % more per pass (twice the TMA copies) but claims one
@@ -1052,7 +1058,8 @@ void run_fused_schedule(const LaunchCtx& ctx_in, const std::vector<Decoded>& gat
       pc.opt = &o;
       pc.plan_only = true;
       pc.launch_counter = &c;
-      run_fused_schedule(pc, gates, tile_qubits);
+      std::vector<FusedPass> tmp;
+      plan_fused_schedule(pc, gates, tile_qubits, tmp);
       return c;
     };
     const uint64_t p7 = count(7), p6 = count(6);
@@ -1064,28 +1071,21 @@ void run_fused_schedule(const LaunchCtx& ctx_in, const std::vector<Decoded>& gat
   std::vector<int> rest;
   for (size_t i = 0; i < gates.size(); ++i)
     if (gates[i].cls != GClass::NOOP) rest.push_back((int)i);
+  auto single = [&](int gi) {
+    FusedPass ps;
+    ps.gate = gi;
+    ps.qmask = qubit_mask(gates[gi]);
+    out.push_back(std::move(ps));
+  };
   if (!tile_cfg(ctx, tile_qubits, &cfg)) {
-    if (ctx.plan_only || ctx.dry_run) {  // host-only callers (lfqs_jit_precompile): no launch
+    if (ctx.plan_only) {
       *ctx.launch_counter += rest.size();
       return;
     }
-    for (int i : rest) launch_gate(ctx, gates[i]);
+    for (int i : rest) single(i);
     return;
   }
-  // LFQS_FUSE_JIT: passes are planned first, compiled in parallel, then launched.
-  struct Pass {
-    int gate = -1;                 // single-gate pass (class kernel)
-    std::unique_ptr<FProg> prog;   // fused pass
-    std::string key;
-  };
-  std::vector<Pass> passes;
-  const bool collect = ctx.jit && (1 << (cfg.K - cfg.L)) <= ctx.opt->fuse_tma_max_chunks;
-  if (ctx.dry_run && !collect && !ctx.plan_only) {  // nothing to compile: count passes only
-    LaunchCtx pc = ctx;
-    pc.plan_only = true;
-    run_fused_schedule(pc, gates, tile_qubits);
-    return;
-  }
+  const bool jit_ok = ctx.jit && (1 << (cfg.K - cfg.L)) <= ctx.opt->fuse_tma_max_chunks;
   constexpr size_t kWindow = 4096;  // gates scanned per pass
   const int max_ops = ctx.phase_tables ? kMaxOps - 16 : kMaxOps;  // room for F_DTAB headers
   std::vector<char> taken(gates.size(), 0);
@@ -1137,41 +1137,45 @@ void run_fused_schedule(const LaunchCtx& ctx_in, const std::vector<Decoded>& gat
     } else if (nops < 2) {
       // Nothing to fuse with the first remaining gate: its class kernel.
       while (taken[rest[head]]) ++head;
-      if (collect) {
-        passes.emplace_back();
-        passes.back().gate = rest[head];
-      } else {
-        launch_gate(ctx, gates[rest[head]]);
-      }
+      single(rest[head]);
       taken[rest[head]] = 1;
     } else {
-      if (collect) {
-        passes.emplace_back();
-        passes.back().prog.reset(new FProg);
-        build_program(ctx, cfg, in_tile, list, *passes.back().prog);
-        passes.back().key = jit_key(*passes.back().prog, cfg.K, ctx.c64, jit_config(ctx, cfg.K));
-      } else {
-        launch_program(ctx, cfg, in_tile, list);
-      }
+      FusedPass ps;
+      ps.prog.reset(new FProg);
+      ps.K = cfg.K;
+      build_program(ctx, cfg, in_tile, list, *ps.prog);
+      for (int gi : picked) ps.qmask |= qubit_mask(gates[gi]);
+      if (jit_ok) ps.key = jit_key(*ps.prog, cfg.K, ctx.c64, jit_config(ctx, cfg.K));
+      out.push_back(std::move(ps));
       for (int gi : picked) taken[gi] = 1;
     }
     while (head < rest.size() && taken[rest[head]]) ++head;
   }
-  if (!collect || ctx.plan_only) return;
+  if (ctx.plan_only || !jit_ok) return;
   std::vector<std::pair<std::string, const FProg*>> items;
-  for (const Pass& ps : passes)
+  for (const FusedPass& ps : out)
     if (ps.prog) items.emplace_back(ps.key, ps.prog.get());
   jit_compile(items, cfg.K, ctx.c64, jit_config(ctx, cfg.K));
-  if (ctx.dry_run) {
+}
+
+void launch_fused_pass(const LaunchCtx& ctx, const std::vector<Decoded>& gates,
+                       const FusedPass& ps) {
+  if (ps.prog)
+    launch_built(ctx, ps.K, *ps.prog, ps.key.empty() ? nullptr : &ps.key);
+  else
+    launch_gate(ctx, gates[ps.gate]);
+}
+
+void run_fused_schedule(const LaunchCtx& ctx, const std::vector<Decoded>& gates,
+                        int tile_qubits) {
+  std::vector<FusedPass> passes;
+  plan_fused_schedule(ctx, gates, tile_qubits, passes);
+  if (ctx.plan_only) return;
+  if (ctx.dry_run) {  // host-only (lfqs_jit_precompile): planned and compiled, not launched
     *ctx.launch_counter += passes.size();
     return;
   }
-  for (const Pass& ps : passes) {
-    if (ps.prog)
-      launch_built(ctx, cfg.K, *ps.prog, &ps.key);
-    else
-      launch_gate(ctx, gates[ps.gate]);
-  }
+  for (const FusedPass& ps : passes) launch_fused_pass(ctx, gates, ps);
 }
 
 }  // namespace lfqs

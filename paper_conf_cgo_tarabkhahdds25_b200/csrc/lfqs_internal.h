@@ -5,6 +5,7 @@
 #include <cuda_runtime.h>
 
 #include <cstdint>
+#include <memory>
 #include <stdexcept>
 #include <string>
 #include <vector>
@@ -153,6 +154,23 @@ bool run_fused_circuit(const LaunchCtx& ctx, const std::vector<Decoded>& gates, 
                        size_t end, int tile_qubits, size_t* consumed);
 // Whole-list fused execution with exact-commutation reordering (fused_kernels.cu).
 void run_fused_schedule(const LaunchCtx& ctx, const std::vector<Decoded>& gates, int tile_qubits);
+
+// One pass of a fused schedule: a single gate's class kernel or a fused tile program.
+struct FProg;  // fused_prog.h
+struct FusedPass {
+  int gate = -1;                 // single-gate pass: index into the gate list
+  std::shared_ptr<FProg> prog;   // fused pass (tile program)
+  std::string key;               // compiled-pass cache key (LFQS_FUSE_JIT), else empty
+  int K = 0;                     // tile qubits of prog
+  uint64_t qmask = 0;            // qubits the pass's gates touch (targets | controls)
+};
+// Plans (and for LFQS_FUSE_JIT compiles) the passes run_fused_schedule would launch.
+void plan_fused_schedule(const LaunchCtx& ctx, const std::vector<Decoded>& gates, int tile_qubits,
+                         std::vector<FusedPass>& out);
+// Launches one planned pass on ctx: the whole shard, or any block of it (amps offset,
+// n_local) that contains every qubit in ps.qmask.
+void launch_fused_pass(const LaunchCtx& ctx, const std::vector<Decoded>& gates,
+                       const FusedPass& ps);
 
 // Reductions (C9): d_out[v], v < 2^nq (nq <= 20, bit s of v = bit qubits[s]); one read
 // pass over the shard whatever nq is; deterministic (fixed grid and summation order).

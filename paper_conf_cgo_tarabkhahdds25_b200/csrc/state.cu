@@ -350,16 +350,38 @@ std::vector<Decoded> State::segment(const std::vector<PlanOp>& ops, size_t b, si
   return seg;
 }
 
-void State::run_range(const std::vector<PlanOp>& ops, size_t b, size_t e, bool fuse, int c,
-                      int v) {
-  if (b >= e) return;
+std::vector<State::ShardRun> State::plan_run(const std::vector<PlanOp>& ops, size_t b, size_t e,
+                                             bool fuse) {
+  std::vector<ShardRun> run(n_shards());
   for (int s = 0; s < n_shards(); ++s) {
+    ShardRun& r = run[s];
+    r.seg = segment(ops, b, e, s);
+    if (fuse) {
+      plan_fused_schedule(ctx(s), r.seg, opt.fuse_tile_qubits, r.passes);
+    } else {  // one pass per gate (LFQS_FUSE_NONE)
+      for (size_t i = 0; i < r.seg.size(); ++i) {
+        FusedPass ps;
+        ps.gate = (int)i;
+        uint64_t m = r.seg[i].cmask;
+        for (int t = 0; t < r.seg[i].m; ++t) m |= 1ull << r.seg[i].targets[t];
+        ps.qmask = m;
+        r.passes.push_back(std::move(ps));
+      }
+    }
+  }
+  return run;
+}
+
+void State::launch_passes(const std::vector<ShardRun>& run, const std::vector<size_t>& from,
+                          const std::vector<size_t>& to, int c, int v) {
+  for (int s = 0; s < n_shards(); ++s) {
+    if (from[s] >= to[s]) continue;
     LaunchCtx x = ctx(s);
     if (c > 0) {
       x.amps = static_cast<unsigned char*>(x.amps) + ((uint64_t)v << (n_local - c)) * ab;
       x.n_local = n_local - c;
     }
-    run_local(x, segment(ops, b, e, s), fuse);
+    for (size_t i = from[s]; i < to[s]; ++i) launch_fused_pass(x, run[s].seg, run[s].passes[i]);
   }
 }
 
@@ -417,74 +439,80 @@ cudaEvent_t State::exchange_part(int l, int g, int c, int v, cudaEvent_t ready) 
   return nullptr;
 }
 
+// Executes planned ops: maximal runs of LOCAL ops are rank-specialised per shard and
+// planned into passes (fused if requested); EXCHANGE ops move data between shards.
+//
 // Global-qubit exchange overlapped with local work (BASELINE north_star
-// "overlapped with local work on separate streams").  The exchange moves data only inside
-// each block whose top c local bits are fixed (its position l is below them; the planner
-// reserves those bits, planner.h), so it splits into 2^c independent parts.  The last local
-// ops before it that do not touch the top c bits (tail [tb, te)) run part by part on the
-// compute stream; part v moves as soon as its tail is done, while the compute stream works
-// on the next part; the first local ops after the exchange that do not touch those bits
-// (head [hb, he)) run on part v as soon as it has landed.  Every op sees exactly the data
-// it would see in the serial order (Eq. 3: ops on disjoint blocks commute), and each
-// part runs the same kernels as the whole shard, so results equal the serial path's for the
-// same segmentation (tests/test_gpu_overlap.py).
-void State::overlapped_exchange(const std::vector<PlanOp>& ops, size_t tb, size_t te,
-                                const PlanOp& x, size_t hb, size_t he, bool fuse, int c) {
-  const int parts = 1 << c;
-  for (int v = 0; v < parts; ++v) {
-    run_range(ops, tb, te, fuse, c, v);
-    LFQS_CUDA_CHECK(cudaEventRecord(part_event(ev_tail, v), stream));
-  }
-  for (int v = 0; v < parts; ++v) {
-    cudaEvent_t done = exchange_part(x.l, x.g, c, v, part_event(ev_tail, v));
-    if (done) LFQS_CUDA_CHECK(cudaStreamWaitEvent(stream, done, 0));
-    run_range(ops, hb, he, fuse, c, v);
-  }
-  ++exchanges;
-  exchange_bytes += (uint64_t)ab << (n_local - 1);
-}
-
-namespace {
-// Does a physical op touch one of the top c local positions?
-bool touches_top(const Decoded& pg, int n_local, int c) {
-  const uint64_t H = ((1ull << c) - 1) << (n_local - c);
-  uint64_t m = pg.cmask;
-  for (int s = 0; s < pg.m; ++s) m |= 1ull << pg.targets[s];
-  return (m & H) != 0;
-}
-}  // namespace
-
-// Executes planned ops: maximal runs of LOCAL ops are rank-specialised per shard
-// and run (fused if requested); EXCHANGE ops move data between shards -- overlapped with
-// the neighbouring local ops when Options::exchange_chunk_bits > 0 and the exchange
-// position lies below the chunk bits, serially otherwise.
+// "overlapped with local work on separate streams"), Options::exchange_chunk_bits = c > 0:
+// an exchange at a position l below the top c local qubits (the planner keeps exchange
+// positions out of the top two, planner.h) moves data only inside each block whose top c
+// bits are fixed, so it splits into 2^c independent parts.  The trailing passes of the run
+// before it that touch none of those c qubits run part by part on the compute stream; part
+// v moves (exchange stream, or the NCCL stream) as soon as its tail is done, while the
+// compute stream goes on with the next part; the leading passes of the next run that touch
+// none of them run on part v as soon as it has landed.  The passes are exactly the ones the
+// serial execution launches (no extra HBM pass), each applied block by block with the same
+// kernels, and every pass sees the data it would see in the serial order (Eq. 3; ops
+// on disjoint blocks commute): results are bit-identical to serial exchanges
+// (tests/test_gpu_overlap.py, tests/test_gpu_p2p.py).  Other exchanges (position among the
+// top c, e.g. during canonicalisation) run serially.
 void State::execute(const std::vector<PlanOp>& ops, bool fuse) {
   std::vector<size_t> ex;
   for (size_t i = 0; i < ops.size(); ++i)
     if (ops[i].kind == PlanOp::EXCHANGE) ex.push_back(i);
+  if (fuse && !opt.fuse_reorder) {  // prefix fusion (a tuning mode): serial, run by run
+    size_t i = 0;
+    for (size_t k = 0; k <= ex.size(); ++k) {
+      const size_t e = k < ex.size() ? ex[k] : ops.size();
+      for (int s = 0; s < n_shards(); ++s) run_local(ctx(s), segment(ops, i, e, s), true);
+      if (k < ex.size()) exchange_data(ops[e].l, ops[e].g);
+      i = e + 1;
+    }
+    return;
+  }
   const int c = overlap_bits();
-  size_t pos = 0;  // first op of the current run not yet executed (a head may be done)
-  for (size_t k = 0; k <= ex.size(); ++k) {
-    const size_t re = k < ex.size() ? ex[k] : ops.size();
+  const uint64_t H = c > 0 ? ((1ull << c) - 1) << (n_local - c) : 0;
+  const int S = n_shards();
+  std::vector<ShardRun> cur = plan_run(ops, 0, ex.empty() ? ops.size() : ex[0], fuse);
+  std::vector<size_t> from(S, 0), end(S);
+  for (size_t k = 0;; ++k) {
+    for (int s = 0; s < S; ++s) end[s] = cur[s].passes.size();
     if (k == ex.size()) {
-      run_range(ops, pos, re, fuse, 0, 0);
+      launch_passes(cur, from, end, 0, 0);
       break;
     }
     const PlanOp& X = ops[ex[k]];
+    const size_t nb = ex[k] + 1, ne = k + 1 < ex.size() ? ex[k + 1] : ops.size();
+    std::vector<ShardRun> next = plan_run(ops, nb, ne, fuse);
     if (c == 0 || X.l >= n_local - c) {
-      run_range(ops, pos, re, fuse, 0, 0);
+      launch_passes(cur, from, end, 0, 0);
       exchange_data(X.l, X.g);
-      pos = ex[k] + 1;
+      cur = std::move(next);
+      std::fill(from.begin(), from.end(), 0);
       continue;
     }
-    size_t ts = re;
-    while (ts > pos && !touches_top(ops[ts - 1].gate, n_local, c)) --ts;
-    run_range(ops, pos, ts, fuse, 0, 0);  // the body of the run
-    const size_t hb = ex[k] + 1, ne = k + 1 < ex.size() ? ex[k + 1] : ops.size();
-    size_t he = hb;
-    while (he < ne && !touches_top(ops[he].gate, n_local, c)) ++he;
-    overlapped_exchange(ops, ts, re, X, hb, he, fuse, c);
-    pos = he;
+    // tail: trailing passes free of the chunk bits; head: leading ones of the next run
+    std::vector<size_t> ts(S), he(S, 0), zero(S, 0);
+    for (int s = 0; s < S; ++s) {
+      ts[s] = end[s];
+      while (ts[s] > from[s] && !(cur[s].passes[ts[s] - 1].qmask & H)) --ts[s];
+      while (he[s] < next[s].passes.size() && !(next[s].passes[he[s]].qmask & H)) ++he[s];
+    }
+    launch_passes(cur, from, ts, 0, 0);  // the body of the run
+    const int parts = 1 << c;
+    for (int v = 0; v < parts; ++v) {
+      launch_passes(cur, ts, end, c, v);
+      LFQS_CUDA_CHECK(cudaEventRecord(part_event(ev_tail, v), stream));
+    }
+    for (int v = 0; v < parts; ++v) {
+      cudaEvent_t done = exchange_part(X.l, X.g, c, v, part_event(ev_tail, v));
+      if (done) LFQS_CUDA_CHECK(cudaStreamWaitEvent(stream, done, 0));
+      launch_passes(next, zero, he, c, v);
+    }
+    ++exchanges;
+    exchange_bytes += (uint64_t)ab << (n_local - 1);
+    cur = std::move(next);
+    from = he;
   }
 }
 

@@ -93,15 +93,20 @@ struct State : lfqs_state {
   int overlap_bits() const;
   cudaEvent_t part_event(std::vector<cudaEvent_t>& pool, int v);
   std::vector<Decoded> segment(const std::vector<PlanOp>& ops, size_t b, size_t e, int shard);
-  // Runs LOCAL ops [b, e) on every shard, whole (c = 0) or on part v of 2^c (the block
-  // whose top c local bits equal v; the ops must not touch those bits).
-  void run_range(const std::vector<PlanOp>& ops, size_t b, size_t e, bool fuse, int c, int v);
+  // A run of LOCAL ops planned into passes, per shard (rank-specialised gates + passes).
+  struct ShardRun {
+    std::vector<Decoded> seg;
+    std::vector<FusedPass> passes;
+  };
+  std::vector<ShardRun> plan_run(const std::vector<PlanOp>& ops, size_t b, size_t e, bool fuse);
+  // Launches passes [from[s], to[s]) of every shard, on the whole shard (c = 0) or on part
+  // v of 2^c (the block whose top c local bits equal v; the passes do not touch them).
+  void launch_passes(const std::vector<ShardRun>& run, const std::vector<size_t>& from,
+                     const std::vector<size_t>& to, int c, int v);
   // One part of an exchange; the data it moves is final once `ready` has fired.  Returns
   // the event the compute stream must wait for before using the part (NULL: the copies
   // already sit on the compute stream, NCCL transport).
   cudaEvent_t exchange_part(int l, int g, int c, int v, cudaEvent_t ready);
-  void overlapped_exchange(const std::vector<PlanOp>& ops, size_t tb, size_t te, const PlanOp& x,
-                           size_t hb, size_t he, bool fuse, int c);
   int n_shards() const { return virt ? world : 1; }
   int rank_of_shard(int shard) const { return virt ? shard : rank; }
   void execute(const std::vector<PlanOp>& ops, bool fuse);

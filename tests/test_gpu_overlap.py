@@ -3,9 +3,9 @@ north_star "overlapped with local work on separate streams"), on the single-GPU 
 partition: the exchange is split into 2^c parts by the top c local qubits, moved on an
 exchange stream while the neighbouring local ops run part by part (state.cu
 overlapped_exchange).  Unfused runs apply exactly the same kernels per amplitude as the
-serial path, so they are bit-identical to it; fused runs may cut passes differently
-(rounding only) and are held to the oracle (<= 1e-12; permutation/diagonal circuits
-bit-exact)."""
+serial path, and fused runs launch exactly the serial run's passes block by block, so
+both are bit-identical to serial exchanges; all are held to the oracle (<= 1e-12;
+permutation/diagonal circuits bit-exact)."""
 import numpy as np
 import pytest
 
@@ -68,10 +68,15 @@ def test_overlap_fused_vs_oracle(L, world, fuse):
     ref = O.run_circuit(n, gates, psi.copy())
     exact = [g for g in W.random_gate_list(n, 300, seed=world + 1, max_controls=2) if g.exact]
     ref_exact = O.run_circuit(n, exact, psi.copy())
+    serial = None
     for bits in (0, 2, 3):
         out, probs, _ = _run(L, n, world, psi, gates, fuse, bits)
         assert np.max(np.abs(out - ref)) <= 1e-12, bits
         np.testing.assert_allclose(probs, O.probs(n, ref, [n - 1, 1]), rtol=1e-12, atol=1e-15)
+        if serial is None:
+            serial = out
+        else:  # the overlapped run launches the serial run's passes, block by block
+            assert np.array_equal(out, serial), bits
         if fuse != "jit+phase":
             out, _, _ = _run(L, n, world, psi, exact, fuse, bits)
             assert np.array_equal(out, ref_exact), bits
