@@ -39,6 +39,7 @@
 #include "cx.cuh"
 #include "fused_prog.h"
 #include "jit.h"
+#include "planner.h"
 #include "lfqs_internal.h"
 
 namespace lfqs {
@@ -382,6 +383,7 @@ __device__ __forceinline__ uint64_t tile_addr(const FTile& tg, uint64_t base, ui
 // (profiles/r01_c64_occupancy.md).
 template <int K, bool DIRECT, class S>
 __global__ void __launch_bounds__(kFThreads, sizeof(S) == 4 ? 4 : 2) k_fused(cx<S>* __restrict__ a,
+                                                        uint64_t tile_off,
                                                         const __grid_constant__ FProg prog) {
   using C = cx<S>;
   constexpr uint32_t T = 1u << K;
@@ -394,7 +396,7 @@ __global__ void __launch_bounds__(kFThreads, sizeof(S) == 4 ? 4 : 2) k_fused(cx<
   const FTile& tg = prog.tile;
   const int lc = tg.lc, nh = tg.nh;
   // Tile base: the tile index with zeros inserted at every tile qubit.
-  uint64_t base = (uint64_t)blockIdx.x << lc;
+  uint64_t base = ((uint64_t)blockIdx.x + tile_off) << lc;  // tile_off: first tile of a block
   for (int i = 0; i < nh; ++i) {
     const int p = tg.hpos[i];
     const uint64_t lo = base & ((1ull << p) - 1);
@@ -742,28 +744,28 @@ void encode(const Decoded& g, const TileMap& tm, FProg& P) {
 }
 
 template <int K, bool DIRECT, class S>
-void launch_kd(const LaunchCtx& ctx, const FProg& P) {
+void launch_kd(const LaunchCtx& ctx, const FProg& P, uint64_t tile_off) {
   const size_t smem = sizeof(cx<S>) << K;
   ensure_smem_attr((const void*)k_fused<K, DIRECT, S>, (int)smem);
   const uint64_t tiles = 1ull << (ctx.n_local - K);
   k_fused<K, DIRECT, S><<<(unsigned)tiles, kFThreads, smem, ctx.stream>>>(
-      reinterpret_cast<cx<S>*>(ctx.amps), P);
+      reinterpret_cast<cx<S>*>(ctx.amps), tile_off, P);
 }
 // TMA bulk copies for tiles of at most fuse_tma_max_chunks chunks (default: all),
 // direct register loads otherwise.
 template <int K>
-void launch_k(const LaunchCtx& ctx, const FProg& P) {
+void launch_k(const LaunchCtx& ctx, const FProg& P, uint64_t tile_off) {
   const bool direct = (1 << P.tile.nh) > ctx.opt->fuse_tma_max_chunks;
   if (ctx.c64) {
     if (direct)
-      launch_kd<K, true, float>(ctx, P);
+      launch_kd<K, true, float>(ctx, P, tile_off);
     else
-      launch_kd<K, false, float>(ctx, P);
+      launch_kd<K, false, float>(ctx, P, tile_off);
   } else {
     if (direct)
-      launch_kd<K, true, double>(ctx, P);
+      launch_kd<K, true, double>(ctx, P, tile_off);
     else
-      launch_kd<K, false, double>(ctx, P);
+      launch_kd<K, false, double>(ctx, P, tile_off);
   }
 }
 
@@ -967,19 +969,22 @@ void build_program(const LaunchCtx& ctx, const TileCfg& cfg, uint64_t in_tile,
 
 // Launches an encoded pass: the compiled kernel of its program (LFQS_FUSE_JIT)
 // or the interpreting kernel k_fused<K>.
-void launch_built(const LaunchCtx& ctx, int K, const FProg& P, const std::string* key = nullptr) {
+// tile_off: the launch covers tiles [tile_off, tile_off + 2^(ctx.n_local - K)) of the state
+// at ctx.amps (a block whose top bits are fixed, for overlapped exchanges; 0 otherwise).
+void launch_built(const LaunchCtx& ctx, int K, const FProg& P, const std::string* key = nullptr,
+                  uint64_t tile_off = 0) {
   if (ctx.jit && (1 << P.tile.nh) <= ctx.opt->fuse_tma_max_chunks) {
     const int jc = jit_config(ctx, K);
-    jit_launch(ctx, P, K, key ? *key : jit_key(P, K, ctx.c64, jc), jc);
+    jit_launch(ctx, P, K, key ? *key : jit_key(P, K, ctx.c64, jc), jc, tile_off);
     ++*ctx.launch_counter;
     return;
   }
   switch (K) {
-    case 8: launch_k<8>(ctx, P); break;
-    case 9: launch_k<9>(ctx, P); break;
-    case 10: launch_k<10>(ctx, P); break;
-    case 11: launch_k<11>(ctx, P); break;
-    default: launch_k<12>(ctx, P); break;
+    case 8: launch_k<8>(ctx, P, tile_off); break;
+    case 9: launch_k<9>(ctx, P, tile_off); break;
+    case 10: launch_k<10>(ctx, P, tile_off); break;
+    case 11: launch_k<11>(ctx, P, tile_off); break;
+    default: launch_k<12>(ctx, P, tile_off); break;
   }
   LFQS_CUDA_CHECK(cudaGetLastError());
   ++*ctx.launch_counter;
@@ -1071,10 +1076,17 @@ void plan_fused_schedule(const LaunchCtx& ctx_in, const std::vector<Decoded>& ga
   std::vector<int> rest;
   for (size_t i = 0; i < gates.size(); ++i)
     if (gates[i].cls != GClass::NOOP) rest.push_back((int)i);
+  auto nd_of = [&](const Decoded& g) {
+    uint64_t m = 0;
+    if (g.cls != GClass::DIAG)
+      for (int t = 0; t < g.m; ++t) m |= 1ull << g.targets[t];
+    return m;
+  };
   auto single = [&](int gi) {
     FusedPass ps;
     ps.gate = gi;
     ps.qmask = qubit_mask(gates[gi]);
+    ps.nd_mask = nd_of(gates[gi]);
     out.push_back(std::move(ps));
   };
   if (!tile_cfg(ctx, tile_qubits, &cfg)) {
@@ -1144,7 +1156,10 @@ void plan_fused_schedule(const LaunchCtx& ctx_in, const std::vector<Decoded>& ga
       ps.prog.reset(new FProg);
       ps.K = cfg.K;
       build_program(ctx, cfg, in_tile, list, *ps.prog);
-      for (int gi : picked) ps.qmask |= qubit_mask(gates[gi]);
+      for (int gi : picked) {
+        ps.qmask |= qubit_mask(gates[gi]);
+        ps.nd_mask |= nd_of(gates[gi]);
+      }
       if (jit_ok) ps.key = jit_key(*ps.prog, cfg.K, ctx.c64, jit_config(ctx, cfg.K));
       out.push_back(std::move(ps));
       for (int gi : picked) taken[gi] = 1;
@@ -1164,6 +1179,30 @@ void launch_fused_pass(const LaunchCtx& ctx, const std::vector<Decoded>& gates,
     launch_built(ctx, ps.K, *ps.prog, ps.key.empty() ? nullptr : &ps.key);
   else
     launch_gate(ctx, gates[ps.gate]);
+}
+
+void launch_fused_pass_block(const LaunchCtx& ctx, const std::vector<Decoded>& gates,
+                             const FusedPass& ps, int c, uint64_t v) {
+  const int n_sub = ctx.n_local - c;
+  require(c >= 0 && n_sub >= 1 && (ps.nd_mask >> n_sub) == 0,
+          "internal: pass not confined to the block");
+  if (ps.prog) {
+    require(n_sub >= ps.K, "internal: block smaller than the pass's tile");
+    LaunchCtx x = ctx;  // same base pointer; the tiles of block v only
+    x.n_local = n_sub;
+    launch_built(x, ps.K, *ps.prog, ps.key.empty() ? nullptr : &ps.key, v << (n_sub - ps.K));
+    return;
+  }
+  // A single gate: its controls / diagonal entries on the block's fixed top bits are
+  // resolved on the host, as the planner does for a rank's global bits (Planner::rank_local
+  // with the block index in the role of the rank), then it runs on the block.
+  Planner blk(ctx.n_local, 1 << c);
+  Decoded lg;
+  if (!blk.rank_local(gates[ps.gate], (int)v, 0, &lg) || lg.cls == GClass::NOOP) return;
+  LaunchCtx x = ctx;
+  x.amps = static_cast<unsigned char*>(ctx.amps) + (v << n_sub) * (ctx.c64 ? 8 : 16);
+  x.n_local = n_sub;
+  launch_gate(x, lg);
 }
 
 void run_fused_schedule(const LaunchCtx& ctx, const std::vector<Decoded>& gates,

@@ -1565,6 +1565,8 @@ struct Gen {
     e("mov.u32 %%ltid, %%tid.x;");
     e("mov.u32 %%bid, %%ctaid.x;");
     e("cvt.u64.u32 %%base, %%bid;");
+    e("ld.param.u64 %%toff, [poff];");  // first tile of the launch (a block of the state)
+    e("add.u64 %%base, %%base, %%toff;");
     e("shl.b64 %%base, %%base, %d;", tg.lc);
     for (int i = 0; i < tg.nh; ++i) {
       const int pp = tg.hpos[i];
@@ -1695,7 +1697,7 @@ struct Gen {
     out += ".shared .align 8 .b64 lfqs_bar;\n";
     out += ".shared .align 16 .b8 lfqs_dtab[" + std::to_string(256 * ES) + "];\n\n";
     const int nc = P.ncoef > 0 ? P.ncoef : 1;
-    out += ".visible .entry lfqs_jit(.param .u64 pa, .param .align 16 .b8 pc[" +
+    out += ".visible .entry lfqs_jit(.param .u64 pa, .param .u64 poff, .param .align 16 .b8 pc[" +
            std::to_string(nc * 16) + "])\n";
     out += ".maxntid " + std::to_string(NT) + ", 1, 1\n.minnctapersm " +
            std::to_string(min_ctas()) + "\n{\n";
@@ -1706,7 +1708,7 @@ struct Gen {
     out += std::string("  .reg .") + FT + " %f<" + std::to_string(nf + 1) + ">;\n";
     out += std::string("  .reg .") + FT + " %vx<" + std::to_string(R) + ">;\n";
     out += std::string("  .reg .") + FT + " %vy<" + std::to_string(R) + ">;\n";
-    out += "  .reg .b64 %ga, %base;\n  .reg .b32 %ltid, %bid, %tile, %dtab, %bar, %taddr;\n";
+    out += "  .reg .b64 %ga, %base, %toff;\n  .reg .b32 %ltid, %bid, %tile, %dtab, %bar, %taddr;\n";
     out += body;
     out += "}\n";
     return out;
@@ -1910,7 +1912,8 @@ size_t jit_cache_size() {
   return g_cache.size();
 }
 
-void jit_launch(const LaunchCtx& ctx, const FProg& P, int K, const std::string& key, int jc) {
+void jit_launch(const LaunchCtx& ctx, const FProg& P, int K, const std::string& key, int jc,
+                uint64_t tile_off) {
   const int nt = jc & JIT_THREADS_MASK;
   std::shared_ptr<Entry> en;
   {
@@ -1952,7 +1955,7 @@ void jit_launch(const LaunchCtx& ctx, const FProg& P, int K, const std::string& 
     }
   }
   void* a = ctx.amps;
-  void* args[2] = {&a, (void*)P.c};
+  void* args[3] = {&a, &tile_off, (void*)P.c};
   const uint64_t tiles = 1ull << (ctx.n_local - K);
   LFQS_CUDA_CHECK(cudaLaunchKernel((const void*)en->kern, dim3((unsigned)tiles), dim3(nt),
                                    args, (size_t)smem, ctx.stream));

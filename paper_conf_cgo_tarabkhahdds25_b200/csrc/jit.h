@@ -25,8 +25,10 @@ std::string jit_key(const FProg& P, int K, bool c64, int jc);
 // Generates and compiles (in parallel, nvPTXCompiler) every pass not yet cached.
 void jit_compile(const std::vector<std::pair<std::string, const FProg*>>& items, int K, bool c64,
                  int jc);
-// Launches the pass (compiling it first if needed) on ctx.stream.
-void jit_launch(const LaunchCtx& ctx, const FProg& P, int K, const std::string& key, int jc);
+// Launches the pass (compiling it first if needed) on ctx.stream: 2^(ctx.n_local - K) tiles,
+// tile indices starting at tile_off (a block of the state whose top bits are fixed).
+void jit_launch(const LaunchCtx& ctx, const FProg& P, int K, const std::string& key, int jc,
+                uint64_t tile_off = 0);
 // Generator configuration for tile size K (LFQS_OPT_JIT_THREADS, LFQS_OPT_JIT_LANE_MOVE).
 int jit_config(const LaunchCtx& ctx, int K);
 size_t jit_cache_size();

@@ -163,6 +163,7 @@ struct FusedPass {
   std::string key;               // compiled-pass cache key (LFQS_FUSE_JIT), else empty
   int K = 0;                     // tile qubits of prog
   uint64_t qmask = 0;            // qubits the pass's gates touch (targets | controls)
+  uint64_t nd_mask = 0;          // targets of its non-diagonal gates (the qubits it mixes)
 };
 // Plans (and for LFQS_FUSE_JIT compiles) the passes run_fused_schedule would launch.
 void plan_fused_schedule(const LaunchCtx& ctx, const std::vector<Decoded>& gates, int tile_qubits,
@@ -171,6 +172,12 @@ void plan_fused_schedule(const LaunchCtx& ctx, const std::vector<Decoded>& gates
 // n_local) that contains every qubit in ps.qmask.
 void launch_fused_pass(const LaunchCtx& ctx, const std::vector<Decoded>& gates,
                        const FusedPass& ps);
+// Launches it on block v of the shard ctx: the amplitudes whose top c bits equal v.  The
+// pass must not mix those bits (ps.nd_mask below n_local - c); controls and diagonal
+// entries on them are resolved for the block (exactly the ops the whole-shard pass applies
+// to these amplitudes, with the same kernels and formulas).
+void launch_fused_pass_block(const LaunchCtx& ctx, const std::vector<Decoded>& gates,
+                             const FusedPass& ps, int c, uint64_t v);
 
 // Reductions (C9): d_out[v], v < 2^nq (nq <= 20, bit s of v = bit qubits[s]); one read
 // pass over the shard whatever nq is; deterministic (fixed grid and summation order).

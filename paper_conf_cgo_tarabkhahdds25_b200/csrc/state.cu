@@ -299,7 +299,7 @@ void State::exchange_data(int l, int g) {
     for (int r = 0; r < world; ++r) {
       if (r >> j & 1) continue;
       const int r2 = r | (1 << j);
-      launch_half_swap(ctx(r), l, ((uint64_t)(r2 - r)) << n_local);
+      launch_half_swap(ctx(r), l, ((uint64_t)(r2 - r)) << n_local, 0, opt.exchange_ctas);
     }
   } else if (p2p) {
     p2p->exchange(ctx(0), l, j, n_local, 0, opt.exchange_ctas);
@@ -362,9 +362,10 @@ std::vector<State::ShardRun> State::plan_run(const std::vector<PlanOp>& ops, siz
       for (size_t i = 0; i < r.seg.size(); ++i) {
         FusedPass ps;
         ps.gate = (int)i;
-        uint64_t m = r.seg[i].cmask;
+        uint64_t m = 0;
         for (int t = 0; t < r.seg[i].m; ++t) m |= 1ull << r.seg[i].targets[t];
-        ps.qmask = m;
+        ps.qmask = m | r.seg[i].cmask;
+        ps.nd_mask = r.seg[i].cls == GClass::DIAG ? 0 : m;
         r.passes.push_back(std::move(ps));
       }
     }
@@ -376,12 +377,13 @@ void State::launch_passes(const std::vector<ShardRun>& run, const std::vector<si
                           const std::vector<size_t>& to, int c, int v) {
   for (int s = 0; s < n_shards(); ++s) {
     if (from[s] >= to[s]) continue;
-    LaunchCtx x = ctx(s);
-    if (c > 0) {
-      x.amps = static_cast<unsigned char*>(x.amps) + ((uint64_t)v << (n_local - c)) * ab;
-      x.n_local = n_local - c;
+    const LaunchCtx x = ctx(s);
+    for (size_t i = from[s]; i < to[s]; ++i) {
+      if (c > 0)
+        launch_fused_pass_block(x, run[s].seg, run[s].passes[i], c, (uint64_t)v);
+      else
+        launch_fused_pass(x, run[s].seg, run[s].passes[i]);
     }
-    for (size_t i = from[s]; i < to[s]; ++i) launch_fused_pass(x, run[s].seg, run[s].passes[i]);
   }
 }
 
@@ -447,10 +449,14 @@ cudaEvent_t State::exchange_part(int l, int g, int c, int v, cudaEvent_t ready) 
 // an exchange at a position l below the top c local qubits (the planner keeps exchange
 // positions out of the top two, planner.h) moves data only inside each block whose top c
 // bits are fixed, so it splits into 2^c independent parts.  The trailing passes of the run
-// before it that touch none of those c qubits run part by part on the compute stream; part
+// before it that do not mix those c qubits run part by part on the compute stream; part
 // v moves (exchange stream, or the NCCL stream) as soon as its tail is done, while the
-// compute stream goes on with the next part; the leading passes of the next run that touch
-// none of them run on part v as soon as it has landed.  The passes are exactly the ones the
+// compute stream goes on with the next part; the leading passes of the next run that do
+// not mix those qubits run on part v as soon as it has landed.  A pass "mixes" a qubit
+// when a non-diagonal gate targets it; controls and diagonal entries on the chunk qubits
+// are resolved per part (fused passes read them from the tile index, which starts at the
+// part's first tile; single gates are specialised on the host), so e.g. every QFT CPhase
+// pass can run part by part.  The passes are exactly the ones the
 // serial execution launches (no extra HBM pass), each applied block by block with the same
 // kernels, and every pass sees the data it would see in the serial order (Eq. 3; ops
 // on disjoint blocks commute): results are bit-identical to serial exchanges
@@ -491,12 +497,16 @@ void State::execute(const std::vector<PlanOp>& ops, bool fuse) {
       std::fill(from.begin(), from.end(), 0);
       continue;
     }
-    // tail: trailing passes free of the chunk bits; head: leading ones of the next run
+    // tail: trailing passes that do not mix the chunk bits (controls and diagonal
+    // entries on them are fine: resolved per block); head: leading ones of the next run
+    auto blockwise = [&](const FusedPass& ps) {
+      return !(ps.nd_mask & H) && (!ps.prog || ps.K <= n_local - c);
+    };
     std::vector<size_t> ts(S), he(S, 0), zero(S, 0);
     for (int s = 0; s < S; ++s) {
       ts[s] = end[s];
-      while (ts[s] > from[s] && !(cur[s].passes[ts[s] - 1].qmask & H)) --ts[s];
-      while (he[s] < next[s].passes.size() && !(next[s].passes[he[s]].qmask & H)) ++he[s];
+      while (ts[s] > from[s] && blockwise(cur[s].passes[ts[s] - 1])) --ts[s];
+      while (he[s] < next[s].passes.size() && blockwise(next[s].passes[he[s]])) ++he[s];
     }
     launch_passes(cur, from, ts, 0, 0);  // the body of the run
     const int parts = 1 << c;
