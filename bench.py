@@ -311,6 +311,76 @@ def run_macro(lfqs, stream, n: int, reps: int, unfused: bool, hbm_peak: float):
 
 
 # ----------------------------------------------------------------------------
+# N > 1: QFT(n_local + log2 N) sharded across the ranks (configs[4] shape)
+# ----------------------------------------------------------------------------
+
+NVLINK_GBPS = 900.0  # NVLink 5 per GPU per direction, nominal (no measured peak here)
+
+
+def run_qft_sharded(lfqs, st, n, n_loc, world, rank, stream, barrier, dist, device_reduce,
+                    hbm_peak, reps):
+    """QFT(n)|x> on the sharded state (n = n_loc + log2 world; 8 GPUs x 2^30: QFT(33), the
+    configs[4] circuit at this per-GPU size), compiled passes + phase tables, exchanges
+    overlapped with local passes; the timed region ends after the final canonicalisation
+    (relabels are not free).  Device time (CUDA events) max over ranks.
+    Combined roofline (SURVEY §8(d) [4]): T_roof = sum of passes x 32 * 2^n_loc B / HBM +
+    exchanges x 16 * 2^(n_loc - 1) B / NVLink, the north-star form with one pass per gate
+    beside it; closed form checked on 64 sampled amplitudes of every rank's shard."""
+    import torch
+    x = int(W.SplitMix64(n).next_u64() & ((1 << n) - 1))
+    gates = W.qft(n)
+    arr = lfqs.marshal_gates(gates)
+    flags = lfqs.FUSE_LOW | lfqs.FUSE_JIT | lfqs.FUSE_PHASE
+
+    def once():
+        st.init_basis(x)
+        barrier()
+        p0, e0 = st.passes(), st.exchange_stats()
+        a = torch.cuda.Event(enable_timing=True)
+        b = torch.cuda.Event(enable_timing=True)
+        a.record(stream)
+        lfqs.lfqs_run_circuit(st.h, arr, flags)
+        st.copy_out(0, 0)  # canonicalise the qubit map (collective), inside the timed region
+        b.record(stream)
+        barrier()
+        e1 = st.exchange_stats()
+        return a.elapsed_time(b), st.passes() - p0, e1[0] - e0[0], e1[1] - e0[1]
+
+    once()  # warm-up: compiles every pass shape
+    runs = [once() for _ in range(reps)]
+    ms_rank = min(r[0] for r in runs)
+    t = torch.tensor([ms_rank], device=device_reduce)
+    dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    ms = float(t.item())
+    _, passes, n_ex, ex_bytes = runs[0]
+    # closed form on this rank's shard (canonical order after the timed canonicalisation)
+    rng = np.random.default_rng(rank + 1)
+    lo = rank << n_loc
+    idx = lo + rng.integers(0, 1 << n_loc, 64)
+    got = np.array([st.copy_out(int(k), 1)[0] for k in idx])
+    ph = ((x * idx.astype(object)) % (1 << n)).astype(np.float64) / (1 << n)
+    err = float(np.max(np.abs(got - np.exp(2j * np.pi * ph) / math.sqrt(2.0 ** n))))
+    e = torch.tensor([err], device=device_reduce, dtype=torch.float64)
+    dist.all_reduce(e, op=dist.ReduceOp.MAX)
+    pb = 32.0 * 2 ** n_loc
+    t_ex = n_ex * 16.0 * 2 ** (n_loc - 1) / (NVLINK_GBPS * 1e9)
+    t_roof = passes * pb / (hbm_peak * 1e9) + t_ex
+    t_roof_gates = len(gates) * pb / (hbm_peak * 1e9) + t_ex
+    return {"circuit": f"QFT({n}) on {world} ranks, 2^{n_loc} amplitudes per rank",
+            "mode": "jit+phase, exchanges overlapped", "gates": len(gates),
+            "ms": round(ms, 3), "gates_per_s": len(gates) / (ms / 1e3),
+            "passes_per_rank": int(passes), "exchanges_per_rank": int(n_ex),
+            "exchange_bytes_per_rank_per_direction": int(ex_bytes),
+            "t_roof_ms": round(t_roof * 1e3, 3), "roof_frac": (t_roof * 1e3) / ms,
+            "t_roof_north_star_ms": round(t_roof_gates * 1e3, 3),
+            "roof_frac_north_star": (t_roof_gates * 1e3) / ms,
+            "roofline_terms": "passes x 32*2^n_loc B / hbm_peak + exchanges x 16*2^(n_loc-1) B "
+                              f"/ {NVLINK_GBPS} GB/s (north star: one pass per gate)",
+            "closed_form_max_abs_err": float(e.item()),
+            "closed_form_rel_err": float(e.item()) * math.sqrt(2.0 ** n)}
+
+
+# ----------------------------------------------------------------------------
 # GPU arm
 # ----------------------------------------------------------------------------
 
@@ -332,6 +402,8 @@ def main():
     ap.add_argument("--macro-reps", type=int, default=3)
     ap.add_argument("--no-macro-unfused", action="store_true",
                     help="skip the strict one-pass-per-gate QFT/GHZ runs of the macro leg")
+    ap.add_argument("--qft-reps", type=int, default=3,
+                    help="N > 1: timed runs of the sharded QFT leg (0: skip)")
     ap.add_argument("--same-device", action="store_true",
                     help="test only: every rank on cuda:0 (exercises the N>1 path on one GPU)")
     ap.add_argument("--transport", default="p2p", choices=["p2p", "nccl"],
@@ -504,6 +576,11 @@ def main():
                   "frac": link_gbps / 900.0 if link_gbps else None,
                   "transport": args.transport}
 
+    qft = None
+    if world > 1 and args.qft_reps > 0:
+        qft = run_qft_sharded(lfqs, st, n, n_loc, world, rank, stream, barrier, dist,
+                              "cpu" if args.same_device else "cuda", hbm_peak, args.qft_reps)
+
     if args.per_gate_json and rank == 0:
         with open(args.per_gate_json, "w") as f:
             json.dump([{"cls": cls, "gate": g.label(), "ms": float(mean_ms[i]),
@@ -513,7 +590,13 @@ def main():
     # end to end through the public API: H2D of the input state from pinned host
     # memory, the sweep, and a D2H read of the measured probabilities each step
     e2e = None
-    if not args.no_e2e:
+    need_gib = 16.0 * 2 ** n_loc / 2 ** 30 * world  # every rank's pinned shard, one host
+    if not args.no_e2e and world > 1 and host_avail_gib() < 1.25 * need_gib:
+        # every rank pins its own 16 GiB shard: skip (and say so) when the host cannot
+        e2e = {"unavailable": f"{world} ranks x {16.0 * 2 ** n_loc / 2 ** 30:.0f} GiB pinned "
+                              f"host buffers exceed 80 % of MemAvailable "
+                              f"({host_avail_gib():.0f} GiB)"}
+    elif not args.no_e2e:
         host = torch.empty(1 << n_loc, dtype=torch.complex128, pin_memory=True)
         hv = host.numpy()
         st.copy_out(rank << n_loc, 1 << n_loc, out=hv)
@@ -584,6 +667,7 @@ def main():
             "roofline": roofline,
             "worst_gate": worst_gate,
             "macro": macro,
+            "qft_sharded": qft,
             "nvlink": nvlink,
             "classes": {k: {kk: (round(vv, 4) if isinstance(vv, float) else vv)
                             for kk, vv in v.items()} for k, v in classes.items()},

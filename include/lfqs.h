@@ -334,6 +334,11 @@ lfqs_status lfqs_state_exchange_stats(const lfqs_state* s, uint64_t* exchanges,
                                       uint64_t* bytes_per_rank);
 /* Number of kernels this state has launched so far (for benchmark accounting). */
 lfqs_status lfqs_kernel_launches(const lfqs_state* s, uint64_t* count);
+/* Number of state passes this state has run so far: one per fused pass or per single-gate
+ * class kernel of lfqs_apply_gate / lfqs_run_circuit (an exchange's swap kernels and
+ * a pass run block by block around an overlapped exchange count once) -- the
+ * denominator of the per-pass HBM roofline (benchmark accounting). */
+lfqs_status lfqs_state_pass_count(const lfqs_state* s, uint64_t* passes);
 /* Tuning knobs (benchmark / test use): LFQS_OPT_LOWQ_SHUFFLE (1: warp-shuffle
  * path for targets < 5; default 0, measured no faster than the 32-byte path), LFQS_OPT_FUSE_TILE_QUBITS (k of the staging
  * tile, default 12). */

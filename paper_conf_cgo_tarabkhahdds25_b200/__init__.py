@@ -61,6 +61,7 @@ EXPORTS = [
     "lfqs_state_init_basis", "lfqs_state_init_random", "lfqs_copy_in", "lfqs_copy_out",
     "lfqs_apply_gate", "lfqs_run_circuit", "lfqs_measure_probs", "lfqs_synchronize",
     "lfqs_state_info", "lfqs_kernel_launches", "lfqs_set_option", "lfqs_last_error",
+    "lfqs_state_pass_count",
     "lfqs_abi_version", "lfqs_plan_circuit", "lfqs_measure_sample", "lfqs_measure_collapse",
     "lfqs_state_create_ex", "lfqs_state_wrap_ex", "lfqs_copy_in_c64", "lfqs_copy_out_c64",
     "lfqs_circuit_compile", "lfqs_circuit_launch", "lfqs_circuit_destroy",
@@ -143,6 +144,7 @@ def lib():
             "lfqs_synchronize": [vp],
             "lfqs_state_info": [vp, ip, ip, ip, ip, C.POINTER(vp)],
             "lfqs_kernel_launches": [vp, C.POINTER(u64)],
+            "lfqs_state_pass_count": [vp, C.POINTER(u64)],
             "lfqs_set_option": [vp, C.c_int, C.c_int64],
             "lfqs_state_create_ex": [C.c_int, C.c_int, C.c_int, vp, C.c_uint32, C.POINTER(vp)],
             "lfqs_state_wrap_ex": [C.c_int, C.c_int, vp, vp, C.c_uint32, C.POINTER(vp)],
@@ -670,6 +672,12 @@ class State:
 
     def launches(self) -> int:
         return lfqs_kernel_launches(self.h)
+
+    def passes(self) -> int:
+        """State passes run so far (fused passes + single-gate kernels; lfqs_state_pass_count)."""
+        c = C.c_uint64()
+        _check(lib().lfqs_state_pass_count(self.h, C.byref(c)))
+        return int(c.value)
 
     def set_option(self, option: int, value: int):
         lfqs_set_option(self.h, option, value)

@@ -501,6 +501,13 @@ lfqs_status lfqs_kernel_launches(const lfqs_state* s, uint64_t* count) {
   });
 }
 
+lfqs_status lfqs_state_pass_count(const lfqs_state* s, uint64_t* passes) {
+  return guarded([&] {
+    require(s != nullptr && passes != nullptr, "NULL argument");
+    *passes = static_cast<const State*>(s)->passes;
+  });
+}
+
 lfqs_status lfqs_set_option(lfqs_state* s, int option, int64_t value) {
   return guarded([&] {
     require(s != nullptr, "NULL state");

@@ -322,7 +322,10 @@ void State::exchange_data(int l, int g) {
 // class kernel per gate.
 void State::run_local(const LaunchCtx& c, const std::vector<Decoded>& gates, bool fuse) {
   if (fuse && opt.fuse_reorder) {
-    run_fused_schedule(c, gates, opt.fuse_tile_qubits);
+    std::vector<FusedPass> ps;
+    plan_fused_schedule(c, gates, opt.fuse_tile_qubits, ps);
+    for (const FusedPass& p : ps) launch_fused_pass(c, gates, p);
+    passes += ps.size();
     return;
   }
   size_t i = 0;
@@ -334,6 +337,7 @@ void State::run_local(const LaunchCtx& c, const std::vector<Decoded>& gates, boo
       launch_gate(c, gates[i]);
       ++i;
     }
+    ++passes;
   }
 }
 
@@ -378,6 +382,7 @@ void State::launch_passes(const std::vector<ShardRun>& run, const std::vector<si
   for (int s = 0; s < n_shards(); ++s) {
     if (from[s] >= to[s]) continue;
     const LaunchCtx x = ctx(s);
+    if (c == 0 || v == 0) passes += to[s] - from[s];
     for (size_t i = from[s]; i < to[s]; ++i) {
       if (c > 0)
         launch_fused_pass_block(x, run[s].seg, run[s].passes[i], c, (uint64_t)v);
@@ -536,6 +541,7 @@ void State::apply(const Decoded& g) {
   DeviceGuard dg(device);
   if (world == 1) {
     launch_gate(ctx(0), g);
+    if (g.cls != GClass::NOOP) ++passes;
     return;
   }
   std::vector<PlanOp> ops;

@@ -35,6 +35,7 @@ struct State : lfqs_state {
   cudaStream_t stream = nullptr;
   bool own_stream = false;
   uint64_t launches = 0;
+  uint64_t passes = 0;          // state passes run (lfqs_state_pass_count)
   Options opt;
   double* d_partials = nullptr; // reduction scratch (grown on demand)
   double* d_probs = nullptr;    // 2^nq result bins (grown on demand)
