@@ -12,8 +12,11 @@
 #include <nccl.h>
 
 #include <algorithm>
+#include <chrono>
+#include <cstdlib>
 #include <cstring>
 #include <string>
+#include <thread>
 
 #include "comm.h"
 
@@ -51,7 +54,7 @@ Comm::Comm(int rank_, int world_, const uint8_t uid[128], size_t stage_bytes)
 }
 
 Comm::~Comm() {
-  cudaStreamSynchronize(cstream);
+  if (comm) cudaStreamSynchronize(cstream);
   for (int i = 0; i < 2; ++i) {
     cudaFree(stage[i]);
     cudaEventDestroy(ev_recv[i]);
@@ -60,13 +63,14 @@ Comm::~Comm() {
   cudaEventDestroy(ev_start);
   cudaFree(d_reduce);
   cudaStreamDestroy(cstream);
-  ncclCommDestroy(comm);
+  if (comm) ncclCommDestroy(comm);
 }
 
 // Exchanges the amplitudes at `pieces` (offset, count in amplitudes, in this
 // rank's shard) with the same pieces of `partner`, in place.
 void Comm::exchange(void* shard, int amp_bytes, const std::vector<Piece>& pieces, int partner,
                     cudaStream_t compute, cudaEvent_t ready) {
+  require(comm != nullptr, "NCCL communicator was aborted after an earlier error");
   // The comm stream must see every kernel the exchanged data depends on: `ready`, or
   // everything already queued on the compute stream.
   if (ready == nullptr) {
@@ -97,7 +101,37 @@ void Comm::exchange(void* shard, int amp_bytes, const std::vector<Piece>& pieces
   }
 }
 
+void Comm::wait(cudaStream_t s) {
+  double timeout_s = 300.0;
+  if (const char* e = std::getenv("LFQS_NCCL_TIMEOUT_S")) timeout_s = std::atof(e);
+  const auto t0 = std::chrono::steady_clock::now();
+  for (unsigned spin = 0;; ++spin) {
+    const cudaError_t q = cudaStreamQuery(s);
+    if (q == cudaSuccess) return;
+    if (q != cudaErrorNotReady) LFQS_CUDA_CHECK(q);
+    ncclResult_t async = ncclSuccess;
+    LFQS_NCCL_CHECK(ncclCommGetAsyncError(comm, &async));
+    if (async != ncclSuccess && async != ncclInProgress) {
+      ncclCommAbort(comm);
+      comm = nullptr;
+      throw Error(LFQS_ERR_NCCL, std::string("NCCL asynchronous error: ") +
+                                     ncclGetErrorString(async));
+    }
+    const double el =
+        std::chrono::duration<double>(std::chrono::steady_clock::now() - t0).count();
+    if (timeout_s > 0 && el > timeout_s) {
+      ncclCommAbort(comm);
+      comm = nullptr;
+      throw Error(LFQS_ERR_NCCL, "NCCL operation did not complete within " +
+                                     std::to_string(timeout_s) + " s (peer lost?); "
+                                     "communicator aborted");
+    }
+    std::this_thread::sleep_for(std::chrono::microseconds(spin < 100 ? 20 : 500));
+  }
+}
+
 void Comm::allreduce_sum(double* d, size_t count, cudaStream_t s) {
+  require(comm != nullptr, "NCCL communicator was aborted after an earlier error");
   LFQS_NCCL_CHECK(ncclAllReduce(d, d, count, ncclDouble, ncclSum, comm, s));
 }
 

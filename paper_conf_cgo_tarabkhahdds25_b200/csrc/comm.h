@@ -34,6 +34,10 @@ struct Comm {
   void exchange(void* shard, int amp_bytes, const std::vector<Piece>& pieces, int partner,
                 cudaStream_t compute, cudaEvent_t ready = nullptr);
   void allreduce_sum(double* d, size_t count, cudaStream_t s);
+  // Waits for stream s while polling ncclCommGetAsyncError: a failed or hung peer
+  // (no progress for timeout_s seconds; LFQS_NCCL_TIMEOUT_S, default 300) aborts the
+  // communicator and throws LFQS_ERR_NCCL instead of blocking forever.
+  void wait(cudaStream_t s);
 };
 
 }  // namespace lfqs

@@ -220,9 +220,16 @@ void State::init_random(uint64_t seed) {
     launch_init_random(ctx(s), seed, (uint64_t)rank_of_shard(s) << n_local);
 }
 
+void State::wait_stream() {
+  if (comm)
+    comm->wait(stream);
+  else
+    LFQS_CUDA_CHECK(cudaStreamSynchronize(stream));
+}
+
 void State::synchronize() {
   DeviceGuard dg(device);
-  LFQS_CUDA_CHECK(cudaStreamSynchronize(stream));
+  wait_stream();
   LFQS_CUDA_CHECK(cudaGetLastError());
   if (p2p) p2p->check();
 }
@@ -257,7 +264,7 @@ void State::copy_raw(uint64_t offset, uint64_t count, void* host, bool to_device
     else
       LFQS_CUDA_CHECK(cudaMemcpyAsync(h, dev, bytes, cudaMemcpyDeviceToHost, stream));
   }
-  LFQS_CUDA_CHECK(cudaStreamSynchronize(stream));
+  wait_stream();
 }
 
 void State::copy(uint64_t offset, uint64_t count, double* host, bool to_device) {
@@ -734,7 +741,7 @@ void State::local_probs(int shard, const int* lq, int nl, double* host) {
   launch_probs(ctx(shard), lq, nl, d_partials, partials_cap, d_probs);
   LFQS_CUDA_CHECK(cudaMemcpyAsync(host, d_probs, sizeof(double) << nl, cudaMemcpyDeviceToHost,
                                   stream));
-  LFQS_CUDA_CHECK(cudaStreamSynchronize(stream));
+  wait_stream();
 }
 
 void State::measure_probs(const int* qubits, int nq, double* out) {
@@ -778,7 +785,7 @@ void State::measure_probs(const int* qubits, int nq, double* out) {
     comm->allreduce_sum(d, nb, stream);
     LFQS_CUDA_CHECK(cudaMemcpyAsync(full.data(), d, sizeof(double) * nb, cudaMemcpyDeviceToHost,
                                     stream));
-    LFQS_CUDA_CHECK(cudaStreamSynchronize(stream));
+    wait_stream();
     if (d != comm->d_reduce) cudaFree(d);
   }
   std::memcpy(out, full.data(), sizeof(double) * nb);

@@ -80,6 +80,9 @@ struct State : lfqs_state {
   // Zeroes amplitudes whose measured bits != outcome, scales the rest by `scale`.
   void collapse(const int* qubits, int nq, uint64_t outcome, double scale);
   void synchronize();
+  // Waits for the state's stream (NCCL states: polling the communicator's async errors
+  // with a timeout, Comm::wait).
+  void wait_stream();
   void* shard_ptr() const { return amps; }
 
  private:
