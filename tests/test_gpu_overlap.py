@@ -100,3 +100,25 @@ def test_overlap_graph_capture_and_per_gate_apply(L):
         for g in gates:
             st.apply(g)
         assert np.max(np.abs(st.copy_out() - ref)) <= 1e-12
+
+
+def test_pass_count(L):
+    """lfqs_state_pass_count: one per single-gate kernel or fused pass; a pass run block by
+    block around an overlapped exchange counts once (the per-pass roofline denominator)."""
+    n = 14
+    gates = W.random_gate_list(n, 50, seed=3, max_controls=1)
+    with L.State.create(n) as st:
+        p0 = st.passes()
+        st.run_circuit(gates)
+        assert st.passes() - p0 == len([g for g in gates if g.kind != "I"])
+        p0, l0 = st.passes(), st.launches()
+        st.run_circuit(gates, fuse="jit")
+        assert 2 <= st.passes() - p0 <= st.launches() - l0
+    for bits in (0, 2):
+        with L.State.virtual(n, 4) as st:
+            st.set_option(L.OPT_EXCHANGE_CHUNK_BITS, bits)
+            st.run_circuit(W.qft(n), fuse="jit")
+            if bits == 0:
+                serial = st.passes()
+            else:
+                assert st.passes() == serial
