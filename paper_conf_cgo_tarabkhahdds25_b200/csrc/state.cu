@@ -340,11 +340,12 @@ void State::run_local(const LaunchCtx& c, const std::vector<Decoded>& gates, boo
     size_t used = 0;
     if (fuse && run_fused_circuit(c, gates, i, gates.size(), opt.fuse_tile_qubits, &used)) {
       i += used;
+      ++passes;
     } else {
       launch_gate(c, gates[i]);
+      if (gates[i].cls != GClass::NOOP) ++passes;
       ++i;
     }
-    ++passes;
   }
 }
 
