@@ -44,8 +44,12 @@ def main():
                         W.Gate("UNITARY2", (5, 3), (0, 11), (), U2),
                         W.Gate("UNITARY3", (1, 2, 3), (), (), U3),
                         W.Gate("UNITARY3", (4, 1, 5), (7,), (), U3)])
+        # line-shaped reads: fixed bits on qubits 1 / 2 (controls, one-entry diagonals)
+        st.run_circuit([W.TOFFOLI(1, 2, 5), W.TOFFOLI(1, 2, 0), W.CZ(1, 2), W.Gate("S", (1,)),
+                        W.CNOT(2, 9), W.Gate("T", (2,), (7,))])
         st.measure_probs([0, 3, 13])
         st.measure_probs(list(range(12)))
+        st.measure_probs(list(range(13, -1, -1)))  # 14 qubits: two-level binning
         st.sample([1, 2], np.linspace(0, 0.99, 7))
         st.collapse([5], 1)
         st.synchronize()
@@ -54,10 +58,14 @@ def main():
         st.run_circuit(gates)
         st.measure_probs([0, 1])
         st.collapse([0], 0)
-    with L.State.virtual(n, 4) as st:
+    with L.State.virtual(n, 4) as st:  # exchanges overlapped with passes (exchange stream)
         st.init_random(2)
         st.run_circuit(gates, fuse=True)
+        st.set_option(L.OPT_EXCHANGE_CTAS, 8)  # grid-limited swap kernel
+        st.run_circuit(gates, fuse="jit")
+        st.run_circuit(gates[:80])
         st.copy_out(0, 16)
+        st.measure_probs(list(range(n)))
     print("sanitize workload done")
 
 
