@@ -433,6 +433,14 @@ lfqs_status lfqs_state_pass_count(const lfqs_state* s, uint64_t* passes);
                                      persistent grid-stride kernel); 0 (default): one
                                      thread per pair.  A small grid saturates NVLink and
                                      leaves the SMs to the overlapped local passes */
+#define LFQS_OPT_FUSE_MERGE_2Q 22 /* 1 (default): inside a fused pass, a dense 1-target gate
+                                     adjacent (in commuting order) to a 2-target gate on a
+                                     superset of its qubit is multiplied into the 4x4 on the
+                                     host, and two 2-target gates on the same pair are
+                                     multiplied, when the product has no more complex
+                                     multiply-adds per amplitude than the separate gates
+                                     (e.g. Sycamore-like 1-target layers into fSim).
+                                     Rounding changes only (dense tolerance class) */
 lfqs_status lfqs_set_option(lfqs_state* s, int option, int64_t value);
 const char* lfqs_last_error(void);
 int lfqs_abi_version(void);

@@ -652,6 +652,7 @@ inline double2 D2(cplx z) { return make_double2(z.re, z.im); }
 int coef_count(const Decoded& g) {
   const int d = 1 << g.m;
   if (g.m == 1) return 4;
+  if (g.m == 2) return 16;  // a 2-target gate may absorb 1-target gates (merge_2q): dense
   switch (g.cls) {
     case GClass::DIAG: return d;  // upper bound (DIAG1 uses 1)
     case GClass::PERM_X: case GClass::PERM_Y: case GClass::PERM_SWAP: return 0;
@@ -895,6 +896,122 @@ void merge_phase_runs(FProg& P, bool split) {
   P.nops = no;
 }
 
+// ---- 2-target merges (LFQS_OPT_FUSE_MERGE_2Q) ---------------------------------------
+// A dense 1-target gate next to a 2-target gate on a superset of its qubit (nothing in
+// between touches it, so they are adjacent in the commuting order, Eq. 3) is folded
+// into the 4x4 matrix on the host, and two 2-target gates on the same pair are multiplied,
+// when the product costs no more complex multiply-adds per amplitude than the gates did
+// separately (nonzeros / 4 for a 4x4, nonzeros / 2 for a 2x2).  Sycamore-like cycles (a
+// dense 1-target gate on each qubit, then fSim on pairs) lose about a quarter of their FP64
+// work; the heavy passes are FP64-bound (profiles/r02_heavy_passes.md).  Rounding changes
+// only (dense tolerance class); permutation / diagonal-only pairs never merge.
+int nnz_of(const cplx* M, int d) {
+  int c = 0;
+  for (int i = 0; i < d * d; ++i) c += (M[i].re != 0.0 || M[i].im != 0.0);
+  return c;
+}
+void mat4_mul(const cplx* A, const cplx* B, cplx* C) {  // C = A B (row-major 4x4)
+  for (int r = 0; r < 4; ++r)
+    for (int c = 0; c < 4; ++c) {
+      double re = 0.0, im = 0.0;
+      for (int k = 0; k < 4; ++k) {
+        const cplx x = A[r * 4 + k], y = B[k * 4 + c];
+        re += x.re * y.re - x.im * y.im;
+        im += x.re * y.im + x.im * y.re;
+      }
+      C[r * 4 + c] = cplx{re, im};
+    }
+}
+// U on local bit `msb` ? 1 : 0 of a 4x4 (targets[0] = local bit 1): U (x) I or I (x) U.
+void embed2(const cplx* U, bool msb, cplx* E) {
+  for (int r = 0; r < 4; ++r)
+    for (int c = 0; c < 4; ++c) {
+      const int ur = msb ? r >> 1 : r & 1, uc = msb ? c >> 1 : c & 1;
+      const int or_ = msb ? r & 1 : r >> 1, oc = msb ? c & 1 : c >> 1;
+      E[r * 4 + c] = or_ == oc ? U[ur * 2 + uc] : cplx{0.0, 0.0};
+    }
+}
+// M with its two local bits exchanged (the same gate with targets listed the other way).
+void swap_bits4(const cplx* M, cplx* O) {
+  auto p = [](int j) { return ((j & 1) << 1) | (j >> 1); };
+  for (int r = 0; r < 4; ++r)
+    for (int c = 0; c < 4; ++c) O[p(r) * 4 + p(c)] = M[r * 4 + c];
+}
+void set_dense4(Decoded& a, const cplx* M) {
+  for (int i = 0; i < 16; ++i) a.M[i] = M[i];
+  a.cls = GClass::DENSE;
+  a.is_h = false;
+  a.kind = LFQS_UNITARY2;
+}
+
+template <class LastTouching>
+bool merge_2q(std::vector<Decoded>& prog, Decoded& g, LastTouching&& last_touching) {
+  const uint64_t gq = qubit_mask(g);
+  if (g.m == 1 && g.cls == GClass::DENSE) {
+    // g after a 2-target gate a on (a0, a1) that g's target belongs to
+    const long k = last_touching(gq);
+    if (k < 0) return false;
+    Decoded& a = prog[k];
+    const int t = g.targets[0];
+    if (a.m != 2 || a.cmask != g.cmask || (a.targets[0] != t && a.targets[1] != t) ||
+        (a.cls != GClass::DENSE && a.cls != GClass::PERM_SWAP && a.cls != GClass::DIAG))
+      return false;
+    cplx E[16], P[16];
+    embed2(g.M, a.targets[0] == g.targets[0], E);
+    mat4_mul(E, a.M, P);
+    if (nnz_of(P, 4) > nnz_of(a.M, 4) + 2 * nnz_of(g.M, 2)) return false;
+    set_dense4(a, P);
+    return true;
+  }
+  if (g.m != 2 || (g.cls != GClass::DENSE && g.cls != GClass::PERM_SWAP && g.cls != GClass::DIAG))
+    return false;
+  // two 2-target gates on the same pair
+  const long k = last_touching(gq);
+  if (k >= 0) {
+    Decoded& a = prog[k];
+    if (a.m == 2 && a.cmask == g.cmask && qubit_mask(a) == gq &&
+        (a.cls == GClass::DENSE || g.cls == GClass::DENSE)) {
+      cplx G[16], P[16];
+      if (a.targets[0] == g.targets[0])
+        for (int i = 0; i < 16; ++i) G[i] = g.M[i];
+      else
+        swap_bits4(g.M, G);
+      mat4_mul(G, a.M, P);
+      if (nnz_of(P, 4) <= nnz_of(a.M, 4) + nnz_of(G, 4)) {
+        set_dense4(a, P);
+        return true;
+      }
+    }
+  }
+  // dense 1-target gates on g's targets right before it (nothing in between touches
+  // their qubits): g . (U0 (x) U1)
+  long ks[2] = {-1, -1};
+  int cost_sep = nnz_of(g.M, 4);
+  cplx P[16];
+  for (int i = 0; i < 16; ++i) P[i] = g.M[i];
+  for (int s2 = 0; s2 < 2; ++s2) {
+    const uint64_t q = (1ull << g.targets[s2]) | g.cmask;
+    const long j = last_touching(q);
+    if (j < 0) continue;
+    const Decoded& u = prog[j];
+    if (u.m != 1 || u.cls != GClass::DENSE || u.cmask != g.cmask || u.targets[0] != g.targets[s2])
+      continue;
+    cplx E[16], T[16];
+    embed2(u.M, s2 == 0, E);
+    mat4_mul(P, E, T);
+    for (int i = 0; i < 16; ++i) P[i] = T[i];
+    cost_sep += 2 * nnz_of(u.M, 2);
+    ks[s2] = j;
+  }
+  if (ks[0] < 0 && ks[1] < 0) return false;
+  if (nnz_of(P, 4) > cost_sep) return false;
+  for (long j : ks)
+    if (j >= 0) prog[j].cls = GClass::NOOP;  // absorbed into g
+  set_dense4(g, P);
+  prog.push_back(g);
+  return true;
+}
+
 // Builds the tile geometry for qubit set in_tile (filled up to K qubits), merges
 // same-qubit 1-target runs containing a dense gate, and encodes the program.
 void build_program(const LaunchCtx& ctx, const TileCfg& cfg, uint64_t in_tile,
@@ -931,20 +1048,25 @@ void build_program(const LaunchCtx& ctx, const TileCfg& cfg, uint64_t in_tile,
   // one dense layer.
   std::vector<Decoded> prog;
   prog.reserve(list.size());
+  // index of the last live gate of prog touching any qubit in mask (within 256), or -1
+  auto last_touching = [&](uint64_t mask) -> long {
+    for (size_t k = prog.size(); k-- > 0 && prog.size() - k <= 256;)
+      if (prog[k].cls != GClass::NOOP && (qubit_mask(prog[k]) & mask)) return (long)k;
+    return -1;
+  };
   for (const Decoded* gp : list) {
-    const Decoded& g = *gp;
-    if (g.cls == GClass::NOOP) continue;
+    if (gp->cls == GClass::NOOP) continue;
+    Decoded g = *gp;
+    if (ctx.opt->fuse_merge_2q && merge_2q(prog, g, last_touching)) continue;
     if (!prog.empty()) {
       size_t ai = prog.size() - 1;
       if (ctx.opt->fuse_merge_commuting && g.m == 1) {
-        const uint64_t gq = qubit_mask(g);
-        for (size_t k = prog.size(); k-- > 0 && prog.size() - k <= 256;) {
-          ai = k;
-          if (qubit_mask(prog[k]) & gq) break;
-        }
+        const long k = last_touching(qubit_mask(g));
+        if (k >= 0) ai = (size_t)k;
       }
       Decoded& a = prog[ai];
-      if (a.m == 1 && g.m == 1 && a.targets[0] == g.targets[0] && a.cmask == g.cmask &&
+      if (a.cls != GClass::NOOP && a.m == 1 && g.m == 1 && a.targets[0] == g.targets[0] &&
+          a.cmask == g.cmask &&
           (a.cls == GClass::DENSE || g.cls == GClass::DENSE)) {
         cplx Cm[4];
         for (int r = 0; r < 2; ++r)

@@ -164,3 +164,57 @@ def test_fused_lane_bit_dense_1q(L, low, tma):
             out[fuse] = st.copy_out()
     assert np.max(np.abs(out[True] - ref)) <= 1e-12
     assert np.array_equal(out[True], out["jit"])
+
+
+def _merge2q_cases(n):
+    """Every shape the 2-target merge handles, and some it must refuse."""
+    U = lambda s: W.haar_unitary(1, s)  # noqa: E731
+    U4 = lambda s: W.haar_unitary(2, s)  # noqa: E731
+    fsim = W.fsim(np.pi / 2, np.pi / 6)
+    g = []
+    g += [W.Gate("UNITARY2", (3, 7), (), (), U4(1)), W.Gate("UNITARY1", (3,), (), (), U(2)),
+          W.Gate("H", (7,)), W.Gate("RX", (7,), (), (0.4,))]           # 1q after a U4 (both)
+    g += [W.Gate("U3", (1,), (), (0.3, 0.2, 0.1)), W.Gate("RY", (9,), (), (1.1,)),
+          W.Gate("T", (4,)), W.Gate("UNITARY2", (9, 1), (), (), fsim)]  # 1q before fSim
+    g += [W.Gate("UNITARY2", (9, 1), (), (), fsim),                     # same pair, reversed
+          W.Gate("UNITARY2", (1, 9), (), (), U4(3))]
+    g += [W.Gate("SWAP", (2, 5)), W.Gate("H", (5,)), W.Gate("H", (2,))]  # SWAP absorbs 1q
+    g += [W.Gate("UNITARY2", (0, 6), (8,), (), U4(4)),                  # same controls
+          W.Gate("UNITARY1", (6,), (8,), (), U(5)),
+          W.Gate("UNITARY1", (0,), (), (), U(6))]                       # different controls
+    g += [W.Gate("UNITARY2", (10, 11), (), (), U4(7)), W.CNOT(2, 10),   # blocked by CNOT
+          W.Gate("H", (10,)), W.Gate("H", (11,))]
+    g += W.sycamore_like(2, n // 2, 4, seed=8)
+    return g
+
+
+@pytest.mark.parametrize("fuse", [True, "jit", "jit+phase"])
+def test_merge_2q_matches_oracle_and_unmerged(L, fuse):
+    """LFQS_OPT_FUSE_MERGE_2Q: dense 1-target gates folded into neighbouring 2-target gates
+    (both orders, SWAP, same-pair products, controlled) equal the oracle within 1e-12 and
+    the unmerged fused run within rounding; the interpreter and the pass compiler agree
+    bit for bit; permutation / diagonal circuits stay bit-exact."""
+    n = 12
+    psi = W.random_state(n, 17)
+    gates = _merge2q_cases(n)
+    ref = O.run_circuit(n, gates, psi.copy())
+    outs = {}
+    for m2 in (0, 1):
+        with L.State.create(n) as st:
+            st.set_option(L.OPT_FUSE_MERGE_2Q, m2)
+            st.copy_in(psi)
+            st.run_circuit(gates, fuse=fuse)
+            outs[m2] = st.copy_out()
+        assert np.max(np.abs(outs[m2] - ref)) <= 1e-12, m2
+    assert np.max(np.abs(outs[0] - outs[1])) <= 1e-13
+    if fuse == "jit":
+        with L.State.create(n) as st:  # interpreter with the same merges
+            st.copy_in(psi)
+            st.run_circuit(gates, fuse=True)
+            assert np.array_equal(st.copy_out(), outs[1])
+    exact = [W.Gate("SWAP", (2, 5)), W.CNOT(5, 2), W.Gate("X", (2,)), W.Gate("SWAP", (5, 2)),
+             W.CZ(1, 3), W.Gate("S", (5,))] * 5
+    with L.State.create(n) as st:
+        st.copy_in(psi)
+        st.run_circuit(exact, fuse=fuse)
+        assert np.array_equal(st.copy_out(), O.run_circuit(n, exact, psi.copy()))
