@@ -311,6 +311,55 @@ def run_macro(lfqs, stream, n: int, reps: int, unfused: bool, hbm_peak: float):
 
 
 # ----------------------------------------------------------------------------
+# configs[0]: the 10-qubit micro-benchmark gates (launch-bound regime)
+# ----------------------------------------------------------------------------
+
+def cpu_baseline_small(n, gates, psi):
+    """configs[0]'s cpu_baseline: the oracle (tier B, one host thread) on the whole
+    470-gate circuit; its result is also the reference the GPU runs are checked against."""
+    import oracle
+    t0 = time.perf_counter()
+    ref = oracle.run_circuit(n, gates, psi.copy())
+    return ref, {"kind": "oracle", "cores": 1,
+                 "us_per_gate": (time.perf_counter() - t0) / len(gates) * 1e6}
+
+
+def run_small(lfqs, stream, with_oracle: bool, reps: int = 50):
+    """configs[0] (n = 10: H and Rz on every qubit, CNOT on every ordered pair, Toffoli on
+    every (c1 < c2, t); 470 gates): per-gate class kernels replayed from a CUDA graph, and
+    the compiled fused passes replayed from a CUDA graph, CUDA events over `reps` replays;
+    each checked against the oracle's result on the same seeded state (cpu_baseline_small)."""
+    import torch
+    n = 10
+    gates = W.micro_gates_10q(n)
+    psi = W.random_state(n, 0x1F5)
+    arr = lfqs.marshal_gates(gates)
+    out = {"config": "configs[0]", "n": n, "gates": len(gates)}
+    ref = None
+    if with_oracle:
+        ref, out["cpu_baseline"] = cpu_baseline_small(n, gates, psi)
+    with lfqs.State.create(n, 0, stream=stream) as st:
+        lfqs.lfqs_jit_precompile(n, arr, "jit")
+        for mode, fuse in (("graph_per_gate", False), ("graph_compiled_passes", "jit")):
+            st.copy_in(psi)
+            with st.compile(arr, fuse=fuse) as c:
+                c.launch()
+                err = None if ref is None else float(np.max(np.abs(st.copy_out() - ref)))
+                torch.cuda.synchronize()
+                a = torch.cuda.Event(enable_timing=True)
+                b = torch.cuda.Event(enable_timing=True)
+                a.record(stream)
+                for _ in range(reps):
+                    c.launch()
+                b.record(stream)
+                torch.cuda.synchronize()
+                t = a.elapsed_time(b) / 1e3 / reps
+                out[mode] = {"us_per_gate": t / len(gates) * 1e6, "gates_per_s": len(gates) / t,
+                             "kernels_per_circuit": int(c.kernels), "max_abs_err_vs_oracle": err}
+    return out
+
+
+# ----------------------------------------------------------------------------
 # N > 1: QFT(n_local + log2 N) sharded across the ranks (configs[4] shape)
 # ----------------------------------------------------------------------------
 
@@ -400,6 +449,7 @@ def main():
                     help="configs[2] leg at N = 1: QFT and GHZ at this many qubits after the "
                          "sweep (0: skip)")
     ap.add_argument("--macro-reps", type=int, default=3)
+    ap.add_argument("--no-small", action="store_true", help="skip the configs[0] leg")
     ap.add_argument("--no-macro-unfused", action="store_true",
                     help="skip the strict one-pass-per-gate QFT/GHZ runs of the macro leg")
     ap.add_argument("--qft-reps", type=int, default=3,
@@ -635,6 +685,10 @@ def main():
                       "lfqs_measure_probs"}
         del host
 
+    small = None
+    if world == 1 and not args.no_small:
+        small = run_small(lfqs, stream, with_oracle=not args.no_cpu_baseline)
+
     macro = None
     if world == 1 and args.macro_n > 0:
         st.close()
@@ -667,6 +721,7 @@ def main():
             "roofline": roofline,
             "worst_gate": worst_gate,
             "macro": macro,
+            "small": small,
             "qft_sharded": qft,
             "nvlink": nvlink,
             "classes": {k: {kk: (round(vv, 4) if isinstance(vv, float) else vv)
