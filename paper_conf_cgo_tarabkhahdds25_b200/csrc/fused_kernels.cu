@@ -900,15 +900,27 @@ void merge_phase_runs(FProg& P, bool split) {
 // A dense 1-target gate next to a 2-target gate on a superset of its qubit (nothing in
 // between touches it, so they are adjacent in the commuting order, Eq. 3) is folded
 // into the 4x4 matrix on the host, and two 2-target gates on the same pair are multiplied,
-// when the product costs no more complex multiply-adds per amplitude than the gates did
-// separately (nonzeros / 4 for a 4x4, nonzeros / 2 for a 2x2).  Sycamore-like cycles (a
+// when the product costs fewer FP64 operations per amplitude than the gates did separately
+// (cost_of).  Sycamore-like cycles (a
 // dense 1-target gate on each qubit, then fSim on pairs) lose about a quarter of their FP64
 // work; the heavy passes are FP64-bound (profiles/r02_heavy_passes.md).  Rounding changes
 // only (dense tolerance class); permutation / diagonal-only pairs never merge.
-int nnz_of(const cplx* M, int d) {
+// FP64 operations per amplitude of a d x d gate matrix as the kernels evaluate it: each
+// coefficient costs 2 per nonzero real / imaginary part (x2 for the amplitude's two
+// components), a coefficient +-1 or +-i is a move / negation (1), zeros cost nothing; a
+// permutation class gate is pure moves (0).
+int cost_of(const cplx* M, int d, GClass cls) {
+  if (cls == GClass::PERM_X || cls == GClass::PERM_Y || cls == GClass::PERM_SWAP) return 0;
   int c = 0;
-  for (int i = 0; i < d * d; ++i) c += (M[i].re != 0.0 || M[i].im != 0.0);
-  return c;
+  for (int i = 0; i < d * d; ++i) {
+    const double re = M[i].re, im = M[i].im;
+    if (re == 0.0 && im == 0.0) continue;
+    if ((im == 0.0 && (re == 1.0 || re == -1.0)) || (re == 0.0 && (im == 1.0 || im == -1.0)))
+      c += 1;
+    else
+      c += 2 * (re != 0.0) + 2 * (im != 0.0);
+  }
+  return c * 4 / d;  // x4: per amplitude in units of 1/4 (integer arithmetic)
 }
 void mat4_mul(const cplx* A, const cplx* B, cplx* C) {  // C = A B (row-major 4x4)
   for (int r = 0; r < 4; ++r)
@@ -959,7 +971,8 @@ bool merge_2q(std::vector<Decoded>& prog, Decoded& g, LastTouching&& last_touchi
     cplx E[16], P[16];
     embed2(g.M, a.targets[0] == g.targets[0], E);
     mat4_mul(E, a.M, P);
-    if (nnz_of(P, 4) > nnz_of(a.M, 4) + 2 * nnz_of(g.M, 2)) return false;
+    if (cost_of(P, 4, GClass::DENSE) >= cost_of(a.M, 4, a.cls) + cost_of(g.M, 2, g.cls))
+      return false;
     set_dense4(a, P);
     return true;
   }
@@ -977,7 +990,7 @@ bool merge_2q(std::vector<Decoded>& prog, Decoded& g, LastTouching&& last_touchi
       else
         swap_bits4(g.M, G);
       mat4_mul(G, a.M, P);
-      if (nnz_of(P, 4) <= nnz_of(a.M, 4) + nnz_of(G, 4)) {
+      if (cost_of(P, 4, GClass::DENSE) < cost_of(a.M, 4, a.cls) + cost_of(G, 4, g.cls)) {
         set_dense4(a, P);
         return true;
       }
@@ -986,7 +999,7 @@ bool merge_2q(std::vector<Decoded>& prog, Decoded& g, LastTouching&& last_touchi
   // dense 1-target gates on g's targets right before it (nothing in between touches
   // their qubits): g . (U0 (x) U1)
   long ks[2] = {-1, -1};
-  int cost_sep = nnz_of(g.M, 4);
+  int cost_sep = cost_of(g.M, 4, g.cls);
   cplx P[16];
   for (int i = 0; i < 16; ++i) P[i] = g.M[i];
   for (int s2 = 0; s2 < 2; ++s2) {
@@ -1000,11 +1013,11 @@ bool merge_2q(std::vector<Decoded>& prog, Decoded& g, LastTouching&& last_touchi
     embed2(u.M, s2 == 0, E);
     mat4_mul(P, E, T);
     for (int i = 0; i < 16; ++i) P[i] = T[i];
-    cost_sep += 2 * nnz_of(u.M, 2);
+    cost_sep += cost_of(u.M, 2, u.cls);
     ks[s2] = j;
   }
   if (ks[0] < 0 && ks[1] < 0) return false;
-  if (nnz_of(P, 4) > cost_sep) return false;
+  if (cost_of(P, 4, GClass::DENSE) >= cost_sep) return false;
   for (long j : ks)
     if (j >= 0) prog[j].cls = GClass::NOOP;  // absorbed into g
   set_dense4(g, P);
