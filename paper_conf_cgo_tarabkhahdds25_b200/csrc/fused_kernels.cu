@@ -956,8 +956,39 @@ void set_dense4(Decoded& a, const cplx* M) {
   a.kind = LFQS_UNITARY2;
 }
 
+// A 1-target gate with exactly one control as the 2-target gate it is on (control, target):
+// |0><0| (x) I + |1><1| (x) U, control = local bit 1 (targets[0]).
+Decoded as_two_target(const Decoded& g) {
+  Decoded h = g;
+  const int c = __builtin_ctzll(g.cmask);
+  h.m = 2;
+  h.targets[0] = c;
+  h.targets[1] = g.targets[0];
+  h.targets[2] = 0;
+  h.cmask = 0;
+  h.is_h = false;
+  h.kind = LFQS_UNITARY2;
+  for (int i = 0; i < 16; ++i) h.M[i] = cplx{0.0, 0.0};
+  h.M[0] = h.M[5] = cplx{1.0, 0.0};
+  for (int r = 0; r < 2; ++r)
+    for (int q = 0; q < 2; ++q) h.M[(2 + r) * 4 + 2 + q] = g.M[r * 2 + q];
+  return h;
+}
+
 template <class LastTouching>
-bool merge_2q(std::vector<Decoded>& prog, Decoded& g, LastTouching&& last_touching) {
+bool merge_2q(std::vector<Decoded>& prog, Decoded& g, LastTouching&& last_touching,
+              const TileMap& tm) {
+  if (g.m == 1 && __builtin_popcountll(g.cmask) == 1) {
+    // CZ / CNOT / CPhase / CU: merge in its 4x4 form when that pays (e.g. the dense
+    // 1-target gates on both its qubits right before it); otherwise it stays as it is.
+    Decoded h = as_two_target(g);
+    return merge_2q(prog, h, last_touching, tm);
+  }
+  // A merged gate is dense: both of its targets must be tile qubits (diagonal gates may
+  // act on qubits outside the tile, read from the tile index, a dense one may not).
+  auto in_tile2 = [&](const Decoded& x) {
+    return x.m == 2 && tm.tb[x.targets[0]] >= 0 && tm.tb[x.targets[1]] >= 0;
+  };
   const uint64_t gq = qubit_mask(g);
   if (g.m == 1 && g.cls == GClass::DENSE) {
     // g after a 2-target gate a on (a0, a1) that g's target belongs to
@@ -966,7 +997,7 @@ bool merge_2q(std::vector<Decoded>& prog, Decoded& g, LastTouching&& last_touchi
     Decoded& a = prog[k];
     const int t = g.targets[0];
     if (a.m != 2 || a.cmask != g.cmask || (a.targets[0] != t && a.targets[1] != t) ||
-        (a.cls != GClass::DENSE && a.cls != GClass::PERM_SWAP && a.cls != GClass::DIAG))
+        !in_tile2(a))
       return false;
     cplx E[16], P[16];
     embed2(g.M, a.targets[0] == g.targets[0], E);
@@ -976,8 +1007,7 @@ bool merge_2q(std::vector<Decoded>& prog, Decoded& g, LastTouching&& last_touchi
     set_dense4(a, P);
     return true;
   }
-  if (g.m != 2 || (g.cls != GClass::DENSE && g.cls != GClass::PERM_SWAP && g.cls != GClass::DIAG))
-    return false;
+  if (g.m != 2 || g.cls == GClass::NOOP || !in_tile2(g)) return false;
   // two 2-target gates on the same pair
   const long k = last_touching(gq);
   if (k >= 0) {
@@ -1070,7 +1100,7 @@ void build_program(const LaunchCtx& ctx, const TileCfg& cfg, uint64_t in_tile,
   for (const Decoded* gp : list) {
     if (gp->cls == GClass::NOOP) continue;
     Decoded g = *gp;
-    if (ctx.opt->fuse_merge_2q && merge_2q(prog, g, last_touching)) continue;
+    if (ctx.opt->fuse_merge_2q && merge_2q(prog, g, last_touching, tm)) continue;
     if (!prog.empty()) {
       size_t ai = prog.size() - 1;
       if (ctx.opt->fuse_merge_commuting && g.m == 1) {

@@ -109,3 +109,17 @@ def test_fused_coefficient_budget_counts_merged_gates(lib):
     for rep in range(14):   # X(0) H(0) merge into one U2: 4 coefficients (budgeted 0 + 1 before)
         gates += [W.CNOT(1, 0), W.Gate("X", (0,)), W.Gate("H", (0,))]
     assert L.lfqs_jit_precompile(n, gates, "jit") >= 2
+
+
+@pytest.mark.parametrize("n", [12, 20])
+def test_jit_compiles_merged_programs(lib, n):
+    """Host-only: every fused pass of circuits exercising the 2-target merges (controlled
+    gates in 4x4 form, diagonals acting outside the tile, same-pair products) generates PTX
+    that ptxas accepts (a dense merged gate on a qubit outside the tile would not)."""
+    import workloads as W
+    for s in range(3):
+        for g in (W.random_gate_list(n, 300, seed=s, max_controls=2),
+                  W.sycamore_like(2, n // 2, 6, seed=s), W.random_layered(n, 6, seed=s),
+                  W.qft(n) + W.grover(n, 5, 1)):
+            for mode in ("jit", "jit+phase"):
+                assert L.lfqs_jit_precompile(n, g, mode) >= 1
