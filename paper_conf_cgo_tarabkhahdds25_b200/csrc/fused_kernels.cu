@@ -1016,6 +1016,9 @@ Decoded as_two_target(const Decoded& g) {
 template <class LastTouching>
 bool merge_2q(std::vector<Decoded>& prog, Decoded& g, LastTouching&& last_touching,
               const TileMap& tm) {
+  // Diagonal gates are left alone: they are nearly free inside a pass (phase tables fold
+  // whole runs of them into one lookup) and stay exact.
+  if (g.cls == GClass::DIAG) return false;
   if (g.m == 1 && __builtin_popcountll(g.cmask) == 1) {
     // CZ / CNOT / CPhase / CU: merge in its 4x4 form when that pays (e.g. the dense
     // 1-target gates on both its qubits right before it); otherwise it stays as it is.
@@ -1035,7 +1038,7 @@ bool merge_2q(std::vector<Decoded>& prog, Decoded& g, LastTouching&& last_touchi
     Decoded& a = prog[k];
     const int t = g.targets[0];
     if (a.m != 2 || a.cmask != g.cmask || (a.targets[0] != t && a.targets[1] != t) ||
-        !in_tile2(a))
+        !in_tile2(a) || a.cls == GClass::DIAG)
       return false;
     cplx E[16], P[16];
     embed2(g.M, a.targets[0] == g.targets[0], E);
@@ -1050,7 +1053,7 @@ bool merge_2q(std::vector<Decoded>& prog, Decoded& g, LastTouching&& last_touchi
   const long k = last_touching(gq);
   if (k >= 0) {
     Decoded& a = prog[k];
-    if (a.m == 2 && a.cmask == g.cmask && qubit_mask(a) == gq &&
+    if (a.m == 2 && a.cmask == g.cmask && qubit_mask(a) == gq && a.cls != GClass::DIAG &&
         (a.cls == GClass::DENSE || g.cls == GClass::DENSE)) {
       cplx G[16], P[16];
       if (a.targets[0] == g.targets[0])
