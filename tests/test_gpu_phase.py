@@ -87,10 +87,16 @@ def test_phase_tables_diag_heavy(L, n, tile, low, split):
 @pytest.mark.parametrize("n", [10, 16, 20])
 def test_phase_tables_qft_closed_form(L, n):
     x = (0x9E3779B97F4A7C15 >> (64 - n)) | 1
+    """QFT rows make separable tables (every member a CPhase on one table bit besides the
+    common target bit): built from per-bit factors, interpreter == compiled bit for bit."""
     with L.State.create(n) as st:
         st.init_basis(x)
         st.run_circuit(W.qft(n), fuse="phase")
         a = st.copy_out()
+        st.init_basis(x)
+        st.run_circuit(W.qft(n), fuse="jit+phase")
+        b = st.copy_out()
+    assert np.array_equal(a, b)
     y = np.arange(1 << n, dtype=np.int64)
     ref = np.exp(2j * np.pi * ((x * y) % (1 << n)) / (1 << n)) / np.sqrt(1 << n)
     assert np.max(np.abs(a - ref)) <= 1e-12
