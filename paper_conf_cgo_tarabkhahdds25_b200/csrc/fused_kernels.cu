@@ -462,9 +462,11 @@ __global__ void __launch_bounds__(kFThreads, sizeof(S) == 4 ? 4 : 2) k_fused(cx<
       const int nb = __popc(U);
       __syncthreads();  // the previous table's readers (and tile writers) are done
       if (h.pad0 & kDtabSeparable) {
-        // separable table (separable_table): thread s < 2 nb + 1 multiplies the factors of
-        // slot s (2 b + v: members fixing table bit b to v; 2 nb: members fixing none)
-        if (tid < 2u * nb + 1u) {
+        // separable table (separable_table): slot s (2 b + v: members fixing table bit b to
+        // v; 2 nb: members fixing none) is multiplied out by thread (s mod 8) * 32 + s / 8
+        // -- one lane of each warp, so the slots' chains run on different warps
+        const uint32_t slot_me = (tid & 31u) * 8u + (tid >> 5);
+        if ((tid & 31u) < 3u && slot_me < 2u * nb + 1u) {
           C t = mk<S>(1, 0);
           for (int j = 1; j <= nm; ++j) {
             const FHdr& g = prog.h[o + j];
@@ -472,11 +474,11 @@ __global__ void __launch_bounds__(kFThreads, sizeof(S) == 4 ? 4 : 2) k_fused(cx<
             const uint32_t rel = g.mlo & U;
             const uint32_t slot =
                 rel ? 2u * __popc(U & (rel - 1)) + ((g.plo & rel) ? 1u : 0u) : 2u * nb;
-            if (slot != tid) continue;
+            if (slot != slot_me) continue;
             const C d = cvs<S>(prog.c[g.coef]);
             if (!is_one(d)) t = cmul_fma(d, t);
           }
-          dsep[tid] = t;
+          dsep[slot_me] = t;
         }
         __syncthreads();
         if (tid < (1u << nb)) {
@@ -877,7 +879,7 @@ bool tile_dependent(const FHdr& h) {
 // control lies outside the tile) adds no table bits, but every table entry evaluates it;
 // grouped apart, such members usually share their in-tile bits as a common predicate and
 // form a table of very few entries, so the per-tile build does ~1/256 of the work.
-void merge_phase_runs(FProg& P, bool split) {
+void merge_phase_runs(FProg& P, bool split, bool separable) {
   static thread_local FHdr out[kMaxOps];
   static thread_local FHdr run[kMaxOps];
   int no = 0, o = 0;
@@ -920,7 +922,7 @@ void merge_phase_runs(FProg& P, bool split) {
           t.m = (uint8_t)(j - i);
           t.mlo = sup & ~cm;
           t.plo = cm | (cp << 16);
-          t.pad0 = separable_table(run + i, j - i, t.mlo) ? kDtabSeparable : 0;
+          t.pad0 = separable && separable_table(run + i, j - i, t.mlo) ? kDtabSeparable : 0;
           out[no++] = t;
           --spare;
         }
@@ -1170,7 +1172,8 @@ void build_program(const LaunchCtx& ctx, const TileCfg& cfg, uint64_t in_tile,
     prog.push_back(g);
   }
   for (const Decoded& g : prog) encode(g, tm, P);
-  if (ctx.phase_tables) merge_phase_runs(P, ctx.opt->fuse_phase_split);
+  if (ctx.phase_tables)
+    merge_phase_runs(P, ctx.opt->fuse_phase_split, ctx.opt->fuse_phase_separable);
 }
 
 // Launches an encoded pass: the compiled kernel of its program (LFQS_FUSE_JIT)

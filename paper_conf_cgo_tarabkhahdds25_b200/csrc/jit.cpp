@@ -1023,9 +1023,10 @@ struct Gen {
                            : 2 * nb;
         slot[sl].push_back(o + j);
       }
+      const int nw = NT / 32;  // slot sl on thread (sl mod nw) * 32 + sl / nw
       for (int sl = 0; sl <= 2 * nb; ++sl) {
         const std::string skip = L(), q = p();
-        e("setp.ne.u32 %s, %%ltid, %d;", q.c_str(), sl);
+        e("setp.ne.u32 %s, %%ltid, %d;", q.c_str(), (sl % nw) * 32 + sl / nw);
         e("@%s bra %s;", q.c_str(), skip.c_str());
         Cx t{f(), f()};
         e("mov.%s %s, %s;", FT, t.x.c_str(), c64 ? "0f3F800000" : "0d3FF0000000000000");
