@@ -441,11 +441,6 @@ lfqs_status lfqs_state_pass_count(const lfqs_state* s, uint64_t* passes);
                                      multiply-adds per amplitude than the separate gates
                                      (e.g. Sycamore-like 1-target layers into fSim).
                                      Rounding changes only (dense tolerance class) */
-#define LFQS_OPT_FUSE_PHASE_SEPARABLE 23 /* 1 (default): a phase table whose members are all
-                                     one-entry diagonals fixing at most one table bit (QFT
-                                     rows) is built per tile from per-bit factor products
-                                     instead of evaluating every member for every entry.
-                                     Rounding order only (phase-table tolerance) */
 lfqs_status lfqs_set_option(lfqs_state* s, int option, int64_t value);
 const char* lfqs_last_error(void);
 int lfqs_abi_version(void);

@@ -52,7 +52,6 @@ OPT_LINE_READS = 19
 OPT_EXCHANGE_CHUNK_BITS = 20
 OPT_EXCHANGE_CTAS = 21
 OPT_FUSE_MERGE_2Q = 22
-OPT_FUSE_PHASE_SEPARABLE = 23
 
 STATUS = {0: "OK", -1: "INVALID_ARG", -2: "OUT_OF_MEMORY", -3: "CUDA", -4: "NCCL",
           -5: "UNSUPPORTED"}

@@ -522,7 +522,6 @@ lfqs_status lfqs_set_option(lfqs_state* s, int option, int64_t value) {
       case LFQS_OPT_WIDE256: st->opt.wide256 = value != 0; break;
       case LFQS_OPT_LINE_READS: st->opt.line_reads = value != 0; break;
       case LFQS_OPT_FUSE_MERGE_2Q: st->opt.fuse_merge_2q = value != 0; break;
-      case LFQS_OPT_FUSE_PHASE_SEPARABLE: st->opt.fuse_phase_separable = value != 0; break;
       case LFQS_OPT_EXCHANGE_CHUNK_BITS:
         require(value >= 0 && value <= 4, "LFQS_OPT_EXCHANGE_CHUNK_BITS must be in [0, 4]");
         st->opt.exchange_chunk_bits = (int)value;  // the plan is the same for every value

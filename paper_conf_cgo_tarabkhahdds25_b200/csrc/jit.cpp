@@ -1010,65 +1010,8 @@ struct Gen {
     const uint32_t U = h.mlo, cm = h.plo & 0xffffu, cp = h.plo >> 16;
     const int nb = __builtin_popcount(U);
     sync();
-    if (h.pad0 & kDtabSeparable) {
-      // Separable table (fused_kernels.cu separable_table, same order of operations as
-      // k_fused): thread s multiplies the factors of slot s -- members fixing table bit b
-      // to v (s = 2 b + v) or no table bit (s = 2 nb) -- in member order; then entry e =
-      // C x F[0][e_0] x F[1][e_1] ...
-      std::vector<std::vector<int>> slot(2 * nb + 1);
-      for (int j = 1; j <= nm; ++j) {
-        const FHdr& g = P.h[o + j];
-        const uint32_t rel = g.mlo & U;
-        const int sl = rel ? 2 * __builtin_popcount(U & (rel - 1)) + ((g.plo & rel) ? 1 : 0)
-                           : 2 * nb;
-        slot[sl].push_back(o + j);
-      }
-      const int nw = NT / 32;  // slot sl on thread (sl mod nw) * 32 + sl / nw
-      for (int sl = 0; sl <= 2 * nb; ++sl) {
-        const std::string skip = L(), q = p();
-        e("setp.ne.u32 %s, %%ltid, %d;", q.c_str(), (sl % nw) * 32 + sl / nw);
-        e("@%s bra %s;", q.c_str(), skip.c_str());
-        Cx t{f(), f()};
-        e("mov.%s %s, %s;", FT, t.x.c_str(), c64 ? "0f3F800000" : "0d3FF0000000000000");
-        e("mov.%s %s, %s;", FT, t.y.c_str(), zero().c_str());
-        for (int oj : slot[sl]) {
-          const FHdr& g = P.h[oj];
-          const Cx d = coef(g.coef);
-          if (d.vx == 1.0 && d.vy == 0.0) continue;  // is_one: skipped as in k_fused
-          const std::string ms = L();
-          tile_pred(g.mhi, g.phi, ms);
-          assign(t.x, t.y, cmulf(d, t));
-          label(ms);
-        }
-        const std::string a = r();
-        e("mov.u32 %s, lfqs_dsep;", a.c_str());
-        sts(a, t, sl * ES);
-        label(skip);
-      }
-      sync();
-      for (int k = 0; k * NT < (1 << nb); ++k) {
-        const std::string skip = L(), q = p(), eid = r();
-        e("add.u32 %s, %%ltid, %d;", eid.c_str(), k * NT);
-        e("setp.ge.u32 %s, %s, %u;", q.c_str(), eid.c_str(), 1u << nb);
-        e("@%s bra %s;", q.c_str(), skip.c_str());
-        const std::string ds = r();
-        e("mov.u32 %s, lfqs_dsep;", ds.c_str());
-        Cx t = lds(ds, 2 * nb * ES);
-        for (int b = 0; b < nb; ++b) {
-          const std::string bit = r(), ad = r();
-          e("bfe.u32 %s, %s, %d, 1;", bit.c_str(), eid.c_str(), b);
-          e("mad.lo.u32 %s, %s, %d, %s;", ad.c_str(), bit.c_str(), ES, ds.c_str());
-          const Cx fb = lds(ad, 2 * b * ES);
-          t = cmulf(fb, t);
-        }
-        const std::string a = r();
-        e("mad.lo.u32 %s, %s, %d, %%dtab;", a.c_str(), eid.c_str(), ES);
-        sts(a, t);
-        label(skip);
-      }
-    }
     // Entry e of the table is built by thread e mod NT (entries e = ltid + k NT).
-    for (int k = 0; !(h.pad0 & kDtabSeparable) && k * NT < (1 << nb); ++k) {
+    for (int k = 0; k * NT < (1 << nb); ++k) {
       const std::string skip = L(), q = p(), eid = r();
       e("add.u32 %s, %%ltid, %d;", eid.c_str(), k * NT);
       e("setp.ge.u32 %s, %s, %u;", q.c_str(), eid.c_str(), 1u << nb);
@@ -1752,8 +1695,7 @@ struct Gen {
     out += ".version 8.7\n.target sm_100a\n.address_size 64\n\n";
     out += ".extern .shared .align 128 .b8 lfqs_tile[];\n";
     out += ".shared .align 8 .b64 lfqs_bar;\n";
-    out += ".shared .align 16 .b8 lfqs_dtab[" + std::to_string(256 * ES) + "];\n";
-    out += ".shared .align 16 .b8 lfqs_dsep[" + std::to_string(17 * ES) + "];\n\n";
+    out += ".shared .align 16 .b8 lfqs_dtab[" + std::to_string(256 * ES) + "];\n\n";
     const int nc = P.ncoef > 0 ? P.ncoef : 1;
     out += ".visible .entry lfqs_jit(.param .u64 pa, .param .u64 poff, .param .align 16 .b8 pc[" +
            std::to_string(nc * 16) + "])\n";
