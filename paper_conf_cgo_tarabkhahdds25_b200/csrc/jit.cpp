@@ -1004,13 +1004,41 @@ struct Gen {
     label(skip);
   }
 
-  void op_dtab(int o) {
+  // Phase tables built in the prologue, while the tile's TMA load is in flight: a table
+  // depends only on the tile index and the coefficients, never on amplitudes, so every
+  // table of the pass that fits is built before the first barrier and
+  // each F_DTAB op is then a lookup pass with no barrier of its own (the build latency and
+  // two barriers per table hide behind the load).  Entries beyond prebuild_entries() are
+  // built in place as before.  Entries and arithmetic are exactly
+  // op_dtab's / k_fused's, so results stay bit-identical to the interpreter.
+  // Table entries built in the prologue: 32 KiB (complex128: 2 CTAs per SM with the 64 KiB
+  // tile) or 8 KiB (complex64: 4 CTAs per SM with the 32 KiB tile).
+  int prebuild_entries() const { return c64 ? 1024 : 2048; }
+  std::map<int, int> dtab_off;  // prebuilt F_DTAB op -> entry offset in lfqs_dtab
+  int dtab_pre = 0;             // entries of the prebuilt tables
+  bool dtab_dyn = false;        // some table is built in place (after the prebuilt ones)
+  void plan_prebuild() {
+    for (int o = 0; o < P.nops; ++o) {
+      const FHdr& h = P.h[o];
+      if (h.type != F_DTAB) continue;
+      const int sz = 1 << __builtin_popcount(h.mlo);
+      if (dtab_pre + sz <= prebuild_entries()) {
+        dtab_off[o] = dtab_pre;
+        dtab_pre += sz;
+      } else {
+        dtab_dyn = true;
+      }
+      o += h.m;
+    }
+  }
+  int dtab_entries() const { return std::max(dtab_pre + (dtab_dyn ? 256 : 0), 1); }
+
+  // Builds table `o` into lfqs_dtab entries [off, off + 2^nb): entry e by thread e mod NT.
+  void dtab_build(int o, int off) {
     const FHdr& h = P.h[o];
     const int nm = h.m;
-    const uint32_t U = h.mlo, cm = h.plo & 0xffffu, cp = h.plo >> 16;
+    const uint32_t U = h.mlo, cp = h.plo >> 16;
     const int nb = __builtin_popcount(U);
-    sync();
-    // Entry e of the table is built by thread e mod NT (entries e = ltid + k NT).
     for (int k = 0; k * NT < (1 << nb); ++k) {
       const std::string skip = L(), q = p(), eid = r();
       e("add.u32 %s, %%ltid, %d;", eid.c_str(), k * NT);
@@ -1032,18 +1060,32 @@ struct Gen {
       for (int j = 1; j <= nm; ++j) dtab_member(P.h[o + j], ie, t);
       const std::string a = r();
       e("mad.lo.u32 %s, %s, %d, %%dtab;", a.c_str(), eid.c_str(), ES);
-      sts(a, t);
+      sts(a, t, off * ES);
       label(skip);
     }
-    if (!in_regs) {
-      if (greedy && nreg >= 1) {
-        place(plan_set(o + nm + 1), o + nm + 1);
-        emit_taddr();
+  }
+
+  void op_dtab(int o) {
+    const FHdr& h = P.h[o];
+    const int nm = h.m;
+    const uint32_t U = h.mlo, cm = h.plo & 0xffffu, cp = h.plo >> 16;
+    const auto pre = dtab_off.find(o);
+    const int toff = pre != dtab_off.end() ? pre->second : dtab_pre;
+    if (pre != dtab_off.end()) {
+      ensure_regs(o + nm + 1);
+    } else {
+      sync();
+      dtab_build(o, toff);
+      if (!in_regs) {
+        if (greedy && nreg >= 1) {
+          place(plan_set(o + nm + 1), o + nm + 1);
+          emit_taddr();
+        }
+        tile_to_regs();
+        in_regs = true;
       }
-      tile_to_regs();
-      in_regs = true;
+      sync();
     }
-    sync();
     const std::string end = L();
     skip_unless(thread_pred(cm, cp), end);
     // e(i) = pext(i, U): table-index bit k is tile bit u_k, held by a thread bit
@@ -1065,6 +1107,7 @@ struct Gen {
     }
     const std::string ebase = r();
     e("mad.lo.u32 %s, %s, %d, %%dtab;", ebase.c_str(), et.c_str(), ES);
+    if (toff) e("add.u32 %s, %s, %d;", ebase.c_str(), ebase.c_str(), toff * ES);
     uint32_t ctm, ctv, crm, crp;
     split(cm, cp, ctm, ctv, crm, crp);
     for (int r_ = 0; r_ < R; ++r_) {
@@ -1559,6 +1602,7 @@ struct Gen {
     const uint32_t T = 1u << K;
     const uint32_t bytes = T * ES, chunk_bytes = (uint32_t)ES << tg.lc;
     const int nch = 1 << tg.nh;
+    plan_prebuild();
     // prologue: base, TMA load
     e("ld.param.u64 %%ga, [pa];");
     e("cvta.to.global.u64 %%ga, %%ga;");
@@ -1597,6 +1641,7 @@ struct Gen {
       chunk_loop(nch, chunk_bytes, true);
       label(w0);
     }
+    for (const auto& t : dtab_off) dtab_build(t.first, t.second);  // while the tile loads
     sync();
     {
       const std::string wt = L(), q = p();
@@ -1695,7 +1740,7 @@ struct Gen {
     out += ".version 8.7\n.target sm_100a\n.address_size 64\n\n";
     out += ".extern .shared .align 128 .b8 lfqs_tile[];\n";
     out += ".shared .align 8 .b64 lfqs_bar;\n";
-    out += ".shared .align 16 .b8 lfqs_dtab[" + std::to_string(256 * ES) + "];\n\n";
+    out += ".shared .align 16 .b8 lfqs_dtab[" + std::to_string(dtab_entries() * ES) + "];\n\n";
     const int nc = P.ncoef > 0 ? P.ncoef : 1;
     out += ".visible .entry lfqs_jit(.param .u64 pa, .param .u64 poff, .param .align 16 .b8 pc[" +
            std::to_string(nc * 16) + "])\n";
