@@ -392,7 +392,6 @@ __global__ void __launch_bounds__(kFThreads, sizeof(S) == 4 ? 4 : 2) k_fused(cx<
   C* tile = reinterpret_cast<C*>(smem_raw);
   __shared__ __align__(8) uint64_t bar;
   __shared__ C dtab[256];  // phase table of the current F_DTAB op
-  __shared__ C dsep[2 * 8 + 1];  // factors of a separable table (slot 2 b + v, constant)
   const uint32_t tid = threadIdx.x;
   const FTile& tg = prog.tile;
   const int lc = tg.lc, nh = tg.nh;
@@ -461,32 +460,7 @@ __global__ void __launch_bounds__(kFThreads, sizeof(S) == 4 ? 4 : 2) k_fused(cx<
       const uint32_t U = mlo, cm = plo & 0xffffu, cp = plo >> 16;
       const int nb = __popc(U);
       __syncthreads();  // the previous table's readers (and tile writers) are done
-      if (h.pad0 & kDtabSeparable) {
-        // separable table (separable_table): slot s (2 b + v: members fixing table bit b to
-        // v; 2 nb: members fixing none) is multiplied out by thread (s mod 8) * 32 + s / 8
-        // -- one lane of each warp, so the slots' chains run on different warps
-        const uint32_t slot_me = (tid & 31u) * 8u + (tid >> 5);
-        if ((tid & 31u) < 3u && slot_me < 2u * nb + 1u) {
-          C t = mk<S>(1, 0);
-          for (int j = 1; j <= nm; ++j) {
-            const FHdr& g = prog.h[o + j];
-            if ((base & g.mhi) != g.phi) continue;
-            const uint32_t rel = g.mlo & U;
-            const uint32_t slot =
-                rel ? 2u * __popc(U & (rel - 1)) + ((g.plo & rel) ? 1u : 0u) : 2u * nb;
-            if (slot != slot_me) continue;
-            const C d = cvs<S>(prog.c[g.coef]);
-            if (!is_one(d)) t = cmul_fma(d, t);
-          }
-          dsep[slot_me] = t;
-        }
-        __syncthreads();
-        if (tid < (1u << nb)) {
-          C t = dsep[2 * nb];
-          for (int b = 0; b < nb; ++b) t = cmul_fma(dsep[2 * b + ((tid >> b) & 1u)], t);
-          dtab[tid] = t;
-        }
-      } else if (tid < (1u << nb)) {
+      if (tid < (1u << nb)) {
         // Entry tid: tile pattern with tid's bits deposited at U's positions.
         uint32_t ie = cp, u = U;
         for (int b = 0; b < nb; ++b) {
@@ -850,20 +824,6 @@ uint32_t diag_support(const FHdr& h) {
 // preceded by an F_DTAB header and evaluated as one table per tile.
 constexpr int kMinTable = 3;
 constexpr int kTableBits = 8;
-// A table is separable when every member is a one-entry diagonal fixing at most one table
-// bit (QFT rows: CPhase(k -> q) with q common to the group or outside the tile): then
-// entry e = C x prod_b F[b][bit b of e], where C is the product of the members fixing no
-// table bit and F[b][v] the product of those fixing table bit b to v (each in member
-// order), so a tile builds its table with ~members + 2^nb x nb complex multiplies instead
-// of 2^nb x members (k_fused F_DTAB; jit.cpp builds them in the pass prologue, where the
-// one extra barrier of the two-phase build hides behind the tile load).
-bool separable_table(const FHdr* members, int n, uint32_t U) {
-  for (int k = 0; k < n; ++k) {
-    if (members[k].type != F_DIAG1) return false;
-    if (__builtin_popcount(members[k].mlo & U) > 1) return false;
-  }
-  return true;
-}
 // A diagonal op whose factor depends on the tile (out-of-tile fixed bits or targets).
 bool tile_dependent(const FHdr& h) {
   if (h.mhi != 0) return true;
@@ -923,7 +883,6 @@ void merge_phase_runs(FProg& P, bool split) {
           t.m = (uint8_t)(j - i);
           t.mlo = sup & ~cm;
           t.plo = cm | (cp << 16);
-          t.pad0 = separable_table(run + i, j - i, t.mlo) ? kDtabSeparable : 0;
           out[no++] = t;
           --spare;
         }

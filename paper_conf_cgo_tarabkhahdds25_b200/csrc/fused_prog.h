@@ -22,10 +22,8 @@ struct FHdr {       // 32 bytes
   uint32_t mlo, plo;  // per-amplitude predicate (i & mlo) == plo   (tile bits)
   uint64_t mhi, phi;  // per-tile predicate     (base & mhi) == phi (qubits outside the tile)
   // F_DTAB: m = member count, mlo = table bits U (tile bits), plo = common
-  // predicate cm | cp << 16 (every member requires (i & cm) == cp); mhi = phi = 0;
-  // pad0 = kDtabSeparable when the table factors per table bit (separable_table).
+  // predicate cm | cp << 16 (every member requires (i & cm) == cp); mhi = phi = 0.
 };
-constexpr uint8_t kDtabSeparable = 1;  // FHdr.pad0 of an F_DTAB (fused_kernels.cu)
 constexpr int kMaxOps = 192;
 constexpr int kMaxCoef = 1580;
 constexpr int kMaxHigh = 8;

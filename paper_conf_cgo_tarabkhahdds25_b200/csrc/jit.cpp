@@ -1015,8 +1015,6 @@ struct Gen {
   // tile) or 8 KiB (complex64: 4 CTAs per SM with the 32 KiB tile).
   int prebuild_entries() const { return c64 ? 1024 : 2048; }
   std::map<int, int> dtab_off;  // prebuilt F_DTAB op -> entry offset in lfqs_dtab
-  std::map<int, int> dsep_off;  // prebuilt separable F_DTAB op -> slot offset in lfqs_dsep
-  int dsep_pre = 0;             // slots of the prebuilt separable tables
   int dtab_pre = 0;             // entries of the prebuilt tables
   bool dtab_dyn = false;        // some table is built in place (after the prebuilt ones)
   void plan_prebuild() {
@@ -1027,10 +1025,6 @@ struct Gen {
       if (dtab_pre + sz <= prebuild_entries()) {
         dtab_off[o] = dtab_pre;
         dtab_pre += sz;
-        if (separable(h)) {
-          dsep_off[o] = dsep_pre;
-          dsep_pre += 2 * __builtin_popcount(h.mlo) + 1;
-        }
       } else {
         dtab_dyn = true;
       }
@@ -1038,70 +1032,6 @@ struct Gen {
     }
   }
   int dtab_entries() const { return std::max(dtab_pre + (dtab_dyn ? 256 : 0), 1); }
-
-  // Separable tables (fused_kernels.cu separable_table; the same order of operations as
-  // k_fused): phase 1 -- slot s (members fixing table bit b to v: s = 2 b + v; members
-  // fixing none: s = 2 nb) multiplied out, in member order, by thread (s mod nw) * 32 +
-  // s / nw into lfqs_dsep[dsep_off + s]; phase 2 (after a barrier) -- entry e = C x F[0][e_0]
-  // x F[1][e_1] ... by thread e mod NT.
-  void dtab_sep_slots(int o, int dsep_off) {
-    const FHdr& h = P.h[o];
-    const uint32_t U = h.mlo;
-    const int nb = __builtin_popcount(U);
-    std::vector<std::vector<int>> slot(2 * nb + 1);
-    for (int j = 1; j <= h.m; ++j) {
-      const FHdr& g = P.h[o + j];
-      const uint32_t rel = g.mlo & U;
-      const int sl = rel ? 2 * __builtin_popcount(U & (rel - 1)) + ((g.plo & rel) ? 1 : 0)
-                         : 2 * nb;
-      slot[sl].push_back(o + j);
-    }
-    const int nw = NT / 32;
-    for (int sl = 0; sl <= 2 * nb; ++sl) {
-      const std::string skip = L(), q = p();
-      e("setp.ne.u32 %s, %%ltid, %d;", q.c_str(), (sl % nw) * 32 + sl / nw);
-      e("@%s bra %s;", q.c_str(), skip.c_str());
-      Cx t{f(), f()};
-      e("mov.%s %s, %s;", FT, t.x.c_str(), c64 ? "0f3F800000" : "0d3FF0000000000000");
-      e("mov.%s %s, %s;", FT, t.y.c_str(), zero().c_str());
-      for (int oj : slot[sl]) {
-        const FHdr& g = P.h[oj];
-        const Cx d = coef(g.coef);
-        if (d.vx == 1.0 && d.vy == 0.0) continue;  // is_one: skipped as in k_fused
-        const std::string ms = L();
-        tile_pred(g.mhi, g.phi, ms);
-        assign(t.x, t.y, cmulf(d, t));
-        label(ms);
-      }
-      const std::string a = r();
-      e("mov.u32 %s, lfqs_dsep;", a.c_str());
-      sts(a, t, (dsep_off + sl) * ES);
-      label(skip);
-    }
-  }
-  void dtab_sep_entries(int o, int off, int dsep_off) {
-    const int nb = __builtin_popcount(P.h[o].mlo);
-    for (int k = 0; k * NT < (1 << nb); ++k) {
-      const std::string skip = L(), q = p(), eid = r();
-      e("add.u32 %s, %%ltid, %d;", eid.c_str(), k * NT);
-      e("setp.ge.u32 %s, %s, %u;", q.c_str(), eid.c_str(), 1u << nb);
-      e("@%s bra %s;", q.c_str(), skip.c_str());
-      const std::string ds = r();
-      e("mov.u32 %s, lfqs_dsep;", ds.c_str());
-      Cx t = lds(ds, (dsep_off + 2 * nb) * ES);
-      for (int b = 0; b < nb; ++b) {
-        const std::string bit = r(), ad = r();
-        e("bfe.u32 %s, %s, %d, 1;", bit.c_str(), eid.c_str(), b);
-        e("mad.lo.u32 %s, %s, %d, %s;", ad.c_str(), bit.c_str(), ES, ds.c_str());
-        t = cmulf(lds(ad, (dsep_off + 2 * b) * ES), t);
-      }
-      const std::string a = r();
-      e("mad.lo.u32 %s, %s, %d, %%dtab;", a.c_str(), eid.c_str(), ES);
-      sts(a, t, off * ES);
-      label(skip);
-    }
-  }
-  static bool separable(const FHdr& h) { return (h.pad0 & kDtabSeparable) != 0; }
 
   // Builds table `o` into lfqs_dtab entries [off, off + 2^nb): entry e by thread e mod NT.
   void dtab_build(int o, int off) {
@@ -1145,13 +1075,7 @@ struct Gen {
       ensure_regs(o + nm + 1);
     } else {
       sync();
-      if (separable(h)) {
-        dtab_sep_slots(o, dsep_pre);  // the slots after the prebuilt tables' ones
-        sync();
-        dtab_sep_entries(o, toff, dsep_pre);
-      } else {
-        dtab_build(o, toff);
-      }
+      dtab_build(o, toff);
       if (!in_regs) {
         if (greedy && nreg >= 1) {
           place(plan_set(o + nm + 1), o + nm + 1);
@@ -1717,16 +1641,7 @@ struct Gen {
       chunk_loop(nch, chunk_bytes, true);
       label(w0);
     }
-    // phase tables, while the tile loads (separable ones: slots, one barrier, entries)
-    for (const auto& t : dtab_off)
-      if (separable(P.h[t.first]))
-        dtab_sep_slots(t.first, dsep_off[t.first]);
-      else
-        dtab_build(t.first, t.second);
-    if (dsep_pre > 0) {
-      sync();
-      for (const auto& t : dsep_off) dtab_sep_entries(t.first, dtab_off[t.first], t.second);
-    }
+    for (const auto& t : dtab_off) dtab_build(t.first, t.second);  // while the tile loads
     sync();
     {
       const std::string wt = L(), q = p();
@@ -1825,8 +1740,7 @@ struct Gen {
     out += ".version 8.7\n.target sm_100a\n.address_size 64\n\n";
     out += ".extern .shared .align 128 .b8 lfqs_tile[];\n";
     out += ".shared .align 8 .b64 lfqs_bar;\n";
-    out += ".shared .align 16 .b8 lfqs_dtab[" + std::to_string(dtab_entries() * ES) + "];\n";
-    out += ".shared .align 16 .b8 lfqs_dsep[" + std::to_string((dsep_pre + 17) * ES) + "];\n\n";
+    out += ".shared .align 16 .b8 lfqs_dtab[" + std::to_string(dtab_entries() * ES) + "];\n\n";
     const int nc = P.ncoef > 0 ? P.ncoef : 1;
     out += ".visible .entry lfqs_jit(.param .u64 pa, .param .u64 poff, .param .align 16 .b8 pc[" +
            std::to_string(nc * 16) + "])\n";
