@@ -17,7 +17,7 @@ timeout 600 python bench.py --impl reference --steps 3 --warmup 3 --ref-step-s 6
 timeout 300 python tools/profile_gates.py --n 30 --reps 5 --time --no-shuffle > $O/${TAG}_pergate_n30.txt 2>&1
 timeout 900 ncu --metrics gpu__time_duration.sum,dram__bytes_read.sum,dram__bytes_write.sum \
   --clock-control none --csv --log-file $O/${TAG}_launches.csv \
-  python bench.py --steps 1 --warmup 3 --no-e2e --no-cpu-baseline --macro-n 0 > $O/${TAG}_ncu_bench.out 2>&1
+  python bench.py --steps 1 --warmup 3 --no-e2e --no-cpu-baseline --macro-n 0 --no-small > $O/${TAG}_ncu_bench.out 2>&1
 timeout 900 ncu --set full --clock-control none --import-source on -k regex:k_group_x2 -c 2 \
   -o $O/${TAG}_full_dense1 python tools/profile_gates.py --n 28 --reps 1 --gates RX:12,H:20 \
   > $O/${TAG}_ncu_full.out 2>&1

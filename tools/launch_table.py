@@ -1,6 +1,6 @@
 """Summarises the ncu launch list of one bench step (tools/gpu_evidence.sh: `ncu --metrics
 gpu__time_duration.sum,dram__bytes_read.sum,dram__bytes_write.sum ... bench.py --steps 1
---warmup 3 --no-e2e --no-cpu-baseline --macro-n 0`) into profiles/rNN_launches.md and
+--warmup 3 --no-e2e --no-cpu-baseline --macro-n 0 --no-small`) into profiles/rNN_launches.md and
 profiles/traffic_per_launch.json.
 
 The last 540 gate launches of the capture are the timed step; they are matched, in order,
@@ -52,7 +52,8 @@ def main():
     out = [f"# {tag} — ncu launch list of one bench step (n = 30 sweep, {len(sweep)} launches)", "",
            "Command: `ncu --metrics gpu__time_duration.sum,dram__bytes_read.sum,dram__bytes_write.sum "
            "--clock-control none --csv python bench.py --steps 1 --warmup 3 --no-e2e "
-           "--no-cpu-baseline --macro-n 0` (tools/gpu_evidence.sh); table by `tools/launch_table.py`.",
+           "--no-cpu-baseline --macro-n 0 --no-small` (tools/gpu_evidence.sh); table by "
+           "`tools/launch_table.py`.",
            "ncu times are cold-cache and serialised: compare shares, not absolutes. Bench (CUDA "
            "events, same kernels): see the bench JSON line.", "",
            "| class | launches | ncu ms | share | DRAM bytes/launch (traffic) | SURVEY §8(d) "
