@@ -80,13 +80,17 @@ void Comm::exchange(void* shard, int amp_bytes, const std::vector<Piece>& pieces
   LFQS_CUDA_CHECK(cudaStreamWaitEvent(cstream, ready, 0));
   const uint64_t stage_amps = stage_bytes / amp_bytes;
   unsigned char* base = static_cast<unsigned char*>(shard);
-  int c = 0;
   for (const Piece& pc : pieces) {
     for (uint64_t off = 0; off < pc.count; off += stage_amps) {
       const uint64_t cnt = std::min<uint64_t>(stage_amps, pc.count - off);
       const size_t bytes = cnt * amp_bytes;
-      const int b = c & 1;
-      if (c >= 2) LFQS_CUDA_CHECK(cudaStreamWaitEvent(cstream, ev_free[b], 0));
+      // A staging buffer is reused only after the compute stream has copied its previous
+      // contents out -- also across calls: the parts of an overlapped exchange are separate
+      // calls whose `ready` events may precede the previous part's copies.
+      const int b = next_stage;
+      next_stage ^= 1;
+      if (stage_used[b]) LFQS_CUDA_CHECK(cudaStreamWaitEvent(cstream, ev_free[b], 0));
+      stage_used[b] = true;
       unsigned char* src = base + (pc.offset + off) * amp_bytes;
       LFQS_NCCL_CHECK(ncclGroupStart());
       LFQS_NCCL_CHECK(ncclSend(src, bytes, ncclUint8, partner, comm, cstream));
@@ -96,7 +100,6 @@ void Comm::exchange(void* shard, int amp_bytes, const std::vector<Piece>& pieces
       LFQS_CUDA_CHECK(cudaStreamWaitEvent(compute, ev_recv[b], 0));
       LFQS_CUDA_CHECK(cudaMemcpyAsync(src, stage[b], bytes, cudaMemcpyDeviceToDevice, compute));
       LFQS_CUDA_CHECK(cudaEventRecord(ev_free[b], compute));
-      ++c;
     }
   }
 }

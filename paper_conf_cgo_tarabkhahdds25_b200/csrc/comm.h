@@ -23,6 +23,8 @@ struct Comm {
   unsigned char* stage[2] = {nullptr, nullptr};
   uint64_t stage_bytes = 0;
   cudaEvent_t ev_recv[2], ev_free[2], ev_start;
+  int next_stage = 0;                   // staging buffer of the next chunk
+  bool stage_used[2] = {false, false};  // ev_free[b] marks the end of its last use
   double* d_reduce = nullptr;
 
   static void unique_id(uint8_t uid[128]);
