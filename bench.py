@@ -366,67 +366,90 @@ def run_small(lfqs, stream, with_oracle: bool, reps: int = 50):
 NVLINK_GBPS = 900.0  # NVLink 5 per GPU per direction, nominal (no measured peak here)
 
 
-def run_qft_sharded(lfqs, st, n, n_loc, world, rank, stream, barrier, dist, device_reduce,
-                    hbm_peak, reps):
-    """QFT(n)|x> on the sharded state (n = n_loc + log2 world; 8 GPUs x 2^30: QFT(33), the
-    configs[4] circuit at this per-GPU size), compiled passes + phase tables, exchanges
-    overlapped with local passes; the timed region ends after the final canonicalisation
-    (relabels are not free).  Device time (CUDA events) max over ranks.
-    Combined roofline (SURVEY §8(d) [4]): T_roof = sum of passes x 32 * 2^n_loc B / HBM +
-    exchanges x 16 * 2^(n_loc - 1) B / NVLink, the north-star form with one pass per gate
-    beside it; closed form checked on 64 sampled amplitudes of every rank's shard."""
+def run_sharded_circuits(lfqs, st, n, n_loc, world, rank, stream, barrier, dist, device_reduce,
+                         hbm_peak, reps):
+    """Macro circuits on the sharded state (n = n_loc + log2 world): QFT(n)|x> (8 GPUs x 2^30:
+    QFT(33), the configs[4] circuit at this per-GPU size), and the configs[3] shapes Grover(n)
+    (2 iterations) and a random layered circuit of depth 20 -- compiled passes + phase
+    tables, exchanges overlapped with local passes; the timed region ends after the final
+    canonicalisation (relabels are not free).  Device time (CUDA events), max
+    over ranks.  Combined roofline (SURVEY §8(d) [4]): T_roof = passes x 32 * 2^n_loc B / HBM
+    + exchanges x 16 * 2^(n_loc - 1) B / NVLink, with the north-star form (one pass per gate)
+    beside it.  Checks: QFT and Grover closed forms on 64 sampled amplitudes of every rank's
+    shard (readings R10, R12), the random circuit's norm."""
     import torch
     x = int(W.SplitMix64(n).next_u64() & ((1 << n) - 1))
-    gates = W.qft(n)
-    arr = lfqs.marshal_gates(gates)
+    w = int(W.SplitMix64(n + 1).next_u64() & ((1 << n) - 1))
+    k_it = 2
+    th = math.asin(2.0 ** (-n / 2))
+
+    def qft_ref(idx):
+        ph = ((x * idx.astype(object)) % (1 << n)).astype(np.float64) / (1 << n)
+        return np.exp(2j * np.pi * ph) / math.sqrt(2.0 ** n), math.sqrt(2.0 ** n)
+
+    def grover_ref(idx):
+        ref = np.full(idx.shape, (-1) ** k_it * math.cos((2 * k_it + 1) * th) /
+                      math.sqrt(2.0 ** n - 1), dtype=complex)
+        ref[idx == w] = (-1) ** k_it * math.sin((2 * k_it + 1) * th)
+        return ref, math.sqrt(2.0 ** n)
+
+    circuits = [("qft", W.qft(n), x, qft_ref), ("grover", W.grover(n, w, k_it), 0, grover_ref),
+                ("random", W.random_layered(n, 20, seed=7), 0, None)]
     flags = lfqs.FUSE_LOW | lfqs.FUSE_JIT | lfqs.FUSE_PHASE
+    out = {}
+    for name, gates, init, ref_fn in circuits:
+        arr = lfqs.marshal_gates(gates)
 
-    def once():
-        st.init_basis(x)
-        barrier()
-        p0, e0 = st.passes(), st.exchange_stats()
-        a = torch.cuda.Event(enable_timing=True)
-        b = torch.cuda.Event(enable_timing=True)
-        a.record(stream)
-        lfqs.lfqs_run_circuit(st.h, arr, flags)
-        st.copy_out(0, 0)  # canonicalise the qubit map (collective), inside the timed region
-        b.record(stream)
-        barrier()
-        e1 = st.exchange_stats()
-        return a.elapsed_time(b), st.passes() - p0, e1[0] - e0[0], e1[1] - e0[1]
+        def once():
+            st.init_basis(init)
+            barrier()
+            p0, e0 = st.passes(), st.exchange_stats()
+            a = torch.cuda.Event(enable_timing=True)
+            b = torch.cuda.Event(enable_timing=True)
+            a.record(stream)
+            lfqs.lfqs_run_circuit(st.h, arr, flags)
+            st.copy_out(0, 0)  # canonicalise the qubit map (collective), in the timed region
+            b.record(stream)
+            barrier()
+            e1 = st.exchange_stats()
+            return a.elapsed_time(b), st.passes() - p0, e1[0] - e0[0], e1[1] - e0[1]
 
-    once()  # warm-up: compiles every pass shape
-    runs = [once() for _ in range(reps)]
-    ms_rank = min(r[0] for r in runs)
-    t = torch.tensor([ms_rank], device=device_reduce)
-    dist.all_reduce(t, op=dist.ReduceOp.MAX)
-    ms = float(t.item())
-    _, passes, n_ex, ex_bytes = runs[0]
-    # closed form on this rank's shard (canonical order after the timed canonicalisation)
-    rng = np.random.default_rng(rank + 1)
-    lo = rank << n_loc
-    idx = lo + rng.integers(0, 1 << n_loc, 64)
-    got = np.array([st.copy_out(int(k), 1)[0] for k in idx])
-    ph = ((x * idx.astype(object)) % (1 << n)).astype(np.float64) / (1 << n)
-    err = float(np.max(np.abs(got - np.exp(2j * np.pi * ph) / math.sqrt(2.0 ** n))))
-    e = torch.tensor([err], device=device_reduce, dtype=torch.float64)
-    dist.all_reduce(e, op=dist.ReduceOp.MAX)
-    pb = 32.0 * 2 ** n_loc
-    t_ex = n_ex * 16.0 * 2 ** (n_loc - 1) / (NVLINK_GBPS * 1e9)
-    t_roof = passes * pb / (hbm_peak * 1e9) + t_ex
-    t_roof_gates = len(gates) * pb / (hbm_peak * 1e9) + t_ex
-    return {"circuit": f"QFT({n}) on {world} ranks, 2^{n_loc} amplitudes per rank",
+        once()  # warm-up: compiles every pass shape
+        runs = [once() for _ in range(reps)]
+        t = torch.tensor([min(r[0] for r in runs)], device=device_reduce)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        ms = float(t.item())
+        _, passes, n_ex, ex_bytes = runs[0]
+        if ref_fn is not None:  # closed form on this rank's shard (canonical order)
+            rng = np.random.default_rng(rank + 1)
+            idx = (rank << n_loc) + rng.integers(0, 1 << n_loc, 64)
+            if name == "grover" and (w >> n_loc) == rank:
+                idx[0] = w
+            got = np.array([st.copy_out(int(k), 1)[0] for k in idx])
+            ref, scale = ref_fn(idx)
+            e = torch.tensor([float(np.max(np.abs(got - ref)))], device=device_reduce,
+                             dtype=torch.float64)
+            dist.all_reduce(e, op=dist.ReduceOp.MAX)
+            check = {"closed_form_max_abs_err": float(e.item()),
+                     "closed_form_rel_err": float(e.item()) * scale}
+        else:
+            check = {"norm2": st.norm2()}  # all ranks (reduction across them)
+        pb = 32.0 * 2 ** n_loc
+        t_ex = n_ex * 16.0 * 2 ** (n_loc - 1) / (NVLINK_GBPS * 1e9)
+        t_roof = passes * pb / (hbm_peak * 1e9) + t_ex
+        t_roof_gates = len(gates) * pb / (hbm_peak * 1e9) + t_ex
+        out[f"{name}{n}"] = {
+            "circuit": f"{name}({n}) on {world} ranks, 2^{n_loc} amplitudes per rank",
             "mode": "jit+phase, exchanges overlapped", "gates": len(gates),
             "ms": round(ms, 3), "gates_per_s": len(gates) / (ms / 1e3),
             "passes_per_rank": int(passes), "exchanges_per_rank": int(n_ex),
             "exchange_bytes_per_rank_per_direction": int(ex_bytes),
             "t_roof_ms": round(t_roof * 1e3, 3), "roof_frac": (t_roof * 1e3) / ms,
             "t_roof_north_star_ms": round(t_roof_gates * 1e3, 3),
-            "roof_frac_north_star": (t_roof_gates * 1e3) / ms,
-            "roofline_terms": "passes x 32*2^n_loc B / hbm_peak + exchanges x 16*2^(n_loc-1) B "
-                              f"/ {NVLINK_GBPS} GB/s (north star: one pass per gate)",
-            "closed_form_max_abs_err": float(e.item()),
-            "closed_form_rel_err": float(e.item()) * math.sqrt(2.0 ** n)}
+            "roof_frac_north_star": (t_roof_gates * 1e3) / ms, **check}
+    out["roofline_terms"] = ("passes x 32*2^n_loc B / hbm_peak + exchanges x 16*2^(n_loc-1) B "
+                             f"/ {NVLINK_GBPS} GB/s (north star: one pass per gate)")
+    return out
 
 
 # ----------------------------------------------------------------------------
@@ -453,7 +476,8 @@ def main():
     ap.add_argument("--no-macro-unfused", action="store_true",
                     help="skip the strict one-pass-per-gate QFT/GHZ runs of the macro leg")
     ap.add_argument("--qft-reps", type=int, default=3,
-                    help="N > 1: timed runs of the sharded QFT leg (0: skip)")
+                    help="N > 1: timed runs of each sharded macro circuit (QFT, Grover, "
+                         "random layered; 0: skip)")
     ap.add_argument("--same-device", action="store_true",
                     help="test only: every rank on cuda:0 (exercises the N>1 path on one GPU)")
     ap.add_argument("--transport", default="p2p", choices=["p2p", "nccl"],
@@ -628,8 +652,9 @@ def main():
 
     qft = None
     if world > 1 and args.qft_reps > 0:
-        qft = run_qft_sharded(lfqs, st, n, n_loc, world, rank, stream, barrier, dist,
-                              "cpu" if args.same_device else "cuda", hbm_peak, args.qft_reps)
+        qft = run_sharded_circuits(lfqs, st, n, n_loc, world, rank, stream, barrier, dist,
+                                   "cpu" if args.same_device else "cuda", hbm_peak,
+                                   args.qft_reps)
 
     if args.per_gate_json and rank == 0:
         with open(args.per_gate_json, "w") as f:
@@ -722,7 +747,7 @@ def main():
             "worst_gate": worst_gate,
             "macro": macro,
             "small": small,
-            "qft_sharded": qft,
+            "macro_sharded": qft,
             "nvlink": nvlink,
             "classes": {k: {kk: (round(vv, 4) if isinstance(vv, float) else vv)
                             for kk, vv in v.items()} for k, v in classes.items()},
