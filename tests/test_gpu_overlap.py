@@ -122,3 +122,19 @@ def test_pass_count(L):
                 serial = st.passes()
             else:
                 assert st.passes() == serial
+
+
+def test_exchange_options_validated(L):
+    with L.State.virtual(10, 2) as st:
+        for opt, bad in ((L.OPT_EXCHANGE_CHUNK_BITS, 5), (L.OPT_EXCHANGE_CHUNK_BITS, -1),
+                         (L.OPT_EXCHANGE_CTAS, -1), (L.OPT_EXCHANGE_CTAS, 1 << 20)):
+            with pytest.raises(L.LfqsError) as e:
+                st.set_option(opt, bad)
+            assert e.value.status == -1
+        st.set_option(L.OPT_EXCHANGE_CHUNK_BITS, 4)  # n_local = 9: 9 - 4 >= 4, still valid
+        st.set_option(L.OPT_EXCHANGE_CTAS, 1)
+        psi = W.random_state(10, 3)
+        st.copy_in(psi)
+        gates = W.qft(10)
+        st.run_circuit(gates)
+        assert np.max(np.abs(st.copy_out() - O.run_circuit(10, gates, psi.copy()))) <= 1e-12
