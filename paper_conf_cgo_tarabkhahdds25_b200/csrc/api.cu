@@ -537,8 +537,8 @@ lfqs_status lfqs_set_option(lfqs_state* s, int option, int64_t value) {
         break;
       case LFQS_OPT_FUSE_REORDER: st->opt.fuse_reorder = value != 0; break;
       case LFQS_OPT_JIT_THREADS:
-        require(value == 128 || value == 256 || value == 512,
-                "LFQS_OPT_JIT_THREADS must be 128, 256 or 512");
+        require(value == 0 || value == 128 || value == 256 || value == 512,
+                "LFQS_OPT_JIT_THREADS must be 0 (per pass), 128, 256 or 512");
         st->opt.jit_threads = (int)value;
         break;
       case LFQS_OPT_JIT_LANE_MOVE: st->opt.jit_lane_move = value != 0; break;

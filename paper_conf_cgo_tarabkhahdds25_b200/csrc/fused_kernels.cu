@@ -31,6 +31,7 @@
 #include <cuda_runtime.h>
 
 #include <cstring>
+#include <map>
 #include <memory>
 #include <string>
 #include <type_traits>
@@ -1142,7 +1143,7 @@ void build_program(const LaunchCtx& ctx, const TileCfg& cfg, uint64_t in_tile,
 void launch_built(const LaunchCtx& ctx, int K, const FProg& P, const std::string* key = nullptr,
                   uint64_t tile_off = 0) {
   if (ctx.jit && (1 << P.tile.nh) <= ctx.opt->fuse_tma_max_chunks) {
-    const int jc = jit_config(ctx, K);
+    const int jc = jit_config(ctx, K, &P);
     jit_launch(ctx, P, K, key ? *key : jit_key(P, K, ctx.c64, jc), jc, tile_off);
     ++*ctx.launch_counter;
     return;
@@ -1328,17 +1329,17 @@ void plan_fused_schedule(const LaunchCtx& ctx_in, const std::vector<Decoded>& ga
         ps.qmask |= qubit_mask(gates[gi]);
         ps.nd_mask |= nd_of(gates[gi]);
       }
-      if (jit_ok) ps.key = jit_key(*ps.prog, cfg.K, ctx.c64, jit_config(ctx, cfg.K));
+      if (jit_ok) ps.key = jit_key(*ps.prog, cfg.K, ctx.c64, jit_config(ctx, cfg.K, ps.prog.get()));
       out.push_back(std::move(ps));
       for (int gi : picked) taken[gi] = 1;
     }
     while (head < rest.size() && taken[rest[head]]) ++head;
   }
   if (ctx.plan_only || !jit_ok) return;
-  std::vector<std::pair<std::string, const FProg*>> items;
+  std::map<int, std::vector<std::pair<std::string, const FProg*>>> items;  // per generator config
   for (const FusedPass& ps : out)
-    if (ps.prog) items.emplace_back(ps.key, ps.prog.get());
-  jit_compile(items, cfg.K, ctx.c64, jit_config(ctx, cfg.K));
+    if (ps.prog) items[jit_config(ctx, cfg.K, ps.prog.get())].emplace_back(ps.key, ps.prog.get());
+  for (const auto& it : items) jit_compile(it.second, cfg.K, ctx.c64, it.first);
 }
 
 void launch_fused_pass(const LaunchCtx& ctx, const std::vector<Decoded>& gates,

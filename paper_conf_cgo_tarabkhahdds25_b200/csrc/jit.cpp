@@ -24,6 +24,7 @@
 #include <nvPTXCompiler.h>
 
 #include <atomic>
+#include <cmath>
 #include <condition_variable>
 #include <cstdarg>
 #include <cstdio>
@@ -1942,8 +1943,58 @@ void jit_compile(const std::vector<std::pair<std::string, const FProg*>>& items,
   wait_others();
 }
 
-int jit_config(const LaunchCtx& ctx, int K) {
-  const int t = ctx.opt->jit_threads;
+// FP64 operations per amplitude a pass issues (static estimate from its program): dense
+// 1-target types 4 (H, real / imaginary-off-diagonal) or 8 (general), a 4x4 / 8x8 matrix 2 per
+// nonzero real or imaginary coefficient part per row, one-entry diagonals 4 per affected
+// amplitude; each scaled by the fraction of amplitudes its predicates select.
+double pass_fp64_per_amp(const FProg& P, double* table_work) {
+  double ops = 0.0;
+  *table_work = 0.0;
+  for (int o = 0; o < P.nops; ++o) {
+    const FHdr& h = P.h[o];
+    const double frac =
+        std::ldexp(1.0, -__builtin_popcount(h.mlo) - __builtin_popcountll(h.mhi));
+    const double2* c = P.c + h.coef;
+    auto parts = [&](int n) {
+      int k = 0;
+      for (int i = 0; i < n; ++i) k += 2 * (c[i].x != 0.0) + 2 * (c[i].y != 0.0);
+      return k;
+    };
+    switch (h.type) {
+      case F_DTAB:  // entries x members evaluated per tile
+        *table_work += std::ldexp((double)h.m, __builtin_popcount(h.mlo));
+        o += h.m;
+        break;
+      case F_DIAG1: ops += 4.0 * frac; break;
+      case F_DIAGN: ops += 4.0 * frac; break;
+      case F_H: case F_UR: case F_UI: ops += 4.0 * frac; break;
+      case F_U2: ops += 8.0 * frac; break;
+      case F_U4: ops += parts(16) / 4.0 * frac; break;
+      case F_U8: ops += parts(64) / 8.0 * frac; break;
+      default: break;  // moves
+    }
+  }
+  return ops;
+}
+
+// LFQS_OPT_JIT_THREADS = 0 (auto): 128 threads per CTA (3 CTAs per SM, one more
+// register-held tile bit: fewer tile round trips) for passes whose FP64 work is below ~0.9 of
+// their HBM time and that build no large phase tables; 256 otherwise -- heavy FP64 passes and
+// table-heavy (QFT) passes need 256's 16 warps per SM to hide latency.  Calibrated on the
+// per-pass ncu A/B of profiles/r02_heavy_passes.md (light passes 1.6 -> 1.25 ms with 128,
+// heavy ones 5.5 -> 9.9 ms, QFT table passes 2.3 -> 3.2 ms).
+int auto_threads(const FProg& P, bool c64, int K) {
+  if (c64 || K < 9) return 256;
+  double table_work = 0.0;
+  const double ops = pass_fp64_per_amp(P, &table_work);
+  // FP64 time / HBM time of the pass = ops x 2^n / 1.7e13 per s  /  (32 x 2^n B / 6.5e12 B/s)
+  const double rho = ops * 6.5e12 / (1.7e13 * 32.0);
+  return (table_work < 2048.0 && rho <= 0.9) ? 128 : 256;
+}
+
+int jit_config(const LaunchCtx& ctx, int K, const FProg* P) {
+  int t = ctx.opt->jit_threads;
+  if (t == 0) t = P ? auto_threads(*P, ctx.c64, K) : 256;
   return ((t == 512 && K >= 9) ? 512 : (t == 128 && K >= 8) ? 128 : 256) |
          (ctx.opt->jit_lane_move ? JIT_LANE_MOVE : 0) |
          (ctx.opt->jit_greedy_place ? JIT_GREEDY_PLACE : 0) |

@@ -29,8 +29,9 @@ void jit_compile(const std::vector<std::pair<std::string, const FProg*>>& items,
 // tile indices starting at tile_off (a block of the state whose top bits are fixed).
 void jit_launch(const LaunchCtx& ctx, const FProg& P, int K, const std::string& key, int jc,
                 uint64_t tile_off = 0);
-// Generator configuration for tile size K (LFQS_OPT_JIT_THREADS, LFQS_OPT_JIT_LANE_MOVE).
-int jit_config(const LaunchCtx& ctx, int K);
+// Generator configuration of pass P for tile size K (LFQS_OPT_JIT_THREADS -- 0: chosen per
+// pass from P -- LFQS_OPT_JIT_LANE_MOVE, ...).
+int jit_config(const LaunchCtx& ctx, int K, const FProg* P = nullptr);
 size_t jit_cache_size();
 
 }  // namespace lfqs

@@ -99,7 +99,7 @@ struct Options {
   // beats direct loads for every chunk count up to 128, so TMA is the default.
   int fuse_tma_max_chunks = 256;
   int items_per_thread = 0;  // 0 = library default
-  int jit_threads = 256;     // threads per CTA of compiled passes (128, 256 or 512)
+  int jit_threads = 0;       // threads per CTA of compiled passes (128, 256, 512; 0: per pass)
   int lane_group = 1;  // 1: dense 4x4 on qubits {1, 2} via k_lanegroup; 2: every dense 4x4/8x8
                        // with targets in [1, 5] (test / measurement); 0: never
   int stream_max_prefix = 0;  // lfqs_run_circuit_streamed: max gates run per piece (0: all)

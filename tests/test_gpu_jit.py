@@ -70,12 +70,13 @@ def test_jit_equals_interpreter(L, n, tile, low, reorder):
     assert np.max(np.abs(b - ref)) <= 1e-12
 
 
-@pytest.mark.parametrize("threads", [128, 256, 512])
+@pytest.mark.parametrize("threads", [0, 128, 256, 512])
 @pytest.mark.parametrize("tile", [9, 10, 12])
 @pytest.mark.parametrize("n", [13, 16])
 def test_jit_512_threads_equals_interpreter(L, n, tile, threads):
-    """Compiled passes with 512 threads per CTA (LFQS_OPT_JIT_THREADS): a different
-    thread/register placement of the same per-amplitude arithmetic."""
+    """Compiled passes with 128 / 256 / 512 threads per CTA or chosen per pass (0, the
+    default; LFQS_OPT_JIT_THREADS): a different thread/register placement of the same
+    per-amplitude arithmetic."""
     psi = W.random_state(n, 3 * n + tile)
     gates = _mixed(n, 2000 + n + tile)
     a, _ = _run(L, n, psi, gates, True, tile)
