@@ -61,7 +61,8 @@ def main():
     ap.add_argument("--tile", type=int, default=0)
     ap.add_argument("--low", type=int, default=0)
     ap.add_argument("--reorder", type=int, default=1)
-    ap.add_argument("--jit-threads", type=int, default=256, help="LFQS_OPT_JIT_THREADS (128/256/512)")
+    ap.add_argument("--jit-threads", type=int, default=0,
+                    help="LFQS_OPT_JIT_THREADS (0: per pass, the library default; 128/256/512)")
     ap.add_argument("--lane-move", type=int, default=-1,
                     help="LFQS_OPT_JIT_LANE_MOVE (0/1; -1: library default)")
     ap.add_argument("--phase-split", type=int, default=-1,
@@ -176,7 +177,7 @@ def main():
                        "conv_GBps": 2.0 * ab * 2 ** n * len(gates) / (t / 1e3) / 1e9,
                        "pass_GBps": 2.0 * ab * 2 ** n * passes / (t / 1e3) / 1e9,
                        "dtype": "c64" if args.c64 else "c128", "world": args.world,
-                       "exchanges": x1 - x0, "lane_move": args.lane_move, "merge": args.merge, "merge2q": args.merge2q, "greedy": args.greedy, "lane_reg2": args.lane_reg2, "pool": args.pool, "partial_rt": args.partial_rt, "phase_split": args.phase_split,
+                       "exchanges": x1 - x0, "lane_move": args.lane_move, "merge": args.merge, "merge2q": args.merge2q, "jit_threads": args.jit_threads, "greedy": args.greedy, "lane_reg2": args.lane_reg2, "pool": args.pool, "partial_rt": args.partial_rt, "phase_split": args.phase_split,
                        "hbm_peak_GBps": peak, "peak_source": peak_src}
                 # fraction of the HBM roofline: per pass actually made, and against the
                 # north-star convention of one 2*16*2^n-byte pass per gate
