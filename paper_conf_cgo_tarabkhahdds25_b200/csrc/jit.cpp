@@ -1982,9 +1982,11 @@ double pass_fp64_per_amp(const FProg& P, double* table_work) {
 // their HBM time and that build no large phase tables; 256 otherwise -- heavy FP64 passes and
 // table-heavy (QFT) passes need 256's 16 warps per SM to hide latency.  Calibrated on the
 // per-pass ncu A/B of profiles/r02_heavy_passes.md (light passes 1.6 -> 1.25 ms with 128,
-// heavy ones 5.5 -> 9.9 ms, QFT table passes 2.3 -> 3.2 ms).
+// heavy ones 5.5 -> 9.9 ms, QFT table passes 2.3 -> 3.2 ms).  The same rule for complex64
+// (fp32 arithmetic at twice the rate on half the bytes: about the same ratio): random
+// layered(31) 347 -> 333 ms, Grover 121 -> 116, the others unchanged.
 int auto_threads(const FProg& P, bool c64, int K) {
-  if (c64 || K < 9) return 256;
+  if (K < 9) return 256;
   double table_work = 0.0;
   const double ops = pass_fp64_per_amp(P, &table_work);
   // FP64 time / HBM time of the pass = ops x 2^n / 1.7e13 per s  /  (32 x 2^n B / 6.5e12 B/s)
