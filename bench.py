@@ -623,7 +623,11 @@ def main():
     roofline = {"bound": "hbm",
                 "kernel": f"{dom} class per-gate kernels (apply_kernels.cu k_group_x2 / k_group)",
                 "achieved": dc["alg_GBps"], "peak": hbm_peak, "unit": "GB/s",
-                "frac": dc["alg_GBps"] / hbm_peak, "traffic": traffic, "peak_source": peak_src,
+                "frac": dc["alg_GBps"] / hbm_peak, "traffic": traffic,
+                "traffic_source": "ncu dram__bytes_read.sum + dram__bytes_write.sum per launch, "
+                                  "class mean of the committed capture (profiles/r02_launches.md, "
+                                  "profiles/traffic_per_launch.json)" if traffic else None,
+                "peak_source": peak_src,
                 "bytes_per_launch": dc["alg_bytes"] / dc["gates"],
                 "avg_launch_ms": dc["ms"] / dc["gates"]}
     # N > 1: the global-qubit exchanges (half-shard swaps over NVLink).  A gate that
