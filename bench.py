@@ -623,7 +623,8 @@ def main():
     roofline = {"bound": "hbm",
                 "kernel": f"{dom} class per-gate kernels (apply_kernels.cu k_group_x2 / k_group)",
                 "achieved": dc["alg_GBps"], "peak": hbm_peak, "unit": "GB/s",
-                "frac": dc["alg_GBps"] / hbm_peak, "traffic": traffic,
+                "frac": dc["alg_GBps"] / hbm_peak,
+                "frac_of_nominal_8000GBps": dc["alg_GBps"] / 8000.0, "traffic": traffic,
                 "traffic_source": "ncu dram__bytes_read.sum + dram__bytes_write.sum per launch, "
                                   "class mean of the committed capture (profiles/r02_launches.md, "
                                   "profiles/traffic_per_launch.json)" if traffic else None,
