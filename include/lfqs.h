@@ -332,6 +332,14 @@ lfqs_status lfqs_state_info(const lfqs_state* s, int* n_qubits, int* n_local, in
  * summed.  Counted when the exchange is enqueued (host side, no synchronisation). */
 lfqs_status lfqs_state_exchange_stats(const lfqs_state* s, uint64_t* exchanges,
                                       uint64_t* bytes_per_rank);
+/* Overlapped-exchange accounting (cumulative; benchmark / test use):
+ * exchanges run in parts (LFQS_OPT_EXCHANGE_CHUNK_BITS > 0), local passes run block by block
+ * around them (summed over the state's shards), exchanges whose chunk qubits were not the
+ * top local qubits (LFQS_OPT_EXCHANGE_CHUNK_SELECT), and exchanges chained onto the
+ * previous one (the whole run between them ran block by block).  Any pointer may be NULL. */
+lfqs_status lfqs_state_overlap_stats(const lfqs_state* s, uint64_t* overlapped_exchanges,
+                                     uint64_t* block_passes, uint64_t* strided_exchanges,
+                                     uint64_t* chained_exchanges);
 /* Number of kernels this state has launched so far (for benchmark accounting). */
 lfqs_status lfqs_kernel_launches(const lfqs_state* s, uint64_t* count);
 /* Number of state passes this state has run so far: one per fused pass or per single-gate
@@ -416,19 +424,19 @@ lfqs_status lfqs_state_pass_count(const lfqs_state* s, uint64_t* passes);
                                   tools/probe_sparse.cu); 0: read only the touched groups.
                                   Bit-identical results either way */
 #define LFQS_OPT_EXCHANGE_CHUNK_BITS 20 /* sharded states: each global-qubit exchange is
-                                  split into 2^value parts by the top `value` local qubits
-                                  (the planner never uses the top 2 as exchange positions,
+                                  split into 2^value parts (value in [0, 3]) by `value`
+                                  local "chunk" qubits (LFQS_OPT_EXCHANGE_CHUNK_SELECT; the
+                                  planner never uses the top 2 as exchange positions,
                                   whatever the value, so the plan does not depend on it;
                                   an exchange at a position among the top `value` runs
-                                  serially);
-                                  the local ops right before it and right after it that do
-                                  not touch those qubits run part by part on the state's
+                                  serially when the chunk qubits are the top ones);
+                                  the local passes right before it and right after it that
+                                  do not mix those qubits run part by part on the state's
                                   stream while the parts move on an exchange stream (NCCL:
                                   the communicator's stream) -- exchange overlapped with
-                                  local work.  Default 2; 0: serial exchanges.  Same
-                                  per-amplitude arithmetic; pass boundaries of fused runs
-                                  follow the split (rounding-level differences for dense
-                                  gates only) */
+                                  local work.  Default 2; 0: serial exchanges.  The same
+                                  passes and per-amplitude arithmetic as serial exchanges:
+                                  bit-identical results */
 #define LFQS_OPT_EXCHANGE_CTAS 21 /* grid of the device / P2P exchange swap kernels (a
                                      persistent grid-stride kernel); 0 (default): one
                                      thread per pair.  A small grid saturates NVLink and
@@ -441,6 +449,21 @@ lfqs_status lfqs_state_pass_count(const lfqs_state* s, uint64_t* passes);
                                      multiply-adds per amplitude than the separate gates
                                      (e.g. Sycamore-like 1-target layers into fSim).
                                      Rounding changes only (dense tolerance class) */
+#define LFQS_OPT_EXCHANGE_CHUNK_SELECT 23 /* 1 (default): fused runs on the device / P2P
+                                  transports choose each exchange's chunk qubits among the
+                                  local qubits at or above the fused tile size, the ones
+                                  left unmixed by the most planned ops around the exchange
+                                  (and keep the previous exchange's when the run between
+                                  the two leaves them unmixed: the run then flows block by
+                                  block from one exchange into the next); rank-independent
+                                  (decided from the plan).  0, per-gate runs and NCCL: the
+                                  top local qubits.  Bit-identical results either way */
+#define LFQS_OPT_EXCHANGE_RATE_GBS 24 /* > 0: the device / P2P exchange swap kernel (grid
+                                  LFQS_OPT_EXCHANGE_CTAS, 64 if 0) paces itself to this many
+                                  GB/s per direction -- a link-rate emulation, so that the
+                                  one-GPU virtual partition shows how much of an NVLink
+                                  exchange the overlapped local passes hide; default 0
+                                  (unpaced).  Same results */
 lfqs_status lfqs_set_option(lfqs_state* s, int option, int64_t value);
 const char* lfqs_last_error(void);
 int lfqs_abi_version(void);

@@ -52,6 +52,8 @@ OPT_LINE_READS = 19
 OPT_EXCHANGE_CHUNK_BITS = 20
 OPT_EXCHANGE_CTAS = 21
 OPT_FUSE_MERGE_2Q = 22
+OPT_EXCHANGE_CHUNK_SELECT = 23
+OPT_EXCHANGE_RATE_GBS = 24
 
 STATUS = {0: "OK", -1: "INVALID_ARG", -2: "OUT_OF_MEMORY", -3: "CUDA", -4: "NCCL",
           -5: "UNSUPPORTED"}
@@ -68,6 +70,7 @@ EXPORTS = [
     "lfqs_circuit_compile", "lfqs_circuit_launch", "lfqs_circuit_destroy",
     "lfqs_state_create_p2p", "lfqs_state_p2p_handle", "lfqs_state_p2p_attach",
     "lfqs_state_exchange_stats", "lfqs_jit_precompile", "lfqs_run_circuit_streamed",
+    "lfqs_state_overlap_stats",
 ]
 P2P_HANDLE_BYTES = 256
 STATE_C64 = 1
@@ -140,6 +143,8 @@ def lib():
             "lfqs_state_p2p_handle": [vp, C.POINTER(C.c_uint8)],
             "lfqs_state_p2p_attach": [vp, C.POINTER(C.c_uint8)],
             "lfqs_state_exchange_stats": [vp, C.POINTER(u64), C.POINTER(u64)],
+            "lfqs_state_overlap_stats": [vp, C.POINTER(u64), C.POINTER(u64), C.POINTER(u64),
+                                         C.POINTER(u64)],
             "lfqs_circuit_destroy": [vp],
             "lfqs_measure_probs": [vp, ip, C.c_int, dp, C.c_size_t],
             "lfqs_synchronize": [vp],
@@ -670,6 +675,13 @@ class State:
         a, b = C.c_uint64(), C.c_uint64()
         _check(lib().lfqs_state_exchange_stats(self.h, C.byref(a), C.byref(b)))
         return a.value, b.value
+
+    def overlap_stats(self) -> dict:
+        """Cumulative overlapped-exchange accounting (lfqs_state_overlap_stats)."""
+        v = [C.c_uint64() for _ in range(4)]
+        _check(lib().lfqs_state_overlap_stats(self.h, *[C.byref(x) for x in v]))
+        return dict(zip(("overlapped", "block_passes", "strided", "chained"),
+                        (x.value for x in v)))
 
     def launches(self) -> int:
         return lfqs_kernel_launches(self.h)

@@ -481,6 +481,19 @@ lfqs_status lfqs_state_exchange_stats(const lfqs_state* s, uint64_t* exchanges,
   });
 }
 
+lfqs_status lfqs_state_overlap_stats(const lfqs_state* s, uint64_t* overlapped_exchanges,
+                                     uint64_t* block_passes, uint64_t* strided_exchanges,
+                                     uint64_t* chained_exchanges) {
+  return guarded([&] {
+    require(s != nullptr, "NULL state");
+    const State* st = static_cast<const State*>(s);
+    if (overlapped_exchanges) *overlapped_exchanges = st->ov_exchanges;
+    if (block_passes) *block_passes = st->ov_block_passes;
+    if (strided_exchanges) *strided_exchanges = st->ov_strided;
+    if (chained_exchanges) *chained_exchanges = st->ov_chained;
+  });
+}
+
 lfqs_status lfqs_state_info(const lfqs_state* s, int* n_qubits, int* n_local, int* rank,
                             int* world, void** dev_ptr) {
   return guarded([&] {
@@ -523,8 +536,13 @@ lfqs_status lfqs_set_option(lfqs_state* s, int option, int64_t value) {
       case LFQS_OPT_LINE_READS: st->opt.line_reads = value != 0; break;
       case LFQS_OPT_FUSE_MERGE_2Q: st->opt.fuse_merge_2q = value != 0; break;
       case LFQS_OPT_EXCHANGE_CHUNK_BITS:
-        require(value >= 0 && value <= 4, "LFQS_OPT_EXCHANGE_CHUNK_BITS must be in [0, 4]");
+        require(value >= 0 && value <= 3, "LFQS_OPT_EXCHANGE_CHUNK_BITS must be in [0, 3]");
         st->opt.exchange_chunk_bits = (int)value;  // the plan is the same for every value
+        break;
+      case LFQS_OPT_EXCHANGE_CHUNK_SELECT: st->opt.exchange_chunk_select = value != 0; break;
+      case LFQS_OPT_EXCHANGE_RATE_GBS:
+        require(value >= 0 && value <= 100000, "LFQS_OPT_EXCHANGE_RATE_GBS must be in [0, 100000]");
+        st->opt.exchange_rate_gbs = (int)value;
         break;
       case LFQS_OPT_EXCHANGE_CTAS:
         require(value >= 0 && value <= 65535, "LFQS_OPT_EXCHANGE_CTAS must be in [0, 65535]");

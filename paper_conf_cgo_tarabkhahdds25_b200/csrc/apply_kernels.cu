@@ -376,26 +376,43 @@ __global__ void __launch_bounds__(kThreads) k_lanegroup(cx<S>* __restrict__ a, u
 // (a[k | 2^l], a[k + partner]) for the free indices k (bit l inserted as 0), two
 // adjacent pairs per item when l > 0 (32-B accesses on both sides).
 // ---------------------------------------------------------------------------
+__device__ __forceinline__ uint64_t globaltimer_ns() {
+  uint64_t t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
+
+// Grid-limited exchange swap (persistent, grid-stride).  period_ns > 0 paces it: the
+// grid's j-th round of items starts no earlier than j * period_ns after the CTA started
+// (a link-rate emulation, LFQS_OPT_EXCHANGE_RATE_GBS).
 template <class S>
 __global__ void __launch_bounds__(kThreads) k_xswap(cx<S>* __restrict__ a, uint64_t n_pairs,
-                                                     int l, uint64_t partner) {
+                                                     int l, uint64_t partner, InsertPlan ip,
+                                                     uint64_t period_ns) {
+  // ip inserts 0 at l and the block's fixed bits (never at position 0 when l > 0)
   const uint64_t stride = (uint64_t)gridDim.x * kThreads;
   const uint64_t bit = 1ull << l;
-  if (l > 0) {
-    const uint64_t n_items = n_pairs / 2;
-    for (uint64_t i = (uint64_t)blockIdx.x * kThreads + threadIdx.x; i < n_items; i += stride) {
-      const uint64_t f = i << 1;
-      const uint64_t lo = f & (bit - 1);
-      const uint64_t k = ((f - lo) << 1) | lo;
+  const uint64_t n_items = l > 0 ? n_pairs / 2 : n_pairs;
+  const uint64_t t0 = period_ns ? globaltimer_ns() : 0;
+  uint64_t round = 0;
+  for (uint64_t b0 = (uint64_t)blockIdx.x * kThreads; b0 < n_items; b0 += stride, ++round) {
+    if (period_ns) {
+      if (threadIdx.x == 0)
+        while (globaltimer_ns() < t0 + round * period_ns) {
+        }
+      __syncthreads();
+    }
+    const uint64_t i = b0 + threadIdx.x;
+    if (i >= n_items) continue;
+    if (l > 0) {
+      const uint64_t k = expand<6>(ip, i << 1);
       cx<S> x0, x1, y0, y1;
       ld2(a + (k | bit), x0, x1);
       ld2(a + k + partner, y0, y1);
       st2(a + (k | bit), y0, y1);
       st2(a + k + partner, x0, x1);
-    }
-  } else {
-    for (uint64_t i = (uint64_t)blockIdx.x * kThreads + threadIdx.x; i < n_pairs; i += stride) {
-      const uint64_t k = i << 1;
+    } else {
+      const uint64_t k = expand<6>(ip, i);
       const cx<S> x = ld1(a + (k | 1)), y = ld1(a + k + partner);
       st1(a + (k | 1), y);
       st1(a + k + partner, x);
@@ -760,25 +777,35 @@ void launch_gate_t(const LaunchCtx& ctx, const Decoded& g) {
 
 // Virtual-partition exchange: swap the l=1 half of this shard with the l=0 half
 // of the shard `partner_offset_amps` amplitudes further on (same pass structure
-// as a SWAP gate).
-// n_pairs = 0: all 2^(n_local-1) pairs; otherwise the first n_pairs (the P2P
-// exchange splits the pairs between the two ranks, p2p.cu).  The partner may be
-// any address (a peer GPU's shard mapped by CUDA IPC): the offset wraps mod 2^64.
-void launch_half_swap(const LaunchCtx& ctx, int l, uint64_t partner_offset_amps, uint64_t n_pairs,
-                      int ctas) {
-  const InsertPlan ip = make_plan(1ull << l, 0);
+// as a SWAP gate), over the amplitudes whose bits fix_zero are 0 and fix_one
+// are 1 (a block of an overlapped exchange; the P2P exchange also fixes one bit to split
+// the pairs between the two ranks, p2p.cu).  The partner may be any address (a peer
+// GPU's shard mapped by CUDA IPC): the offset wraps mod 2^64.
+void launch_half_swap(const LaunchCtx& ctx, int l, uint64_t partner_offset_amps, int ctas,
+                      uint64_t fix_zero, uint64_t fix_one) {
+  const uint64_t fixed = fix_zero | fix_one;
+  require(!(fixed >> l & 1) && !(fix_zero & fix_one) && __builtin_popcountll(fixed) <= 4 &&
+              (fixed >> ctx.n_local) == 0 && (l == 0 || !(fixed & 1)),
+          "internal: bad exchange block");
+  const InsertPlan ip = make_plan((1ull << l) | fix_zero, fix_one);
   Offs<2> off{{1ull << l, partner_offset_amps}};
-  if (n_pairs == 0) n_pairs = 1ull << (ctx.n_local - 1);
-  if (ctas > 0) {
+  const uint64_t n_pairs = 1ull << (ctx.n_local - 1 - __builtin_popcountll(fixed));
+  const int rate = ctx.opt->exchange_rate_gbs;
+  if (ctas > 0 || rate > 0) {
     // Grid-limited (persistent, grid-stride) variant: an exchange overlapped with local
     // passes needs only the SMs that saturate the link (NVLink 5: ~900 GB/s per direction,
-    // an eighth of HBM), leaving the rest to the concurrent compute stream.
+    // an eighth of HBM), leaving the rest to the concurrent compute stream.  With a rate
+    // (bytes per direction per ns = GB/s) each round of the grid is paced to it.
+    if (ctas <= 0) ctas = 64;
+    const uint64_t per_item = (uint64_t)(ctx.c64 ? 8 : 16) * (l > 0 ? 2 : 1);
+    const uint64_t period =
+        rate > 0 ? ((uint64_t)ctas * kThreads * per_item + rate - 1) / (uint64_t)rate : 0;
     if (ctx.c64)
       k_xswap<float><<<ctas, kThreads, 0, ctx.stream>>>(reinterpret_cast<cx<float>*>(ctx.amps),
-                                                         n_pairs, l, partner_offset_amps);
+                                                         n_pairs, l, partner_offset_amps, ip, period);
     else
       k_xswap<double><<<ctas, kThreads, 0, ctx.stream>>>(reinterpret_cast<cx<double>*>(ctx.amps),
-                                                          n_pairs, l, partner_offset_amps);
+                                                          n_pairs, l, partner_offset_amps, ip, period);
     LFQS_CUDA_CHECK(cudaGetLastError());
     ++*ctx.launch_counter;
     return;

@@ -384,7 +384,7 @@ __device__ __forceinline__ uint64_t tile_addr(const FTile& tg, uint64_t base, ui
 // (profiles/r01_c64_occupancy.md).
 template <int K, bool DIRECT, class S>
 __global__ void __launch_bounds__(kFThreads, sizeof(S) == 4 ? 4 : 2) k_fused(cx<S>* __restrict__ a,
-                                                        uint64_t tile_off,
+                                                        uint64_t tile_ins,
                                                         const __grid_constant__ FProg prog) {
   using C = cx<S>;
   constexpr uint32_t T = 1u << K;
@@ -396,8 +396,18 @@ __global__ void __launch_bounds__(kFThreads, sizeof(S) == 4 ? 4 : 2) k_fused(cx<
   const uint32_t tid = threadIdx.x;
   const FTile& tg = prog.tile;
   const int lc = tg.lc, nh = tg.nh;
-  // Tile base: the tile index with zeros inserted at every tile qubit.
-  uint64_t base = ((uint64_t)blockIdx.x + tile_off) << lc;  // tile_off: first tile of a block
+  // Tile base: the tile index with zeros inserted at every tile qubit.  tile_ins (a
+  // block of the state, for overlapped exchanges): up to three fixed bits inserted into
+  // the tile index first (tile_insertions()).
+  uint64_t t = blockIdx.x;
+#pragma unroll
+  for (int i = 0; i < 3; ++i) {
+    const uint32_t b = (uint32_t)(tile_ins >> (8 * i)) & 0x7f;
+    const int p = b & 63;
+    const uint64_t lo = t & ((1ull << p) - 1);
+    t = ((t - lo) << 1) | lo | ((uint64_t)(b >> 6) << p);
+  }
+  uint64_t base = t << lc;
   for (int i = 0; i < nh; ++i) {
     const int p = tg.hpos[i];
     const uint64_t lo = base & ((1ull << p) - 1);
@@ -746,28 +756,28 @@ void encode(const Decoded& g, const TileMap& tm, FProg& P) {
 }
 
 template <int K, bool DIRECT, class S>
-void launch_kd(const LaunchCtx& ctx, const FProg& P, uint64_t tile_off) {
+void launch_kd(const LaunchCtx& ctx, const FProg& P, uint64_t tile_ins) {
   const size_t smem = sizeof(cx<S>) << K;
   ensure_smem_attr((const void*)k_fused<K, DIRECT, S>, (int)smem);
   const uint64_t tiles = 1ull << (ctx.n_local - K);
   k_fused<K, DIRECT, S><<<(unsigned)tiles, kFThreads, smem, ctx.stream>>>(
-      reinterpret_cast<cx<S>*>(ctx.amps), tile_off, P);
+      reinterpret_cast<cx<S>*>(ctx.amps), tile_ins, P);
 }
 // TMA bulk copies for tiles of at most fuse_tma_max_chunks chunks (default: all),
 // direct register loads otherwise.
 template <int K>
-void launch_k(const LaunchCtx& ctx, const FProg& P, uint64_t tile_off) {
+void launch_k(const LaunchCtx& ctx, const FProg& P, uint64_t tile_ins) {
   const bool direct = (1 << P.tile.nh) > ctx.opt->fuse_tma_max_chunks;
   if (ctx.c64) {
     if (direct)
-      launch_kd<K, true, float>(ctx, P, tile_off);
+      launch_kd<K, true, float>(ctx, P, tile_ins);
     else
-      launch_kd<K, false, float>(ctx, P, tile_off);
+      launch_kd<K, false, float>(ctx, P, tile_ins);
   } else {
     if (direct)
-      launch_kd<K, true, double>(ctx, P, tile_off);
+      launch_kd<K, true, double>(ctx, P, tile_ins);
     else
-      launch_kd<K, false, double>(ctx, P, tile_off);
+      launch_kd<K, false, double>(ctx, P, tile_ins);
   }
 }
 
@@ -1138,22 +1148,22 @@ void build_program(const LaunchCtx& ctx, const TileCfg& cfg, uint64_t in_tile,
 
 // Launches an encoded pass: the compiled kernel of its program (LFQS_FUSE_JIT)
 // or the interpreting kernel k_fused<K>.
-// tile_off: the launch covers tiles [tile_off, tile_off + 2^(ctx.n_local - K)) of the state
-// at ctx.amps (a block whose top bits are fixed, for overlapped exchanges; 0 otherwise).
+// The launch covers 2^(ctx.n_local - K) tiles; tile_ins (tile_insertions()) fixes up to
+// three more bits of the tile index (a block of the state, for overlapped exchanges).
 void launch_built(const LaunchCtx& ctx, int K, const FProg& P, const std::string* key = nullptr,
-                  uint64_t tile_off = 0) {
+                  uint64_t tile_ins = kNoTileIns) {
   if (ctx.jit && (1 << P.tile.nh) <= ctx.opt->fuse_tma_max_chunks) {
     const int jc = jit_config(ctx, K, &P);
-    jit_launch(ctx, P, K, key ? *key : jit_key(P, K, ctx.c64, jc), jc, tile_off);
+    jit_launch(ctx, P, K, key ? *key : jit_key(P, K, ctx.c64, jc), jc, tile_ins);
     ++*ctx.launch_counter;
     return;
   }
   switch (K) {
-    case 8: launch_k<8>(ctx, P, tile_off); break;
-    case 9: launch_k<9>(ctx, P, tile_off); break;
-    case 10: launch_k<10>(ctx, P, tile_off); break;
-    case 11: launch_k<11>(ctx, P, tile_off); break;
-    default: launch_k<12>(ctx, P, tile_off); break;
+    case 8: launch_k<8>(ctx, P, tile_ins); break;
+    case 9: launch_k<9>(ctx, P, tile_ins); break;
+    case 10: launch_k<10>(ctx, P, tile_ins); break;
+    case 11: launch_k<11>(ctx, P, tile_ins); break;
+    default: launch_k<12>(ctx, P, tile_ins); break;
   }
   LFQS_CUDA_CHECK(cudaGetLastError());
   ++*ctx.launch_counter;
@@ -1350,21 +1360,52 @@ void launch_fused_pass(const LaunchCtx& ctx, const std::vector<Decoded>& gates,
     launch_gate(ctx, gates[ps.gate]);
 }
 
-void launch_fused_pass_block(const LaunchCtx& ctx, const std::vector<Decoded>& gates,
-                             const FusedPass& ps, int c, uint64_t v) {
+// Block v of the chunk qubits (lfqs_internal.h): fused passes fix the chunk bits in the
+// tile index (tile-index insertions), so the pass runs over the block's tiles only; a
+// single gate runs on the contiguous block of the top chunk qubits, its controls and
+// diagonal entries on them resolved on the host as the planner does for a rank's global
+// bits (Planner::rank_local with the block index in the role of the rank).
+bool pass_blockwise(const FusedPass& ps, uint64_t chunk, int n_local) {
+  const int c = __builtin_popcountll(chunk);
+  if (c == 0 || c > 3 || (ps.nd_mask & chunk) || (chunk >> n_local)) return false;
+  if (!ps.prog) return chunk == (((1ull << c) - 1) << (n_local - c));
+  if (ps.K > n_local - c) return false;
+  const FTile& tg = ps.prog->tile;
+  uint64_t in_tile = (1ull << tg.lc) - 1;
+  for (int i = 0; i < tg.nh; ++i) in_tile |= 1ull << tg.hpos[i];
+  return (chunk & in_tile) == 0;
+}
+
+namespace {
+uint64_t tile_insertions(const FTile& tg, uint64_t chunk, uint64_t v) {
+  uint64_t ins = kNoTileIns;
+  int i = 0;
+  for (int q = 0; q < 64; ++q) {
+    if (!(chunk >> q & 1)) continue;
+    int below = 0;  // tile qubits below q
+    for (int h = 0; h < tg.nh; ++h) below += tg.hpos[h] < q;
+    const int tp = q - tg.lc - below;  // q's position in the tile index
+    require(q >= tg.lc && tp >= 0 && tp < 63 && i < 3, "internal: chunk qubit inside the tile");
+    ins &= ~(0xffull << (8 * i));
+    ins |= (uint64_t)(tp | (int)((v >> i) & 1) << 6) << (8 * i);
+    ++i;
+  }
+  return ins;
+}
+}  // namespace
+
+void launch_fused_pass_part(const LaunchCtx& ctx, const std::vector<Decoded>& gates,
+                            const FusedPass& ps, uint64_t chunk, uint64_t v) {
+  require(pass_blockwise(ps, chunk, ctx.n_local), "internal: pass not confined to the block");
+  const int c = __builtin_popcountll(chunk);
   const int n_sub = ctx.n_local - c;
-  require(c >= 0 && n_sub >= 1 && (ps.nd_mask >> n_sub) == 0,
-          "internal: pass not confined to the block");
   if (ps.prog) {
-    require(n_sub >= ps.K, "internal: block smaller than the pass's tile");
-    LaunchCtx x = ctx;  // same base pointer; the tiles of block v only
+    LaunchCtx x = ctx;  // same base pointer; the block's tiles only
     x.n_local = n_sub;
-    launch_built(x, ps.K, *ps.prog, ps.key.empty() ? nullptr : &ps.key, v << (n_sub - ps.K));
+    launch_built(x, ps.K, *ps.prog, ps.key.empty() ? nullptr : &ps.key,
+                 tile_insertions(ps.prog->tile, chunk, v));
     return;
   }
-  // A single gate: its controls / diagonal entries on the block's fixed top bits are
-  // resolved on the host, as the planner does for a rank's global bits (Planner::rank_local
-  // with the block index in the role of the rank), then it runs on the block.
   Planner blk(ctx.n_local, 1 << c);
   Decoded lg;
   if (!blk.rank_local(gates[ps.gate], (int)v, 0, &lg) || lg.cls == GClass::NOOP) return;

@@ -44,6 +44,13 @@ struct FProg {
 };
 static_assert(sizeof(FProg) + 8 <= 32764, "kernel parameter limit");
 
+// Tile-index insertions of a launch (k_fused / compiled passes): byte i (i = 0..2, by
+// ascending position) = position p (bits 0-5, in tile-index space) | value << 6 of a bit
+// inserted into the block index before it becomes the tile base; p = 63 inserts nothing.
+// A launch with insertions covers the tiles of one block of the state (the amplitudes
+// whose chunk qubits hold fixed values -- overlapped exchanges, state.cu).
+constexpr uint64_t kNoTileIns = 0x3f3f3full;
+
 constexpr int kFThreads = 256;
 constexpr int kMinK = 8, kMaxK = 12;
 

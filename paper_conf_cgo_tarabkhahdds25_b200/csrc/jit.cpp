@@ -1610,8 +1610,25 @@ struct Gen {
     e("mov.u32 %%ltid, %%tid.x;");
     e("mov.u32 %%bid, %%ctaid.x;");
     e("cvt.u64.u32 %%base, %%bid;");
-    e("ld.param.u64 %%toff, [poff];");  // first tile of the launch (a block of the state)
-    e("add.u64 %%base, %%base, %%toff;");
+    // tile-index insertions (kNoTileIns: none): the fixed bits of a block of the state
+    e("ld.param.u64 %%toff, [poff];");
+    for (int i = 0; i < 3; ++i) {
+      const std::string x = rd(), b = r(), pp = r(), vv = r(), m = rd(), lo = rd(), v64 = rd();
+      e("shr.u64 %s, %%toff, %d;", x.c_str(), 8 * i);
+      e("cvt.u32.u64 %s, %s;", b.c_str(), x.c_str());
+      e("and.b32 %s, %s, 63;", pp.c_str(), b.c_str());
+      e("bfe.u32 %s, %s, 6, 1;", vv.c_str(), b.c_str());
+      e("mov.b64 %s, 1;", m.c_str());
+      e("shl.b64 %s, %s, %s;", m.c_str(), m.c_str(), pp.c_str());
+      e("sub.u64 %s, %s, 1;", m.c_str(), m.c_str());
+      e("and.b64 %s, %%base, %s;", lo.c_str(), m.c_str());
+      e("sub.u64 %%base, %%base, %s;", lo.c_str());
+      e("shl.b64 %%base, %%base, 1;");
+      e("or.b64 %%base, %%base, %s;", lo.c_str());
+      e("cvt.u64.u32 %s, %s;", v64.c_str(), vv.c_str());
+      e("shl.b64 %s, %s, %s;", v64.c_str(), v64.c_str(), pp.c_str());
+      e("or.b64 %%base, %%base, %s;", v64.c_str());
+    }
     e("shl.b64 %%base, %%base, %d;", tg.lc);
     for (int i = 0; i < tg.nh; ++i) {
       const int pp = tg.hpos[i];
@@ -2011,7 +2028,7 @@ size_t jit_cache_size() {
 }
 
 void jit_launch(const LaunchCtx& ctx, const FProg& P, int K, const std::string& key, int jc,
-                uint64_t tile_off) {
+                uint64_t tile_ins) {
   const int nt = jc & JIT_THREADS_MASK;
   std::shared_ptr<Entry> en;
   {
@@ -2053,7 +2070,7 @@ void jit_launch(const LaunchCtx& ctx, const FProg& P, int K, const std::string& 
     }
   }
   void* a = ctx.amps;
-  void* args[3] = {&a, &tile_off, (void*)P.c};
+  void* args[3] = {&a, &tile_ins, (void*)P.c};
   const uint64_t tiles = 1ull << (ctx.n_local - K);
   LFQS_CUDA_CHECK(cudaLaunchKernel((const void*)en->kern, dim3((unsigned)tiles), dim3(nt),
                                    args, (size_t)smem, ctx.stream));

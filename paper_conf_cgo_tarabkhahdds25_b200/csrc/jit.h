@@ -26,9 +26,9 @@ std::string jit_key(const FProg& P, int K, bool c64, int jc);
 void jit_compile(const std::vector<std::pair<std::string, const FProg*>>& items, int K, bool c64,
                  int jc);
 // Launches the pass (compiling it first if needed) on ctx.stream: 2^(ctx.n_local - K) tiles,
-// tile indices starting at tile_off (a block of the state whose top bits are fixed).
+// with the tile-index insertions tile_ins (fused_prog.h; a block of the state).
 void jit_launch(const LaunchCtx& ctx, const FProg& P, int K, const std::string& key, int jc,
-                uint64_t tile_off = 0);
+                uint64_t tile_ins = kNoTileIns);
 // Generator configuration of pass P for tile size K (LFQS_OPT_JIT_THREADS -- 0: chosen per
 // pass from P -- LFQS_OPT_JIT_LANE_MOVE, ...).
 int jit_config(const LaunchCtx& ctx, int K, const FProg* P = nullptr);

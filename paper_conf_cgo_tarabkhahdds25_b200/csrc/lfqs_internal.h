@@ -85,11 +85,14 @@ struct Options {
   bool wide256 = true;       // two adjacent groups per item, 32-byte accesses
   bool line_reads = true;    // fixed bits 1-2 -> store predicate, whole-line reads (apply_kernels.cu)
   // Global-qubit exchanges overlapped with local work (state.cu execute): the
-  // exchange is split into 2^exchange_chunk_bits parts by the top local qubits; the last
+  // exchange is split into 2^exchange_chunk_bits parts by as many local qubits; the last
   // local ops before it and the first after it run part by part on the compute stream
   // while the parts move on the exchange stream.  0 bits: serial exchanges.
   int exchange_chunk_bits = 2;
+  bool exchange_chunk_select = true;  // chunk qubits chosen per exchange (state.cu choose_chunk)
   int exchange_ctas = 0;     // grid of the (device / P2P) exchange swap kernels; 0: full grid
+  int exchange_rate_gbs = 0; // > 0: the swap kernel paced to this many GB/s per direction
+                             // (a link-rate emulation for the one-GPU virtual partition)
   int fuse_tile_qubits = 12;
   int fuse_low_qubits = 0;   // contiguous low qubits of a fused tile (chunk = 2^L amps);
                              // 0: auto, 7 or 6 by planned pass count (fused_kernels.cu)
@@ -142,12 +145,13 @@ void launch_gate(const LaunchCtx& ctx, const Decoded& g);
 // The same on a structure-of-arrays shard (soa_kernels.cu).
 void launch_gate_soa(const LaunchCtx& ctx, const Decoded& g);
 // Half-shard swap for the global-qubit exchange: the l=1 half of the shard at
-// ctx.amps with the l=0 half of the shard partner_offset_amps further on (first
-// n_pairs pairs; 0 = all).
+// ctx.amps with the l=0 half of the shard partner_offset_amps further on, restricted to
+// the amplitudes whose bits fix_zero are 0 and fix_one are 1 (a block of an overlapped
+// exchange, or one rank's share of the pairs; <= 4 fixed bits, none at l).
 // ctas > 0: a grid of at most that many CTAs (persistent grid-stride kernel) -- for
 // exchanges overlapped with local passes on another stream.
-void launch_half_swap(const LaunchCtx& ctx, int l, uint64_t partner_offset_amps,
-                      uint64_t n_pairs = 0, int ctas = 0);
+void launch_half_swap(const LaunchCtx& ctx, int l, uint64_t partner_offset_amps, int ctas = 0,
+                      uint64_t fix_zero = 0, uint64_t fix_one = 0);
 
 // Fused staging of gates[begin..): applies the longest prefix that fits one tile
 // program in one HBM pass; false if fewer than two gates fuse (fused_kernels.cu).
@@ -173,12 +177,16 @@ void plan_fused_schedule(const LaunchCtx& ctx, const std::vector<Decoded>& gates
 // n_local) that contains every qubit in ps.qmask.
 void launch_fused_pass(const LaunchCtx& ctx, const std::vector<Decoded>& gates,
                        const FusedPass& ps);
-// Launches it on block v of the shard ctx: the amplitudes whose top c bits equal v.  The
-// pass must not mix those bits (ps.nd_mask below n_local - c); controls and diagonal
-// entries on them are resolved for the block (exactly the ops the whole-shard pass applies
-// to these amplitudes, with the same kernels and formulas).
-void launch_fused_pass_block(const LaunchCtx& ctx, const std::vector<Decoded>& gates,
-                             const FusedPass& ps, int c, uint64_t v);
+// Block v of the chunk qubits `chunk` (<= 3 positions of the shard): the amplitudes whose
+// chunk bits, read in ascending position order, spell v.  A pass can run block by block
+// when it does not mix the chunk qubits (pass_blockwise): a fused pass whose tile holds
+// none of them (they are fixed bits of its tile index), or a single gate when the chunk
+// qubits are the top ones of the shard (a contiguous block).  Controls and diagonal
+// entries on them are resolved for the block -- exactly the ops the whole-shard pass
+// applies to these amplitudes, with the same kernels and formulas.
+bool pass_blockwise(const FusedPass& ps, uint64_t chunk, int n_local);
+void launch_fused_pass_part(const LaunchCtx& ctx, const std::vector<Decoded>& gates,
+                            const FusedPass& ps, uint64_t chunk, uint64_t v);
 
 // Reductions (C9): d_out[v], v < 2^nq (nq <= 20, bit s of v = bit qubits[s]); one read
 // pass over the shard whatever nq is; deterministic (fixed grid and summation order).

@@ -180,23 +180,31 @@ void P2P::barrier_all(cudaStream_t s) {
   LFQS_CUDA_CHECK(cudaGetLastError());
 }
 
-void P2P::exchange(const LaunchCtx& ctx, int l, int j, int n_sub, uint64_t offset, int ctas) {
+void P2P::exchange(const LaunchCtx& ctx, int l, int j, uint64_t chunk, uint64_t v, int ctas) {
   const int partner = rank ^ (1 << j);
   const int b = (rank >> j) & 1;
   const int low = b ? partner : rank, high = b ? rank : partner;
   const int ab = ctx.c64 ? 8 : 16;
-  require(l < n_sub && n_sub >= 2, "internal: exchange position outside the block");
-  // Pairs (low[k | 2^l], high[k]) for k with bit l = 0.  The index bit hb splits
-  // them: rank b swaps the pairs whose bit hb equals b.
-  const int hb = (l == n_sub - 1) ? n_sub - 2 : n_sub - 1;
+  const int nl = ctx.n_local;
+  require(l < nl && nl >= 2 && !(chunk >> l & 1) && (chunk >> nl) == 0,
+          "internal: exchange position inside the block's fixed bits");
+  // Pairs (low[k | 2^l], high[k]) for k with bit l = 0 in the block.  The highest free
+  // index bit hb splits them: rank b swaps the pairs whose bit hb equals b.
+  int hb = nl - 1;
+  while (hb == l || (chunk >> hb & 1)) --hb;
+  require(hb >= 1, "internal: no free bit to split the exchange");
+  uint64_t fz = 0, fo = 0;
+  int i = 0;
+  for (int q = 0; q < nl; ++q)
+    if (chunk >> q & 1) ((v >> i++ & 1) ? fo : fz) |= 1ull << q;
+  (b ? fo : fz) |= 1ull << hb;
   const int64_t d = reinterpret_cast<intptr_t>(peer_amps[high]) -
                     reinterpret_cast<intptr_t>(peer_amps[low]);
   require(d % (2 * ab) == 0, "internal: peer shards are not 32-byte aligned");
   barrier_pair(partner, ctx.stream);  // both blocks are final up to here
   LaunchCtx c = ctx;
-  c.amps = peer_amps[low] + (offset + ((uint64_t)b << hb)) * ab;
-  c.n_local = n_sub;
-  launch_half_swap(c, l, (uint64_t)(d / ab), 1ull << (n_sub - 2), ctas);
+  c.amps = peer_amps[low];
+  launch_half_swap(c, l, (uint64_t)(d / ab), ctas, fz, fo);
   barrier_pair(partner, ctx.stream);  // both halves swapped before either moves on
 }
 

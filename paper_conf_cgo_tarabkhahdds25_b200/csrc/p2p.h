@@ -44,10 +44,10 @@ struct P2P {
   void barrier_all(cudaStream_t s);
   // In-place half-shard exchange with the partner across global bit j (local
   // position l): this rank swaps its half of the pairs.  The exchange covers the
-  // 2^n_sub amplitudes from amplitude `offset` of both shards (a whole shard: offset 0,
-  // n_sub = n_local; one part of an overlapped exchange: a contiguous 2^n_sub block),
-  // on ctx.stream (barriers included); ctas > 0 bounds the swap kernel's grid.
-  void exchange(const LaunchCtx& ctx, int l, int j, int n_sub, uint64_t offset = 0,
+  // amplitudes of both shards whose bits `chunk` spell v in ascending position order
+  // (a whole shard: chunk = 0; one block of an overlapped exchange otherwise), on
+  // ctx.stream (barriers included); ctas > 0 bounds the swap kernel's grid.
+  void exchange(const LaunchCtx& ctx, int l, int j, uint64_t chunk = 0, uint64_t v = 0,
                 int ctas = 0);
   // out[0..count) = sum over ranks (in rank order) of every rank's in[0..count)
   // (host arrays).  Synchronous.

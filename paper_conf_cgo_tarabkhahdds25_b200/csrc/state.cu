@@ -306,10 +306,10 @@ void State::exchange_data(int l, int g) {
     for (int r = 0; r < world; ++r) {
       if (r >> j & 1) continue;
       const int r2 = r | (1 << j);
-      launch_half_swap(ctx(r), l, ((uint64_t)(r2 - r)) << n_local, 0, opt.exchange_ctas);
+      launch_half_swap(ctx(r), l, ((uint64_t)(r2 - r)) << n_local, opt.exchange_ctas);
     }
   } else if (p2p) {
-    p2p->exchange(ctx(0), l, j, n_local, 0, opt.exchange_ctas);
+    p2p->exchange(ctx(0), l, j, 0, 0, opt.exchange_ctas);
   } else {
     const int b = (rank >> j) & 1;
     std::vector<Piece> pieces;
@@ -386,14 +386,14 @@ std::vector<State::ShardRun> State::plan_run(const std::vector<PlanOp>& ops, siz
 }
 
 void State::launch_passes(const std::vector<ShardRun>& run, const std::vector<size_t>& from,
-                          const std::vector<size_t>& to, int c, int v) {
+                          const std::vector<size_t>& to, uint64_t chunk, uint64_t v) {
   for (int s = 0; s < n_shards(); ++s) {
     if (from[s] >= to[s]) continue;
     const LaunchCtx x = ctx(s);
-    if (c == 0 || v == 0) passes += to[s] - from[s];
+    if (chunk == 0 || v == 0) passes += to[s] - from[s];
     for (size_t i = from[s]; i < to[s]; ++i) {
-      if (c > 0)
-        launch_fused_pass_block(x, run[s].seg, run[s].passes[i], c, (uint64_t)v);
+      if (chunk)
+        launch_fused_pass_part(x, run[s].seg, run[s].passes[i], chunk, v);
       else
         launch_fused_pass(x, run[s].seg, run[s].passes[i]);
     }
@@ -415,33 +415,121 @@ cudaEvent_t State::part_event(std::vector<cudaEvent_t>& pool, int v) {
   return pool[v];
 }
 
-cudaEvent_t State::exchange_part(int l, int g, int c, int v, cudaEvent_t ready) {
-  const int j = g - n_local, ns = n_local - c;
-  const uint64_t off = (uint64_t)v << ns;
+// Chunk qubits of the exchange ops[ex[k]] (0: run it serially).  The choice depends only
+// on the planned ops, never on a rank's own passes, so every rank of a P2P / NCCL state
+// picks the same blocks.  Per-gate execution (no fused passes) and the NCCL transport use
+// the top c local qubits (contiguous blocks, single-gate passes can run on them; NCCL
+// sends each block's pieces).  Fused execution on the device / P2P transports picks the
+// c positions among the local qubits at or above the tile size (a fused pass holds such a
+// qubit in its tile only when it mixes it, fused_kernels.cu) that stay unmixed longest
+// around the exchange: the most ops before it (back to the previous exchange) plus after
+// it (to the next one) free of non-diagonal gates on them; the previous exchange's chunk
+// qubits win when the whole run between the two leaves them unmixed (the run then runs
+// block by block between the two exchanges' parts: a pipeline, state.cu execute).
+uint64_t State::choose_chunk(const std::vector<PlanOp>& ops, const std::vector<size_t>& ex,
+                             size_t k, bool fuse, uint64_t prev) const {
+  const int c = overlap_bits();
+  if (c == 0) return 0;
+  const PlanOp& X = ops[ex[k]];
+  const uint64_t top = ((1ull << c) - 1) << (n_local - c);
+  const bool strided = fuse && (virt || p2p) && opt.exchange_chunk_select;
+  if (!strided) return (top >> X.l & 1) ? 0 : top;
+  const size_t b = k > 0 ? ex[k - 1] + 1 : 0, e = k + 1 < ex.size() ? ex[k + 1] : ops.size();
+  auto mixed = [&](const PlanOp& o) -> uint64_t {
+    uint64_t m = 0;
+    if (o.kind == PlanOp::EXCHANGE) return ~0ull;
+    if (o.gate.cls != GClass::DIAG && o.gate.cls != GClass::NOOP)
+      for (int t = 0; t < o.gate.m; ++t) m |= 1ull << o.gate.targets[t];
+    return m;
+  };
+  uint64_t run_mixed = 0;  // mixed by the run between the previous exchange and this one
+  for (size_t i = b; i < ex[k]; ++i) run_mixed |= mixed(ops[i]);
+  if (prev && !(prev >> X.l & 1) && !(run_mixed & prev)) return prev;
+  const int lo = std::max(opt.fuse_tile_qubits, 1);
+  if (n_local - lo < c + 1) return (top >> X.l & 1) ? 0 : top;
+  // ops before / after the exchange free of mixing, per position
+  int before[64], after[64];
+  for (int q = 0; q < 64; ++q) before[q] = after[q] = 0;
+  uint64_t seen = 0;
+  for (size_t i = ex[k]; i-- > b;) {
+    const uint64_t m = mixed(ops[i]);
+    seen |= m;
+    for (int q = lo; q < n_local; ++q)
+      if (!(seen >> q & 1)) ++before[q];
+  }
+  seen = 0;
+  for (size_t i = ex[k] + 1; i < e; ++i) {
+    const uint64_t m = mixed(ops[i]);
+    seen |= m;
+    for (int q = lo; q < n_local; ++q)
+      if (!(seen >> q & 1)) ++after[q];
+  }
+  std::vector<int> cand;
+  for (int q = lo; q < n_local; ++q)
+    if (q != X.l) cand.push_back(q);
+  uint64_t best = 0;
+  long best_score = -1;
+  auto consider = [&](uint64_t m) {
+    int tb = 1 << 30, ta = 1 << 30;
+    for (int q = 0; q < 64; ++q)
+      if (m >> q & 1) tb = std::min(tb, before[q]), ta = std::min(ta, after[q]);
+    const long sc = (long)tb + ta;
+    // ties: the top qubits (the contiguous blocks of the serial planner), then higher ones
+    if (sc > best_score || (sc == best_score && (m == top || (best != top && m > best)))) {
+      best = m;
+      best_score = sc;
+    }
+  };
+  const int nc = (int)cand.size();
+  for (int i0 = 0; i0 < nc; ++i0) {
+    const uint64_t m0 = 1ull << cand[i0];
+    if (c == 1) { consider(m0); continue; }
+    for (int i1 = i0 + 1; i1 < nc; ++i1) {
+      const uint64_t m1 = m0 | 1ull << cand[i1];
+      if (c == 2) { consider(m1); continue; }
+      for (int i2 = i1 + 1; i2 < nc; ++i2) consider(m1 | 1ull << cand[i2]);
+    }
+  }
+  return best;
+}
+
+cudaEvent_t State::exchange_part(int l, int g, uint64_t chunk, uint64_t v, cudaEvent_t ready) {
+  const int j = g - n_local;
   if (virt || p2p) {
-    if (xstream == nullptr)
-      LFQS_CUDA_CHECK(cudaStreamCreateWithFlags(&xstream, cudaStreamNonBlocking));
+    if (xstream == nullptr) {
+      // highest priority: the link transfer is on the critical path, so its CTAs are
+      // dispatched ahead of the compute stream's pending tiles
+      int lo = 0, hi = 0;
+      LFQS_CUDA_CHECK(cudaDeviceGetStreamPriorityRange(&lo, &hi));
+      LFQS_CUDA_CHECK(cudaStreamCreateWithPriority(&xstream, cudaStreamNonBlocking, hi));
+    }
     LFQS_CUDA_CHECK(cudaStreamWaitEvent(xstream, ready, 0));
+    uint64_t fz = 0, fo = 0;
+    int i = 0;
+    for (int q = 0; q < n_local; ++q)
+      if (chunk >> q & 1) ((v >> i++ & 1) ? fo : fz) |= 1ull << q;
     if (virt) {
       for (int r = 0; r < world; ++r) {
         if (r >> j & 1) continue;
         const int r2 = r | (1 << j);
         LaunchCtx x = ctx(r);
         x.stream = xstream;
-        x.amps = static_cast<unsigned char*>(x.amps) + off * ab;
-        x.n_local = ns;
-        launch_half_swap(x, l, ((uint64_t)(r2 - r)) << n_local, 0, opt.exchange_ctas);
+        launch_half_swap(x, l, ((uint64_t)(r2 - r)) << n_local, opt.exchange_ctas, fz, fo);
       }
     } else {
       LaunchCtx x = ctx(0);
       x.stream = xstream;
-      p2p->exchange(x, l, j, ns, off, opt.exchange_ctas);
+      p2p->exchange(x, l, j, chunk, v, opt.exchange_ctas);
     }
-    cudaEvent_t done = part_event(ev_done, v);
+    cudaEvent_t done = part_event(ev_done, (int)v);
     LFQS_CUDA_CHECK(cudaEventRecord(done, xstream));
     return done;
   }
-  // NCCL: this part's half (local bit l = 1 - own global bit) as contiguous pieces.
+  // NCCL: the top c local qubits (choose_chunk); this part's half (local bit l = 1 - own
+  // global bit) as contiguous pieces.
+  const int c = __builtin_popcountll(chunk), ns = n_local - c;
+  require(chunk == ((1ull << c) - 1) << ns, "internal: NCCL exchange blocks must be the top qubits");
+  const uint64_t off = v << ns;
   const int b = (rank >> j) & 1;
   std::vector<Piece> pieces;
   if (l == ns - 1) {
@@ -459,22 +547,22 @@ cudaEvent_t State::exchange_part(int l, int g, int c, int v, cudaEvent_t ready) 
 //
 // Global-qubit exchange overlapped with local work (BASELINE north_star
 // "overlapped with local work on separate streams"), Options::exchange_chunk_bits = c > 0:
-// an exchange at a position l below the top c local qubits (the planner keeps exchange
-// positions out of the top two, planner.h) moves data only inside each block whose top c
-// bits are fixed, so it splits into 2^c independent parts.  The trailing passes of the run
-// before it that do not mix those c qubits run part by part on the compute stream; part
-// v moves (exchange stream, or the NCCL stream) as soon as its tail is done, while the
-// compute stream goes on with the next part; the leading passes of the next run that do
-// not mix those qubits run on part v as soon as it has landed.  A pass "mixes" a qubit
-// when a non-diagonal gate targets it; controls and diagonal entries on the chunk qubits
-// are resolved per part (fused passes read them from the tile index, which starts at the
-// part's first tile; single gates are specialised on the host), so e.g. every QFT CPhase
-// pass can run part by part.  The passes are exactly the ones the
-// serial execution launches (no extra HBM pass), each applied block by block with the same
-// kernels, and every pass sees the data it would see in the serial order (Eq. 3; ops
-// on disjoint blocks commute): results are bit-identical to serial exchanges
-// (tests/test_gpu_overlap.py, tests/test_gpu_p2p.py).  Other exchanges (position among the
-// top c, e.g. during canonicalisation) run serially.
+// an exchange at local position l moves data only inside each block of the state whose c
+// chunk qubits (choose_chunk; never l) hold fixed values, so it splits into 2^c
+// independent parts.  The trailing passes of the run before it that do not mix the chunk
+// qubits run part by part on the compute stream; part v moves (exchange stream, or the
+// NCCL stream) as soon as its tail is done, while the compute stream goes on with the
+// next part; the leading passes of the next run that do not mix them run on part v as
+// soon as it has landed.  When those leading passes are the whole run and the next
+// exchange uses the same chunk qubits, its part v starts as soon as part v's run is done
+// (a pipeline across consecutive exchanges).  A pass "mixes" a qubit when a non-diagonal
+// gate targets it; controls and diagonal entries on the chunk qubits are resolved per
+// part (fused passes take them as fixed bits of the tile index; single gates are
+// specialised on the host), so e.g. every QFT CPhase pass can run part by part.  The
+// passes are exactly the ones the serial execution launches (no extra HBM pass), each
+// applied block by block with the same kernels, and every pass sees the data it would see
+// in the serial order (Eq. 3; ops on disjoint blocks commute): results are
+// bit-identical to serial exchanges (tests/test_gpu_overlap.py, tests/test_gpu_p2p.py).
 void State::execute(const std::vector<PlanOp>& ops, bool fuse) {
   std::vector<size_t> ex;
   for (size_t i = 0; i < ops.size(); ++i)
@@ -489,11 +577,10 @@ void State::execute(const std::vector<PlanOp>& ops, bool fuse) {
     }
     return;
   }
-  const int c = overlap_bits();
-  const uint64_t H = c > 0 ? ((1ull << c) - 1) << (n_local - c) : 0;
   const int S = n_shards();
   std::vector<ShardRun> cur = plan_run(ops, 0, ex.empty() ? ops.size() : ex[0], fuse);
   std::vector<size_t> from(S, 0), end(S);
+  uint64_t prev = 0;  // chunk of the previous exchange if its leading passes were its whole run
   for (size_t k = 0;; ++k) {
     for (int s = 0; s < S; ++s) end[s] = cur[s].passes.size();
     if (k == ex.size()) {
@@ -503,37 +590,51 @@ void State::execute(const std::vector<PlanOp>& ops, bool fuse) {
     const PlanOp& X = ops[ex[k]];
     const size_t nb = ex[k] + 1, ne = k + 1 < ex.size() ? ex[k + 1] : ops.size();
     std::vector<ShardRun> next = plan_run(ops, nb, ne, fuse);
-    if (c == 0 || X.l >= n_local - c) {
+    const uint64_t chunk = choose_chunk(ops, ex, k, fuse, prev);
+    if (chunk == 0) {
       launch_passes(cur, from, end, 0, 0);
       exchange_data(X.l, X.g);
       cur = std::move(next);
       std::fill(from.begin(), from.end(), 0);
+      prev = 0;
       continue;
     }
-    // tail: trailing passes that do not mix the chunk bits (controls and diagonal
-    // entries on them are fine: resolved per block); head: leading ones of the next run
-    auto blockwise = [&](const FusedPass& ps) {
-      return !(ps.nd_mask & H) && (!ps.prog || ps.K <= n_local - c);
-    };
+    // tail: trailing passes that do not mix the chunk qubits; head: leading ones of the
+    // next run
     std::vector<size_t> ts(S), he(S, 0), zero(S, 0);
+    bool chained = prev == chunk, whole = true;
     for (int s = 0; s < S; ++s) {
       ts[s] = end[s];
-      while (ts[s] > from[s] && blockwise(cur[s].passes[ts[s] - 1])) --ts[s];
-      while (he[s] < next[s].passes.size() && blockwise(next[s].passes[he[s]])) ++he[s];
+      while (ts[s] > from[s] && pass_blockwise(cur[s].passes[ts[s] - 1], chunk, n_local)) --ts[s];
+      while (he[s] < next[s].passes.size() && pass_blockwise(next[s].passes[he[s]], chunk, n_local))
+        ++he[s];
+      chained &= from[s] == end[s];
+      whole &= he[s] == next[s].passes.size();
     }
-    launch_passes(cur, from, ts, 0, 0);  // the body of the run
-    const int parts = 1 << c;
-    for (int v = 0; v < parts; ++v) {
-      launch_passes(cur, ts, end, c, v);
-      LFQS_CUDA_CHECK(cudaEventRecord(part_event(ev_tail, v), stream));
+    const int parts = 1 << __builtin_popcountll(chunk);
+    if (!chained) {
+      // (chained: the whole run between the previous exchange and this one already ran
+      // part by part, each part's ev_tail recorded after it)
+      launch_passes(cur, from, ts, 0, 0);  // the body of the run
+      for (int v = 0; v < parts; ++v) {
+        launch_passes(cur, ts, end, chunk, (uint64_t)v);
+        LFQS_CUDA_CHECK(cudaEventRecord(part_event(ev_tail, v), stream));
+      }
     }
     for (int v = 0; v < parts; ++v) {
-      cudaEvent_t done = exchange_part(X.l, X.g, c, v, part_event(ev_tail, v));
+      cudaEvent_t done = exchange_part(X.l, X.g, chunk, (uint64_t)v, part_event(ev_tail, v));
       if (done) LFQS_CUDA_CHECK(cudaStreamWaitEvent(stream, done, 0));
-      launch_passes(next, zero, he, c, v);
+      launch_passes(next, zero, he, chunk, (uint64_t)v);
+      if (whole) LFQS_CUDA_CHECK(cudaEventRecord(part_event(ev_tail, v), stream));
     }
     ++exchanges;
     exchange_bytes += (uint64_t)ab << (n_local - 1);
+    ++ov_exchanges;
+    for (int s = 0; s < S; ++s) ov_block_passes += (end[s] - ts[s]) + he[s];
+    const int c = __builtin_popcountll(chunk);
+    ov_strided += chunk != ((1ull << c) - 1) << (n_local - c);
+    ov_chained += chained;
+    prev = whole ? chunk : 0;
     cur = std::move(next);
     from = he;
   }

@@ -45,6 +45,7 @@ struct State : lfqs_state {
   P2P* p2p = nullptr;           // CUDA-IPC peer transport (instead of comm)
   // exchange statistics (benchmark accounting)
   uint64_t exchanges = 0, exchange_bytes = 0;
+  uint64_t ov_exchanges = 0, ov_block_passes = 0, ov_strided = 0, ov_chained = 0;
 
   static State* create_local(int n, int device, cudaStream_t stream, void* borrowed,
                              bool c64 = false, bool soa = false);
@@ -103,14 +104,18 @@ struct State : lfqs_state {
     std::vector<FusedPass> passes;
   };
   std::vector<ShardRun> plan_run(const std::vector<PlanOp>& ops, size_t b, size_t e, bool fuse);
-  // Launches passes [from[s], to[s]) of every shard, on the whole shard (c = 0) or on part
-  // v of 2^c (the block whose top c local bits equal v; the passes do not touch them).
+  // Launches passes [from[s], to[s]) of every shard, on the whole shard (chunk = 0) or on
+  // block v of the chunk qubits (the passes do not mix them: pass_blockwise).
   void launch_passes(const std::vector<ShardRun>& run, const std::vector<size_t>& from,
-                     const std::vector<size_t>& to, int c, int v);
-  // One part of an exchange; the data it moves is final once `ready` has fired.  Returns
-  // the event the compute stream must wait for before using the part (NULL: the copies
+                     const std::vector<size_t>& to, uint64_t chunk, uint64_t v);
+  // Chunk qubits of the overlapped exchange ops[ex[k]] (0: serial); prev: the previous
+  // exchange's, when its run may continue block by block.
+  uint64_t choose_chunk(const std::vector<PlanOp>& ops, const std::vector<size_t>& ex, size_t k,
+                        bool fuse, uint64_t prev) const;
+  // One block of an exchange; the data it moves is final once `ready` has fired.  Returns
+  // the event the compute stream must wait for before using the block (NULL: the copies
   // already sit on the compute stream, NCCL transport).
-  cudaEvent_t exchange_part(int l, int g, int c, int v, cudaEvent_t ready);
+  cudaEvent_t exchange_part(int l, int g, uint64_t chunk, uint64_t v, cudaEvent_t ready);
   int n_shards() const { return virt ? world : 1; }
   int rank_of_shard(int shard) const { return virt ? shard : rank; }
   void execute(const std::vector<PlanOp>& ops, bool fuse);

@@ -57,6 +57,28 @@ def worker(rank, world, port, n, seed, out_q):
                 outs.append(st.copy_out()[lo:hi])
         report["overlap"] = (all(np.array_equal(outs[0], o) for o in outs[1:]),
                              float(np.max(np.abs(outs[1] - ref[lo:hi]))))
+        # fused (compiled) passes with the chunk qubits chosen per exchange (strided blocks
+        # below the top qubits: fixed tile-index bits, swap kernels with fixed bits; the
+        # choice is made from the plan, so every rank picks the same blocks) vs top-qubit
+        # blocks vs serial exchanges: the same passes, so the same bits
+        nf = 16
+        lf, hf = rank << (nf - (world.bit_length() - 1)), (rank + 1) << (nf - (world.bit_length() - 1))
+        psif = W.random_state(nf, seed + 3)
+        gf = W.qft(nf) + W.random_layered(nf, 3, seed=seed) + W.random_gate_list(nf, 80, seed=seed)
+        reff = O.run_circuit(nf, gf, psif.copy())
+        outs, strided = [], 0
+        for bits, sel, ctas in ((0, 1, 0), (2, 0, 0), (2, 1, 0), (2, 1, 8)):
+            with L.State.p2p(nf, rank, world) as st:
+                st.set_option(L.OPT_FUSE_TILE_QUBITS, 8)
+                st.set_option(L.OPT_EXCHANGE_CHUNK_BITS, bits)
+                st.set_option(L.OPT_EXCHANGE_CHUNK_SELECT, sel)
+                st.set_option(L.OPT_EXCHANGE_CTAS, ctas)
+                st.copy_in(psif)
+                st.run_circuit(gf, fuse="jit")
+                outs.append(st.copy_out()[lf:hf])
+                strided += st.overlap_stats()["strided"] if sel else 0
+        report["overlap_fused"] = (all(np.array_equal(outs[0], o) for o in outs[1:]),
+                                   float(np.max(np.abs(outs[0] - reff[lf:hf]))), strided)
         # one gate at a time through lfqs_apply_gate (planner per gate, exchanges included)
         with L.State.p2p(n, rank, world) as st:
             st.copy_in(psi)

@@ -82,6 +82,66 @@ def test_overlap_fused_vs_oracle(L, world, fuse):
             assert np.array_equal(out, ref_exact), bits
 
 
+@pytest.mark.parametrize("fuse", [True, "jit", "jit+phase"])
+@pytest.mark.parametrize("world,n,tile", [(4, 20, 12), (2, 16, 8), (8, 17, 8)])
+def test_chunk_select_bit_identical(L, world, n, tile, fuse):
+    """LFQS_OPT_EXCHANGE_CHUNK_SELECT: each exchange's chunk qubits are chosen among the
+    local qubits at or above the tile size (fixed bits of the fused passes' tile index,
+    strided blocks for the swap kernels), and consecutive exchanges sharing them are
+    chained block by block.  The passes are the serial run's: bit-identical to serial
+    exchanges and to the top-qubit blocks, within 1e-12 of the oracle; strided and
+    chained exchanges do occur."""
+    psi = W.random_state(n, 5 + world)
+    gates = (W.qft(n) + W.random_layered(n, 3, seed=world) +
+             W.random_gate_list(n, 120, seed=world, max_controls=2) + W.ghz(n))
+    ref = O.run_circuit(n, gates, psi.copy())
+    outs, stats = {}, {}
+    for bits, sel, ctas, rate in ((0, 1, 0, 0), (2, 0, 0, 0), (2, 1, 0, 0), (3, 1, 8, 0),
+                                  (1, 1, 0, 0), (2, 1, 0, 200)):
+        with L.State.virtual(n, world) as st:
+            st.set_option(L.OPT_FUSE_TILE_QUBITS, tile)
+            st.set_option(L.OPT_EXCHANGE_CHUNK_BITS, bits)
+            st.set_option(L.OPT_EXCHANGE_CHUNK_SELECT, sel)
+            st.set_option(L.OPT_EXCHANGE_CTAS, ctas)
+            st.set_option(L.OPT_EXCHANGE_RATE_GBS, rate)
+            st.copy_in(psi)
+            st.run_circuit(gates, fuse=fuse)
+            outs[bits, sel, rate] = st.copy_out()
+            stats[bits, sel, rate] = st.overlap_stats()
+    serial = outs[0, 1, 0]
+    assert np.max(np.abs(serial - ref)) <= 1e-12
+    for k, o in outs.items():
+        assert np.array_equal(o, serial), (k, stats[k])
+    assert stats[0, 1, 0]["overlapped"] == 0
+    st2 = stats[2, 1, 0]
+    assert st2["overlapped"] > 0 and st2["block_passes"] > 0 and st2["strided"] > 0, st2
+    assert stats[2, 0, 0]["strided"] == 0
+
+
+def test_chunk_select_chains_exchanges(L):
+    """Consecutive exchanges whose run between them leaves the chunk qubits unmixed run as
+    a pipeline (part v of the second exchange starts when part v of the run is done): QFT
+    on 8 shards takes the Hadamards of its three global qubits one after another, with only
+    the swapped-in qubit mixed (and phase tables) between the exchanges."""
+    n, world = 18, 8
+    psi = W.random_state(n, 4)
+    gates = W.qft(n) + W.random_gate_list(n, 100, seed=11, max_controls=1)
+    ref = O.run_circuit(n, gates, psi.copy())
+    with L.State.virtual(n, world) as st:
+        st.set_option(L.OPT_FUSE_TILE_QUBITS, 8)
+        st.copy_in(psi)
+        st.run_circuit(gates, fuse="jit+phase")
+        got = st.copy_out()
+        stats = st.overlap_stats()
+        st.set_option(L.OPT_EXCHANGE_CHUNK_BITS, 0)
+        st.copy_in(psi)
+        st.run_circuit(gates, fuse="jit+phase")
+        serial = st.copy_out()
+    assert np.max(np.abs(got - ref)) <= 1e-12
+    assert np.array_equal(got, serial)
+    assert stats["overlapped"] > 0 and stats["chained"] > 0, stats
+
+
 def test_overlap_graph_capture_and_per_gate_apply(L):
     """The exchange stream forks from and joins the capturing stream (lfqs_circuit_compile
     on a virtual partition), and per-gate lfqs_apply_gate overlaps its own exchange."""
@@ -126,12 +186,12 @@ def test_pass_count(L):
 
 def test_exchange_options_validated(L):
     with L.State.virtual(10, 2) as st:
-        for opt, bad in ((L.OPT_EXCHANGE_CHUNK_BITS, 5), (L.OPT_EXCHANGE_CHUNK_BITS, -1),
+        for opt, bad in ((L.OPT_EXCHANGE_CHUNK_BITS, 4), (L.OPT_EXCHANGE_CHUNK_BITS, -1),
                          (L.OPT_EXCHANGE_CTAS, -1), (L.OPT_EXCHANGE_CTAS, 1 << 20)):
             with pytest.raises(L.LfqsError) as e:
                 st.set_option(opt, bad)
             assert e.value.status == -1
-        st.set_option(L.OPT_EXCHANGE_CHUNK_BITS, 4)  # n_local = 9: 9 - 4 >= 4, still valid
+        st.set_option(L.OPT_EXCHANGE_CHUNK_BITS, 3)  # n_local = 9: 9 - 3 >= 4, still valid
         st.set_option(L.OPT_EXCHANGE_CTAS, 1)
         psi = W.random_state(10, 3)
         st.copy_in(psi)

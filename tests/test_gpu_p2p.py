@@ -53,5 +53,7 @@ def test_p2p_sharded_circuits(world):
         assert payload["apply"] <= 1e-12
         same, err = payload["overlap"]
         assert same and err <= 1e-12, (rank, same, err)
+        same, err, strided = payload["overlap_fused"]
+        assert same and err <= 1e-12 and (strided > 0 or world > 2), (rank, same, err, strided)
         same, err = payload["streamed"]
         assert same and err <= 1e-12, (rank, same, err)

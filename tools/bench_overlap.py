@@ -31,6 +31,9 @@ def main():
     ap.add_argument("--mode", default="jit+phase")
     ap.add_argument("--ctas", default="0,32,16,8")
     ap.add_argument("--bits", default="0,1,2,3")
+    ap.add_argument("--select", default="1", help="LFQS_OPT_EXCHANGE_CHUNK_SELECT values")
+    ap.add_argument("--tile", type=int, default=12)
+    ap.add_argument("--rate", default="0", help="LFQS_OPT_EXCHANGE_RATE_GBS values (0: unpaced)")
     ap.add_argument("--reps", type=int, default=3)
     args = ap.parse_args()
     import torch
@@ -67,28 +70,39 @@ def main():
                       "ms": round(t1, 3)}), flush=True)
     with L.State.virtual(n, args.world, 0, stream=s) as st:
         if flags & L.FUSE_JIT:  # compile every pass shape outside the timed region
+            st.set_option(L.OPT_FUSE_TILE_QUBITS, args.tile)
             for b in [int(v) for v in args.bits.split(",")]:
                 st.set_option(L.OPT_EXCHANGE_CHUNK_BITS, b)
                 st.init_basis(0)
                 L.lfqs_run_circuit(st.h, arr, flags)
             torch.cuda.synchronize()
-        for ctas in [int(v) for v in args.ctas.split(",")]:
+        st.set_option(L.OPT_FUSE_TILE_QUBITS, args.tile)
+        for ctas, rate in [(int(v), int(r)) for v in args.ctas.split(",")
+                           for r in args.rate.split(",")]:
             st.set_option(L.OPT_EXCHANGE_CTAS, ctas)
+            st.set_option(L.OPT_EXCHANGE_RATE_GBS, rate)
             serial = None
             for b in [int(v) for v in args.bits.split(",")]:
-                st.set_option(L.OPT_EXCHANGE_CHUNK_BITS, b)
-                x0 = st.exchange_stats()[0]
-                t = timed(st)
-                nx = (st.exchange_stats()[0] - x0) // (args.reps + 1)
-                rec = {"circuit": args.circuit, "mode": args.mode, "n": n, "world": args.world,
-                       "exchange_ctas": ctas, "chunk_bits": b, "ms": round(t, 3),
-                       "exchanges": int(nx), "unsharded_ms": round(t1, 3),
-                       "exposed_exchange_ms": round(t - t1, 3)}
-                if b == 0:
-                    serial = t
-                elif serial is not None and serial > t1:
-                    rec["hidden_frac"] = round((serial - t) / (serial - t1), 3)
-                print(json.dumps(rec), flush=True)
+                for sel in ([1] if b == 0 else [int(v) for v in args.select.split(",")]):
+                    st.set_option(L.OPT_EXCHANGE_CHUNK_BITS, b)
+                    st.set_option(L.OPT_EXCHANGE_CHUNK_SELECT, sel)
+                    x0 = st.exchange_stats()[0]
+                    o0 = st.overlap_stats()
+                    t = timed(st)
+                    nx = (st.exchange_stats()[0] - x0) // (args.reps + 1)
+                    o1 = st.overlap_stats()
+                    ov = {k: (o1[k] - o0[k]) // (args.reps + 1) for k in o1}
+                    rec = {"circuit": args.circuit, "mode": args.mode, "n": n,
+                           "world": args.world, "exchange_ctas": ctas, "rate_gbs": rate,
+                           "chunk_bits": b,
+                           "chunk_select": sel, "ms": round(t, 3), "exchanges": int(nx),
+                           "overlap": ov, "unsharded_ms": round(t1, 3),
+                           "exposed_exchange_ms": round(t - t1, 3)}
+                    if b == 0:
+                        serial = t
+                    elif serial is not None and serial > t1:
+                        rec["hidden_frac"] = round((serial - t) / (serial - t1), 3)
+                    print(json.dumps(rec), flush=True)
 
 
 if __name__ == "__main__":
