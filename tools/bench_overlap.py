@@ -1,15 +1,23 @@
 """Exchange/compute overlap on one GPU: a virtual partition into `world` shards
 runs a circuit with serial exchanges (LFQS_OPT_EXCHANGE_CHUNK_BITS = 0) and overlapped
-ones (2^c parts on an exchange stream while the neighbouring local passes run part by part),
-with the exchange swap kernel's grid limited to `ctas` CTAs -- a small grid moves the
-exchange at a link-like rate (NVLink 5: ~0.9 TB/s per direction, an eighth of HBM) and
-leaves the SMs to the local passes, which is what an exchange over NVLink looks like to
-the GPU.  The same circuit on an unsharded state (world = 1) gives the local work alone.
+ones (2^c blocks on a high-priority exchange stream while the neighbouring local passes run
+block by block; LFQS_OPT_EXCHANGE_CHUNK_SELECT picks the chunk qubits per exchange).  The
+exchange swap kernel is grid-limited (`--ctas`) and optionally paced (`--rate`, GB/s per
+direction per shard pair): what an exchange over NVLink looks like to the GPU -- a
+link-bound transfer that leaves most SMs and most of the HBM bandwidth to the passes.
 
-    python tools/bench_overlap.py --n 32 --world 4 --circuit qft --ctas 0,16,8
+Pacing ratio: on P real GPUs every rank runs its own shard's passes (time C) and all shard
+pairs exchange at once at the link rate R; the virtual partition runs the P shards' passes
+back to back (P * C) and its P/2 pair exchanges one after another, so the virtual swap at
+R/2 per pair keeps exchange time : pass time equal to the real one (R = 900 GB/s NVLink 5
+-> --rate 450).  The same circuit on an unsharded state (world = 1) gives the local work
+alone.
 
-Prints one JSON object per (ctas, chunk bits): ms, exchanges, exposed exchange time
-(ms - unsharded ms) and the fraction of the serial exchange time hidden by overlapping.
+    python tools/bench_overlap.py --n 32 --world 4 --circuit qft --ctas 64 --rate 450
+
+Prints one JSON object per (ctas, rate, chunk bits, select): ms, exchanges, the overlap
+accounting (lfqs_state_overlap_stats), the exposed exchange time (ms - unsharded ms) and
+the fraction of the serial exchange time hidden by overlapping.
 """
 import argparse
 import json
@@ -29,11 +37,11 @@ def main():
     ap.add_argument("--world", type=int, default=4)
     ap.add_argument("--circuit", default="qft")
     ap.add_argument("--mode", default="jit+phase")
-    ap.add_argument("--ctas", default="0,32,16,8")
-    ap.add_argument("--bits", default="0,1,2,3")
-    ap.add_argument("--select", default="1", help="LFQS_OPT_EXCHANGE_CHUNK_SELECT values")
+    ap.add_argument("--ctas", default="64")
+    ap.add_argument("--bits", default="0,2,3")
+    ap.add_argument("--select", default="0,1", help="LFQS_OPT_EXCHANGE_CHUNK_SELECT values")
     ap.add_argument("--tile", type=int, default=12)
-    ap.add_argument("--rate", default="0", help="LFQS_OPT_EXCHANGE_RATE_GBS values (0: unpaced)")
+    ap.add_argument("--rate", default="450", help="LFQS_OPT_EXCHANGE_RATE_GBS values (0: unpaced)")
     ap.add_argument("--reps", type=int, default=3)
     args = ap.parse_args()
     import torch

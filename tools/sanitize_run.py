@@ -66,6 +66,18 @@ def main():
         st.run_circuit(gates[:80])
         st.copy_out(0, 16)
         st.measure_probs(list(range(n)))
+    # chunk qubits chosen per exchange (strided blocks: fixed tile-index bits, swap kernels
+    # with fixed bits), chained exchanges, the paced swap kernel
+    with L.State.virtual(16, 4) as st:
+        st.init_random(5)
+        st.set_option(L.OPT_FUSE_TILE_QUBITS, 8)
+        g16 = W.qft(16) + W.random_layered(16, 3, seed=4)
+        st.run_circuit(g16, fuse="jit+phase")
+        st.set_option(L.OPT_EXCHANGE_RATE_GBS, 200)
+        st.set_option(L.OPT_EXCHANGE_CHUNK_BITS, 3)
+        st.run_circuit(g16, fuse=True)
+        assert st.overlap_stats()["strided"] > 0
+        st.measure_probs([0, 15])
     print("sanitize workload done")
 
 
