@@ -464,6 +464,11 @@ lfqs_status lfqs_state_pass_count(const lfqs_state* s, uint64_t* passes);
                                   one-GPU virtual partition shows how much of an NVLink
                                   exchange the overlapped local passes hide; default 0
                                   (unpaced).  Same results */
+#define LFQS_OPT_FUSE_H_SCALE 25 /* 1 (default): in a fused pass with k >= 2 unpredicated
+                                  Hadamards, one carries the whole scale (1/sqrt 2)^k and the
+                                  others compute the unscaled butterfly (a + b, a - b): 2 FP64
+                                  multiplies per amplitude fewer per Hadamard.  Rounding
+                                  changes only (dense tolerance class) */
 lfqs_status lfqs_set_option(lfqs_state* s, int option, int64_t value);
 const char* lfqs_last_error(void);
 int lfqs_abi_version(void);

@@ -30,6 +30,7 @@
 // complex64, NEXT-4); the program's coefficients are stored in double.
 #include <cuda_runtime.h>
 
+#include <cmath>
 #include <cstring>
 #include <map>
 #include <memory>
@@ -851,6 +852,31 @@ bool tile_dependent(const FHdr& h) {
 // control lies outside the tile) adds no table bits, but every table entry evaluates it;
 // grouped apart, such members usually share their in-tile bits as a common predicate and
 // form a table of very few entries, so the per-tile build does ~1/256 of the work.
+// Hadamard scales folded (LFQS_OPT_FUSE_H_SCALE, default 1).  Every amplitude of a tile
+// passes through each unpredicated Hadamard exactly once, so the k factors 1/sqrt(2) of a
+// pass's k >= 2 unpredicated F_H ops are one uniform scalar (1/sqrt(2))^k: the last of them
+// carries it (2^(-k/2) exactly for even k) and the others compute the unscaled butterfly
+// (a + b, a - b) -- coefficient 1, an exact product the pass compiler drops.  Linear ops
+// commute with a scalar, so the pass computes the same state up to rounding (dense
+// tolerance class; H is dense): 2 FP64 multiplies per amplitude per folded Hadamard fewer
+// (QFT / Grover / QPE passes).  Interpreter and pass compiler run the same program.
+void fold_h_scales(FProg& P) {
+  int k = 0, last = -1;
+  for (int o = 0; o < P.nops; ++o) {
+    const FHdr& h = P.h[o];
+    if (h.type == F_H && h.mlo == 0 && h.mhi == 0) {
+      ++k;
+      last = o;
+    }
+  }
+  if (k < 2) return;
+  const double s = (k & 1) ? std::ldexp(M_SQRT1_2, -(k - 1) / 2) : std::ldexp(1.0, -k / 2);
+  for (int o = 0; o < P.nops; ++o) {
+    const FHdr& h = P.h[o];
+    if (h.type == F_H && h.mlo == 0 && h.mhi == 0) P.c[h.coef] = double2{o == last ? s : 1.0, 0.0};
+  }
+}
+
 void merge_phase_runs(FProg& P, bool split) {
   static thread_local FHdr out[kMaxOps];
   static thread_local FHdr run[kMaxOps];
@@ -1143,6 +1169,7 @@ void build_program(const LaunchCtx& ctx, const TileCfg& cfg, uint64_t in_tile,
     prog.push_back(g);
   }
   for (const Decoded& g : prog) encode(g, tm, P);
+  if (ctx.opt->fuse_h_scale) fold_h_scales(P);
   if (ctx.phase_tables) merge_phase_runs(P, ctx.opt->fuse_phase_split);
 }
 

@@ -454,6 +454,7 @@ struct Gen {
   struct Op2 {
     int type;
     std::string s;                  // F_H
+    bool s1 = false;                // F_H coefficient exactly 1: the unscaled butterfly
     std::string m00, m01, m10, m11; // F_UR
     std::string d0, e01, e10, d1;   // F_UI
     Cx c0, c1, c2, c3, n0, n1, n2, n3;  // F_U2 (n*.x = -c*.y)
@@ -463,7 +464,12 @@ struct Gen {
     o.type = h.type;
     const int c = h.coef;
     switch (h.type) {
-      case F_H: o.s = coef_re(c); break;
+      case F_H: {
+        const Cx k = coef(c);
+        o.s = k.x;
+        o.s1 = k.vx == 1.0;
+        break;
+      }
       case F_UR:
         o.m00 = coef_re(c); o.m01 = coef_re(c + 1); o.m10 = coef_re(c + 2); o.m11 = coef_re(c + 3);
         break;
@@ -479,6 +485,8 @@ struct Gen {
     }
     return o;
   }
+  // s * v of F_H; with s == 1 (fold_h_scales) the exact product is dropped
+  std::string hs(const Op2& o, const std::string& v) { return o.s1 ? v : mul(o.s, v); }
   void pair(const Op2& o, Cx& a0, Cx& a1) {
     const Cx x0 = a0, x1 = a1;
     switch (o.type) {
@@ -488,8 +496,8 @@ struct Gen {
         a1 = {neg(x0.y), x0.x};
         return;
       case F_H:
-        a0 = {mul(o.s, add(x0.x, x1.x)), mul(o.s, add(x0.y, x1.y))};
-        a1 = {mul(o.s, sub(x0.x, x1.x)), mul(o.s, sub(x0.y, x1.y))};
+        a0 = {hs(o, add(x0.x, x1.x)), hs(o, add(x0.y, x1.y))};
+        a1 = {hs(o, sub(x0.x, x1.x)), hs(o, sub(x0.y, x1.y))};
         return;
       case F_UR:
         a0 = {fma(o.m01, x1.x, mul(o.m00, x0.x)), fma(o.m01, x1.y, mul(o.m00, x0.y))};
@@ -554,7 +562,7 @@ struct Gen {
       case F_H: {
         // s (p + (bit ? -a : a))
         const std::string ax = sel(neg(a.x), a.x, bit), ay = sel(neg(a.y), a.y, bit);
-        return {mul(o.s, add(pp.x, ax)), mul(o.s, add(pp.y, ay))};
+        return {hs(o, add(pp.x, ax)), hs(o, add(pp.y, ay))};
       }
       case F_UR:
         return {fma(l.B, pp.x, mul(l.A, a.x)), fma(l.B, pp.y, mul(l.A, a.y))};
@@ -577,7 +585,7 @@ struct Gen {
       case F_Y: return bit ? Cx{neg(pp.y), pp.x} : Cx{pp.y, neg(pp.x)};
       case F_H: {
         const std::string ax = bit ? neg(a.x) : a.x, ay = bit ? neg(a.y) : a.y;
-        return {mul(o.s, add(pp.x, ax)), mul(o.s, add(pp.y, ay))};
+        return {hs(o, add(pp.x, ax)), hs(o, add(pp.y, ay))};
       }
       case F_UR: {
         const std::string& A = bit ? o.m11 : o.m00;
@@ -1984,7 +1992,8 @@ double pass_fp64_per_amp(const FProg& P, double* table_work) {
         break;
       case F_DIAG1: ops += 4.0 * frac; break;
       case F_DIAGN: ops += 4.0 * frac; break;
-      case F_H: case F_UR: case F_UI: ops += 4.0 * frac; break;
+      case F_H: ops += (c[0].x == 1.0 ? 2.0 : 4.0) * frac; break;
+      case F_UR: case F_UI: ops += 4.0 * frac; break;
       case F_U2: ops += 8.0 * frac; break;
       case F_U4: ops += parts(16) / 4.0 * frac; break;
       case F_U8: ops += parts(64) / 8.0 * frac; break;

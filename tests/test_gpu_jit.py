@@ -215,3 +215,32 @@ def test_jit_precompile_then_run(L):
     got, passes = _run(L, n, psi, gates, "jit")
     assert passes == k
     assert np.max(np.abs(got - O.run_circuit(n, gates, psi.copy()))) <= 1e-12
+
+
+@pytest.mark.parametrize("c64", [False, True])
+@pytest.mark.parametrize("fuse", ["jit", "jit+phase"])
+def test_h_scale_folding(L, fuse, c64):
+    """LFQS_OPT_FUSE_H_SCALE: a pass's unpredicated Hadamards compute unscaled butterflies
+    and one of them carries (1/sqrt 2)^k.  Compiled == interpreted bit for bit with the
+    folding on and off; within the dense tolerance of the oracle and of the unfolded pass
+    (QFT, Grover and an H layer: passes with many Hadamards, controlled H left alone)."""
+    n = 14
+    psi = W.random_state(n, 21)
+    gates = (W.qft(n) + W.grover(n, 1234, 1) + [W.Gate("H", (q,)) for q in range(n)] +
+             [W.Gate("H", (3,), (9,)), W.Gate("H", (10,), (2, 5))] +
+             W.random_gate_list(n, 80, seed=5, max_controls=2))
+    ref = O.run_circuit(n, gates, psi.copy())
+    tol = 1e-5 if c64 else 1e-12
+    interp = True if fuse == "jit" else "phase"  # the interpreter of the same passes
+    outs = {}
+    for hs in (0, 1):
+        for f in (interp, fuse):
+            with L.State.create(n, c64=c64) as st:
+                st.set_option(L.OPT_FUSE_H_SCALE, hs)
+                st.copy_in(psi)
+                st.run_circuit(gates, fuse=f)
+                outs[hs, f] = st.copy_out()
+            assert np.max(np.abs(outs[hs, f] - ref)) <= tol, (hs, f)
+    for hs in (0, 1):  # interpreter == pass compiler
+        assert np.array_equal(outs[hs, interp], outs[hs, fuse]), hs
+    assert not np.array_equal(outs[0, fuse], outs[1, fuse])  # the folding did change the passes
