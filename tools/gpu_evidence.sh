@@ -28,6 +28,10 @@ timeout 2400 python tools/bench_circuits.py --n 30 --modes jit+phase,unfused --o
 timeout 2400 python tools/bench_circuits.py --n 33 --reps 1 --circuits qft,ghz,qpe,grover,random,sycamore --modes jit+phase > $O/${TAG}_circuits_n33.jsonl 2>&1
 timeout 900 python tools/bench_circuits.py --n 31 --c64 --circuits qft,ghz,random --modes jit+phase > $O/${TAG}_circuits_c64_n31.jsonl 2>&1
 timeout 600 python tools/bench_small.py > $O/${TAG}_small.jsonl 2>&1
+timeout 600 python -m torch.distributed.run --nnodes=1 --nproc-per-node 2 --master-addr 127.0.0.1 \
+  --master-port 29517 bench.py --gpus 2 --same-device --qubits-per-gpu 28 --steps 2 --warmup 3 \
+  > $O/${TAG}_bench_n2_same_device.json 2> $O/${TAG}_bench_n2.err
+timeout 900 python tools/bench_overlap.py --n 32 --world 4 --circuit qft --bits 0,2 > $O/${TAG}_overlap_qft32_w4.jsonl 2>&1
 for tool in memcheck racecheck synccheck; do
   timeout 900 compute-sanitizer --tool $tool --print-limit 20 python tools/sanitize_run.py > $O/${TAG}_sanitize_$tool.txt 2>&1
 done
