@@ -373,6 +373,11 @@ __device__ __forceinline__ cx<S> diag_factor(const FHdr& g, const double2* pc, u
   return cvs<S>(c[j]);
 }
 
+// A phase-table member that holds for every entry of its table (jit.cpp hoisted_member).
+__device__ __forceinline__ bool dtab_hoisted(const FHdr& g, uint32_t cm) {
+  return g.type == F_DIAG1 && g.mlo == cm;
+}
+
 // Global amplitude index of tile element i (chunk = i >> lc, offset = low lc bits).
 __device__ __forceinline__ uint64_t tile_addr(const FTile& tg, uint64_t base, uint32_t i) {
   uint64_t off = base | (i & ((1u << tg.lc) - 1));
@@ -480,11 +485,23 @@ __global__ void __launch_bounds__(kFThreads, sizeof(S) == 4 ? 4 : 2) k_fused(cx<
           u &= u - 1;
           ie |= ((tid >> b) & 1u) << pos;
         }
-        C t = mk<S>(1, 0);
+        // Members that hold for every entry (one-entry diagonals whose tile-bit predicate
+        // is the common one: decided by the tile index alone) are a per-tile factor C; with
+        // >= 2 of them the entry is C * (the other members' product), each product in
+        // program order -- the pass compiler computes C once per tile (jit.cpp
+        // dtab_factor), the same values.
+        int nh = 0;
+        for (int j = 1; j <= nm; ++j) nh += dtab_hoisted(prog.h[o + j], cm);
+        C t = mk<S>(1, 0), cf = mk<S>(1, 0);
         for (int j = 1; j <= nm; ++j) {
           const C d = diag_factor<S>(prog.h[o + j], prog.c, base, ie);
-          if (!is_one(d)) t = cmul_fma(d, t);
+          if (is_one(d)) continue;
+          if (nh >= 2 && dtab_hoisted(prog.h[o + j], cm))
+            cf = cmul_fma(d, cf);
+          else
+            t = cmul_fma(d, t);
         }
+        if (nh >= 2) t = cmul_fma(cf, t);
         dtab[tid] = t;
       }
       if (!in_regs) {

@@ -1025,6 +1025,7 @@ struct Gen {
   int prebuild_entries() const { return c64 ? 1024 : 2048; }
   std::map<int, int> dtab_off;  // prebuilt F_DTAB op -> entry offset in lfqs_dtab
   int dtab_pre = 0;             // entries of the prebuilt tables
+  int n_dtabc = 0;              // prebuilt tables with hoisted members (lfqs_dtabc slots)
   bool dtab_dyn = false;        // some table is built in place (after the prebuilt ones)
   void plan_prebuild() {
     for (int o = 0; o < P.nops; ++o) {
@@ -1042,12 +1043,59 @@ struct Gen {
   }
   int dtab_entries() const { return std::max(dtab_pre + (dtab_dyn ? 256 : 0), 1); }
 
+  // Members of table `o` that hold for every entry (one-entry diagonals whose tile-bit
+  // predicate is the table's common predicate; only tile bits outside the table, i.e. the
+  // tile index, decide them): a per-tile factor.  With >= 2 of them the table is
+  // C * partial[e] -- C their product (program order), partial[e] the other members'
+  // (program order) -- exactly as k_fused builds it (fused_kernels.cu dtab_hoisted).
+  static bool hoisted_member(const FHdr& g, uint32_t cm) { return g.type == F_DIAG1 && g.mlo == cm; }
+  int n_hoisted(int o) const {
+    const FHdr& h = P.h[o];
+    const uint32_t cm = h.plo & 0xffffu;
+    int k = 0;
+    for (int j = 1; j <= h.m; ++j) k += hoisted_member(P.h[o + j], cm);
+    return k;
+  }
+  // C of table o into `c` (registers): the hoisted members' product.
+  void dtab_factor(int o, Cx& c) {
+    const FHdr& h = P.h[o];
+    const uint32_t cm = h.plo & 0xffffu;
+    e("mov.%s %s, %s;", FT, c.x.c_str(), c64 ? "0f3F800000" : "0d3FF0000000000000");
+    e("mov.%s %s, %s;", FT, c.y.c_str(), zero().c_str());
+    for (int j = 1; j <= h.m; ++j) {
+      const FHdr& g = P.h[o + j];
+      if (!hoisted_member(g, cm)) continue;
+      const std::string skip = L();
+      tile_pred(g.mhi, g.phi, skip);
+      const Cx d = coef(g.coef);
+      if (!(d.vx == 1.0 && d.vy == 0.0)) assign(c.x, c.y, cmulf(d, c));
+      label(skip);
+    }
+  }
+
   // Builds table `o` into lfqs_dtab entries [off, off + 2^nb): entry e by thread e mod NT.
-  void dtab_build(int o, int off) {
+  // hslot >= 0 (a prebuilt table with hoisted members): the entries are the partial
+  // products and thread 32 + hslot writes C to lfqs_dtabc[hslot] (dtab_finalize multiplies
+  // them after the next barrier); otherwise every thread applies C itself.
+  void dtab_build(int o, int off, int hslot = -1) {
     const FHdr& h = P.h[o];
     const int nm = h.m;
-    const uint32_t U = h.mlo, cp = h.plo >> 16;
+    const uint32_t U = h.mlo, cm = h.plo & 0xffffu, cp = h.plo >> 16;
     const int nb = __builtin_popcount(U);
+    const bool hoist = n_hoisted(o) >= 2;
+    Cx c{f(), f()};
+    if (hoist && hslot >= 0) {
+      const std::string skip = L(), q = p();
+      e("setp.ne.u32 %s, %%ltid, %d;", q.c_str(), 32 + hslot);
+      e("@%s bra %s;", q.c_str(), skip.c_str());
+      dtab_factor(o, c);
+      const std::string a = r();
+      e("mov.u32 %s, lfqs_dtabc;", a.c_str());
+      sts(a, c, hslot * ES);
+      label(skip);
+    } else if (hoist) {
+      dtab_factor(o, c);
+    }
     for (int k = 0; k * NT < (1 << nb); ++k) {
       const std::string skip = L(), q = p(), eid = r();
       e("add.u32 %s, %%ltid, %d;", eid.c_str(), k * NT);
@@ -1066,10 +1114,32 @@ struct Gen {
       Cx t{f(), f()};
       e("mov.%s %s, %s;", FT, t.x.c_str(), c64 ? "0f3F800000" : "0d3FF0000000000000");
       e("mov.%s %s, %s;", FT, t.y.c_str(), zero().c_str());
-      for (int j = 1; j <= nm; ++j) dtab_member(P.h[o + j], ie, t);
+      for (int j = 1; j <= nm; ++j)
+        if (!hoist || !hoisted_member(P.h[o + j], cm)) dtab_member(P.h[o + j], ie, t);
+      if (hoist && hslot < 0) assign(t.x, t.y, cmulf(c, t));
       const std::string a = r();
       e("mad.lo.u32 %s, %s, %d, %%dtab;", a.c_str(), eid.c_str(), ES);
       sts(a, t, off * ES);
+      label(skip);
+    }
+  }
+  // After the barrier that follows the prologue builds: entries of the prebuilt tables
+  // with hoisted members times their C (each thread its own entries).
+  void dtab_finalize(int o, int off, int hslot) {
+    const FHdr& h = P.h[o];
+    const int nb = __builtin_popcount(h.mlo);
+    const std::string ca = r();
+    e("mov.u32 %s, lfqs_dtabc;", ca.c_str());
+    const Cx c = lds(ca, hslot * ES);
+    for (int k = 0; k * NT < (1 << nb); ++k) {
+      const std::string skip = L(), q = p(), eid = r();
+      e("add.u32 %s, %%ltid, %d;", eid.c_str(), k * NT);
+      e("setp.ge.u32 %s, %s, %u;", q.c_str(), eid.c_str(), 1u << nb);
+      e("@%s bra %s;", q.c_str(), skip.c_str());
+      const std::string a = r();
+      e("mad.lo.u32 %s, %s, %d, %%dtab;", a.c_str(), eid.c_str(), ES);
+      const Cx t = lds(a, off * ES);
+      sts(a, cmulf(c, t), off * ES);
       label(skip);
     }
   }
@@ -1667,8 +1737,20 @@ struct Gen {
       chunk_loop(nch, chunk_bytes, true);
       label(w0);
     }
-    for (const auto& t : dtab_off) dtab_build(t.first, t.second);  // while the tile loads
+    // while the tile loads; tables with hoisted members: partial entries here, C by one
+    // thread each, multiplied in after the barrier
+    std::vector<std::pair<int, int>> fin;  // (table op, slot)
+    for (const auto& t : dtab_off) {
+      const int hs = n_hoisted(t.first) >= 2 && (int)fin.size() < NT - 32 ? (int)fin.size() : -1;
+      if (hs >= 0) fin.emplace_back(t.first, hs);
+      dtab_build(t.first, t.second, hs);
+    }
     sync();
+    if (!fin.empty()) {
+      for (const auto& t : fin) dtab_finalize(t.first, dtab_off[t.first], t.second);
+      sync();
+    }
+    n_dtabc = (int)fin.size();
     {
       const std::string wt = L(), q = p();
       label(wt);
@@ -1766,7 +1848,8 @@ struct Gen {
     out += ".version 8.7\n.target sm_100a\n.address_size 64\n\n";
     out += ".extern .shared .align 128 .b8 lfqs_tile[];\n";
     out += ".shared .align 8 .b64 lfqs_bar;\n";
-    out += ".shared .align 16 .b8 lfqs_dtab[" + std::to_string(dtab_entries() * ES) + "];\n\n";
+    out += ".shared .align 16 .b8 lfqs_dtab[" + std::to_string(dtab_entries() * ES) + "];\n";
+    out += ".shared .align 16 .b8 lfqs_dtabc[" + std::to_string(std::max(n_dtabc, 1) * ES) + "];\n\n";
     const int nc = P.ncoef > 0 ? P.ncoef : 1;
     out += ".visible .entry lfqs_jit(.param .u64 pa, .param .u64 poff, .param .align 16 .b8 pc[" +
            std::to_string(nc * 16) + "])\n";

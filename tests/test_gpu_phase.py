@@ -146,3 +146,22 @@ def test_phase_flag_rejected_alone_is_harmless(L):
     b, k0 = _run(L, n, psi, gates, False)
     assert np.array_equal(a, b) and k == k0
     assert math.isfinite(float(np.abs(a).sum()))
+
+
+@pytest.mark.parametrize("c64", [False, True])
+@pytest.mark.parametrize("tile", [8, 12])
+def test_hoisted_table_factors(L, tile, c64):
+    """Phase-table members decided by the tile index alone (QFT's CPhase rows to qubits
+    outside the tile; controlled diagonals with controls outside the tile) form a per-tile
+    factor the pass compiler computes once per tile (one thread, after a barrier) and the
+    interpreter per entry -- the same products in the same order, so compiled == interpreted
+    bit for bit; within the tolerance of the oracle."""
+    n = 18
+    psi = W.random_state(n, 8)
+    x = 0x2B3C5
+    gates = W.qft(n) + W.qpe(n - 1, x) + diag_heavy(n, 300, 3)
+    ref = O.run_circuit(n, gates, psi.copy())
+    a, _ = _run(L, n, psi, gates, "phase", tile=tile, c64=c64)
+    b, _ = _run(L, n, psi, gates, "jit+phase", tile=tile, c64=c64)
+    assert np.array_equal(a, b)
+    assert np.max(np.abs(b - ref)) <= (2e-5 if c64 else 1e-12)
