@@ -580,7 +580,12 @@ void State::execute(const std::vector<PlanOp>& ops, bool fuse) {
   const int S = n_shards();
   std::vector<ShardRun> cur = plan_run(ops, 0, ex.empty() ? ops.size() : ex[0], fuse);
   std::vector<size_t> from(S, 0), end(S);
-  uint64_t prev = 0;  // chunk of the previous exchange if its leading passes were its whole run
+  // chunk qubits of the previous exchange (0: serial).  choose_chunk keeps them when the
+  // planned ops in between leave them unmixed -- a rank-independent decision (P2P ranks
+  // must pick the same blocks); whether this rank's passes in between all ran block by
+  // block (so the exchanges chain) is a local scheduling matter.
+  uint64_t prev = 0;
+  bool prev_whole = false;  // the previous exchange's leading passes were its whole run
   for (size_t k = 0;; ++k) {
     for (int s = 0; s < S; ++s) end[s] = cur[s].passes.size();
     if (k == ex.size()) {
@@ -597,12 +602,13 @@ void State::execute(const std::vector<PlanOp>& ops, bool fuse) {
       cur = std::move(next);
       std::fill(from.begin(), from.end(), 0);
       prev = 0;
+      prev_whole = false;
       continue;
     }
     // tail: trailing passes that do not mix the chunk qubits; head: leading ones of the
     // next run
     std::vector<size_t> ts(S), he(S, 0), zero(S, 0);
-    bool chained = prev == chunk, whole = true;
+    bool chained = prev == chunk && prev_whole, whole = true;
     for (int s = 0; s < S; ++s) {
       ts[s] = end[s];
       while (ts[s] > from[s] && pass_blockwise(cur[s].passes[ts[s] - 1], chunk, n_local)) --ts[s];
@@ -634,7 +640,8 @@ void State::execute(const std::vector<PlanOp>& ops, bool fuse) {
     const int c = __builtin_popcountll(chunk);
     ov_strided += chunk != ((1ull << c) - 1) << (n_local - c);
     ov_chained += chained;
-    prev = whole ? chunk : 0;
+    prev = chunk;
+    prev_whole = whole;
     cur = std::move(next);
     from = he;
   }
