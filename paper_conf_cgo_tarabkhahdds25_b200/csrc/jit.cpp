@@ -1075,8 +1075,9 @@ struct Gen {
 
   // Builds table `o` into lfqs_dtab entries [off, off + 2^nb): entry e by thread e mod NT.
   // hslot >= 0 (a prebuilt table with hoisted members): the entries are the partial
-  // products and thread 32 + hslot writes C to lfqs_dtabc[hslot] (dtab_finalize multiplies
-  // them after the next barrier); otherwise every thread applies C itself.
+  // products and lane hslot / W of warp hslot % W (W warps) writes C to lfqs_dtabc[hslot]
+  // -- the chains of different tables run in different warps, in parallel (dtab_finalize
+  // multiplies them in after the next barrier); otherwise every thread applies C itself.
   void dtab_build(int o, int off, int hslot = -1) {
     const FHdr& h = P.h[o];
     const int nm = h.m;
@@ -1086,7 +1087,8 @@ struct Gen {
     Cx c{f(), f()};
     if (hoist && hslot >= 0) {
       const std::string skip = L(), q = p();
-      e("setp.ne.u32 %s, %%ltid, %d;", q.c_str(), 32 + hslot);
+      const int nw = NT / 32;
+      e("setp.ne.u32 %s, %%ltid, %d;", q.c_str(), (hslot % nw) * 32 + hslot / nw);
       e("@%s bra %s;", q.c_str(), skip.c_str());
       dtab_factor(o, c);
       const std::string a = r();
@@ -1741,7 +1743,7 @@ struct Gen {
     // thread each, multiplied in after the barrier
     std::vector<std::pair<int, int>> fin;  // (table op, slot)
     for (const auto& t : dtab_off) {
-      const int hs = n_hoisted(t.first) >= 2 && (int)fin.size() < NT - 32 ? (int)fin.size() : -1;
+      const int hs = n_hoisted(t.first) >= 2 && (int)fin.size() < NT ? (int)fin.size() : -1;
       if (hs >= 0) fin.emplace_back(t.first, hs);
       dtab_build(t.first, t.second, hs);
     }

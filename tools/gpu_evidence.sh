@@ -32,7 +32,8 @@ timeout 600 python -m torch.distributed.run --nnodes=1 --nproc-per-node 2 --mast
   --master-port 29517 bench.py --gpus 2 --same-device --qubits-per-gpu 28 --steps 2 --warmup 3 \
   > $O/${TAG}_bench_n2_same_device.json 2> $O/${TAG}_bench_n2.err
 timeout 900 python tools/bench_overlap.py --n 32 --world 4 --circuit qft --bits 0,2 > $O/${TAG}_overlap_qft32_w4.jsonl 2>&1
-for tool in memcheck racecheck synccheck; do
-  timeout 900 compute-sanitizer --tool $tool --print-limit 20 python tools/sanitize_run.py > $O/${TAG}_sanitize_$tool.txt 2>&1
-done
+# compute-sanitizer is closed on this GPU pool (round 2); tools/sanitize_run.py is the
+# workload the r01/r02 sanitizer passes ran (profiles/r0*_sanitizers.md); run here without
+# the sanitizer it still exercises every kernel family once and checks its own results.
+timeout 600 python tools/sanitize_run.py > $O/${TAG}_sanitize_workload.txt 2>&1
 echo done
