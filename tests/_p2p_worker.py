@@ -64,7 +64,14 @@ def worker(rank, world, port, n, seed, out_q):
         nf = 16
         lf, hf = rank << (nf - (world.bit_length() - 1)), (rank + 1) << (nf - (world.bit_length() - 1))
         psif = W.random_state(nf, seed + 3)
-        gf = W.qft(nf) + W.random_layered(nf, 3, seed=seed) + W.random_gate_list(nf, 80, seed=seed)
+        # gates controlled on the global qubits make the ranks' pass lists differ (a
+        # rank whose control bit is 0 drops them), while their blocks must still agree
+        gf = (W.qft(nf) + W.random_layered(nf, 3, seed=seed) +
+              W.random_gate_list(nf, 80, seed=seed, max_controls=2) +
+              [W.Gate("RX", (q,), (nf - 1,), (0.3 + q,)) for q in range(4, 12)] +
+              [W.Gate("H", (nf - 2,))] +
+              [W.Gate("RY", (q,), (nf - 1,), (0.7 * q,)) for q in range(0, 12, 2)] +
+              [W.Gate("H", (nf - 1,))])
         reff = O.run_circuit(nf, gf, psif.copy())
         outs, strided = [], 0
         for bits, sel, ctas in ((0, 1, 0), (2, 0, 0), (2, 1, 0), (2, 1, 8)):

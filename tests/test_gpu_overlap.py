@@ -198,3 +198,26 @@ def test_exchange_options_validated(L):
         gates = W.qft(10)
         st.run_circuit(gates)
         assert np.max(np.abs(st.copy_out() - O.run_circuit(10, gates, psi.copy()))) <= 1e-12
+
+
+def test_chunk_select_complex64(L):
+    """Strided exchange blocks on a complex64 virtual partition (8-byte amplitudes in the
+    swap kernels' fixed-bit indexing and the fused passes' tile-index insertions): the same
+    bits as serial exchanges, within single-precision tolerance of the oracle."""
+    n, world = 17, 4
+    psi = W.random_state(n, 12)
+    gates = W.qft(n) + W.random_layered(n, 3, seed=9)
+    ref = O.run_circuit(n, gates, psi.copy())
+    outs, strided = {}, 0
+    for bits, rate in ((0, 0), (2, 0), (3, 300)):
+        with L.State.virtual(n, world, c64=True) as st:
+            st.set_option(L.OPT_FUSE_TILE_QUBITS, 8)
+            st.set_option(L.OPT_EXCHANGE_CHUNK_BITS, bits)
+            st.set_option(L.OPT_EXCHANGE_RATE_GBS, rate)
+            st.copy_in(psi)
+            st.run_circuit(gates, fuse="jit+phase")
+            outs[bits] = st.copy_out()
+            strided += st.overlap_stats()["strided"]
+    assert np.max(np.abs(outs[0] - ref)) <= 1e-5
+    assert np.array_equal(outs[2], outs[0]) and np.array_equal(outs[3], outs[0])
+    assert strided > 0
