@@ -469,6 +469,12 @@ lfqs_status lfqs_state_pass_count(const lfqs_state* s, uint64_t* passes);
                                   others compute the unscaled butterfly (a + b, a - b): 2 FP64
                                   multiplies per amplitude fewer per Hadamard.  Rounding
                                   changes only (dense tolerance class) */
+#define LFQS_OPT_FUSE_PHASE_EXTRACT 26 /* 1 (default): a fused pass's uncontrolled dense
+                                  1-target gates that are a global phase times a real matrix
+                                  or a real-diagonal / imaginary-off-diagonal one (sqrt X,
+                                  sqrt Y, ...) run in that 4-operation form, the phases
+                                  multiplied into one other dense 1-target gate of the pass.
+                                  Rounding changes only (dense tolerance class) */
 lfqs_status lfqs_set_option(lfqs_state* s, int option, int64_t value);
 const char* lfqs_last_error(void);
 int lfqs_abi_version(void);

@@ -877,6 +877,88 @@ bool tile_dependent(const FHdr& h) {
 // commute with a scalar, so the pass computes the same state up to rounding (dense
 // tolerance class; H is dense): 2 FP64 multiplies per amplitude per folded Hadamard fewer
 // (QFT / Grover / QPE passes).  Interpreter and pass compiler run the same program.
+// Global phase of a dense 1-target matrix (static matrix specialisation, up to a
+// phase): U = z R, |z| = 1, with R real (kind 1: F_UR) or with a real diagonal and an
+// imaginary off-diagonal (kind 2: F_UI) -- 4 FP64 operations per amplitude instead of 8.
+// The parts dropped from R must be below 1e-15 of the largest entry (e.g. sqrt(X) =
+// e^{i pi/4} Rx(pi/2), sqrt(Y) = e^{i pi/4} Ry(pi/2)).  Returns 0 when U has no such form.
+int phase_real_form(const cplx* M, cplx* R, cplx* z) {
+  double best = 0.0;
+  for (int i = 0; i < 4; ++i) best = std::max(best, std::hypot(M[i].re, M[i].im));
+  if (best == 0.0) return 0;
+  const double tol = 1e-15 * best;
+  for (int i = 0; i < 4; ++i) {
+    if (std::hypot(M[i].re, M[i].im) < 0.25 * best) continue;
+    for (int rot = 0; rot < 2; ++rot) {
+      const double a = std::atan2(M[i].im, M[i].re) + (rot ? M_PI / 2 : 0.0);
+      const double zr = std::cos(a), zi = std::sin(a);
+      cplx T[4];
+      for (int k = 0; k < 4; ++k)  // conj(z) * M
+        T[k] = cplx{M[k].re * zr + M[k].im * zi, M[k].im * zr - M[k].re * zi};
+      bool real = true, ui = true;
+      for (int k = 0; k < 4; ++k) {
+        real &= std::fabs(T[k].im) <= tol;
+        ui &= (k == 0 || k == 3) ? std::fabs(T[k].im) <= tol : std::fabs(T[k].re) <= tol;
+      }
+      if (!real && !ui) continue;
+      for (int k = 0; k < 4; ++k) {
+        R[k] = T[k];
+        if (real || k == 0 || k == 3)
+          R[k].im = 0.0;
+        else
+          R[k].re = 0.0;
+      }
+      *z = cplx{zr, zi};
+      return real ? 1 : 2;
+    }
+  }
+  return 0;
+}
+
+// Global phases taken out of a pass's dense 1-target gates (LFQS_OPT_FUSE_PHASE_EXTRACT,
+// default 1).  Every unpredicated F_U2 op that is z R with R of a 4-operation form
+// (phase_real_form) becomes that form, and the product of the z's -- a uniform scalar,
+// which commutes with every linear op of the pass -- is multiplied into one remaining
+// unpredicated F_U2 op's coefficients (a gate without such a form, else the last
+// convertible one stays F_U2 and carries it).  4 FP64 operations per amplitude fewer per
+// converted gate; rounding changes only (dense tolerance class).  Interpreter and pass
+// compiler run the same program.
+void extract_phases(FProg& P) {
+  std::vector<int> conv;
+  int carrier = -1;
+  for (int o = 0; o < P.nops; ++o) {
+    const FHdr& h = P.h[o];
+    if (h.type != F_U2 || h.mlo || h.mhi) continue;
+    cplx M[4], R[4], z;
+    for (int k = 0; k < 4; ++k) M[k] = cplx{P.c[h.coef + k].x, P.c[h.coef + k].y};
+    if (phase_real_form(M, R, &z))
+      conv.push_back(o);
+    else
+      carrier = o;
+  }
+  if (conv.empty()) return;
+  if (carrier < 0) {
+    if (conv.size() < 2) return;
+    carrier = conv.back();
+    conv.pop_back();
+  }
+  cplx Z{1.0, 0.0};
+  for (int o : conv) {
+    FHdr& h = P.h[o];
+    cplx M[4], R[4], z;
+    for (int k = 0; k < 4; ++k) M[k] = cplx{P.c[h.coef + k].x, P.c[h.coef + k].y};
+    const int kind = phase_real_form(M, R, &z);
+    h.type = kind == 1 ? F_UR : F_UI;
+    for (int k = 0; k < 4; ++k) P.c[h.coef + k] = D2(R[k]);
+    Z = cplx{Z.re * z.re - Z.im * z.im, Z.re * z.im + Z.im * z.re};
+  }
+  const FHdr& hc = P.h[carrier];
+  for (int k = 0; k < 4; ++k) {
+    const double2 c = P.c[hc.coef + k];
+    P.c[hc.coef + k] = make_double2(Z.re * c.x - Z.im * c.y, Z.re * c.y + Z.im * c.x);
+  }
+}
+
 void fold_h_scales(FProg& P) {
   int k = 0, last = -1;
   for (int o = 0; o < P.nops; ++o) {
@@ -963,6 +1045,16 @@ void merge_phase_runs(FProg& P, bool split) {
 // coefficient costs 2 per nonzero real / imaginary part (x2 for the amplitude's two
 // components), a coefficient +-1 or +-i is a move / negation (1), zeros cost nothing; a
 // permutation class gate is pure moves (0).
+int cost_of(const cplx* M, int d, GClass cls);
+// A dense 1-target gate as a pass runs it: without controls, its phase-real form when it has
+// one (extract_phases; the phase goes to a carrier op at no cost).
+int cost_1q(const Decoded& u, bool extract) {
+  cplx R[4], z;
+  if (extract && u.cmask == 0 && u.cls == GClass::DENSE && phase_real_form(u.M, R, &z))
+    return cost_of(R, 2, GClass::DENSE);
+  return cost_of(u.M, 2, u.cls);
+}
+
 int cost_of(const cplx* M, int d, GClass cls) {
   if (cls == GClass::PERM_X || cls == GClass::PERM_Y || cls == GClass::PERM_SWAP) return 0;
   int c = 0;
@@ -1031,7 +1123,7 @@ Decoded as_two_target(const Decoded& g) {
 
 template <class LastTouching>
 bool merge_2q(std::vector<Decoded>& prog, Decoded& g, LastTouching&& last_touching,
-              const TileMap& tm) {
+              const TileMap& tm, bool extract) {
   // Diagonal gates are left alone: they are nearly free inside a pass (phase tables fold
   // whole runs of them into one lookup) and stay exact.
   if (g.cls == GClass::DIAG) return false;
@@ -1039,7 +1131,7 @@ bool merge_2q(std::vector<Decoded>& prog, Decoded& g, LastTouching&& last_touchi
     // CZ / CNOT / CPhase / CU: merge in its 4x4 form when that pays (e.g. the dense
     // 1-target gates on both its qubits right before it); otherwise it stays as it is.
     Decoded h = as_two_target(g);
-    return merge_2q(prog, h, last_touching, tm);
+    return merge_2q(prog, h, last_touching, tm, extract);
   }
   // A merged gate is dense: both of its targets must be tile qubits (diagonal gates may
   // act on qubits outside the tile, read from the tile index, a dense one may not).
@@ -1059,7 +1151,7 @@ bool merge_2q(std::vector<Decoded>& prog, Decoded& g, LastTouching&& last_touchi
     cplx E[16], P[16];
     embed2(g.M, a.targets[0] == g.targets[0], E);
     mat4_mul(E, a.M, P);
-    if (cost_of(P, 4, GClass::DENSE) >= cost_of(a.M, 4, a.cls) + cost_of(g.M, 2, g.cls))
+    if (cost_of(P, 4, GClass::DENSE) >= cost_of(a.M, 4, a.cls) + cost_1q(g, extract))
       return false;
     set_dense4(a, P);
     return true;
@@ -1100,7 +1192,7 @@ bool merge_2q(std::vector<Decoded>& prog, Decoded& g, LastTouching&& last_touchi
     embed2(u.M, s2 == 0, E);
     mat4_mul(P, E, T);
     for (int i = 0; i < 16; ++i) P[i] = T[i];
-    cost_sep += cost_of(u.M, 2, u.cls);
+    cost_sep += cost_1q(u, extract);
     ks[s2] = j;
   }
   if (ks[0] < 0 && ks[1] < 0) return false;
@@ -1157,7 +1249,8 @@ void build_program(const LaunchCtx& ctx, const TileCfg& cfg, uint64_t in_tile,
   for (const Decoded* gp : list) {
     if (gp->cls == GClass::NOOP) continue;
     Decoded g = *gp;
-    if (ctx.opt->fuse_merge_2q && merge_2q(prog, g, last_touching, tm)) continue;
+    if (ctx.opt->fuse_merge_2q && merge_2q(prog, g, last_touching, tm, ctx.opt->fuse_phase_extract))
+      continue;
     if (!prog.empty()) {
       size_t ai = prog.size() - 1;
       if (ctx.opt->fuse_merge_commuting && g.m == 1) {
@@ -1186,6 +1279,7 @@ void build_program(const LaunchCtx& ctx, const TileCfg& cfg, uint64_t in_tile,
     prog.push_back(g);
   }
   for (const Decoded& g : prog) encode(g, tm, P);
+  if (ctx.opt->fuse_phase_extract) extract_phases(P);
   if (ctx.opt->fuse_h_scale) fold_h_scales(P);
   if (ctx.phase_tables) merge_phase_runs(P, ctx.opt->fuse_phase_split);
 }

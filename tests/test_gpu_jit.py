@@ -244,3 +244,36 @@ def test_h_scale_folding(L, fuse, c64):
     for hs in (0, 1):  # interpreter == pass compiler
         assert np.array_equal(outs[hs, interp], outs[hs, fuse]), hs
     assert not np.array_equal(outs[0, fuse], outs[1, fuse])  # the folding did change the passes
+
+
+@pytest.mark.parametrize("c64", [False, True])
+@pytest.mark.parametrize("fuse", ["jit", "jit+phase"])
+def test_phase_extraction(L, fuse, c64):
+    """LFQS_OPT_FUSE_PHASE_EXTRACT: dense 1-target gates that are a global phase times a
+    4-operation form (sqrt X = e^{i pi/4} Rx(pi/2), sqrt Y = e^{i pi/4} Ry(pi/2), phased
+    Rx / Ry) run in that form with the phases carried by one other gate of the pass.
+    Compiled == interpreted bit for bit with the extraction on and off; within the dense
+    tolerance of the oracle (Sycamore-like cycles, random layered, controlled sqrt X left
+    alone)."""
+    n = 15
+    psi = W.random_state(n, 33)
+    sx = np.exp(1j * np.pi / 4) * np.array([[1, -1j], [-1j, 1]]) / np.sqrt(2)
+    ph = np.exp(0.37j) * np.array([[np.cos(0.4), -np.sin(0.4)], [np.sin(0.4), np.cos(0.4)]])
+    gates = (W.sycamore_like(3, 5, 6, seed=2) + W.random_layered(n, 3, seed=4) +
+             [W.Gate("UNITARY1", (q,), (), (), ph if q % 2 else sx) for q in range(n)] +
+             [W.Gate("UNITARY1", (3,), (7,), (), sx), W.Gate("UNITARY1", (9,), (), (), ph)])
+    ref = O.run_circuit(n, gates, psi.copy())
+    tol = 2e-5 if c64 else 1e-12
+    interp = True if fuse == "jit" else "phase"
+    outs = {}
+    for pe in (0, 1):
+        for f in (interp, fuse):
+            with L.State.create(n, c64=c64) as st:
+                st.set_option(L.OPT_FUSE_PHASE_EXTRACT, pe)
+                st.copy_in(psi)
+                st.run_circuit(gates, fuse=f)
+                outs[pe, f] = st.copy_out()
+            assert np.max(np.abs(outs[pe, f] - ref)) <= tol, (pe, f)
+    for pe in (0, 1):
+        assert np.array_equal(outs[pe, interp], outs[pe, fuse]), pe
+    assert not np.array_equal(outs[0, fuse], outs[1, fuse])

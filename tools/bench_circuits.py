@@ -79,6 +79,8 @@ def main():
                     help="LFQS_OPT_FUSE_MERGE_COMMUTING (0/1; -1: library default)")
     ap.add_argument("--merge2q", type=int, default=-1,
                     help="LFQS_OPT_FUSE_MERGE_2Q (0/1; -1: library default)")
+    ap.add_argument("--pextract", type=int, default=-1,
+                    help="LFQS_OPT_FUSE_PHASE_EXTRACT (0/1; -1: library default)")
     ap.add_argument("--hscale", type=int, default=-1,
                     help="LFQS_OPT_FUSE_H_SCALE (0/1; -1: library default)")
     ap.add_argument("--c64", action="store_true", help="complex64 state (NEXT-4)")
@@ -145,6 +147,8 @@ def main():
             st.set_option(L.OPT_JIT_LANE_MOVE, args.lane_move)
         if args.hscale >= 0:
             st.set_option(L.OPT_FUSE_H_SCALE, args.hscale)
+        if args.pextract >= 0:
+            st.set_option(L.OPT_FUSE_PHASE_EXTRACT, args.pextract)
         for name in args.circuits.split(","):
             gates, init, meta = circuits[name]
             arr = L.marshal_gates(gates)
@@ -181,7 +185,7 @@ def main():
                        "conv_GBps": 2.0 * ab * 2 ** n * len(gates) / (t / 1e3) / 1e9,
                        "pass_GBps": 2.0 * ab * 2 ** n * passes / (t / 1e3) / 1e9,
                        "dtype": "c64" if args.c64 else "c128", "world": args.world,
-                       "exchanges": x1 - x0, "lane_move": args.lane_move, "merge": args.merge, "merge2q": args.merge2q, "jit_threads": args.jit_threads, "greedy": args.greedy, "lane_reg2": args.lane_reg2, "pool": args.pool, "partial_rt": args.partial_rt, "phase_split": args.phase_split, "hscale": args.hscale,
+                       "exchanges": x1 - x0, "lane_move": args.lane_move, "merge": args.merge, "merge2q": args.merge2q, "jit_threads": args.jit_threads, "greedy": args.greedy, "lane_reg2": args.lane_reg2, "pool": args.pool, "partial_rt": args.partial_rt, "phase_split": args.phase_split, "hscale": args.hscale, "pextract": args.pextract,
                        "hbm_peak_GBps": peak, "peak_source": peak_src}
                 # fraction of the HBM roofline: per pass actually made, and against the
                 # north-star convention of one 2*16*2^n-byte pass per gate
