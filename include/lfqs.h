@@ -475,6 +475,11 @@ lfqs_status lfqs_state_pass_count(const lfqs_state* s, uint64_t* passes);
                                   sqrt Y, ...) run in that 4-operation form, the phases
                                   multiplied into one other dense 1-target gate of the pass.
                                   Rounding changes only (dense tolerance class) */
+#define LFQS_OPT_CANON_FUSE 27 /* sharded states, 1 (default): the local SWAP / X passes
+                                  that restore the canonical qubit map (copy_in / copy_out /
+                                  the end of a compiled circuit) run fused, a run of them in
+                                  one tile pass, and their exchanges overlap like a circuit's;
+                                  0: one pass per SWAP.  Moves only: bit-identical */
 lfqs_status lfqs_set_option(lfqs_state* s, int option, int64_t value);
 const char* lfqs_last_error(void);
 int lfqs_abi_version(void);

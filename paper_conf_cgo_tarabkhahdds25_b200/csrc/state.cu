@@ -647,10 +647,19 @@ void State::execute(const std::vector<PlanOp>& ops, bool fuse) {
   }
 }
 
+// The canonicalising ops are local SWAP passes (and X passes for global flips) between
+// exchanges: moves only, so they run fused (LFQS_OPT_CANON_FUSE, default 1) -- runs of
+// SWAPs share one tile pass, bit-identical to one pass per SWAP, and the exchanges between
+// them may take strided chunk qubits and overlap with them (QFT(33) on 8 ranks: 8 SWAP
+// passes -> 3).  The interpreting kernel runs them (no compiled passes outside a run).
 void State::canonicalize() {
   std::vector<PlanOp> ops;
   plan.plan_canonicalize(ops);
-  execute(ops, false);
+  const bool j = jit, pt = phase_tables;
+  jit = phase_tables = false;
+  execute(ops, opt.canon_fuse && !soa);
+  jit = j;
+  phase_tables = pt;
 }
 
 void State::apply(const Decoded& g) {

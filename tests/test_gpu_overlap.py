@@ -221,3 +221,27 @@ def test_chunk_select_complex64(L):
     assert np.max(np.abs(outs[0] - ref)) <= 1e-5
     assert np.array_equal(outs[2], outs[0]) and np.array_equal(outs[3], outs[0])
     assert strided > 0
+
+
+@pytest.mark.parametrize("world", [2, 8])
+def test_canonicalize_fused(L, world):
+    """LFQS_OPT_CANON_FUSE: the SWAP passes that restore the canonical map run fused (a run
+    of them in one tile pass) with their exchanges overlapped -- moves only, so copy_out is
+    bit-identical to one pass per SWAP, in fewer passes."""
+    n = 18
+    psi = W.random_state(n, 41)
+    gates = W.qft(n) + W.random_gate_list(n, 60, seed=6, max_controls=1)
+    ref = O.run_circuit(n, gates, psi.copy())
+    outs, canon_passes = {}, {}
+    for cf in (0, 1):
+        with L.State.virtual(n, world) as st:
+            st.set_option(L.OPT_CANON_FUSE, cf)
+            st.set_option(L.OPT_FUSE_TILE_QUBITS, 10)
+            st.copy_in(psi)
+            st.run_circuit(gates, fuse="jit+phase")
+            p0 = st.passes()
+            outs[cf] = st.copy_out()  # canonicalises
+            canon_passes[cf] = st.passes() - p0
+    assert np.array_equal(outs[0], outs[1])
+    assert np.max(np.abs(outs[1] - ref)) <= 1e-12
+    assert canon_passes[1] <= canon_passes[0], canon_passes
