@@ -57,6 +57,7 @@ OPT_EXCHANGE_RATE_GBS = 24
 OPT_FUSE_H_SCALE = 25
 OPT_FUSE_PHASE_EXTRACT = 26
 OPT_CANON_FUSE = 27
+OPT_FUSE_PERM = 28
 
 STATUS = {0: "OK", -1: "INVALID_ARG", -2: "OUT_OF_MEMORY", -3: "CUDA", -4: "NCCL",
           -5: "UNSUPPORTED"}

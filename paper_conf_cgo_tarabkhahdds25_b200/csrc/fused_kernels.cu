@@ -1361,9 +1361,161 @@ bool run_fused_circuit(const LaunchCtx& ctx, const std::vector<Decoded>& gates, 
 // launching anything; launch_fused_pass runs one of them on any block of the state whose
 // qubits include every qubit the pass touches (the executor runs boundary passes of an
 // overlapped exchange part by part, state.cu).
-void plan_fused_schedule(const LaunchCtx& ctx_in, const std::vector<Decoded>& gates,
+// ---- bit-permutation pass (LFQS_OPT_FUSE_PERM) -------------------------------------------
+// A run of SWAP gates composes into a permutation pi of the index bits (SWAP
+// moves amplitudes only).  When pi is an involution (disjoint transpositions: QFT's final
+// bit reversal), the tile bits S = {0..L-1} u pi({0..L-1}) are closed under it, and so is
+// the rest: tile t (the free bits) maps to tile sigma(t), with sigma(sigma(t)) = t.  One CTA
+// per tile pair loads both tiles (coalesced runs of 2^L amplitudes), then writes each
+// destination element from the shared-memory copy of its source: every amplitude read
+// and written once -- one HBM pass for the whole SWAP run instead of one per few SWAPs.
+// Moves only: bit-identical to the SWAP gates.
+constexpr int kPermMaxBits = 10;  // tile bits (2 tiles x 1024 x 16 B = 32 KiB of smem)
+
+template <class S>
+__global__ void __launch_bounds__(256) k_bitperm(cx<S>* __restrict__ a,
+                                                 const __grid_constant__ PermArgs A) {
+  extern __shared__ __align__(16) unsigned char perm_smem[];
+  cx<S>* sm = reinterpret_cast<cx<S>*>(perm_smem);
+  const uint64_t t = blockIdx.x;
+  uint64_t pt = 0, bt = 0, bp = 0;
+  for (int k = 0; k < A.nf; ++k) {
+    const uint64_t b = (t >> k) & 1;
+    pt |= b << A.fdst[k];
+    bt |= b << A.fbit[k];
+  }
+  if (pt < t) return;  // the partner's CTA moves this pair
+  for (int k = 0; k < A.nf; ++k) bp |= ((pt >> k) & 1) << A.fbit[k];
+  const uint32_t T = 1u << A.ns;
+  auto dep = [&](uint32_t e) {
+    uint64_t o = 0;
+    for (int k = 0; k < A.ns; ++k) o |= (uint64_t)((e >> k) & 1) << A.sbit[k];
+    return o;
+  };
+  const bool pair = pt != t;
+  for (uint32_t e = threadIdx.x; e < T; e += 256) {
+    const uint64_t o = dep(e);
+    sm[e] = ld1(a + (bt | o));
+    if (pair) sm[T + e] = ld1(a + (bp | o));
+  }
+  __syncthreads();
+  for (uint32_t e = threadIdx.x; e < T; e += 256) {
+    // destination element e holds the source element whose bit k is e's bit sdst[k]
+    uint32_t src = 0;
+    for (int k = 0; k < A.ns; ++k) src |= ((e >> A.sdst[k]) & 1u) << k;
+    const uint64_t o = dep(e);
+    st1(a + (bp | o), sm[src]);
+    if (pair) st1(a + (bt | o), sm[T + src]);
+  }
+}
+
+void launch_bitperm(const LaunchCtx& ctx, const PermArgs& A) {
+  const uint64_t tiles = 1ull << A.nf;
+  require(tiles < (1ull << 31), "internal: bit-permutation grid too large");
+  const size_t smem = (size_t)2 * (ctx.c64 ? 8 : 16) << A.ns;
+  if (ctx.c64)
+    k_bitperm<float><<<(unsigned)tiles, 256, smem, ctx.stream>>>(
+        reinterpret_cast<cx<float>*>(ctx.amps), A);
+  else
+    k_bitperm<double><<<(unsigned)tiles, 256, smem, ctx.stream>>>(
+        reinterpret_cast<cx<double>*>(ctx.amps), A);
+  LFQS_CUDA_CHECK(cudaGetLastError());
+  ++*ctx.launch_counter;
+}
+
+// The trailing run of uncontrolled SWAPs of `gates` (NOOPs skipped) as one permutation pass:
+// *end = index of its first gate.  False when the run is shorter than 3 SWAPs, not an
+// involution, or the shard too small.
+bool plan_swap_suffix(const LaunchCtx& ctx, const std::vector<Decoded>& gates, size_t* end,
+                      PermArgs* pa, uint64_t* moved) {
+  const int nl = ctx.n_local;
+  size_t i = gates.size();
+  int count = 0;
+  while (i > 0) {
+    const Decoded& g = gates[i - 1];
+    if (g.cls == GClass::NOOP) {
+      --i;
+      continue;
+    }
+    if (g.cls != GClass::PERM_SWAP || g.cmask != 0 || g.m != 2) break;
+    --i;
+    ++count;
+  }
+  if (count < 3) return false;
+  int pi[64];  // pi[q]: the position the data bit at q ends at
+  for (int q = 0; q < 64; ++q) pi[q] = q;
+  for (size_t k = i; k < gates.size(); ++k) {
+    const Decoded& g = gates[k];
+    if (g.cls == GClass::NOOP) continue;
+    const int x = g.targets[0], y = g.targets[1];
+    for (int q = 0; q < nl; ++q) pi[q] = pi[q] == x ? y : pi[q] == y ? x : pi[q];
+  }
+  for (int q = 0; q < nl; ++q)
+    if (pi[pi[q]] != q) return false;
+  uint64_t S = 0;
+  for (int L = 1; L <= nl; ++L) {  // the most low bits whose closure fits
+    uint64_t s2 = 0;
+    for (int q = 0; q < L; ++q) s2 |= (1ull << q) | (1ull << pi[q]);
+    if (__builtin_popcountll(s2) > kPermMaxBits) break;
+    S = s2;
+  }
+  if ((S & 31) != 31 || nl - __builtin_popcountll(S) < 1) return false;
+  PermArgs A;
+  int sidx[64], fidx[64];
+  for (int q = 0; q < nl; ++q) {
+    if (S >> q & 1) {
+      sidx[q] = A.ns;
+      A.sbit[A.ns++] = (uint8_t)q;
+    } else {
+      fidx[q] = A.nf;
+      A.fbit[A.nf++] = (uint8_t)q;
+    }
+  }
+  for (int k = 0; k < A.ns; ++k) A.sdst[k] = (uint8_t)sidx[pi[A.sbit[k]]];
+  for (int k = 0; k < A.nf; ++k) A.fdst[k] = (uint8_t)fidx[pi[A.fbit[k]]];
+  uint64_t mv = 0;
+  for (int q = 0; q < nl; ++q)
+    if (pi[q] != q) mv |= 1ull << q;
+  *pa = A;
+  *moved = mv;
+  *end = i;
+  return true;
+}
+
+void plan_fused_schedule(const LaunchCtx& ctx_in, const std::vector<Decoded>& gates_in,
                          int tile_qubits, std::vector<FusedPass>& out) {
   out.clear();
+  // A trailing run of SWAPs becomes one bit-permutation pass, appended after the other
+  // passes when this function returns (plan-only: counted).
+  struct PermTail {
+    const LaunchCtx& c;
+    std::vector<FusedPass>& o;
+    std::shared_ptr<PermArgs> pa;
+    uint64_t moved = 0;
+    ~PermTail() {
+      if (!pa) return;
+      if (c.plan_only) {
+        ++*c.launch_counter;
+        return;
+      }
+      FusedPass ps;
+      ps.perm = pa;
+      ps.qmask = ps.nd_mask = moved;
+      o.push_back(std::move(ps));
+    }
+  } tail{ctx_in, out, nullptr, 0};
+  std::vector<Decoded> trimmed;
+  const std::vector<Decoded>* gp = &gates_in;
+  if (ctx_in.opt->fuse_perm && !ctx_in.soa) {
+    size_t end = 0;
+    PermArgs pa;
+    if (plan_swap_suffix(ctx_in, gates_in, &end, &pa, &tail.moved)) {
+      tail.pa = std::make_shared<PermArgs>(pa);
+      trimmed.assign(gates_in.begin(), gates_in.begin() + end);
+      gp = &trimmed;
+    }
+  }
+  const std::vector<Decoded>& gates = *gp;
   // LFQS_OPT_FUSE_LOW_QUBITS = 0 (auto): plan the passes (host only) with 7 and with 6
   // contiguous low qubits per tile and take 6 only when it saves >= 20 % of the passes --
   // a 1-KiB-chunk tile costs ~10 % more per pass (twice the TMA copies) but claims one
@@ -1492,7 +1644,9 @@ void plan_fused_schedule(const LaunchCtx& ctx_in, const std::vector<Decoded>& ga
 
 void launch_fused_pass(const LaunchCtx& ctx, const std::vector<Decoded>& gates,
                        const FusedPass& ps) {
-  if (ps.prog)
+  if (ps.perm)
+    launch_bitperm(ctx, *ps.perm);
+  else if (ps.prog)
     launch_built(ctx, ps.K, *ps.prog, ps.key.empty() ? nullptr : &ps.key);
   else
     launch_gate(ctx, gates[ps.gate]);
@@ -1505,7 +1659,7 @@ void launch_fused_pass(const LaunchCtx& ctx, const std::vector<Decoded>& gates,
 // bits (Planner::rank_local with the block index in the role of the rank).
 bool pass_blockwise(const FusedPass& ps, uint64_t chunk, int n_local) {
   const int c = __builtin_popcountll(chunk);
-  if (c == 0 || c > 3 || (ps.nd_mask & chunk) || (chunk >> n_local)) return false;
+  if (c == 0 || c > 3 || ps.perm || (ps.nd_mask & chunk) || (chunk >> n_local)) return false;
   if (!ps.prog) return chunk == (((1ull << c) - 1) << (n_local - c));
   if (ps.K > n_local - c) return false;
   const FTile& tg = ps.prog->tile;

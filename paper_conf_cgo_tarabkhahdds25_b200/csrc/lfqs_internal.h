@@ -108,6 +108,7 @@ struct Options {
   int stream_max_prefix = 0;  // lfqs_run_circuit_streamed: max gates run per piece (0: all)
   bool fuse_phase_split = false;     // phase tables: tile-invariant / tile-dependent groups
   bool fuse_merge_commuting = true;  // merge same-qubit 1-target gates across commuting gates
+  bool fuse_perm = true;     // trailing SWAP runs as one bit-permutation pass (k_bitperm)
   bool canon_fuse = true;     // canonicalising SWAP passes fused (State::canonicalize)
   bool fuse_phase_extract = true;  // global phases of dense 1-target gates (extract_phases)
   bool fuse_h_scale = true;   // Hadamard scales of a fused pass folded into one (fold_h_scales)
@@ -163,9 +164,22 @@ bool run_fused_circuit(const LaunchCtx& ctx, const std::vector<Decoded>& gates, 
 // Whole-list fused execution with exact-commutation reordering (fused_kernels.cu).
 void run_fused_schedule(const LaunchCtx& ctx, const std::vector<Decoded>& gates, int tile_qubits);
 
-// One pass of a fused schedule: a single gate's class kernel or a fused tile program.
+// A qubit permutation that is an involution (a run of disjoint-cycle SWAPs: QFT's final
+// bit reversal) applied in one pass (fused_kernels.cu k_bitperm): the tile bits are closed
+// under it, so tile t's data goes to tile sigma(t) with its bits permuted inside the tile.
+struct PermArgs {
+  int ns = 0, nf = 0;      // tile bits, tile-index bits
+  uint8_t sbit[16] = {};   // element bit k <-> position sbit[k] (ascending)
+  uint8_t sdst[16] = {};   // element bit k of the source goes to element bit sdst[k]
+  uint8_t fbit[48] = {};   // tile-index bit k <-> position fbit[k] (ascending)
+  uint8_t fdst[48] = {};   // tile-index bit k goes to tile-index bit fdst[k]
+};
+
+// One pass of a fused schedule: a single gate's class kernel, a fused tile program, or a
+// bit-permutation pass.
 struct FProg;  // fused_prog.h
 struct FusedPass {
+  std::shared_ptr<PermArgs> perm;  // bit-permutation pass (a trailing run of SWAPs)
   int gate = -1;                 // single-gate pass: index into the gate list
   std::shared_ptr<FProg> prog;   // fused pass (tile program)
   std::string key;               // compiled-pass cache key (LFQS_FUSE_JIT), else empty

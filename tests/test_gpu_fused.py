@@ -218,3 +218,53 @@ def test_merge_2q_matches_oracle_and_unmerged(L, fuse):
         st.copy_in(psi)
         st.run_circuit(exact, fuse=fuse)
         assert np.array_equal(st.copy_out(), O.run_circuit(n, exact, psi.copy()))
+
+
+@pytest.mark.parametrize("c64", [False, True])
+@pytest.mark.parametrize("n", [12, 16, 21])
+def test_bitperm_pass(n, c64):
+    """LFQS_OPT_FUSE_PERM: a fused run ending in >= 3 SWAPs whose composition is an
+    involution (QFT's bit reversal, disjoint SWAPs) applies them as one bit-permutation
+    pass.  Moves only: an exact circuit with such a tail is bit-identical with the pass on
+    and off and to the oracle; QFT within tolerance, compiled == interpreted; a cyclic SWAP
+    chain (not an involution) falls back to the tile passes."""
+    import torch
+    if not torch.cuda.is_available():
+        pytest.skip("needs a GPU")
+    import paper_conf_cgo_tarabkhahdds25_b200 as L
+    psi = W.random_state(n, 77 + n)
+    rev = [W.Gate("SWAP", (q, n - 1 - q)) for q in range(n // 2)]
+    exact = [g for g in W.random_gate_list(n, 120, seed=n, max_controls=2) if g.exact]
+    cases = {"rev": exact + rev,
+             "pairs": exact + [W.Gate("SWAP", (0, 7)), W.Gate("SWAP", (3, n - 2)),
+                               W.Gate("SWAP", (1, 9)), W.Gate("SWAP", (2, n - 1)),
+                               W.Gate("SWAP", (4, 6))],
+             "cycle": exact + [W.Gate("SWAP", (0, 5)), W.Gate("SWAP", (5, 9)),
+                               W.Gate("SWAP", (9, n - 1))]}
+    tol = 0.0
+    for name, gates in cases.items():
+        ref = O.run_circuit(n, gates, psi.copy())
+        outs = []
+        for perm in (0, 1):
+            for fuse in (True, "jit"):
+                with L.State.create(n, c64=c64) as st:
+                    st.set_option(L.OPT_FUSE_PERM, perm)
+                    st.copy_in(psi)
+                    st.run_circuit(gates, fuse=fuse)
+                    outs.append(st.copy_out())
+        for o in outs[1:]:
+            assert np.array_equal(o, outs[0]), name
+        if not c64:
+            assert np.array_equal(outs[0], ref), name
+    qft = W.qft(n)
+    ref = O.run_circuit(n, qft, psi.copy())
+    res = {}
+    for perm in (0, 1):
+        for fuse in ("phase", "jit+phase"):
+            with L.State.create(n, c64=c64) as st:
+                st.set_option(L.OPT_FUSE_PERM, perm)
+                st.copy_in(psi)
+                st.run_circuit(qft, fuse=fuse)
+                res[perm, fuse] = st.copy_out()
+            assert np.max(np.abs(res[perm, fuse] - ref)) <= (2e-5 if c64 else 1e-12)
+    assert np.array_equal(res[1, "phase"], res[1, "jit+phase"])

@@ -79,6 +79,8 @@ def main():
                     help="LFQS_OPT_FUSE_MERGE_COMMUTING (0/1; -1: library default)")
     ap.add_argument("--merge2q", type=int, default=-1,
                     help="LFQS_OPT_FUSE_MERGE_2Q (0/1; -1: library default)")
+    ap.add_argument("--perm", type=int, default=-1,
+                    help="LFQS_OPT_FUSE_PERM (0/1; -1: library default)")
     ap.add_argument("--pextract", type=int, default=-1,
                     help="LFQS_OPT_FUSE_PHASE_EXTRACT (0/1; -1: library default)")
     ap.add_argument("--hscale", type=int, default=-1,
@@ -114,6 +116,9 @@ def main():
         # light programs: fused-pass memory efficiency (one H per qubit; X pairs)
         "hlayer": ([W.Gate("H", (q,)) for q in range(n)], lambda st: st.init_basis(0), {}),
         "xlow": ([W.Gate("X", (0,)), W.Gate("X", (1,))], lambda st: st.init_basis(0), {}),
+        # QFT's final bit reversal alone (one bit-permutation pass, LFQS_OPT_FUSE_PERM)
+        "bitrev": ([W.Gate("SWAP", (q, n - 1 - q)) for q in range(n // 2)],
+                   lambda st: st.init_basis(0), {}),
         "xhigh": ([W.Gate("X", (n - 1,)), W.Gate("X", (n - 5,))], lambda st: st.init_basis(0), {}),
     }
     ab = 8 if args.c64 else 16
@@ -149,6 +154,8 @@ def main():
             st.set_option(L.OPT_FUSE_H_SCALE, args.hscale)
         if args.pextract >= 0:
             st.set_option(L.OPT_FUSE_PHASE_EXTRACT, args.pextract)
+        if args.perm >= 0:
+            st.set_option(L.OPT_FUSE_PERM, args.perm)
         for name in args.circuits.split(","):
             gates, init, meta = circuits[name]
             arr = L.marshal_gates(gates)
@@ -185,7 +192,7 @@ def main():
                        "conv_GBps": 2.0 * ab * 2 ** n * len(gates) / (t / 1e3) / 1e9,
                        "pass_GBps": 2.0 * ab * 2 ** n * passes / (t / 1e3) / 1e9,
                        "dtype": "c64" if args.c64 else "c128", "world": args.world,
-                       "exchanges": x1 - x0, "lane_move": args.lane_move, "merge": args.merge, "merge2q": args.merge2q, "jit_threads": args.jit_threads, "greedy": args.greedy, "lane_reg2": args.lane_reg2, "pool": args.pool, "partial_rt": args.partial_rt, "phase_split": args.phase_split, "hscale": args.hscale, "pextract": args.pextract,
+                       "exchanges": x1 - x0, "lane_move": args.lane_move, "merge": args.merge, "merge2q": args.merge2q, "jit_threads": args.jit_threads, "greedy": args.greedy, "lane_reg2": args.lane_reg2, "pool": args.pool, "partial_rt": args.partial_rt, "phase_split": args.phase_split, "hscale": args.hscale, "pextract": args.pextract, "perm": args.perm,
                        "hbm_peak_GBps": peak, "peak_source": peak_src}
                 # fraction of the HBM roofline: per pass actually made, and against the
                 # north-star convention of one 2*16*2^n-byte pass per gate
