@@ -480,10 +480,11 @@ lfqs_status lfqs_state_pass_count(const lfqs_state* s, uint64_t* passes);
                                   the end of a compiled circuit) run fused, a run of them in
                                   one tile pass, and their exchanges overlap like a circuit's;
                                   0: one pass per SWAP.  Moves only: bit-identical */
-#define LFQS_OPT_FUSE_PERM 28 /* 1 (default): a fused run ending in >= 3 uncontrolled SWAPs
-                                  whose composition is an involution (QFT's bit reversal)
-                                  applies them as one bit-permutation pass (tile pairs
-                                  closed under the permutation).  Moves only: bit-identical */
+#define LFQS_OPT_FUSE_PERM 28 /* 1 (default, auto tile size): a fused run ending in >= 3
+                                  uncontrolled SWAPs whose composition is an involution
+                                  (QFT's bit reversal) applies them as one bit-permutation
+                                  pass (tile pairs closed under the permutation); 8..12: that
+                                  many tile bits at most; 0: off.  Moves only: bit-identical */
 lfqs_status lfqs_set_option(lfqs_state* s, int option, int64_t value);
 const char* lfqs_last_error(void);
 int lfqs_abi_version(void);

@@ -538,7 +538,11 @@ lfqs_status lfqs_set_option(lfqs_state* s, int option, int64_t value) {
       case LFQS_OPT_FUSE_H_SCALE: st->opt.fuse_h_scale = value != 0; break;
       case LFQS_OPT_FUSE_PHASE_EXTRACT: st->opt.fuse_phase_extract = value != 0; break;
       case LFQS_OPT_CANON_FUSE: st->opt.canon_fuse = value != 0; break;
-      case LFQS_OPT_FUSE_PERM: st->opt.fuse_perm = value != 0; break;
+      case LFQS_OPT_FUSE_PERM:
+        require(value == 0 || value == 1 || (value >= 8 && value <= 12),
+                "LFQS_OPT_FUSE_PERM must be 0, 1 or a tile size in [8, 12]");
+        st->opt.fuse_perm = (int)value;
+        break;
       case LFQS_OPT_EXCHANGE_CHUNK_BITS:
         require(value >= 0 && value <= 3, "LFQS_OPT_EXCHANGE_CHUNK_BITS must be in [0, 3]");
         st->opt.exchange_chunk_bits = (int)value;  // the plan is the same for every value

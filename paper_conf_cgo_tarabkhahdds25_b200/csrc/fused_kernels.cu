@@ -1370,13 +1370,17 @@ bool run_fused_circuit(const LaunchCtx& ctx, const std::vector<Decoded>& gates, 
 // destination element from the shared-memory copy of its source: every amplitude read
 // and written once -- one HBM pass for the whole SWAP run instead of one per few SWAPs.
 // Moves only: bit-identical to the SWAP gates.
-constexpr int kPermMaxBits = 10;  // tile bits (2 tiles x 1024 x 16 B = 32 KiB of smem)
 
-template <class S>
+template <class S, int EPT>
 __global__ void __launch_bounds__(256) k_bitperm(cx<S>* __restrict__ a,
                                                  const __grid_constant__ PermArgs A) {
   extern __shared__ __align__(16) unsigned char perm_smem[];
   cx<S>* sm = reinterpret_cast<cx<S>*>(perm_smem);
+  constexpr uint32_t T = 256u * EPT;  // 2^ns elements per tile
+  // shared-memory slot of element e: one 16-B pad per 32 elements, so that the gather by
+  // permuted index (lanes 32 elements apart for a bit reversal) hits distinct banks
+  constexpr uint32_t TP = T + T / 32;
+  auto slot = [](uint32_t e) { return e + (e >> 5); };
   const uint64_t t = blockIdx.x;
   uint64_t pt = 0, bt = 0, bp = 0;
   for (int k = 0; k < A.nf; ++k) {
@@ -1386,39 +1390,67 @@ __global__ void __launch_bounds__(256) k_bitperm(cx<S>* __restrict__ a,
   }
   if (pt < t) return;  // the partner's CTA moves this pair
   for (int k = 0; k < A.nf; ++k) bp |= ((pt >> k) & 1) << A.fbit[k];
-  const uint32_t T = 1u << A.ns;
   auto dep = [&](uint32_t e) {
     uint64_t o = 0;
-    for (int k = 0; k < A.ns; ++k) o |= (uint64_t)((e >> k) & 1) << A.sbit[k];
+#pragma unroll
+    for (int k = 0; k < 16; ++k)
+      if (k < A.ns) o |= (uint64_t)((e >> k) & 1) << A.sbit[k];
     return o;
   };
   const bool pair = pt != t;
-  for (uint32_t e = threadIdx.x; e < T; e += 256) {
-    const uint64_t o = dep(e);
-    sm[e] = ld1(a + (bt | o));
-    if (pair) sm[T + e] = ld1(a + (bp | o));
+  // every load of both tiles in flight before the first shared-memory store
+  cx<S> v[2 * EPT];
+#pragma unroll
+  for (int r = 0; r < EPT; ++r) {
+    const uint64_t o = dep(r * 256u + threadIdx.x);
+    v[r] = ld1(a + (bt | o));
+    if (pair) v[EPT + r] = ld1(a + (bp | o));
+  }
+#pragma unroll
+  for (int r = 0; r < EPT; ++r) {
+    sm[slot(r * 256u + threadIdx.x)] = v[r];
+    if (pair) sm[TP + slot(r * 256u + threadIdx.x)] = v[EPT + r];
   }
   __syncthreads();
-  for (uint32_t e = threadIdx.x; e < T; e += 256) {
+#pragma unroll
+  for (int r = 0; r < EPT; ++r) {
     // destination element e holds the source element whose bit k is e's bit sdst[k]
+    const uint32_t e = r * 256u + threadIdx.x;
     uint32_t src = 0;
-    for (int k = 0; k < A.ns; ++k) src |= ((e >> A.sdst[k]) & 1u) << k;
+#pragma unroll
+    for (int k = 0; k < 16; ++k)
+      if (k < A.ns) src |= ((e >> A.sdst[k]) & 1u) << k;
     const uint64_t o = dep(e);
-    st1(a + (bp | o), sm[src]);
-    if (pair) st1(a + (bt | o), sm[T + src]);
+    st1(a + (bp | o), sm[slot(src)]);
+    if (pair) st1(a + (bt | o), sm[TP + slot(src)]);
+  }
+}
+
+template <class S>
+void launch_bitperm_t(const LaunchCtx& ctx, const PermArgs& A, unsigned tiles) {
+  const size_t smem = (size_t)2 * sizeof(cx<S>) * ((1u << A.ns) + (1u << A.ns) / 32);
+  auto* p = reinterpret_cast<cx<S>*>(ctx.amps);
+  auto go = [&](auto kern) {
+    ensure_smem_attr((const void*)kern, (int)smem);
+    kern<<<tiles, 256, smem, ctx.stream>>>(p, A);
+  };
+  switch (A.ns) {
+    case 8: go(k_bitperm<S, 1>); break;
+    case 9: go(k_bitperm<S, 2>); break;
+    case 10: go(k_bitperm<S, 4>); break;
+    case 11: go(k_bitperm<S, 8>); break;
+    default: go(k_bitperm<S, 16>); break;
   }
 }
 
 void launch_bitperm(const LaunchCtx& ctx, const PermArgs& A) {
   const uint64_t tiles = 1ull << A.nf;
-  require(tiles < (1ull << 31), "internal: bit-permutation grid too large");
-  const size_t smem = (size_t)2 * (ctx.c64 ? 8 : 16) << A.ns;
+  require(tiles < (1ull << 31) && A.ns >= 8 && A.ns <= 12,
+          "internal: bad bit-permutation pass geometry");
   if (ctx.c64)
-    k_bitperm<float><<<(unsigned)tiles, 256, smem, ctx.stream>>>(
-        reinterpret_cast<cx<float>*>(ctx.amps), A);
+    launch_bitperm_t<float>(ctx, A, (unsigned)tiles);
   else
-    k_bitperm<double><<<(unsigned)tiles, 256, smem, ctx.stream>>>(
-        reinterpret_cast<cx<double>*>(ctx.amps), A);
+    launch_bitperm_t<double>(ctx, A, (unsigned)tiles);
   LFQS_CUDA_CHECK(cudaGetLastError());
   ++*ctx.launch_counter;
 }
@@ -1444,6 +1476,9 @@ bool plan_swap_suffix(const LaunchCtx& ctx, const std::vector<Decoded>& gates, s
   if (count < 3) return false;
   int pi[64];  // pi[q]: the position the data bit at q ends at
   for (int q = 0; q < 64; ++q) pi[q] = q;
+  // tile bits: auto (1) = 10 for complex128 (2 x 16 KiB tiles; 12 bits' 2 x 64 KiB allow one
+  // CTA per SM: 8.0 -> 11.3 ms for the n = 30 bit reversal), 12 for complex64 (15.2 -> 13.9)
+  const int max_bits = ctx.opt->fuse_perm == 1 ? (ctx.c64 ? 12 : 10) : ctx.opt->fuse_perm;
   for (size_t k = i; k < gates.size(); ++k) {
     const Decoded& g = gates[k];
     if (g.cls == GClass::NOOP) continue;
@@ -1456,10 +1491,11 @@ bool plan_swap_suffix(const LaunchCtx& ctx, const std::vector<Decoded>& gates, s
   for (int L = 1; L <= nl; ++L) {  // the most low bits whose closure fits
     uint64_t s2 = 0;
     for (int q = 0; q < L; ++q) s2 |= (1ull << q) | (1ull << pi[q]);
-    if (__builtin_popcountll(s2) > kPermMaxBits) break;
+    if (__builtin_popcountll(s2) > max_bits) break;
     S = s2;
   }
-  if ((S & 31) != 31 || nl - __builtin_popcountll(S) < 1) return false;
+  if ((S & 31) != 31 || __builtin_popcountll(S) < 8 || nl - __builtin_popcountll(S) < 1)
+    return false;
   PermArgs A;
   int sidx[64], fidx[64];
   for (int q = 0; q < nl; ++q) {
@@ -1506,7 +1542,7 @@ void plan_fused_schedule(const LaunchCtx& ctx_in, const std::vector<Decoded>& ga
   } tail{ctx_in, out, nullptr, 0};
   std::vector<Decoded> trimmed;
   const std::vector<Decoded>* gp = &gates_in;
-  if (ctx_in.opt->fuse_perm && !ctx_in.soa) {
+  if (ctx_in.opt->fuse_perm != 0 && !ctx_in.soa) {
     size_t end = 0;
     PermArgs pa;
     if (plan_swap_suffix(ctx_in, gates_in, &end, &pa, &tail.moved)) {

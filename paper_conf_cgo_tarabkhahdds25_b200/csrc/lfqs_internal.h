@@ -108,7 +108,8 @@ struct Options {
   int stream_max_prefix = 0;  // lfqs_run_circuit_streamed: max gates run per piece (0: all)
   bool fuse_phase_split = false;     // phase tables: tile-invariant / tile-dependent groups
   bool fuse_merge_commuting = true;  // merge same-qubit 1-target gates across commuting gates
-  bool fuse_perm = true;     // trailing SWAP runs as one bit-permutation pass (k_bitperm)
+  int fuse_perm = 1;         // trailing SWAP runs as one bit-permutation pass (k_bitperm)
+                             // with at most this many tile bits (0: off, 1: auto)
   bool canon_fuse = true;     // canonicalising SWAP passes fused (State::canonicalize)
   bool fuse_phase_extract = true;  // global phases of dense 1-target gates (extract_phases)
   bool fuse_h_scale = true;   // Hadamard scales of a fused pass folded into one (fold_h_scales)
