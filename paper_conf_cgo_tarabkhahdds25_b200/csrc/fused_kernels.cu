@@ -1455,31 +1455,22 @@ void launch_bitperm(const LaunchCtx& ctx, const PermArgs& A) {
   ++*ctx.launch_counter;
 }
 
-// The trailing run of uncontrolled SWAPs of `gates` (NOOPs skipped) as one permutation pass:
-// *end = index of its first gate.  False when the run is shorter than 3 SWAPs, not an
-// involution, or the shard too small.
-bool plan_swap_suffix(const LaunchCtx& ctx, const std::vector<Decoded>& gates, size_t* end,
-                      PermArgs* pa, uint64_t* moved) {
+bool is_plain_swap(const Decoded& g) {
+  return g.cls == GClass::PERM_SWAP && g.cmask == 0 && g.m == 2;
+}
+
+// The SWAPs of gates[b, e) (NOOPs skipped) as one permutation pass.  False when the
+// composition is not an involution or the shard is too small for closed tiles.
+bool plan_swap_run(const LaunchCtx& ctx, const std::vector<Decoded>& gates, size_t b, size_t e,
+                   PermArgs* pa, uint64_t* moved) {
   const int nl = ctx.n_local;
-  size_t i = gates.size();
-  int count = 0;
-  while (i > 0) {
-    const Decoded& g = gates[i - 1];
-    if (g.cls == GClass::NOOP) {
-      --i;
-      continue;
-    }
-    if (g.cls != GClass::PERM_SWAP || g.cmask != 0 || g.m != 2) break;
-    --i;
-    ++count;
-  }
-  if (count < 3) return false;
+  const size_t i = b;
   int pi[64];  // pi[q]: the position the data bit at q ends at
   for (int q = 0; q < 64; ++q) pi[q] = q;
   // tile bits: auto (1) = 10 for complex128 (2 x 16 KiB tiles; 12 bits' 2 x 64 KiB allow one
   // CTA per SM: 8.0 -> 11.3 ms for the n = 30 bit reversal), 12 for complex64 (15.2 -> 13.9)
   const int max_bits = ctx.opt->fuse_perm == 1 ? (ctx.c64 ? 12 : 10) : ctx.opt->fuse_perm;
-  for (size_t k = i; k < gates.size(); ++k) {
+  for (size_t k = i; k < e; ++k) {
     const Decoded& g = gates[k];
     if (g.cls == GClass::NOOP) continue;
     const int x = g.targets[0], y = g.targets[1];
@@ -1514,44 +1505,100 @@ bool plan_swap_suffix(const LaunchCtx& ctx, const std::vector<Decoded>& gates, s
     if (pi[q] != q) mv |= 1ull << q;
   *pa = A;
   *moved = mv;
-  *end = i;
   return true;
 }
 
-void plan_fused_schedule(const LaunchCtx& ctx_in, const std::vector<Decoded>& gates_in,
+void plan_fused_core(const LaunchCtx& ctx_in, const std::vector<Decoded>& gates,
+                     int tile_qubits, std::vector<FusedPass>& out);
+
+// A trailing run of >= 3 uncontrolled SWAPs whose composition is an involution (QFT's final
+// bit reversal) becomes a bit-permutation pass after the fused passes of the gates before
+// it, when that saves passes (LFQS_OPT_FUSE_PERM).
+void plan_fused_schedule(const LaunchCtx& ctx_in, const std::vector<Decoded>& gates,
                          int tile_qubits, std::vector<FusedPass>& out) {
   out.clear();
-  // A trailing run of SWAPs becomes one bit-permutation pass, appended after the other
-  // passes when this function returns (plan-only: counted).
-  struct PermTail {
-    const LaunchCtx& c;
-    std::vector<FusedPass>& o;
+  struct Run {
+    size_t b, e;
     std::shared_ptr<PermArgs> pa;
-    uint64_t moved = 0;
-    ~PermTail() {
-      if (!pa) return;
-      if (c.plan_only) {
-        ++*c.launch_counter;
-        return;
-      }
-      FusedPass ps;
-      ps.perm = pa;
-      ps.qmask = ps.nd_mask = moved;
-      o.push_back(std::move(ps));
-    }
-  } tail{ctx_in, out, nullptr, 0};
-  std::vector<Decoded> trimmed;
-  const std::vector<Decoded>* gp = &gates_in;
+    uint64_t moved;
+  };
+  std::vector<Run> runs;
   if (ctx_in.opt->fuse_perm != 0 && !ctx_in.soa) {
-    size_t end = 0;
-    PermArgs pa;
-    if (plan_swap_suffix(ctx_in, gates_in, &end, &pa, &tail.moved)) {
-      tail.pa = std::make_shared<PermArgs>(pa);
-      trimmed.assign(gates_in.begin(), gates_in.begin() + end);
-      gp = &trimmed;
+    for (size_t k = 0; k < gates.size();) {
+      if (!is_plain_swap(gates[k])) {
+        ++k;
+        continue;
+      }
+      size_t e = k;
+      int count = 0;
+      while (e < gates.size() && (is_plain_swap(gates[e]) || gates[e].cls == GClass::NOOP)) {
+        count += is_plain_swap(gates[e]);
+        ++e;
+      }
+      // trailing runs only: a run inside a circuit splits its fused runs, and the passes
+      // around it got heavier than the SWAPs saved (QPE(30) with its inverse QFT's leading
+      // bit reversal as a pass: 12 -> 9 passes but 67.7 -> 78.0 ms)
+      size_t t = e;
+      while (t < gates.size() && gates[t].cls == GClass::NOOP) ++t;
+      PermArgs pa;
+      uint64_t mv = 0;
+      if (count >= 3 && t == gates.size() && plan_swap_run(ctx_in, gates, k, e, &pa, &mv))
+        runs.push_back(Run{k, e, std::make_shared<PermArgs>(pa), mv});
+      k = e;
     }
   }
-  const std::vector<Decoded>& gates = *gp;
+  Options o = *ctx_in.opt;
+  o.fuse_perm = 0;
+  LaunchCtx sub = ctx_in;
+  sub.opt = &o;
+  if (!runs.empty() && !ctx_in.plan_only) {
+    // keep the permutation passes only if they save passes: SWAPs next to diagonal-only
+    // work (an inverse QFT's leading bit reversal after QPE's controlled phases) already
+    // ride in passes that have tile slots to spare (host-only pass counts)
+    auto count = [&](bool with) {
+      uint64_t c = 0;
+      LaunchCtx pc = with ? ctx_in : sub;
+      pc.plan_only = true;
+      pc.launch_counter = &c;
+      std::vector<FusedPass> tmp;
+      plan_fused_schedule(pc, gates, tile_qubits, tmp);
+      return c;
+    };
+    if (count(true) >= count(false)) runs.clear();
+  }
+  if (runs.empty()) {
+    plan_fused_core(ctx_in, gates, tile_qubits, out);
+    return;
+  }
+  auto segment = [&](size_t b, size_t e) {
+    if (b >= e) return;
+    std::vector<Decoded> part(gates.begin() + b, gates.begin() + e);
+    std::vector<FusedPass> tmp;
+    plan_fused_core(sub, part, tile_qubits, tmp);
+    for (FusedPass& ps : tmp) {
+      if (!ps.prog && !ps.perm) ps.gate += (int)b;
+      out.push_back(std::move(ps));
+    }
+  };
+  size_t at = 0;
+  for (const Run& r : runs) {
+    segment(at, r.b);
+    if (ctx_in.plan_only) {
+      ++*ctx_in.launch_counter;
+    } else {
+      FusedPass ps;
+      ps.perm = r.pa;
+      ps.qmask = ps.nd_mask = r.moved;
+      out.push_back(std::move(ps));
+    }
+    at = r.e;
+  }
+  segment(at, gates.size());
+}
+
+void plan_fused_core(const LaunchCtx& ctx_in, const std::vector<Decoded>& gates,
+                     int tile_qubits, std::vector<FusedPass>& out) {
+  out.clear();
   // LFQS_OPT_FUSE_LOW_QUBITS = 0 (auto): plan the passes (host only) with 7 and with 6
   // contiguous low qubits per tile and take 6 only when it saves >= 20 % of the passes --
   // a 1-KiB-chunk tile costs ~10 % more per pass (twice the TMA copies) but claims one
@@ -1569,7 +1616,7 @@ void plan_fused_schedule(const LaunchCtx& ctx_in, const std::vector<Decoded>& ga
       pc.plan_only = true;
       pc.launch_counter = &c;
       std::vector<FusedPass> tmp;
-      plan_fused_schedule(pc, gates, tile_qubits, tmp);
+      plan_fused_core(pc, gates, tile_qubits, tmp);
       return c;
     };
     const uint64_t p7 = count(7), p6 = count(6);

@@ -268,3 +268,32 @@ def test_bitperm_pass(n, c64):
                 res[perm, fuse] = st.copy_out()
             assert np.max(np.abs(res[perm, fuse] - ref)) <= (2e-5 if c64 else 1e-12)
     assert np.array_equal(res[1, "phase"], res[1, "jit+phase"])
+
+
+def test_bitperm_inside_circuit():
+    """A SWAP run inside a circuit (an inverse QFT's leading bit reversal in QPE) is split
+    out as a permutation pass only when that saves passes; either way the result equals the
+    run without permutation passes within tolerance, and exact circuits stay bit-exact."""
+    import torch
+    if not torch.cuda.is_available():
+        pytest.skip("needs a GPU")
+    import paper_conf_cgo_tarabkhahdds25_b200 as L
+    n = 17
+    psi = W.random_state(n, 5)
+    rev = [W.Gate("SWAP", (q, n - 1 - q)) for q in range(n // 2)]
+    exact = [g for g in W.random_gate_list(n, 100, seed=3, max_controls=1) if g.exact]
+    for gates, bitexact in ((W.qpe(n - 1, 0x5A5A), False), (exact + rev + exact, True),
+                            (W.qft(n) + W.random_layered(n, 2, seed=1) + W.qft_inverse(n), False)):
+        ref = O.run_circuit(n, gates, psi.copy())
+        outs = []
+        for perm in (0, 1):
+            with L.State.create(n) as st:
+                st.set_option(L.OPT_FUSE_PERM, perm)
+                st.copy_in(psi)
+                st.run_circuit(gates, fuse="jit+phase" if not bitexact else "jit")
+                outs.append(st.copy_out())
+        for o in outs:
+            if bitexact:
+                assert np.array_equal(o, ref)
+            else:
+                assert np.max(np.abs(o - ref)) <= 1e-12
