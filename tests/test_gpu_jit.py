@@ -277,3 +277,27 @@ def test_phase_extraction(L, fuse, c64):
     for pe in (0, 1):
         assert np.array_equal(outs[pe, interp], outs[pe, fuse]), pe
     assert not np.array_equal(outs[0, fuse], outs[1, fuse])
+
+
+def test_qft33_full_size_sampled(L):
+    """configs[2] at full size in the bench's launch configuration (compiled passes + phase
+    tables: folded Hadamard scales, hoisted table factors, the bit-permutation pass for the
+    final SWAPs): QFT(33)|x> against its closed form e^{2 pi i x y / 2^33} / 2^16.5 on
+    sampled amplitudes (the state does not fit the host oracle), and the norm."""
+    import torch
+    n = 33
+    free = torch.cuda.mem_get_info()[0]
+    if free < (16 << n) + (4 << 30):
+        pytest.skip("needs a 128 GiB state")
+    x = 0x1A2B3C4D5 & ((1 << n) - 1)
+    rng = np.random.default_rng(3)
+    idx = np.unique(np.concatenate([rng.integers(0, 1 << n, 200), [0, 1, (1 << n) - 1]]))
+    with L.State.create(n) as st:
+        st.init_basis(x)
+        st.run_circuit(W.qft(n), fuse="jit+phase")
+        got = np.array([st.copy_out(int(k), 1)[0] for k in idx])
+        norm = st.norm2()
+    ref = np.exp(2j * np.pi * ((x * idx.astype(object)) % (1 << n)).astype(np.float64) / (1 << n)) \
+        / np.sqrt(2.0 ** n)
+    assert np.max(np.abs(got - ref)) <= 1e-12
+    assert abs(norm - 1.0) <= 1e-12
