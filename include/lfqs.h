@@ -485,6 +485,13 @@ lfqs_status lfqs_state_pass_count(const lfqs_state* s, uint64_t* passes);
                                   (QFT's bit reversal) applies them as one bit-permutation
                                   pass (tile pairs closed under the permutation); 8..12: that
                                   many tile bits at most; 0: off.  Moves only: bit-identical */
+#define LFQS_OPT_EXCHANGE_WIDE 29 /* sharded states on the device / P2P transports, 1
+                                  (default): the planner may exchange a global qubit with any
+                                  local position >= 3 (Belady over all of them; the swap kernel
+                                  moves any block in place), and canonicalisation needs no
+                                  SWAP pass to bring a low qubit to the top first; 0: the top
+                                  window the NCCL transport uses.  Results within tolerance
+                                  (a different plan) */
 lfqs_status lfqs_set_option(lfqs_state* s, int option, int64_t value);
 const char* lfqs_last_error(void);
 int lfqs_abi_version(void);

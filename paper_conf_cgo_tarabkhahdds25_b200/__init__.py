@@ -58,6 +58,7 @@ OPT_FUSE_H_SCALE = 25
 OPT_FUSE_PHASE_EXTRACT = 26
 OPT_CANON_FUSE = 27
 OPT_FUSE_PERM = 28
+OPT_EXCHANGE_WIDE = 29
 
 STATUS = {0: "OK", -1: "INVALID_ARG", -2: "OUT_OF_MEMORY", -3: "CUDA", -4: "NCCL",
           -5: "UNSUPPORTED"}

@@ -538,6 +538,7 @@ lfqs_status lfqs_set_option(lfqs_state* s, int option, int64_t value) {
       case LFQS_OPT_FUSE_H_SCALE: st->opt.fuse_h_scale = value != 0; break;
       case LFQS_OPT_FUSE_PHASE_EXTRACT: st->opt.fuse_phase_extract = value != 0; break;
       case LFQS_OPT_CANON_FUSE: st->opt.canon_fuse = value != 0; break;
+      case LFQS_OPT_EXCHANGE_WIDE: st->opt.exchange_wide = value != 0; break;
       case LFQS_OPT_FUSE_PERM:
         require(value == 0 || value == 1 || (value >= 8 && value <= 12),
                 "LFQS_OPT_FUSE_PERM must be 0, 1 or a tile size in [8, 12]");

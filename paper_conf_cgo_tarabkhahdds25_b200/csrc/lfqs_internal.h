@@ -110,6 +110,7 @@ struct Options {
   bool fuse_merge_commuting = true;  // merge same-qubit 1-target gates across commuting gates
   int fuse_perm = 1;         // trailing SWAP runs as one bit-permutation pass (k_bitperm)
                              // with at most this many tile bits (0: off, 1: auto)
+  bool exchange_wide = true;  // device / P2P transports: exchanges at any local position >= 3
   bool canon_fuse = true;     // canonicalising SWAP passes fused (State::canonicalize)
   bool fuse_phase_extract = true;  // global phases of dense 1-target gates (extract_phases)
   bool fuse_h_scale = true;   // Hadamard scales of a fused pass folded into one (fold_h_scales)

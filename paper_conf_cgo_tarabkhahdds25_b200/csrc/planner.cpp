@@ -102,7 +102,7 @@ void Planner::plan_canonicalize(std::vector<PlanOp>& out) {
   // low position l would split the exchanged half-shard into 2^(n_local-1-l) pieces of
   // 2^l amplitudes (the NCCL transport sends one message per piece).  A qubit that sits
   // lower is first moved to the top local position by one local SWAP pass.
-  const int wlo = std::max(0, n_local - kSwapWindow);
+  const int wlo = swap_lo >= 0 ? std::min(swap_lo, n_local - 1) : std::max(0, n_local - kSwapWindow);
   for (int G = n - 1; G >= n_local; --G) {
     int P = l2p[G];
     if (P == G) continue;
@@ -170,7 +170,7 @@ void Planner::plan_gate(const Decoded& g, std::vector<PlanOp>& out,
       int l = -1, best = -1;
       const int rsv = std::max(0, std::min(reserve_top, n_local - 4));
       const int top = n_local - 1 - rsv;
-      const int lo = std::max(0, top + 1 - kSwapWindow);
+      const int lo = swap_lo >= 0 ? std::min(swap_lo, top) : std::max(0, top + 1 - kSwapWindow);
       for (int p = top; p >= lo; --p) {
         if (tmask >> p & 1) continue;
         const int score = next_use ? (*next_use)[p2l[p]] : 0;

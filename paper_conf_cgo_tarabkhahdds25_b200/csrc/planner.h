@@ -39,6 +39,10 @@ struct Planner {
   // the one used furthest in the future (Belady), among the top kSwapWindow
   // local positions (so exchanged pieces stay >= 2^(n_local - kSwapWindow) amps).
   static constexpr int kSwapWindow = 8;
+  // >= 0: exchange positions may go down to this local position instead (the device and
+  // P2P transports swap any block in place, so small pieces cost nothing extra there; the
+  // NCCL transport keeps the window for its message sizes).  Set per run by the State.
+  int swap_lo = -1;
   // The top reserve_top local positions are never chosen as the exchange position l by
   // plan_gate: they are the chunk bits of overlapped exchanges (state.cu execute), which
   // split an exchange into parts by them while the neighbouring local ops run part by part.

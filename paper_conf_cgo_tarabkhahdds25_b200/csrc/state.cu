@@ -652,8 +652,13 @@ void State::execute(const std::vector<PlanOp>& ops, bool fuse) {
 // SWAPs share one tile pass, bit-identical to one pass per SWAP, and the exchanges between
 // them may take strided chunk qubits and overlap with them (QFT(33) on 8 ranks: 8 SWAP
 // passes -> 3).  The interpreting kernel runs them (no compiled passes outside a run).
+void State::plan_window() {
+  plan.swap_lo = (opt.exchange_wide && (virt || p2p)) ? std::min(3, n_local - 1) : -1;
+}
+
 void State::canonicalize() {
   std::vector<PlanOp> ops;
+  plan_window();
   plan.plan_canonicalize(ops);
   const bool j = jit, pt = phase_tables;
   jit = phase_tables = false;
@@ -670,6 +675,7 @@ void State::apply(const Decoded& g) {
     return;
   }
   std::vector<PlanOp> ops;
+  plan_window();
   plan.plan_gate(g, ops);
   execute(ops, false);
 }
@@ -691,6 +697,7 @@ void State::run(const std::vector<Decoded>& gates, uint32_t flags) {
     return;
   }
   std::vector<PlanOp> ops;
+  plan_window();
   plan.plan_circuit(gates, ops);  // Belady lookahead over the whole circuit
   execute(ops, fuse);
 }
@@ -766,6 +773,7 @@ void State::run_streamed(const void* host, const std::vector<Decoded>& gates, ui
     run_local(ctx(0), rest, fuse);
   } else {
     std::vector<PlanOp> ops;
+    plan_window();
     plan.plan_circuit(rest, ops);  // exchanges for the global qubits, as in run()
     execute(ops, fuse);
   }

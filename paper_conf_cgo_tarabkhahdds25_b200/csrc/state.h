@@ -122,6 +122,7 @@ struct State : lfqs_state {
   void run_local(const LaunchCtx& c, const std::vector<Decoded>& gates, bool fuse);
   void exchange_data(int l, int g);  // swap physical positions l (local) and g (global)
   void canonicalize();
+  void plan_window();  // the planner's exchange window for this state's transport
 };
 
 // A circuit captured by State::compile; launch() replays it on the state's stream.
