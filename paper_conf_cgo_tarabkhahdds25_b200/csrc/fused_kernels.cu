@@ -1383,14 +1383,23 @@ __global__ void __launch_bounds__(256) k_bitperm(cx<S>* __restrict__ a,
   auto slot = [](uint32_t e) { return e + (e >> 5); };
   const uint64_t t = blockIdx.x;
   uint64_t pt = 0, bt = 0, bp = 0;
-  for (int k = 0; k < A.nf; ++k) {
-    const uint64_t b = (t >> k) & 1;
-    pt |= b << A.fdst[k];
-    bt |= b << A.fbit[k];
+  if (A.f0 >= 0 && A.rev) {  // QFT's bit reversal: contiguous tile-index bits, reversed
+    pt = __brevll(t) >> (64 - A.nf);
+    if (pt < t) return;  // the partner's CTA moves this pair
+    bt = t << A.f0;
+    bp = pt << A.f0;
+  } else {
+    for (int k = 0; k < A.nf; ++k) {
+      const uint64_t b = (t >> k) & 1;
+      pt |= b << A.fdst[k];
+      bt |= b << A.fbit[k];
+    }
+    if (pt < t) return;  // the partner's CTA moves this pair
+    for (int k = 0; k < A.nf; ++k) bp |= ((pt >> k) & 1) << A.fbit[k];
   }
-  if (pt < t) return;  // the partner's CTA moves this pair
-  for (int k = 0; k < A.nf; ++k) bp |= ((pt >> k) & 1) << A.fbit[k];
   auto dep = [&](uint32_t e) {
+    if (A.s_lo >= 0)  // two runs of tile bits: [0, s_lo) and [s_h0, ...)
+      return (uint64_t)(e & ((1u << A.s_lo) - 1)) | ((uint64_t)(e >> A.s_lo) << A.s_h0);
     uint64_t o = 0;
 #pragma unroll
     for (int k = 0; k < 16; ++k)
@@ -1398,11 +1407,30 @@ __global__ void __launch_bounds__(256) k_bitperm(cx<S>* __restrict__ a,
     return o;
   };
   const bool pair = pt != t;
+  // element e = r * 256 + tid: its offset and its source element are ORs of a per-thread
+  // part (tid's bits) and a per-r part (the same for every thread) -- the bit loops run once
+  auto srcmap = [&](uint32_t e) {
+    if (A.srev) return __brev(e) >> (32 - A.ns);
+    uint32_t src = 0;
+#pragma unroll
+    for (int k = 0; k < 16; ++k)
+      if (k < A.ns) src |= ((e >> A.sdst[k]) & 1u) << k;
+    return src;
+  };
+  const uint64_t dt = dep(threadIdx.x);
+  const uint32_t st = srcmap(threadIdx.x);
+  uint64_t dr[EPT];
+  uint32_t sr[EPT];
+#pragma unroll
+  for (int r = 0; r < EPT; ++r) {
+    dr[r] = dep(r * 256u);
+    sr[r] = srcmap(r * 256u);
+  }
   // every load of both tiles in flight before the first shared-memory store
   cx<S> v[2 * EPT];
 #pragma unroll
   for (int r = 0; r < EPT; ++r) {
-    const uint64_t o = dep(r * 256u + threadIdx.x);
+    const uint64_t o = dt | dr[r];
     v[r] = ld1(a + (bt | o));
     if (pair) v[EPT + r] = ld1(a + (bp | o));
   }
@@ -1415,12 +1443,8 @@ __global__ void __launch_bounds__(256) k_bitperm(cx<S>* __restrict__ a,
 #pragma unroll
   for (int r = 0; r < EPT; ++r) {
     // destination element e holds the source element whose bit k is e's bit sdst[k]
-    const uint32_t e = r * 256u + threadIdx.x;
-    uint32_t src = 0;
-#pragma unroll
-    for (int k = 0; k < 16; ++k)
-      if (k < A.ns) src |= ((e >> A.sdst[k]) & 1u) << k;
-    const uint64_t o = dep(e);
+    const uint32_t src = st | sr[r];
+    const uint64_t o = dt | dr[r];
     st1(a + (bp | o), sm[slot(src)]);
     if (pair) st1(a + (bt | o), sm[TP + slot(src)]);
   }
@@ -1500,6 +1524,23 @@ bool plan_swap_run(const LaunchCtx& ctx, const std::vector<Decoded>& gates, size
   }
   for (int k = 0; k < A.ns; ++k) A.sdst[k] = (uint8_t)sidx[pi[A.sbit[k]]];
   for (int k = 0; k < A.nf; ++k) A.fdst[k] = (uint8_t)fidx[pi[A.fbit[k]]];
+  bool contig = A.nf > 0, rev = A.nf > 0;
+  for (int k = 0; k < A.nf; ++k) {
+    contig &= A.fbit[k] == A.fbit[0] + k;
+    rev &= A.fdst[k] == A.nf - 1 - k;
+  }
+  if (contig) A.f0 = A.fbit[0];
+  A.rev = rev;
+  int lo = 0;
+  while (lo < A.ns && A.sbit[lo] == lo) ++lo;
+  bool two_runs = true, srev = true;
+  for (int k = lo; k < A.ns; ++k) two_runs &= A.sbit[k] == A.sbit[lo] + (k - lo);
+  for (int k = 0; k < A.ns; ++k) srev &= A.sdst[k] == A.ns - 1 - k;
+  if (two_runs) {
+    A.s_lo = lo;
+    A.s_h0 = lo < A.ns ? A.sbit[lo] : 0;
+  }
+  A.srev = srev;
   uint64_t mv = 0;
   for (int q = 0; q < nl; ++q)
     if (pi[q] != q) mv |= 1ull << q;

@@ -175,6 +175,10 @@ struct PermArgs {
   uint8_t sdst[16] = {};   // element bit k of the source goes to element bit sdst[k]
   uint8_t fbit[48] = {};   // tile-index bit k <-> position fbit[k] (ascending)
   uint8_t fdst[48] = {};   // tile-index bit k goes to tile-index bit fdst[k]
+  int f0 = -1;             // >= 0: the tile-index bits are positions f0 .. f0 + nf - 1
+  int rev = 0;             // 1: sigma reverses the tile-index bits (fdst[k] = nf - 1 - k)
+  int s_lo = -1, s_h0 = 0; // >= 0: tile bits = positions [0, s_lo) and [s_h0, s_h0 + ns - s_lo)
+  int srev = 0;            // 1: the tile bits are reversed too (sdst[k] = ns - 1 - k)
 };
 
 // One pass of a fused schedule: a single gate's class kernel, a fused tile program, or a
