@@ -1491,9 +1491,9 @@ bool plan_swap_run(const LaunchCtx& ctx, const std::vector<Decoded>& gates, size
   const size_t i = b;
   int pi[64];  // pi[q]: the position the data bit at q ends at
   for (int q = 0; q < 64; ++q) pi[q] = q;
-  // tile bits: auto (1) = 10 for complex128 (2 x 16 KiB tiles; 12 bits' 2 x 64 KiB allow one
-  // CTA per SM: 8.0 -> 11.3 ms for the n = 30 bit reversal), 12 for complex64 (15.2 -> 13.9)
-  const int max_bits = ctx.opt->fuse_perm == 1 ? (ctx.c64 ? 12 : 10) : ctx.opt->fuse_perm;
+  // tile bits: auto (1) = 10 (complex128: 2 x 16 KiB tiles; 12 bits' 2 x 64 KiB allow one
+  // CTA per SM: 5.97 -> 10.2 ms for the n = 30 bit reversal; complex64 n = 31: 5.66 vs 8.18)
+  const int max_bits = ctx.opt->fuse_perm == 1 ? 10 : ctx.opt->fuse_perm;
   for (size_t k = i; k < e; ++k) {
     const Decoded& g = gates[k];
     if (g.cls == GClass::NOOP) continue;
