@@ -31,6 +31,8 @@
 #include <cuda_runtime.h>
 
 #include <cmath>
+#include <cstdlib>
+#include <cstdio>
 #include <cstring>
 #include <map>
 #include <memory>
@@ -1640,7 +1642,7 @@ void plan_fused_schedule(const LaunchCtx& ctx_in, const std::vector<Decoded>& ga
 void plan_fused_core(const LaunchCtx& ctx_in, const std::vector<Decoded>& gates,
                      int tile_qubits, std::vector<FusedPass>& out) {
   out.clear();
-  // LFQS_OPT_FUSE_LOW_QUBITS = 0 (auto): plan the passes (host only) with 7 and with 6
+  // LFQS_OPT_FUSE_LOW_QUBITS = 0 (auto): plan the passes (host only) with 7, 6 and 5
   // contiguous low qubits per tile and take 6 only when it saves >= 20 % of the passes --
   // a 1-KiB-chunk tile costs ~10 % more per pass (twice the TMA copies) but claims one
   // more qubit (measured at n = 30: QFT 65 -> 60 ms, Grover 113 -> 109, GHZ 26 -> 24 with
@@ -1663,6 +1665,12 @@ void plan_fused_core(const LaunchCtx& ctx_in, const std::vector<Decoded>& gates,
     const uint64_t p7 = count(7), p6 = count(6);
     auto_opt = *ctx_in.opt;
     auto_opt.fuse_low_qubits = (p6 * 5 <= p7 * 4) ? 6 : 7;
+    // 5 low qubits (512-B chunks, 128 bulk copies per tile: +46 % per pass for Grover(33))
+    // only when that cuts the passes to <= 65 %: many light passes at large n (Grover(33):
+    // 26 -> 16 passes, 1052 -> 947 ms); FP64-heavy circuits lose (random layered(33): 46 ->
+    // 35 passes but 2514 -> 2764 ms), and their pass counts fall less
+    const uint64_t pb = auto_opt.fuse_low_qubits == 6 ? p6 : p7, p5 = count(5);
+    if (p5 * 20 <= pb * 13) auto_opt.fuse_low_qubits = 5;
     ctx.opt = &auto_opt;
   }
   TileCfg cfg;
