@@ -660,11 +660,16 @@ void State::canonicalize() {
   std::vector<PlanOp> ops;
   plan_window();
   plan.plan_canonicalize(ops);
-  const bool j = jit, pt = phase_tables;
+  struct Restore {  // the run's pass-compiler flags, also when execute throws
+    bool &j, &pt;
+    const bool j0, pt0;
+    ~Restore() {
+      j = j0;
+      pt = pt0;
+    }
+  } restore{jit, phase_tables, jit, phase_tables};
   jit = phase_tables = false;
   execute(ops, opt.canon_fuse && !soa);
-  jit = j;
-  phase_tables = pt;
 }
 
 void State::apply(const Decoded& g) {
