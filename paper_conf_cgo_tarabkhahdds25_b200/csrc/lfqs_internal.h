@@ -12,7 +12,19 @@
 
 #include "../../include/lfqs.h"
 
+#include <nvtx3/nvToolsExt.h>
+
 namespace lfqs {
+
+// NVTX range over a host-side phase (a circuit run, an exchange, canonicalisation,
+// a measurement) for nsys / ncu --nvtx timelines (SURVEY §5 tracing); header-only NVTX3,
+// a no-op unless a tool is attached.
+struct NvtxRange {
+  explicit NvtxRange(const char* name) { nvtxRangePushA(name); }
+  ~NvtxRange() { nvtxRangePop(); }
+  NvtxRange(const NvtxRange&) = delete;
+  NvtxRange& operator=(const NvtxRange&) = delete;
+};
 
 // Thrown inside the library, converted to lfqs_status at the ABI boundary.
 struct Error : std::runtime_error {

@@ -596,6 +596,7 @@ void State::execute(const std::vector<PlanOp>& ops, bool fuse) {
     const size_t nb = ex[k] + 1, ne = k + 1 < ex.size() ? ex[k + 1] : ops.size();
     std::vector<ShardRun> next = plan_run(ops, nb, ne, fuse);
     const uint64_t chunk = choose_chunk(ops, ex, k, fuse, prev);
+    NvtxRange nv(chunk ? "lfqs_exchange_overlapped" : "lfqs_exchange");
     if (chunk == 0) {
       launch_passes(cur, from, end, 0, 0);
       exchange_data(X.l, X.g);
@@ -657,6 +658,7 @@ void State::plan_window() {
 }
 
 void State::canonicalize() {
+  NvtxRange nv("lfqs_canonicalize");
   std::vector<PlanOp> ops;
   plan_window();
   plan.plan_canonicalize(ops);
@@ -687,6 +689,7 @@ void State::apply(const Decoded& g) {
 
 void State::run(const std::vector<Decoded>& gates, uint32_t flags) {
   DeviceGuard dg(device);
+  NvtxRange nv("lfqs_run_circuit");
   const bool fuse = (flags & LFQS_FUSE_LOW) != 0;
   if (fuse && soa)
     throw Error(LFQS_ERR_UNSUPPORTED, "fused passes need an AOS state (LFQS_STATE_SOA is per-gate only)");
@@ -717,6 +720,7 @@ void State::run(const std::vector<Decoded>& gates, uint32_t flags) {
 // copy_in + run; fused, the prefix and the rest form separate passes (rounding only).
 void State::run_streamed(const void* host, const std::vector<Decoded>& gates, uint32_t flags,
                          int chunk_bits) {
+  NvtxRange nv("lfqs_run_circuit_streamed");
   DeviceGuard dg(device);
   require(!virt && !soa, "streamed runs need an AOS state on one GPU or one shard per rank");
   require(chunk_bits >= 0 && chunk_bits <= 8 && chunk_bits < n_local,
@@ -876,6 +880,7 @@ void State::local_probs(int shard, const int* lq, int nl, double* host) {
 }
 
 void State::measure_probs(const int* qubits, int nq, double* out) {
+  NvtxRange nv("lfqs_measure_probs");
   DeviceGuard dg(device);
   const size_t nb = size_t(1) << nq;
   if (world == 1) {
