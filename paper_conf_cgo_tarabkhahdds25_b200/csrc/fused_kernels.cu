@@ -914,6 +914,22 @@ int phase_real_form(const cplx* M, cplx* R, cplx* z) {
       return real ? 1 : 2;
     }
   }
+  // kind 3: a real diagonal after the phase, any off-diagonal (sqrt W = e^{i pi/4} R): stays
+  // F_U2, the pass compiler drops the diagonal's zero imaginary parts (12 FP64 operations per
+  // pair instead of 16)
+  for (int i = 0; i < 4; i += 3) {
+    if (std::hypot(M[i].re, M[i].im) < 0.25 * best) continue;
+    const double a = std::atan2(M[i].im, M[i].re);
+    const double zr = std::cos(a), zi = std::sin(a);
+    cplx T[4];
+    for (int k = 0; k < 4; ++k)
+      T[k] = cplx{M[k].re * zr + M[k].im * zi, M[k].im * zr - M[k].re * zi};
+    if (std::fabs(T[0].im) > tol || std::fabs(T[3].im) > tol) continue;
+    for (int k = 0; k < 4; ++k) R[k] = T[k];
+    R[0].im = R[3].im = 0.0;
+    *z = cplx{zr, zi};
+    return 3;
+  }
   return 0;
 }
 
@@ -933,7 +949,9 @@ void extract_phases(FProg& P) {
     if (h.type != F_U2 || h.mlo || h.mhi) continue;
     cplx M[4], R[4], z;
     for (int k = 0; k < 4; ++k) M[k] = cplx{P.c[h.coef + k].x, P.c[h.coef + k].y};
-    if (phase_real_form(M, R, &z))
+    const int kind = phase_real_form(M, R, &z);
+    // kind 3 pays only if the diagonal had imaginary parts to drop
+    if (kind == 1 || kind == 2 || (kind == 3 && (M[0].im != 0.0 || M[3].im != 0.0)))
       conv.push_back(o);
     else
       carrier = o;
@@ -950,7 +968,7 @@ void extract_phases(FProg& P) {
     cplx M[4], R[4], z;
     for (int k = 0; k < 4; ++k) M[k] = cplx{P.c[h.coef + k].x, P.c[h.coef + k].y};
     const int kind = phase_real_form(M, R, &z);
-    h.type = kind == 1 ? F_UR : F_UI;
+    h.type = kind == 1 ? F_UR : kind == 2 ? F_UI : F_U2;
     for (int k = 0; k < 4; ++k) P.c[h.coef + k] = D2(R[k]);
     Z = cplx{Z.re * z.re - Z.im * z.im, Z.re * z.im + Z.im * z.re};
   }
