@@ -296,11 +296,14 @@ lfqs_status lfqs_measure_collapse(lfqs_state* s, const int* qubits, int n_q, uin
  *     this rank exchanges, in place, its amplitudes whose bit l equals
  *     1 - bit (g - n_local) of `rank` with the same positions of partner rank
  *     rank ^ 2^(g - n_local).
- * canonicalize != 0 appends the ops that restore the identity qubit map.
+ * canonicalize: bit 0 appends the ops that restore the identity qubit map; bit 1
+ * (LFQS_PLAN_WIDE) plans with the device / P2P transports' exchange window (any local
+ * position >= 3, LFQS_OPT_EXCHANGE_WIDE) instead of the NCCL-sized top window.
  * Returns LFQS_ERR_INVALID_ARG with *n_ops = required length if capacity is
  * too small.  The ops array must outlive any use of gate.matrix. */
 #define LFQS_PLAN_LOCAL 0
 #define LFQS_PLAN_EXCHANGE 1
+#define LFQS_PLAN_WIDE 2
 typedef struct {
   int32_t kind;
   int32_t l;

@@ -511,17 +511,20 @@ class PlanGate:
         return f"{self.kind}c{list(self.controls)}{list(self.targets)}"
 
 
-def lfqs_plan_circuit(n_qubits: int, world: int, rank: int, gates, canonicalize: bool = True):
+def lfqs_plan_circuit(n_qubits: int, world: int, rank: int, gates, canonicalize: bool = True,
+                      wide: bool = False):
     """Host-only planner query (no GPU).  Returns a list of
-    ("local", PlanGate) and ("exchange", l, g) tuples for `rank` (include/lfqs.h)."""
+    ("local", PlanGate) and ("exchange", l, g) tuples for `rank` (include/lfqs.h).
+    wide: the device / P2P transports' exchange window (LFQS_PLAN_WIDE)."""
     arr, n, keep = marshal_gates(gates)
     need = C.c_size_t(0)
-    rc = lib().lfqs_plan_circuit(n_qubits, world, rank, arr, n, int(canonicalize), None, 0,
+    flags = int(bool(canonicalize)) | (2 if wide else 0)
+    rc = lib().lfqs_plan_circuit(n_qubits, world, rank, arr, n, flags, None, 0,
                                  C.byref(need))
     if rc != 0 and need.value == 0:
         _check(rc)
     ops = (LfqsPlanOp * max(1, need.value))()
-    _check(lib().lfqs_plan_circuit(n_qubits, world, rank, arr, n, int(canonicalize), ops,
+    _check(lib().lfqs_plan_circuit(n_qubits, world, rank, arr, n, flags, ops,
                                    need.value, C.byref(need)))
     out = []
     for i in range(need.value):

@@ -341,6 +341,7 @@ lfqs_status lfqs_plan_circuit(int n_qubits, int world, int rank, const lfqs_gate
     require(n_qubits >= 1 && n_qubits <= 40, "n_qubits must be in [1, 40]");
     require(world >= 1 && rank >= 0 && rank < world, "bad rank / world");
     Planner plan(n_qubits, world);
+    if (canonicalize & LFQS_PLAN_WIDE) plan.swap_lo = std::min(3, plan.n_local - 1);
     std::vector<PlanOp> raw;
     std::vector<Decoded> dec;
     for (size_t i = 0; i < n_gates; ++i) {
@@ -359,7 +360,7 @@ lfqs_status lfqs_plan_circuit(int n_qubits, int world, int rank, const lfqs_gate
     } else {
       plan.plan_circuit(dec, raw);  // the same planning State::run uses
     }
-    if (canonicalize) plan.plan_canonicalize(raw);
+    if (canonicalize & 1) plan.plan_canonicalize(raw);
     // Rank-specialise and convert.
     std::vector<lfqs_plan_op> out;
     for (const PlanOp& op : raw) {
