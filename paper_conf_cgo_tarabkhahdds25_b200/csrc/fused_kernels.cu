@@ -1631,6 +1631,9 @@ void plan_fused_schedule(const LaunchCtx& ctx_in, const std::vector<Decoded>& ga
     plan_fused_core(ctx_in, gates, tile_qubits, out);
     return;
   }
+  // the automatic low-qubit choice compares whole-run pass counts, permutation passes
+  // included (QFT(30): 6 vs 5 passes -> L = 7, 36.7 ms, not L = 6's 38.7 ms)
+  o.auto_extra_passes = (int)runs.size();
   auto segment = [&](size_t b, size_t e) {
     if (b >= e) return;
     std::vector<Decoded> part(gates.begin() + b, gates.begin() + e);
@@ -1682,12 +1685,13 @@ void plan_fused_core(const LaunchCtx& ctx_in, const std::vector<Decoded>& gates,
     };
     const uint64_t p7 = count(7), p6 = count(6);
     auto_opt = *ctx_in.opt;
-    auto_opt.fuse_low_qubits = (p6 * 5 <= p7 * 4) ? 6 : 7;
+    const uint64_t x = (uint64_t)ctx_in.opt->auto_extra_passes;
+    auto_opt.fuse_low_qubits = ((p6 + x) * 5 <= (p7 + x) * 4) ? 6 : 7;
     // 5 low qubits (512-B chunks, 128 bulk copies per tile: +46 % per pass for Grover(33))
     // only when that cuts the passes to <= 65 %: many light passes at large n (Grover(33):
     // 26 -> 16 passes, 1052 -> 947 ms); FP64-heavy circuits lose (random layered(33): 46 ->
     // 35 passes but 2514 -> 2764 ms), and their pass counts fall less
-    const uint64_t pb = auto_opt.fuse_low_qubits == 6 ? p6 : p7, p5 = count(5);
+    const uint64_t pb = (auto_opt.fuse_low_qubits == 6 ? p6 : p7) + x, p5 = count(5) + x;
     if (p5 * 20 <= pb * 13) auto_opt.fuse_low_qubits = 5;
     ctx.opt = &auto_opt;
   }

@@ -120,6 +120,7 @@ struct Options {
   int stream_max_prefix = 0;  // lfqs_run_circuit_streamed: max gates run per piece (0: all)
   bool fuse_phase_split = false;     // phase tables: tile-invariant / tile-dependent groups
   bool fuse_merge_commuting = true;  // merge same-qubit 1-target gates across commuting gates
+  int auto_extra_passes = 0;  // internal: passes planned outside the auto-tiled run
   int fuse_perm = 1;         // trailing SWAP runs as one bit-permutation pass (k_bitperm)
                              // with at most this many tile bits (0: off, 1: auto)
   bool exchange_wide = true;  // device / P2P transports: exchanges at any local position >= 3
