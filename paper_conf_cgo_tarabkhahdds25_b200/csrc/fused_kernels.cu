@@ -1687,6 +1687,14 @@ void plan_fused_core(const LaunchCtx& ctx_in, const std::vector<Decoded>& gates,
     auto_opt = *ctx_in.opt;
     const uint64_t x = (uint64_t)ctx_in.opt->auto_extra_passes;
     auto_opt.fuse_low_qubits = ((p6 + x) * 5 <= (p7 + x) * 4) ? 6 : 7;
+    // moves and Hadamards only (GHZ): passes are pure HBM streams, so 6 low qubits pay as
+    // soon as they save more than the ~10 % a 1-KiB-chunk pass costs extra (GHZ(33): 6 -> 5
+    // passes, 225 -> 204 ms); phase tables and dense gates keep the 20 % rule
+    bool light = true;
+    for (const Decoded& g : gates)
+      light &= g.cls == GClass::NOOP || g.cls == GClass::PERM_X || g.cls == GClass::PERM_Y ||
+               g.cls == GClass::PERM_SWAP || g.is_h;
+    if (light && (p6 + x) * 11 < (p7 + x) * 10) auto_opt.fuse_low_qubits = 6;
     // 5 low qubits (512-B chunks, 128 bulk copies per tile: +46 % per pass for Grover(33))
     // only when that cuts the passes to <= 65 %: many light passes at large n (Grover(33):
     // 26 -> 16 passes, 1052 -> 947 ms); FP64-heavy circuits lose (random layered(33): 46 ->
